@@ -1,0 +1,254 @@
+/*
+ * stg.h — C ABI of libstg, the B200 (sm_100a) hot path of STGraph
+ * (Cherian et al., "STGraph: A Framework for Temporal Graph Neural Networks").
+ *
+ * Citations: "P:Lnnn" = /root/reference/PAPER.md line nnn (section in brackets);
+ * "C<k>" = reading k in DESIGN.md §Readings.
+ *
+ * Conventions (all entry points):
+ *  - Every array argument is a DEVICE pointer (cudaMalloc'd or torch-owned)
+ *    unless marked (host).  Floating point is fp32 row-major; ids are int32.
+ *  - Ownership: the caller owns every buffer it passes; inputs are only read
+ *    during the call (plus the documented by-reference retention of the state
+ *    stack).  The library owns graph / snapshot / stack storage, freed by the
+ *    matching *_destroy.  Views (stg_csr_view) are BORROWED.
+ *  - Streams: every call is ordered on the given stream (NULL = legacy default
+ *    stream).  Only *_create calls synchronise the host.  stg_dtdg_get_* never
+ *    synchronise: every snapshot size E_t is fixed at create time.
+ *  - Errors: calls return a status and never throw or abort across the ABI.
+ *    Argument checks are synchronous; asynchronous CUDA faults surface as
+ *    STG_ERR_CUDA on a later call.  stg_last_error() gives a thread-local text.
+ *  - Limits: V < 2^30, every edge count < 2^31 (else STG_ERR_OUT_OF_RANGE).
+ */
+#ifndef STG_H_
+#define STG_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* stg_stream_t;   /* == cudaStream_t */
+
+typedef enum {
+  STG_OK = 0,
+  STG_ERR_INVALID_ARG = 1,   /* NULL / negative / misaligned argument */
+  STG_ERR_OUT_OF_RANGE = 2,  /* id outside [0,V), t outside [0,T), size overflow */
+  STG_ERR_NO_MEMORY = 3,     /* device or host allocation failed */
+  STG_ERR_CUDA = 4,          /* a CUDA runtime error (possibly from earlier async work) */
+  STG_ERR_NCCL = 5,          /* reserved for collective failures */
+  STG_ERR_STATE = 6          /* object in the wrong state, e.g. pop of an empty state stack */
+} stg_status;
+
+/* Thread-local description of the last non-OK status returned on this thread. */
+const char* stg_last_error(void);
+/* Library version as an integer MAJOR*10000 + MINOR*100 + PATCH. */
+int32_t stg_version(void);
+/* Number of device kernels this library launched since load (all threads). */
+int64_t stg_kernel_launch_count(void);
+
+/* Optional allocator hook (e.g. PyTorch's caching allocator).  alloc returns a
+ * device pointer of >= bytes (256-byte aligned) or NULL; free releases it.
+ * Both are called from the host thread that calls into the library.  Passing
+ * NULL restores cudaMalloc/cudaFree.  Must be set before objects are created. */
+typedef void* (*stg_alloc_fn)(size_t bytes, stg_stream_t stream, void* ctx);
+typedef void (*stg_free_fn)(void* ptr, stg_stream_t stream, void* ctx);
+stg_status stg_set_allocator(stg_alloc_fn alloc, stg_free_fn free_fn, void* ctx);
+
+/* Graph creation flags. */
+enum {
+  STG_SELF_LOOPS = 1u << 0,     /* add (v,v) for every v (idempotent; reading C1/C11).
+                                   In a DTDG the loops are pinned: never deleted. */
+  STG_EDGE_IDS = 1u << 1,       /* compute out_eid, the shared edge labels (C6) */
+  STG_VALIDATE = 1u << 2,       /* DTDG: reject ill-formed batches (duplicate adds, adds of
+                                   present edges, deletes of absent edges) instead of
+                                   normalising them (reading C9) */
+  STG_NORM_DGL_BOTH = 1u << 3   /* n_src = out_deg^-1/2, n_dst = in_deg^-1/2 (default:
+                                   both = in_deg^-1/2, PyG gcn_norm, reading C1) */
+};
+
+/* Row-block sharding: an object created with a non-NULL
+ * stg_dist holds only the destination rows [row_begin,row_end) of the
+ * forward in-CSR and, for the backward out-CSR, only the edges whose
+ * destination lies in that block (rows = all sources).  NULL = whole graph. */
+typedef struct {
+  int32_t rank, world;
+  int32_t row_begin, row_end;
+} stg_dist;
+
+/* A BORROWED view of one snapshot.  Valid until the owning object is destroyed
+ * or, for a DTDG, until the next stg_dtdg_get_* call on it.  Layout (Fig. 3,
+ * P:L183-185):
+ *   forward CSR  : in_rowptr[R+1] (R = row_end-row_begin, local rows),
+ *                  in_col[E] = source ids ascending within a row,
+ *                  in_row[E] = the destination id of every in-edge (COO)
+ *   backward CSR : out_rowptr[V+1], out_col[E] = destination ids ascending,
+ *                  out_row[E] = the source id of every out-edge (COO)
+ *   out_eid[E]   : in-CSR position of out-edge j (shared edge label), or NULL
+ *   in_deg/out_deg[V], in_ids/out_ids[V] = vertices by degree desc, id asc
+ *   norm_src/norm_dst[V] fp32 GCN normalisation vectors (reading C1)
+ *   in_sched/out_sched: library-internal degree-bucket schedules for the
+ *   aggregation kernels (may be NULL in caller-built views).
+ *   workspace: library-internal scratch handle (may be NULL). */
+typedef struct {
+  int32_t num_nodes;
+  int32_t row_begin, row_end;
+  int32_t timestamp;            /* -1 for a static graph */
+  int64_t num_edges;            /* edges held by this view (local edges if sharded) */
+  const int32_t *in_rowptr, *in_col, *in_row;
+  const int32_t *out_rowptr, *out_col, *out_row;
+  const int32_t *out_eid;
+  const int32_t *in_deg, *out_deg, *in_ids, *out_ids;
+  const float *norm_src, *norm_dst;
+  const int32_t *in_sched, *out_sched;
+  void* workspace;
+} stg_csr_view;
+
+typedef struct stg_graph stg_graph;
+typedef struct stg_dtdg stg_dtdg;
+typedef struct stg_state_stack stg_state_stack;
+
+/* ---- static graph (Definition II.1; STGraphBase) ----
+ * Builds the edge SET {(src[i],dst[i])} (duplicates removed, loops added with
+ * STG_SELF_LOOPS), both CSRs, degrees, node_ids, norms and (STG_EDGE_IDS) the
+ * shared edge labels, all on the device.  src/dst: E device ids in [0,V).
+ * Synchronises `stream`.  *out is owned by the caller; free with _destroy. */
+stg_status stg_static_graph_create(int32_t V, int64_t E, const int32_t* src, const int32_t* dst,
+                                   uint32_t flags, const stg_dist* dist, stg_stream_t stream,
+                                   stg_graph** out);
+stg_status stg_graph_view(const stg_graph* g, stg_csr_view* out);
+void stg_graph_destroy(stg_graph* g);
+
+/* ---- DTDG (Definition II.2; GPMAGraph behaviour) ----
+ * Base snapshot S_0 = {(src0,dst0)} plus per-timestamp batches: batch t is
+ * add_src/add_dst[add_off[t] .. add_off[t+1]) and likewise for deletes, with
+ * S_t = (S_{t-1} \ D_t) ∪ A_t.  add_off/del_off are HOST arrays of
+ * T+1 int64; batch 0 must be empty.  The batches are normalised here to the
+ * effective deltas A'_t = A_t \ S_{t-1}, D'_t = (D_t \ A_t) ∩ S_{t-1} (reading C9),
+ * stored on the device in both (dst,src) and (src,dst) order; every E_t is then
+ * known.  Synchronises `stream`. */
+stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0, const int32_t* dst0,
+                           const int64_t* add_off, const int32_t* add_src, const int32_t* add_dst,
+                           const int64_t* del_off, const int32_t* del_src, const int32_t* del_dst,
+                           uint32_t flags, const stg_dist* dist, stg_stream_t stream, stg_dtdg** out);
+/* Get-Graph(G, t) (Algorithm 2; reading C8): returns the
+ * snapshot for t built on demand from the nearest cached snapshot (base, the
+ * forward head, the backward cursor) by applying |Δt| delta steps on `stream`. */
+stg_status stg_dtdg_get_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, stg_csr_view* out);
+/* Get-Backward-Graph(G, t): the same snapshot t for the backward pass,
+ * reached from the backward cursor by reverse updates, without disturbing the
+ * cached forward head (which the next sequence starts from). */
+stg_status stg_dtdg_get_backward_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, stg_csr_view* out);
+int64_t stg_dtdg_num_edges(const stg_dtdg* g, int32_t t);    /* -1 if t out of range */
+int32_t stg_dtdg_num_timestamps(const stg_dtdg* g);
+/* Number of effective added / deleted edges of step t (0 for t = 0). */
+int64_t stg_dtdg_num_deltas(const stg_dtdg* g, int32_t t, int32_t deletes);
+void stg_dtdg_destroy(stg_dtdg* g);
+
+/* ---- GCN aggregation (north_star) ----
+ * forward : y[v,:] = n_dst[v] · Σ_{u∈N_in(v)} n_src[u] · x[u,:]   over the in-CSR,
+ *           for the local rows v of the view (y row i ↔ vertex row_begin+i).
+ * backward: gx[u,:] = n_src[u] · Σ_{v∈N_out(u)} n_dst[v] · gy[v,:] over the out-CSR
+ *           (the exact transpose), for all V sources (partial sums if sharded).
+ * x/gy: [V,W] (forward: all sources) with leading dimension ldx >= W;
+ * y/gx: leading dimension ldy >= W.  fp32 accumulation in a fixed order per
+ * row: results are deterministic run to run (no float atomics; reading C20).
+ * Float4 path when W, ldx, ldy are multiples of 4 and x, y are 16-byte aligned. */
+stg_status stg_gcn_aggregate_fwd(const stg_csr_view* g, int32_t W, const float* x, int64_t ldx,
+                                 float* y, int64_t ldy, stg_stream_t stream);
+stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* gy, int64_t ldgy,
+                                 float* gx, int64_t ldgx, stg_stream_t stream);
+/* General form used by both: backward=0 → in-CSR, 1 → out-CSR;
+ *   out[r,:] = scale_row[r] · Σ_{c∈row r} scale_col[c] · in[c,:] + bias[:]
+ * with scale_row / scale_col / bias each optional (NULL = 1 / 1 / 0). */
+stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t W,
+                                const float* in, int64_t ldin, float* out, int64_t ldout,
+                                const float* scale_row, const float* scale_col, const float* bias,
+                                stg_stream_t stream);
+
+/* ---- TGCN (GCN + GRU; reading C13-C15) ----
+ * W [F,3H] (gates z|r|h), b [3H], L [3][2H][H] (gate g: rows 0..H-1 = L_g¹ act
+ * on C_g, rows H..2H-1 = L_g² act on H or R⊙H), l [3][H]. */
+typedef struct {
+  int32_t F, H;
+  const float *W, *b, *L, *l;
+} stg_tgcn_params;
+typedef struct {
+  float *W, *b, *L, *l;        /* gradients, ACCUMULATED (+=), same layouts */
+} stg_tgcn_grads;
+
+/* State Stack: LIFO of per-timestamp forward state.  Each push
+ * stores C_t [V,3H] in the stack's device arena (capacity_bytes) and retains
+ * H_prev BY REFERENCE: the caller keeps that buffer unmodified until the
+ * matching backward pops it (reading A8: only {H_{t-1}, C_t} are saved). */
+stg_status stg_state_stack_create(int64_t capacity_bytes, stg_state_stack** out);
+int32_t stg_state_stack_depth(const stg_state_stack* s);
+void stg_state_stack_destroy(stg_state_stack* s);
+
+/* Forward step at one timestamp (a7):
+ *   P' = diag(n_src)·X·W;  C = diag(n_dst)·A·P' + b;  GRU gates;  H_next.
+ * X [V,F], H_prev/H_next [V,H] (all vertices; sharded views compute the local
+ * rows of C and H_next only).  stack == NULL: inference, nothing retained. */
+stg_status stg_tgcn_step(const stg_csr_view* g_fwd, const stg_tgcn_params* p, const float* X,
+                         const float* H_prev, float* H_next, stg_state_stack* stack,
+                         stg_stream_t stream);
+/* Backward step (a8): pops {H_prev, C} pushed by the matching forward step and,
+ * given dH_next = dℓ/dH_t (total), writes dH_prev = dℓ/dH_{t-1} and accumulates
+ * parameter gradients.  g_bwd must be the snapshot of the same t (its out-CSR
+ * carries dP = Âᵀ·dC).  dH_prev may alias nothing else. */
+stg_status stg_tgcn_step_backward(const stg_csr_view* g_bwd, const stg_tgcn_params* p, const float* X,
+                                  const float* dH_next, float* dH_prev, stg_tgcn_grads* grads,
+                                  stg_state_stack* stack, stg_stream_t stream);
+
+/* Surrogate MSE head (timing only; A15): ŷ_v = Σ_k ReLU(H_vk)·w_o[k] + b_o[0],
+ *   ℓ = mean_v (ŷ_v − y_v)².
+ * loss_accum (device scalar, may be NULL) += ℓ.  If dH != NULL: dH (+)= dℓ/dH
+ * (accumulate=1 adds into dH, 0 overwrites) and dw_o/db_o (if non-NULL) += grads. */
+stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o,
+                        const float* b_o, float* loss_accum, float* dH, int32_t accumulate,
+                        float* dw_o, float* db_o, stg_stream_t stream);
+
+/* p -= lr·g over n elements (the per-sequence optimiser step, reading C17). */
+stg_status stg_sgd_update(float* p, const float* g, int64_t n, float lr, stg_stream_t stream);
+
+/* Algorithm 1 for ONE sequence s = [t0, t0+S): forward for t ∈ s
+ * (DTDG: Get-Graph, graph-stack push; state-stack push; step; loss), then
+ * backward in LIFO order (graph-stack pop, Get-Backward-Graph, head gradient,
+ * step_backward).  Exactly one of `graph` / `dtdg` is non-NULL.
+ * X (host)[S] device pointers to X_t [V,F]; Y (host)[S] device pointers to y_t [V];
+ * H0 [V,H] initial state (detached); H_seq [S][V,H] receives H_t (H_seq[S-1] is
+ * the state the next sequence starts from, reading C15); G_work [2][V,H] scratch.
+ * Gradients (grads, dw_o, db_o) and loss_accum are accumulated. */
+stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
+                                   const stg_tgcn_params* p, const float* w_o, const float* b_o,
+                                   const float* const* X, const float* const* Y, const float* H0,
+                                   float* H_seq, float* G_work, stg_tgcn_grads* grads, float* dw_o,
+                                   float* db_o, float* loss_accum, stg_state_stack* stack,
+                                   stg_stream_t stream);
+
+/* ---- multi-GPU helpers ----
+ * nnz-balanced destination row blocks: bounds (host)[world+1] with bounds[0]=0,
+ * bounds[world]=V, block k ≈ E/world in-edges.  in_rowptr is a DEVICE [V+1]
+ * array of a whole-graph view.  Synchronises `stream`. */
+stg_status stg_partition_rows(int32_t V, const int32_t* in_rowptr, int32_t world, int32_t* bounds,
+                              stg_stream_t stream);
+
+/* Per-phase device timing with CUDA events recorded on the launching stream
+ * around each phase (bench.py; the GNN vs graph-update split of Fig. 9,
+ * P:L316/L345).  phase: 0 aggregation fwd, 1 aggregation bwd, 2 snapshot
+ * build (Get-Graph / Get-Backward-Graph), 3 P' = X·W, 4 GRU fwd, 5 GRU bwd,
+ * 6 dW, 7 head.  stg_profile_read synchronises on the recorded events and
+ * returns the accumulated milliseconds and count (reset != 0 clears them). */
+stg_status stg_profile_enable(int32_t on);
+stg_status stg_profile_read(int32_t phase, double* total_ms, int64_t* count, int32_t reset);
+
+/* Stream-ordered byte copy (kind: 0 device->device, 1 host->device,
+ * 2 device->host); lets bindings read borrowed view arrays. */
+stg_status stg_memcpy(void* dst, const void* src, size_t bytes, int32_t kind, stg_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STG_H_ */

@@ -115,13 +115,16 @@ void orc_csr_build(int32_t V, int64_t n, const uint64_t* S, int32_t dgl_both,
     in_col[in_rowptr[v] + fill[v]++] = ksrc(S[i]);
   }
   free(fill);
-  /* shared edge labels: the in-CSR position of every out-edge (linear search) */
+  /* shared edge labels: the in-CSR position of every out-edge (the row of v
+   * is sorted ascending, so the position of u is found by bisection) */
   for (int32_t u = 0; u < V; ++u)
     for (int32_t j = out_rowptr[u]; j < out_rowptr[u + 1]; ++j) {
-      int32_t v = out_col[j], e = -1;
-      for (int32_t k = in_rowptr[v]; k < in_rowptr[v + 1]; ++k)
-        if (in_col[k] == u) { e = k; break; }
-      out_eid[j] = e;
+      int32_t v = out_col[j], lo = in_rowptr[v], hi = in_rowptr[v + 1];
+      while (lo < hi) {
+        int32_t mid = lo + (hi - lo) / 2;
+        if (in_col[mid] < u) lo = mid + 1; else hi = mid;
+      }
+      out_eid[j] = (lo < in_rowptr[v + 1] && in_col[lo] == u) ? lo : -1;
     }
   node_ids(V, in_deg, in_ids);    /* forward pass order: in-degree */
   node_ids(V, out_deg, out_ids);  /* backward pass order: out-degree */

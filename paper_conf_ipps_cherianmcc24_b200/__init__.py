@@ -1,0 +1,394 @@
+"""Python binding of libstg — the B200 (sm_100a) hot path of STGraph.
+
+Argument marshalling only: every step of the path runs in libstg's CUDA
+kernels (csrc/).  Functions keep the C-ABI names of include/stg.h.  PyTorch is
+used for device memory and streams; there is NO CPU fallback — importing this
+package fails loudly when libstg.so is missing, and every call raises StgError
+on a non-OK status.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libstg.so")
+
+STG_SELF_LOOPS = 1 << 0
+STG_EDGE_IDS = 1 << 1
+STG_VALIDATE = 1 << 2
+STG_NORM_DGL_BOTH = 1 << 3
+
+STATUS = {0: "STG_OK", 1: "STG_ERR_INVALID_ARG", 2: "STG_ERR_OUT_OF_RANGE", 3: "STG_ERR_NO_MEMORY",
+          4: "STG_ERR_CUDA", 5: "STG_ERR_NCCL", 6: "STG_ERR_STATE"}
+
+
+class StgError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__("%s: %s" % (STATUS.get(status, status), msg))
+        self.status = status
+
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError("libstg.so not built (%s); run __graft_entry__.build()" % LIB_PATH)
+
+_P = ctypes.c_void_p
+_i32, _i64, _u32, _f32 = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_float
+
+
+class stg_dist(ctypes.Structure):
+    _fields_ = [("rank", _i32), ("world", _i32), ("row_begin", _i32), ("row_end", _i32)]
+
+
+class stg_csr_view(ctypes.Structure):
+    _fields_ = [("num_nodes", _i32), ("row_begin", _i32), ("row_end", _i32), ("timestamp", _i32),
+                ("num_edges", _i64),
+                ("in_rowptr", _P), ("in_col", _P), ("in_row", _P),
+                ("out_rowptr", _P), ("out_col", _P), ("out_row", _P),
+                ("out_eid", _P),
+                ("in_deg", _P), ("out_deg", _P), ("in_ids", _P), ("out_ids", _P),
+                ("norm_src", _P), ("norm_dst", _P),
+                ("in_sched", _P), ("out_sched", _P),
+                ("workspace", _P)]
+
+
+class stg_tgcn_params(ctypes.Structure):
+    _fields_ = [("F", _i32), ("H", _i32), ("W", _P), ("b", _P), ("L", _P), ("l", _P)]
+
+
+class stg_tgcn_grads(ctypes.Structure):
+    _fields_ = [("W", _P), ("b", _P), ("L", _P), ("l", _P)]
+
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+
+def _decl(name, argtypes, restype=_i32):
+    f = getattr(_lib, name)
+    f.argtypes = argtypes
+    f.restype = restype
+    return f
+
+
+_decl("stg_last_error", [], ctypes.c_char_p)
+_decl("stg_version", [], _i32)
+_decl("stg_kernel_launch_count", [], _i64)
+_decl("stg_memcpy", [_P, _P, ctypes.c_size_t, _i32, _P])
+_decl("stg_static_graph_create", [_i32, _i64, _P, _P, _u32, _P, _P, ctypes.POINTER(_P)])
+_decl("stg_graph_view", [_P, ctypes.POINTER(stg_csr_view)])
+_decl("stg_graph_destroy", [_P], None)
+_decl("stg_dtdg_create", [_i32, _i32, _i64, _P, _P, _P, _P, _P, _P, _P, _P, _u32, _P, _P, ctypes.POINTER(_P)])
+_decl("stg_dtdg_get_snapshot", [_P, _i32, _P, ctypes.POINTER(stg_csr_view)])
+_decl("stg_dtdg_get_backward_snapshot", [_P, _i32, _P, ctypes.POINTER(stg_csr_view)])
+_decl("stg_dtdg_num_edges", [_P, _i32], _i64)
+_decl("stg_dtdg_num_timestamps", [_P], _i32)
+_decl("stg_dtdg_num_deltas", [_P, _i32, _i32], _i64)
+_decl("stg_dtdg_destroy", [_P], None)
+_decl("stg_gcn_aggregate_fwd", [ctypes.POINTER(stg_csr_view), _i32, _P, _i64, _P, _i64, _P])
+_decl("stg_gcn_aggregate_bwd", [ctypes.POINTER(stg_csr_view), _i32, _P, _i64, _P, _i64, _P])
+_decl("stg_gcn_aggregate_ex", [ctypes.POINTER(stg_csr_view), _i32, _i32, _P, _i64, _P, _i64, _P, _P, _P, _P])
+_decl("stg_state_stack_create", [_i64, ctypes.POINTER(_P)])
+_decl("stg_state_stack_depth", [_P], _i32)
+_decl("stg_state_stack_destroy", [_P], None)
+_decl("stg_tgcn_step", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn_params), _P, _P, _P, _P, _P])
+_decl("stg_tgcn_step_backward", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn_params), _P, _P, _P,
+                                 ctypes.POINTER(stg_tgcn_grads), _P, _P])
+_decl("stg_mse_head", [_i32, _i32, _P, _P, _P, _P, _P, _P, _i32, _P, _P, _P])
+_decl("stg_sgd_update", [_P, _P, _i64, _f32, _P])
+_decl("stg_tgcn_train_sequence", [_P, _P, _i32, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P,
+                                  ctypes.POINTER(_P), ctypes.POINTER(_P), _P, _P, _P,
+                                  ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P, _P])
+_decl("stg_partition_rows", [_i32, _P, _i32, ctypes.POINTER(_i32), _P])
+
+ABI_SYMBOLS = [
+    "stg_last_error", "stg_version", "stg_kernel_launch_count", "stg_set_allocator", "stg_memcpy",
+    "stg_static_graph_create", "stg_graph_view", "stg_graph_destroy",
+    "stg_dtdg_create", "stg_dtdg_get_snapshot", "stg_dtdg_get_backward_snapshot", "stg_dtdg_num_edges",
+    "stg_dtdg_num_timestamps", "stg_dtdg_num_deltas", "stg_dtdg_destroy",
+    "stg_gcn_aggregate_fwd", "stg_gcn_aggregate_bwd", "stg_gcn_aggregate_ex",
+    "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
+    "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_sgd_update", "stg_tgcn_train_sequence",
+    "stg_partition_rows",
+]
+
+
+def _check(status: int):
+    if status != 0:
+        raise StgError(status, _lib.stg_last_error().decode(errors="replace"))
+
+
+def _stream(stream=None):
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _ptr(t):
+    if t is None:
+        return None
+    if not t.is_cuda:
+        raise StgError(1, "expected a CUDA tensor")
+    if not t.is_contiguous():
+        raise StgError(1, "expected a contiguous tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _dev_i32(a):
+    if isinstance(a, torch.Tensor):
+        return a.to(device="cuda", dtype=torch.int32).contiguous()
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.int32)).cuda()
+
+
+def kernel_launch_count() -> int:
+    return int(_lib.stg_kernel_launch_count())
+
+
+def version() -> int:
+    return int(_lib.stg_version())
+
+
+# ---------------------------------------------------------------- graphs
+class Graph:
+    """Owner of a stg_graph* (static graph)."""
+
+    def __init__(self, handle, keep=()):
+        self.handle = handle
+        self._keep = keep
+
+    def view(self) -> stg_csr_view:
+        return stg_graph_view(self)
+
+    def close(self):
+        if self.handle:
+            _lib.stg_graph_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Dtdg:
+    """Owner of a stg_dtdg* (discrete-time dynamic graph)."""
+
+    def __init__(self, handle):
+        self.handle = handle
+
+    @property
+    def T(self) -> int:
+        return int(_lib.stg_dtdg_num_timestamps(self.handle))
+
+    def num_edges(self, t: int) -> int:
+        return int(_lib.stg_dtdg_num_edges(self.handle, t))
+
+    def num_deltas(self, t: int, deletes: bool) -> int:
+        return int(_lib.stg_dtdg_num_deltas(self.handle, t, int(deletes)))
+
+    def close(self):
+        if self.handle:
+            _lib.stg_dtdg_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def stg_static_graph_create(V: int, src, dst, flags: int = 0, stream=None) -> Graph:
+    s, d = _dev_i32(src), _dev_i32(dst)
+    out = ctypes.c_void_p()
+    _check(_lib.stg_static_graph_create(V, s.numel(), _ptr(s), _ptr(d), flags, None, _stream(stream),
+                                        ctypes.byref(out)))
+    return Graph(out)
+
+
+def stg_graph_view(g: Graph) -> stg_csr_view:
+    v = stg_csr_view()
+    _check(_lib.stg_graph_view(g.handle, ctypes.byref(v)))
+    return v
+
+
+def stg_dtdg_create(V: int, T: int, src0, dst0, add_off, add_src, add_dst, del_off, del_src, del_dst,
+                    flags: int = 0, stream=None) -> Dtdg:
+    s0, d0 = _dev_i32(src0), _dev_i32(dst0)
+    a_s, a_d = _dev_i32(add_src), _dev_i32(add_dst)
+    r_s, r_d = _dev_i32(del_src), _dev_i32(del_dst)
+    ao = np.ascontiguousarray(add_off, dtype=np.int64)
+    do = np.ascontiguousarray(del_off, dtype=np.int64)
+    if ao.size != T + 1 or do.size != T + 1:
+        raise StgError(1, "offset arrays must have T+1 entries")
+    out = ctypes.c_void_p()
+    _check(_lib.stg_dtdg_create(V, T, s0.numel(), _ptr(s0), _ptr(d0),
+                                ao.ctypes.data_as(_P), _ptr(a_s) if a_s.numel() else None,
+                                _ptr(a_d) if a_d.numel() else None,
+                                do.ctypes.data_as(_P), _ptr(r_s) if r_s.numel() else None,
+                                _ptr(r_d) if r_d.numel() else None,
+                                flags, None, _stream(stream), ctypes.byref(out)))
+    torch.cuda.current_stream().synchronize()
+    return Dtdg(out)
+
+
+def stg_dtdg_get_snapshot(d: Dtdg, t: int, stream=None) -> stg_csr_view:
+    v = stg_csr_view()
+    _check(_lib.stg_dtdg_get_snapshot(d.handle, t, _stream(stream), ctypes.byref(v)))
+    return v
+
+
+def stg_dtdg_get_backward_snapshot(d: Dtdg, t: int, stream=None) -> stg_csr_view:
+    v = stg_csr_view()
+    _check(_lib.stg_dtdg_get_backward_snapshot(d.handle, t, _stream(stream), ctypes.byref(v)))
+    return v
+
+
+def view_arrays(v: stg_csr_view, stream=None) -> dict:
+    """Copies of the view's arrays as CUDA tensors (for tests / inspection)."""
+    V, E = v.num_nodes, v.num_edges
+    R = v.row_end - v.row_begin
+    spec = {"in_rowptr": (R + 1, torch.int32), "in_col": (E, torch.int32), "in_row": (E, torch.int32),
+            "out_rowptr": (V + 1, torch.int32), "out_col": (E, torch.int32), "out_row": (E, torch.int32),
+            "out_eid": (E, torch.int32), "in_deg": (V, torch.int32), "out_deg": (V, torch.int32),
+            "in_ids": (V, torch.int32), "out_ids": (V, torch.int32), "norm_src": (V, torch.float32),
+            "norm_dst": (V, torch.float32)}
+    out = {}
+    for k, (n, dt) in spec.items():
+        p = getattr(v, k)
+        if not p:
+            continue
+        t = torch.empty(n, dtype=dt, device="cuda")
+        if n:
+            _check(_lib.stg_memcpy(ctypes.c_void_p(t.data_ptr()), ctypes.c_void_p(p), t.numel() * t.element_size(),
+                                   0, _stream(stream)))
+        out[k] = t
+    for k in ("in_sched", "out_sched"):
+        p = getattr(v, k)
+        if p:
+            hdr = torch.empty(2, dtype=torch.int32, device="cuda")
+            _check(_lib.stg_memcpy(ctypes.c_void_p(hdr.data_ptr()), ctypes.c_void_p(p), 8, 0, _stream(stream)))
+            out[k] = hdr
+    return out
+
+
+# ---------------------------------------------------------------- aggregation
+def _out2d(x, rows, W, out):
+    if out is None:
+        out = torch.empty((rows, W), dtype=torch.float32, device=x.device)
+    return out
+
+
+def stg_gcn_aggregate_fwd(v: stg_csr_view, x: torch.Tensor, y: torch.Tensor = None, stream=None):
+    W = x.shape[1]
+    y = _out2d(x, v.row_end - v.row_begin, W, y)
+    _check(_lib.stg_gcn_aggregate_fwd(ctypes.byref(v), W, _ptr(x), x.stride(0), _ptr(y), y.stride(0),
+                                      _stream(stream)))
+    return y
+
+
+def stg_gcn_aggregate_bwd(v: stg_csr_view, gy: torch.Tensor, gx: torch.Tensor = None, stream=None):
+    W = gy.shape[1]
+    gx = _out2d(gy, v.num_nodes, W, gx)
+    _check(_lib.stg_gcn_aggregate_bwd(ctypes.byref(v), W, _ptr(gy), gy.stride(0), _ptr(gx), gx.stride(0),
+                                      _stream(stream)))
+    return gx
+
+
+def stg_gcn_aggregate_ex(v: stg_csr_view, backward: bool, x: torch.Tensor, out: torch.Tensor = None,
+                         scale_row=None, scale_col=None, bias=None, stream=None):
+    W = x.shape[1]
+    rows = v.num_nodes if backward else v.row_end - v.row_begin
+    out = _out2d(x, rows, W, out)
+    _check(_lib.stg_gcn_aggregate_ex(ctypes.byref(v), int(backward), W, _ptr(x), x.stride(0), _ptr(out),
+                                     out.stride(0), _ptr(scale_row), _ptr(scale_col), _ptr(bias), _stream(stream)))
+    return out
+
+
+# ---------------------------------------------------------------- TGCN
+class StateStack:
+    def __init__(self, capacity_bytes: int):
+        h = ctypes.c_void_p()
+        _check(_lib.stg_state_stack_create(int(capacity_bytes), ctypes.byref(h)))
+        self.handle = h
+
+    @property
+    def depth(self) -> int:
+        return int(_lib.stg_state_stack_depth(self.handle))
+
+    def close(self):
+        if self.handle:
+            _lib.stg_state_stack_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def stg_state_stack_create(capacity_bytes: int) -> StateStack:
+    return StateStack(capacity_bytes)
+
+
+def make_params(p: dict) -> stg_tgcn_params:
+    F, H3 = p["W"].shape
+    return stg_tgcn_params(F, H3 // 3, _ptr(p["W"]), _ptr(p["b"]), _ptr(p["L"]), _ptr(p["l"]))
+
+
+def make_grads(g: dict) -> stg_tgcn_grads:
+    return stg_tgcn_grads(_ptr(g["W"]), _ptr(g["b"]), _ptr(g["L"]), _ptr(g["l"]))
+
+
+def stg_tgcn_step(v: stg_csr_view, params: dict, X, H_prev, H_next=None, stack: StateStack = None, stream=None):
+    if H_next is None:
+        H_next = torch.empty_like(H_prev)
+    P = make_params(params)
+    _check(_lib.stg_tgcn_step(ctypes.byref(v), ctypes.byref(P), _ptr(X), _ptr(H_prev), _ptr(H_next),
+                              stack.handle if stack else None, _stream(stream)))
+    return H_next
+
+
+def stg_tgcn_step_backward(v: stg_csr_view, params: dict, X, dH_next, grads: dict, stack: StateStack,
+                           dH_prev=None, stream=None):
+    if dH_prev is None:
+        dH_prev = torch.empty_like(dH_next)
+    P = make_params(params)
+    G = make_grads(grads)
+    _check(_lib.stg_tgcn_step_backward(ctypes.byref(v), ctypes.byref(P), _ptr(X), _ptr(dH_next), _ptr(dH_prev),
+                                       ctypes.byref(G), stack.handle, _stream(stream)))
+    return dH_prev
+
+
+def stg_mse_head(Hn, y, w_o, b_o, loss_accum=None, dH=None, accumulate=False, dw_o=None, db_o=None, stream=None):
+    V, H = Hn.shape
+    _check(_lib.stg_mse_head(V, H, _ptr(Hn), _ptr(y), _ptr(w_o), _ptr(b_o), _ptr(loss_accum), _ptr(dH),
+                             int(accumulate), _ptr(dw_o), _ptr(db_o), _stream(stream)))
+
+
+def stg_sgd_update(p: torch.Tensor, g: torch.Tensor, lr: float, stream=None):
+    _check(_lib.stg_sgd_update(_ptr(p), _ptr(g), p.numel(), float(lr), _stream(stream)))
+
+
+def stg_tgcn_train_sequence(source, t0: int, S: int, params: dict, w_o, b_o, Xs, Ys, H0, H_seq, G_work,
+                            grads: dict, dw_o, db_o, loss_accum, stack: StateStack, stream=None):
+    """Algorithm 1 over one sequence; `source` is a Graph or a Dtdg."""
+    P = make_params(params)
+    G = make_grads(grads)
+    xp = (_P * S)(*[x.data_ptr() for x in Xs])
+    yp = (_P * S)(*[y.data_ptr() for y in Ys])
+    graph = source.handle if isinstance(source, Graph) else None
+    dtdg = source.handle if isinstance(source, Dtdg) else None
+    _check(_lib.stg_tgcn_train_sequence(graph, dtdg, t0, S, ctypes.byref(P), _ptr(w_o), _ptr(b_o), xp, yp,
+                                        _ptr(H0), _ptr(H_seq), _ptr(G_work), ctypes.byref(G), _ptr(dw_o),
+                                        _ptr(db_o), _ptr(loss_accum), stack.handle, _stream(stream)))
+
+
+def stg_partition_rows(V: int, in_rowptr: torch.Tensor, world: int, stream=None) -> list:
+    b = (_i32 * (world + 1))()
+    _check(_lib.stg_partition_rows(V, _ptr(in_rowptr), world, b, _stream(stream)))
+    return list(b)

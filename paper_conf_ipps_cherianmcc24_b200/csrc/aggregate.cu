@@ -1,0 +1,378 @@
+// aggregate.cu — vertex-centric GCN aggregation for sm_100a (north_star; P:L72,
+// L195, L322).  One kernel serves the forward (in-CSR) and the backward
+// (out-CSR, the exact transpose):
+//
+//   out[r,:] = scale_row[r] · Σ_{j ∈ row r} scale_col[col[j]] · in[col[j],:] + bias
+//
+// Design:
+//  * feature-adaptive thread groups (the paper's FA-TGA): a row is
+//    owned by a group of G lanes; each lane holds VPL 128-bit vectors of the
+//    row (G·VPL·4 >= W), so a 32-lane warp works on 32/G rows at once;
+//  * rows are taken in node_ids order (degree-descending presort)
+//    so the rows sharing a warp have similar degrees;
+//  * rows with more than kHubChunk edges are split into fixed chunks of
+//    kHubChunk edges (hub items first); the last chunk to finish sums the
+//    chunk partials in a fixed order — deterministic, no float atomics;
+//  * column indices are loaded coalesced, one per lane, and broadcast with
+//    __shfl_sync; feature rows are gathered with 128-bit ld.global.nc;
+//  * U independent accumulators per vector bound every sequential fp32 chain
+//    to <= 64 terms (reading C19/C20 error bound).
+//  * persistent grid of (#SMs × resident blocks), grid-stride over work items.
+#include <map>
+#include <mutex>
+
+#include "graph.cuh"
+
+namespace stg {
+namespace {
+
+constexpr int kAggThreads = 256;
+
+struct AggArgs {
+  int32_t R;
+  const int32_t* rowptr;
+  const int32_t* col;
+  const int32_t* ids;
+  const int32_t* sched;
+  const float* srow;
+  const float* scol;
+  const float* bias;
+  int32_t W;  // columns of this launch
+  const float* x;
+  int64_t ldx;
+  float* y;
+  int64_t ldy;
+  float* partials;  // [chunks][W]
+  int32_t* counters;
+};
+
+template <int VEC> struct VecT;
+template <> struct VecT<4> { using T = float4; };
+template <> struct VecT<1> { using T = float; };
+
+__device__ __forceinline__ float4 ldg_v(const float4* p) { return __ldg(p); }
+__device__ __forceinline__ float ldg_v(const float* p) { return __ldg(p); }
+__device__ __forceinline__ float4 ldcg_v(const float4* p) { return __ldcg(p); }
+__device__ __forceinline__ float ldcg_v(const float* p) { return __ldcg(p); }
+__device__ __forceinline__ void zero(float4& a) { a = make_float4(0.f, 0.f, 0.f, 0.f); }
+__device__ __forceinline__ void zero(float& a) { a = 0.f; }
+__device__ __forceinline__ void fma_v(float4& a, float s, const float4& b) {
+  a.x = fmaf(s, b.x, a.x); a.y = fmaf(s, b.y, a.y); a.z = fmaf(s, b.z, a.z); a.w = fmaf(s, b.w, a.w);
+}
+__device__ __forceinline__ void fma_v(float& a, float s, const float& b) { a = fmaf(s, b, a); }
+__device__ __forceinline__ void add_v(float4& a, const float4& b) { a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w; }
+__device__ __forceinline__ void add_v(float& a, const float& b) { a += b; }
+__device__ __forceinline__ float4 scale_bias(float s, const float4& a, const float* bias, int c0) {
+  float4 r;
+  r.x = s * a.x; r.y = s * a.y; r.z = s * a.z; r.w = s * a.w;
+  if (bias) { r.x += bias[c0]; r.y += bias[c0 + 1]; r.z += bias[c0 + 2]; r.w += bias[c0 + 3]; }
+  return r;
+}
+__device__ __forceinline__ float scale_bias(float s, const float& a, const float* bias, int c0) {
+  float r = s * a;
+  if (bias) r += bias[c0];
+  return r;
+}
+
+template <int VEC, int G, int VPL, int U, bool SCOL>
+__global__ void __launch_bounds__(kAggThreads) k_aggregate(const AggArgs a) {
+  using VT = typename VecT<VEC>::T;
+  constexpr int NG = 32 / G;                  // row groups per warp
+  constexpr int IPL = U > G ? U / G : 1;       // column indices per lane per batch
+  constexpr int B = G * IPL;                   // edges per batch (multiple of U)
+  static_assert(B % U == 0, "batch must be a multiple of U");
+  const unsigned FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const int gi = lane / G, gl = lane % G;
+  const int32_t n_hub = a.sched ? a.sched[0] : 0;
+  const int32_t n_chunks = a.sched ? a.sched[1] : 0;
+  const int32_t* cptr = a.sched ? a.sched + 2 : nullptr;
+  const int64_t total = (int64_t)n_chunks + (a.R - n_hub);
+  const int64_t warp_id = ((int64_t)blockIdx.x * kAggThreads + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * kAggThreads) >> 5;
+
+  for (int64_t base = warp_id * NG; base < total; base += nwarps * NG) {
+    const int64_t item = base + gi;
+    const bool valid = item < total;
+    int32_t v = 0, beg = 0, end = 0, hub = -1;
+    if (valid) {
+      if (item < n_chunks) {
+        int32_t lo = 0, hi = n_hub;           // largest h with cptr[h] <= item
+        while (lo < hi) {
+          int32_t mid = (lo + hi + 1) >> 1;
+          if (cptr[mid] <= item) lo = mid; else hi = mid - 1;
+        }
+        hub = lo;
+        v = a.ids[lo];
+        int32_t rb = a.rowptr[v], re = a.rowptr[v + 1];
+        beg = rb + (int32_t)(item - cptr[lo]) * kHubChunk;
+        end = min(beg + kHubChunk, re);
+      } else {
+        int64_t li = n_hub + (item - n_chunks);
+        v = a.ids ? a.ids[li] : (int32_t)li;
+        beg = a.rowptr[v];
+        end = a.rowptr[v + 1];
+      }
+    }
+    const int32_t n = end - beg;
+    const int32_t nmax = __reduce_max_sync(FULL, n);
+
+    VT acc[U][VPL];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) zero(acc[u][c]);
+
+    for (int32_t e0 = 0; e0 < nmax; e0 += B) {
+      int32_t idx[IPL];
+      float sc[IPL];
+#pragma unroll
+      for (int q = 0; q < IPL; ++q) {
+        int32_t e = e0 + q * G + gl;
+        idx[q] = e < n ? __ldg(a.col + beg + e) : -1;
+        sc[q] = (SCOL && idx[q] >= 0) ? __ldg(a.scol + idx[q]) : 1.0f;
+      }
+#pragma unroll
+      for (int k = 0; k < B; k += U) {
+        VT val[U][VPL];
+        float ss[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int j = k + u;
+          const int src = gi * G + (j % G);
+          const int32_t uu = __shfl_sync(FULL, idx[j / G], src);
+          ss[u] = SCOL ? __shfl_sync(FULL, sc[j / G], src) : 1.0f;
+          const VT* xr = reinterpret_cast<const VT*>(a.x + (int64_t)(uu < 0 ? 0 : uu) * a.ldx);
+#pragma unroll
+          for (int c = 0; c < VPL; ++c) {
+            const int cv = c * G + gl;
+            if (uu >= 0 && cv * VEC < a.W) val[u][c] = ldg_v(xr + cv);
+            else zero(val[u][c]);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int c = 0; c < VPL; ++c) {
+            if (SCOL) fma_v(acc[u][c], ss[u], val[u][c]);
+            else add_v(acc[u][c], val[u][c]);
+          }
+      }
+    }
+    // pairwise combine of the U accumulators
+#pragma unroll
+    for (int w = 1; w < U; w <<= 1)
+#pragma unroll
+      for (int u = 0; u < U; u += 2 * w)
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) add_v(acc[u][c], acc[u + w][c]);
+
+    const bool hubitem = valid && hub >= 0;
+    if (valid && !hubitem) {
+      const float s = a.srow ? a.srow[v] : 1.0f;
+      VT* yr = reinterpret_cast<VT*>(a.y + (int64_t)v * a.ldy);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv * VEC < a.W) yr[cv] = scale_bias(s, acc[0][c], a.bias, cv * VEC);
+      }
+    }
+    if (hubitem) {
+      VT* pr = reinterpret_cast<VT*>(a.partials + item * (int64_t)a.W);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv * VEC < a.W) pr[cv] = acc[0][c];
+      }
+      __threadfence();
+    }
+    __syncwarp();
+    int32_t ticket = 0;
+    if (hubitem && gl == 0) ticket = atomicAdd(a.counters + hub, 1);
+    ticket = __shfl_sync(FULL, ticket, gi * G);
+    const bool last = hubitem && ticket == (cptr[hub + 1] - cptr[hub]) - 1;
+    if (last) {
+      __threadfence();
+      const int32_t cb = cptr[hub], ce = cptr[hub + 1];
+      VT tot[VPL];
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) zero(tot[c]);
+      for (int32_t c0 = cb; c0 < ce; c0 += 16) {      // two-level fixed-order sum
+        VT blk[VPL];
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) zero(blk[c]);
+        const int32_t c1 = min(c0 + 16, ce);
+        for (int32_t ch = c0; ch < c1; ++ch) {
+          const VT* pr = reinterpret_cast<const VT*>(a.partials + (int64_t)ch * a.W);
+#pragma unroll
+          for (int c = 0; c < VPL; ++c) {
+            const int cv = c * G + gl;
+            if (cv * VEC < a.W) add_v(blk[c], ldcg_v(pr + cv));
+          }
+        }
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) add_v(tot[c], blk[c]);
+      }
+      const float s = a.srow ? a.srow[v] : 1.0f;
+      VT* yr = reinterpret_cast<VT*>(a.y + (int64_t)v * a.ldy);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv * VEC < a.W) yr[cv] = scale_bias(s, tot[c], a.bias, cv * VEC);
+      }
+      if (gl == 0) a.counters[hub] = 0;             // self-reset for the next call
+    }
+  }
+}
+
+using KernelFn = void (*)(const AggArgs);
+
+template <int VEC, int G, bool SCOL>
+KernelFn pick_vpl(int vpl) {
+  switch (vpl) {
+    case 1: return k_aggregate<VEC, G, 1, 4, SCOL>;
+    case 2: return k_aggregate<VEC, G, 2, 4, SCOL>;
+    case 3: return k_aggregate<VEC, G, 3, 2, SCOL>;
+    default: return k_aggregate<VEC, G, 4, 2, SCOL>;
+  }
+}
+
+template <int VEC, bool SCOL>
+KernelFn pick_g(int g, int vpl) {
+  switch (g) {
+    case 1: return pick_vpl<VEC, 1, SCOL>(vpl);
+    case 2: return pick_vpl<VEC, 2, SCOL>(vpl);
+    case 4: return pick_vpl<VEC, 4, SCOL>(vpl);
+    case 8: return pick_vpl<VEC, 8, SCOL>(vpl);
+    case 16: return pick_vpl<VEC, 16, SCOL>(vpl);
+    default: return pick_vpl<VEC, 32, SCOL>(vpl);
+  }
+}
+
+KernelFn pick(int vec, int g, int vpl, bool scol) {
+  if (vec == 4) return scol ? pick_g<4, true>(g, vpl) : pick_g<4, false>(g, vpl);
+  return scol ? pick_g<1, true>(g, vpl) : pick_g<1, false>(g, vpl);
+}
+
+int max_blocks_for(KernelFn fn) {
+  static std::mutex mu;
+  static std::map<KernelFn, int> cache;
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = cache.find(fn);
+  if (it != cache.end()) return it->second;
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kAggThreads, 0) != cudaSuccess || per_sm < 1) {
+    cudaGetLastError();
+    per_sm = 1;
+  }
+  int b = per_sm * num_sms();
+  cache[fn] = b;
+  return b;
+}
+
+}  // namespace
+
+// Launch plan: vector width, group size, vectors per lane for W columns.
+struct AggPlan {
+  int vec, g, vpl, wmax;
+};
+static AggPlan plan_for(int32_t W, bool vec4) {
+  AggPlan p;
+  p.vec = vec4 ? 4 : 1;
+  int nv = W / p.vec;
+  if (nv > 128) nv = 128;                 // column-split into 128-vector launches
+  int g = 1;
+  while (g < 32 && g * 4 < nv) g <<= 1;
+  p.g = g;
+  p.vpl = (nv + g - 1) / g;
+  p.wmax = 128 * p.vec;
+  return p;
+}
+
+stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
+                            float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
+                            cudaStream_t s) {
+  if (!gv) return fail(STG_ERR_INVALID_ARG, "aggregate: view is NULL");
+  if (W < 1) return fail(STG_ERR_INVALID_ARG, "aggregate: W=%d < 1", W);
+  if (ldin < W || ldout < W) return fail(STG_ERR_INVALID_ARG, "aggregate: leading dimension < W");
+  if (!in || !out) return fail(STG_ERR_INVALID_ARG, "aggregate: NULL input/output");
+  const int32_t R = backward ? gv->num_nodes : gv->row_end - gv->row_begin;
+  if (R <= 0) return STG_OK;
+  AggArgs a{};
+  a.R = R;
+  a.rowptr = backward ? gv->out_rowptr : gv->in_rowptr;
+  a.col = backward ? gv->out_col : gv->in_col;
+  a.ids = backward ? gv->out_ids : gv->in_ids;
+  a.sched = backward ? gv->out_sched : gv->in_sched;
+  if (!a.rowptr || (gv->num_edges > 0 && !a.col))
+    return fail(STG_ERR_INVALID_ARG, "aggregate: view lacks the %s CSR", backward ? "backward" : "forward");
+  if (a.sched && (!a.ids || !gv->workspace)) a.sched = nullptr;
+  a.srow = srow;
+  a.scol = scol;
+  a.bias = bias;
+  const bool vec4 = (W % 4 == 0) && (ldin % 4 == 0) && (ldout % 4 == 0) &&
+                    ((uintptr_t)in % 16 == 0) && ((uintptr_t)out % 16 == 0);
+  const AggPlan p0 = plan_for(W, vec4);
+  const int64_t chunks_bound = a.sched ? 2 * (gv->num_edges / kHubChunk) + 2 : 0;
+  AggWs* ws = static_cast<AggWs*>(gv->workspace);
+  if (a.sched) {
+    const int32_t wl = W < p0.wmax ? W : p0.wmax;
+    STG_TRY(ws->partials.alloc((size_t)chunks_bound * wl + 4, s));
+    const int64_t ncnt = sched_cap(gv->num_edges) + 1;
+    if (ws->counters_n < ncnt) {
+      STG_TRY(ws->counters.alloc(ncnt, s));
+      STG_CUDA(cudaMemsetAsync(ws->counters.p, 0, sizeof(int32_t) * ncnt, s));
+      ws->counters_n = ncnt;
+    }
+    a.partials = ws->partials.p;
+    a.counters = ws->counters.p;
+  }
+  const int64_t items_bound = (int64_t)R + chunks_bound + 1;
+  ProfScope prof(backward ? PH_AGG_BWD : PH_AGG_FWD, s);
+  for (int32_t c0 = 0; c0 < W; c0 += p0.wmax) {
+    const int32_t wl = (W - c0) < p0.wmax ? (W - c0) : p0.wmax;
+    const AggPlan p = plan_for(wl, vec4);
+    a.W = wl;
+    a.x = in + c0;
+    a.ldx = ldin;
+    a.y = out + c0;
+    a.ldy = ldout;
+    a.bias = bias ? bias + c0 : nullptr;
+    KernelFn fn = pick(p.vec, p.g, p.vpl, scol != nullptr);
+    const int rows_per_block = (kAggThreads / 32) * (32 / p.g);
+    int64_t blocks = ceil_div(items_bound, rows_per_block);
+    const int64_t mb = max_blocks_for(fn);
+    if (blocks > mb) blocks = mb;
+    if (blocks < 1) blocks = 1;
+    fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(a);
+    count_launch();
+  }
+  return check_launch("aggregate");
+}
+
+}  // namespace stg
+
+extern "C" {
+
+stg_status stg_gcn_aggregate_fwd(const stg_csr_view* g, int32_t W, const float* x, int64_t ldx, float* y,
+                                 int64_t ldy, stg_stream_t stream) {
+  if (!g) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_fwd: view is NULL");
+  return stg::aggregate_launch(g, 0, W, x, ldx, y, ldy, g->norm_dst ? g->norm_dst + g->row_begin : nullptr,
+                               g->norm_src, nullptr, (cudaStream_t)stream);
+}
+
+stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* gy, int64_t ldgy, float* gx,
+                                 int64_t ldgx, stg_stream_t stream) {
+  if (!g) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_bwd: view is NULL");
+  return stg::aggregate_launch(g, 1, W, gy, ldgy, gx, ldgx, g->norm_src, g->norm_dst, nullptr,
+                               (cudaStream_t)stream);
+}
+
+stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t W, const float* in, int64_t ldin,
+                                float* out, int64_t ldout, const float* scale_row, const float* scale_col,
+                                const float* bias, stg_stream_t stream) {
+  return stg::aggregate_launch(g, backward, W, in, ldin, out, ldout, scale_row, scale_col, bias,
+                               (cudaStream_t)stream);
+}
+
+}  // extern "C"

@@ -1,0 +1,162 @@
+// common.cu — error strings, allocator hook, launch counter.
+#include "common.cuh"
+
+#include <mutex>
+#include <vector>
+
+namespace stg {
+
+static thread_local std::string t_err;
+std::atomic<int64_t> g_launches{0};
+
+static stg_alloc_fn g_alloc = nullptr;
+static stg_free_fn g_free = nullptr;
+static void* g_ctx = nullptr;
+
+void set_error(const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  t_err = buf;
+}
+
+stg_status fail(stg_status s, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  t_err = buf;
+  return s;
+}
+
+stg_status cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
+  return fail(STG_ERR_CUDA, "%s failed at %s:%d: %s (%s)", what, file, line, cudaGetErrorName(e),
+              cudaGetErrorString(e));
+}
+
+stg_status check_launch(const char* what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(STG_ERR_CUDA, "kernel launch %s: %s", what, cudaGetErrorString(e));
+  return STG_OK;
+}
+
+void* dmalloc(size_t bytes, cudaStream_t s) {
+  if (g_alloc) return g_alloc(bytes, (stg_stream_t)s, g_ctx);
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return p;
+}
+
+void dfree(void* p, cudaStream_t s) {
+  if (!p) return;
+  if (g_free) { g_free(p, (stg_stream_t)s, g_ctx); return; }
+  cudaFree(p);
+}
+
+int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
+struct Prof {
+  std::mutex mu;
+  bool on = false;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pending[PH_COUNT];
+  std::vector<cudaEvent_t> pool;
+  double total[PH_COUNT] = {};
+  int64_t count[PH_COUNT] = {};
+};
+static Prof& prof() {
+  static Prof p;
+  return p;
+}
+bool prof_on() { return prof().on; }
+cudaEvent_t prof_event() {
+  Prof& p = prof();
+  std::lock_guard<std::mutex> lk(p.mu);
+  if (!p.pool.empty()) {
+    cudaEvent_t e = p.pool.back();
+    p.pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+void prof_push(int phase, cudaEvent_t a, cudaEvent_t b) {
+  Prof& p = prof();
+  std::lock_guard<std::mutex> lk(p.mu);
+  p.pending[phase].emplace_back(a, b);
+}
+
+}  // namespace stg
+
+extern "C" {
+
+stg_status stg_profile_enable(int32_t on) {
+  stg::prof().on = on != 0;
+  return STG_OK;
+}
+
+stg_status stg_profile_read(int32_t phase, double* total_ms, int64_t* count, int32_t reset) {
+  using namespace stg;
+  if (phase < 0 || phase >= PH_COUNT) return fail(STG_ERR_OUT_OF_RANGE, "stg_profile_read: phase %d", phase);
+  Prof& p = prof();
+  std::lock_guard<std::mutex> lk(p.mu);
+  for (auto& pr : p.pending[phase]) {
+    if (cudaEventSynchronize(pr.second) != cudaSuccess) return fail(STG_ERR_CUDA, "stg_profile_read: event sync");
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, pr.first, pr.second);
+    p.total[phase] += ms;
+    p.count[phase] += 1;
+    p.pool.push_back(pr.first);
+    p.pool.push_back(pr.second);
+  }
+  p.pending[phase].clear();
+  if (total_ms) *total_ms = p.total[phase];
+  if (count) *count = p.count[phase];
+  if (reset) { p.total[phase] = 0.0; p.count[phase] = 0; }
+  return STG_OK;
+}
+
+const char* stg_last_error(void) { return stg::t_err.c_str(); }
+
+int32_t stg_version(void) { return 100; }
+
+int64_t stg_kernel_launch_count(void) { return stg::g_launches.load(); }
+
+stg_status stg_set_allocator(stg_alloc_fn alloc, stg_free_fn free_fn, void* ctx) {
+  if ((alloc == nullptr) != (free_fn == nullptr))
+    return stg::fail(STG_ERR_INVALID_ARG, "stg_set_allocator: alloc and free must both be set or both NULL");
+  stg::g_alloc = alloc;
+  stg::g_free = free_fn;
+  stg::g_ctx = ctx;
+  return STG_OK;
+}
+
+}  // extern "C"
+
+extern "C" {
+// Byte copy on a stream (kind: 0 = device->device, 1 = host->device, 2 = device->host).
+// Used by the Python binding to read back borrowed view arrays.
+stg_status stg_memcpy(void* dst, const void* src, size_t bytes, int32_t kind, stg_stream_t stream) {
+  if (!bytes) return STG_OK;
+  if (!dst || !src) return stg::fail(STG_ERR_INVALID_ARG, "stg_memcpy: NULL pointer");
+  cudaMemcpyKind k = kind == 1 ? cudaMemcpyHostToDevice : (kind == 2 ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice);
+  cudaError_t e = cudaMemcpyAsync(dst, src, bytes, k, (cudaStream_t)stream);
+  if (e != cudaSuccess) return stg::fail(STG_ERR_CUDA, "stg_memcpy: %s", cudaGetErrorString(e));
+  return STG_OK;
+}
+}

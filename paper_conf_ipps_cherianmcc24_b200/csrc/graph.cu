@@ -1,0 +1,473 @@
+// graph.cu — snapshot builders (static graph create, CSR pair, node_ids, edge
+// labels, hub schedule) and the DTDG delta-apply step.  Hand-written sm_100a
+// kernels; the paper's Thrust/CUB routines and Algorithm 3's atomic
+// transpose are replaced by sort/merge constructions that give
+// the canonical (ascending-neighbour) order deterministically (reading C3/C7).
+#include "graph.cuh"
+#include "prims.cuh"
+
+namespace stg {
+
+BuildWs* buildws_create() { return new BuildWs(); }
+void buildws_destroy(BuildWs* w) { delete w; }
+
+static inline unsigned grid_for(int64_t n, int threads, int64_t max_blocks = 148 * 16) {
+  int64_t b = ceil_div(n > 0 ? n : 1, threads);
+  return (unsigned)(b < max_blocks ? b : max_blocks);
+}
+
+stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl) {
+  V = V_;
+  cap = cap_ > 0 ? cap_ : 1;
+  nb = 1;
+  while ((int64_t(1) << nb) < (int64_t)V) ++nb;
+  edge_ids = eids;
+  dgl_both = dgl;
+  const int64_t sc = 2 + sched_cap(cap) + 1;
+  STG_TRY(in_rowptr.alloc(V + 1)); STG_TRY(out_rowptr.alloc(V + 1));
+  STG_TRY(in_col.alloc(cap)); STG_TRY(in_row.alloc(cap));
+  STG_TRY(out_col.alloc(cap)); STG_TRY(out_row.alloc(cap));
+  if (eids) STG_TRY(out_eid.alloc(cap));
+  STG_TRY(in_deg.alloc(V)); STG_TRY(out_deg.alloc(V));
+  STG_TRY(in_ids.alloc(V)); STG_TRY(out_ids.alloc(V));
+  STG_TRY(in_sched.alloc(sc)); STG_TRY(out_sched.alloc(sc));
+  STG_TRY(norm_src.alloc(V)); STG_TRY(norm_dst.alloc(V));
+  return STG_OK;
+}
+
+void Snapshot::view(stg_csr_view* v, AggWs* ws) const {
+  v->num_nodes = V;
+  v->row_begin = 0;
+  v->row_end = V;
+  v->timestamp = t;
+  v->num_edges = E;
+  v->in_rowptr = in_rowptr.p; v->in_col = in_col.p; v->in_row = in_row.p;
+  v->out_rowptr = out_rowptr.p; v->out_col = out_col.p; v->out_row = out_row.p;
+  v->out_eid = edge_ids ? out_eid.p : nullptr;
+  v->in_deg = in_deg.p; v->out_deg = out_deg.p; v->in_ids = in_ids.p; v->out_ids = out_ids.p;
+  v->norm_src = norm_src.p; v->norm_dst = norm_dst.p;
+  v->in_sched = in_sched.p; v->out_sched = out_sched.p;
+  v->workspace = ws;
+}
+
+// ------------------------------------------------------------------ kernels
+__global__ void k_unpack(const uint64_t* __restrict__ keys, int64_t E, int nb, int32_t* __restrict__ row,
+                         int32_t* __restrict__ col) {
+  const uint64_t mask = (uint64_t(1) << nb) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t k = keys[i];
+    row[i] = (int32_t)(k >> nb);
+    col[i] = (int32_t)(k & mask);
+  }
+}
+
+__global__ void k_swap_keys(const uint64_t* __restrict__ in, int64_t E, int nb, uint64_t* __restrict__ out) {
+  const uint64_t mask = (uint64_t(1) << nb) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t k = in[i];
+    out[i] = ((k & mask) << nb) | (k >> nb);
+  }
+}
+
+// rowptr of a row-sorted COO: rowptr[v] = first index with row >= v.
+__global__ void k_rowptr(const int32_t* __restrict__ rows, int64_t E, int32_t V, int32_t* __restrict__ rowptr) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= E; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t prev = i == 0 ? -1 : rows[i - 1];
+    int32_t cur = i == E ? V : rows[i];
+    for (int32_t v = prev + 1; v <= cur; ++v) rowptr[v] = (int32_t)i;
+  }
+}
+
+__global__ void k_deg(const int32_t* __restrict__ rowptr, int32_t V, int32_t* __restrict__ deg) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
+    deg[v] = rowptr[v + 1] - rowptr[v];
+}
+
+// GCN normalisation vectors (reading C1): IEEE 1/sqrtf, 0 for degree 0.
+__global__ void k_norm(const int32_t* __restrict__ in_deg, const int32_t* __restrict__ out_deg, int32_t V,
+                       int dgl_both, float* __restrict__ n_src, float* __restrict__ n_dst) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+    int32_t di = in_deg[v];
+    float nd = di > 0 ? 1.0f / sqrtf((float)di) : 0.0f;
+    n_dst[v] = nd;
+    if (dgl_both) {
+      int32_t d = out_deg[v];
+      n_src[v] = d > 0 ? 1.0f / sqrtf((float)d) : 0.0f;
+    } else {
+      n_src[v] = nd;
+    }
+  }
+}
+
+// node_ids sort keys: ascending (mask - deg) == descending degree; the stable
+// sort keeps ascending ids among equal degrees (reading C4).
+__global__ void k_deg_keys(const int32_t* __restrict__ deg, int32_t V, uint32_t mask, uint32_t* __restrict__ keys,
+                           int32_t* __restrict__ vals) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+    keys[v] = mask - (uint32_t)deg[v];
+    vals[v] = v;
+  }
+}
+
+// sched[0] = number of hub rows (deg > kHubChunk) = length of that prefix of ids.
+__global__ void k_sched_count(const int32_t* __restrict__ ids, const int32_t* __restrict__ deg, int32_t V,
+                              int64_t m, int32_t* __restrict__ sched) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= m; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t dprev = i == 0 ? INT32_MAX : deg[ids[i - 1]];
+    int32_t dcur = i >= V ? 0 : deg[ids[i]];
+    if (dprev > kHubChunk && dcur <= kHubChunk) sched[0] = (int32_t)i;
+  }
+}
+
+struct ChunkIn {
+  const int32_t* ids;
+  const int32_t* deg;
+  __device__ int64_t operator()(int64_t i) const {
+    int32_t d = deg[ids[i]];
+    return d > kHubChunk ? (d + kHubChunk - 1) / kHubChunk : 0;
+  }
+};
+struct StoreExcl32 {
+  int32_t* o;
+  __device__ void operator()(int64_t i, int64_t ex, int64_t) const { o[i] = (int32_t)ex; }
+};
+
+// shared edge labels: out_eid[j] = in-CSR position of out-edge j = (u -> v)
+__global__ void k_out_eid(const int32_t* __restrict__ out_row, const int32_t* __restrict__ out_col, int64_t E,
+                          const int32_t* __restrict__ in_rowptr, const int32_t* __restrict__ in_col,
+                          int32_t* __restrict__ out_eid) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < E; j += (int64_t)gridDim.x * blockDim.x) {
+    int32_t u = out_row[j], v = out_col[j];
+    int32_t lo = in_rowptr[v], hi = in_rowptr[v + 1];
+    while (lo < hi) {
+      int32_t mid = (lo + hi) >> 1;
+      if (in_col[mid] < u) lo = mid + 1; else hi = mid;
+    }
+    out_eid[j] = lo;
+  }
+}
+
+struct UniqIn {
+  const uint64_t* k;
+  __device__ int64_t operator()(int64_t i) const { return i == 0 || k[i] != k[i - 1]; }
+};
+struct UniqOut {
+  const uint64_t* k;
+  uint64_t* o;
+  __device__ void operator()(int64_t i, int64_t ex, int64_t f) const {
+    if (f) o[ex] = k[i];
+  }
+};
+
+stg_status sort_unique_keys(uint64_t** keys, uint64_t** alt, int64_t n, int nbits, int64_t* d_count, BuildWs& ws,
+                            cudaStream_t s) {
+  uint32_t* nov = nullptr;
+  STG_TRY((radix_sort<uint64_t, uint32_t>(keys, alt, nullptr, &nov, n, 0, nbits, ws.radix, s)));
+  STG_TRY(scan(UniqIn{*keys}, UniqOut{*keys, *alt}, n, ws.scan, s, d_count));
+  std::swap(*keys, *alt);
+  return STG_OK;
+}
+
+stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s) {
+  const int32_t V = g.V;
+  STG_TRY(ws.dkey.alloc(V)); STG_TRY(ws.dkey_alt.alloc(V));
+  STG_TRY(ws.dval_alt.alloc(V));
+  // degrees are bounded by V (edge sets have no multi-edges)
+  const int dbits = bits_for(V);
+  const uint32_t mask = (uint32_t)((uint64_t(1) << dbits) - 1);
+  const int64_t m = std::min<int64_t>(V, sched_cap(g.cap));
+  for (int dir = 0; dir < 2; ++dir) {
+    int32_t* deg = dir == 0 ? g.in_deg.p : g.out_deg.p;
+    int32_t* ids = dir == 0 ? g.in_ids.p : g.out_ids.p;
+    int32_t* sched = dir == 0 ? g.in_sched.p : g.out_sched.p;
+    uint32_t* k = ws.dkey.p; uint32_t* ka = ws.dkey_alt.p;
+    int32_t* vv = ids; int32_t* va = ws.dval_alt.p;
+    k_deg_keys<<<grid_for(V, 256), 256, 0, s>>>(deg, V, mask, k, vv);
+    count_launch();
+    STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, dbits, ws.radix, s)));
+    if (vv != ids) {
+      STG_CUDA(cudaMemcpyAsync(ids, vv, sizeof(int32_t) * V, cudaMemcpyDeviceToDevice, s));
+    }
+    k_sched_count<<<grid_for(m + 1, 256), 256, 0, s>>>(ids, deg, V, m, sched);
+    count_launch();
+    // chunk_ptr (exclusive) in sched[2..2+m], total chunks in sched[2+m] and sched[1]
+    STG_TRY(scan(ChunkIn{ids, deg}, StoreExcl32{sched + 2}, m, ws.scan, s, nullptr, sched + 2 + m));
+    STG_CUDA(cudaMemcpyAsync(sched + 1, sched + 2 + m, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
+  }
+  return check_launch("build_ids_and_sched");
+}
+
+stg_status build_out_eid(Snapshot& g, cudaStream_t s) {
+  if (!g.edge_ids) return STG_OK;
+  k_out_eid<<<grid_for(g.E, 256), 256, 0, s>>>(g.out_row.p, g.out_col.p, g.E, g.in_rowptr.p, g.in_col.p,
+                                              g.out_eid.p);
+  count_launch();
+  return check_launch("out_eid");
+}
+
+stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& g, BuildWs& ws, cudaStream_t s) {
+  const int32_t V = g.V;
+  g.E = E;
+  // backward CSR (rows = src): keys are already (src, dst)-sorted
+  k_unpack<<<grid_for(E, 256), 256, 0, s>>>(keys, E, g.nb, g.out_row.p, g.out_col.p);
+  k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.out_row.p, E, V, g.out_rowptr.p);
+  count_launch(2);
+  // forward CSR (rows = dst): re-key as (dst, src) and sort (the transpose)
+  STG_TRY(ws.kalt.alloc(2 * (size_t)(E > 0 ? E : 1)));
+  uint64_t* a = ws.kalt.p;
+  uint64_t* b = ws.kalt.p + (E > 0 ? E : 1);
+  k_swap_keys<<<grid_for(E, 256), 256, 0, s>>>(keys, E, g.nb, a);
+  count_launch();
+  uint32_t* nov = nullptr;
+  STG_TRY((radix_sort<uint64_t, uint32_t>(&a, &b, nullptr, &nov, E, 0, 2 * g.nb, ws.radix, s)));
+  k_unpack<<<grid_for(E, 256), 256, 0, s>>>(a, E, g.nb, g.in_row.p, g.in_col.p);
+  k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.in_row.p, E, V, g.in_rowptr.p);
+  k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.in_rowptr.p, V, g.in_deg.p);
+  k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.out_rowptr.p, V, g.out_deg.p);
+  k_norm<<<grid_for(V, 256), 256, 0, s>>>(g.in_deg.p, g.out_deg.p, V, g.dgl_both, g.norm_src.p, g.norm_dst.p);
+  count_launch(5);
+  STG_TRY(check_launch("build_from_out_keys"));
+  STG_TRY(build_ids_and_sched(g, ws, s));
+  return build_out_eid(g, s);
+}
+
+// -------------------------------------------------------------- delta apply
+// touch[row] = {add_lo, add_hi, del_lo, del_hi} into the sorted delta lists.
+__global__ void k_touch_mark(const uint64_t* __restrict__ d, int64_t n, int nb, int comp, int4* __restrict__ touch) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t r = (int32_t)(d[i] >> nb);
+    bool first = i == 0 || (int32_t)(d[i - 1] >> nb) != r;
+    bool last = i == n - 1 || (int32_t)(d[i + 1] >> nb) != r;
+    int* t = reinterpret_cast<int*>(touch + r);
+    if (first) t[2 * comp] = (int)i;
+    if (last) t[2 * comp + 1] = (int)(i + 1);
+  }
+}
+
+__global__ void k_touch_clear(const uint64_t* __restrict__ d, int64_t n, int nb, int4* __restrict__ touch) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    touch[(int32_t)(d[i] >> nb)] = make_int4(0, 0, 0, 0);
+}
+
+struct NewDegIn {
+  const int32_t* deg;
+  const int4* touch;
+  __device__ int64_t operator()(int64_t v) const {
+    int4 t = touch[v];
+    return deg[v] + (t.y - t.x) - (t.w - t.z);
+  }
+};
+struct RowptrOut {
+  int32_t* rowptr;
+  int32_t* deg;
+  __device__ void operator()(int64_t v, int64_t ex, int64_t d) const {
+    rowptr[v] = (int32_t)ex;
+    deg[v] = (int32_t)d;
+  }
+};
+
+__device__ __forceinline__ int64_t lb_keys(const uint64_t* a, int64_t lo, int64_t hi, uint64_t k) {
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (a[mid] < k) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// Surviving old edges move to new_rowptr[v] + i - (#dels < c) + (#adds < c).
+__global__ void k_merge_old(const int32_t* __restrict__ orow, const int32_t* __restrict__ ocol,
+                            const int32_t* __restrict__ orowptr, int64_t E_old,
+                            const int32_t* __restrict__ nrowptr, const int4* __restrict__ touch,
+                            const uint64_t* __restrict__ adds, const uint64_t* __restrict__ dels, int nb,
+                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < E_old; j += (int64_t)gridDim.x * blockDim.x) {
+    int32_t v = orow[j], c = ocol[j];
+    int4 t = touch[v];
+    int64_t pos = (int64_t)nrowptr[v] + (j - orowptr[v]);
+    if (t.y != t.x || t.w != t.z) {
+      uint64_t key = ((uint64_t)v << nb) | (uint64_t)c;
+      int64_t dl = lb_keys(dels, t.z, t.w, key);
+      if (dl < t.w && dels[dl] == key) continue;  // deleted
+      int64_t al = lb_keys(adds, t.x, t.y, key);
+      pos += (al - t.x) - (dl - t.z);
+    }
+    nrow[pos] = v;
+    ncol[pos] = c;
+  }
+}
+
+// Added edge a of row v lands at new_rowptr[v] + (a - add_lo) + (#old < c) - (#dels < c).
+__global__ void k_merge_add(const uint64_t* __restrict__ adds, int64_t nadd, const uint64_t* __restrict__ dels,
+                            int nb, const int32_t* __restrict__ ocol, const int32_t* __restrict__ orowptr,
+                            const int32_t* __restrict__ nrowptr, const int4* __restrict__ touch,
+                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol) {
+  const uint64_t mask = (uint64_t(1) << nb) - 1;
+  for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < nadd; a += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t key = adds[a];
+    int32_t v = (int32_t)(key >> nb), c = (int32_t)(key & mask);
+    int4 t = touch[v];
+    int32_t lo = orowptr[v], hi = orowptr[v + 1];
+    int32_t b = lo, e = hi;
+    while (b < e) {
+      int32_t mid = (b + e) >> 1;
+      if (ocol[mid] < c) b = mid + 1; else e = mid;
+    }
+    int64_t dl = lb_keys(dels, t.z, t.w, key);
+    int64_t pos = (int64_t)nrowptr[v] + (a - t.x) + (b - lo) - (dl - t.z);
+    nrow[pos] = v;
+    ncol[pos] = c;
+  }
+}
+
+static stg_status apply_dir(int32_t V, int nb, const int32_t* orow, const int32_t* ocol, const int32_t* orowptr,
+                            const int32_t* odeg, int64_t E_old, int32_t* nrow, int32_t* ncol, int32_t* nrowptr,
+                            int32_t* ndeg, const DirDelta& d, int4* touch, BuildWs& ws, cudaStream_t s) {
+  if (d.nadd) { k_touch_mark<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, nb, 0, touch); count_launch(); }
+  if (d.ndel) { k_touch_mark<<<grid_for(d.ndel, 256), 256, 0, s>>>(d.del, d.ndel, nb, 1, touch); count_launch(); }
+  STG_TRY(scan(NewDegIn{odeg, touch}, RowptrOut{nrowptr, ndeg}, V, ws.scan, s, nullptr, nrowptr + V));
+  if (E_old) {
+    k_merge_old<<<grid_for(E_old, 256), 256, 0, s>>>(orow, ocol, orowptr, E_old, nrowptr, touch, d.add, d.del, nb,
+                                                    nrow, ncol);
+    count_launch();
+  }
+  if (d.nadd) {
+    k_merge_add<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, d.del, nb, ocol, orowptr, nrowptr, touch, nrow,
+                                                     ncol);
+    count_launch();
+  }
+  if (d.nadd) { k_touch_clear<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, nb, touch); count_launch(); }
+  if (d.ndel) { k_touch_clear<<<grid_for(d.ndel, 256), 256, 0, s>>>(d.del, d.ndel, nb, touch); count_launch(); }
+  return check_launch("apply_dir");
+}
+
+stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
+                       int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws, cudaStream_t s) {
+  const int32_t V = src.V;
+  STG_TRY(apply_dir(V, src.nb, src.in_row.p, src.in_col.p, src.in_rowptr.p, src.in_deg.p, src.E, dst.in_row.p,
+                    dst.in_col.p, dst.in_rowptr.p, dst.in_deg.p, in_dir, touch_in, ws, s));
+  STG_TRY(apply_dir(V, src.nb, src.out_row.p, src.out_col.p, src.out_rowptr.p, src.out_deg.p, src.E,
+                    dst.out_row.p, dst.out_col.p, dst.out_rowptr.p, dst.out_deg.p, out_dir, touch_out, ws, s));
+  dst.E = E_new;
+  dst.t = t_new;
+  k_norm<<<grid_for(V, 256), 256, 0, s>>>(dst.in_deg.p, dst.out_deg.p, V, dst.dgl_both, dst.norm_src.p,
+                                         dst.norm_dst.p);
+  count_launch();
+  STG_TRY(build_ids_and_sched(dst, ws, s));
+  return build_out_eid(dst, s);
+}
+
+// ------------------------------------------------------------ static graph
+__global__ void k_validate_pack(const int32_t* __restrict__ src, const int32_t* __restrict__ dst, int64_t E,
+                                int32_t V, int nb, int loops, uint64_t* __restrict__ keys, int32_t* __restrict__ bad) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E + (loops ? V : 0);
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t a, b;
+    if (i < E) { a = src[i]; b = dst[i]; }
+    else { a = b = (int32_t)(i - E); }
+    if ((unsigned)a >= (unsigned)V || (unsigned)b >= (unsigned)V) { atomicExch(bad, 1); a = b = 0; }
+    keys[i] = ((uint64_t)a << nb) | (uint64_t)b;
+  }
+}
+
+}  // namespace stg
+
+using namespace stg;
+
+extern "C" {
+
+stg_status stg_static_graph_create(int32_t V, int64_t E, const int32_t* src, const int32_t* dst, uint32_t flags,
+                                   const stg_dist* dist, stg_stream_t stream, stg_graph** out) {
+  if (!out) return fail(STG_ERR_INVALID_ARG, "stg_static_graph_create: out is NULL");
+  *out = nullptr;
+  if (V < 1 || V >= (1 << 30)) return fail(STG_ERR_OUT_OF_RANGE, "stg_static_graph_create: V=%d outside [1,2^30)", V);
+  if (E < 0) return fail(STG_ERR_INVALID_ARG, "stg_static_graph_create: E < 0");
+  if (E + ((flags & STG_SELF_LOOPS) ? V : 0) >= (int64_t(1) << 31))
+    return fail(STG_ERR_OUT_OF_RANGE, "stg_static_graph_create: E=%lld >= 2^31", (long long)E);
+  if (E > 0 && (!src || !dst)) return fail(STG_ERR_INVALID_ARG, "stg_static_graph_create: src/dst NULL");
+  if (dist) return fail(STG_ERR_INVALID_ARG, "stg_static_graph_create: row-block sharding is not implemented for static graphs");
+  cudaStream_t s = (cudaStream_t)stream;
+  auto* g = new stg_graph();
+  BuildWs ws;
+  const int loops = (flags & STG_SELF_LOOPS) ? 1 : 0;
+  const int64_t n = E + (loops ? V : 0);
+  Snapshot& sn = g->snap;
+  stg_status st = sn.alloc(V, n, (flags & STG_EDGE_IDS) != 0, (flags & STG_NORM_DGL_BOTH) != 0);
+  DArray<uint64_t> k1, k2;
+  DArray<int32_t> bad;
+  DArray<int64_t> cnt;
+  if (st == STG_OK) st = k1.alloc(n);
+  if (st == STG_OK) st = k2.alloc(n);
+  if (st == STG_OK) st = bad.alloc(1);
+  if (st == STG_OK) st = cnt.alloc(1);
+  int32_t hbad = 0;
+  int64_t E2 = 0;
+  if (st == STG_OK) {
+    sn.t = -1;
+    cudaMemsetAsync(bad.p, 0, sizeof(int32_t), s);
+    k_validate_pack<<<grid_for(n, 256), 256, 0, s>>>(src, dst, E, V, sn.nb, loops, k1.p, bad.p);
+    count_launch();
+    uint64_t* a = k1.p; uint64_t* b = k2.p;
+    st = sort_unique_keys(&a, &b, n, 2 * sn.nb, cnt.p, ws, s);
+    if (st == STG_OK) {
+      if (cudaMemcpyAsync(&hbad, bad.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+          cudaMemcpyAsync(&E2, cnt.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+          cudaStreamSynchronize(s) != cudaSuccess)
+        st = fail(STG_ERR_CUDA, "stg_static_graph_create: %s", cudaGetErrorString(cudaGetLastError()));
+    }
+    if (st == STG_OK && hbad) st = fail(STG_ERR_OUT_OF_RANGE, "stg_static_graph_create: vertex id outside [0,%d)", V);
+    if (st == STG_OK) st = build_from_out_keys(a, E2, sn, ws, s);
+    if (st == STG_OK && cudaStreamSynchronize(s) != cudaSuccess)
+      st = fail(STG_ERR_CUDA, "stg_static_graph_create: %s", cudaGetErrorString(cudaGetLastError()));
+  }
+  if (st != STG_OK) { delete g; return st; }
+  *out = g;
+  return STG_OK;
+}
+
+stg_status stg_graph_view(const stg_graph* g, stg_csr_view* out) {
+  if (!g || !out) return fail(STG_ERR_INVALID_ARG, "stg_graph_view: NULL argument");
+  g->snap.view(out, const_cast<AggWs*>(&g->ws));
+  return STG_OK;
+}
+
+void stg_graph_destroy(stg_graph* g) {
+  if (g) cudaDeviceSynchronize();
+  delete g;
+}
+
+}  // extern "C"
+
+namespace stg {
+// bounds[k] = first row r with rowptr[r] >= k·E/world (nnz-balanced blocks).
+__global__ void k_partition(const int32_t* __restrict__ rowptr, int32_t V, int32_t world, int32_t* __restrict__ b) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k > world) return;
+  if (k == 0) { b[0] = 0; return; }
+  if (k == world) { b[world] = V; return; }
+  const int64_t E = rowptr[V];
+  const int64_t target = (E * k + world - 1) / world;
+  int32_t lo = 0, hi = V;
+  while (lo < hi) {
+    int32_t mid = (lo + hi) >> 1;
+    if (rowptr[mid] < target) lo = mid + 1; else hi = mid;
+  }
+  b[k] = lo;
+}
+}  // namespace stg
+
+extern "C" stg_status stg_partition_rows(int32_t V, const int32_t* in_rowptr, int32_t world, int32_t* bounds,
+                                         stg_stream_t stream) {
+  using namespace stg;
+  if (V < 1 || world < 1 || !in_rowptr || !bounds) return fail(STG_ERR_INVALID_ARG, "stg_partition_rows: bad arguments");
+  cudaStream_t s = (cudaStream_t)stream;
+  DArray<int32_t> d;
+  STG_TRY(d.alloc(world + 1));
+  k_partition<<<(world + 128) / 128, 128, 0, s>>>(in_rowptr, V, world, d.p);
+  count_launch();
+  STG_CUDA(cudaMemcpyAsync(bounds, d.p, sizeof(int32_t) * (world + 1), cudaMemcpyDeviceToHost, s));
+  STG_CUDA(cudaStreamSynchronize(s));
+  // blocks must be non-decreasing; enforce (equal bounds = empty block)
+  for (int k = 1; k <= world; ++k)
+    if (bounds[k] < bounds[k - 1]) bounds[k] = bounds[k - 1];
+  return STG_OK;
+}

@@ -1,0 +1,77 @@
+// graph.cuh — device-resident snapshot (the STGraphBase arrays)
+// and the builders shared by static graphs and DTDG snapshots.
+#pragma once
+
+#include "common.cuh"
+
+namespace stg {
+
+// Rows with more than kHubChunk in-edges are split into chunks of kHubChunk
+// edges (degree-bucketed schedule); each light row / hub chunk is
+// one work item of the aggregation kernel.  128 keeps every fp32 accumulator
+// chain <= 64 terms.
+constexpr int32_t kHubChunk = 128;
+
+inline int64_t sched_cap(int64_t E) { return E / (kHubChunk + 1) + 2; }
+
+// Aggregation scratch owned by a graph / dtdg object: hub-chunk partial sums
+// and per-hub-row completion counters (self-resetting, zero between calls).
+struct AggWs {
+  DArray<float> partials;
+  DArray<int32_t> counters;
+  int64_t counters_n = 0;
+};
+
+struct Snapshot {
+  int32_t V = 0, nb = 1;   // nb: bits per id in packed keys
+  int32_t t = -1;
+  int64_t E = 0, cap = 0;  // current edges, edge capacity
+  bool edge_ids = false, dgl_both = false;
+  DArray<int32_t> in_rowptr, in_col, in_row, in_deg, in_ids;
+  DArray<int32_t> out_rowptr, out_col, out_row, out_deg, out_ids, out_eid;
+  DArray<int32_t> in_sched, out_sched;  // [2 + sched_cap(cap) + 1]
+  DArray<float> norm_src, norm_dst;
+
+  stg_status alloc(int32_t V_, int64_t cap_, bool eids, bool dgl);
+  void view(stg_csr_view* v, AggWs* ws) const;
+};
+
+// Shared builder scratch (radix sort / scan buffers), grow-only.
+struct BuildWs;
+BuildWs* buildws_create();
+void buildws_destroy(BuildWs*);
+
+// Build every array of `out` from the sorted unique packed out-keys
+// (src << nb | dst) of the snapshot edge set.  No host synchronisation.
+stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& out, BuildWs& ws, cudaStream_t s);
+
+// Sort + unique packed keys in place.  keys/alt hold n entries; on return
+// *keys points to the sorted unique keys; the unique count is written to
+// *d_count (device).  Does not synchronise.
+stg_status sort_unique_keys(uint64_t** keys, uint64_t** alt, int64_t n, int nbits, int64_t* d_count,
+                            BuildWs& ws, cudaStream_t s);
+
+// Recompute degrees' dependents: node_ids (both directions) and the hub
+// schedules.  Needs deg arrays and rowptrs set.
+stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s);
+stg_status build_out_eid(Snapshot& g, cudaStream_t s);
+
+// Delta application (DTDG Get-Graph / Get-Backward-Graph step).  For one
+// direction: the sorted packed deltas (row << nb | col) of that direction.
+struct DirDelta {
+  const uint64_t* add;
+  int64_t nadd;
+  const uint64_t* del;
+  int64_t ndel;
+};
+stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
+                       int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws,
+                       cudaStream_t s);
+
+}  // namespace stg
+
+// Opaque objects of the C ABI.
+struct stg_graph {
+  stg::Snapshot snap;
+  stg::AggWs ws;
+};

@@ -1,0 +1,672 @@
+// tgcn.cu — TGCN step (GCN + GRU, readings C13-C15), State Stack,
+// surrogate MSE head, SGD, and Algorithm 1's per-sequence driver.
+//
+// Per timestamp (a7):  P' = diag(n_src)·X·W   (k_xw, row-scale epilogue)
+//                      C  = diag(n_dst)·A·P' + b  (aggregation kernel, bias epilogue)
+//                      Z, R, Ĥ, H'               (k_gru_fwd, fused)
+// Backward (a8):       k_gru_bwd (recompute gates, chain rule, dC' = n_dst⊙dC,
+//                      per-block parameter-gradient partials) → aggregation over
+//                      the out-CSR (dP) → k_dw (Xᵀ·dP partials) → fixed-order
+//                      reduction.  No float atomics: deterministic run to run.
+#include <algorithm>
+#include <mutex>
+#include <vector>
+
+#include "graph.cuh"
+
+namespace stg {
+stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
+                            float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
+                            cudaStream_t s);
+}
+
+namespace stg {
+namespace {
+
+constexpr int kT = 256;  // threads per block for the TGCN kernels
+
+__device__ __forceinline__ float sigm(float a) { return 1.0f / (1.0f + expf(-a)); }
+
+// ---------------------------------------------------------------- P' = n ⊙ XW
+// Row tile of 32 rows; W [F, N] and the X tile live in shared memory.
+__global__ void __launch_bounds__(kT) k_xw(int32_t V, int32_t F, int32_t N, const float* __restrict__ X,
+                                           const float* __restrict__ W, const float* __restrict__ rs,
+                                           float* __restrict__ P) {
+  extern __shared__ float sm[];
+  float* sW = sm;                 // [F][N]
+  float* sX = sm + F * N;         // [32][F]
+  constexpr int BR = 32;
+  for (int i = threadIdx.x; i < F * N; i += kT) sW[i] = W[i];
+  const int64_t ntiles = (V + BR - 1) / BR;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * BR;
+    __syncthreads();
+    for (int i = threadIdx.x; i < BR * F; i += kT) {
+      int64_t r = r0 + i / F;
+      sX[i] = r < V ? X[r * F + i % F] : 0.0f;
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < BR * N; o += kT) {
+      const int r = o / N, c = o % N;
+      if (r0 + r >= V) continue;
+      const float* xr = sX + r * F;
+      float acc = 0.0f;
+      for (int f = 0; f < F; ++f) acc = fmaf(xr[f], sW[f * N + c], acc);
+      P[(r0 + r) * N + c] = rs ? rs[r0 + r] * acc : acc;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- GRU forward
+// Row tile of BR rows.  smem: L [3][2H][H], l [3][H], C [BR][3H], H [BR][H],
+// Z, R, RH [BR][H].
+template <int BR>
+__global__ void __launch_bounds__(kT) k_gru_fwd(int32_t V, int32_t H, const float* __restrict__ C,
+                                                const float* __restrict__ Hp, const float* __restrict__ L,
+                                                const float* __restrict__ l, float* __restrict__ Hn) {
+  extern __shared__ float sm[];
+  const int H3 = 3 * H, LG = 2 * H * H;
+  float* sL = sm;
+  float* sl = sL + 3 * LG;
+  float* sC = sl + H3;
+  float* sH = sC + BR * H3;
+  float* sZ = sH + BR * H;
+  float* sR = sZ + BR * H;
+  float* sRH = sR + BR * H;
+  for (int i = threadIdx.x; i < 3 * LG; i += kT) sL[i] = L[i];
+  for (int i = threadIdx.x; i < H3; i += kT) sl[i] = l[i];
+  const float* Lz = sL; const float* Lr = sL + LG; const float* Lh = sL + 2 * LG;
+  const int64_t ntiles = (V + BR - 1) / BR;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * BR;
+    __syncthreads();
+    for (int i = threadIdx.x; i < BR * H3; i += kT) {
+      int64_t r = r0 + i / H3;
+      sC[i] = r < V ? C[r * H3 + i % H3] : 0.0f;
+    }
+    for (int i = threadIdx.x; i < BR * H; i += kT) {
+      int64_t r = r0 + i / H;
+      sH[i] = r < V ? Hp[r * H + i % H] : 0.0f;
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < BR * H; o += kT) {
+      const int r = o / H, j = o % H;
+      const float* cz = sC + r * H3; const float* cr = cz + H; const float* hv = sH + r * H;
+      float az = sl[j], ar = sl[H + j];
+      for (int i = 0; i < H; ++i) {
+        az = fmaf(cz[i], Lz[i * H + j], az);
+        az = fmaf(hv[i], Lz[(H + i) * H + j], az);
+        ar = fmaf(cr[i], Lr[i * H + j], ar);
+        ar = fmaf(hv[i], Lr[(H + i) * H + j], ar);
+      }
+      const float z = sigm(az), rr = sigm(ar);
+      sZ[o] = z; sR[o] = rr; sRH[o] = rr * hv[j];
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < BR * H; o += kT) {
+      const int r = o / H, j = o % H;
+      if (r0 + r >= V) continue;
+      const float* ch = sC + r * H3 + 2 * H; const float* rh = sRH + r * H;
+      float ah = sl[2 * H + j];
+      for (int i = 0; i < H; ++i) {
+        ah = fmaf(ch[i], Lh[i * H + j], ah);
+        ah = fmaf(rh[i], Lh[(H + i) * H + j], ah);
+      }
+      const float hh = tanhf(ah), z = sZ[o];
+      Hn[(r0 + r) * H + j] = z * sH[o] + (1.0f - z) * hh;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- GRU backward
+// Recomputes Z, R, Ĥ from {C, H} (A8), applies the chain rule,
+// writes dC' = n_dst ⊙ dC and dH_prev, and accumulates per-block partials of
+// [dL (6H²) | dl (3H) | db (3H)] in a fixed row order.
+template <int BR>
+__global__ void __launch_bounds__(kT) k_gru_bwd(int32_t V, int32_t H, const float* __restrict__ C,
+                                                const float* __restrict__ Hp, const float* __restrict__ G,
+                                                const float* __restrict__ L, const float* __restrict__ l,
+                                                const float* __restrict__ ndst, float* __restrict__ dCs,
+                                                float* __restrict__ dHp, float* __restrict__ part) {
+  extern __shared__ float sm[];
+  const int H3 = 3 * H, LG = 2 * H * H, HH = H * H;
+  const int NP = 6 * HH + 6 * H;     // partial layout: dL[3][2H][H], dl[3][H], db[3H]
+  float* sL = sm;
+  float* sl = sL + 3 * LG;
+  float* sC = sl + H3;
+  float* sH = sC + BR * H3;
+  float* sG = sH + BR * H;
+  float* sZ = sG + BR * H;
+  float* sR = sZ + BR * H;
+  float* sHh = sR + BR * H;
+  float* sdaz = sHh + BR * H;
+  float* sdar = sdaz + BR * H;
+  float* sdah = sdar + BR * H;
+  float* sdC = sdah + BR * H;        // [BR][3H] unscaled dC
+  float* sAcc = sdC + BR * H3;       // [NP]
+  for (int i = threadIdx.x; i < 3 * LG; i += kT) sL[i] = L[i];
+  for (int i = threadIdx.x; i < H3; i += kT) sl[i] = l[i];
+  for (int i = threadIdx.x; i < NP; i += kT) sAcc[i] = 0.0f;
+  const float* Lz = sL; const float* Lr = sL + LG; const float* Lh = sL + 2 * LG;
+  const int64_t ntiles = (V + BR - 1) / BR;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * BR;
+    __syncthreads();
+    for (int i = threadIdx.x; i < BR * H3; i += kT) {
+      int64_t r = r0 + i / H3;
+      sC[i] = r < V ? C[r * H3 + i % H3] : 0.0f;
+    }
+    for (int i = threadIdx.x; i < BR * H; i += kT) {
+      int64_t r = r0 + i / H;
+      sH[i] = r < V ? Hp[r * H + i % H] : 0.0f;
+      sG[i] = r < V ? G[r * H + i % H] : 0.0f;
+    }
+    __syncthreads();
+    // gates (identical arithmetic to k_gru_fwd)
+    for (int o = threadIdx.x; o < BR * H; o += kT) {
+      const int r = o / H, j = o % H;
+      const float* cz = sC + r * H3; const float* cr = cz + H; const float* hv = sH + r * H;
+      float az = sl[j], ar = sl[H + j];
+      for (int i = 0; i < H; ++i) {
+        az = fmaf(cz[i], Lz[i * H + j], az);
+        az = fmaf(hv[i], Lz[(H + i) * H + j], az);
+        ar = fmaf(cr[i], Lr[i * H + j], ar);
+        ar = fmaf(hv[i], Lr[(H + i) * H + j], ar);
+      }
+      sZ[o] = sigm(az); sR[o] = sigm(ar);
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < BR * H; o += kT) {
+      const int r = o / H, j = o % H;
+      const float* ch = sC + r * H3 + 2 * H; const float* hv = sH + r * H; const float* rr = sR + r * H;
+      float ah = sl[2 * H + j];
+      for (int i = 0; i < H; ++i) {
+        ah = fmaf(ch[i], Lh[i * H + j], ah);
+        ah = fmaf(rr[i] * hv[i], Lh[(H + i) * H + j], ah);
+      }
+      const float hh = tanhf(ah);
+      sHh[o] = hh;
+      const float g = sG[o], z = sZ[o];
+      const float dZ = g * (hv[j] - hh), dHh = g * (1.0f - z);
+      sdah[o] = dHh * (1.0f - hh * hh);
+      sdaz[o] = dZ * z * (1.0f - z);
+    }
+    __syncthreads();
+    // dC_h, dRH -> dR -> da_r ; dH accumulates in sG (reused as dH after G is consumed)
+    for (int o = threadIdx.x; o < BR * H; o += kT) {
+      const int r = o / H, i = o % H;
+      const float* dah = sdah + r * H;
+      float s1 = 0.0f, s2 = 0.0f;
+      for (int j = 0; j < H; ++j) {
+        s1 = fmaf(dah[j], Lh[i * H + j], s1);
+        s2 = fmaf(dah[j], Lh[(H + i) * H + j], s2);
+      }
+      sdC[r * H3 + 2 * H + i] = s1;
+      const float rr = sR[o], hv = sH[o];
+      sdar[o] = s2 * hv * rr * (1.0f - rr);
+      sHh[o] = s2 * rr;             // dH contribution through R⊙H (Ĥ no longer needed)
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < BR * H; o += kT) {
+      const int r = o / H, i = o % H;
+      const float* dar = sdar + r * H; const float* daz = sdaz + r * H;
+      float sr1 = 0.0f, sr2 = 0.0f, sz1 = 0.0f, sz2 = 0.0f;
+      for (int j = 0; j < H; ++j) {
+        sr1 = fmaf(dar[j], Lr[i * H + j], sr1);
+        sr2 = fmaf(dar[j], Lr[(H + i) * H + j], sr2);
+        sz1 = fmaf(daz[j], Lz[i * H + j], sz1);
+        sz2 = fmaf(daz[j], Lz[(H + i) * H + j], sz2);
+      }
+      sdC[r * H3 + H + i] = sr1;
+      sdC[r * H3 + i] = sz1;
+      const int64_t row = r0 + r;
+      if (row < V) dHp[row * H + i] = sG[o] * sZ[o] + sHh[o] + (sr2 + sz2);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < BR * H3; i += kT) {
+      int64_t r = r0 + i / H3;
+      if (r < V) dCs[r * H3 + i % H3] = ndst[r] * sdC[i];
+    }
+    // parameter-gradient partials (each entry owned by one thread; rows in order)
+    const int nrows = (int)(V - r0 < BR ? V - r0 : BR);
+    for (int e = threadIdx.x; e < NP; e += kT) {
+      float acc = sAcc[e];
+      if (e < 6 * HH) {
+        const int g = e / LG, rem = e % LG, i = rem / H, j = rem % H;
+        const float* da = g == 0 ? sdaz : (g == 1 ? sdar : sdah);
+        for (int r = 0; r < nrows; ++r) {
+          float a;
+          if (i < H) a = sC[r * H3 + g * H + i];
+          else a = (g == 2) ? sR[r * H + (i - H)] * sH[r * H + (i - H)] : sH[r * H + (i - H)];
+          acc = fmaf(a, da[r * H + j], acc);
+        }
+      } else if (e < 6 * HH + 3 * H) {
+        const int g = (e - 6 * HH) / H, j = (e - 6 * HH) % H;
+        const float* da = g == 0 ? sdaz : (g == 1 ? sdar : sdah);
+        for (int r = 0; r < nrows; ++r) acc += da[r * H + j];
+      } else {
+        const int c = e - 6 * HH - 3 * H;
+        for (int r = 0; r < nrows; ++r) acc += sdC[r * H3 + c];
+      }
+      sAcc[e] = acc;
+    }
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < NP; e += kT) part[(int64_t)blockIdx.x * NP + e] = sAcc[e];
+}
+
+// ---------------------------------------------------------------- dW partials
+// dW[f,c] += Σ_v X[v,f]·dP[v,c]; block-private accumulators, rows in order.
+__global__ void __launch_bounds__(kT) k_dw(int32_t V, int32_t F, int32_t N, const float* __restrict__ X,
+                                           const float* __restrict__ dP, float* __restrict__ part) {
+  extern __shared__ float sm[];
+  constexpr int BR = 32;
+  float* sX = sm;              // [BR][F]
+  float* sD = sX + BR * F;     // [BR][N]
+  float* sAcc = sD + BR * N;   // [F][N]
+  for (int i = threadIdx.x; i < F * N; i += kT) sAcc[i] = 0.0f;
+  const int64_t ntiles = (V + BR - 1) / BR;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * BR;
+    __syncthreads();
+    for (int i = threadIdx.x; i < BR * F; i += kT) {
+      int64_t r = r0 + i / F;
+      sX[i] = r < V ? X[r * F + i % F] : 0.0f;
+    }
+    for (int i = threadIdx.x; i < BR * N; i += kT) {
+      int64_t r = r0 + i / N;
+      sD[i] = r < V ? dP[r * N + i % N] : 0.0f;
+    }
+    __syncthreads();
+    const int nrows = (int)(V - r0 < BR ? V - r0 : BR);
+    for (int e = threadIdx.x; e < F * N; e += kT) {
+      const int f = e / N, c = e % N;
+      float acc = sAcc[e];
+      for (int r = 0; r < nrows; ++r) acc = fmaf(sX[r * F + f], sD[r * N + c], acc);
+      sAcc[e] = acc;
+    }
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < F * N; e += kT) part[(int64_t)blockIdx.x * F * N + e] = sAcc[e];
+}
+
+// out[e] += Σ_b part[b][e], blocks of 16 summed first (fixed order).
+__global__ void k_reduce_part(const float* __restrict__ part, int32_t nb, int32_t n, float* __restrict__ out0,
+                              int32_t n0, float* __restrict__ out1, int32_t n1, float* __restrict__ out2) {
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
+    float tot = 0.0f;
+    for (int b0 = 0; b0 < nb; b0 += 16) {
+      float blk = 0.0f;
+      const int b1 = min(b0 + 16, nb);
+      for (int b = b0; b < b1; ++b) blk += part[(int64_t)b * n + e];
+      tot += blk;
+    }
+    if (e < n0) out0[e] += tot;
+    else if (e < n0 + n1) out1[e - n0] += tot;
+    else out2[e - n0 - n1] += tot;
+  }
+}
+
+// ---------------------------------------------------------------- MSE head
+// One warp per row.  Per-block partials [loss | dw_o (H) | db_o] (fp32 for the
+// gradients, fp64 for the loss).
+__global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t H, const float* __restrict__ Hn,
+                                                 const float* __restrict__ y, const float* __restrict__ w_o,
+                                                 const float* __restrict__ b_o, float* __restrict__ dH, int accumulate,
+                                                 int want_grad, double* __restrict__ lpart,
+                                                 float* __restrict__ gpart) {
+  __shared__ double sl[kT / 32];
+  __shared__ float sg[kT / 32][65];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  double lacc = 0.0;
+  float gw0 = 0.0f, gw1 = 0.0f, gb = 0.0f;     // lane owns k = lane and lane + 32
+  const float b = b_o[0];
+  const float invV = 1.0f / (float)V;
+  for (int64_t v = (int64_t)blockIdx.x * (kT / 32) + w; v < V; v += (int64_t)gridDim.x * (kT / 32)) {
+    const float* h = Hn + v * H;
+    float h0 = lane < H ? h[lane] : 0.0f, h1 = lane + 32 < H ? h[lane + 32] : 0.0f;
+    float r0 = fmaxf(h0, 0.0f), r1 = fmaxf(h1, 0.0f);
+    float s = (lane < H ? r0 * w_o[lane] : 0.0f) + (lane + 32 < H ? r1 * w_o[lane + 32] : 0.0f);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float e = (s + b) - y[v];
+    lacc += (double)e * (double)e;
+    if (want_grad) {
+      const float g = 2.0f * e * invV;
+      if (dH) {
+        if (lane < H) {
+          float d = h0 > 0.0f ? g * w_o[lane] : 0.0f;
+          dH[v * H + lane] = accumulate ? dH[v * H + lane] + d : d;
+        }
+        if (lane + 32 < H) {
+          float d = h1 > 0.0f ? g * w_o[lane + 32] : 0.0f;
+          dH[v * H + lane + 32] = accumulate ? dH[v * H + lane + 32] + d : d;
+        }
+      }
+      gw0 = fmaf(g, r0, gw0);
+      gw1 = fmaf(g, r1, gw1);
+      gb += g;
+    }
+  }
+  if (lane == 0) sl[w] = lacc;
+  sg[w][lane] = gw0;
+  sg[w][lane + 32] = gw1;
+  if (lane == 0) sg[w][64] = gb;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int i = 0; i < kT / 32; ++i) t += sl[i];
+    lpart[blockIdx.x] = t;
+  }
+  for (int k = threadIdx.x; k < H + 1; k += kT) {
+    float t = 0.0f;
+    const int src = k < H ? k : 64;
+    for (int i = 0; i < kT / 32; ++i) t += sg[i][src];
+    gpart[(int64_t)blockIdx.x * (H + 1) + k] = t;
+  }
+}
+
+__global__ void k_mse_reduce(int32_t nb, int32_t H, int32_t V, const double* __restrict__ lpart,
+                             const float* __restrict__ gpart, float* __restrict__ loss, float* __restrict__ dw_o,
+                             float* __restrict__ db_o) {
+  if (blockIdx.x == 0 && threadIdx.x == 0 && loss) {
+    double t = 0.0;
+    for (int b = 0; b < nb; ++b) t += lpart[b];
+    *loss += (float)(t / (double)V);
+  }
+  for (int k = threadIdx.x; k < H + 1; k += blockDim.x) {
+    float t = 0.0f;
+    for (int b = 0; b < nb; ++b) t += gpart[(int64_t)b * (H + 1) + k];
+    if (k < H) { if (dw_o) dw_o[k] += t; }
+    else if (db_o) db_o[0] += t;
+  }
+}
+
+__global__ void k_sgd(float* __restrict__ p, const float* __restrict__ g, int64_t n, float lr) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] -= lr * g[i];
+}
+
+int grid_blocks(const void* fn, size_t smem, int64_t tiles) {
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kT, smem) != cudaSuccess || per_sm < 1) {
+    cudaGetLastError();
+    per_sm = 1;
+  }
+  int64_t b = (int64_t)per_sm * num_sms();
+  if (tiles < b) b = tiles;
+  return (int)(b < 1 ? 1 : b);
+}
+
+template <class K>
+stg_status set_smem(K fn, size_t smem) {
+  if (smem > 48 * 1024) STG_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  return STG_OK;
+}
+
+}  // namespace
+
+// Scratch used by the TGCN kernels (grow-only).
+struct TgcnWs {
+  DArray<float> P, dC, dP, part_gru, part_dw, gpart;
+  DArray<double> lpart;
+};
+
+}  // namespace stg
+
+using namespace stg;
+
+struct StackEntry {
+  const float* Hp;
+  float* C;
+  int32_t V, H;
+  size_t bytes;
+};
+
+struct stg_state_stack {
+  DArray<unsigned char> arena;
+  size_t cap = 0, top = 0;
+  std::vector<StackEntry> entries;
+  TgcnWs ws;
+};
+
+static TgcnWs& global_ws() {
+  static TgcnWs ws;
+  return ws;
+}
+
+static stg_status check_params(const stg_tgcn_params* p) {
+  if (!p || !p->W || !p->b || !p->L || !p->l) return fail(STG_ERR_INVALID_ARG, "tgcn: NULL parameter pointer");
+  if (p->F < 1 || p->H < 1) return fail(STG_ERR_INVALID_ARG, "tgcn: F=%d H=%d must be >= 1", p->F, p->H);
+  if (p->H > 64) return fail(STG_ERR_INVALID_ARG, "tgcn: H=%d > 64 is not supported", p->H);
+  if ((size_t)p->F * 3 * p->H * 4 + 32 * p->F * 4 > 200 * 1024)
+    return fail(STG_ERR_INVALID_ARG, "tgcn: F=%d too large for the resident-weight kernel", p->F);
+  return STG_OK;
+}
+
+static size_t gru_fwd_smem(int H, int BR) { return sizeof(float) * (6 * H * H + 3 * H + BR * 3 * H + 4 * BR * H); }
+static size_t gru_bwd_smem(int H, int BR) {
+  return sizeof(float) * (6 * H * H + 3 * H + BR * 3 * H + 8 * BR * H + BR * 3 * H + 6 * H * H + 6 * H);
+}
+
+extern "C" {
+
+stg_status stg_state_stack_create(int64_t capacity_bytes, stg_state_stack** out) {
+  if (!out || capacity_bytes < 0) return fail(STG_ERR_INVALID_ARG, "stg_state_stack_create: bad arguments");
+  auto* s = new stg_state_stack();
+  s->cap = (size_t)capacity_bytes;
+  if (s->cap) {
+    stg_status st = s->arena.alloc(s->cap);
+    if (st != STG_OK) { delete s; return st; }
+  }
+  *out = s;
+  return STG_OK;
+}
+
+int32_t stg_state_stack_depth(const stg_state_stack* s) { return s ? (int32_t)s->entries.size() : -1; }
+
+void stg_state_stack_destroy(stg_state_stack* s) {
+  if (s) cudaDeviceSynchronize();
+  delete s;
+}
+
+stg_status stg_tgcn_step(const stg_csr_view* g, const stg_tgcn_params* p, const float* X, const float* H_prev,
+                         float* H_next, stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_params(p));
+  if (!g || !X || !H_prev || !H_next) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step: NULL argument");
+  if (g->row_begin != 0 || g->row_end != g->num_nodes)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step: sharded views are driven from Python (DESIGN.md §Multi-GPU)");
+  cudaStream_t s = (cudaStream_t)stream;
+  const int32_t V = g->num_nodes, F = p->F, H = p->H, H3 = 3 * H;
+  TgcnWs& ws = stack ? stack->ws : global_ws();
+  STG_TRY(ws.P.alloc((size_t)V * H3));
+  float* C = nullptr;
+  const size_t cbytes = sizeof(float) * (size_t)V * H3;
+  if (stack) {
+    const size_t need = (cbytes + 255) & ~size_t(255);
+    if (stack->top + need > stack->cap)
+      return fail(STG_ERR_NO_MEMORY, "stg_tgcn_step: state stack full (%zu + %zu > %zu bytes)", stack->top, need,
+                  stack->cap);
+    C = reinterpret_cast<float*>(stack->arena.p + stack->top);
+  } else {
+    STG_TRY(ws.dC.alloc((size_t)V * H3));
+    C = ws.dC.p;
+  }
+  // P' = diag(n_src)·X·W
+  {
+    ProfScope prof(PH_XW, s);
+    const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
+    STG_TRY(set_smem(k_xw, smem));
+    const int nb = grid_blocks((const void*)k_xw, smem, (V + 31) / 32);
+    k_xw<<<nb, kT, smem, s>>>(V, F, H3, X, p->W, g->norm_src, ws.P.p);
+    count_launch();
+  }
+  // C = diag(n_dst)·A·P' + b
+  STG_TRY(aggregate_launch(g, 0, H3, ws.P.p, H3, C, H3, g->norm_dst, nullptr, p->b, s));
+  // GRU
+  ProfScope prof_gru(PH_GRU_FWD, s);
+  if (H <= 32) {
+    const size_t smem = gru_fwd_smem(H, 32);
+    STG_TRY(set_smem(k_gru_fwd<32>, smem));
+    const int nb = grid_blocks((const void*)k_gru_fwd<32>, smem, (V + 31) / 32);
+    k_gru_fwd<32><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
+  } else {
+    const size_t smem = gru_fwd_smem(H, 16);
+    STG_TRY(set_smem(k_gru_fwd<16>, smem));
+    const int nb = grid_blocks((const void*)k_gru_fwd<16>, smem, (V + 15) / 16);
+    k_gru_fwd<16><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
+  }
+  count_launch();
+  STG_TRY(check_launch("stg_tgcn_step"));
+  if (stack) {
+    const size_t need = (cbytes + 255) & ~size_t(255);
+    stack->entries.push_back(StackEntry{H_prev, C, V, H, need});
+    stack->top += need;
+  }
+  return STG_OK;
+}
+
+stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* p, const float* X,
+                                  const float* dH_next, float* dH_prev, stg_tgcn_grads* grads,
+                                  stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_params(p));
+  if (!g || !X || !dH_next || !dH_prev || !grads || !stack)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward: NULL argument");
+  if (!grads->W || !grads->b || !grads->L || !grads->l)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward: NULL gradient pointer");
+  if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn_step_backward: state stack is empty");
+  const StackEntry e = stack->entries.back();
+  const int32_t V = g->num_nodes, F = p->F, H = p->H, H3 = 3 * H;
+  if (e.V != V || e.H != H) return fail(STG_ERR_STATE, "stg_tgcn_step_backward: stack top does not match (V,H)");
+  cudaStream_t s = (cudaStream_t)stream;
+  TgcnWs& ws = stack->ws;
+  STG_TRY(ws.dC.alloc((size_t)V * H3));
+  STG_TRY(ws.dP.alloc((size_t)V * H3));
+  // GRU backward + partials of dL, dl, db
+  ProfScope* prof_gru = new ProfScope(PH_GRU_BWD, s);
+  const int BR = H <= 32 ? 16 : 4;
+  const size_t smem = gru_bwd_smem(H, BR);
+  const int NP = 6 * H * H + 6 * H;
+  int nbg;
+  if (BR == 16) {
+    STG_TRY(set_smem(k_gru_bwd<16>, smem));
+    nbg = grid_blocks((const void*)k_gru_bwd<16>, smem, (V + 15) / 16);
+  } else {
+    STG_TRY(set_smem(k_gru_bwd<4>, smem));
+    nbg = grid_blocks((const void*)k_gru_bwd<4>, smem, (V + 3) / 4);
+  }
+  STG_TRY(ws.part_gru.alloc((size_t)nbg * NP));
+  if (BR == 16)
+    k_gru_bwd<16><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, g->norm_dst, ws.dC.p, dH_prev,
+                                        ws.part_gru.p);
+  else
+    k_gru_bwd<4><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, g->norm_dst, ws.dC.p, dH_prev,
+                                       ws.part_gru.p);
+  count_launch();
+  k_reduce_part<<<(NP + 255) / 256, 256, 0, s>>>(ws.part_gru.p, nbg, NP, grads->L, 6 * H * H, grads->l, 3 * H,
+                                                 grads->b);
+  count_launch();
+  delete prof_gru;
+  // dP = diag(n_src)·Aᵀ·(n_dst ⊙ dC) over the out-CSR
+  STG_TRY(aggregate_launch(g, 1, H3, ws.dC.p, H3, ws.dP.p, H3, g->norm_src, nullptr, nullptr, s));
+  // dW += Xᵀ·dP
+  {
+    ProfScope prof(PH_DW, s);
+    const size_t sm2 = sizeof(float) * (size_t)(32 * F + 32 * H3 + F * H3);
+    STG_TRY(set_smem(k_dw, sm2));
+    const int nb = grid_blocks((const void*)k_dw, sm2, (V + 31) / 32);
+    STG_TRY(ws.part_dw.alloc((size_t)nb * F * H3));
+    k_dw<<<nb, kT, sm2, s>>>(V, F, H3, X, ws.dP.p, ws.part_dw.p);
+    k_reduce_part<<<(F * H3 + 255) / 256, 256, 0, s>>>(ws.part_dw.p, nb, F * H3, grads->W, F * H3, nullptr, 0,
+                                                       nullptr);
+    count_launch(2);
+  }
+  STG_TRY(check_launch("stg_tgcn_step_backward"));
+  stack->entries.pop_back();
+  stack->top -= e.bytes;
+  return STG_OK;
+}
+
+stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o, const float* b_o,
+                        float* loss_accum, float* dH, int32_t accumulate, float* dw_o, float* db_o,
+                        stg_stream_t stream) {
+  if (V < 1 || H < 1 || H > 64 || !Hn || !y || !w_o || !b_o)
+    return fail(STG_ERR_INVALID_ARG, "stg_mse_head: bad arguments (V=%d H=%d)", V, H);
+  cudaStream_t s = (cudaStream_t)stream;
+  TgcnWs& ws = global_ws();
+  int nb = (int)std::min<int64_t>((V + 7) / 8, (int64_t)num_sms() * 4);
+  STG_TRY(ws.lpart.alloc(nb));
+  STG_TRY(ws.gpart.alloc((size_t)nb * (H + 1)));
+  const int want = (dH || dw_o || db_o) ? 1 : 0;
+  ProfScope prof(PH_HEAD, s);
+  k_mse_head<<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p);
+  k_mse_reduce<<<1, 64, 0, s>>>(nb, H, V, ws.lpart.p, ws.gpart.p, loss_accum, want ? dw_o : nullptr,
+                                want ? db_o : nullptr);
+  count_launch(2);
+  return check_launch("stg_mse_head");
+}
+
+stg_status stg_sgd_update(float* p, const float* g, int64_t n, float lr, stg_stream_t stream) {
+  if (n < 0 || (n > 0 && (!p || !g))) return fail(STG_ERR_INVALID_ARG, "stg_sgd_update: bad arguments");
+  if (!n) return STG_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  k_sgd<<<(unsigned)std::min<int64_t>(ceil_div(n, 256), 4096), 256, 0, s>>>(p, g, n, lr);
+  count_launch();
+  return check_launch("stg_sgd_update");
+}
+
+stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
+                                   const stg_tgcn_params* p, const float* w_o, const float* b_o,
+                                   const float* const* X, const float* const* Y, const float* H0, float* H_seq,
+                                   float* G_work, stg_tgcn_grads* grads, float* dw_o, float* db_o,
+                                   float* loss_accum, stg_state_stack* stack, stg_stream_t stream) {
+  if ((graph == nullptr) == (dtdg == nullptr))
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence: exactly one of graph / dtdg must be given");
+  if (S < 1 || !X || !Y || !H0 || !H_seq || !G_work || !stack)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence: bad arguments");
+  STG_TRY(check_params(p));
+  stg_csr_view view;
+  int32_t V;
+  if (graph) {
+    STG_TRY(stg_graph_view(graph, &view));
+    V = view.num_nodes;
+  } else {
+    if (t0 < 0 || t0 + S > stg_dtdg_num_timestamps(dtdg))
+      return fail(STG_ERR_OUT_OF_RANGE, "stg_tgcn_train_sequence: [%d,%d) outside the DTDG", t0, t0 + S);
+    STG_TRY(stg_dtdg_get_snapshot(dtdg, t0, stream, &view));
+    V = view.num_nodes;
+  }
+  const int32_t H = p->H;
+  const size_t VH = (size_t)V * H;
+  std::vector<int32_t> graph_stack;
+  // forward, Algorithm 1 lines 7-16
+  for (int32_t i = 0; i < S; ++i) {
+    const int32_t t = t0 + i;
+    if (dtdg) {
+      if (i > 0) STG_TRY(stg_dtdg_get_snapshot(dtdg, t, stream, &view));   // Get-Graph (Alg. 2)
+      graph_stack.push_back(t);                                             // graph-stack.push(t)
+    }
+    const float* Hp = i == 0 ? H0 : H_seq + (size_t)(i - 1) * VH;
+    STG_TRY(stg_tgcn_step(&view, p, X[i], Hp, H_seq + (size_t)i * VH, stack, stream));   // push + fwdprop
+    STG_TRY(stg_mse_head(V, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr, nullptr,
+                         stream));                                          // loss += loss-fn(out)
+  }
+  // backward in LIFO order, lines 18-25
+  float* G = G_work;
+  float* Gn = G_work + VH;
+  STG_CUDA(cudaMemsetAsync(G, 0, sizeof(float) * VH, (cudaStream_t)stream));
+  for (int32_t i = S - 1; i >= 0; --i) {
+    if (dtdg) {
+      const int32_t t = graph_stack.back();
+      graph_stack.pop_back();
+      STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, t, stream, &view));     // Get-Backward-Graph
+    }
+    // G = dℓ_t/dH_t + dH from step t+1
+    STG_TRY(stg_mse_head(V, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, nullptr, G, 1, dw_o, db_o, stream));
+    STG_TRY(stg_tgcn_step_backward(&view, p, X[i], G, Gn, grads, stack, stream));   // pop + bwdprop
+    std::swap(G, Gn);
+  }
+  return STG_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,144 @@
+"""GPU parity: on-demand DTDG snapshots (Get-Graph / Get-Backward-Graph) are
+bit-exact against the oracle's cumulative rebuild, in every access order."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from helpers import assert_graph_equal, cond_err, to_gpu
+
+pytestmark = pytest.mark.gpu
+
+
+def _create(stg, d, flags):
+    return stg.stg_dtdg_create(d.V, d.T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                               d.del_dst, flags)
+
+
+def _oracle_snaps(d, loops):
+    return [oracle.csr(d.V, S) for S in oracle.snapshot_sets_fold(d, self_loops=loops)]
+
+
+@pytest.fixture(scope="module", params=["C4", "C5s"])
+def dtdg_case(request, stg):
+    d = gen.dtdg(gen.CONFIGS[request.param])
+    refs = {loops: _oracle_snaps(d, loops) for loops in (False, True)}
+    return request.param, d, refs
+
+
+@pytest.mark.parametrize("loops", [False, True])
+def test_forward_walk_bit_exact(stg, dtdg_case, loops):
+    name, d, refs = dtdg_case
+    flags = stg.STG_EDGE_IDS | (stg.STG_SELF_LOOPS if loops else 0)
+    g = _create(stg, d, flags)
+    assert g.T == d.T
+    for t in range(d.T):
+        assert g.num_edges(t) == refs[loops][t]["E"], t
+    for t in range(d.T):
+        v = stg.stg_dtdg_get_snapshot(g, t)
+        assert v.timestamp == t
+        assert_graph_equal(stg.view_arrays(v), refs[loops][t], tag=(name, "fwd", t))
+
+
+@pytest.mark.parametrize("loops", [False, True])
+def test_backward_walk_and_random_access(stg, dtdg_case, loops):
+    name, d, refs = dtdg_case
+    flags = stg.STG_EDGE_IDS | (stg.STG_SELF_LOOPS if loops else 0)
+    g = _create(stg, d, flags)
+    T = d.T
+    # Algorithm 1 pattern: sequences of S forward, then backward in LIFO order
+    S = 4
+    for t0 in range(0, T, S):
+        ts = list(range(t0, min(T, t0 + S)))
+        for t in ts:
+            assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_snapshot(g, t)), refs[loops][t], tag=(name, "f", t))
+        for t in reversed(ts):
+            v = stg.stg_dtdg_get_backward_snapshot(g, t)
+            assert_graph_equal(stg.view_arrays(v), refs[loops][t], tag=(name, "b", t))
+    # random access, both kinds
+    rng = np.random.default_rng(0)
+    for _ in range(12):
+        t = int(rng.integers(0, T))
+        f = stg.stg_dtdg_get_backward_snapshot if rng.integers(0, 2) else stg.stg_dtdg_get_snapshot
+        assert_graph_equal(stg.view_arrays(f(g, t)), refs[loops][t], tag=(name, "r", t))
+    # full backward walk from the end to 0
+    stg.stg_dtdg_get_snapshot(g, T - 1)
+    for t in reversed(range(T)):
+        assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_backward_snapshot(g, t)), refs[loops][t],
+                           tag=(name, "bw", t))
+
+
+def test_snapshot_aggregation(stg, dtdg_case):
+    name, d, refs = dtdg_case
+    g = _create(stg, d, stg.STG_SELF_LOOPS)
+    W = 64
+    for t in (0, 1, d.T // 2, d.T - 1):
+        v = stg.stg_dtdg_get_snapshot(g, t)
+        x = gen.uniform_pm1(t, 77, d.V * W).reshape(d.V, W).astype(np.float64)
+        y = stg.stg_gcn_aggregate_fwd(v, to_gpu(x)).cpu().numpy()
+        ref = refs[True][t]
+        assert cond_err(y, oracle.aggregate_fwd(ref, x), oracle.aggregate_scale(ref, x)) <= 1e-5
+        vb = stg.stg_dtdg_get_backward_snapshot(g, t)
+        gx = stg.stg_gcn_aggregate_bwd(vb, to_gpu(x)).cpu().numpy()
+        assert cond_err(gx, oracle.aggregate_bwd(ref, x), oracle.aggregate_scale(ref, x, bwd=True)) <= 1e-5
+
+
+def _noisy(seed, V=300, T=9):
+    """Raw batches with duplicates, deletes of absent edges, add∩delete and loops."""
+    rng = np.random.default_rng(seed)
+    s0, d0 = rng.integers(0, V, 2000), rng.integers(0, V, 2000)
+    A, D = [(np.zeros(0, int), np.zeros(0, int))], [(np.zeros(0, int), np.zeros(0, int))]
+    for t in range(1, T):
+        na, nd = int(rng.integers(0, 300)), int(rng.integers(0, 300))
+        a = (rng.integers(0, V, na), rng.integers(0, V, na))
+        dd = (rng.integers(0, V, nd), rng.integers(0, V, nd))
+        if na > 10:   # add ∩ delete and duplicates
+            dd = (np.concatenate([dd[0], a[0][:5]]), np.concatenate([dd[1], a[1][:5]]))
+            a = (np.concatenate([a[0], a[0][:5]]), np.concatenate([a[1], a[1][:5]]))
+        A.append(a); D.append(dd)
+    off = lambda L: np.concatenate([[0], np.cumsum([x[0].size for x in L])]).astype(np.int64)
+    cat = lambda L, i: np.concatenate([x[i] for x in L]).astype(np.int32)
+    return gen.DTDG(V=V, T=T, W=0, slide=0, ev_src=None, ev_dst=None, src0=s0.astype(np.int32),
+                    dst0=d0.astype(np.int32), add_off=off(A), add_src=cat(A, 0), add_dst=cat(A, 1),
+                    del_off=off(D), del_src=cat(D, 0), del_dst=cat(D, 1))
+
+
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("loops", [False, True])
+def test_raw_batches_are_normalised(stg, seed, loops):
+    d = _noisy(seed)
+    refs = _oracle_snaps(d, loops)
+    g = _create(stg, d, stg.STG_EDGE_IDS | (stg.STG_SELF_LOOPS if loops else 0))
+    for t in range(d.T):
+        assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_snapshot(g, t)), refs[t], tag=(seed, t))
+    for t in reversed(range(d.T)):
+        assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_backward_snapshot(g, t)), refs[t], tag=(seed, "b", t))
+    # effective delta counts equal the oracle's normalisation
+    S_prev = None
+    for t, S in enumerate(oracle.snapshot_sets_fold(d, self_loops=loops)):
+        if t:
+            A, D = oracle.batch(d, t)
+            a, dd = oracle.effective_deltas(S_prev, A, D, pinned_loops=loops)
+            assert g.num_deltas(t, False) == a.size and g.num_deltas(t, True) == dd.size
+        S_prev = S
+
+
+def test_validate_rejects_ineffective_batches(stg):
+    d = _noisy(1)
+    with pytest.raises(stg.StgError) as e:
+        _create(stg, d, stg.STG_VALIDATE)
+    assert e.value.status == 1
+
+
+def test_bad_arguments(stg):
+    d = gen.dtdg(gen.CONFIGS["C5s"])
+    g = _create(stg, d, 0)
+    with pytest.raises(stg.StgError) as e:
+        stg.stg_dtdg_get_snapshot(g, d.T)
+    assert e.value.status == 2
+    bad_off = d.add_off.copy()
+    bad_off[1] = 1
+    with pytest.raises(stg.StgError):
+        stg.stg_dtdg_create(d.V, d.T, d.src0, d.dst0, bad_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                            d.del_dst, 0)

@@ -1,0 +1,168 @@
+"""GPU parity: TGCN step forward/backward and Algorithm 1 sequences vs the oracle.
+
+Tolerances: H' is compared in absolute terms (|H'| < 1)
+at 2e-5; parameter gradients normwise per tensor at 1e-4 · max|ref|; the
+sequence loss at 1e-5 relative.
+"""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from helpers import to_gpu
+
+pytestmark = pytest.mark.gpu
+
+H_TOL = 2e-5
+G_TOL = 1e-4
+
+
+def _params(F, H, seed):
+    p = gen.tgcn_params(F, H, seed)
+    return p, {k: to_gpu(v) for k, v in p.items()}
+
+
+def _zero_grads(F, H):
+    return {"W": torch.zeros(F, 3 * H, device="cuda"), "b": torch.zeros(3 * H, device="cuda"),
+            "L": torch.zeros(3, 2 * H, H, device="cuda"), "l": torch.zeros(3, H, device="cuda")}
+
+
+def _normwise(a, ref):
+    a = np.asarray(a, np.float64)
+    ref = np.asarray(ref, np.float64)
+    den = np.max(np.abs(ref))
+    return float(np.max(np.abs(a - ref)) / (den if den > 0 else 1.0))
+
+
+def _graph(stg, name):
+    cfg = gen.CONFIGS[name]
+    if cfg.kind == "static":
+        s, d = gen.static_edges(cfg)
+        return cfg, stg.stg_static_graph_create(cfg.V, s, d, stg.STG_SELF_LOOPS), \
+            oracle.static_graph(cfg.V, s, d, self_loops=True)
+    dd = gen.dtdg(cfg)
+    S0 = next(oracle.snapshot_sets_fold(dd, self_loops=True))
+    return cfg, stg.stg_static_graph_create(cfg.V, oracle.unkey(S0)[0], oracle.unkey(S0)[1], 0), oracle.csr(cfg.V, S0)
+
+
+@pytest.mark.parametrize("name,H", [("C1", 16), ("C2", 32), ("C6", 16), ("C5s", 32), ("C2", 64), ("C1", 5)])
+def test_tgcn_step_parity(stg, name, H):
+    cfg, g, ref = _graph(stg, name)
+    V, F = cfg.V, cfg.F
+    p, pg = _params(F, H, 11)
+    X = gen.features(cfg, 5)
+    Hp = gen.uniform_pm1(3, 3, V * H).reshape(V, H)
+    Xg, Hg = to_gpu(X), to_gpu(Hp)
+    stack = stg.stg_state_stack_create(64 << 20)
+    Hn = stg.stg_tgcn_step(g.view(), pg, Xg, Hg, stack=stack)
+    f = oracle.tgcn_fwd(ref, p, X, Hp)
+    err = np.max(np.abs(Hn.cpu().numpy() - f["Hn"]))
+    assert err <= H_TOL, err
+    # backward with a random upstream gradient
+    G = gen.uniform_pm1(4, 4, V * H).reshape(V, H)
+    grads = _zero_grads(F, H)
+    dHp = stg.stg_tgcn_step_backward(g.view(), pg, Xg, to_gpu(G), grads, stack)
+    assert stack.depth == 0
+    rg = oracle.zero_grads(F, H)
+    rdH = oracle.tgcn_bwd(ref, p, X, Hp, f, G, rg)
+    assert _normwise(dHp.cpu().numpy(), rdH) <= G_TOL
+    for k in ("W", "b", "L", "l"):
+        e = _normwise(grads[k].cpu().numpy(), rg[k])
+        assert e <= G_TOL, (k, e)
+
+
+def test_tgcn_inference_and_stack_errors(stg):
+    cfg, g, ref = _graph(stg, "C1")
+    p, pg = _params(cfg.F, cfg.H, 1)
+    X = to_gpu(gen.features(cfg, 0))
+    H0 = torch.zeros(cfg.V, cfg.H, device="cuda")
+    Hn = stg.stg_tgcn_step(g.view(), pg, X, H0)          # no stack: inference
+    f = oracle.tgcn_fwd(ref, p, gen.features(cfg, 0), np.zeros((cfg.V, cfg.H)))
+    assert np.max(np.abs(Hn.cpu().numpy() - f["Hn"])) <= H_TOL
+    stack = stg.stg_state_stack_create(1 << 20)
+    with pytest.raises(stg.StgError) as e:
+        stg.stg_tgcn_step_backward(g.view(), pg, X, H0, _zero_grads(cfg.F, cfg.H), stack)
+    assert e.value.status == 6
+    tiny = stg.stg_state_stack_create(16)
+    with pytest.raises(stg.StgError) as e:
+        stg.stg_tgcn_step(g.view(), pg, X, H0, stack=tiny)
+    assert e.value.status == 3
+
+
+def test_zero_parameters_closed_form(stg):
+    cfg, g, _ = _graph(stg, "C2")
+    pg = {k: torch.zeros_like(v) for k, v in _params(cfg.F, cfg.H, 0)[1].items()}
+    Hp = to_gpu(gen.uniform_pm1(1, 1, cfg.V * cfg.H).reshape(cfg.V, cfg.H))
+    Hn = stg.stg_tgcn_step(g.view(), pg, to_gpu(gen.features(cfg, 0)), Hp)
+    assert torch.equal(Hn, 0.5 * Hp)
+
+
+def _run_sequence(stg, source, cfg, pg, Xs, Ys, H0, S, t0):
+    V, H, F = cfg.V, pg["L"].shape[2], cfg.F
+    grads = _zero_grads(F, H)
+    dw = torch.zeros(H, device="cuda")
+    db = torch.zeros(1, device="cuda")
+    loss = torch.zeros(1, device="cuda")
+    Hseq = torch.empty(S, V, H, device="cuda")
+    Gw = torch.empty(2, V, H, device="cuda")
+    stack = stg.stg_state_stack_create(S * V * 3 * H * 4 + (1 << 20))
+    stg.stg_tgcn_train_sequence(source, t0, S, pg, pg["w_o"], pg["b_o"], Xs, Ys, H0, Hseq, Gw, grads, dw, db,
+                                loss, stack)
+    assert stack.depth == 0
+    return loss.item(), grads, dw, db, Hseq
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_train_sequence_static(stg, name):
+    cfg = gen.CONFIGS[name]
+    s, d = gen.static_edges(cfg)
+    g = stg.stg_static_graph_create(cfg.V, s, d, stg.STG_SELF_LOOPS)
+    ref = oracle.static_graph(cfg.V, s, d, self_loops=True)
+    S, t0 = 8, 16
+    p, pg = _params(cfg.F, cfg.H, 2)
+    Xs = [gen.features(cfg, t0 + i) for i in range(S)]
+    Ys = [gen.labels(cfg, t0 + i) for i in range(S)]
+    H0 = gen.uniform_pm1(8, 8, cfg.V * cfg.H).reshape(cfg.V, cfg.H)
+    loss, grads, dw, db, Hseq = _run_sequence(stg, g, cfg, pg, [to_gpu(x) for x in Xs], [to_gpu(y) for y in Ys],
+                                              to_gpu(H0), S, t0)
+    rl, rg, rH = oracle.train_sequence([ref] * S, [ref] * S, p, Xs, Ys, H0)
+    assert abs(loss - rl) <= 1e-5 * abs(rl)
+    assert np.max(np.abs(Hseq[-1].cpu().numpy() - rH)) <= H_TOL
+    for k in ("W", "b", "L", "l"):
+        assert _normwise(grads[k].cpu().numpy(), rg[k]) <= G_TOL, k
+    assert _normwise(dw.cpu().numpy(), rg["w_o"]) <= G_TOL
+    assert _normwise(db.cpu().numpy(), rg["b_o"]) <= G_TOL
+
+
+@pytest.mark.parametrize("name", ["C4", "C5s"])
+def test_train_sequence_dtdg(stg, name):
+    cfg = gen.CONFIGS[name]
+    d = gen.dtdg(cfg)
+    g = stg.stg_dtdg_create(d.V, d.T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                            d.del_dst, stg.STG_SELF_LOOPS)
+    snaps = [oracle.csr(d.V, S) for S in oracle.snapshot_sets_fold(d, self_loops=True)]
+    H = cfg.H
+    p, pg = _params(cfg.F, H, 3)
+    H0 = np.zeros((cfg.V, H))
+    Hc = to_gpu(H0)
+    S = 4
+    for t0 in (0, S, 2 * S):             # three consecutive sequences (cached head reuse)
+        Xs = [gen.features(cfg, t0 + i) for i in range(S)]
+        Ys = [gen.labels(cfg, t0 + i) for i in range(S)]
+        loss, grads, dw, db, Hseq = _run_sequence(stg, g, cfg, pg, [to_gpu(x) for x in Xs],
+                                                  [to_gpu(y) for y in Ys], Hc, S, t0)
+        rl, rg, rH = oracle.train_sequence(snaps[t0:t0 + S], snaps[t0:t0 + S], p, Xs, Ys, H0)
+        assert abs(loss - rl) <= 1e-5 * abs(rl), (t0, loss, rl)
+        assert np.max(np.abs(Hseq[-1].cpu().numpy() - rH)) <= H_TOL
+        for k in ("W", "b", "L", "l"):
+            assert _normwise(grads[k].cpu().numpy(), rg[k]) <= G_TOL, (t0, k)
+        H0 = rH
+        Hc = Hseq[-1].clone()
+
+
+def test_sgd_update(stg):
+    p = torch.arange(10, dtype=torch.float32, device="cuda")
+    g = torch.ones(10, device="cuda")
+    stg.stg_sgd_update(p, g, 0.5)
+    assert torch.equal(p, torch.arange(10, dtype=torch.float32, device="cuda") - 0.5)
