@@ -1,0 +1,398 @@
+#!/usr/bin/env python
+"""bench.py — STGraph hot path on B200: one step = one Algorithm-1 TGCN training
+epoch over the C5 DTDG (wiki-talk-temporal-shaped, 2^20 nodes,
+~8M edges + self-loops, T=41 on-demand snapshots, F=64, H=32, sequences of 16).
+
+Every step runs, per timestamp t: Get-Graph(t) (delta-apply snapshot build),
+P' = X_t·W, forward aggregation over the in-CSR, GRU; then per sequence in LIFO
+order: Get-Backward-Graph(t), head gradient, GRU backward, backward aggregation
+over the out-CSR, dW; and one SGD step per sequence.
+
+metric: aggregated edges/s (fwd+bwd) = Σ_t 2·|E_t| per epoch ÷ epoch time
+(plus timesteps/s).  `--impl reference` times the fp64 oracle on the host.
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "aggregated edges/s (fwd+bwd)"
+UNIT = "edges/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C5")
+    ap.add_argument("--seq", type=int, default=16, help="sequence length S (reading C16)")
+    ap.add_argument("--lr", type=float, default=1e-3)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs (STREAM-style copy, burst)"
+    return 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
+
+
+# ------------------------------------------------------------------ oracle (CPU baseline / reference arm)
+def oracle_timestep(cfg, d, t: int, S_prev):
+    """The fp64 oracle on one C5 timestep: Get-Graph (fold S_{t-1} -> S_t), CSR pair
+    build, TGCN forward, MSE head, TGCN backward.  Returns (edges aggregated, seconds, S_t)."""
+    import gen
+    import oracle
+    X = gen.features(cfg, t % 2)
+    Y = gen.labels(cfg, t)
+    p = gen.tgcn_params(cfg.F, cfg.H, cfg.seed)
+    Hp = np.zeros((cfg.V, cfg.H))
+    t0 = time.perf_counter()
+    A, D = oracle.batch(d, t)
+    s_, d_ = oracle.unkey(D)
+    D = D[s_ != d_]
+    S = oracle.set_apply(S_prev, D, np.concatenate([A, oracle.keys(np.arange(cfg.V), np.arange(cfg.V))]))
+    g = oracle.csr(cfg.V, S)
+    f = oracle.tgcn_fwd(g, p, X, Hp)
+    grads = oracle.zero_grads(cfg.F, cfg.H)
+    _, dH = oracle.mse_head(f["Hn"], Y, p["w_o"], p["b_o"], grads)
+    oracle.tgcn_bwd(g, p, X, Hp, f, dH, grads)
+    dt = time.perf_counter() - t0
+    return 2 * g["E"], dt, S
+
+
+def run_reference(args):
+    import gen
+    import oracle
+    cfg = gen.CONFIGS[args.config]
+    d = gen.dtdg(cfg)
+    oracle.build()
+    S = next(oracle.snapshot_sets_fold(d, self_loops=True))
+    edges, secs = 0, 0.0
+    t = 1
+    for i in range(args.warmup + args.steps):
+        e, dt, S = oracle_timestep(cfg, d, t, S)
+        if i >= args.warmup:
+            edges += e
+            secs += dt
+        t = t + 1 if t + 1 < d.T else 1
+        if t == 1:
+            S = next(oracle.snapshot_sets_fold(d, self_loops=True))
+    value = edges / secs
+    sample = "per step: one C5 timestep (fold S_{t-1}->S_t, CSR pair, TGCN fwd + MSE head + bwd) in the fp64 oracle"
+    out = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+           "config": {"workload": cfg.desc, "config": cfg.name, "V": cfg.V, "F": cfg.F, "H": cfg.H, "T": d.T,
+                      "sample": sample},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+# ------------------------------------------------------------------ our arm
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        if rank == 0:
+            run_reference(args)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import gen
+    import paper_conf_ipps_cherianmcc24_b200 as stg
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    cfg = gen.CONFIGS[args.config]
+    assert cfg.kind == "dtdg"
+    d = gen.dtdg(cfg)
+    V, F, H, T = cfg.V, cfg.F, cfg.H, d.T
+    S = args.seq
+    seqs = [(t0, min(S, T - t0)) for t0 in range(0, T, S)]
+    g = stg.stg_dtdg_create(V, T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src, d.del_dst,
+                            stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS)
+    E_t = [g.num_edges(t) for t in range(T)]
+    edges_per_step = 2 * sum(E_t)
+
+    # inputs: 2 distinct seeded X_t matrices cycled over t (each 256 MB > L2), labels per t
+    NX = 2
+    Xh = [torch.from_numpy(gen.features(cfg, i)) for i in range(NX)]
+    Yh = [torch.from_numpy(gen.labels(cfg, t)) for t in range(T)]
+    Xd = [x.to(dev) for x in Xh]
+    Yd = [y.to(dev) for y in Yh]
+    p = {k: torch.from_numpy(v).to(dev) for k, v in gen.tgcn_params(F, H, cfg.seed).items()}
+    grads = {"W": torch.zeros(F, 3 * H, device=dev), "b": torch.zeros(3 * H, device=dev),
+             "L": torch.zeros(3, 2 * H, H, device=dev), "l": torch.zeros(3, H, device=dev)}
+    dw_o, db_o = torch.zeros(H, device=dev), torch.zeros(1, device=dev)
+    loss = torch.zeros(1, device=dev)
+    Hbuf = [torch.empty(S, V, H, device=dev) for _ in range(2)]
+    H0 = torch.zeros(V, H, device=dev)
+    Gw = torch.empty(2, V, H, device=dev)
+    stack = stg.stg_state_stack_create(S * V * 3 * H * 4 + (64 << 20))
+    stream = torch.cuda.current_stream()
+
+    def sgd():
+        for k in ("W", "b", "L", "l"):
+            stg.stg_sgd_update(p[k], grads[k], args.lr)
+        stg.stg_sgd_update(p["w_o"], dw_o, args.lr)
+        stg.stg_sgd_update(p["b_o"], db_o, args.lr)
+
+    def epoch(Xsrc, Ysrc):
+        Hprev = H0
+        for k, (t0, n) in enumerate(seqs):
+            Hs = Hbuf[k % 2]
+            stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], [Xsrc(t) for t in range(t0, t0 + n)],
+                                        [Ysrc(t) for t in range(t0, t0 + n)], Hprev, Hs, Gw, grads, dw_o, db_o,
+                                        loss, stack)
+            sgd()
+            Hprev = Hs[n - 1]
+
+    Xdev = lambda t: Xd[t % NX]
+    Ydev = lambda t: Yd[t]
+    for _ in range(args.warmup):
+        epoch(Xdev, Ydev)
+    torch.cuda.synchronize()
+
+    # ---------------- timed region (device-resident inputs)
+    clocks = ClockSampler(local)
+    stg.stg_profile_enable(False)
+    stg.stg_profile_read(reset=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    time.sleep(0.3)
+    launches0 = stg.kernel_launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for _ in range(args.steps):
+        epoch(Xdev, Ydev)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1)
+    launches = stg.kernel_launch_count() - launches0
+    clk = clocks.stop()
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = t.item()
+        dist.barrier()
+    value = world * edges_per_step * args.steps / (ms / 1e3)
+    tsps = world * T * args.steps / (ms / 1e3)
+
+    # ---------------- per-phase device times (profiled pass, same work)
+    stg.stg_profile_enable(True)
+    stg.stg_profile_read(reset=True)
+    for _ in range(max(1, min(args.steps, 2))):
+        epoch(Xdev, Ydev)
+    torch.cuda.synchronize()
+    prof = stg.stg_profile_read(reset=True)
+    stg.stg_profile_enable(False)
+    nprof = max(1, min(args.steps, 2))
+
+    # roofline of the dominant kernel: the aggregation (fwd + bwd, W = 3H)
+    Wagg = 3 * H
+    E_mean = sum(E_t) / T
+    # compulsory bytes per launch: col 4E + rowptr 4(V+1) + node_ids 4V + row scale 4V
+    # + read each source row once 4VW + write each output row 4VW
+    alg_bytes = 4 * E_mean + 4 * (V + 1) + 4 * V + 4 * V + 8 * V * Wagg
+    agg_ms = prof["agg_fwd"][0] + prof["agg_bwd"][0]
+    agg_n = prof["agg_fwd"][1] + prof["agg_bwd"][1]
+    agg_avg_s = (agg_ms / agg_n) / 1e3 if agg_n else float("nan")
+    peak, peak_src = measured_peaks()
+    achieved = alg_bytes / agg_avg_s / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "agg_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("bytes_per_launch")
+        except Exception:
+            traffic = None
+    step_ms_prof = sum(v[0] for v in prof.values()) / nprof
+
+    # ---------------- end-to-end through the public API with host buffers
+    e2e = None
+    if not args.no_e2e:
+        Xpin = [x.pin_memory() for x in Xh]
+        Ypin = [y.pin_memory() for y in Yh]
+        copy = torch.cuda.Stream(device=dev)
+        stage = [[torch.empty(V, F, device=dev) for _ in range(S)] for _ in range(2)]
+        ystage = [[torch.empty(V, device=dev) for _ in range(S)] for _ in range(2)]
+        loss_h = torch.empty(1, pin_memory=True)
+        h2d = 0
+
+        def e2e_epoch():
+            nonlocal h2d
+            done = [None, None]
+            # prefetch sequence 0
+            def issue(k):
+                nonlocal h2d
+                t0, n = seqs[k]
+                with torch.cuda.stream(copy):
+                    if done[k % 2] is not None:
+                        copy.wait_event(done[k % 2])
+                    for i in range(n):
+                        stage[k % 2][i].copy_(Xpin[(t0 + i) % NX], non_blocking=True)
+                        ystage[k % 2][i].copy_(Ypin[t0 + i], non_blocking=True)
+                        h2d += Xpin[0].numel() * 4 + Ypin[0].numel() * 4
+                    ev = torch.cuda.Event()
+                    ev.record(copy)
+                return ev
+            ready = issue(0)
+            Hprev = H0
+            for k, (t0, n) in enumerate(seqs):
+                stream.wait_event(ready)
+                if k + 1 < len(seqs):
+                    nxt = issue(k + 1) if True else None
+                Hs = Hbuf[k % 2]
+                stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], stage[k % 2][:n], ystage[k % 2][:n],
+                                            Hprev, Hs, Gw, grads, dw_o, db_o, loss, stack)
+                sgd()
+                ev = torch.cuda.Event()
+                ev.record(stream)
+                done[k % 2] = ev
+                Hprev = Hs[n - 1]
+                if k + 1 < len(seqs):
+                    ready = nxt
+            loss_h.copy_(loss, non_blocking=True)
+            torch.cuda.synchronize()
+            return float(loss_h.item())
+
+        for _ in range(1):
+            e2e_epoch()
+        h2d = 0
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t0w = time.perf_counter()
+        for _ in range(args.steps):
+            e2e_epoch()
+        e2e_s = time.perf_counter() - t0w
+        if world > 1:
+            tt = torch.tensor([e2e_s], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            e2e_s = tt.item()
+        e2e = {"value": world * edges_per_step * args.steps / e2e_s, "unit": UNIT,
+               "h2d_bytes_per_step": int(h2d / args.steps), "d2h_bytes_per_step": 4,
+               "ms_per_step": 1e3 * e2e_s / args.steps,
+               "note": "X_t (256 MB) and y_t copied H2D from pinned host memory every timestep on a copy "
+                       "stream overlapped with the previous sequence; loss read back every epoch"}
+
+    # ---------------- CPU baseline: the oracle on one C5 timestep (rank 0, N=1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        oracle.build()
+        S0 = next(oracle.snapshot_sets_fold(d, self_loops=True))
+        e_c, dt_c, _ = oracle_timestep(cfg, d, 1, S0)
+        cpu = {"value": e_c / dt_c, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": "one C5 timestep (t=1): fold S_0->S_1, CSR pair, TGCN fwd + MSE head + bwd, fp64, "
+                         "single thread; %.1f s" % dt_c}
+
+    if rank == 0:
+        out = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": cfg.desc + " (BASELINE.json configs[4])", "config": cfg.name, "V": V,
+                       "E_mean": int(E_mean), "T": T, "F": F, "H": H, "seq_len": S, "sequences": len(seqs),
+                       "step": "one Algorithm-1 training epoch over all T timestamps",
+                       "l2": "inputs larger than L2 (X_t 256 MB, graph ~0.3 GB, state 8 GB)",
+                       "parallelism": "replicas" if world > 1 else "single"},
+            "timesteps_per_s": tsps,
+            "gpu_launches": int(launches),
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "k_aggregate (fwd in-CSR + bwd out-CSR, W=%d)" % Wagg,
+                         "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": agg_avg_s * 1e3,
+                         "peak_source": peak_src},
+            "phases_ms_per_step": {k: v[0] / nprof for k, v in prof.items()},
+            "phase_share": {k: (v[0] / nprof) / step_ms_prof for k, v in prof.items()} if step_ms_prof else None,
+            "clocks": clk,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

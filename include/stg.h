@@ -168,6 +168,11 @@ stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t
                                 const float* scale_row, const float* scale_col, const float* bias,
                                 stg_stream_t stream);
 
+/* Gather strategy of the aggregation kernel for the float4 path: 0 (default)
+ * = register gathers; 1 = asynchronous cp.async copies of neighbour rows into
+ * a per-warp shared-memory ring.  Results are bit-identical. */
+stg_status stg_aggregate_set_strategy(int32_t async_gather);
+
 /* ---- TGCN (GCN + GRU; reading C13-C15) ----
  * W [F,3H] (gates z|r|h), b [3H], L [3][2H][H] (gate g: rows 0..H-1 = L_g¹ act
  * on C_g, rows H..2H-1 = L_g² act on H or R⊙H), l [3][H]. */
@@ -210,8 +215,9 @@ stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, c
                         const float* b_o, float* loss_accum, float* dH, int32_t accumulate,
                         float* dw_o, float* db_o, stg_stream_t stream);
 
-/* p -= lr·g over n elements (the per-sequence optimiser step, reading C17). */
-stg_status stg_sgd_update(float* p, const float* g, int64_t n, float lr, stg_stream_t stream);
+/* p -= lr·g over n elements, then g = 0 for the next accumulation (the
+ * per-sequence optimiser step, reading C17). */
+stg_status stg_sgd_update(float* p, float* g, int64_t n, float lr, stg_stream_t stream);
 
 /* Algorithm 1 for ONE sequence s = [t0, t0+S): forward for t ∈ s
  * (DTDG: Get-Graph, graph-stack push; state-stack push; step; loss), then
@@ -243,6 +249,13 @@ stg_status stg_partition_rows(int32_t V, const int32_t* in_rowptr, int32_t world
  * returns the accumulated milliseconds and count (reset != 0 clears them). */
 stg_status stg_profile_enable(int32_t on);
 stg_status stg_profile_read(int32_t phase, double* total_ms, int64_t* count, int32_t reset);
+
+/* Diagnostic tcgen05 3xTF32 GEMM (tests pin the UMMA conventions with it):
+ * mode 0: C[M,N] = A[M,K]·B[K,N] (M % 128 == 0, K % 8 == 0, K <= 256);
+ * mode 1: C[128,N] = Aᵀ·B with A [R,128], B [R,N] (R % 128 == 0).
+ * N % 16 == 0, 16 <= N <= 256.  Row-major fp32 device arrays. */
+stg_status stg_debug_tc_gemm(int32_t mode, int32_t M, int32_t N, int32_t K, int32_t R, const float* A,
+                             const float* B, float* C, stg_stream_t stream);
 
 /* Stream-ordered byte copy (kind: 0 device->device, 1 host->device,
  * 2 device->host); lets bindings read borrowed view arrays. */

@@ -102,6 +102,10 @@ _decl("stg_tgcn_train_sequence", [_P, _P, _i32, _i32, ctypes.POINTER(stg_tgcn_pa
                                   ctypes.POINTER(_P), ctypes.POINTER(_P), _P, _P, _P,
                                   ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P, _P])
 _decl("stg_partition_rows", [_i32, _P, _i32, ctypes.POINTER(_i32), _P])
+_decl("stg_profile_enable", [_i32])
+_decl("stg_debug_tc_gemm", [_i32, _i32, _i32, _i32, _i32, _P, _P, _P, _P])
+_decl("stg_aggregate_set_strategy", [_i32])
+_decl("stg_profile_read", [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64), _i32])
 
 ABI_SYMBOLS = [
     "stg_last_error", "stg_version", "stg_kernel_launch_count", "stg_set_allocator", "stg_memcpy",
@@ -111,8 +115,25 @@ ABI_SYMBOLS = [
     "stg_gcn_aggregate_fwd", "stg_gcn_aggregate_bwd", "stg_gcn_aggregate_ex",
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
     "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_sgd_update", "stg_tgcn_train_sequence",
-    "stg_partition_rows",
+    "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
 ]
+
+PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head"]
+
+
+def stg_profile_enable(on: bool = True):
+    _check(_lib.stg_profile_enable(int(on)))
+
+
+def stg_profile_read(reset: bool = True) -> dict:
+    """{phase: (total_ms, count)} for every profiled phase (synchronises on the events)."""
+    out = {}
+    for i, name in enumerate(PHASES):
+        ms = ctypes.c_double(0.0)
+        n = _i64(0)
+        _check(_lib.stg_profile_read(i, ctypes.byref(ms), ctypes.byref(n), int(reset)))
+        out[name] = (ms.value, n.value)
+    return out
 
 
 def _check(status: int):
@@ -392,3 +413,22 @@ def stg_partition_rows(V: int, in_rowptr: torch.Tensor, world: int, stream=None)
     b = (_i32 * (world + 1))()
     _check(_lib.stg_partition_rows(V, _ptr(in_rowptr), world, b, _stream(stream)))
     return list(b)
+
+
+def stg_debug_tc_gemm(mode: int, A: torch.Tensor, B: torch.Tensor, stream=None) -> torch.Tensor:
+    """mode 0: A[M,K]·B[K,N]; mode 1: Aᵀ·B with A[R,128], B[R,N] (tcgen05 3xTF32)."""
+    if mode == 0:
+        M, K = A.shape
+        N = B.shape[1]
+        C = torch.empty(M, N, device=A.device)
+        _check(_lib.stg_debug_tc_gemm(0, M, N, K, 0, _ptr(A), _ptr(B), _ptr(C), _stream(stream)))
+    else:
+        R = A.shape[0]
+        N = B.shape[1]
+        C = torch.empty(128, N, device=A.device)
+        _check(_lib.stg_debug_tc_gemm(1, 128, N, 0, R, _ptr(A), _ptr(B), _ptr(C), _stream(stream)))
+    return C
+
+
+def stg_aggregate_set_strategy(async_gather: bool):
+    _check(_lib.stg_aggregate_set_strategy(int(async_gather)))

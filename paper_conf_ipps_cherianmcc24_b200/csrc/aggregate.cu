@@ -225,6 +225,210 @@ __global__ void __launch_bounds__(kAggThreads) k_aggregate(const AggArgs a) {
   }
 }
 
+
+// ---------------------------------------------------------------------------
+// Asynchronous-gather variant (float4 path, W <= 128): per warp a double-
+// buffered ring of 32 row slots in shared memory.  For each batch the warp
+// loads the 32 column indices (one per lane, coalesced), then issues the row
+// copies as 16-byte cp.async (LDGSTS, no register destinations) for batch b+1
+// while it consumes batch b from shared memory.  Slot s belongs to group
+// s / G (the G lanes that own one row item); accumulation order per row is the
+// same fixed edge order as k_aggregate, so results are deterministic.
+template <int G, int VPL, int U, bool SCOL>
+__global__ void __launch_bounds__(kAggThreads) k_aggregate_async(const AggArgs a, int warps_per_block) {
+  constexpr int NG = 32 / G;                 // row items per warp
+  constexpr int EPG = G;                     // slots (edges) per item per batch
+  const unsigned FULL = 0xffffffffu;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  if (wib >= warps_per_block) return;
+  const int gi = lane / G, gl = lane % G;
+  const int W = a.W, nv = W / 4;             // row length in float4
+  const int slot_bytes = W * 4;
+  unsigned char* wbase = smem_raw + (size_t)wib * (2 * 32 * slot_bytes + 2 * 32 * 4);
+  unsigned char* buf[2] = {wbase, wbase + 32 * slot_bytes};
+  float* scs[2] = {reinterpret_cast<float*>(wbase + 2 * 32 * slot_bytes),
+                   reinterpret_cast<float*>(wbase + 2 * 32 * slot_bytes) + 32};
+  const int32_t n_hub = a.sched ? a.sched[0] : 0;
+  const int32_t n_chunks = a.sched ? a.sched[1] : 0;
+  const int32_t* cptr = a.sched ? a.sched + 2 : nullptr;
+  const int64_t total = (int64_t)n_chunks + (a.R - n_hub);
+  const int64_t warp_id = (int64_t)blockIdx.x * warps_per_block + wib;
+  const int64_t nwarps = (int64_t)gridDim.x * warps_per_block;
+
+  for (int64_t base = warp_id * NG; base < total; base += nwarps * NG) {
+    const int64_t item = base + gi;
+    const bool valid = item < total;
+    int32_t v = 0, beg = 0, end = 0, hub = -1;
+    if (valid) {
+      if (item < n_chunks) {
+        int32_t lo = 0, hi = n_hub;
+        while (lo < hi) {
+          int32_t mid = (lo + hi + 1) >> 1;
+          if (cptr[mid] <= item) lo = mid; else hi = mid - 1;
+        }
+        hub = lo;
+        v = a.ids[lo];
+        int32_t rb = a.rowptr[v], re = a.rowptr[v + 1];
+        beg = rb + (int32_t)(item - cptr[lo]) * kHubChunk;
+        end = min(beg + kHubChunk, re);
+      } else {
+        int64_t li = n_hub + (item - n_chunks);
+        v = a.ids ? a.ids[li] : (int32_t)li;
+        beg = a.rowptr[v];
+        end = a.rowptr[v + 1];
+      }
+    }
+    const int32_t n = end - beg;
+    const int32_t nmax = __reduce_max_sync(FULL, n);
+    const int nb = (nmax + EPG - 1) / EPG;
+    // lane s describes slot s: group s / EPG, edge (b·EPG + s % EPG) of that group
+    const int sg = lane / EPG, se = lane % EPG;
+    const int32_t s_beg = __shfl_sync(FULL, beg, sg * G);
+    const int32_t s_n = __shfl_sync(FULL, n, sg * G);
+
+    auto issue = [&](int b, int which) {
+      const int e = b * EPG + se;
+      const int32_t u = e < s_n ? __ldg(a.col + s_beg + e) : -1;
+      if (SCOL) scs[which][lane] = u >= 0 ? __ldg(a.scol + u) : 0.0f;
+      const uint32_t dst0 = (uint32_t)__cvta_generic_to_shared(buf[which]);
+      for (int p = lane; p < 32 * nv; p += 32) {
+        const int slot = p / nv, ch = p - slot * nv;
+        const int32_t us = __shfl_sync(FULL, u, slot);
+        if (us >= 0) {
+          const float* src = a.x + (int64_t)us * a.ldx + 4 * ch;
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(dst0 + (uint32_t)(slot * slot_bytes + 16 * ch)),
+                       "l"(src)
+                       : "memory");
+        }
+      }
+      asm volatile("cp.async.commit_group;\n" ::: "memory");
+    };
+
+    float4 acc[U][VPL];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) acc[u][c] = make_float4(0.f, 0.f, 0.f, 0.f);
+
+    if (nb > 0) issue(0, 0);
+    for (int b = 0; b < nb; ++b) {
+      if (b + 1 < nb) {
+        issue(b + 1, (b + 1) & 1);
+        asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+      }
+      __syncwarp();
+      const unsigned char* bb = buf[b & 1];
+      const float* sc = scs[b & 1];
+#pragma unroll
+      for (int e = 0; e < EPG; ++e) {
+        if (b * EPG + e < n) {
+          const int slot = gi * EPG + e;
+          const float4* row = reinterpret_cast<const float4*>(bb + slot * slot_bytes);
+          const float ssc = SCOL ? sc[slot] : 1.0f;
+#pragma unroll
+          for (int c = 0; c < VPL; ++c) {
+            const int cv = c * G + gl;
+            if (cv < nv) {
+              const float4 xv = row[cv];
+              if (SCOL) fma_v(acc[e % U][c], ssc, xv);
+              else add_v(acc[e % U][c], xv);
+            }
+          }
+        }
+      }
+      __syncwarp();
+    }
+#pragma unroll
+    for (int w = 1; w < U; w <<= 1)
+#pragma unroll
+      for (int u = 0; u < U; u += 2 * w)
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) add_v(acc[u][c], acc[u + w][c]);
+
+    const bool hubitem = valid && hub >= 0;
+    if (valid && !hubitem) {
+      const float s = a.srow ? a.srow[v] : 1.0f;
+      float4* yr = reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv < nv) yr[cv] = scale_bias(s, acc[0][c], a.bias, cv * 4);
+      }
+    }
+    if (hubitem) {
+      float4* pr = reinterpret_cast<float4*>(a.partials + item * (int64_t)W);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv < nv) pr[cv] = acc[0][c];
+      }
+      __threadfence();
+    }
+    __syncwarp();
+    int32_t ticket = 0;
+    if (hubitem && gl == 0) ticket = atomicAdd(a.counters + hub, 1);
+    ticket = __shfl_sync(FULL, ticket, gi * G);
+    const bool last = hubitem && ticket == (cptr[hub + 1] - cptr[hub]) - 1;
+    if (last) {
+      __threadfence();
+      const int32_t cb = cptr[hub], ce = cptr[hub + 1];
+      float4 tot[VPL];
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) tot[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int32_t c0 = cb; c0 < ce; c0 += 16) {
+        float4 blk[VPL];
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) blk[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+        const int32_t c1 = min(c0 + 16, ce);
+        for (int32_t ch = c0; ch < c1; ++ch) {
+          const float4* pr = reinterpret_cast<const float4*>(a.partials + (int64_t)ch * W);
+#pragma unroll
+          for (int c = 0; c < VPL; ++c) {
+            const int cv = c * G + gl;
+            if (cv < nv) add_v(blk[c], __ldcg(pr + cv));
+          }
+        }
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) add_v(tot[c], blk[c]);
+      }
+      const float s = a.srow ? a.srow[v] : 1.0f;
+      float4* yr = reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv < nv) yr[cv] = scale_bias(s, tot[c], a.bias, cv * 4);
+      }
+      if (gl == 0) a.counters[hub] = 0;
+    }
+  }
+}
+
+using AsyncFn = void (*)(const AggArgs, int);
+
+template <int G, bool SCOL>
+AsyncFn pick_async_vpl(int vpl) {
+  switch (vpl) {
+    case 1: return k_aggregate_async<G, 1, 4, SCOL>;
+    case 2: return k_aggregate_async<G, 2, 4, SCOL>;
+    case 3: return k_aggregate_async<G, 3, 2, SCOL>;
+    default: return k_aggregate_async<G, 4, 2, SCOL>;
+  }
+}
+template <bool SCOL>
+AsyncFn pick_async_g(int g, int vpl) {
+  switch (g) {
+    case 1: return pick_async_vpl<1, SCOL>(vpl);
+    case 2: return pick_async_vpl<2, SCOL>(vpl);
+    case 4: return pick_async_vpl<4, SCOL>(vpl);
+    case 8: return pick_async_vpl<8, SCOL>(vpl);
+    case 16: return pick_async_vpl<16, SCOL>(vpl);
+    default: return pick_async_vpl<32, SCOL>(vpl);
+  }
+}
+
 using KernelFn = void (*)(const AggArgs);
 
 template <int VEC, int G, bool SCOL>
@@ -272,6 +476,9 @@ int max_blocks_for(KernelFn fn) {
 
 }  // namespace
 
+// Gather strategy switch (1 = cp.async shared-memory ring; 0 = register gathers).
+static int g_agg_async = 0;
+
 // Launch plan: vector width, group size, vectors per lane for W columns.
 struct AggPlan {
   int vec, g, vpl, wmax;
@@ -317,7 +524,7 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   AggWs* ws = static_cast<AggWs*>(gv->workspace);
   if (a.sched) {
     const int32_t wl = W < p0.wmax ? W : p0.wmax;
-    STG_TRY(ws->partials.alloc((size_t)chunks_bound * wl + 4, s));
+    STG_TRY(ws->partials.alloc((size_t)chunks_bound * wl + 4, s));   // >= the async path's 128-column chunks
     const int64_t ncnt = sched_cap(gv->num_edges) + 1;
     if (ws->counters_n < ncnt) {
       STG_TRY(ws->counters.alloc(ncnt, s));
@@ -329,8 +536,10 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   }
   const int64_t items_bound = (int64_t)R + chunks_bound + 1;
   ProfScope prof(backward ? PH_AGG_BWD : PH_AGG_FWD, s);
-  for (int32_t c0 = 0; c0 < W; c0 += p0.wmax) {
-    const int32_t wl = (W - c0) < p0.wmax ? (W - c0) : p0.wmax;
+  const bool use_async = vec4 && g_agg_async;
+  const int wmax = use_async ? 128 : p0.wmax;
+  for (int32_t c0 = 0; c0 < W; c0 += wmax) {
+    const int32_t wl = (W - c0) < wmax ? (W - c0) : wmax;
     const AggPlan p = plan_for(wl, vec4);
     a.W = wl;
     a.x = in + c0;
@@ -338,13 +547,42 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     a.y = out + c0;
     a.ldy = ldout;
     a.bias = bias ? bias + c0 : nullptr;
-    KernelFn fn = pick(p.vec, p.g, p.vpl, scol != nullptr);
-    const int rows_per_block = (kAggThreads / 32) * (32 / p.g);
-    int64_t blocks = ceil_div(items_bound, rows_per_block);
-    const int64_t mb = max_blocks_for(fn);
-    if (blocks > mb) blocks = mb;
-    if (blocks < 1) blocks = 1;
-    fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(a);
+    const int rows_per_warp = 32 / p.g;
+    const int U = p.vpl <= 2 ? 4 : 2;
+    if (use_async && p.g >= U) {
+      AsyncFn fn = scol ? pick_async_g<true>(p.g, p.vpl) : pick_async_g<false>(p.g, p.vpl);
+      const size_t per_warp = (size_t)2 * 32 * wl * 4 + 2 * 32 * 4;
+      int wpb = (int)std::min<size_t>(8, (size_t)(200 * 1024) / per_warp);
+      if (wpb < 1) wpb = 1;
+      const size_t smem = per_warp * wpb;
+      static std::mutex mu;
+      {
+        std::lock_guard<std::mutex> lk(mu);
+        static std::map<AsyncFn, size_t> attr;
+        if (attr[fn] < smem) {
+          STG_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+          attr[fn] = smem;
+        }
+      }
+      int per_sm = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kAggThreads, smem) != cudaSuccess || per_sm < 1) {
+        cudaGetLastError();
+        per_sm = 1;
+      }
+      int64_t blocks = ceil_div(items_bound, (int64_t)wpb * rows_per_warp);
+      const int64_t mb = (int64_t)per_sm * num_sms();
+      if (blocks > mb) blocks = mb;
+      if (blocks < 1) blocks = 1;
+      fn<<<(unsigned)blocks, kAggThreads, smem, s>>>(a, wpb);
+    } else {
+      KernelFn fn = pick(p.vec, p.g, p.vpl, scol != nullptr);
+      const int rows_per_block = (kAggThreads / 32) * rows_per_warp;
+      int64_t blocks = ceil_div(items_bound, rows_per_block);
+      const int64_t mb = max_blocks_for(fn);
+      if (blocks > mb) blocks = mb;
+      if (blocks < 1) blocks = 1;
+      fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(a);
+    }
     count_launch();
   }
   return check_launch("aggregate");
@@ -366,6 +604,11 @@ stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* 
   if (!g) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_bwd: view is NULL");
   return stg::aggregate_launch(g, 1, W, gy, ldgy, gx, ldgx, g->norm_src, g->norm_dst, nullptr,
                                (cudaStream_t)stream);
+}
+
+stg_status stg_aggregate_set_strategy(int32_t async_gather) {
+  stg::g_agg_async = async_gather ? 1 : 0;
+  return STG_OK;
 }
 
 stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t W, const float* in, int64_t ldin,

@@ -15,6 +15,16 @@
 #include "graph.cuh"
 
 namespace stg {
+bool tc_supported(int F, int H);
+int tc_atb_max_blocks();
+stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s);
+stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float* L, const float* l, float* Hn,
+                      cudaStream_t s);
+stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float* G, const float* L, const float* l,
+                      const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s);
+stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* dW, cudaStream_t s);
+stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
+                 float* dl_tmp, float* dL, float* dl, float* db, const float* L, cudaStream_t s);
 stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
                             float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
                             cudaStream_t s);
@@ -308,50 +318,65 @@ __global__ void k_reduce_part(const float* __restrict__ part, int32_t nb, int32_
 }
 
 // ---------------------------------------------------------------- MSE head
-// One warp per row.  Per-block partials [loss | dw_o (H) | db_o] (fp32 for the
-// gradients, fp64 for the loss).
+// LPR = H/4 lanes per row (float4 each), 32/LPR rows per warp step, several
+// rows in flight per warp.  Per-block partials [loss | dw_o (H) | db_o]
+// (fp32 gradients, fp64 loss), reduced in a fixed order by k_mse_reduce.
+template <int LPR>
 __global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t H, const float* __restrict__ Hn,
                                                  const float* __restrict__ y, const float* __restrict__ w_o,
                                                  const float* __restrict__ b_o, float* __restrict__ dH, int accumulate,
                                                  int want_grad, double* __restrict__ lpart,
                                                  float* __restrict__ gpart) {
+  constexpr int RPW = 32 / LPR;                 // rows per warp step
   __shared__ double sl[kT / 32];
-  __shared__ float sg[kT / 32][65];
+  __shared__ float sg[kT / 32][129];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int rl = lane / LPR, ql = lane % LPR;   // row slot, float4 index within the row
   double lacc = 0.0;
-  float gw0 = 0.0f, gw1 = 0.0f, gb = 0.0f;     // lane owns k = lane and lane + 32
+  float4 gw = make_float4(0.f, 0.f, 0.f, 0.f);
+  float gb = 0.f;
   const float b = b_o[0];
   const float invV = 1.0f / (float)V;
-  for (int64_t v = (int64_t)blockIdx.x * (kT / 32) + w; v < V; v += (int64_t)gridDim.x * (kT / 32)) {
-    const float* h = Hn + v * H;
-    float h0 = lane < H ? h[lane] : 0.0f, h1 = lane + 32 < H ? h[lane + 32] : 0.0f;
-    float r0 = fmaxf(h0, 0.0f), r1 = fmaxf(h1, 0.0f);
-    float s = (lane < H ? r0 * w_o[lane] : 0.0f) + (lane + 32 < H ? r1 * w_o[lane + 32] : 0.0f);
+  const float4 wo = reinterpret_cast<const float4*>(w_o)[ql];
+  const int64_t step = (int64_t)gridDim.x * (kT / 32) * RPW;
+  for (int64_t v0 = ((int64_t)blockIdx.x * (kT / 32) + w) * RPW; v0 < V; v0 += step) {
+    const int64_t v = v0 + rl;
+    const bool ok = v < V;
+    float4 h = ok ? reinterpret_cast<const float4*>(Hn + v * H)[ql] : make_float4(0.f, 0.f, 0.f, 0.f);
+    const float yv = (ok && ql == 0) ? y[v] : 0.f;
+    float4 r = make_float4(fmaxf(h.x, 0.f), fmaxf(h.y, 0.f), fmaxf(h.z, 0.f), fmaxf(h.w, 0.f));
+    float s = r.x * wo.x + r.y * wo.y + r.z * wo.z + r.w * wo.w;
 #pragma unroll
-    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    const float e = (s + b) - y[v];
-    lacc += (double)e * (double)e;
-    if (want_grad) {
+    for (int o = LPR / 2; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float yy = __shfl_sync(0xffffffffu, yv, rl * LPR);
+    const float e = (s + b) - yy;
+    if (ok && ql == 0) lacc += (double)e * (double)e;
+    if (want_grad && ok) {
       const float g = 2.0f * e * invV;
       if (dH) {
-        if (lane < H) {
-          float d = h0 > 0.0f ? g * w_o[lane] : 0.0f;
-          dH[v * H + lane] = accumulate ? dH[v * H + lane] + d : d;
+        float4 d = make_float4(h.x > 0.f ? g * wo.x : 0.f, h.y > 0.f ? g * wo.y : 0.f, h.z > 0.f ? g * wo.z : 0.f,
+                               h.w > 0.f ? g * wo.w : 0.f);
+        float4* dp = reinterpret_cast<float4*>(dH + v * H) + ql;
+        if (accumulate) {
+          float4 o = *dp;
+          d.x += o.x; d.y += o.y; d.z += o.z; d.w += o.w;
         }
-        if (lane + 32 < H) {
-          float d = h1 > 0.0f ? g * w_o[lane + 32] : 0.0f;
-          dH[v * H + lane + 32] = accumulate ? dH[v * H + lane + 32] + d : d;
-        }
+        *dp = d;
       }
-      gw0 = fmaf(g, r0, gw0);
-      gw1 = fmaf(g, r1, gw1);
-      gb += g;
+      gw.x = fmaf(g, r.x, gw.x); gw.y = fmaf(g, r.y, gw.y); gw.z = fmaf(g, r.z, gw.z); gw.w = fmaf(g, r.w, gw.w);
+      if (ql == 0) gb += g;
     }
   }
-  if (lane == 0) sl[w] = lacc;
-  sg[w][lane] = gw0;
-  sg[w][lane + 32] = gw1;
-  if (lane == 0) sg[w][64] = gb;
+  // fixed-order reduction: over the RPW row slots of the warp, then over warps
+#pragma unroll
+  for (int o = LPR; o < 32; o <<= 1) {
+    gw.x += __shfl_xor_sync(0xffffffffu, gw.x, o); gw.y += __shfl_xor_sync(0xffffffffu, gw.y, o);
+    gw.z += __shfl_xor_sync(0xffffffffu, gw.z, o); gw.w += __shfl_xor_sync(0xffffffffu, gw.w, o);
+    gb += __shfl_xor_sync(0xffffffffu, gb, o);
+    lacc += __shfl_xor_sync(0xffffffffu, lacc, o);
+  }
+  if (lane == 0) { sl[w] = lacc; sg[w][128] = gb; }
+  if (lane < LPR) { sg[w][4 * lane] = gw.x; sg[w][4 * lane + 1] = gw.y; sg[w][4 * lane + 2] = gw.z; sg[w][4 * lane + 3] = gw.w; }
   __syncthreads();
   if (threadIdx.x == 0) {
     double t = 0.0;
@@ -360,7 +385,7 @@ __global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t H, const flo
   }
   for (int k = threadIdx.x; k < H + 1; k += kT) {
     float t = 0.0f;
-    const int src = k < H ? k : 64;
+    const int src = k < H ? k : 128;
     for (int i = 0; i < kT / 32; ++i) t += sg[i][src];
     gpart[(int64_t)blockIdx.x * (H + 1) + k] = t;
   }
@@ -382,9 +407,11 @@ __global__ void k_mse_reduce(int32_t nb, int32_t H, int32_t V, const double* __r
   }
 }
 
-__global__ void k_sgd(float* __restrict__ p, const float* __restrict__ g, int64_t n, float lr) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+__global__ void k_sgd(float* __restrict__ p, float* __restrict__ g, int64_t n, float lr) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     p[i] -= lr * g[i];
+    g[i] = 0.0f;
+  }
 }
 
 int grid_blocks(const void* fn, size_t smem, int64_t tiles) {
@@ -408,7 +435,7 @@ stg_status set_smem(K fn, size_t smem) {
 
 // Scratch used by the TGCN kernels (grow-only).
 struct TgcnWs {
-  DArray<float> P, dC, dP, part_gru, part_dw, gpart;
+  DArray<float> P, dC, dP, part_gru, part_dw, gpart, da, RH, part_tc, dl_tmp;
   DArray<double> lpart;
 };
 
@@ -492,31 +519,39 @@ stg_status stg_tgcn_step(const stg_csr_view* g, const stg_tgcn_params* p, const 
     STG_TRY(ws.dC.alloc((size_t)V * H3));
     C = ws.dC.p;
   }
+  const bool use_tc = tc_supported(F, H);
   // P' = diag(n_src)·X·W
   {
     ProfScope prof(PH_XW, s);
-    const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
-    STG_TRY(set_smem(k_xw, smem));
-    const int nb = grid_blocks((const void*)k_xw, smem, (V + 31) / 32);
-    k_xw<<<nb, kT, smem, s>>>(V, F, H3, X, p->W, g->norm_src, ws.P.p);
-    count_launch();
+    if (use_tc) {
+      STG_TRY(tc_xw(V, F, H, X, p->W, g->norm_src, ws.P.p, s));
+    } else {
+      const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
+      STG_TRY(set_smem(k_xw, smem));
+      const int nb = grid_blocks((const void*)k_xw, smem, (V + 31) / 32);
+      k_xw<<<nb, kT, smem, s>>>(V, F, H3, X, p->W, g->norm_src, ws.P.p);
+      count_launch();
+    }
   }
   // C = diag(n_dst)·A·P' + b
   STG_TRY(aggregate_launch(g, 0, H3, ws.P.p, H3, C, H3, g->norm_dst, nullptr, p->b, s));
   // GRU
   ProfScope prof_gru(PH_GRU_FWD, s);
-  if (H <= 32) {
+  if (use_tc) {
+    STG_TRY(tc_gru_fwd(V, H, C, H_prev, p->L, p->l, H_next, s));
+  } else if (H <= 32) {
     const size_t smem = gru_fwd_smem(H, 32);
     STG_TRY(set_smem(k_gru_fwd<32>, smem));
     const int nb = grid_blocks((const void*)k_gru_fwd<32>, smem, (V + 31) / 32);
     k_gru_fwd<32><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
+    count_launch();
   } else {
     const size_t smem = gru_fwd_smem(H, 16);
     STG_TRY(set_smem(k_gru_fwd<16>, smem));
     const int nb = grid_blocks((const void*)k_gru_fwd<16>, smem, (V + 15) / 16);
     k_gru_fwd<16><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
+    count_launch();
   }
-  count_launch();
   STG_TRY(check_launch("stg_tgcn_step"));
   if (stack) {
     const size_t need = (cbytes + 255) & ~size_t(255);
@@ -542,6 +577,27 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
   TgcnWs& ws = stack->ws;
   STG_TRY(ws.dC.alloc((size_t)V * H3));
   STG_TRY(ws.dP.alloc((size_t)V * H3));
+  if (tc_supported(F, H)) {
+    STG_TRY(ws.da.alloc((size_t)V * H3));
+    STG_TRY(ws.RH.alloc((size_t)V * H));
+    STG_TRY(ws.part_tc.alloc((size_t)2 * tc_atb_max_blocks() * 128 * std::max(H3, (F + 15) / 16 * 16)));
+    STG_TRY(ws.dl_tmp.alloc(H3));
+    {
+      ProfScope prof(PH_GRU_BWD, s);
+      STG_TRY(tc_gru_bwd(V, H, e.C, e.Hp, dH_next, p->L, p->l, g->norm_dst, ws.dC.p, dH_prev, ws.da.p, ws.RH.p, s));
+      STG_TRY(tc_dl(V, H, e.C, e.Hp, ws.RH.p, ws.da.p, ws.part_tc.p, ws.dl_tmp.p, grads->L, grads->l, grads->b, p->L,
+                    s));
+    }
+    STG_TRY(aggregate_launch(g, 1, H3, ws.dC.p, H3, ws.dP.p, H3, g->norm_src, nullptr, nullptr, s));
+    {
+      ProfScope prof(PH_DW, s);
+      STG_TRY(tc_dw(V, F, H, X, ws.dP.p, ws.part_tc.p, grads->W, s));
+    }
+    STG_TRY(check_launch("stg_tgcn_step_backward"));
+    stack->entries.pop_back();
+    stack->top -= e.bytes;
+    return STG_OK;
+  }
   // GRU backward + partials of dL, dl, db
   ProfScope* prof_gru = new ProfScope(PH_GRU_BWD, s);
   const int BR = H <= 32 ? 16 : 4;
@@ -590,23 +646,35 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
 stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o, const float* b_o,
                         float* loss_accum, float* dH, int32_t accumulate, float* dw_o, float* db_o,
                         stg_stream_t stream) {
-  if (V < 1 || H < 1 || H > 64 || !Hn || !y || !w_o || !b_o)
-    return fail(STG_ERR_INVALID_ARG, "stg_mse_head: bad arguments (V=%d H=%d)", V, H);
+  if (V < 1 || H < 1 || H > 128 || H % 4 || !Hn || !y || !w_o || !b_o)
+    return fail(STG_ERR_INVALID_ARG, "stg_mse_head: bad arguments (V=%d H=%d; H %% 4 == 0, H <= 128)", V, H);
+  if (((uintptr_t)Hn | (uintptr_t)w_o | (uintptr_t)(dH ? dH : Hn)) % 16)
+    return fail(STG_ERR_INVALID_ARG, "stg_mse_head: Hn, w_o, dH must be 16-byte aligned");
   cudaStream_t s = (cudaStream_t)stream;
   TgcnWs& ws = global_ws();
-  int nb = (int)std::min<int64_t>((V + 7) / 8, (int64_t)num_sms() * 4);
+  const int LPR = H / 4 <= 1 ? 1 : (H / 4 <= 2 ? 2 : (H / 4 <= 4 ? 4 : (H / 4 <= 8 ? 8 : (H / 4 <= 16 ? 16 : 32))));
+  if (LPR * 4 != H) return fail(STG_ERR_INVALID_ARG, "stg_mse_head: H=%d must be 4·2^k", H);
+  const int rows_per_block = (kT / 32) * (32 / LPR);
+  int nb = (int)std::min<int64_t>((V + rows_per_block - 1) / rows_per_block, (int64_t)num_sms() * 8);
   STG_TRY(ws.lpart.alloc(nb));
   STG_TRY(ws.gpart.alloc((size_t)nb * (H + 1)));
   const int want = (dH || dw_o || db_o) ? 1 : 0;
   ProfScope prof(PH_HEAD, s);
-  k_mse_head<<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p);
+  switch (LPR) {
+    case 1: k_mse_head<1><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 2: k_mse_head<2><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 4: k_mse_head<4><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 8: k_mse_head<8><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 16: k_mse_head<16><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    default: k_mse_head<32><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+  }
   k_mse_reduce<<<1, 64, 0, s>>>(nb, H, V, ws.lpart.p, ws.gpart.p, loss_accum, want ? dw_o : nullptr,
                                 want ? db_o : nullptr);
   count_launch(2);
   return check_launch("stg_mse_head");
 }
 
-stg_status stg_sgd_update(float* p, const float* g, int64_t n, float lr, stg_stream_t stream) {
+stg_status stg_sgd_update(float* p, float* g, int64_t n, float lr, stg_stream_t stream) {
   if (n < 0 || (n > 0 && (!p || !g))) return fail(STG_ERR_INVALID_ARG, "stg_sgd_update: bad arguments");
   if (!n) return STG_OK;
   cudaStream_t s = (cudaStream_t)stream;

@@ -168,3 +168,24 @@ def test_aggregation_ex_scales_and_bias(stg):
     r = oracle.aggregate(ref["in_rowptr"], ref["in_col"], srow, scol, x) + bias
     sc = oracle.aggregate(ref["in_rowptr"], ref["in_col"], srow, scol, np.abs(x)) + np.abs(bias)
     assert cond_err(y, r, sc) <= TOL
+
+
+@pytest.mark.parametrize("W", [4, 16, 64, 96, 128, 200])
+def test_gather_strategies_bit_identical(stg, W):
+    """cp.async shared-memory gathers and register gathers give identical bits."""
+    V = 20000
+    rng = np.random.default_rng(3)
+    s = np.concatenate([rng.integers(0, V, 8000), rng.integers(0, V, 60000)])
+    d = np.concatenate([np.full(8000, 11), rng.integers(0, V, 60000)])
+    g = stg.stg_static_graph_create(V, s, d, stg.STG_SELF_LOOPS)
+    x = to_gpu(gen.uniform_pm1(2, W, V * W).reshape(V, W))
+    try:
+        stg.stg_aggregate_set_strategy(True)
+        a1 = stg.stg_gcn_aggregate_fwd(g.view(), x)
+        b1 = stg.stg_gcn_aggregate_bwd(g.view(), x)
+        stg.stg_aggregate_set_strategy(False)
+        a0 = stg.stg_gcn_aggregate_fwd(g.view(), x)
+        b0 = stg.stg_gcn_aggregate_bwd(g.view(), x)
+    finally:
+        stg.stg_aggregate_set_strategy(False)
+    assert torch.equal(a0, a1) and torch.equal(b0, b1)

@@ -1,8 +1,11 @@
 """GPU parity: TGCN step forward/backward and Algorithm 1 sequences vs the oracle.
 
 Tolerances: H' is compared in absolute terms (|H'| < 1)
-at 2e-5; parameter gradients normwise per tensor at 1e-4 · max|ref|; the
-sequence loss at 1e-5 relative.
+at 2e-5; the sequence loss at 1e-5 relative; parameter gradients normwise per
+tensor at g_tol(n) = max(1e-4, 1e-6·sqrt(n)) · max|ref|, n = rows reduced
+(V · timestamps): a gradient is a sum of n row terms of random sign, so its
+norm is ~sqrt(n) times smaller than the sum of |terms| that bounds the fp32 /
+3xTF32 rounding (per-term relative error <= 2^-20).
 """
 import numpy as np
 import pytest
@@ -16,6 +19,10 @@ pytestmark = pytest.mark.gpu
 
 H_TOL = 2e-5
 G_TOL = 1e-4
+
+
+def g_tol(n_rows: int) -> float:
+    return max(1e-4, 1e-6 * float(np.sqrt(n_rows)))
 
 
 def _params(F, H, seed):
@@ -69,7 +76,7 @@ def test_tgcn_step_parity(stg, name, H):
     assert _normwise(dHp.cpu().numpy(), rdH) <= G_TOL
     for k in ("W", "b", "L", "l"):
         e = _normwise(grads[k].cpu().numpy(), rg[k])
-        assert e <= G_TOL, (k, e)
+        assert e <= g_tol(V), (k, e)
 
 
 def test_tgcn_inference_and_stack_errors(stg):
@@ -130,9 +137,9 @@ def test_train_sequence_static(stg, name):
     assert abs(loss - rl) <= 1e-5 * abs(rl)
     assert np.max(np.abs(Hseq[-1].cpu().numpy() - rH)) <= H_TOL
     for k in ("W", "b", "L", "l"):
-        assert _normwise(grads[k].cpu().numpy(), rg[k]) <= G_TOL, k
-    assert _normwise(dw.cpu().numpy(), rg["w_o"]) <= G_TOL
-    assert _normwise(db.cpu().numpy(), rg["b_o"]) <= G_TOL
+        assert _normwise(grads[k].cpu().numpy(), rg[k]) <= g_tol(cfg.V * S), k
+    assert _normwise(dw.cpu().numpy(), rg["w_o"]) <= g_tol(cfg.V * S)
+    assert _normwise(db.cpu().numpy(), rg["b_o"]) <= g_tol(cfg.V * S)
 
 
 @pytest.mark.parametrize("name", ["C4", "C5s"])
@@ -156,7 +163,7 @@ def test_train_sequence_dtdg(stg, name):
         assert abs(loss - rl) <= 1e-5 * abs(rl), (t0, loss, rl)
         assert np.max(np.abs(Hseq[-1].cpu().numpy() - rH)) <= H_TOL
         for k in ("W", "b", "L", "l"):
-            assert _normwise(grads[k].cpu().numpy(), rg[k]) <= G_TOL, (t0, k)
+            assert _normwise(grads[k].cpu().numpy(), rg[k]) <= g_tol(cfg.V * S), (t0, k)
         H0 = rH
         Hc = Hseq[-1].clone()
 
@@ -166,3 +173,4 @@ def test_sgd_update(stg):
     g = torch.ones(10, device="cuda")
     stg.stg_sgd_update(p, g, 0.5)
     assert torch.equal(p, torch.arange(10, dtype=torch.float32, device="cuda") - 0.5)
+    assert torch.count_nonzero(g) == 0
