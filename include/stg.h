@@ -168,10 +168,14 @@ stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t
                                 const float* scale_row, const float* scale_col, const float* bias,
                                 stg_stream_t stream);
 
-/* Gather strategy of the aggregation kernel for the float4 path: 0 (default)
- * = register gathers; 1 = asynchronous cp.async copies of neighbour rows into
- * a per-warp shared-memory ring.  Results are bit-identical. */
-stg_status stg_aggregate_set_strategy(int32_t async_gather);
+/* Work decomposition of the aggregation kernel (float4 path):
+ * 0 (default) = degree-ordered row items (node_ids order, hub rows chunked;
+ *     FA-TGA lane groups, register gathers);  1 = as 0 with cp.async gathers;
+ * 2 = edge-parallel: warps stream contiguous 128-edge chunks of the CSR
+ *     (nnz-balanced) with TMA bulk row copies, rows split across chunks
+ *     finished in chunk order (W >= 64, views with the COO row array).
+ * Every strategy is deterministic; 0 and 1 are bit-identical. */
+stg_status stg_aggregate_set_strategy(int32_t strategy);
 
 /* ---- TGCN (GCN + GRU; reading C13-C15) ----
  * W [F,3H] (gates z|r|h), b [3H], L [3][2H][H] (gate g: rows 0..H-1 = L_g¹ act

@@ -430,5 +430,6 @@ def stg_debug_tc_gemm(mode: int, A: torch.Tensor, B: torch.Tensor, stream=None) 
     return C
 
 
-def stg_aggregate_set_strategy(async_gather: bool):
-    _check(_lib.stg_aggregate_set_strategy(int(async_gather)))
+def stg_aggregate_set_strategy(strategy: int):
+    """0 = degree-ordered row items (default), 1 = row items with cp.async gathers, 2 = edge-parallel TMA."""
+    _check(_lib.stg_aggregate_set_strategy(int(strategy)))

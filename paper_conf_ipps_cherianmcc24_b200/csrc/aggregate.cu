@@ -429,6 +429,294 @@ AsyncFn pick_async_g(int g, int vpl) {
   }
 }
 
+// ---------------------------------------------------------------------------
+// Edge-parallel ("merge-path") variant for W <= 128 float4 rows: warp w streams
+// the contiguous edge chunks c = w, w + nwarps, ... of kEdgeChunk edges.  Column
+// and row ids are read 32 at a time (coalesced) and broadcast; 8 feature-row
+// gathers are in flight per lane; a row is flushed when the row id changes.
+// Rows fully inside a chunk are written directly; a row split across chunks
+// [c_a, c_b] leaves one partial per chunk (slot 2c_a+1, then 2c for c > c_a) and
+// the last chunk to finish (atomic ticket per row, self-resetting) sums them in
+// chunk order.  Two accumulators alternate on edge parity: every fp32 chain is
+// <= 64 terms, results are deterministic, no float atomics.
+constexpr int kEdgeChunk = 128;
+
+struct EdgeArgs {
+  int32_t R;
+  int64_t E;
+  const int32_t* rowptr;
+  const int32_t* col;
+  const int32_t* row;
+  const float* srow;
+  const float* scol;
+  const float* bias;
+  int32_t W;
+  const float* x;
+  int64_t ldx;
+  float* y;
+  int64_t ldy;
+  float* partials;   // [2 * nchunks][W]
+  int32_t* counters; // [R]
+};
+
+__device__ __forceinline__ void edge_write_row(const EdgeArgs& a, int32_t r, float4 v, int lane, int nv) {
+  if (lane < nv) {
+    const float s = a.srow ? a.srow[r] : 1.0f;
+    reinterpret_cast<float4*>(a.y + (int64_t)r * a.ldy)[lane] = scale_bias(s, v, a.bias, 4 * lane);
+  }
+}
+
+template <bool SCOL>
+__global__ void __launch_bounds__(kAggThreads) k_agg_edges(const EdgeArgs a) {
+  constexpr int U = 8;
+  const unsigned FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const int nv = a.W / 4;
+  const int64_t nchunks = (a.E + kEdgeChunk - 1) / kEdgeChunk;
+  const int64_t warp_id = ((int64_t)blockIdx.x * kAggThreads + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * kAggThreads) >> 5;
+  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int64_t c = warp_id; c < nchunks; c += nwarps) {
+    const int64_t e0 = c * kEdgeChunk, e1 = (a.E < e0 + kEdgeChunk) ? a.E : e0 + kEdgeChunk;
+    const int32_t r_first = a.row[e0], r_last = a.row[e1 - 1];
+    const bool start_open = e0 > a.rowptr[r_first];
+    const bool end_open = e1 < a.rowptr[r_last + 1];
+    // empty rows in the gap before this chunk (and after the last chunk)
+    {
+      const int32_t gap0 = c == 0 ? 0 : a.row[e0 - 1] + 1;
+      for (int32_t r = gap0; r < r_first; ++r) edge_write_row(a, r, z4, lane, nv);
+      if (c == nchunks - 1)
+        for (int32_t r = r_last + 1; r < a.R; ++r) edge_write_row(a, r, z4, lane, nv);
+    }
+    int32_t cur = r_first;
+    float4 acc0 = z4, acc1 = z4;
+    auto flush = [&](int32_t r) {
+      float4 v = acc0;
+      add_v(v, acc1);
+      const bool open_s = (r == r_first) && start_open, open_e = (r == r_last) && end_open;
+      if (!open_s && !open_e) {
+        edge_write_row(a, r, v, lane, nv);
+        return;
+      }
+      const int64_t slot = open_s ? 2 * c : 2 * c + 1;
+      if (lane < nv) reinterpret_cast<float4*>(a.partials + slot * a.W)[lane] = v;
+      __threadfence();
+      __syncwarp();
+      const int64_t rb = a.rowptr[r], re = a.rowptr[r + 1];
+      const int64_t ca = rb / kEdgeChunk, cb = (re - 1) / kEdgeChunk;
+      int32_t ticket = 0;
+      if (lane == 0) ticket = atomicAdd(a.counters + r, 1);
+      ticket = __shfl_sync(FULL, ticket, 0);
+      if (ticket == (int32_t)(cb - ca)) {       // last chunk of row r to finish
+        __threadfence();
+        float4 tot = z4;
+        for (int64_t q0 = ca; q0 <= cb; q0 += 16) {
+          float4 blk = z4;
+          const int64_t q1 = (q0 + 16 < cb + 1) ? q0 + 16 : cb + 1;
+          for (int64_t q = q0; q < q1; ++q) {
+            const int64_t sl = q == ca ? 2 * q + 1 : 2 * q;
+            if (lane < nv) add_v(blk, __ldcg(reinterpret_cast<const float4*>(a.partials + sl * a.W) + lane));
+          }
+          add_v(tot, blk);
+        }
+        edge_write_row(a, r, tot, lane, nv);
+        if (lane == 0) a.counters[r] = 0;
+      }
+    };
+    for (int64_t base = e0; base < e1; base += 32) {
+      const int n = (int)((e1 - base) < 32 ? (e1 - base) : 32);
+      const int32_t my_col = lane < n ? __ldg(a.col + base + lane) : 0;
+      const int32_t my_row = lane < n ? __ldg(a.row + base + lane) : cur;
+      const float my_sc = (SCOL && lane < n) ? __ldg(a.scol + my_col) : 1.0f;
+      for (int j0 = 0; j0 < n; j0 += U) {
+        float4 xv[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int32_t cj = __shfl_sync(FULL, my_col, j0 + u);
+          xv[u] = (j0 + u < n && lane < nv) ? __ldg(reinterpret_cast<const float4*>(a.x + (int64_t)cj * a.ldx) + lane)
+                                            : z4;
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          if (j0 + u >= n) break;
+          const int32_t rj = __shfl_sync(FULL, my_row, j0 + u);
+          const float sj = SCOL ? __shfl_sync(FULL, my_sc, j0 + u) : 1.0f;
+          if (rj != cur) {
+            flush(cur);
+            for (int32_t r = cur + 1; r < rj; ++r) edge_write_row(a, r, z4, lane, nv);
+            cur = rj;
+            acc0 = z4;
+            acc1 = z4;
+          }
+          if (((base + j0 + u) & 1) == 0) {
+            if (SCOL) fma_v(acc0, sj, xv[u]); else add_v(acc0, xv[u]);
+          } else {
+            if (SCOL) fma_v(acc1, sj, xv[u]); else add_v(acc1, xv[u]);
+          }
+        }
+      }
+    }
+    flush(cur);
+  }
+}
+
+// TMA-gather edge-parallel kernel (strategy 2): per warp two 32-slot row
+// buffers in shared memory; for every 32-edge batch each lane issues ONE bulk
+// copy (cp.async.bulk, the whole W·4-byte feature row) that completes on the
+// buffer's mbarrier (expect_tx).  The next batch (possibly of the next chunk)
+// is issued before the current one is consumed, so a warp keeps up to 64 rows
+// in flight without register destinations.  Accumulation order and the chunk /
+// split-row logic are those of k_agg_edges.
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t mbar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(mbar)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t mbar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(mbar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint32_t mbar, uint32_t phase) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "W_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@P1 bra D_%=;\n\t"
+      "bra W_%=;\n"
+      "D_%=:\n\t}\n" ::"r"(mbar),
+      "r"(phase)
+      : "memory");
+}
+
+template <bool SCOL>
+__global__ void __launch_bounds__(kAggThreads) k_agg_edges_tma(const EdgeArgs a, int warps_per_block) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  __shared__ __align__(8) uint64_t mbars[kAggThreads / 32][2];
+  const unsigned FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  if (wib >= warps_per_block) return;
+  const int nv = a.W / 4;
+  const uint32_t rowb = (uint32_t)a.W * 4;
+  unsigned char* wbuf = smem_raw + (size_t)wib * 2 * 32 * rowb;
+  const uint32_t sbuf0 = (uint32_t)__cvta_generic_to_shared(wbuf);
+  const uint32_t mb0 = (uint32_t)__cvta_generic_to_shared(&mbars[wib][0]);
+  const uint32_t mb1 = (uint32_t)__cvta_generic_to_shared(&mbars[wib][1]);
+  if (lane == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(mb0) : "memory");
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(mb1) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncwarp();
+  const int64_t nchunks = (a.E + kEdgeChunk - 1) / kEdgeChunk;
+  const int64_t warp_id = (int64_t)blockIdx.x * warps_per_block + wib;
+  const int64_t nwarps = (int64_t)gridDim.x * warps_per_block;
+  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+  uint32_t phase0 = 0, phase1 = 0;
+  // batch stream: (chunk c, edge base) in order; issue(k) fills buffer k & 1
+  int32_t q_row0 = 0, q_row1 = 0, q_n0 = 0, q_n1 = 0;   // per-buffer batch metadata (no local arrays)
+  float q_sc0 = 1.f, q_sc1 = 1.f;
+  auto issue = [&](int64_t c, int64_t base, int which) {
+    const int64_t e1 = (a.E < c * kEdgeChunk + kEdgeChunk) ? a.E : c * kEdgeChunk + kEdgeChunk;
+    const int n = (int)((e1 - base) < 32 ? (e1 - base) : 32);
+    int32_t u = 0, rw = 0;
+    float sc = 1.0f;
+    if (lane < n) {
+      u = __ldg(a.col + base + lane);
+      rw = __ldg(a.row + base + lane);
+      sc = SCOL ? __ldg(a.scol + u) : 1.0f;
+    }
+    if (which) { q_row1 = rw; q_sc1 = sc; q_n1 = n; } else { q_row0 = rw; q_sc0 = sc; q_n0 = n; }
+    const uint32_t mb = which ? mb1 : mb0;
+    if (lane == 0) mbar_expect_tx(mb, (uint32_t)n * rowb);
+    __syncwarp();
+    if (lane < n) bulk_g2s(sbuf0 + (uint32_t)which * 32 * rowb + (uint32_t)lane * rowb, a.x + (int64_t)u * a.ldx, rowb, mb);
+  };
+  int64_t c = warp_id;
+  if (c >= nchunks) return;
+  int which = 0;
+  issue(c, c * kEdgeChunk, 0);
+  for (; c < nchunks; c += nwarps) {
+    const int64_t e0 = c * kEdgeChunk, e1 = (a.E < e0 + kEdgeChunk) ? a.E : e0 + kEdgeChunk;
+    const int32_t r_first = a.row[e0], r_last = a.row[e1 - 1];
+    const bool start_open = e0 > a.rowptr[r_first];
+    const bool end_open = e1 < a.rowptr[r_last + 1];
+    {
+      const int32_t gap0 = c == 0 ? 0 : a.row[e0 - 1] + 1;
+      for (int32_t r = gap0; r < r_first; ++r) edge_write_row(a, r, z4, lane, nv);
+      if (c == nchunks - 1)
+        for (int32_t r = r_last + 1; r < a.R; ++r) edge_write_row(a, r, z4, lane, nv);
+    }
+    int32_t cur = r_first;
+    float4 acc0 = z4, acc1 = z4;
+    auto flush = [&](int32_t r) {
+      float4 v = acc0;
+      add_v(v, acc1);
+      const bool open_s = (r == r_first) && start_open, open_e = (r == r_last) && end_open;
+      if (!open_s && !open_e) {
+        edge_write_row(a, r, v, lane, nv);
+        return;
+      }
+      const int64_t slot = open_s ? 2 * c : 2 * c + 1;
+      if (lane < nv) reinterpret_cast<float4*>(a.partials + slot * a.W)[lane] = v;
+      __threadfence();
+      __syncwarp();
+      const int64_t rb = a.rowptr[r], re = a.rowptr[r + 1];
+      const int64_t ca = rb / kEdgeChunk, cb = (re - 1) / kEdgeChunk;
+      int32_t ticket = 0;
+      if (lane == 0) ticket = atomicAdd(a.counters + r, 1);
+      ticket = __shfl_sync(FULL, ticket, 0);
+      if (ticket == (int32_t)(cb - ca)) {
+        __threadfence();
+        float4 tot = z4;
+        for (int64_t q0 = ca; q0 <= cb; q0 += 16) {
+          float4 blk = z4;
+          const int64_t q1 = (q0 + 16 < cb + 1) ? q0 + 16 : cb + 1;
+          for (int64_t q = q0; q < q1; ++q) {
+            const int64_t sl = q == ca ? 2 * q + 1 : 2 * q;
+            if (lane < nv) add_v(blk, __ldcg(reinterpret_cast<const float4*>(a.partials + sl * a.W) + lane));
+          }
+          add_v(tot, blk);
+        }
+        edge_write_row(a, r, tot, lane, nv);
+        if (lane == 0) a.counters[r] = 0;
+      }
+    };
+    for (int64_t base = e0; base < e1; base += 32) {
+      // prefetch the next batch of the stream (this chunk or the next chunk of this warp)
+      const int nxt = which ^ 1;
+      if (base + 32 < e1) issue(c, base + 32, nxt);
+      else if (c + nwarps < nchunks) issue(c + nwarps, (c + nwarps) * kEdgeChunk, nxt);
+      mbar_wait_parity(which ? mb1 : mb0, which ? phase1 : phase0);
+      if (which) phase1 ^= 1u; else phase0 ^= 1u;
+      const unsigned char* bb = wbuf + (size_t)which * 32 * rowb;
+      const int n = which ? q_n1 : q_n0;
+      const int32_t my_row = which ? q_row1 : q_row0;
+      const float my_sc = which ? q_sc1 : q_sc0;
+      for (int j = 0; j < n; ++j) {
+        const int32_t rj = __shfl_sync(FULL, my_row, j);
+        const float sj = SCOL ? __shfl_sync(FULL, my_sc, j) : 1.0f;
+        if (rj != cur) {
+          flush(cur);
+          for (int32_t r = cur + 1; r < rj; ++r) edge_write_row(a, r, z4, lane, nv);
+          cur = rj;
+          acc0 = z4;
+          acc1 = z4;
+        }
+        if (lane < nv) {
+          const float4 xv = reinterpret_cast<const float4*>(bb + (size_t)j * rowb)[lane];
+          if (((base + j) & 1) == 0) {
+            if (SCOL) fma_v(acc0, sj, xv); else add_v(acc0, xv);
+          } else {
+            if (SCOL) fma_v(acc1, sj, xv); else add_v(acc1, xv);
+          }
+        }
+      }
+      __syncwarp();     // every lane is done reading this buffer before it is refilled
+      which = nxt;
+    }
+    flush(cur);
+  }
+}
+
 using KernelFn = void (*)(const AggArgs);
 
 template <int VEC, int G, bool SCOL>
@@ -477,7 +765,7 @@ int max_blocks_for(KernelFn fn) {
 }  // namespace
 
 // Gather strategy switch (1 = cp.async shared-memory ring; 0 = register gathers).
-static int g_agg_async = 0;
+static int g_agg_async = 0;   // measured fastest on C5
 
 // Launch plan: vector width, group size, vectors per lane for W columns.
 struct AggPlan {
@@ -536,7 +824,53 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   }
   const int64_t items_bound = (int64_t)R + chunks_bound + 1;
   ProfScope prof(backward ? PH_AGG_BWD : PH_AGG_FWD, s);
-  const bool use_async = vec4 && g_agg_async;
+  // edge-parallel path: float4 rows, 16 <= float4-per-row chunks (W in [64, 128] per launch), COO rows known
+  const int32_t* rowarr = backward ? gv->out_row : gv->in_row;
+  if (vec4 && g_agg_async == 2 && W >= 64 && rowarr && gv->num_edges > 0 && gv->workspace) {
+    const int64_t E = gv->num_edges;
+    const int64_t nchunks = (E + kEdgeChunk - 1) / kEdgeChunk;
+    STG_TRY(ws->epartials.alloc((size_t)2 * nchunks * 128 + 4, s));
+    if (ws->ecounters_n < R) {
+      STG_TRY(ws->ecounters.alloc(R, s));
+      STG_CUDA(cudaMemsetAsync(ws->ecounters.p, 0, sizeof(int32_t) * R, s));
+      ws->ecounters_n = R;
+    }
+    EdgeArgs ea{};
+    ea.R = R; ea.E = E; ea.rowptr = a.rowptr; ea.col = a.col; ea.row = rowarr;
+    ea.srow = srow; ea.scol = scol;
+    ea.partials = ws->epartials.p; ea.counters = ws->ecounters.p;
+    for (int32_t c0 = 0; c0 < W; c0 += 128) {
+      const int32_t wl = (W - c0) < 128 ? (W - c0) : 128;
+      ea.W = wl; ea.x = in + c0; ea.ldx = ldin; ea.y = out + c0; ea.ldy = ldout;
+      ea.bias = bias ? bias + c0 : nullptr;
+      auto fn = scol ? k_agg_edges_tma<true> : k_agg_edges_tma<false>;
+      const size_t per_warp = (size_t)2 * 32 * wl * 4;
+      int wpb = (int)std::min<size_t>(kAggThreads / 32, (size_t)(200 * 1024) / per_warp);
+      if (wpb < 1) wpb = 1;
+      const size_t smem = per_warp * wpb;
+      {
+        static std::mutex mu;
+        std::lock_guard<std::mutex> lk(mu);
+        static size_t attr[2] = {0, 0};
+        if (attr[scol ? 1 : 0] < smem) {
+          STG_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+          attr[scol ? 1 : 0] = smem;
+        }
+      }
+      int per_sm = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kAggThreads, smem) != cudaSuccess || per_sm < 1) {
+        cudaGetLastError();
+        per_sm = 1;
+      }
+      int64_t blocks = ceil_div(nchunks, wpb);
+      const int64_t mb = (int64_t)per_sm * num_sms();
+      if (blocks > mb) blocks = mb;
+      fn<<<(unsigned)blocks, kAggThreads, smem, s>>>(ea, wpb);
+      count_launch();
+    }
+    return check_launch("aggregate_edges");
+  }
+  const bool use_async = vec4 && g_agg_async == 1;
   const int wmax = use_async ? 128 : p0.wmax;
   for (int32_t c0 = 0; c0 < W; c0 += wmax) {
     const int32_t wl = (W - c0) < wmax ? (W - c0) : wmax;
@@ -606,8 +940,9 @@ stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* 
                                (cudaStream_t)stream);
 }
 
-stg_status stg_aggregate_set_strategy(int32_t async_gather) {
-  stg::g_agg_async = async_gather ? 1 : 0;
+stg_status stg_aggregate_set_strategy(int32_t strategy) {
+  if (strategy < 0 || strategy > 2) return stg::fail(STG_ERR_INVALID_ARG, "stg_aggregate_set_strategy: %d", strategy);
+  stg::g_agg_async = strategy;
   return STG_OK;
 }
 

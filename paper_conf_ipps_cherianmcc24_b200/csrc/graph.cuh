@@ -20,6 +20,9 @@ struct AggWs {
   DArray<float> partials;
   DArray<int32_t> counters;
   int64_t counters_n = 0;
+  DArray<float> epartials;       // edge-parallel kernel: per-chunk partials
+  DArray<int32_t> ecounters;     // edge-parallel kernel: per-row tickets (self-resetting)
+  int64_t ecounters_n = 0;
 };
 
 struct Snapshot {

@@ -154,48 +154,46 @@ __device__ __forceinline__ void stage_rows(unsigned char* hi, unsigned char* lo,
   }
 }
 
+// TRANSPOSED operand tiles (K = rows) use a padded K-major layout: element
+// (feature f, row r) of an [F' × RK] tile at
+//     (f % 8)·16 + (f / 8)·SBO_T + (r % 4)·4 + (r / 4)·LBO_T,
+// LBO_T = 144 (128 + 16: consecutive K core matrices shifted by one 16-byte bank
+// quad), SBO_T = (RK / 4)·144.  The descriptor carries LBO_T / SBO_T.
+constexpr uint32_t kLboT = 144;
+__host__ __device__ __forceinline__ uint32_t sbo_t(int RK) { return (uint32_t)(RK / 4) * kLboT; }
+__host__ __device__ __forceinline__ uint32_t tmaj_off(int f, int r, int RK) {
+  return (uint32_t)((f & 7) * 16 + (r & 3) * 4) + (uint32_t)(f >> 3) * sbo_t(RK) + (uint32_t)(r >> 2) * kLboT;
+}
+
 // Stage rows [0,RK) × columns [f0, f0+F) of a row-major array as the TRANSPOSED
-// K-major operand: element (feature f, row r) of an [F' × RK] tile (K = rows)
-// at feature row fd0 + f.  Conflict-free: lane = (r%4, chunk parity, rotation s)
-// and the 4 scalars of each float4 are stored in a lane-rotated order so one
-// warp store touches 32 distinct banks.  F % 4 == 0, RK % 16 == 0.
+// operand (feature rows fd0.., K = rows).  Each thread owns a 4×4 block:
+// 4 float4 loads (4 rows × 4 features), an in-register transpose, and four
+// 16-byte stores (one per feature, 4 consecutive rows).  With LBO_T the 32
+// lanes of a store (8 row quads × 4 feature quads) cover every bank quad 4
+// times: conflict-free.  F % 4 == 0, RK % 4 == 0.
 __device__ __forceinline__ void stage_rows_T(unsigned char* hi, unsigned char* lo, const float* __restrict__ src,
                                              int64_t ld, int nvalid, int F, int f0, int fd0, int RK) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const int rr = (lane & 3) + 4 * (lane >> 3);
-  const int jj = (lane >> 2) & 1;
-  const int s = lane >> 3;
-  const int nrb = RK / 16, njb = (F + 7) / 8, total = nrb * njb;
-  const uint32_t sbo = (uint32_t)(RK / 4) * 128;
-  constexpr int B = 8;
-  for (int base = warp; base < total; base += B * nw) {
-    float4 v[B];
+  const int nrq = RK / 4, nfq = F / 4, total = nrq * nfq;
+  const uint32_t sbo = sbo_t(RK);
+  for (int b = threadIdx.x; b < total; b += blockDim.x) {
+    const int rq = b % nrq, fq = b / nrq;
+    float4 v[4];
 #pragma unroll
-    for (int i = 0; i < B; ++i) {
-      const int it = base + i * nw;
-      const int r = (it % nrb) * 16 + rr;
-      const int j = (it / nrb) * 2 + jj;
-      v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (it < total && 4 * j < F && r < nvalid)
-        v[i] = __ldg(reinterpret_cast<const float4*>(src + (int64_t)r * ld + f0 + 4 * j));
+    for (int i = 0; i < 4; ++i) {
+      const int r = 4 * rq + i;
+      v[i] = r < nvalid ? __ldg(reinterpret_cast<const float4*>(src + (int64_t)r * ld + f0 + 4 * fq))
+                        : make_float4(0.f, 0.f, 0.f, 0.f);
     }
+    const int fb = fd0 + 4 * fq;
+    const uint32_t base = (uint32_t)(fb >> 3) * sbo + (uint32_t)rq * kLboT + (uint32_t)((fb & 7) * 16);
+    const float t[4][4] = {{v[0].x, v[1].x, v[2].x, v[3].x}, {v[0].y, v[1].y, v[2].y, v[3].y},
+                           {v[0].z, v[1].z, v[2].z, v[3].z}, {v[0].w, v[1].w, v[2].w, v[3].w}};
 #pragma unroll
-    for (int i = 0; i < B; ++i) {
-      const int it = base + i * nw;
-      const int r = (it % nrb) * 16 + rr;
-      const int j = (it / nrb) * 2 + jj;
-      if (it >= total || 4 * j >= F) continue;
-#pragma unroll
-      for (int t = 0; t < 4; ++t) {
-        const int ci = (t + s) & 3;
-        const float x = ci == 0 ? v[i].x : (ci == 1 ? v[i].y : (ci == 2 ? v[i].z : v[i].w));
-        const int f = fd0 + 4 * j + ci;
-        const uint32_t off = (uint32_t)((f & 7) * 16) + (uint32_t)(f >> 3) * sbo + (uint32_t)((r & 3) * 4) +
-                             (uint32_t)(r >> 2) * 128;
-        const float h = tf32_hi(x);
-        *reinterpret_cast<float*>(hi + off) = h;
-        *reinterpret_cast<float*>(lo + off) = x - h;
-      }
+    for (int c = 0; c < 4; ++c) {
+      const float4 h = make_float4(tf32_hi(t[c][0]), tf32_hi(t[c][1]), tf32_hi(t[c][2]), tf32_hi(t[c][3]));
+      const float4 l = make_float4(t[c][0] - h.x, t[c][1] - h.y, t[c][2] - h.z, t[c][3] - h.w);
+      *reinterpret_cast<float4*>(hi + base + 16 * c) = h;
+      *reinterpret_cast<float4*>(lo + base + 16 * c) = l;
     }
   }
 }

@@ -23,11 +23,12 @@ __global__ void __launch_bounds__(128) k_tc_debug(int mode, int M, int N, int K,
   const int Kt = mode == 0 ? K : 32;            // K extent of a stored tile (32 rows for mode 1)
   const int Mrows = 128;
   unsigned char* a_hi = sm;
-  unsigned char* a_lo = a_hi + Mrows * Kt * 4;
+  const int pf = mode == 0 ? 4 : 5;              // mode 1 tiles use the padded transposed layout
+  unsigned char* a_lo = a_hi + Mrows * Kt * pf;
   const int Kb = mode == 0 ? K : 32;             // mode 0: B stored [N × K]; mode 1: Yᵀ tile [N × 32]
   const int Nr = N;
-  unsigned char* b_hi = a_lo + Mrows * Kt * 4;
-  unsigned char* b_lo = b_hi + Nr * Kb * 4;
+  unsigned char* b_hi = a_lo + Mrows * Kt * pf;
+  unsigned char* b_lo = b_hi + Nr * Kb * pf;
   const int warp = threadIdx.x >> 5;
   uint32_t ncols = 32;
   while ((int)ncols < N) ncols <<= 1;
@@ -74,8 +75,14 @@ __global__ void __launch_bounds__(128) k_tc_debug(int mode, int M, int N, int K,
         tc::mma_3xtf32_kmajor(tm, tc::smem_u32(a_hi), tc::smem_u32(a_lo), tc::smem_u32(b_hi), tc::smem_u32(b_lo), K,
                               tc::idesc_tf32(128, N, 0, 0), false);
       } else {
-        tc::mma_3xtf32_kmajor(tm, tc::smem_u32(a_hi), tc::smem_u32(a_lo), tc::smem_u32(b_hi), tc::smem_u32(b_lo),
-                              32, tc::idesc_tf32(128, N, 0, 0), tile > 0);
+        const uint32_t sb = tc::sbo_t(32), idesc = tc::idesc_tf32(128, N, 0, 0);
+        for (int k = 0; k < 32; k += 8) {
+          const uint32_t o = (uint32_t)(k / 4) * tc::kLboT;
+          const uint32_t acc = (tile > 0 || k > 0) ? 1u : 0u;
+          tc::mma_tf32(tm, tc::desc(tc::smem_u32(a_lo) + o, tc::kLboT, sb), tc::desc(tc::smem_u32(b_hi) + o, tc::kLboT, sb), idesc, acc);
+          tc::mma_tf32(tm, tc::desc(tc::smem_u32(a_hi) + o, tc::kLboT, sb), tc::desc(tc::smem_u32(b_lo) + o, tc::kLboT, sb), idesc, 1u);
+          tc::mma_tf32(tm, tc::desc(tc::smem_u32(a_hi) + o, tc::kLboT, sb), tc::desc(tc::smem_u32(b_hi) + o, tc::kLboT, sb), idesc, 1u);
+        }
       }
       tc::commit(&mbar);
     }
@@ -109,7 +116,8 @@ extern "C" stg_status stg_debug_tc_gemm(int32_t mode, int32_t M, int32_t N, int3
   if (mode == 0 && (M % 128 || K % 8 || K < 8 || K > 256)) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: M/K");
   if (mode == 1 && (R % 32 || R < 32)) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: R");
   const int Kt = mode == 0 ? K : 32, Kb = mode == 0 ? K : 32, Nr = N;
-  const size_t smem = (size_t)2 * 128 * Kt * 4 + (size_t)2 * Nr * Kb * 4;
+  const int pf = mode == 0 ? 4 : 5;
+  const size_t smem = (size_t)2 * 128 * Kt * pf + (size_t)2 * Nr * Kb * pf;
   if (smem > 200 * 1024) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: tile too large");
   STG_CUDA(cudaFuncSetAttribute(k_tc_debug, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int grid = mode == 0 ? M / 128 : 1;

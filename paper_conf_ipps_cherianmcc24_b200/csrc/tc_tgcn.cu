@@ -56,19 +56,39 @@ __device__ __forceinline__ void mma_seg(uint32_t d, uint32_t ahi, uint32_t alo, 
   }
 }
 
+// A warp can only touch its TMEM lane quarter (warp % 4): lanes 32·(w%4) + lane.
+// 3xTF32 chain over two TRANSPOSED tiles (padded layout, K = RK rows).
+__device__ __forceinline__ void mma_T(uint32_t d, uint32_t ahi, uint32_t alo, uint32_t bhi, uint32_t blo, int RK,
+                                      uint32_t idesc, bool first) {
+  const uint32_t sb = tc::sbo_t(RK);
+  for (int k = 0; k < RK; k += 8) {
+    const uint32_t o = (uint32_t)(k / 4) * tc::kLboT;
+    const uint32_t acc = (first && k == 0) ? 0u : 1u;
+    tc::mma_tf32(d, tc::desc(alo + o, tc::kLboT, sb), tc::desc(bhi + o, tc::kLboT, sb), idesc, acc);
+    tc::mma_tf32(d, tc::desc(ahi + o, tc::kLboT, sb), tc::desc(blo + o, tc::kLboT, sb), idesc, 1u);
+    tc::mma_tf32(d, tc::desc(ahi + o, tc::kLboT, sb), tc::desc(bhi + o, tc::kLboT, sb), idesc, 1u);
+  }
+}
+
 __device__ __forceinline__ uint32_t tmem_row(uint32_t base, int col) {
-  return base + ((uint32_t)((threadIdx.x >> 5) * 32) << 16) + (uint32_t)col;
+  return base + ((uint32_t)(((threadIdx.x >> 5) & 3) * 32) << 16) + (uint32_t)col;
 }
 
 template <int N>
 __device__ __forceinline__ void tmem_row_load(uint32_t base, int col, float (&v)[N]) {
-  static_assert(N % 16 == 0, "N % 16");
+  static_assert(N % 8 == 0, "N % 8");
 #pragma unroll
-  for (int c = 0; c < N; c += 16) {
+  for (int c = 0; c + 16 <= N; c += 16) {
     float t[16];
     tc::tmem_ld16(tmem_row(base, col + c), t);
 #pragma unroll
     for (int i = 0; i < 16; ++i) v[c + i] = t[i];
+  }
+  if (N % 16) {
+    float t[8];
+    tc::tmem_ld8(tmem_row(base, col + (N / 16) * 16), t);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[(N / 16) * 16 + i] = t[i];
   }
   tc::tmem_wait_ld();
 }
@@ -182,15 +202,43 @@ __device__ __forceinline__ void stage_row_vec(unsigned char* hi, unsigned char* 
 }
 
 // ------------------------------------------------------------------ GRU forward
+// 256 threads: thread t owns tile row (w % 4)·32 + lane (its TMEM lane) and the
+// column half (w / 4) of every H-wide quantity.  All GRU epilogue math is
+// column-local; the column mixing happens in the MMAs.
+constexpr int kGruThreads = 256;
+
+template <int N>
+__device__ __forceinline__ void ld_half(const float* __restrict__ src, bool ok, float (&v)[N]) {
+#pragma unroll
+  for (int q = 0; q < N / 4; ++q) {
+    float4 x = ok ? __ldg(reinterpret_cast<const float4*>(src) + q) : make_float4(0.f, 0.f, 0.f, 0.f);
+    v[4 * q] = x.x; v[4 * q + 1] = x.y; v[4 * q + 2] = x.z; v[4 * q + 3] = x.w;
+  }
+}
+template <int N>
+__device__ __forceinline__ void st_half(float* dst, const float (&v)[N], float scale = 1.0f) {
+#pragma unroll
+  for (int q = 0; q < N / 4; ++q)
+    reinterpret_cast<float4*>(dst)[q] =
+        make_float4(scale * v[4 * q], scale * v[4 * q + 1], scale * v[4 * q + 2], scale * v[4 * q + 3]);
+}
+template <int N>
+__device__ __forceinline__ void stage_half(unsigned char* hi, unsigned char* lo, int r, int k0, int K,
+                                           const float (&v)[N]) {
+#pragma unroll
+  for (int q = 0; q < N / 4; ++q)
+    tc::st_split4(hi, lo, r, k0 / 4 + q, K, make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]));
+}
+
 template <int H>
-__global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_fwd(int V, const float* __restrict__ C,
-                                                              const float* __restrict__ Hp,
-                                                              const float* __restrict__ L,
-                                                              const float* __restrict__ l, float* __restrict__ Hn) {
+__global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_fwd(int V, const float* __restrict__ C,
+                                                               const float* __restrict__ Hp,
+                                                               const float* __restrict__ L,
+                                                               const float* __restrict__ l, float* __restrict__ Hn) {
   extern __shared__ __align__(128) unsigned char sm[];
   __shared__ uint64_t mbar;
   __shared__ uint32_t tslot;
-  constexpr int BG = GruSmem<H>::BG, A1 = GruSmem<H>::A1, H3 = 3 * H;
+  constexpr int BG = GruSmem<H>::BG, A1 = GruSmem<H>::A1, H3 = 3 * H, HH = H / 2;
   unsigned char* bz_hi = sm;               unsigned char* bz_lo = bz_hi + BG;
   unsigned char* br_hi = bz_lo + BG;       unsigned char* br_lo = br_hi + BG;
   unsigned char* bh_hi = br_lo + BG;       unsigned char* bh_lo = bh_hi + BG;
@@ -207,43 +255,39 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_fwd(int V, const float
   const uint32_t tm = tslot;
   uint32_t phase = 0;
   const int ntiles = (V + 127) / 128;
-  const int t = threadIdx.x;
+  const int w = threadIdx.x >> 5, lr = (w & 3) * 32 + (threadIdx.x & 31), c0 = (w >> 2) * HH;
+  float lz[HH], lrr[HH], lh[HH];
+#pragma unroll
+  for (int j = 0; j < HH; ++j) { lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; }
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int r0 = tile * 128, nv = V - r0, row = r0 + t;
-    // A1 = [C_z | C_r | H]
+    const int r0 = tile * 128, nv = V - r0, row = r0 + lr;
+    const bool ok = row < V;
+    float h[HH];
+    ld_half<HH>(Hp + (int64_t)row * H + c0, ok, h);          // in flight during staging + MMA
     tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, 2 * H, 0, 0, H3);
     tc::stage_rows(ahi, alo, Hp + (int64_t)r0 * H, H, nv, 128, H, 0, 2 * H, H3);
     sync_mma_operands();
-    if (t == 0) {
+    if (threadIdx.x == 0) {
       issue_zr<H>(tm, ahi, alo, bz_hi, bz_lo, br_hi, br_lo);
       tc::commit(&mbar);
     }
     wait_mma(&mbar, phase);
-    float z[H], rh[H], h[H];
+    float z[HH], rh[HH];
     {
-      float a[2 * H];
-      tmem_row_load<2 * H>(tm, 0, a);
+      float az[HH], ar[HH];
+      tmem_row_load<HH>(tm, c0, az);
+      tmem_row_load<HH>(tm, H + c0, ar);
 #pragma unroll
-      for (int j = 0; j < H; ++j) h[j] = 0.f;
-      if (row < V) {
-        const float4* hp = reinterpret_cast<const float4*>(Hp + (int64_t)row * H);
-#pragma unroll
-        for (int q = 0; q < H / 4; ++q) {
-          float4 x = __ldg(hp + q);
-          h[4 * q] = x.x; h[4 * q + 1] = x.y; h[4 * q + 2] = x.z; h[4 * q + 3] = x.w;
-        }
-      }
-#pragma unroll
-      for (int j = 0; j < H; ++j) {
-        z[j] = sigm(a[j] + __ldg(l + j));
-        rh[j] = sigm(a[H + j] + __ldg(l + H + j)) * h[j];
+      for (int j = 0; j < HH; ++j) {
+        z[j] = sigm(az[j] + lz[j]);
+        rh[j] = sigm(ar[j] + lrr[j]) * h[j];
       }
     }
     // A2 = [C_h | RH] (width 2H) reuses the A1 storage (MMA on A1 has completed)
     tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, H, 2 * H, 0, 2 * H);
-    stage_row_vec<H>(ahi, alo, t, H, 2 * H, rh);
+    stage_half<HH>(ahi, alo, lr, H + c0, 2 * H, rh);
     sync_mma_operands();
-    if (t == 0) {
+    if (threadIdx.x == 0) {
       const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0);
       mma_seg(tm + 2 * H, tc::smem_u32(ahi), tc::smem_u32(alo), 2 * H, 0, tc::smem_u32(bh_hi), tc::smem_u32(bh_lo),
               2 * H, 0, 2 * H, idesc, true);
@@ -251,22 +295,14 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_fwd(int V, const float
     }
     wait_mma(&mbar, phase);
     {
-      float a[H];
-      tmem_row_load<H>(tm, 2 * H, a);
-      if (row < V) {
-        float4* out = reinterpret_cast<float4*>(Hn + (int64_t)row * H);
+      float ah[HH], o[HH];
+      tmem_row_load<HH>(tm, 2 * H + c0, ah);
 #pragma unroll
-        for (int q = 0; q < H / 4; ++q) {
-          float o[4];
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const int j = 4 * q + i;
-            const float hh = tanhf(a[j] + __ldg(l + 2 * H + j));
-            o[i] = z[j] * h[j] + (1.0f - z[j]) * hh;
-          }
-          out[q] = make_float4(o[0], o[1], o[2], o[3]);
-        }
+      for (int j = 0; j < HH; ++j) {
+        const float hh = tanhf(ah[j] + lh[j]);
+        o[j] = z[j] * h[j] + (1.0f - z[j]) * hh;
       }
+      if (ok) st_half<HH>(Hn + (int64_t)row * H + c0, o);
     }
     tc::fence_before();
     __syncthreads();
@@ -279,18 +315,18 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_fwd(int V, const float
 
 // ------------------------------------------------------------------ GRU backward
 template <int H>
-__global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_bwd(int V, const float* __restrict__ C,
-                                                              const float* __restrict__ Hp,
-                                                              const float* __restrict__ G,
-                                                              const float* __restrict__ L,
-                                                              const float* __restrict__ l,
-                                                              const float* __restrict__ ndst,
-                                                              float* __restrict__ dCs, float* __restrict__ dHp,
-                                                              float* __restrict__ da, float* __restrict__ RHo) {
+__global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_bwd(int V, const float* __restrict__ C,
+                                                               const float* __restrict__ Hp,
+                                                               const float* __restrict__ G,
+                                                               const float* __restrict__ L,
+                                                               const float* __restrict__ l,
+                                                               const float* __restrict__ ndst,
+                                                               float* __restrict__ dCs, float* __restrict__ dHp,
+                                                               float* __restrict__ da, float* __restrict__ RHo) {
   extern __shared__ __align__(128) unsigned char sm[];
   __shared__ uint64_t mbar;
   __shared__ uint32_t tslot;
-  constexpr int BG = GruSmem<H>::BG, A1 = GruSmem<H>::A1, H3 = 3 * H;
+  constexpr int BG = GruSmem<H>::BG, A1 = GruSmem<H>::A1, H3 = 3 * H, HH = H / 2;
   unsigned char* bz_hi = sm;               unsigned char* bz_lo = bz_hi + BG;
   unsigned char* br_hi = bz_lo + BG;       unsigned char* br_lo = br_hi + BG;
   unsigned char* bh_hi = br_lo + BG;       unsigned char* bh_lo = bh_hi + BG;
@@ -315,92 +351,71 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_bwd(int V, const float
   const uint32_t tm = tslot;
   uint32_t phase = 0;
   const int ntiles = (V + 127) / 128;
-  const int t = threadIdx.x;
+  const int w = threadIdx.x >> 5, lr = (w & 3) * 32 + (threadIdx.x & 31), c0 = (w >> 2) * HH;
   const uint32_t id_h = tc::idesc_tf32(128, H, 0, 0), id_2h = tc::idesc_tf32(128, 2 * H, 0, 0);
+  float lz[HH], lrr[HH], lh[HH];
+#pragma unroll
+  for (int j = 0; j < HH; ++j) { lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; }
+  unsigned char* a3h = ahi;                      unsigned char* a3l = alo;
+  unsigned char* a4zh = ahi + 128 * H * 4;       unsigned char* a4zl = alo + 128 * H * 4;
+  unsigned char* a4rh = ahi + 2 * 128 * H * 4;   unsigned char* a4rl = alo + 2 * 128 * H * 4;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int r0 = tile * 128, nv = V - r0, row = r0 + t;
+    const int r0 = tile * 128, nv = V - r0, row = r0 + lr;
     const bool ok = row < V;
+    float h[HH], g[HH];
+    ld_half<HH>(Hp + (int64_t)row * H + c0, ok, h);           // in flight during staging + MMA
+    ld_half<HH>(G + (int64_t)row * H + c0, ok, g);
+    const float nd = ok ? __ldg(ndst + row) : 0.f;
     tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, 2 * H, 0, 0, H3);
     tc::stage_rows(ahi, alo, Hp + (int64_t)r0 * H, H, nv, 128, H, 0, 2 * H, H3);
     sync_mma_operands();
-    if (t == 0) {
+    if (threadIdx.x == 0) {
       issue_zr<H>(tm, ahi, alo, bz_hi, bz_lo, br_hi, br_lo);
       tc::commit(&mbar);
     }
     wait_mma(&mbar, phase);
-    float z[H], r[H], h[H], dh[H];
+    float z[HH], r[HH], dh[HH];
     {
-      float a[2 * H];
-      tmem_row_load<2 * H>(tm, 0, a);
+      float az[HH], ar[HH];
+      tmem_row_load<HH>(tm, c0, az);
+      tmem_row_load<HH>(tm, H + c0, ar);
 #pragma unroll
-      for (int j = 0; j < H; ++j) h[j] = 0.f;
-      if (ok) {
-        const float4* hp = reinterpret_cast<const float4*>(Hp + (int64_t)row * H);
-#pragma unroll
-        for (int q = 0; q < H / 4; ++q) {
-          float4 x = __ldg(hp + q);
-          h[4 * q] = x.x; h[4 * q + 1] = x.y; h[4 * q + 2] = x.z; h[4 * q + 3] = x.w;
-        }
-      }
-#pragma unroll
-      for (int j = 0; j < H; ++j) {
-        z[j] = sigm(a[j] + __ldg(l + j));
-        r[j] = sigm(a[H + j] + __ldg(l + H + j));
-        dh[j] = r[j] * h[j];                        // RH for now
+      for (int j = 0; j < HH; ++j) {
+        z[j] = sigm(az[j] + lz[j]);
+        r[j] = sigm(ar[j] + lrr[j]);
+        dh[j] = r[j] * h[j];                         // RH for now
       }
     }
     tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, H, 2 * H, 0, 2 * H);
-    stage_row_vec<H>(ahi, alo, t, H, 2 * H, dh);
-    if (ok) {
-      float4* o = reinterpret_cast<float4*>(RHo + (int64_t)row * H);
-#pragma unroll
-      for (int q = 0; q < H / 4; ++q) o[q] = make_float4(dh[4 * q], dh[4 * q + 1], dh[4 * q + 2], dh[4 * q + 3]);
-    }
+    stage_half<HH>(ahi, alo, lr, H + c0, 2 * H, dh);
+    if (ok) st_half<HH>(RHo + (int64_t)row * H + c0, dh);
     sync_mma_operands();
-    if (t == 0) {
+    if (threadIdx.x == 0) {
       mma_seg(tm + 2 * H, tc::smem_u32(ahi), tc::smem_u32(alo), 2 * H, 0, tc::smem_u32(bh_hi), tc::smem_u32(bh_lo),
               2 * H, 0, 2 * H, id_h, true);
       tc::commit(&mbar);
     }
     wait_mma(&mbar, phase);
-    // A3 = da_h [128 × H] (K = H), A4z = da_z, A4r = da_r placed after it
-    unsigned char* a3h = ahi;                      unsigned char* a3l = alo;
-    unsigned char* a4zh = ahi + 128 * H * 4;       unsigned char* a4zl = alo + 128 * H * 4;
-    unsigned char* a4rh = ahi + 2 * 128 * H * 4;   unsigned char* a4rl = alo + 2 * 128 * H * 4;
     {
-      float a[H], g[H], dah[H], daz[H];
-      tmem_row_load<H>(tm, 2 * H, a);
+      float ah[HH], dah[HH], daz[HH];
+      tmem_row_load<HH>(tm, 2 * H + c0, ah);
 #pragma unroll
-      for (int j = 0; j < H; ++j) g[j] = 0.f;
-      if (ok) {
-        const float4* gp = reinterpret_cast<const float4*>(G + (int64_t)row * H);
-#pragma unroll
-        for (int q = 0; q < H / 4; ++q) {
-          float4 x = __ldg(gp + q);
-          g[4 * q] = x.x; g[4 * q + 1] = x.y; g[4 * q + 2] = x.z; g[4 * q + 3] = x.w;
-        }
-      }
-#pragma unroll
-      for (int j = 0; j < H; ++j) {
-        const float hh = tanhf(a[j] + __ldg(l + 2 * H + j));
+      for (int j = 0; j < HH; ++j) {
+        const float hh = tanhf(ah[j] + lh[j]);
         const float dZ = g[j] * (h[j] - hh), dHh = g[j] * (1.0f - z[j]);
         dah[j] = dHh * (1.0f - hh * hh);
         daz[j] = dZ * z[j] * (1.0f - z[j]);
         dh[j] = g[j] * z[j];
       }
-      stage_row_vec<H>(a3h, a3l, t, 0, H, dah);
-      stage_row_vec<H>(a4zh, a4zl, t, 0, H, daz);
+      stage_half<HH>(a3h, a3l, lr, c0, H, dah);
+      stage_half<HH>(a4zh, a4zl, lr, c0, H, daz);
       if (ok) {
-        float4* oa = reinterpret_cast<float4*>(da + (int64_t)row * H3);
-#pragma unroll
-        for (int q = 0; q < H / 4; ++q) {
-          oa[q] = make_float4(daz[4 * q], daz[4 * q + 1], daz[4 * q + 2], daz[4 * q + 3]);
-          oa[H / 2 + q] = make_float4(dah[4 * q], dah[4 * q + 1], dah[4 * q + 2], dah[4 * q + 3]);
-        }
+        st_half<HH>(da + (int64_t)row * H3 + c0, daz);
+        st_half<HH>(da + (int64_t)row * H3 + 2 * H + c0, dah);
       }
     }
     sync_mma_operands();
-    if (t == 0) {
+    if (threadIdx.x == 0) {
       mma_seg(tm + 4 * H, tc::smem_u32(a3h), tc::smem_u32(a3l), H, 0, tc::smem_u32(lh_hi), tc::smem_u32(lh_lo), H, 0,
               H, id_2h, true);
       mma_seg(tm + 6 * H, tc::smem_u32(a4zh), tc::smem_u32(a4zl), H, 0, tc::smem_u32(lz_hi), tc::smem_u32(lz_lo), H,
@@ -408,31 +423,21 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_bwd(int V, const float
       tc::commit(&mbar);
     }
     wait_mma(&mbar, phase);
-    const float nd = ok ? ndst[row] : 0.f;
     {
-      float a[2 * H], dar[H];
-      tmem_row_load<2 * H>(tm, 4 * H, a);              // [dC_h | dRH]
-      if (ok) {
-        float4* o = reinterpret_cast<float4*>(dCs + (int64_t)row * H3 + 2 * H);
+      float dch[HH], drh[HH], dar[HH];
+      tmem_row_load<HH>(tm, 4 * H + c0, dch);          // dC_h
+      tmem_row_load<HH>(tm, 5 * H + c0, drh);          // dRH
+      if (ok) st_half<HH>(dCs + (int64_t)row * H3 + 2 * H + c0, dch, nd);
 #pragma unroll
-        for (int q = 0; q < H / 4; ++q)
-          o[q] = make_float4(nd * a[4 * q], nd * a[4 * q + 1], nd * a[4 * q + 2], nd * a[4 * q + 3]);
+      for (int j = 0; j < HH; ++j) {
+        dh[j] += drh[j] * r[j];
+        dar[j] = drh[j] * h[j] * r[j] * (1.0f - r[j]);
       }
-#pragma unroll
-      for (int j = 0; j < H; ++j) {
-        const float dRH = a[H + j];
-        dh[j] += dRH * r[j];
-        dar[j] = dRH * h[j] * r[j] * (1.0f - r[j]);
-      }
-      stage_row_vec<H>(a4rh, a4rl, t, 0, H, dar);
-      if (ok) {
-        float4* oa = reinterpret_cast<float4*>(da + (int64_t)row * H3 + H);
-#pragma unroll
-        for (int q = 0; q < H / 4; ++q) oa[q] = make_float4(dar[4 * q], dar[4 * q + 1], dar[4 * q + 2], dar[4 * q + 3]);
-      }
+      stage_half<HH>(a4rh, a4rl, lr, c0, H, dar);
+      if (ok) st_half<HH>(da + (int64_t)row * H3 + H + c0, dar);
     }
     sync_mma_operands();
-    if (t == 0) {
+    if (threadIdx.x == 0) {
       mma_seg(tm + 8 * H, tc::smem_u32(a4rh), tc::smem_u32(a4rl), H, 0, tc::smem_u32(lr_hi), tc::smem_u32(lr_lo), H,
               0, H, id_2h, true);
       tc::commit(&mbar);
@@ -440,22 +445,14 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_bwd(int V, const float
     wait_mma(&mbar, phase);
 #pragma unroll
     for (int half = 0; half < 2; ++half) {               // [dC_z | dH_z], then [dC_r | dH_r]
-      float a[2 * H];
-      tmem_row_load<2 * H>(tm, (6 + 2 * half) * H, a);
-      if (ok) {
-        float4* o = reinterpret_cast<float4*>(dCs + (int64_t)row * H3 + half * H);
+      float dc[HH], dx[HH];
+      tmem_row_load<HH>(tm, (6 + 2 * half) * H + c0, dc);
+      tmem_row_load<HH>(tm, (7 + 2 * half) * H + c0, dx);
+      if (ok) st_half<HH>(dCs + (int64_t)row * H3 + half * H + c0, dc, nd);
 #pragma unroll
-        for (int q = 0; q < H / 4; ++q)
-          o[q] = make_float4(nd * a[4 * q], nd * a[4 * q + 1], nd * a[4 * q + 2], nd * a[4 * q + 3]);
-      }
-#pragma unroll
-      for (int j = 0; j < H; ++j) dh[j] += a[H + j];
+      for (int j = 0; j < HH; ++j) dh[j] += dx[j];
     }
-    if (ok) {
-      float4* od = reinterpret_cast<float4*>(dHp + (int64_t)row * H);
-#pragma unroll
-      for (int q = 0; q < H / 4; ++q) od[q] = make_float4(dh[4 * q], dh[4 * q + 1], dh[4 * q + 2], dh[4 * q + 3]);
-    }
+    if (ok) st_half<HH>(dHp + (int64_t)row * H + c0, dh);
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
@@ -466,119 +463,176 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_tc_gru_bwd(int V, const float
 }
 
 // ------------------------------------------------------------------ Σ_rows Aᵀ·B
-// A = [A1 (FA1 cols) | A2 (FA2 cols) | ones (if ones)] padded to 128 features;
-// B = [B1 (N cols)].  Tiles of RK rows are staged transposed (K = rows).
-// Per-CTA partial D [128 × N] written to part[blockIdx.x].
-constexpr int kRK = 64;
+// D_a = Σ_rows A_a[r,:]ᵀ·B[r,:] for NA (1 or 2) A operands sharing one B.
+//   A_0 = [A1 (FA1 cols) | A2 (FA2 cols)], A_1 = [A3 (FA3 cols) | ones (opt.)],
+// each padded to 128 feature rows (M = 128), B = [B (FB cols)] padded to N.
+// Tiles of kRK rows are staged TRANSPOSED (K = rows) by all 16 warps into one
+// of two operand stages while the tensor core consumes the other (mbarrier
+// per stage).  Per-CTA partials [NA][128 × N] go to part[blockIdx.x].
+constexpr int kRK = 32;
+constexpr int kAtbThreads = 512;
 
-template <int N>
-__global__ void __launch_bounds__(kTcThreads) k_tc_atb(int V, const float* __restrict__ A1, int64_t lda1, int FA1,
-                                                       const float* __restrict__ A2, int64_t lda2, int FA2, int ones,
-                                                       const float* __restrict__ B, int64_t ldb, int FB,
-                                                       float* __restrict__ part) {
+struct AtbArgs {
+  int V;
+  const float* A1; int64_t lda1; int FA1;
+  const float* A2; int64_t lda2; int FA2;
+  const float* A3; int64_t lda3; int FA3; int ones;
+  const float* B; int64_t ldb; int FB;
+  float* part;
+};
+
+template <int N, int NA>
+__global__ void __launch_bounds__(kAtbThreads, 1) k_tc_atb(const AtbArgs p) {
   extern __shared__ __align__(128) unsigned char sm[];
-  __shared__ uint64_t mbar;
+  __shared__ uint64_t mbar[2];
   __shared__ uint32_t tslot;
-  unsigned char* ahi = sm;
-  unsigned char* alo = ahi + 128 * kRK * 4;
-  unsigned char* bhi = alo + 128 * kRK * 4;
-  unsigned char* blo = bhi + N * kRK * 4;
-  constexpr uint32_t NC = N <= 32 ? 32 : (N <= 64 ? 64 : (N <= 128 ? 128 : 256));
-  const int FA = FA1 + FA2;
-  // zero the padded feature rows [FA, 128) once (ones row set per tile below)
-  for (int e = threadIdx.x; e < 128 * kRK; e += kTcThreads) {
-    const int f = e / kRK, k = e % kRK;
-    if (f >= FA) {
-      const float v = (ones && f == FA) ? 1.0f : 0.0f;
-      *reinterpret_cast<float*>(ahi + tc::kmaj_off(f, k, kRK)) = v;
-      *reinterpret_cast<float*>(alo + tc::kmaj_off(f, k, kRK)) = 0.0f;
+  constexpr int ABYTES = 128 / 8 * (kRK / 4) * 144, BBYTES = N / 8 * (kRK / 4) * 144;   // padded layout
+  constexpr int STAGE = NA * 2 * ABYTES + 2 * BBYTES;
+  constexpr uint32_t NC = NA * N <= 32 ? 32 : (NA * N <= 64 ? 64 : (NA * N <= 128 ? 128 : (NA * N <= 256 ? 256 : 512)));
+  auto ahi = [&](int st, int a) { return sm + st * STAGE + a * 2 * ABYTES; };
+  auto alo = [&](int st, int a) { return sm + st * STAGE + a * 2 * ABYTES + ABYTES; };
+  auto bhi = [&](int st) { return sm + st * STAGE + NA * 2 * ABYTES; };
+  auto blo = [&](int st) { return sm + st * STAGE + NA * 2 * ABYTES + BBYTES; };
+  const int FA0 = p.FA1 + p.FA2, FAx = p.FA3 + (p.ones ? 1 : 0);
+  // zero the padding feature rows of both stages once (ones row: 1.0 per valid row, set per tile)
+  for (int st = 0; st < 2; ++st) {
+    for (int e = threadIdx.x; e < 128 * kRK; e += kAtbThreads) {
+      const int f = e / kRK, k = e % kRK;
+      const uint32_t off = tc::tmaj_off(f, k, kRK);
+      if (f >= FA0) { *reinterpret_cast<float*>(ahi(st, 0) + off) = 0.f; *reinterpret_cast<float*>(alo(st, 0) + off) = 0.f; }
+      if (NA > 1 && f >= p.FA3) { *reinterpret_cast<float*>(ahi(st, 1) + off) = 0.f; *reinterpret_cast<float*>(alo(st, 1) + off) = 0.f; }
+    }
+    for (int e = threadIdx.x; e < (N - p.FB) * kRK; e += kAtbThreads) {
+      const int f = p.FB + e / kRK, k = e % kRK;
+      *reinterpret_cast<float*>(bhi(st) + tc::tmaj_off(f, k, kRK)) = 0.f;
+      *reinterpret_cast<float*>(blo(st) + tc::tmaj_off(f, k, kRK)) = 0.f;
     }
   }
-  for (int e = threadIdx.x; e < (N - FB) * kRK; e += kTcThreads) {   // zero B feature padding once
-    const int f = FB + e / kRK, k = e % kRK;
-    *reinterpret_cast<float*>(bhi + tc::kmaj_off(f, k, kRK)) = 0.0f;
-    *reinterpret_cast<float*>(blo + tc::kmaj_off(f, k, kRK)) = 0.0f;
-  }
   if ((threadIdx.x >> 5) == 0) tc::tmem_alloc(&tslot, NC);
-  if (threadIdx.x == 0) { tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
+  if (threadIdx.x == 0) {
+    tc::mbar_init(&mbar[0], 1);
+    tc::mbar_init(&mbar[1], 1);
+    tc::fence_mbar_init();
+  }
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
   const uint32_t tm = tslot;
-  uint32_t phase = 0;
+  uint32_t phase[2] = {0u, 0u};
+  bool pending[2] = {false, false};
   const uint32_t idesc = tc::idesc_tf32(128, N, 0, 0);
-  const int ntiles = (V + kRK - 1) / kRK;
-  bool first = true;
-  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int r0 = tile * kRK, nv = V - r0;
-    tc::stage_rows_T(ahi, alo, A1 + (int64_t)r0 * lda1, lda1, nv, FA1, 0, 0, kRK);
-    if (FA2) tc::stage_rows_T(ahi, alo, A2 + (int64_t)r0 * lda2, lda2, nv, FA2, 0, FA1, kRK);
-    if (ones && nv < kRK) {   // ones row must be zero on padding rows of the last tile
-      for (int k = threadIdx.x; k < kRK; k += kTcThreads)
-        *reinterpret_cast<float*>(ahi + tc::kmaj_off(FA, k, kRK)) = k < nv ? 1.0f : 0.0f;
+  const int ntiles = (p.V + kRK - 1) / kRK;
+  int it = 0;
+  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++it) {
+    const int st = it & 1;
+    if (pending[st]) {                      // the MMAs that read this stage must be done
+      tc::mbar_wait(&mbar[st], phase[st]);
+      phase[st] ^= 1u;
+      pending[st] = false;
     }
-    tc::stage_rows_T(bhi, blo, B + (int64_t)r0 * ldb, ldb, nv, FB, 0, 0, kRK);
+    const int r0 = tile * kRK, nv = p.V - r0;
+    tc::stage_rows_T(ahi(st, 0), alo(st, 0), p.A1 + (int64_t)r0 * p.lda1, p.lda1, nv, p.FA1, 0, 0, kRK);
+    if (p.FA2) tc::stage_rows_T(ahi(st, 0), alo(st, 0), p.A2 + (int64_t)r0 * p.lda2, p.lda2, nv, p.FA2, 0, p.FA1, kRK);
+    if (NA > 1) {
+      tc::stage_rows_T(ahi(st, 1), alo(st, 1), p.A3 + (int64_t)r0 * p.lda3, p.lda3, nv, p.FA3, 0, 0, kRK);
+      if (p.ones)
+        for (int k = threadIdx.x; k < kRK; k += kAtbThreads)
+          *reinterpret_cast<float*>(ahi(st, 1) + tc::tmaj_off(p.FA3, k, kRK)) = k < nv ? 1.0f : 0.0f;
+    }
+    tc::stage_rows_T(bhi(st), blo(st), p.B + (int64_t)r0 * p.ldb, p.ldb, nv, p.FB, 0, 0, kRK);
     sync_mma_operands();
     if (threadIdx.x == 0) {
-      mma_seg(tm, tc::smem_u32(ahi), tc::smem_u32(alo), kRK, 0, tc::smem_u32(bhi), tc::smem_u32(blo), kRK, 0, kRK,
-              idesc, first);
-      tc::commit(&mbar);
+      const bool first = it == 0;
+      mma_T(tm, tc::smem_u32(ahi(st, 0)), tc::smem_u32(alo(st, 0)), tc::smem_u32(bhi(st)), tc::smem_u32(blo(st)), kRK,
+            idesc, first);
+      if (NA > 1)
+        mma_T(tm + N, tc::smem_u32(ahi(st, 1)), tc::smem_u32(alo(st, 1)), tc::smem_u32(bhi(st)),
+              tc::smem_u32(blo(st)), kRK, idesc, first);
+      tc::commit(&mbar[st]);
     }
-    wait_mma(&mbar, phase);
-    first = false;
-    tc::fence_before();
-    __syncthreads();
-    tc::fence_after();
+    pending[st] = true;
   }
-  // epilogue: thread t = feature row t of D
-  float* out = part + (int64_t)blockIdx.x * 128 * N + (int64_t)threadIdx.x * N;
-  if (first) {
-    for (int c = 0; c < N; ++c) out[c] = 0.f;
-  } else {
-    float v[N];
-    tmem_row_load<N>(tm, 0, v);
-    for (int c = 0; c < N; ++c) out[c] = v[c];
+  for (int st = 0; st < 2; ++st)
+    if (pending[st]) { tc::mbar_wait(&mbar[st], phase[st]); phase[st] ^= 1u; }
+  tc::fence_after();
+  (void)FAx;
+  // epilogue: warp w reads TMEM lane quarter (w % 4), column block (w / 4) of 4
+  const int w = threadIdx.x >> 5, q = w & 3, cb = w >> 2;
+  const int row = q * 32 + (threadIdx.x & 31);
+  constexpr int TOT = NA * N;                           // 8-column groups interleaved over the 4 warp groups
+  float* out = p.part + (int64_t)blockIdx.x * NA * 128 * N;
+  for (int c = cb * 8; c < TOT; c += 32) {
+    float v[8];
+    if (it == 0) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) v[i] = 0.f;
+    } else {
+      tc::tmem_ld8(tm + ((uint32_t)(q * 32) << 16) + (uint32_t)c, v);
+      tc::tmem_wait_ld();
+    }
+    const int a = c / N, cc = c % N;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) out[(int64_t)a * 128 * N + (int64_t)row * N + cc + i] = v[i];
   }
   tc::fence_before();
   __syncthreads();
   if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
 }
 
-// out[i] += Σ_b part[b][map(i)] in a fixed order (blocks of 16), for the
-// [rows × cols] sub-block starting at (row0, col0) of the [128 × N] partials;
-// transpose != 0 writes out[c*rows + r].
-__global__ void k_tc_reduce(const float* __restrict__ part, int nb, int N, int row0, int rows, int col0, int cols,
-                            int transpose, float* __restrict__ out) {
-  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < rows * cols; e += gridDim.x * blockDim.x) {
-    const int r = e / cols, c = e % cols;
-    const int64_t src = (int64_t)(row0 + r) * N + col0 + c;
-    float tot = 0.f;
+// Fixed-order sum of the per-CTA partials: tot[e] = Σ_b part[b][e] (blocks of 16).
+__global__ void k_tc_sum_parts(const float* __restrict__ part, int nb, int n, float* __restrict__ tot) {
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
+    float t = 0.f;
     for (int b0 = 0; b0 < nb; b0 += 16) {
       float blk = 0.f;
       const int b1 = min(b0 + 16, nb);
-      for (int b = b0; b < b1; ++b) blk += part[(int64_t)b * 128 * N + src];
-      tot += blk;
+      for (int b = b0; b < b1; ++b) blk += part[(int64_t)b * n + e];
+      t += blk;
     }
-    out[transpose ? (int64_t)c * rows + r : (int64_t)r * cols + c] += tot;
+    tot[e] = t;
   }
 }
 
-// db = Σ_rows dC = dl_g·L_g¹ᵀ per gate (linear in the per-gate sums of da).
-__global__ void k_db_from_dl(int H, const float* __restrict__ dl_new, const float* __restrict__ L,
-                             float* __restrict__ db) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= 3 * H) return;
-  const int g = c / H, i = c % H;
-  const float* Lg = L + (int64_t)g * 2 * H * H;
-  float s = 0.f;
-  for (int j = 0; j < H; ++j) s = fmaf(dl_new[g * H + j], Lg[i * H + j], s);
-  db[c] += s;
+// Scatter the dL / dl / db pieces out of tot = [D1 (128 × 3H) | D2 (128 × 3H)]:
+//   D1 rows: C_z | C_r | C_h | H,  D2 rows: RH | ones;  columns da_z | da_r | da_h
+__global__ void k_dl_scatter(int H, const float* __restrict__ tot, const float* __restrict__ L,
+                             float* __restrict__ dL, float* __restrict__ dl, float* __restrict__ db) {
+  const int H3 = 3 * H, LG = 2 * H * H;
+  const float* D1 = tot;
+  const float* D2 = tot + 128 * H3;
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < 6 * H * H + 6 * H; e += gridDim.x * blockDim.x) {
+    if (e < 6 * H * H) {
+      const int g = e / LG, rem = e % LG, i = rem / H, j = rem % H;
+      float v;
+      if (i < H) v = D1[(g * H + i) * H3 + g * H + j];                 // C_gᵀ da_g
+      else if (g < 2) v = D1[(3 * H + i - H) * H3 + g * H + j];       // Hᵀ da_z, Hᵀ da_r
+      else v = D2[(i - H) * H3 + 2 * H + j];                          // RHᵀ da_h
+      dL[e] += v;
+    } else if (e < 6 * H * H + 3 * H) {
+      const int c = e - 6 * H * H;
+      dl[c] += D2[H * H3 + c];                                        // ones row: Σ_rows da
+    } else {
+      const int c = e - 6 * H * H - 3 * H, g = c / H, i = c % H;      // db_g = dl_g · L_g¹ᵀ
+      const float* Lg = L + (int64_t)g * LG;
+      float s = 0.f;
+      for (int j = 0; j < H; ++j) s = fmaf(D2[H * H3 + g * H + j], Lg[i * H + j], s);
+      db[c] += s;
+    }
+  }
+}
+
+// dW[f][c] += tot[c][f]  (tot = D = dPᵀ·X, [128 × Np])
+__global__ void k_dw_scatter(int F, int N3, int Np, const float* __restrict__ tot, float* __restrict__ dW) {
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < F * N3; e += gridDim.x * blockDim.x) {
+    const int f = e / N3, c = e % N3;
+    dW[e] += tot[c * Np + f];
+  }
 }
 
 template <class K>
-int occupancy_blocks(K fn, size_t smem) {
+int occupancy_blocks(K fn, size_t smem, int threads = kTcThreads) {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kTcThreads, smem) != cudaSuccess || per_sm < 1) {
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem) != cudaSuccess || per_sm < 1) {
     cudaGetLastError();
     per_sm = 1;
   }
@@ -595,7 +649,7 @@ stg_status prep(K fn, size_t smem) {
 
 // ------------------------------------------------------------------ host side
 bool tc_supported(int F, int H) { return (H == 16 || H == 32) && F % 4 == 0 && F <= 128 && F >= 4; }
-// part for tc_dw / tc_dl: 2 · tc_atb_max_blocks() · 128 · max(3H, roundup16(F)) floats
+// part for tc_dw / tc_dl: tc_atb_max_blocks() · 2 · 128 · 128 floats; tot: 2 · 128 · 128
 
 stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s) {
   const int N = 3 * H, Kp = (F + 7) / 8 * 8;
@@ -620,13 +674,13 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
   if (H == 32) {
     const size_t smem = 6 * GruSmem<32>::BG + 2 * GruSmem<32>::A1;
     STG_TRY(prep(k_tc_gru_fwd<32>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_fwd<32>, smem));
-    k_tc_gru_fwd<32><<<nb, kTcThreads, smem, s>>>(V, C, Hp, L, l, Hn);
+    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_fwd<32>, smem, kGruThreads));
+    k_tc_gru_fwd<32><<<nb, kGruThreads, smem, s>>>(V, C, Hp, L, l, Hn);
   } else {
     const size_t smem = 6 * GruSmem<16>::BG + 2 * GruSmem<16>::A1;
     STG_TRY(prep(k_tc_gru_fwd<16>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_fwd<16>, smem));
-    k_tc_gru_fwd<16><<<nb, kTcThreads, smem, s>>>(V, C, Hp, L, l, Hn);
+    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_fwd<16>, smem, kGruThreads));
+    k_tc_gru_fwd<16><<<nb, kGruThreads, smem, s>>>(V, C, Hp, L, l, Hn);
   }
   count_launch();
   return check_launch("tc_gru_fwd");
@@ -638,84 +692,77 @@ stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float
   if (H == 32) {
     const size_t smem = 12 * GruSmem<32>::BG + 2 * GruSmem<32>::A1;
     STG_TRY(prep(k_tc_gru_bwd<32>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_bwd<32>, smem));
-    k_tc_gru_bwd<32><<<nb, kTcThreads, smem, s>>>(V, C, Hp, G, L, l, ndst, dCs, dHp, da, RH);
+    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_bwd<32>, smem, kGruThreads));
+    k_tc_gru_bwd<32><<<nb, kGruThreads, smem, s>>>(V, C, Hp, G, L, l, ndst, dCs, dHp, da, RH);
   } else {
     const size_t smem = 12 * GruSmem<16>::BG + 2 * GruSmem<16>::A1;
     STG_TRY(prep(k_tc_gru_bwd<16>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_bwd<16>, smem));
-    k_tc_gru_bwd<16><<<nb, kTcThreads, smem, s>>>(V, C, Hp, G, L, l, ndst, dCs, dHp, da, RH);
+    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_bwd<16>, smem, kGruThreads));
+    k_tc_gru_bwd<16><<<nb, kGruThreads, smem, s>>>(V, C, Hp, G, L, l, ndst, dCs, dHp, da, RH);
   }
   count_launch();
   return check_launch("tc_gru_bwd");
 }
 
-// part must hold grid_max * 128 * N floats; returns the number of partial blocks.
-template <int N>
-static stg_status atb(int V, const float* A1, int64_t lda1, int FA1, const float* A2, int64_t lda2, int FA2, int ones,
-                      const float* B, int64_t ldb, int FB, float* part, int max_blocks, int* nb_out, cudaStream_t s) {
-  const size_t smem = (size_t)2 * 128 * kRK * 4 + (size_t)2 * N * kRK * 4;
-  STG_TRY(prep(k_tc_atb<N>, smem));
-  const int ntiles = (V + kRK - 1) / kRK;
-  int nb = std::min(std::min(ntiles, occupancy_blocks(k_tc_atb<N>, smem)), max_blocks);
+int tc_atb_max_blocks() { return num_sms(); }
+
+template <int N, int NA>
+static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
+  constexpr int STAGE = NA * 2 * (128 / 8) * (kRK / 4) * 144 + 2 * (N / 8) * (kRK / 4) * 144;
+  const size_t smem = 2 * (size_t)STAGE;
+  STG_CUDA(cudaFuncSetAttribute(k_tc_atb<N, NA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int ntiles = (args.V + kRK - 1) / kRK;
+  int nb = std::min(ntiles, tc_atb_max_blocks());
   if (nb < 1) nb = 1;
-  k_tc_atb<N><<<nb, kTcThreads, smem, s>>>(V, A1, lda1, FA1, A2, lda2, FA2, ones, B, ldb, FB, part);
+  k_tc_atb<N, NA><<<nb, kAtbThreads, smem, s>>>(args);
   count_launch();
   *nb_out = nb;
   return check_launch("tc_atb");
 }
 
-int tc_atb_max_blocks() { return 2 * num_sms(); }
-
-// dW[f][c] += Σ_v X[v,f]·dP[v,c]  via D = dPᵀ·X  ([3H pad 128] × F)
-stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* dW, cudaStream_t s) {
+// dW[f][c] += Σ_v X[v,f]·dP[v,c]  via D = dPᵀ·X  ([3H pad 128] × roundup16(F)).
+// part: tc_atb_max_blocks() · 2 · 128 · 128 floats; tot: 2 · 128 · 128 floats.
+stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* tot, float* dW,
+                 cudaStream_t s) {
+  AtbArgs a{};
+  a.V = V; a.A1 = dP; a.lda1 = 3 * H; a.FA1 = 3 * H; a.B = X; a.ldb = F; a.FB = F; a.part = part;
   int nb = 0;
   const int Np = (F + 15) / 16 * 16;
   switch (Np) {
-    case 16: STG_TRY(atb<16>(V, dP, 3 * H, 3 * H, nullptr, 0, 0, 0, X, F, F, part, tc_atb_max_blocks(), &nb, s)); break;
-    case 32: STG_TRY(atb<32>(V, dP, 3 * H, 3 * H, nullptr, 0, 0, 0, X, F, F, part, tc_atb_max_blocks(), &nb, s)); break;
-    case 48: STG_TRY(atb<48>(V, dP, 3 * H, 3 * H, nullptr, 0, 0, 0, X, F, F, part, tc_atb_max_blocks(), &nb, s)); break;
-    case 64: STG_TRY(atb<64>(V, dP, 3 * H, 3 * H, nullptr, 0, 0, 0, X, F, F, part, tc_atb_max_blocks(), &nb, s)); break;
-    case 96: STG_TRY(atb<96>(V, dP, 3 * H, 3 * H, nullptr, 0, 0, 0, X, F, F, part, tc_atb_max_blocks(), &nb, s)); break;
-    case 128: STG_TRY(atb<128>(V, dP, 3 * H, 3 * H, nullptr, 0, 0, 0, X, F, F, part, tc_atb_max_blocks(), &nb, s)); break;
+    case 16: STG_TRY((atb<16, 1>(a, &nb, s))); break;
+    case 32: STG_TRY((atb<32, 1>(a, &nb, s))); break;
+    case 48: STG_TRY((atb<48, 1>(a, &nb, s))); break;
+    case 64: STG_TRY((atb<64, 1>(a, &nb, s))); break;
+    case 96: STG_TRY((atb<96, 1>(a, &nb, s))); break;
+    case 128: STG_TRY((atb<128, 1>(a, &nb, s))); break;
     default: return fail(STG_ERR_INVALID_ARG, "tc_dw: F=%d", F);
   }
-  // D row c (dP feature) × column f (X feature) -> dW[f][c] (transpose)
-  k_tc_reduce<<<(3 * H * F + 255) / 256, 256, 0, s>>>(part, nb, Np, 0, 3 * H, 0, F, 1, dW);
-  count_launch();
+  const int n = 128 * Np;
+  k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
+  k_dw_scatter<<<(F * 3 * H + 255) / 256, 256, 0, s>>>(F, 3 * H, Np, tot, dW);
+  count_launch(2);
   return check_launch("tc_dw");
 }
 
-// dL, dl, db from C, H, RH, da (see k_tc_gru_bwd).  scratch: part (2 × max_blocks × 128 × 3H), dl_tmp [3H].
+// dL, dl, db from C, H, RH, da (see k_tc_gru_bwd) with ONE reduction kernel:
+//   D1 = [C_z|C_r|C_h|H]ᵀ·da,  D2 = [RH|1]ᵀ·da  (da = [da_z|da_r|da_h]).
 stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
-                 float* dl_tmp, float* dL, float* dl, float* db, const float* L, cudaStream_t s) {
-  const int H3 = 3 * H, LG = 2 * H * H;
-  int nb1 = 0, nb2 = 0;
-  float* part2 = part + (size_t)tc_atb_max_blocks() * 128 * H3;
-  // D1 = [C_z|C_r|C_h|H]ᵀ · [da_z|da_r|da_h]   (4H = 128 feature rows for H = 32)
-  // D2 = [RH | 1]ᵀ · [da_z|da_r|da_h]
-  if (H == 32) {
-    STG_TRY(atb<96>(V, C, H3, H3, Hp, H, H, 0, da, H3, H3, part, tc_atb_max_blocks(), &nb1, s));
-    STG_TRY(atb<96>(V, RH, H, H, nullptr, 0, 0, 1, da, H3, H3, part2, tc_atb_max_blocks(), &nb2, s));
-  } else {
-    STG_TRY(atb<48>(V, C, H3, H3, Hp, H, H, 0, da, H3, H3, part, tc_atb_max_blocks(), &nb1, s));
-    STG_TRY(atb<48>(V, RH, H, H, nullptr, 0, 0, 1, da, H3, H3, part2, tc_atb_max_blocks(), &nb2, s));
-  }
-  for (int g = 0; g < 3; ++g) {
-    // dL_g¹ [H × H] = D1 block (rows gH.., cols gH..); dL_g² (z, r) = D1 rows 3H.., cols gH..
-    k_tc_reduce<<<(H * H + 255) / 256, 256, 0, s>>>(part, nb1, H3, g * H, H, g * H, H, 0, dL + g * LG);
-    if (g < 2)
-      k_tc_reduce<<<(H * H + 255) / 256, 256, 0, s>>>(part, nb1, H3, 3 * H, H, g * H, H, 0, dL + g * LG + H * H);
-    else
-      k_tc_reduce<<<(H * H + 255) / 256, 256, 0, s>>>(part2, nb2, H3, 0, H, 2 * H, H, 0, dL + g * LG + H * H);
-  }
-  cudaMemsetAsync(dl_tmp, 0, sizeof(float) * H3, s);
-  k_tc_reduce<<<1, 256, 0, s>>>(part2, nb2, H3, H, 1, 0, H3, 0, dl_tmp);
-  k_db_from_dl<<<1, 128, 0, s>>>(H, dl_tmp, L, db);
-  count_launch(7);
-  // dl += dl_tmp
-  k_tc_reduce<<<1, 256, 0, s>>>(part2, nb2, H3, H, 1, 0, H3, 0, dl);
-  count_launch();
+                 float* tot, float* dL, float* dl, float* db, const float* L, cudaStream_t s) {
+  const int H3 = 3 * H;
+  AtbArgs a{};
+  a.V = V;
+  a.A1 = C; a.lda1 = H3; a.FA1 = H3;
+  a.A2 = Hp; a.lda2 = H; a.FA2 = H;
+  a.A3 = RH; a.lda3 = H; a.FA3 = H; a.ones = 1;
+  a.B = da; a.ldb = H3; a.FB = H3;
+  a.part = part;
+  int nb = 0;
+  if (H == 32) STG_TRY((atb<96, 2>(a, &nb, s)));
+  else STG_TRY((atb<48, 2>(a, &nb, s)));
+  const int n = 2 * 128 * H3;
+  k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
+  k_dl_scatter<<<(6 * H * H + 6 * H + 255) / 256, 256, 0, s>>>(H, tot, L, dL, dl, db);
+  count_launch(2);
   return check_launch("tc_dl");
 }
 

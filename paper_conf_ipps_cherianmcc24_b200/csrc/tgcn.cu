@@ -22,9 +22,10 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
                       cudaStream_t s);
 stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float* G, const float* L, const float* l,
                       const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s);
-stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* dW, cudaStream_t s);
+stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* tot, float* dW,
+                 cudaStream_t s);
 stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
-                 float* dl_tmp, float* dL, float* dl, float* db, const float* L, cudaStream_t s);
+                 float* tot, float* dL, float* dl, float* db, const float* L, cudaStream_t s);
 stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
                             float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
                             cudaStream_t s);
@@ -580,8 +581,8 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
   if (tc_supported(F, H)) {
     STG_TRY(ws.da.alloc((size_t)V * H3));
     STG_TRY(ws.RH.alloc((size_t)V * H));
-    STG_TRY(ws.part_tc.alloc((size_t)2 * tc_atb_max_blocks() * 128 * std::max(H3, (F + 15) / 16 * 16)));
-    STG_TRY(ws.dl_tmp.alloc(H3));
+    STG_TRY(ws.part_tc.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));
+    STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
     {
       ProfScope prof(PH_GRU_BWD, s);
       STG_TRY(tc_gru_bwd(V, H, e.C, e.Hp, dH_next, p->L, p->l, g->norm_dst, ws.dC.p, dH_prev, ws.da.p, ws.RH.p, s));
@@ -591,7 +592,7 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
     STG_TRY(aggregate_launch(g, 1, H3, ws.dC.p, H3, ws.dP.p, H3, g->norm_src, nullptr, nullptr, s));
     {
       ProfScope prof(PH_DW, s);
-      STG_TRY(tc_dw(V, F, H, X, ws.dP.p, ws.part_tc.p, grads->W, s));
+      STG_TRY(tc_dw(V, F, H, X, ws.dP.p, ws.part_tc.p, ws.dl_tmp.p, grads->W, s));
     }
     STG_TRY(check_launch("stg_tgcn_step_backward"));
     stack->entries.pop_back();
