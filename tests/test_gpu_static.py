@@ -210,3 +210,13 @@ def test_every_strategy_matches_oracle(stg, strategy, W):
             assert torch.equal(y1, y2)               # deterministic
     finally:
         stg.stg_aggregate_set_strategy(0)
+
+
+def test_device_partition_matches_host(stg):
+    from paper_conf_ipps_cherianmcc24_b200 import parallel
+    cfg = gen.CONFIGS["C2"]
+    s, d = gen.static_edges(cfg)
+    g = stg.stg_static_graph_create(cfg.V, s, d, stg.STG_SELF_LOOPS)
+    rp = stg.view_arrays(g.view())["in_rowptr"]
+    for world in (1, 2, 4, 8):
+        assert stg.stg_partition_rows(cfg.V, rp, world) == parallel.row_blocks(rp.cpu().numpy(), world)
