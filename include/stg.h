@@ -168,14 +168,25 @@ stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t
                                 const float* scale_row, const float* scale_col, const float* bias,
                                 stg_stream_t stream);
 
-/* Work decomposition of the aggregation kernel (float4 path):
- * 0 (default) = degree-ordered row items (node_ids order, hub rows chunked;
- *     FA-TGA lane groups, register gathers);  1 = as 0 with cp.async gathers;
- * 2 = edge-parallel: warps stream contiguous 128-edge chunks of the CSR
- *     (nnz-balanced) with TMA bulk row copies, rows split across chunks
- *     finished in chunk order (W >= 64, views with the COO row array).
- * Every strategy is deterministic; 0 and 1 are bit-identical. */
+/* Work decomposition of the aggregation (process-wide; every strategy is
+ * deterministic, uses no float atomics, and keeps each fp32 chain <= 64 terms).
+ * The snapshot schedule lists rows in node_ids order (degree presort,
+ * P:L175/L322) as items of <= 64 edges (hub rows cut into chunks).
+ * 2 (default) = edge stream: a warp walks the concatenated edge lists of 32
+ *     items, gathering several neighbour rows at once across row boundaries
+ *     (float4 path, 32 < W <= 128 per column launch; wider W is split into
+ *     launches of <= 128 columns; otherwise strategy 1 is used);
+ * 1 = pipelined items: FA-TGA lane groups serve 32/G rows per warp
+ *     with the next items' descriptors and columns prefetched (float4 path);
+ * 0 = row items with register gathers (any width/alignment; also the path of
+ *     caller-built views without a schedule). */
 stg_status stg_aggregate_set_strategy(int32_t strategy);
+/* Tunables of strategy 2 (STG_ERR_INVALID_ARG for a bad key/value):
+ * key 0: neighbour rows in flight per warp, 4 | 8 | 16 (default 16);
+ * key 1: minimum resident blocks per SM (register budget), 2..6 (default 3;
+ *        supported pairs (rows, blocks): (4,6) (8,4) (16,2) (16,3));
+ * key 2: 32 | 64 (default 32): strategy 2 serves launch widths above this. */
+stg_status stg_aggregate_set_param(int32_t key, int64_t value);
 
 /* ---- TGCN (GCN + GRU; reading C13-C15) ----
  * W [F,3H] (gates z|r|h), b [3H], L [3][2H][H] (gate g: rows 0..H-1 = L_g¹ act

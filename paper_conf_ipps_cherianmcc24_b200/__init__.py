@@ -105,6 +105,7 @@ _decl("stg_partition_rows", [_i32, _P, _i32, ctypes.POINTER(_i32), _P])
 _decl("stg_profile_enable", [_i32])
 _decl("stg_debug_tc_gemm", [_i32, _i32, _i32, _i32, _i32, _P, _P, _P, _P])
 _decl("stg_aggregate_set_strategy", [_i32])
+_decl("stg_aggregate_set_param", [_i32, _i64])
 _decl("stg_profile_read", [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64), _i32])
 
 ABI_SYMBOLS = [
@@ -116,6 +117,7 @@ ABI_SYMBOLS = [
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
     "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_sgd_update", "stg_tgcn_train_sequence",
     "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
+    "stg_aggregate_set_param",
 ]
 
 PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head"]
@@ -431,5 +433,13 @@ def stg_debug_tc_gemm(mode: int, A: torch.Tensor, B: torch.Tensor, stream=None) 
 
 
 def stg_aggregate_set_strategy(strategy: int):
-    """0 = degree-ordered row items (default), 1 = row items with cp.async gathers, 2 = edge-parallel TMA."""
+    """2 = edge stream (default), 1 = pipelined row items, 0 = row items (include/stg.h)."""
     _check(_lib.stg_aggregate_set_strategy(int(strategy)))
+
+
+AGG_ROWS_IN_FLIGHT, AGG_MIN_BLOCKS, AGG_STREAM_WMIN = 0, 1, 2
+
+
+def stg_aggregate_set_param(key: int, value: int):
+    """Edge-stream tunables (include/stg.h): 0 rows in flight, 1 min blocks/SM, 2 min width."""
+    _check(_lib.stg_aggregate_set_param(int(key), int(value)))

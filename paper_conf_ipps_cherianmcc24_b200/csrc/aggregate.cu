@@ -1,23 +1,30 @@
 // aggregate.cu — vertex-centric GCN aggregation for sm_100a (north_star; P:L72,
-// L195, L322).  One kernel serves the forward (in-CSR) and the backward
+// L195, L322).  One kernel family serves the forward (in-CSR) and the backward
 // (out-CSR, the exact transpose):
 //
 //   out[r,:] = scale_row[r] · Σ_{j ∈ row r} scale_col[col[j]] · in[col[j],:] + bias
 //
-// Design:
-//  * feature-adaptive thread groups (the paper's FA-TGA): a row is
-//    owned by a group of G lanes; each lane holds VPL 128-bit vectors of the
-//    row (G·VPL·4 >= W), so a 32-lane warp works on 32/G rows at once;
-//  * rows are taken in node_ids order (degree-descending presort)
-//    so the rows sharing a warp have similar degrees;
-//  * rows with more than kHubChunk edges are split into fixed chunks of
-//    kHubChunk edges (hub items first); the last chunk to finish sums the
-//    chunk partials in a fixed order — deterministic, no float atomics;
-//  * column indices are loaded coalesced, one per lane, and broadcast with
-//    __shfl_sync; feature rows are gathered with 128-bit ld.global.nc;
-//  * U independent accumulators per vector bound every sequential fp32 chain
-//    to <= 64 terms (reading C19/C20 error bound).
-//  * persistent grid of (#SMs × resident blocks), grid-stride over work items.
+// Work list: the snapshot's schedule (graph.cuh) lists the rows in node_ids
+// order (degree-descending presort) as work items of <= 64 edges
+// (hub rows are cut into 64-edge chunks).  Three decompositions
+// (stg_aggregate_set_strategy; DESIGN.md §Aggregation has the measurements):
+//
+//  2 (default, 64 < W <= 128 per launch) k_agg_stream: a warp takes 32 items
+//    at a time from a work queue, scans their edge counts and walks their
+//    concatenated edge lists in 32-edge batches, gathering D neighbour rows at
+//    once ACROSS row boundaries (lane c holds float4 column c of a row), with
+//    the next batch's column ids and the next group's descriptors in flight;
+//    hub chunks leave partial sums that k_agg_hubs adds in fixed order.
+//  1 k_agg_items: a warp serves 32/G rows at once (feature-adaptive lane
+//    groups, the paper's FA-TGA) with a three-stage prefetch across
+//    items (descriptor i+2, first column batch of i+1, gathers of i); the last
+//    chunk of a hub row to finish sums the chunk partials (atomic ticket).
+//  0 k_aggregate: the same lane groups without the schedule prefetch; also the
+//    path for caller-built views without a schedule.
+//
+// Every fp32 chain is <= 64 terms (one accumulator per <= 64-edge item; hub
+// partials are summed in blocks of 16 then in a fixed order), there are no
+// float atomics, and every result is deterministic run to run (reading C20).
 #include <map>
 #include <mutex>
 
@@ -86,7 +93,7 @@ __global__ void __launch_bounds__(kAggThreads) k_aggregate(const AggArgs a) {
   const int gi = lane / G, gl = lane % G;
   const int32_t n_hub = a.sched ? a.sched[0] : 0;
   const int32_t n_chunks = a.sched ? a.sched[1] : 0;
-  const int32_t* cptr = a.sched ? a.sched + 2 : nullptr;
+  const int32_t* cptr = a.sched ? a.sched + a.sched[2] : nullptr;
   const int64_t total = (int64_t)n_chunks + (a.R - n_hub);
   const int64_t warp_id = ((int64_t)blockIdx.x * kAggThreads + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * kAggThreads) >> 5;
@@ -227,226 +234,10 @@ __global__ void __launch_bounds__(kAggThreads) k_aggregate(const AggArgs a) {
 
 
 // ---------------------------------------------------------------------------
-// Asynchronous-gather variant (float4 path, W <= 128): per warp a double-
-// buffered ring of 32 row slots in shared memory.  For each batch the warp
-// loads the 32 column indices (one per lane, coalesced), then issues the row
-// copies as 16-byte cp.async (LDGSTS, no register destinations) for batch b+1
-// while it consumes batch b from shared memory.  Slot s belongs to group
-// s / G (the G lanes that own one row item); accumulation order per row is the
-// same fixed edge order as k_aggregate, so results are deterministic.
-template <int G, int VPL, int U, bool SCOL>
-__global__ void __launch_bounds__(kAggThreads) k_aggregate_async(const AggArgs a, int warps_per_block) {
-  constexpr int NG = 32 / G;                 // row items per warp
-  constexpr int EPG = G;                     // slots (edges) per item per batch
-  const unsigned FULL = 0xffffffffu;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  if (wib >= warps_per_block) return;
-  const int gi = lane / G, gl = lane % G;
-  const int W = a.W, nv = W / 4;             // row length in float4
-  const int slot_bytes = W * 4;
-  unsigned char* wbase = smem_raw + (size_t)wib * (2 * 32 * slot_bytes + 2 * 32 * 4);
-  unsigned char* buf[2] = {wbase, wbase + 32 * slot_bytes};
-  float* scs[2] = {reinterpret_cast<float*>(wbase + 2 * 32 * slot_bytes),
-                   reinterpret_cast<float*>(wbase + 2 * 32 * slot_bytes) + 32};
-  const int32_t n_hub = a.sched ? a.sched[0] : 0;
-  const int32_t n_chunks = a.sched ? a.sched[1] : 0;
-  const int32_t* cptr = a.sched ? a.sched + 2 : nullptr;
-  const int64_t total = (int64_t)n_chunks + (a.R - n_hub);
-  const int64_t warp_id = (int64_t)blockIdx.x * warps_per_block + wib;
-  const int64_t nwarps = (int64_t)gridDim.x * warps_per_block;
-
-  for (int64_t base = warp_id * NG; base < total; base += nwarps * NG) {
-    const int64_t item = base + gi;
-    const bool valid = item < total;
-    int32_t v = 0, beg = 0, end = 0, hub = -1;
-    if (valid) {
-      if (item < n_chunks) {
-        int32_t lo = 0, hi = n_hub;
-        while (lo < hi) {
-          int32_t mid = (lo + hi + 1) >> 1;
-          if (cptr[mid] <= item) lo = mid; else hi = mid - 1;
-        }
-        hub = lo;
-        v = a.ids[lo];
-        int32_t rb = a.rowptr[v], re = a.rowptr[v + 1];
-        beg = rb + (int32_t)(item - cptr[lo]) * kHubChunk;
-        end = min(beg + kHubChunk, re);
-      } else {
-        int64_t li = n_hub + (item - n_chunks);
-        v = a.ids ? a.ids[li] : (int32_t)li;
-        beg = a.rowptr[v];
-        end = a.rowptr[v + 1];
-      }
-    }
-    const int32_t n = end - beg;
-    const int32_t nmax = __reduce_max_sync(FULL, n);
-    const int nb = (nmax + EPG - 1) / EPG;
-    // lane s describes slot s: group s / EPG, edge (b·EPG + s % EPG) of that group
-    const int sg = lane / EPG, se = lane % EPG;
-    const int32_t s_beg = __shfl_sync(FULL, beg, sg * G);
-    const int32_t s_n = __shfl_sync(FULL, n, sg * G);
-
-    auto issue = [&](int b, int which) {
-      const int e = b * EPG + se;
-      const int32_t u = e < s_n ? __ldg(a.col + s_beg + e) : -1;
-      if (SCOL) scs[which][lane] = u >= 0 ? __ldg(a.scol + u) : 0.0f;
-      const uint32_t dst0 = (uint32_t)__cvta_generic_to_shared(buf[which]);
-      for (int p = lane; p < 32 * nv; p += 32) {
-        const int slot = p / nv, ch = p - slot * nv;
-        const int32_t us = __shfl_sync(FULL, u, slot);
-        if (us >= 0) {
-          const float* src = a.x + (int64_t)us * a.ldx + 4 * ch;
-          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(dst0 + (uint32_t)(slot * slot_bytes + 16 * ch)),
-                       "l"(src)
-                       : "memory");
-        }
-      }
-      asm volatile("cp.async.commit_group;\n" ::: "memory");
-    };
-
-    float4 acc[U][VPL];
-#pragma unroll
-    for (int u = 0; u < U; ++u)
-#pragma unroll
-      for (int c = 0; c < VPL; ++c) acc[u][c] = make_float4(0.f, 0.f, 0.f, 0.f);
-
-    if (nb > 0) issue(0, 0);
-    for (int b = 0; b < nb; ++b) {
-      if (b + 1 < nb) {
-        issue(b + 1, (b + 1) & 1);
-        asm volatile("cp.async.wait_group 1;\n" ::: "memory");
-      } else {
-        asm volatile("cp.async.wait_group 0;\n" ::: "memory");
-      }
-      __syncwarp();
-      const unsigned char* bb = buf[b & 1];
-      const float* sc = scs[b & 1];
-#pragma unroll
-      for (int e = 0; e < EPG; ++e) {
-        if (b * EPG + e < n) {
-          const int slot = gi * EPG + e;
-          const float4* row = reinterpret_cast<const float4*>(bb + slot * slot_bytes);
-          const float ssc = SCOL ? sc[slot] : 1.0f;
-#pragma unroll
-          for (int c = 0; c < VPL; ++c) {
-            const int cv = c * G + gl;
-            if (cv < nv) {
-              const float4 xv = row[cv];
-              if (SCOL) fma_v(acc[e % U][c], ssc, xv);
-              else add_v(acc[e % U][c], xv);
-            }
-          }
-        }
-      }
-      __syncwarp();
-    }
-#pragma unroll
-    for (int w = 1; w < U; w <<= 1)
-#pragma unroll
-      for (int u = 0; u < U; u += 2 * w)
-#pragma unroll
-        for (int c = 0; c < VPL; ++c) add_v(acc[u][c], acc[u + w][c]);
-
-    const bool hubitem = valid && hub >= 0;
-    if (valid && !hubitem) {
-      const float s = a.srow ? a.srow[v] : 1.0f;
-      float4* yr = reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy);
-#pragma unroll
-      for (int c = 0; c < VPL; ++c) {
-        const int cv = c * G + gl;
-        if (cv < nv) yr[cv] = scale_bias(s, acc[0][c], a.bias, cv * 4);
-      }
-    }
-    if (hubitem) {
-      float4* pr = reinterpret_cast<float4*>(a.partials + item * (int64_t)W);
-#pragma unroll
-      for (int c = 0; c < VPL; ++c) {
-        const int cv = c * G + gl;
-        if (cv < nv) pr[cv] = acc[0][c];
-      }
-      __threadfence();
-    }
-    __syncwarp();
-    int32_t ticket = 0;
-    if (hubitem && gl == 0) ticket = atomicAdd(a.counters + hub, 1);
-    ticket = __shfl_sync(FULL, ticket, gi * G);
-    const bool last = hubitem && ticket == (cptr[hub + 1] - cptr[hub]) - 1;
-    if (last) {
-      __threadfence();
-      const int32_t cb = cptr[hub], ce = cptr[hub + 1];
-      float4 tot[VPL];
-#pragma unroll
-      for (int c = 0; c < VPL; ++c) tot[c] = make_float4(0.f, 0.f, 0.f, 0.f);
-      for (int32_t c0 = cb; c0 < ce; c0 += 16) {
-        float4 blk[VPL];
-#pragma unroll
-        for (int c = 0; c < VPL; ++c) blk[c] = make_float4(0.f, 0.f, 0.f, 0.f);
-        const int32_t c1 = min(c0 + 16, ce);
-        for (int32_t ch = c0; ch < c1; ++ch) {
-          const float4* pr = reinterpret_cast<const float4*>(a.partials + (int64_t)ch * W);
-#pragma unroll
-          for (int c = 0; c < VPL; ++c) {
-            const int cv = c * G + gl;
-            if (cv < nv) add_v(blk[c], __ldcg(pr + cv));
-          }
-        }
-#pragma unroll
-        for (int c = 0; c < VPL; ++c) add_v(tot[c], blk[c]);
-      }
-      const float s = a.srow ? a.srow[v] : 1.0f;
-      float4* yr = reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy);
-#pragma unroll
-      for (int c = 0; c < VPL; ++c) {
-        const int cv = c * G + gl;
-        if (cv < nv) yr[cv] = scale_bias(s, tot[c], a.bias, cv * 4);
-      }
-      if (gl == 0) a.counters[hub] = 0;
-    }
-  }
-}
-
-using AsyncFn = void (*)(const AggArgs, int);
-
-template <int G, bool SCOL>
-AsyncFn pick_async_vpl(int vpl) {
-  switch (vpl) {
-    case 1: return k_aggregate_async<G, 1, 4, SCOL>;
-    case 2: return k_aggregate_async<G, 2, 4, SCOL>;
-    case 3: return k_aggregate_async<G, 3, 2, SCOL>;
-    default: return k_aggregate_async<G, 4, 2, SCOL>;
-  }
-}
-template <bool SCOL>
-AsyncFn pick_async_g(int g, int vpl) {
-  switch (g) {
-    case 1: return pick_async_vpl<1, SCOL>(vpl);
-    case 2: return pick_async_vpl<2, SCOL>(vpl);
-    case 4: return pick_async_vpl<4, SCOL>(vpl);
-    case 8: return pick_async_vpl<8, SCOL>(vpl);
-    case 16: return pick_async_vpl<16, SCOL>(vpl);
-    default: return pick_async_vpl<32, SCOL>(vpl);
-  }
-}
-
-// ---------------------------------------------------------------------------
-// Edge-parallel ("merge-path") variant for W <= 128 float4 rows: warp w streams
-// the contiguous edge chunks c = w, w + nwarps, ... of kEdgeChunk edges.  Column
-// and row ids are read 32 at a time (coalesced) and broadcast; 8 feature-row
-// gathers are in flight per lane; a row is flushed when the row id changes.
-// Rows fully inside a chunk are written directly; a row split across chunks
-// [c_a, c_b] leaves one partial per chunk (slot 2c_a+1, then 2c for c > c_a) and
-// the last chunk to finish (atomic ticket per row, self-resetting) sums them in
-// chunk order.  Two accumulators alternate on edge parity: every fp32 chain is
-// <= 64 terms, results are deterministic, no float atomics.
-constexpr int kEdgeChunk = 128;
-
-struct EdgeArgs {
-  int32_t R;
-  int64_t E;
-  const int32_t* rowptr;
+// Arguments of the schedule-driven kernels (strategies 1 and 2).
+struct Agg2Args {
+  const int32_t* sched;
   const int32_t* col;
-  const int32_t* row;
   const float* srow;
   const float* scol;
   const float* bias;
@@ -455,266 +246,386 @@ struct EdgeArgs {
   int64_t ldx;
   float* y;
   int64_t ldy;
-  float* partials;   // [2 * nchunks][W]
-  int32_t* counters; // [R]
+  float* partials;
+  int32_t* counters;
 };
 
-__device__ __forceinline__ void edge_write_row(const EdgeArgs& a, int32_t r, float4 v, int lane, int nv) {
-  if (lane < nv) {
-    const float s = a.srow ? a.srow[r] : 1.0f;
-    reinterpret_cast<float4*>(a.y + (int64_t)r * a.ldy)[lane] = scale_bias(s, v, a.bias, 4 * lane);
-  }
-}
-
-template <bool SCOL>
-__global__ void __launch_bounds__(kAggThreads) k_agg_edges(const EdgeArgs a) {
-  constexpr int U = 8;
+// Strategy 1: software-pipelined degree-ordered items.  A warp serves 32/G
+// items at once (G lanes × VPL float4 per row) and runs a three-stage pipeline
+// across its items: item i+2's descriptor and item i+1's first column batch
+// are loaded while item i's neighbour rows are gathered; inside an item the
+// next column batch is loaded while the current one is gathered.
+template <int G, int VPL, int BT, bool SCOL>
+__global__ void __launch_bounds__(kAggThreads, 4) k_agg_items(const Agg2Args a) {
+  constexpr int NG = 32 / G;
+  static_assert(BT <= G && G % BT == 0, "BT must divide G");
   const unsigned FULL = 0xffffffffu;
-  const int lane = threadIdx.x & 31;
-  const int nv = a.W / 4;
-  const int64_t nchunks = (a.E + kEdgeChunk - 1) / kEdgeChunk;
+  const int lane = threadIdx.x & 31, gi = lane / G, gl = lane % G;
+  const int64_t total = a.sched[3];
+  const int32_t* cptr = a.sched + a.sched[2];
+  const int4* items = reinterpret_cast<const int4*>(a.sched + kSchedHdr);
   const int64_t warp_id = ((int64_t)blockIdx.x * kAggThreads + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * kAggThreads) >> 5;
+  const int64_t stride = (((int64_t)gridDim.x * kAggThreads) >> 5) * NG;
+  const int nv = a.W >> 2;
   const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
-  for (int64_t c = warp_id; c < nchunks; c += nwarps) {
-    const int64_t e0 = c * kEdgeChunk, e1 = (a.E < e0 + kEdgeChunk) ? a.E : e0 + kEdgeChunk;
-    const int32_t r_first = a.row[e0], r_last = a.row[e1 - 1];
-    const bool start_open = e0 > a.rowptr[r_first];
-    const bool end_open = e1 < a.rowptr[r_last + 1];
-    // empty rows in the gap before this chunk (and after the last chunk)
-    {
-      const int32_t gap0 = c == 0 ? 0 : a.row[e0 - 1] + 1;
-      for (int32_t r = gap0; r < r_first; ++r) edge_write_row(a, r, z4, lane, nv);
-      if (c == nchunks - 1)
-        for (int32_t r = r_last + 1; r < a.R; ++r) edge_write_row(a, r, z4, lane, nv);
-    }
-    int32_t cur = r_first;
-    float4 acc0 = z4, acc1 = z4;
-    auto flush = [&](int32_t r) {
-      float4 v = acc0;
-      add_v(v, acc1);
-      const bool open_s = (r == r_first) && start_open, open_e = (r == r_last) && end_open;
-      if (!open_s && !open_e) {
-        edge_write_row(a, r, v, lane, nv);
-        return;
+
+  int64_t item = warp_id * NG + gi;
+  int4 m0 = item < total ? __ldcs(items + item) : make_int4(0, 0, 0, -2);
+  int4 m1 = item + stride < total ? __ldcs(items + item + stride) : make_int4(0, 0, 0, -2);
+  int32_t idx0 = gl < m0.z ? __ldcs(a.col + m0.y + gl) : -1;
+  float s0 = (a.srow && m0.w > -2) ? __ldg(a.srow + m0.x) : 1.0f;
+
+  for (int64_t base = warp_id * NG; base < total; base += stride, item += stride) {
+    // stage 1: descriptor of item i+2; stage 2: first column batch (+ row scale) of item i+1
+    const int64_t i2 = item + 2 * stride;
+    const int4 m2 = i2 < total ? __ldcs(items + i2) : make_int4(0, 0, 0, -2);
+    const int32_t idx1 = gl < m1.z ? __ldcs(a.col + m1.y + gl) : -1;
+    const float s1 = (a.srow && m1.w > -2) ? __ldg(a.srow + m1.x) : 1.0f;
+    // stage 3: gather item i
+    const int32_t n = m0.z;
+    const int32_t nmax = __reduce_max_sync(FULL, n);
+    float4 acc[VPL];
+#pragma unroll
+    for (int c = 0; c < VPL; ++c) acc[c] = z4;
+    int32_t cur = idx0;
+    for (int32_t e0 = 0; e0 < nmax; e0 += G) {
+      const int32_t en = e0 + G + gl;
+      const int32_t nxt = en < n ? __ldcs(a.col + m0.y + en) : -1;
+      const float sc = (SCOL && cur >= 0) ? __ldg(a.scol + cur) : 1.0f;
+      const int32_t jn = nmax - e0;             // warp-uniform
+#pragma unroll
+      for (int j0 = 0; j0 < G; j0 += BT) {
+        if (j0 < jn) {
+          float4 val[BT][VPL];
+          float ss[BT];
+#pragma unroll
+          for (int b = 0; b < BT; ++b) {
+            const int32_t uf = __shfl_sync(FULL, cur, gi * G + j0 + b);
+            ss[b] = SCOL ? __shfl_sync(FULL, sc, gi * G + j0 + b) : 1.0f;
+            const bool ok = uf >= 0;
+            const float4* xr = reinterpret_cast<const float4*>(a.x + (int64_t)(ok ? uf : 0) * a.ldx);
+#pragma unroll
+            for (int c = 0; c < VPL; ++c) {
+              const int cv = c * G + gl;
+              val[b][c] = (ok && cv < nv) ? __ldg(xr + cv) : z4;
+            }
+          }
+#pragma unroll
+          for (int b = 0; b < BT; ++b)
+#pragma unroll
+            for (int c = 0; c < VPL; ++c) {
+              if (SCOL) fma_v(acc[c], ss[b], val[b][c]);
+              else add_v(acc[c], val[b][c]);
+            }
+        }
       }
-      const int64_t slot = open_s ? 2 * c : 2 * c + 1;
-      if (lane < nv) reinterpret_cast<float4*>(a.partials + slot * a.W)[lane] = v;
+      cur = nxt;
+    }
+    const bool valid = m0.w > -2;
+    const int32_t hub = m0.w;
+    const int32_t v = m0.x;
+    if (valid && hub < 0) {
+      float4* yr = reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv < nv) __stcs(yr + cv, scale_bias(s0, acc[c], a.bias, cv * 4));
+      }
+    }
+    const bool hubitem = valid && hub >= 0;
+    if (hubitem) {
+      float4* pr = reinterpret_cast<float4*>(a.partials + item * (int64_t)a.W);
+#pragma unroll
+      for (int c = 0; c < VPL; ++c) {
+        const int cv = c * G + gl;
+        if (cv < nv) pr[cv] = acc[c];
+      }
       __threadfence();
-      __syncwarp();
-      const int64_t rb = a.rowptr[r], re = a.rowptr[r + 1];
-      const int64_t ca = rb / kEdgeChunk, cb = (re - 1) / kEdgeChunk;
-      int32_t ticket = 0;
-      if (lane == 0) ticket = atomicAdd(a.counters + r, 1);
-      ticket = __shfl_sync(FULL, ticket, 0);
-      if (ticket == (int32_t)(cb - ca)) {       // last chunk of row r to finish
-        __threadfence();
-        float4 tot = z4;
-        for (int64_t q0 = ca; q0 <= cb; q0 += 16) {
-          float4 blk = z4;
-          const int64_t q1 = (q0 + 16 < cb + 1) ? q0 + 16 : cb + 1;
-          for (int64_t q = q0; q < q1; ++q) {
-            const int64_t sl = q == ca ? 2 * q + 1 : 2 * q;
-            if (lane < nv) add_v(blk, __ldcg(reinterpret_cast<const float4*>(a.partials + sl * a.W) + lane));
-          }
-          add_v(tot, blk);
-        }
-        edge_write_row(a, r, tot, lane, nv);
-        if (lane == 0) a.counters[r] = 0;
-      }
-    };
-    for (int64_t base = e0; base < e1; base += 32) {
-      const int n = (int)((e1 - base) < 32 ? (e1 - base) : 32);
-      const int32_t my_col = lane < n ? __ldg(a.col + base + lane) : 0;
-      const int32_t my_row = lane < n ? __ldg(a.row + base + lane) : cur;
-      const float my_sc = (SCOL && lane < n) ? __ldg(a.scol + my_col) : 1.0f;
-      for (int j0 = 0; j0 < n; j0 += U) {
-        float4 xv[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const int32_t cj = __shfl_sync(FULL, my_col, j0 + u);
-          xv[u] = (j0 + u < n && lane < nv) ? __ldg(reinterpret_cast<const float4*>(a.x + (int64_t)cj * a.ldx) + lane)
-                                            : z4;
-        }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          if (j0 + u >= n) break;
-          const int32_t rj = __shfl_sync(FULL, my_row, j0 + u);
-          const float sj = SCOL ? __shfl_sync(FULL, my_sc, j0 + u) : 1.0f;
-          if (rj != cur) {
-            flush(cur);
-            for (int32_t r = cur + 1; r < rj; ++r) edge_write_row(a, r, z4, lane, nv);
-            cur = rj;
-            acc0 = z4;
-            acc1 = z4;
-          }
-          if (((base + j0 + u) & 1) == 0) {
-            if (SCOL) fma_v(acc0, sj, xv[u]); else add_v(acc0, xv[u]);
-          } else {
-            if (SCOL) fma_v(acc1, sj, xv[u]); else add_v(acc1, xv[u]);
-          }
-        }
-      }
     }
-    flush(cur);
-  }
-}
-
-// TMA-gather edge-parallel kernel (strategy 2): per warp two 32-slot row
-// buffers in shared memory; for every 32-edge batch each lane issues ONE bulk
-// copy (cp.async.bulk, the whole W·4-byte feature row) that completes on the
-// buffer's mbarrier (expect_tx).  The next batch (possibly of the next chunk)
-// is issued before the current one is consumed, so a warp keeps up to 64 rows
-// in flight without register destinations.  Accumulation order and the chunk /
-// split-row logic are those of k_agg_edges.
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t mbar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(mbar)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint32_t mbar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(mbar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait_parity(uint32_t mbar, uint32_t phase) {
-  asm volatile(
-      "{\n\t.reg .pred P1;\n"
-      "W_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-      "@P1 bra D_%=;\n\t"
-      "bra W_%=;\n"
-      "D_%=:\n\t}\n" ::"r"(mbar),
-      "r"(phase)
-      : "memory");
-}
-
-template <bool SCOL>
-__global__ void __launch_bounds__(kAggThreads) k_agg_edges_tma(const EdgeArgs a, int warps_per_block) {
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  __shared__ __align__(8) uint64_t mbars[kAggThreads / 32][2];
-  const unsigned FULL = 0xffffffffu;
-  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  if (wib >= warps_per_block) return;
-  const int nv = a.W / 4;
-  const uint32_t rowb = (uint32_t)a.W * 4;
-  unsigned char* wbuf = smem_raw + (size_t)wib * 2 * 32 * rowb;
-  const uint32_t sbuf0 = (uint32_t)__cvta_generic_to_shared(wbuf);
-  const uint32_t mb0 = (uint32_t)__cvta_generic_to_shared(&mbars[wib][0]);
-  const uint32_t mb1 = (uint32_t)__cvta_generic_to_shared(&mbars[wib][1]);
-  if (lane == 0) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(mb0) : "memory");
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(mb1) : "memory");
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-  }
-  __syncwarp();
-  const int64_t nchunks = (a.E + kEdgeChunk - 1) / kEdgeChunk;
-  const int64_t warp_id = (int64_t)blockIdx.x * warps_per_block + wib;
-  const int64_t nwarps = (int64_t)gridDim.x * warps_per_block;
-  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
-  uint32_t phase0 = 0, phase1 = 0;
-  // batch stream: (chunk c, edge base) in order; issue(k) fills buffer k & 1
-  int32_t q_row0 = 0, q_row1 = 0, q_n0 = 0, q_n1 = 0;   // per-buffer batch metadata (no local arrays)
-  float q_sc0 = 1.f, q_sc1 = 1.f;
-  auto issue = [&](int64_t c, int64_t base, int which) {
-    const int64_t e1 = (a.E < c * kEdgeChunk + kEdgeChunk) ? a.E : c * kEdgeChunk + kEdgeChunk;
-    const int n = (int)((e1 - base) < 32 ? (e1 - base) : 32);
-    int32_t u = 0, rw = 0;
-    float sc = 1.0f;
-    if (lane < n) {
-      u = __ldg(a.col + base + lane);
-      rw = __ldg(a.row + base + lane);
-      sc = SCOL ? __ldg(a.scol + u) : 1.0f;
-    }
-    if (which) { q_row1 = rw; q_sc1 = sc; q_n1 = n; } else { q_row0 = rw; q_sc0 = sc; q_n0 = n; }
-    const uint32_t mb = which ? mb1 : mb0;
-    if (lane == 0) mbar_expect_tx(mb, (uint32_t)n * rowb);
     __syncwarp();
-    if (lane < n) bulk_g2s(sbuf0 + (uint32_t)which * 32 * rowb + (uint32_t)lane * rowb, a.x + (int64_t)u * a.ldx, rowb, mb);
-  };
-  int64_t c = warp_id;
-  if (c >= nchunks) return;
-  int which = 0;
-  issue(c, c * kEdgeChunk, 0);
-  for (; c < nchunks; c += nwarps) {
-    const int64_t e0 = c * kEdgeChunk, e1 = (a.E < e0 + kEdgeChunk) ? a.E : e0 + kEdgeChunk;
-    const int32_t r_first = a.row[e0], r_last = a.row[e1 - 1];
-    const bool start_open = e0 > a.rowptr[r_first];
-    const bool end_open = e1 < a.rowptr[r_last + 1];
-    {
-      const int32_t gap0 = c == 0 ? 0 : a.row[e0 - 1] + 1;
-      for (int32_t r = gap0; r < r_first; ++r) edge_write_row(a, r, z4, lane, nv);
-      if (c == nchunks - 1)
-        for (int32_t r = r_last + 1; r < a.R; ++r) edge_write_row(a, r, z4, lane, nv);
-    }
-    int32_t cur = r_first;
-    float4 acc0 = z4, acc1 = z4;
-    auto flush = [&](int32_t r) {
-      float4 v = acc0;
-      add_v(v, acc1);
-      const bool open_s = (r == r_first) && start_open, open_e = (r == r_last) && end_open;
-      if (!open_s && !open_e) {
-        edge_write_row(a, r, v, lane, nv);
-        return;
-      }
-      const int64_t slot = open_s ? 2 * c : 2 * c + 1;
-      if (lane < nv) reinterpret_cast<float4*>(a.partials + slot * a.W)[lane] = v;
-      __threadfence();
-      __syncwarp();
-      const int64_t rb = a.rowptr[r], re = a.rowptr[r + 1];
-      const int64_t ca = rb / kEdgeChunk, cb = (re - 1) / kEdgeChunk;
+    if (__any_sync(FULL, hubitem)) {
       int32_t ticket = 0;
-      if (lane == 0) ticket = atomicAdd(a.counters + r, 1);
-      ticket = __shfl_sync(FULL, ticket, 0);
-      if (ticket == (int32_t)(cb - ca)) {
+      if (hubitem && gl == 0) ticket = atomicAdd(a.counters + hub, 1);
+      ticket = __shfl_sync(FULL, ticket, gi * G);
+      const bool last = hubitem && ticket == (cptr[hub + 1] - cptr[hub]) - 1;
+      if (last) {
         __threadfence();
-        float4 tot = z4;
-        for (int64_t q0 = ca; q0 <= cb; q0 += 16) {
-          float4 blk = z4;
-          const int64_t q1 = (q0 + 16 < cb + 1) ? q0 + 16 : cb + 1;
-          for (int64_t q = q0; q < q1; ++q) {
-            const int64_t sl = q == ca ? 2 * q + 1 : 2 * q;
-            if (lane < nv) add_v(blk, __ldcg(reinterpret_cast<const float4*>(a.partials + sl * a.W) + lane));
+        const int32_t cb = cptr[hub], ce = cptr[hub + 1];
+        float4 tot[VPL];
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) tot[c] = z4;
+        for (int32_t q0 = cb; q0 < ce; q0 += 16) {      // two-level fixed-order sum
+          float4 blk[VPL];
+#pragma unroll
+          for (int c = 0; c < VPL; ++c) blk[c] = z4;
+          const int32_t q1 = min(q0 + 16, ce);
+          for (int32_t q = q0; q < q1; ++q) {
+            const float4* pr = reinterpret_cast<const float4*>(a.partials + (int64_t)q * a.W);
+#pragma unroll
+            for (int c = 0; c < VPL; ++c) {
+              const int cv = c * G + gl;
+              if (cv < nv) add_v(blk[c], __ldcg(pr + cv));
+            }
           }
-          add_v(tot, blk);
+#pragma unroll
+          for (int c = 0; c < VPL; ++c) add_v(tot[c], blk[c]);
         }
-        edge_write_row(a, r, tot, lane, nv);
-        if (lane == 0) a.counters[r] = 0;
+        float4* yr = reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy);
+#pragma unroll
+        for (int c = 0; c < VPL; ++c) {
+          const int cv = c * G + gl;
+          if (cv < nv) __stcs(yr + cv, scale_bias(s0, tot[c], a.bias, cv * 4));
+        }
+        if (gl == 0) a.counters[hub] = 0;             // self-reset for the next call
+      }
+    }
+    m0 = m1; m1 = m2; idx0 = idx1; s0 = s1;
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Strategy 2: edge stream over groups of 32 work items (16 < W/4 <= 32 float4
+// per launch).  A warp claims the next group of 32 consecutive schedule items
+// from a global queue (largest first: hub chunks lead the schedule), scans
+// their edge counts and walks the concatenated edge list in batches of 32
+// positions: lane l resolves position b·32+l to (item, column id) by a 5-step
+// binary search over the scan (shared memory), and the warp gathers D
+// neighbour rows at a time (lane c holds float4 column c of the row)
+// REGARDLESS of item boundaries, so short rows do not serialise on latency.
+// The next batch's column ids and the next group's descriptors (cp.async into
+// shared memory) are in flight while the current batch is gathered.  An item's
+// sum is flushed when the stream crosses into the next item: light rows are
+// written (s_v·Σ + bias), hub chunks store their partial for k_agg_hubs.
+// Hub rows of k_agg_stream: every chunk item stored its partial sum (unscaled) at
+// partials[item].  One CTA per hub row (grid-stride over the hub rows, which
+// lead node_ids: largest first): warp w sums chunk blocks w, w+8, ... (16
+// chunk partials per block, loaded together, added in chunk order) into
+// shared memory, then a fixed pairwise tree over the blocks gives the row sum
+// (deterministic: the tree shape depends only on the chunk count), written as
+// y[v] = s_v·Σ + bias.  Rows with more than 64 blocks run in rounds of 64.
+constexpr int kHubBlk = 16, kHubRound = 64;
+__global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_t* __restrict__ ids) {
+  __shared__ float4 blk[kHubRound][32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int32_t n_hub = a.sched[0];
+  const int32_t* cptr = a.sched + a.sched[2];
+  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+  const int nv = a.W >> 2;
+  const int c = lane < nv ? lane : nv - 1;
+  // big hubs (more than one block of chunks) lead the schedule: n_big = first h
+  // with cptr[h+1] - cptr[h] <= kHubBlk (chunk counts are non-increasing)
+  int32_t lo = 0, hi = n_hub;
+  while (lo < hi) {
+    const int32_t mid = (lo + hi) >> 1;
+    if (cptr[mid + 1] - cptr[mid] > kHubBlk) lo = mid + 1; else hi = mid;
+  }
+  const int32_t n_big = lo;
+  // (1) big hubs: one CTA each, blocks of 16 chunk partials per warp, fixed tree
+  for (int32_t h = blockIdx.x; h < n_big; h += gridDim.x) {
+    const int32_t cb = cptr[h], ce = cptr[h + 1], v = ids[h];
+    const int32_t nblk = (ce - cb + kHubBlk - 1) / kHubBlk;
+    float4 tot = z4;
+    for (int32_t r0 = 0; r0 < nblk; r0 += kHubRound) {
+      const int nr = min(kHubRound, nblk - r0);
+      for (int b = warp; b < nr; b += 8) {
+        const int32_t q0 = cb + (r0 + b) * kHubBlk, q1 = min(q0 + kHubBlk, ce);
+        float4 p[kHubBlk];
+#pragma unroll
+        for (int i = 0; i < kHubBlk; ++i)
+          p[i] = q0 + i < q1 ? __ldcg(reinterpret_cast<const float4*>(a.partials + (int64_t)(q0 + i) * a.W) + c) : z4;
+        float4 sb = p[0];
+#pragma unroll
+        for (int i = 1; i < kHubBlk; ++i) add_v(sb, p[i]);
+        blk[b][lane] = sb;
+      }
+      __syncthreads();
+      for (int st = 1; st < nr; st <<= 1) {            // fixed pairwise tree over the blocks
+        for (int e = threadIdx.x; e < nr * 32; e += 256) {
+          const int b = e >> 5, l = e & 31;
+          if ((b % (2 * st)) == 0 && b + st < nr) add_v(blk[b][l], blk[b + st][l]);
+        }
+        __syncthreads();
+      }
+      if (warp == 0) add_v(tot, blk[0][lane]);
+      __syncthreads();
+    }
+    if (warp == 0 && lane < nv) {
+      const float sv = a.srow ? a.srow[v] : 1.0f;
+      __stcs(reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy) + lane, scale_bias(sv, tot, a.bias, 4 * lane));
+    }
+  }
+  // (2) hubs of <= 16 chunks: one warp each, all chunk partials loaded together
+  const int64_t nw = (int64_t)gridDim.x * 8;
+  for (int64_t h = n_big + (int64_t)blockIdx.x * 8 + warp; h < n_hub; h += nw) {
+    const int32_t cb = cptr[h], ce = cptr[h + 1], v = ids[h];
+    float4 p[kHubBlk];
+#pragma unroll
+    for (int i = 0; i < kHubBlk; ++i)
+      p[i] = cb + i < ce ? __ldcg(reinterpret_cast<const float4*>(a.partials + (int64_t)(cb + i) * a.W) + c) : z4;
+    float4 sb = p[0];
+#pragma unroll
+    for (int i = 1; i < kHubBlk; ++i) add_v(sb, p[i]);
+    if (lane < nv) {
+      const float sv = a.srow ? a.srow[v] : 1.0f;
+      __stcs(reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy) + lane, scale_bias(sv, sb, a.bias, 4 * lane));
+    }
+  }
+}
+
+template <int D, int MINB, bool SCOL>
+__global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args a, uint32_t* __restrict__ queue) {
+  constexpr int NW = kAggThreads / 32;
+  __shared__ __align__(16) int4 s_items[NW][2][32];
+  __shared__ int32_t s_excl[NW][32], s_v[NW][32], s_beg[NW][32], s_hub[NW][32];
+  const unsigned FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t total = a.sched[3];
+  const int4* items = reinterpret_cast<const int4*>(a.sched + kSchedHdr);
+  const uint32_t ngroups = (uint32_t)((total + 31) / 32);
+  const int nv = a.W >> 2;
+  const bool lane_on = lane < nv;
+  const float4* xl = reinterpret_cast<const float4*>(a.x) + (lane_on ? lane : nv - 1);
+  const uint32_t ld4 = (uint32_t)(a.ldx >> 2);
+  int32_t* ex = s_excl[w];
+  auto fetch = [&](uint32_t g, int buf) {         // cp.async the 32 descriptors of group g
+    const int64_t it = (int64_t)g * 32 + lane;
+    const uint32_t dst = (uint32_t)__cvta_generic_to_shared(&s_items[w][buf][lane]);
+    const int4* src = items + (it < total ? it : 0);
+    const int bytes = (g < ngroups && it < total) ? 16 : 0;
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst), "l"(src), "r"(bytes) : "memory");
+    asm volatile("cp.async.commit_group;\n" ::: "memory");
+  };
+  uint32_t grp = 0;
+  if (lane == 0) grp = atomicAdd(queue, 1u);
+  grp = __shfl_sync(FULL, grp, 0);
+  int buf = 0;
+  fetch(grp, 0);
+  while (grp < ngroups) {
+    const uint32_t g_cur = grp;
+    if (lane == 0) grp = atomicAdd(queue, 1u);         // claim + prefetch the next group
+    grp = __shfl_sync(FULL, grp, 0);
+    fetch(grp, buf ^ 1);
+    asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+    __syncwarp();
+    int4 m = s_items[w][buf][lane];
+    buf ^= 1;
+    if ((int64_t)g_cur * 32 + lane >= total) m = make_int4(0, 0, 0, -2);
+    const int32_t nl = m.w > -2 ? m.z : 0;
+    int32_t incl = nl;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t t = __shfl_up_sync(FULL, incl, o);
+      if (lane >= o) incl += t;
+    }
+    const int32_t N = __shfl_sync(FULL, incl, 31);
+    ex[lane] = incl - nl;
+    s_v[w][lane] = m.x;
+    s_beg[w][lane] = m.y;
+    s_hub[w][lane] = m.w;
+    const float sl = (a.srow && m.w > -2) ? __ldg(a.srow + m.x) : 1.0f;
+    const unsigned zmask = __ballot_sync(FULL, m.w > -2 && nl == 0);
+    __syncwarp();
+    for (unsigned zm = zmask; zm; zm &= zm - 1) {      // rows without edges: y = bias
+      const int32_t vz = s_v[w][__ffs(zm) - 1];
+      if (lane_on)
+        __stcs(reinterpret_cast<float4*>(a.y + (int64_t)vz * a.ldy) + lane,
+               scale_bias(0.f, make_float4(0.f, 0.f, 0.f, 0.f), a.bias, 4 * lane));
+    }
+    auto resolve = [&](int32_t pos, int32_t& u, int32_t& k) {
+      int32_t lo = 0;
+#pragma unroll
+      for (int st = 16; st >= 1; st >>= 1)
+        if (lo + st <= 31 && ex[lo + st] <= pos) lo += st;
+      k = lo;
+      u = pos < N ? __ldcs(a.col + s_beg[w][lo] + (pos - ex[lo])) : 0;
+    };
+    auto flush = [&](int c, const float4& sum) {
+      const float sv = __shfl_sync(FULL, sl, c);
+      const int32_t hub = s_hub[w][c];
+      if (lane_on) {
+        if (hub < 0)
+          __stcs(reinterpret_cast<float4*>(a.y + (int64_t)s_v[w][c] * a.ldy) + lane, scale_bias(sv, sum, a.bias, 4 * lane));
+        else
+          reinterpret_cast<float4*>(a.partials + ((int64_t)g_cur * 32 + c) * a.W)[lane] = sum;
       }
     };
-    for (int64_t base = e0; base < e1; base += 32) {
-      // prefetch the next batch of the stream (this chunk or the next chunk of this warp)
-      const int nxt = which ^ 1;
-      if (base + 32 < e1) issue(c, base + 32, nxt);
-      else if (c + nwarps < nchunks) issue(c + nwarps, (c + nwarps) * kEdgeChunk, nxt);
-      mbar_wait_parity(which ? mb1 : mb0, which ? phase1 : phase0);
-      if (which) phase1 ^= 1u; else phase0 ^= 1u;
-      const unsigned char* bb = wbuf + (size_t)which * 32 * rowb;
-      const int n = which ? q_n1 : q_n0;
-      const int32_t my_row = which ? q_row1 : q_row0;
-      const float my_sc = which ? q_sc1 : q_sc0;
-      for (int j = 0; j < n; ++j) {
-        const int32_t rj = __shfl_sync(FULL, my_row, j);
-        const float sj = SCOL ? __shfl_sync(FULL, my_sc, j) : 1.0f;
-        if (rj != cur) {
-          flush(cur);
-          for (int32_t r = cur + 1; r < rj; ++r) edge_write_row(a, r, z4, lane, nv);
-          cur = rj;
-          acc0 = z4;
-          acc1 = z4;
+    int32_t u0, k0;
+    resolve(lane, u0, k0);
+    int cur = -1;
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int32_t b0 = 0; b0 < N; b0 += 32) {
+      const int32_t nb = min(32, N - b0);
+      // item boundaries of this batch: bit j = edge j starts a new item.  The
+      // first position past the stream end is a boundary to the dummy item -1,
+      // so a partial last step needs no per-edge bounds checks.
+      const int32_t kp = __shfl_up_sync(FULL, k0, 1);
+      const int32_t kc = lane < nb ? k0 : -1;
+      const uint32_t bm = __ballot_sync(FULL, lane <= nb && (lane == 0 ? kc != cur : (lane == nb || kc != kp)));
+      float sc = 1.0f;
+      if (SCOL && lane < nb) sc = __ldg(a.scol + u0);
+      const int32_t uc = u0;
+      if (b0 + 32 < N) resolve(b0 + 32 + lane, u0, k0);  // next batch in flight
+      for (int32_t j0 = 0; j0 < nb; j0 += D) {
+        float4 v[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) {
+          const uint32_t u = (uint32_t)__shfl_sync(FULL, uc, (j0 + d) & 31);
+          v[d] = __ldg(xl + (size_t)u * ld4);
         }
-        if (lane < nv) {
-          const float4 xv = reinterpret_cast<const float4*>(bb + (size_t)j * rowb)[lane];
-          if (((base + j) & 1) == 0) {
-            if (SCOL) fma_v(acc0, sj, xv); else add_v(acc0, xv);
+#pragma unroll
+        for (int d = 0; d < D; ++d) {
+          const float sj = SCOL ? __shfl_sync(FULL, sc, (j0 + d) & 31) : 1.0f;
+          if ((bm >> ((j0 + d) & 31)) & 1u) {
+            if (cur >= 0) flush(cur, acc);
+            cur = __shfl_sync(FULL, kc, (j0 + d) & 31);
+            if (SCOL) { acc = make_float4(0.f, 0.f, 0.f, 0.f); fma_v(acc, sj, v[d]); }
+            else acc = v[d];
           } else {
-            if (SCOL) fma_v(acc1, sj, xv); else add_v(acc1, xv);
+            if (SCOL) fma_v(acc, sj, v[d]);
+            else add_v(acc, v[d]);
           }
         }
       }
-      __syncwarp();     // every lane is done reading this buffer before it is refilled
-      which = nxt;
     }
-    flush(cur);
+    if (cur >= 0) flush(cur, acc);
+    __syncwarp();
   }
+  asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+}
+
+using ItemsFn = void (*)(const Agg2Args);
+template <int G, int VPL, bool SCOL>
+ItemsFn pick_items_vpl() {
+  return k_agg_items<G, VPL, (G >= 4 ? 4 : G), SCOL>;
+}
+template <int G, bool SCOL>
+ItemsFn pick_items_g(int vpl) {
+  switch (vpl) {
+    case 1: return pick_items_vpl<G, 1, SCOL>();
+    case 2: return pick_items_vpl<G, 2, SCOL>();
+    case 3: return pick_items_vpl<G, 3, SCOL>();
+    default: return pick_items_vpl<G, 4, SCOL>();
+  }
+}
+template <bool SCOL>
+ItemsFn pick_items(int g, int vpl) {
+  switch (g) {
+    case 1: return pick_items_g<1, SCOL>(vpl);
+    case 2: return pick_items_g<2, SCOL>(vpl);
+    case 4: return pick_items_g<4, SCOL>(vpl);
+    case 8: return pick_items_g<8, SCOL>(vpl);
+    case 16: return pick_items_g<16, SCOL>(vpl);
+    default: return pick_items_g<32, SCOL>(vpl);
+  }
+}
+
+using StreamFn = void (*)(const Agg2Args, uint32_t*);
+StreamFn pick_stream(int d, int minb, bool scol) {
+#define STG_STREAM(DD, MB) \
+  if (d == DD && minb == MB) return scol ? k_agg_stream<DD, MB, true> : k_agg_stream<DD, MB, false>;
+  STG_STREAM(4, 6) STG_STREAM(8, 4) STG_STREAM(16, 2) STG_STREAM(16, 3)
+#undef STG_STREAM
+  return scol ? k_agg_stream<16, 3, true> : k_agg_stream<16, 3, false>;
 }
 
 using KernelFn = void (*)(const AggArgs);
@@ -764,24 +675,35 @@ int max_blocks_for(KernelFn fn) {
 
 }  // namespace
 
-// Gather strategy switch (1 = cp.async shared-memory ring; 0 = register gathers).
-static int g_agg_async = 0;   // measured fastest on C5
-
-// Launch plan: vector width, group size, vectors per lane for W columns.
-struct AggPlan {
-  int vec, g, vpl, wmax;
+// Work decomposition (stg_aggregate_set_strategy) and strategy-2 tunables.
+static int g_strategy = 2;
+struct AggTune {
+  int d = 16;        // rows in flight per warp (stream kernel)
+  int minb = 3;      // min resident blocks per SM (register budget of the stream kernel)
+  int wmin = 32;     // stream kernel for wmin < W_launch <= 128
 };
-static AggPlan plan_for(int32_t W, bool vec4) {
-  AggPlan p;
-  p.vec = vec4 ? 4 : 1;
-  int nv = W / p.vec;
-  if (nv > 128) nv = 128;                 // column-split into 128-vector launches
-  int g = 1;
-  while (g < 32 && g * 4 < nv) g <<= 1;
-  p.g = g;
-  p.vpl = (nv + g - 1) / g;
-  p.wmax = 128 * p.vec;
-  return p;
+static AggTune g_tune;
+
+static int occupancy_grid(const void* fn) {
+  static std::mutex mu;
+  static std::map<const void*, int> cache;
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = cache.find(fn);
+  if (it != cache.end()) return it->second;
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kAggThreads, 0) != cudaSuccess || per_sm < 1) {
+    cudaGetLastError();
+    per_sm = 1;
+  }
+  return cache[fn] = per_sm * num_sms();
+}
+
+// lane-group size G and float4 per lane for nv float4 columns (vpl_max float4 per lane)
+static void lane_groups(int nv, int vpl_max, int* g, int* vpl) {
+  int gg = 1;
+  while (gg < 32 && gg * vpl_max < nv) gg <<= 1;
+  *g = gg;
+  *vpl = (nv + gg - 1) / gg;
 }
 
 stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
@@ -807,12 +729,12 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   a.bias = bias;
   const bool vec4 = (W % 4 == 0) && (ldin % 4 == 0) && (ldout % 4 == 0) &&
                     ((uintptr_t)in % 16 == 0) && ((uintptr_t)out % 16 == 0);
-  const AggPlan p0 = plan_for(W, vec4);
-  const int64_t chunks_bound = a.sched ? 2 * (gv->num_edges / kHubChunk) + 2 : 0;
+  // column split: launches of <= 512 columns (strategies 0/1) or <= 128 (strategy 2)
+  const int32_t cmax = vec4 ? 512 : 128;
+  const int64_t chunks_bound = a.sched ? (gv->num_edges / kHubChunk) + 2 : 0;
   AggWs* ws = static_cast<AggWs*>(gv->workspace);
   if (a.sched) {
-    const int32_t wl = W < p0.wmax ? W : p0.wmax;
-    STG_TRY(ws->partials.alloc((size_t)chunks_bound * wl + 4, s));   // >= the async path's 128-column chunks
+    STG_TRY(ws->partials.alloc((size_t)chunks_bound * std::min(W, cmax) + 4, s));
     const int64_t ncnt = sched_cap(gv->num_edges) + 1;
     if (ws->counters_n < ncnt) {
       STG_TRY(ws->counters.alloc(ncnt, s));
@@ -824,99 +746,63 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   }
   const int64_t items_bound = (int64_t)R + chunks_bound + 1;
   ProfScope prof(backward ? PH_AGG_BWD : PH_AGG_FWD, s);
-  // edge-parallel path: float4 rows, 16 <= float4-per-row chunks (W in [64, 128] per launch), COO rows known
-  const int32_t* rowarr = backward ? gv->out_row : gv->in_row;
-  if (vec4 && g_agg_async == 2 && W >= 64 && rowarr && gv->num_edges > 0 && gv->workspace) {
-    const int64_t E = gv->num_edges;
-    const int64_t nchunks = (E + kEdgeChunk - 1) / kEdgeChunk;
-    STG_TRY(ws->epartials.alloc((size_t)2 * nchunks * 128 + 4, s));
-    if (ws->ecounters_n < R) {
-      STG_TRY(ws->ecounters.alloc(R, s));
-      STG_CUDA(cudaMemsetAsync(ws->ecounters.p, 0, sizeof(int32_t) * R, s));
-      ws->ecounters_n = R;
+
+  // strategy 2: edge stream, in near-equal column chunks of <= 128 columns
+  const int nsplit = (int)ceil_div(W, 128);
+  const int32_t wsplit = (int32_t)(ceil_div(ceil_div(W, 4), nsplit) * 4);
+  if (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128) {
+    STG_TRY(ws->queue.alloc(nsplit, s));
+    STG_CUDA(cudaMemsetAsync(ws->queue.p, 0, sizeof(uint32_t) * nsplit, s));
+    const StreamFn fn = pick_stream(g_tune.d, g_tune.minb, scol != nullptr);
+    const int64_t blocks = std::min<int64_t>(occupancy_grid((const void*)fn), ceil_div(items_bound, 32 * 8) + 1);
+    const int32_t* hids = backward ? gv->out_ids : gv->in_ids;
+    for (int k = 0; k < nsplit; ++k) {
+      const int32_t c0 = k * wsplit, wl = std::min(wsplit, W - c0);
+      Agg2Args b{};
+      b.sched = a.sched; b.col = a.col; b.srow = srow; b.scol = scol;
+      b.partials = a.partials; b.counters = a.counters;
+      b.W = wl; b.x = in + c0; b.ldx = ldin; b.y = out + c0; b.ldy = ldout;
+      b.bias = bias ? bias + c0 : nullptr;
+      fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(b, ws->queue.p + k);
+      k_agg_hubs<<<(unsigned)(4 * num_sms()), 256, 0, s>>>(b, hids);
+      count_launch(2);
     }
-    EdgeArgs ea{};
-    ea.R = R; ea.E = E; ea.rowptr = a.rowptr; ea.col = a.col; ea.row = rowarr;
-    ea.srow = srow; ea.scol = scol;
-    ea.partials = ws->epartials.p; ea.counters = ws->ecounters.p;
-    for (int32_t c0 = 0; c0 < W; c0 += 128) {
-      const int32_t wl = (W - c0) < 128 ? (W - c0) : 128;
-      ea.W = wl; ea.x = in + c0; ea.ldx = ldin; ea.y = out + c0; ea.ldy = ldout;
-      ea.bias = bias ? bias + c0 : nullptr;
-      auto fn = scol ? k_agg_edges_tma<true> : k_agg_edges_tma<false>;
-      const size_t per_warp = (size_t)2 * 32 * wl * 4;
-      int wpb = (int)std::min<size_t>(kAggThreads / 32, (size_t)(200 * 1024) / per_warp);
-      if (wpb < 1) wpb = 1;
-      const size_t smem = per_warp * wpb;
-      {
-        static std::mutex mu;
-        std::lock_guard<std::mutex> lk(mu);
-        static size_t attr[2] = {0, 0};
-        if (attr[scol ? 1 : 0] < smem) {
-          STG_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-          attr[scol ? 1 : 0] = smem;
-        }
-      }
-      int per_sm = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kAggThreads, smem) != cudaSuccess || per_sm < 1) {
-        cudaGetLastError();
-        per_sm = 1;
-      }
-      int64_t blocks = ceil_div(nchunks, wpb);
-      const int64_t mb = (int64_t)per_sm * num_sms();
-      if (blocks > mb) blocks = mb;
-      fn<<<(unsigned)blocks, kAggThreads, smem, s>>>(ea, wpb);
+    return check_launch("aggregate_stream");
+  }
+  // strategy 1: pipelined items
+  if (vec4 && g_strategy >= 1 && a.sched) {
+    for (int32_t c0 = 0; c0 < W; c0 += cmax) {
+      const int32_t wl = std::min(cmax, W - c0);
+      int g, vpl;
+      lane_groups(wl / 4, 2, &g, &vpl);
+      Agg2Args b{};
+      b.sched = a.sched; b.col = a.col; b.srow = srow; b.scol = scol;
+      b.partials = a.partials; b.counters = a.counters;
+      b.W = wl; b.x = in + c0; b.ldx = ldin; b.y = out + c0; b.ldy = ldout;
+      b.bias = bias ? bias + c0 : nullptr;
+      const ItemsFn fn = scol ? pick_items<true>(g, vpl) : pick_items<false>(g, vpl);
+      const int64_t blocks = std::max<int64_t>(
+          1, std::min<int64_t>(occupancy_grid((const void*)fn), ceil_div(items_bound, (kAggThreads / 32) * (32 / g))));
+      fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(b);
       count_launch();
     }
-    return check_launch("aggregate_edges");
+    return check_launch("aggregate_items");
   }
-  const bool use_async = vec4 && g_agg_async == 1;
-  const int wmax = use_async ? 128 : p0.wmax;
-  for (int32_t c0 = 0; c0 < W; c0 += wmax) {
-    const int32_t wl = (W - c0) < wmax ? (W - c0) : wmax;
-    const AggPlan p = plan_for(wl, vec4);
+  // strategy 0: row items with register gathers (any width / alignment, any view)
+  for (int32_t c0 = 0; c0 < W; c0 += cmax) {
+    const int32_t wl = std::min(cmax, W - c0);
+    int g, vpl;
+    lane_groups(vec4 ? wl / 4 : wl, 4, &g, &vpl);
     a.W = wl;
     a.x = in + c0;
     a.ldx = ldin;
     a.y = out + c0;
     a.ldy = ldout;
     a.bias = bias ? bias + c0 : nullptr;
-    const int rows_per_warp = 32 / p.g;
-    const int U = p.vpl <= 2 ? 4 : 2;
-    if (use_async && p.g >= U) {
-      AsyncFn fn = scol ? pick_async_g<true>(p.g, p.vpl) : pick_async_g<false>(p.g, p.vpl);
-      const size_t per_warp = (size_t)2 * 32 * wl * 4 + 2 * 32 * 4;
-      int wpb = (int)std::min<size_t>(8, (size_t)(200 * 1024) / per_warp);
-      if (wpb < 1) wpb = 1;
-      const size_t smem = per_warp * wpb;
-      static std::mutex mu;
-      {
-        std::lock_guard<std::mutex> lk(mu);
-        static std::map<AsyncFn, size_t> attr;
-        if (attr[fn] < smem) {
-          STG_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-          attr[fn] = smem;
-        }
-      }
-      int per_sm = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kAggThreads, smem) != cudaSuccess || per_sm < 1) {
-        cudaGetLastError();
-        per_sm = 1;
-      }
-      int64_t blocks = ceil_div(items_bound, (int64_t)wpb * rows_per_warp);
-      const int64_t mb = (int64_t)per_sm * num_sms();
-      if (blocks > mb) blocks = mb;
-      if (blocks < 1) blocks = 1;
-      fn<<<(unsigned)blocks, kAggThreads, smem, s>>>(a, wpb);
-    } else {
-      KernelFn fn = pick(p.vec, p.g, p.vpl, scol != nullptr);
-      const int rows_per_block = (kAggThreads / 32) * rows_per_warp;
-      int64_t blocks = ceil_div(items_bound, rows_per_block);
-      const int64_t mb = max_blocks_for(fn);
-      if (blocks > mb) blocks = mb;
-      if (blocks < 1) blocks = 1;
-      fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(a);
-    }
+    const KernelFn fn = pick(vec4 ? 4 : 1, g, vpl, scol != nullptr);
+    const int64_t blocks = std::max<int64_t>(
+        1, std::min<int64_t>(max_blocks_for(fn), ceil_div(items_bound, (kAggThreads / 32) * (32 / g))));
+    fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(a);
     count_launch();
   }
   return check_launch("aggregate");
@@ -942,8 +828,28 @@ stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* 
 
 stg_status stg_aggregate_set_strategy(int32_t strategy) {
   if (strategy < 0 || strategy > 2) return stg::fail(STG_ERR_INVALID_ARG, "stg_aggregate_set_strategy: %d", strategy);
-  stg::g_agg_async = strategy;
+  stg::g_strategy = strategy;
   return STG_OK;
+}
+
+stg_status stg_aggregate_set_param(int32_t key, int64_t value) {
+  switch (key) {
+    case 0:
+      if (value != 4 && value != 8 && value != 16) break;
+      stg::g_tune.d = (int)value;
+      return STG_OK;
+    case 1:
+      if (value < 2 || value > 6) break;
+      stg::g_tune.minb = (int)value;
+      return STG_OK;
+    case 2:
+      if (value != 32 && value != 64) break;
+      stg::g_tune.wmin = (int)value;
+      return STG_OK;
+    default:
+      break;
+  }
+  return stg::fail(STG_ERR_INVALID_ARG, "stg_aggregate_set_param: key %d value %lld", key, (long long)value);
 }
 
 stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t W, const float* in, int64_t ldin,

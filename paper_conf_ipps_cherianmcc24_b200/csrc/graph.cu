@@ -23,7 +23,7 @@ stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl) {
   while ((int64_t(1) << nb) < (int64_t)V) ++nb;
   edge_ids = eids;
   dgl_both = dgl;
-  const int64_t sc = 2 + sched_cap(cap) + 1;
+  const int64_t sc = sched_size(V, cap);
   STG_TRY(in_rowptr.alloc(V + 1)); STG_TRY(out_rowptr.alloc(V + 1));
   STG_TRY(in_col.alloc(cap)); STG_TRY(in_row.alloc(cap));
   STG_TRY(out_col.alloc(cap)); STG_TRY(out_row.alloc(cap));
@@ -119,6 +119,36 @@ __global__ void k_sched_count(const int32_t* __restrict__ ids, const int32_t* __
   }
 }
 
+// Work items in node_ids order (layout in graph.cuh): hub chunks, then light rows.
+__global__ void k_items(const int32_t* __restrict__ ids, const int32_t* __restrict__ rowptr, int32_t V,
+                        int64_t cap_items, int64_t coff, int32_t* __restrict__ sched) {
+  const int32_t n_hub = sched[0], n_chunks = sched[1];
+  const int32_t* cptr = sched + coff;
+  const int64_t total = (int64_t)n_chunks + V - n_hub;
+  int4* items = reinterpret_cast<int4*>(sched + kSchedHdr);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total && i < cap_items;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    if (i < n_chunks) {
+      int32_t lo = 0, hi = n_hub;      // largest h with cptr[h] <= i
+      while (lo < hi) {
+        int32_t mid = (lo + hi + 1) >> 1;
+        if (cptr[mid] <= i) lo = mid; else hi = mid - 1;
+      }
+      const int32_t v = ids[lo], rb = rowptr[v], re = rowptr[v + 1];
+      const int32_t beg = rb + (int32_t)(i - cptr[lo]) * kHubChunk;
+      items[i] = make_int4(v, beg, min(kHubChunk, re - beg), lo);
+    } else {
+      const int32_t v = ids[n_hub + (i - n_chunks)];
+      const int32_t rb = rowptr[v];
+      items[i] = make_int4(v, rb, rowptr[v + 1] - rb, -1);
+    }
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    sched[2] = (int32_t)coff;
+    sched[3] = (int32_t)total;
+  }
+}
+
 struct ChunkIn {
   const int32_t* ids;
   const int32_t* deg;
@@ -188,11 +218,16 @@ stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s) {
     if (vv != ids) {
       STG_CUDA(cudaMemcpyAsync(ids, vv, sizeof(int32_t) * V, cudaMemcpyDeviceToDevice, s));
     }
+    const int32_t* rowptr = dir == 0 ? g.in_rowptr.p : g.out_rowptr.p;
+    const int64_t coff = sched_cptr_off(V, g.cap);
     k_sched_count<<<grid_for(m + 1, 256), 256, 0, s>>>(ids, deg, V, m, sched);
     count_launch();
-    // chunk_ptr (exclusive) in sched[2..2+m], total chunks in sched[2+m] and sched[1]
-    STG_TRY(scan(ChunkIn{ids, deg}, StoreExcl32{sched + 2}, m, ws.scan, s, nullptr, sched + 2 + m));
-    STG_CUDA(cudaMemcpyAsync(sched + 1, sched + 2 + m, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
+    // chunk_ptr (exclusive) in cptr[0..m], total chunks in cptr[m] and sched[1]
+    STG_TRY(scan(ChunkIn{ids, deg}, StoreExcl32{sched + coff}, m, ws.scan, s, nullptr, sched + coff + m));
+    STG_CUDA(cudaMemcpyAsync(sched + 1, sched + coff + m, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
+    const int64_t icap = sched_items_cap(V, g.cap);
+    k_items<<<grid_for(icap, 256), 256, 0, s>>>(ids, rowptr, V, icap, coff, sched);
+    count_launch();
   }
   return check_launch("build_ids_and_sched");
 }

@@ -2,17 +2,35 @@
 // and the builders shared by static graphs and DTDG snapshots.
 #pragma once
 
+#include <algorithm>
+
 #include "common.cuh"
 
 namespace stg {
 
 // Rows with more than kHubChunk in-edges are split into chunks of kHubChunk
 // edges (degree-bucketed schedule); each light row / hub chunk is
-// one work item of the aggregation kernel.  128 keeps every fp32 accumulator
-// chain <= 64 terms.
-constexpr int32_t kHubChunk = 128;
+// one work item of the aggregation kernel.  64 keeps every fp32 accumulator
+// chain <= 64 terms with a single accumulator.
+constexpr int32_t kHubChunk = 64;
 
+// upper bound on the number of hub rows (deg > kHubChunk) of an E-edge graph
 inline int64_t sched_cap(int64_t E) { return E / (kHubChunk + 1) + 2; }
+
+// Degree-bucketed schedule of one CSR direction (int32 array `sched`):
+//   sched[0] = n_hub    rows with deg > kHubChunk (the prefix ids[0, n_hub))
+//   sched[1] = n_chunks total hub chunks
+//   sched[2] = cptr_off offset (in int32) of cptr[0..n_hub] (exclusive chunk prefix)
+//   sched[3] = n_items  = n_chunks + V - n_hub
+//   sched[4 ..]         = items, int4 {v, beg, n, hub} in node_ids order: hub
+//                         chunks first (hub = index into ids / cptr), then the
+//                         light rows (hub = -1).  n <= kHubChunk.
+constexpr int64_t kSchedHdr = 4;
+inline int64_t sched_items_cap(int64_t V, int64_t E) { return V + E / kHubChunk + 2; }
+inline int64_t sched_cptr_off(int64_t V, int64_t E) { return kSchedHdr + 4 * sched_items_cap(V, E); }
+inline int64_t sched_size(int64_t V, int64_t E) {
+  return sched_cptr_off(V, E) + std::min<int64_t>(V, sched_cap(E)) + 2;
+}
 
 // Aggregation scratch owned by a graph / dtdg object: hub-chunk partial sums
 // and per-hub-row completion counters (self-resetting, zero between calls).
@@ -20,9 +38,7 @@ struct AggWs {
   DArray<float> partials;
   DArray<int32_t> counters;
   int64_t counters_n = 0;
-  DArray<float> epartials;       // edge-parallel kernel: per-chunk partials
-  DArray<int32_t> ecounters;     // edge-parallel kernel: per-row tickets (self-resetting)
-  int64_t ecounters_n = 0;
+  DArray<uint32_t> queue;        // edge-stream work-queue heads, one per column chunk (reset per launch)
 };
 
 struct Snapshot {
@@ -32,7 +48,7 @@ struct Snapshot {
   bool edge_ids = false, dgl_both = false;
   DArray<int32_t> in_rowptr, in_col, in_row, in_deg, in_ids;
   DArray<int32_t> out_rowptr, out_col, out_row, out_deg, out_ids, out_eid;
-  DArray<int32_t> in_sched, out_sched;  // [2 + sched_cap(cap) + 1]
+  DArray<int32_t> in_sched, out_sched;  // [sched_size(V, cap)], layout above
   DArray<float> norm_src, norm_dst;
 
   stg_status alloc(int32_t V_, int64_t cap_, bool eids, bool dgl);

@@ -14,10 +14,10 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C5")
 ap.add_argument("--S", type=int, default=4)
 ap.add_argument("--seqs", type=int, default=1)
-ap.add_argument("--async-gather", type=int, default=-1)
+ap.add_argument("--strategy", type=int, default=-1)
 a = ap.parse_args()
-if a.async_gather >= 0:
-    stg.stg_aggregate_set_strategy(bool(a.async_gather))
+if a.strategy >= 0:
+    stg.stg_aggregate_set_strategy(a.strategy)
 cfg = gen.CONFIGS[a.config]
 d = gen.dtdg(cfg)
 V, F, H, S = cfg.V, cfg.F, cfg.H, a.S
