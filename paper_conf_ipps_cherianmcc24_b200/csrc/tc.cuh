@@ -68,6 +68,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t* mbar, uint32_t phase) {
       : "memory");
 }
 
+// plain arrive (count 1) on an mbarrier from a thread
+__device__ __forceinline__ void mbar_arrive(uint64_t* mbar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(mbar)) : "memory");
+}
+
 __device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 // make generic-proxy st.shared visible to the tensor core (async proxy)
@@ -152,6 +157,105 @@ __device__ __forceinline__ void stage_rows(unsigned char* hi, unsigned char* lo,
       if (it < total && j < nj) st_split4(hi, lo, r, (k0 >> 2) + j, Ktile, v[i]);
     }
   }
+}
+
+// As stage_rows, executed by a group of nthr threads (tid = index in the
+// group, a multiple of 32 threads) instead of the whole block: producer warps
+// of a warp-specialised kernel.  All loads of the thread are issued before the
+// first store (up to 16 float4 in flight per thread).
+template <int MAXB = 16>
+__device__ __forceinline__ void stage_rows_grp(unsigned char* hi, unsigned char* lo, const float* __restrict__ src,
+                                               int64_t ld, int nvalid, int rows, int F, int f0, int k0, int Ktile,
+                                               int tid, int nthr) {
+  const int lane = tid & 31, warp = tid >> 5, nw = nthr >> 5;
+  const int nj = F / 4, njb = (nj + 3) / 4, nrb = rows / 8, total = nrb * njb;
+  for (int base = warp; base < total; base += MAXB * nw) {
+    float4 v[MAXB];
+#pragma unroll
+    for (int i = 0; i < MAXB; ++i) {
+      const int it = base + i * nw;
+      const int r = (it % nrb) * 8 + (lane & 7);
+      const int j = (it / nrb) * 4 + (lane >> 3);
+      v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (it < total && j < nj && r < nvalid)
+        v[i] = __ldg(reinterpret_cast<const float4*>(src + (int64_t)r * ld + f0 + 4 * j));
+    }
+#pragma unroll
+    for (int i = 0; i < MAXB; ++i) {
+      const int it = base + i * nw;
+      const int r = (it % nrb) * 8 + (lane & 7);
+      const int j = (it / nrb) * 4 + (lane >> 3);
+      if (it < total && j < nj) st_split4(hi, lo, r, (k0 >> 2) + j, Ktile, v[i]);
+    }
+  }
+}
+
+// Two-phase form of stage_rows_grp for register prefetch: grp_load issues the
+// thread's (at most MAXB) float4 loads of a tile, grp_store splits and stores
+// them; a producer loads tile i+1 while it waits for a free ring slot.
+template <int MAXB>
+__device__ __forceinline__ void grp_load(float4 (&v)[MAXB], const float* __restrict__ src, int64_t ld, int nvalid,
+                                         int rows, int F, int f0, int tid, int nthr) {
+  const int lane = tid & 31, warp = tid >> 5, nw = nthr >> 5;
+  const int nj = F / 4, njb = (nj + 3) / 4, nrb = rows / 8, total = nrb * njb;
+#pragma unroll
+  for (int i = 0; i < MAXB; ++i) {
+    const int it = warp + i * nw;
+    const int r = (it % nrb) * 8 + (lane & 7);
+    const int j = (it / nrb) * 4 + (lane >> 3);
+    v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (it < total && j < nj && r < nvalid) v[i] = __ldg(reinterpret_cast<const float4*>(src + (int64_t)r * ld + f0 + 4 * j));
+  }
+}
+template <int MAXB>
+__device__ __forceinline__ void grp_store(const float4 (&v)[MAXB], unsigned char* hi, unsigned char* lo, int rows,
+                                          int F, int k0, int Ktile, int tid, int nthr) {
+  const int lane = tid & 31, warp = tid >> 5, nw = nthr >> 5;
+  const int nj = F / 4, njb = (nj + 3) / 4, nrb = rows / 8, total = nrb * njb;
+#pragma unroll
+  for (int i = 0; i < MAXB; ++i) {
+    const int it = warp + i * nw;
+    const int r = (it % nrb) * 8 + (lane & 7);
+    const int j = (it / nrb) * 4 + (lane >> 3);
+    if (it < total && j < nj) st_split4(hi, lo, r, (k0 >> 2) + j, Ktile, v[i]);
+  }
+}
+
+// Coalesced row-tile store for a thread-per-row epilogue: the 32 lanes of a
+// warp each hold one row (NC float4 columns) in registers.  The rows go to a
+// per-warp shared-memory stage with an odd row pitch of kStagePitch<NC> float4
+// (so the row-per-lane writes and the chunk-parallel reads are free of bank
+// conflicts), then the warp writes them out chunk-parallel: lane l stores chunk
+// q = it·32 + l of the 32-row block (row q / NC, column q % NC), i.e. lanes
+// write consecutive 16-byte chunks of a row instead of 32 scattered rows per
+// instruction.  dst row r = dst + (row0 + r)·ld (16-byte aligned); rows >=
+// nvalid are not written.  stage: 32 · kStagePitch<NC> float4 of this warp.
+template <int NC>
+constexpr int kStagePitch = NC + 1 + (NC & 1);
+
+// Write the warp's 32 staged rows out chunk-parallel (after the lanes filled
+// their rows of the stage; includes the __syncwarp on both sides).
+template <int NC>
+__device__ __forceinline__ void flush_stage_rows(const float4* stage, float* dst, int64_t ld, int row0, int nvalid) {
+  constexpr int P = kStagePitch<NC>;
+  const int lane = threadIdx.x & 31;
+  __syncwarp();
+#pragma unroll 4
+  for (int it = 0; it < NC; ++it) {
+    const int q = it * 32 + lane;
+    const int r = q / NC, c = q % NC;
+    if (r < nvalid) reinterpret_cast<float4*>(dst + (int64_t)(row0 + r) * ld)[c] = stage[r * P + c];
+  }
+  __syncwarp();
+}
+
+template <int NC>
+__device__ __forceinline__ void store_rows_coalesced(float4* stage, const float4 (&v)[NC], float* dst, int64_t ld,
+                                                     int row0, int nvalid) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int c = 0; c < NC; ++c) stage[lane * kStagePitch<NC> + c] = v[c];
+  flush_stage_rows<NC>(stage, dst, ld, row0, nvalid);
 }
 
 // TRANSPOSED operand tiles (K = rows) use a padded K-major layout: element

@@ -16,6 +16,7 @@
 //
 // The equations are those of SURVEY §8(c) (readings C13-C15).
 #include <algorithm>
+#include <cstdlib>
 #include <map>
 #include <mutex>
 
@@ -147,6 +148,120 @@ __global__ void __launch_bounds__(kTcThreads) k_tc_xw(int V, int F, int Kp, cons
   tc::fence_before();
   __syncthreads();
   if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
+}
+
+// ------------------------------------------------------------------ X·W, pipelined
+// Warp-specialised persistent kernel (13 warps):
+//   warps 4-11 producers, two groups of 4 warps taking alternate tiles: each
+//              group stages its tile (3xTF32 hi/lo split) into its own slot of
+//              a 2-slot shared-memory ring and arrives full[slot]; the group's
+//              next tile is loaded into registers before it waits for the
+//              slot to free up, so two tiles of loads are in flight per SM;
+//   warp  12   one lane issues the tcgen05 MMAs of a tile into one of two TMEM
+//              accumulators and commits empty[slot] and tfull[acc];
+//   warps 0-3  epilogue: thread = tile row = TMEM lane, tcgen05.ld, release
+//              the accumulator (tempty[acc]), scale by n_src, and store P'
+//              through a per-warp shared stage so that lanes write consecutive
+//              16-byte chunks (a thread-per-row store pattern is capped at
+//              ~2.5 TB/s, scripts/store_bench.py).
+constexpr int kXwThreads = 416;
+constexpr int kXwStages = 2;
+
+template <int N>
+__global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int Kp, const float* __restrict__ X,
+                                                              const float* __restrict__ W,
+                                                              const float* __restrict__ rs, float* __restrict__ P,
+                                                              int dbg) {
+  extern __shared__ __align__(128) unsigned char sm[];
+  __shared__ uint64_t full[kXwStages], empty[kXwStages], tfull[2], tempty[2];
+  __shared__ uint32_t tslot;
+  constexpr uint32_t NC = N <= 32 ? 32 : (N <= 64 ? 64 : (N <= 128 ? 128 : 256));
+  constexpr int NQ = N / 4;
+  const int ABYTES = 128 * Kp * 4;
+  unsigned char* bhi = sm;
+  unsigned char* blo = bhi + N * Kp * 4;
+  unsigned char* abase = blo + N * Kp * 4;
+  auto ahi = [&](int st) { return abase + (size_t)st * 2 * ABYTES; };
+  auto alo = [&](int st) { return abase + (size_t)st * 2 * ABYTES + ABYTES; };
+  float4* ostage = reinterpret_cast<float4*>(abase + (size_t)kXwStages * 2 * ABYTES);   // 4 warps x 32 rows
+  const int warp = threadIdx.x >> 5;
+  tc::stage_weight_T(bhi, blo, W, F, N, Kp, N);
+  for (int i = threadIdx.x; i < kXwStages * 2 * 128 * Kp; i += blockDim.x)   // zero the K padding once
+    reinterpret_cast<float*>(abase)[i] = 0.f;
+  if (warp == 12) tc::tmem_alloc(&tslot, 2 * NC);
+  if (threadIdx.x == 0) {
+    for (int st = 0; st < kXwStages; ++st) { tc::mbar_init(&full[st], 128); tc::mbar_init(&empty[st], 1); }
+    for (int b = 0; b < 2; ++b) { tc::mbar_init(&tfull[b], 1); tc::mbar_init(&tempty[b], 128); }
+    tc::fence_mbar_init();
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  const int ntiles = (V + 127) / 128;
+  if (warp >= 4 && warp < 12) {                      // ---- producers (group = slot)
+    // a 128 x F (F <= 64) tile = at most 16 float4 per producer thread
+    const int grp = (warp - 4) >> 2, tid = threadIdx.x - 128 - 128 * grp;
+    float4 v[16];
+    int tile = blockIdx.x + grp * gridDim.x;
+    if (tile < ntiles && !(dbg & 4)) tc::grp_load<16>(v, X + (int64_t)tile * 128 * F, F, V - tile * 128, 128, F, 0, tid, 128);
+    for (int k = 0; tile < ntiles; tile += 2 * gridDim.x, ++k) {
+      if (k > 0) tc::mbar_wait(&empty[grp], (k - 1) & 1);
+      if (!(dbg & 8)) tc::grp_store<16>(v, ahi(grp), alo(grp), 128, F, 0, Kp, tid, 128);
+      tc::fence_proxy_async();
+      tc::mbar_arrive(&full[grp]);
+      const int nt = tile + 2 * gridDim.x;
+      if (nt < ntiles && !(dbg & 4)) tc::grp_load<16>(v, X + (int64_t)nt * 128 * F, F, V - nt * 128, 128, F, 0, tid, 128);
+    }
+  } else if (warp == 12) {                           // ---- MMA issuer
+    if ((threadIdx.x & 31) == 0) {
+      const uint32_t idesc = tc::idesc_tf32(128, N, 0, 0);
+      int i = 0;
+      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+        const int st = i & 1, k = i >> 1;            // tile i lives in slot i % 2, accumulator i % 2
+        tc::mbar_wait(&full[st], k & 1);
+        if (k > 0) tc::mbar_wait(&tempty[st], (k - 1) & 1);
+        tc::fence_after();
+        if (!(dbg & 2))
+          mma_seg(tm + st * NC, tc::smem_u32(ahi(st)), tc::smem_u32(alo(st)), Kp, 0, tc::smem_u32(bhi),
+                  tc::smem_u32(blo), Kp, 0, Kp, idesc, true);
+        tc::commit(&empty[st]);
+        tc::commit(&tfull[st]);
+      }
+    }
+  } else if (warp < 4) {                             // ---- epilogue
+    float4* stage = ostage + warp * 32 * tc::kStagePitch<NQ>;
+    int i = 0;
+    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+      const int b = i & 1, kb = i >> 1;
+      const int row = tile * 128 + threadIdx.x;
+      const float sc = (rs && row < V) ? __ldg(rs + row) : 1.0f;
+      tc::mbar_wait(&tfull[b], kb & 1);
+      tc::fence_after();
+      // TMEM -> registers in 16-column pieces -> scaled row in this warp's stage
+      const int lane = threadIdx.x & 31;
+#pragma unroll
+      for (int c0 = 0; c0 < N; c0 += 16) {
+        float v[16];
+        tmem_row_load<16>(tm + b * NC, c0, v);
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          stage[lane * tc::kStagePitch<NQ> + c0 / 4 + q] =
+              make_float4(sc * v[4 * q], sc * v[4 * q + 1], sc * v[4 * q + 2], sc * v[4 * q + 3]);
+      }
+      tc::fence_before();
+      tc::mbar_arrive(&tempty[b]);
+      if (!(dbg & 1)) {
+        const int wr0 = tile * 128 + warp * 32;
+        tc::flush_stage_rows<NQ>(stage, P, N, wr0, V - wr0);
+      } else {
+        __syncwarp();
+      }
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 12) tc::tmem_free(tm, 2 * NC);
 }
 
 // ------------------------------------------------------------------ GRU shared pieces
@@ -653,16 +768,31 @@ bool tc_supported(int F, int H) { return (H == 16 || H == 32) && F % 4 == 0 && F
 
 stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s) {
   const int N = 3 * H, Kp = (F + 7) / 8 * 8;
-  const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)2 * 128 * Kp * 4;
   const int ntiles = (V + 127) / 128;
-  if (H == 32) {
-    STG_TRY(prep(k_tc_xw<96>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_xw<96>, smem));
-    k_tc_xw<96><<<nb, kTcThreads, smem, s>>>(V, F, Kp, X, W, rs, P);
-  } else {
-    STG_TRY(prep(k_tc_xw<48>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_xw<48>, smem));
-    k_tc_xw<48><<<nb, kTcThreads, smem, s>>>(V, F, Kp, X, W, rs, P);
+  if (Kp <= 64) {                     // pipelined kernel (2-stage ring of 128 x Kp tiles + output stage)
+    const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)kXwStages * 2 * 128 * Kp * 4 +
+                        (size_t)128 * (N / 4 + 1 + ((N / 4) & 1)) * 16;
+    const int nb = std::min(ntiles, num_sms());
+    const char* dv = getenv("STG_XW_DEBUG");       // timing experiments only: skip parts of the pipeline
+    const int dbg = dv ? atoi(dv) : 0;
+    if (H == 32) {
+      STG_TRY(prep(k_tc_xw_pipe<96>, smem));
+      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg);
+    } else {
+      STG_TRY(prep(k_tc_xw_pipe<48>, smem));
+      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg);
+    }
+  } else {                            // 64 < F <= 128: one tile per CTA at a time
+    const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)2 * 128 * Kp * 4;
+    if (H == 32) {
+      STG_TRY(prep(k_tc_xw<96>, smem));
+      const int nb = std::min(ntiles, occupancy_blocks(k_tc_xw<96>, smem));
+      k_tc_xw<96><<<nb, kTcThreads, smem, s>>>(V, F, Kp, X, W, rs, P);
+    } else {
+      STG_TRY(prep(k_tc_xw<48>, smem));
+      const int nb = std::min(ntiles, occupancy_blocks(k_tc_xw<48>, smem));
+      k_tc_xw<48><<<nb, kTcThreads, smem, s>>>(V, F, Kp, X, W, rs, P);
+    }
   }
   count_launch();
   return check_launch("tc_xw");

@@ -53,12 +53,20 @@ def _graph(stg, name):
     return cfg, stg.stg_static_graph_create(cfg.V, oracle.unkey(S0)[0], oracle.unkey(S0)[1], 0), oracle.csr(cfg.V, S0)
 
 
-@pytest.mark.parametrize("name,H", [("C1", 16), ("C2", 32), ("C6", 16), ("C5s", 32), ("C2", 64), ("C1", 5)])
-def test_tgcn_step_parity(stg, name, H):
+@pytest.mark.parametrize("name,H,F", [("C1", 16, None), ("C2", 32, None), ("C6", 16, None), ("C5s", 32, None),
+                                      ("C2", 64, None), ("C1", 5, None), ("C2", 32, 12), ("C2", 32, 96),
+                                      ("C2", 16, 128), ("C5s", 32, 40)])
+def test_tgcn_step_parity(stg, name, H, F):
+    """F overrides cover every X·W path: pipelined (F <= 64, incl. K padding) and
+    one-tile-at-a-time (64 < F <= 128)."""
     cfg, g, ref = _graph(stg, name)
-    V, F = cfg.V, cfg.F
+    V = cfg.V
+    if F is None:
+        F = cfg.F
+        X = gen.features(cfg, 5)
+    else:
+        X = gen.uniform_pm1(9, F, V * F).reshape(V, F)
     p, pg = _params(F, H, 11)
-    X = gen.features(cfg, 5)
     Hp = gen.uniform_pm1(3, 3, V * H).reshape(V, H)
     Xg, Hg = to_gpu(X), to_gpu(Hp)
     stack = stg.stg_state_stack_create(64 << 20)
