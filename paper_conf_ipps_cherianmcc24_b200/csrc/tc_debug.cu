@@ -3,6 +3,11 @@
 //   mode 0: C[M,N] = A[M,K] · B[K,N]            (K-major A and B, M = 128·tiles)
 //   mode 1: C[128,N] = Xᵀ·Y, X[R,128], Y[R,N]    (MN-major views, R = 128·tiles,
 //           accumulated across tiles in TMEM — the reduction form of dW / dL)
+//   mode 2: as mode 0 with the A operand (hi/lo) written to TENSOR MEMORY by
+//           the threads (tcgen05.st, thread = row) and read by the MMA from there
+//   mode 3: ONE tf32 MMA on unsplit fp32 operands (A raw · B raw): the test
+//           compares it with truncated and rounded tf32 products to pin the
+//           hardware's fp32 -> tf32 input conversion
 #include "common.cuh"
 #include "tc.cuh"
 
@@ -20,18 +25,19 @@ __global__ void __launch_bounds__(128) k_tc_debug(int mode, int M, int N, int K,
   extern __shared__ __align__(1024) unsigned char sm[];
   __shared__ uint64_t mbar;
   __shared__ uint32_t tslot;
-  const int Kt = mode == 0 ? K : 32;            // K extent of a stored tile (32 rows for mode 1)
+  const int Kt = mode != 1 ? K : 32;            // K extent of a stored tile (32 rows for mode 1)
   const int Mrows = 128;
   unsigned char* a_hi = sm;
-  const int pf = mode == 0 ? 4 : 5;              // mode 1 tiles use the padded transposed layout
+  const int pf = mode != 1 ? 4 : 5;              // mode 1 tiles use the padded transposed layout
   unsigned char* a_lo = a_hi + Mrows * Kt * pf;
-  const int Kb = mode == 0 ? K : 32;             // mode 0: B stored [N × K]; mode 1: Yᵀ tile [N × 32]
+  const int Kb = mode != 1 ? K : 32;             // modes 0/2/3: B stored [N × K]; mode 1: Yᵀ tile [N × 32]
   const int Nr = N;
   unsigned char* b_hi = a_lo + Mrows * Kt * pf;
   unsigned char* b_lo = b_hi + Nr * Kb * pf;
   const int warp = threadIdx.x >> 5;
   uint32_t ncols = 32;
   while ((int)ncols < N) ncols <<= 1;
+  if (mode == 2) ncols = 512;                     // [0,256) accumulator, [256, 256+2K) A hi/lo
   if (warp == 0) tc::tmem_alloc(&tslot, ncols);
   if (threadIdx.x == 0) {
     tc::mbar_init(&mbar, 1);
@@ -42,21 +48,41 @@ __global__ void __launch_bounds__(128) k_tc_debug(int mode, int M, int N, int K,
   tc::fence_after();
   const uint32_t tm = tslot;
   uint32_t phase = 0;
-  const int tiles = mode == 0 ? 1 : R / 32;
-  const int row0 = mode == 0 ? blockIdx.x * 128 : 0;
+  const int tiles = mode != 1 ? 1 : R / 32;
+  const int row0 = mode != 1 ? blockIdx.x * 128 : 0;
   for (int tile = 0; tile < tiles; ++tile) {
     // ---- stage operands
-    if (mode == 0) {
-      for (int e = threadIdx.x; e < 128 * (K / 4); e += 128) {
+    if (mode == 2) {
+      const int r = threadIdx.x;                      // thread = row = TMEM lane (warp w -> lanes 32w..)
+      for (int k0 = 0; k0 < K; k0 += 8) {
+        float hv[8], lv[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const float v = A[(int64_t)(row0 + r) * K + k0 + i];
+          hv[i] = tc::tf32_hi(v);
+          lv[i] = v - hv[i];
+        }
+        tc::tmem_st8(tm + ((uint32_t)(warp * 32) << 16) + (uint32_t)(256 + k0), hv);
+        tc::tmem_st8(tm + ((uint32_t)(warp * 32) << 16) + (uint32_t)(256 + K + k0), lv);
+      }
+      tc::tmem_wait_st();
+    }
+    if (mode == 0 || mode == 2 || mode == 3) {
+      for (int e = threadIdx.x; mode != 2 && e < 128 * (K / 4); e += 128) {
         const int rl = e & 7, j = (e >> 3) % (K / 4), rg = e / (8 * (K / 4));
         const int r = rg * 8 + rl;
         float4 v = *reinterpret_cast<const float4*>(A + (int64_t)(row0 + r) * K + 4 * j);
-        tc::st_split4(a_hi, a_lo, r, j, K, v);
+        if (mode == 3) {            // raw fp32 as the "hi" operand
+          const uint32_t off = (uint32_t)((r & 7) * 16 + (r >> 3) * (K / 4) * 128 + j * 128);
+          *reinterpret_cast<float4*>(a_hi + off) = v;
+        } else {
+          tc::st_split4(a_hi, a_lo, r, j, K, v);
+        }
       }
       for (int e = threadIdx.x; e < N * K; e += 128) {   // B[k][n] -> K-major [n][k]
         const int n = e / K, k = e % K;
         const float v = B[(int64_t)k * N + n];
-        const float h = tc::tf32_hi(v);
+        const float h = mode == 3 ? v : tc::tf32_hi(v);
         *reinterpret_cast<float*>(b_hi + tc::kmaj_off(n, k, K)) = h;
         *reinterpret_cast<float*>(b_lo + tc::kmaj_off(n, k, K)) = v - h;
       }
@@ -74,6 +100,22 @@ __global__ void __launch_bounds__(128) k_tc_debug(int mode, int M, int N, int K,
       if (mode == 0) {
         tc::mma_3xtf32_kmajor(tm, tc::smem_u32(a_hi), tc::smem_u32(a_lo), tc::smem_u32(b_hi), tc::smem_u32(b_lo), K,
                               tc::idesc_tf32(128, N, 0, 0), false);
+      } else if (mode == 3) {
+        const uint32_t idesc = tc::idesc_tf32(128, N, 0, 0), sbo = (uint32_t)(K / 4) * 128;
+        for (int k = 0; k < K; k += 8) {
+          const uint32_t off = (uint32_t)(k / 4) * 128;
+          tc::mma_tf32(tm, tc::desc(tc::smem_u32(a_hi) + off, 128, sbo), tc::desc(tc::smem_u32(b_hi) + off, 128, sbo),
+                       idesc, k > 0 ? 1u : 0u);
+        }
+      } else if (mode == 2) {
+        const uint32_t idesc = tc::idesc_tf32(128, N, 0, 0), sbo = (uint32_t)(K / 4) * 128;
+        for (int k = 0; k < K; k += 8) {
+          const uint32_t off = (uint32_t)(k / 4) * 128;
+          const uint64_t bh = tc::desc(tc::smem_u32(b_hi) + off, 128, sbo), bl = tc::desc(tc::smem_u32(b_lo) + off, 128, sbo);
+          tc::mma_tf32_ts(tm, tm + 256 + K + k, bh, idesc, k > 0 ? 1u : 0u);   // A_lo·B_hi
+          tc::mma_tf32_ts(tm, tm + 256 + k, bl, idesc, 1u);                    // A_hi·B_lo
+          tc::mma_tf32_ts(tm, tm + 256 + k, bh, idesc, 1u);                    // A_hi·B_hi
+        }
       } else {
         const uint32_t sb = tc::sbo_t(32), idesc = tc::idesc_tf32(128, N, 0, 0);
         for (int k = 0; k < 32; k += 8) {
@@ -113,14 +155,16 @@ extern "C" stg_status stg_debug_tc_gemm(int32_t mode, int32_t M, int32_t N, int3
                                         const float* B, float* C, stg_stream_t stream) {
   using namespace stg;
   if (N % 16 || N < 16 || N > 256) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: N=%d", N);
-  if (mode == 0 && (M % 128 || K % 8 || K < 8 || K > 256)) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: M/K");
+  if (mode < 0 || mode > 3) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: mode=%d", mode);
+  if (mode != 1 && (M % 128 || K % 8 || K < 8 || K > 256)) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: M/K");
+  if (mode == 2 && K > 128) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: K > 128 for TMEM A");
   if (mode == 1 && (R % 32 || R < 32)) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: R");
-  const int Kt = mode == 0 ? K : 32, Kb = mode == 0 ? K : 32, Nr = N;
-  const int pf = mode == 0 ? 4 : 5;
+  const int Kt = mode != 1 ? K : 32, Kb = mode != 1 ? K : 32, Nr = N;
+  const int pf = mode != 1 ? 4 : 5;
   const size_t smem = (size_t)2 * 128 * Kt * pf + (size_t)2 * Nr * Kb * pf;
   if (smem > 200 * 1024) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: tile too large");
   STG_CUDA(cudaFuncSetAttribute(k_tc_debug, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const int grid = mode == 0 ? M / 128 : 1;
+  const int grid = mode != 1 ? M / 128 : 1;
   k_tc_debug<<<grid, 128, smem, (cudaStream_t)stream>>>(mode, M, N, K, R, A, B, C);
   count_launch();
   return check_launch("stg_debug_tc_gemm");

@@ -428,6 +428,193 @@ __global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_fwd(int V, const floa
   if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, 128);
 }
 
+// ------------------------------------------------------------------ GRU forward, v2
+// One persistent CTA per SM, 8 warps; thread = (tile row = TMEM lane, column
+// half).  Inputs arrive by TMA bulk row copies (one per row and tensor) into a
+// double-buffered shared-memory raw tile with odd 16-byte row pitches (the
+// row-per-lane reads are bank-conflict-free); the copies of tile i+2 are issued
+// as soon as tile i has been moved into tensor memory.  The MMA A operands
+// live in TENSOR MEMORY (tcgen05.mma ... [a_tmem]): the hardware reads fp32 as
+// tf32 by truncation (pinned by tests/test_gpu_tc.py), so hi = the raw value
+// and only lo = x - trunc(x) is computed.  TMEM columns (units of H):
+//   [0,3H) [C_z|C_r|H] hi, [3H,6H) lo, [6H,7H) C_h hi, [7H,8H) lo,
+//   [8H,9H) acc z, [9H,10H) acc r, [10H,11H) RH hi, [11H,12H) lo, [12H,13H) acc h.
+// H' leaves through a per-warp shared stage (coalesced 64-byte row segments).
+template <int H>
+struct GruF2 {
+  static constexpr int H3 = 3 * H, HH = H / 2, NQ = HH / 4;
+  static constexpr int PC = H3 + 4, PH = H + 4;           // raw row pitches in floats (odd multiples of 16 B)
+  static constexpr int RAWC = 128 * PC * 4, RAWH = 128 * PH * 4, RAW = RAWC + RAWH;
+  static constexpr int BG = H * 2 * H * 4;
+  static constexpr int STAGE = 32 * tc::kStagePitch<NQ> * 16;
+  static constexpr int SMEM = 6 * BG + 2 * RAW + 8 * STAGE;
+  static constexpr uint32_t TCOLS = 13 * H <= 256 ? 256 : 512;
+};
+
+// 3xTF32 chain with A in tensor memory (columns a_hi.., a_lo..) and B in smem.
+__device__ __forceinline__ void mma_ts_seg(uint32_t d, uint32_t a_hi, uint32_t a_lo, uint32_t bhi, uint32_t blo,
+                                           int b_K, int b_k0, int len, uint32_t idesc, bool first) {
+  const uint32_t sb = (uint32_t)(b_K / 4) * 128;
+  for (int k = 0; k < len; k += 8) {
+    const uint32_t ob = (uint32_t)((b_k0 + k) / 4) * 128;
+    const uint64_t dh = tc::desc(bhi + ob, 128, sb), dl = tc::desc(blo + ob, 128, sb);
+    tc::mma_tf32_ts(d, a_lo + k, dh, idesc, (first && k == 0) ? 0u : 1u);
+    tc::mma_tf32_ts(d, a_hi + k, dl, idesc, 1u);
+    tc::mma_tf32_ts(d, a_hi + k, dh, idesc, 1u);
+  }
+}
+
+// HH fp32 values of a shared raw row -> TMEM (hi = raw, lo = raw - trunc(raw)) at columns (hi, lo)
+template <int HH>
+__device__ __forceinline__ void raw_to_tmem(const float* src, uint32_t t_hi, uint32_t t_lo, float (&v)[HH]) {
+#pragma unroll
+  for (int q = 0; q < HH / 4; ++q) {
+    const float4 x = reinterpret_cast<const float4*>(src)[q];
+    v[4 * q] = x.x; v[4 * q + 1] = x.y; v[4 * q + 2] = x.z; v[4 * q + 3] = x.w;
+  }
+  float lo[HH];
+#pragma unroll
+  for (int j = 0; j < HH; ++j) lo[j] = v[j] - tc::tf32_hi(v[j]);
+  if constexpr (HH == 16) {
+    tc::tmem_st16(t_hi, v);
+    tc::tmem_st16(t_lo, lo);
+  } else {
+    static_assert(HH == 8, "HH");
+    tc::tmem_st8(t_hi, v);
+    tc::tmem_st8(t_lo, lo);
+  }
+}
+
+template <int H>
+__global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const float* __restrict__ C, const float* __restrict__ Hp,
+                                                        const float* __restrict__ L, const float* __restrict__ l,
+                                                        float* __restrict__ Hn) {
+  using G = GruF2<H>;
+  constexpr int H3 = G::H3, HH = G::HH, NQ = G::NQ;
+  extern __shared__ __align__(128) unsigned char sm[];
+  __shared__ uint64_t full[2], mma_bar;
+  __shared__ uint32_t tslot;
+  unsigned char* bz_hi = sm;            unsigned char* bz_lo = bz_hi + G::BG;
+  unsigned char* br_hi = bz_lo + G::BG; unsigned char* br_lo = br_hi + G::BG;
+  unsigned char* bh_hi = br_lo + G::BG; unsigned char* bh_lo = bh_hi + G::BG;
+  unsigned char* raw0 = sm + 6 * G::BG;
+  auto rawC = [&](int b) { return reinterpret_cast<float*>(raw0 + (size_t)b * G::RAW); };
+  auto rawH = [&](int b) { return reinterpret_cast<float*>(raw0 + (size_t)b * G::RAW + G::RAWC); };
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, hf = warp >> 2;
+  const int lr = q * 32 + lane, c0 = hf * HH;
+  float4* stage = reinterpret_cast<float4*>(raw0 + 2 * (size_t)G::RAW) + warp * 32 * tc::kStagePitch<NQ>;
+  const int LG = 2 * H * H;
+  stage_gate_weights<H>(bz_hi, bz_lo, L);
+  stage_gate_weights<H>(br_hi, br_lo, L + LG);
+  stage_gate_weights<H>(bh_hi, bh_lo, L + 2 * LG);
+  if (warp == 0) tc::tmem_alloc(&tslot, G::TCOLS);
+  if (threadIdx.x == 0) {
+    tc::mbar_init(&full[0], 1); tc::mbar_init(&full[1], 1); tc::mbar_init(&mma_bar, 1);
+    tc::fence_mbar_init();
+  }
+  tc::fence_proxy_async();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  const uint32_t tq = tm + ((uint32_t)(q * 32) << 16);   // this thread's TMEM lane quarter
+  const int ntiles = (V + 127) / 128;
+  float lz[HH], lrr[HH], lh[HH];
+#pragma unroll
+  for (int j = 0; j < HH; ++j) { lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; }
+  auto issue = [&](int tile, int b) {                   // TMA row copies of tile into raw buffer b
+    if (tile >= ntiles) return;
+    const int r0 = tile * 128, nv = min(128, V - r0);
+    if (threadIdx.x == 0) tc::mbar_expect_tx(&full[b], (uint32_t)nv * (H3 + H) * 4);
+    if (lr < nv) {
+      if (hf == 0) tc::bulk_g2s(rawC(b) + lr * G::PC, C + (int64_t)(r0 + lr) * H3, H3 * 4, &full[b]);
+      else tc::bulk_g2s(rawH(b) + lr * G::PH, Hp + (int64_t)(r0 + lr) * H, H * 4, &full[b]);
+    }
+  };
+  issue(blockIdx.x, 0);
+  issue(blockIdx.x + gridDim.x, 1);
+  const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0);
+  uint32_t mph = 0;
+  int i = 0;
+  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+    const int b = i & 1, r0 = tile * 128, nv = min(128, V - r0);
+    tc::mbar_wait(&full[b], (i >> 1) & 1);
+    // raw tile -> tensor-memory A operands; this thread's half of H stays in registers
+    float h[HH];
+    {
+      float t[HH];
+      const float* rc = rawC(b) + lr * G::PC;
+      raw_to_tmem<HH>(rc + c0, tq + c0, tq + 3 * H + c0, t);                    // C_z
+      raw_to_tmem<HH>(rc + H + c0, tq + H + c0, tq + 4 * H + c0, t);            // C_r
+      raw_to_tmem<HH>(rc + 2 * H + c0, tq + 6 * H + c0, tq + 7 * H + c0, t);    // C_h
+      raw_to_tmem<HH>(rawH(b) + lr * G::PH + c0, tq + 2 * H + c0, tq + 5 * H + c0, h);   // H
+    }
+    tc::tmem_wait_st();
+    tc::fence_before();
+    __syncthreads();
+    issue(tile + 2 * gridDim.x, b);                    // raw buffer b is free
+    if (threadIdx.x == 0) {
+      tc::fence_after();
+      const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
+      mma_ts_seg(tm + 8 * H, tm + 0, tm + 3 * H, zh, zl, 2 * H, 0, H, idesc, true);          // z: C_z part
+      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, idesc, false);     //    H part
+      mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, idesc, true);         // r: C_r part
+      mma_ts_seg(tm + 9 * H, tm + 2 * H, tm + 5 * H, rh_, rl, 2 * H, H, H, idesc, false);    //    H part
+      tc::commit(&mma_bar);
+    }
+    tc::mbar_wait(&mma_bar, mph);
+    mph ^= 1;
+    tc::fence_after();
+    float z[HH];
+    {
+      float az[HH], ar[HH], rh[HH], lo[HH];
+      tmem_row_load<HH>(tm + 8 * H, c0, az);
+      tmem_row_load<HH>(tm + 9 * H, c0, ar);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        z[j] = sigm(az[j] + lz[j]);
+        rh[j] = sigm(ar[j] + lrr[j]) * h[j];
+        lo[j] = rh[j] - tc::tf32_hi(rh[j]);
+      }
+      if constexpr (HH == 16) { tc::tmem_st16(tq + 10 * H + c0, rh); tc::tmem_st16(tq + 11 * H + c0, lo); }
+      else { tc::tmem_st8(tq + 10 * H + c0, rh); tc::tmem_st8(tq + 11 * H + c0, lo); }
+    }
+    tc::tmem_wait_st();
+    tc::fence_before();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      tc::fence_after();
+      const uint32_t hh_ = tc::smem_u32(bh_hi), hl = tc::smem_u32(bh_lo);
+      mma_ts_seg(tm + 12 * H, tm + 6 * H, tm + 7 * H, hh_, hl, 2 * H, 0, H, idesc, true);    // h: C_h part
+      mma_ts_seg(tm + 12 * H, tm + 10 * H, tm + 11 * H, hh_, hl, 2 * H, H, H, idesc, false); //    RH part
+      tc::commit(&mma_bar);
+    }
+    tc::mbar_wait(&mma_bar, mph);
+    mph ^= 1;
+    tc::fence_after();
+    {
+      float ah[HH];
+      tmem_row_load<HH>(tm + 12 * H, c0, ah);
+      float4* srow = stage + lane * tc::kStagePitch<NQ>;
+#pragma unroll
+      for (int qq = 0; qq < NQ; ++qq) {
+        float o[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int j = 4 * qq + e;
+          const float hh = tanhf(ah[j] + lh[j]);
+          o[e] = z[j] * h[j] + (1.0f - z[j]) * hh;
+        }
+        srow[qq] = make_float4(o[0], o[1], o[2], o[3]);
+      }
+      tc::flush_stage_rows<NQ>(stage, Hn + c0, H, r0 + q * 32, nv - q * 32);
+    }
+    tc::fence_before();
+  }
+  __syncthreads();
+  if (warp == 0) tc::tmem_free(tm, G::TCOLS);
+}
+
 // ------------------------------------------------------------------ GRU backward
 template <int H>
 __global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_bwd(int V, const float* __restrict__ C,
@@ -801,16 +988,13 @@ stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const floa
 stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float* L, const float* l, float* Hn,
                       cudaStream_t s) {
   const int ntiles = (V + 127) / 128;
+  const int nb = std::min(ntiles, num_sms());
   if (H == 32) {
-    const size_t smem = 6 * GruSmem<32>::BG + 2 * GruSmem<32>::A1;
-    STG_TRY(prep(k_tc_gru_fwd<32>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_fwd<32>, smem, kGruThreads));
-    k_tc_gru_fwd<32><<<nb, kGruThreads, smem, s>>>(V, C, Hp, L, l, Hn);
+    STG_TRY(prep(k_tc_gru_fwd2<32>, GruF2<32>::SMEM));
+    k_tc_gru_fwd2<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, C, Hp, L, l, Hn);
   } else {
-    const size_t smem = 6 * GruSmem<16>::BG + 2 * GruSmem<16>::A1;
-    STG_TRY(prep(k_tc_gru_fwd<16>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_fwd<16>, smem, kGruThreads));
-    k_tc_gru_fwd<16><<<nb, kGruThreads, smem, s>>>(V, C, Hp, L, l, Hn);
+    STG_TRY(prep(k_tc_gru_fwd2<16>, GruF2<16>::SMEM));
+    k_tc_gru_fwd2<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, C, Hp, L, l, Hn);
   }
   count_launch();
   return check_launch("tc_gru_fwd");

@@ -31,3 +31,40 @@ def test_tc_gemm_mn_major_reduction(stg, R, N):
     C = stg.stg_debug_tc_gemm(1, to_gpu(X), to_gpu(Y)).cpu().numpy()
     err = np.max(np.abs(C - X.T @ Y) / _cond(X.T, Y))
     assert err < 2e-6, err
+
+
+@pytest.mark.parametrize("M,K,N", [(128, 8, 16), (128, 64, 96), (256, 96, 64), (128, 128, 32), (128, 32, 256)])
+def test_tc_gemm_a_in_tmem(stg, M, K, N):
+    """A operand written to tensor memory by the threads (tcgen05.st, lane = row,
+    column = k) and read by tcgen05.mma.kind::tf32 [d], [a_tmem], b_desc."""
+    A = gen.uniform_pm1(5, M + K, M * K).reshape(M, K).astype(np.float64)
+    B = gen.uniform_pm1(6, K + N, K * N).reshape(K, N).astype(np.float64)
+    C = stg.stg_debug_tc_gemm(2, to_gpu(A), to_gpu(B)).cpu().numpy()
+    err = np.max(np.abs(C - A @ B) / _cond(A, B))
+    assert err < 2e-6, err
+
+
+def _tf32_trunc(x):
+    u = np.asarray(x, np.float32).view(np.uint32) & np.uint32(0xFFFFE000)
+    return u.view(np.float32).astype(np.float64)
+
+
+def _tf32_rna(x):
+    u = np.asarray(x, np.float32).view(np.uint32).astype(np.uint64)
+    u = ((u + np.uint64(0x1000)) & np.uint64(0xFFFFE000)).astype(np.uint32)
+    return u.view(np.float32).astype(np.float64)
+
+
+def test_tf32_input_conversion(stg):
+    """Pins how kind::tf32 reads fp32 operands: one unsplit pass equals the
+    product of the TRUNCATED (low 13 mantissa bits dropped) operands, which is
+    why 3xTF32 takes hi = a & 0xFFFFE000 and lo = a - hi."""
+    M, K, N = 128, 64, 64
+    A = gen.uniform_pm1(7, 1, M * K).reshape(M, K).astype(np.float64)
+    B = gen.uniform_pm1(8, 1, K * N).reshape(K, N).astype(np.float64)
+    C = stg.stg_debug_tc_gemm(3, to_gpu(A), to_gpu(B)).cpu().numpy()
+    cond = _cond(A, B)
+    e_trunc = np.max(np.abs(C - _tf32_trunc(A) @ _tf32_trunc(B)) / cond)
+    e_rna = np.max(np.abs(C - _tf32_rna(A) @ _tf32_rna(B)) / cond)
+    print("tf32 conversion: err vs truncation %.3g, vs round-nearest %.3g" % (e_trunc, e_rna))
+    assert e_trunc < 1e-6 and e_rna > 1e-5, (e_trunc, e_rna)
