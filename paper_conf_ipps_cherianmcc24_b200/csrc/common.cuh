@@ -2,6 +2,7 @@
 // kernel launch accounting.  Product code only (no oracle code is reachable).
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <atomic>
@@ -84,6 +85,12 @@ struct Scratch {
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 int num_sms();
+
+// 2-D TMA descriptor of a row-major fp32 matrix [rows × cols] (row stride ld
+// elements, 16-byte aligned), box [box_rows × box_cols] with 128-byte swizzle
+// (box_cols·4 <= 128).  Encoded through the driver entry point (no libcuda link).
+stg_status make_tmap_f32(CUtensorMap* out, const float* base, uint64_t rows, uint64_t cols, uint64_t ld,
+                         uint32_t box_cols, uint32_t box_rows);
 
 // ---------------------------------------------------------------- profiler
 // Per-phase device time with CUDA events on the launching stream (bench.py and

@@ -14,6 +14,8 @@
 //   A·B ≈ A_lo·B_hi + A_hi·B_lo + A_hi·B_hi, accumulated in fp32 in TMEM.
 #pragma once
 
+#include <cuda.h>
+
 #include <cstdint>
 
 namespace stg {
@@ -78,6 +80,17 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* mbar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
 }
+
+// 2-D TMA tensor load of box (c0, r0) of a tensor map into shared memory
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int c0, int r0, uint64_t* mbar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(r0), "r"(smem_u32(mbar))
+      : "memory");
+}
+// byte offset of 16-byte chunk c (0..7) of row r in a 128-byte-swizzled box (rows of 128 B)
+__device__ __forceinline__ uint32_t swz128(int r, int c) { return (uint32_t)(r * 128 + ((c ^ (r & 7)) << 4)); }
 
 // plain arrive (count 1) on an mbarrier from a thread
 __device__ __forceinline__ void mbar_arrive(uint64_t* mbar) {

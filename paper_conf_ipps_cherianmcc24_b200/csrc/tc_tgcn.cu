@@ -284,7 +284,7 @@ __device__ __forceinline__ void stage_gate_weights(unsigned char* hi, unsigned c
 template <int H>
 __device__ __forceinline__ void stage_plain(unsigned char* hi, unsigned char* lo, const float* __restrict__ Lg) {
   // Lg [2H][H] row-major is already K-major as [N = 2H rows × K = H]
-  for (int e = threadIdx.x; e < 2 * H * H; e += kTcThreads) {
+  for (int e = threadIdx.x; e < 2 * H * H; e += blockDim.x) {
     const int n = e / H, k = e % H;
     const float v = Lg[e];
     const float h = tc::tf32_hi(v);
@@ -430,24 +430,27 @@ __global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_fwd(int V, const floa
 
 // ------------------------------------------------------------------ GRU forward, v2
 // One persistent CTA per SM, 8 warps; thread = (tile row = TMEM lane, column
-// half).  Inputs arrive by TMA bulk row copies (one per row and tensor) into a
-// double-buffered shared-memory raw tile with odd 16-byte row pitches (the
-// row-per-lane reads are bank-conflict-free); the copies of tile i+2 are issued
-// as soon as tile i has been moved into tensor memory.  The MMA A operands
-// live in TENSOR MEMORY (tcgen05.mma ... [a_tmem]): the hardware reads fp32 as
-// tf32 by truncation (pinned by tests/test_gpu_tc.py), so hi = the raw value
-// and only lo = x - trunc(x) is computed.  TMEM columns (units of H):
+// half).  Inputs arrive by 2-D TMA tensor loads (boxes of 128 rows x 32 fp32,
+// 128-byte swizzle, so the row-per-lane reads below are bank-conflict-free)
+// into a double-buffered raw tile; tile i+2 is requested as soon as tile i
+// has been moved into tensor memory.  The MMA A operands live in TENSOR
+// MEMORY (tcgen05.mma ... [a_tmem]): the hardware reads fp32 as tf32 by
+// truncation (pinned by tests/test_gpu_tc.py), so hi = the raw value and only
+// lo = x - trunc(x) is computed.  TMEM columns (units of H):
 //   [0,3H) [C_z|C_r|H] hi, [3H,6H) lo, [6H,7H) C_h hi, [7H,8H) lo,
 //   [8H,9H) acc z, [9H,10H) acc r, [10H,11H) RH hi, [11H,12H) lo, [12H,13H) acc h.
 // H' leaves through a per-warp shared stage (coalesced 64-byte row segments).
+constexpr int kBox = 128 * 32 * 4;       // one TMA box: 128 rows x 32 fp32 (16 KB)
+
 template <int H>
 struct GruF2 {
   static constexpr int H3 = 3 * H, HH = H / 2, NQ = HH / 4;
-  static constexpr int PC = H3 + 4, PH = H + 4;           // raw row pitches in floats (odd multiples of 16 B)
-  static constexpr int RAWC = 128 * PC * 4, RAWH = 128 * PH * 4, RAW = RAWC + RAWH;
+  static constexpr int NBC = (H3 + 31) / 32, NBH = (H + 31) / 32;   // boxes per C / H tile
+  static constexpr int RAW = (NBC + NBH) * kBox;
   static constexpr int BG = H * 2 * H * 4;
   static constexpr int STAGE = 32 * tc::kStagePitch<NQ> * 16;
-  static constexpr int SMEM = 6 * BG + 2 * RAW + 8 * STAGE;
+  static constexpr int WOFF = 2 * RAW;                              // weights after the raw buffers
+  static constexpr int SMEM = WOFF + 6 * BG + 8 * STAGE + 1024;     // + alignment slack
   static constexpr uint32_t TCOLS = 13 * H <= 256 ? 256 : 512;
 };
 
@@ -464,12 +467,16 @@ __device__ __forceinline__ void mma_ts_seg(uint32_t d, uint32_t a_hi, uint32_t a
   }
 }
 
-// HH fp32 values of a shared raw row -> TMEM (hi = raw, lo = raw - trunc(raw)) at columns (hi, lo)
+// HH fp32 values (columns col..col+HH of row r) of a raw tile made of 128x32
+// swizzled boxes -> TMEM (hi = raw, lo = raw - trunc(raw)) at columns (t_hi, t_lo)
 template <int HH>
-__device__ __forceinline__ void raw_to_tmem(const float* src, uint32_t t_hi, uint32_t t_lo, float (&v)[HH]) {
+__device__ __forceinline__ void raw_to_tmem(const unsigned char* tile, int r, int col, uint32_t t_hi, uint32_t t_lo,
+                                            float (&v)[HH]) {
+  const unsigned char* box = tile + (col / 32) * kBox;
+  const int c16 = (col % 32) / 4;
 #pragma unroll
   for (int q = 0; q < HH / 4; ++q) {
-    const float4 x = reinterpret_cast<const float4*>(src)[q];
+    const float4 x = *reinterpret_cast<const float4*>(box + tc::swz128(r, c16 + q));
     v[4 * q] = x.x; v[4 * q + 1] = x.y; v[4 * q + 2] = x.z; v[4 * q + 3] = x.w;
   }
   float lo[HH];
@@ -486,23 +493,24 @@ __device__ __forceinline__ void raw_to_tmem(const float* src, uint32_t t_hi, uin
 }
 
 template <int H>
-__global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const float* __restrict__ C, const float* __restrict__ Hp,
+__global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_constant__ CUtensorMap tmC,
+                                                        const __grid_constant__ CUtensorMap tmH,
                                                         const float* __restrict__ L, const float* __restrict__ l,
                                                         float* __restrict__ Hn) {
   using G = GruF2<H>;
-  constexpr int H3 = G::H3, HH = G::HH, NQ = G::NQ;
-  extern __shared__ __align__(128) unsigned char sm[];
+  constexpr int HH = G::HH, NQ = G::NQ;
+  extern __shared__ unsigned char sm_raw[];
+  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full[2], mma_bar;
   __shared__ uint32_t tslot;
-  unsigned char* bz_hi = sm;            unsigned char* bz_lo = bz_hi + G::BG;
+  unsigned char* bz_hi = sm + G::WOFF;  unsigned char* bz_lo = bz_hi + G::BG;
   unsigned char* br_hi = bz_lo + G::BG; unsigned char* br_lo = br_hi + G::BG;
   unsigned char* bh_hi = br_lo + G::BG; unsigned char* bh_lo = bh_hi + G::BG;
-  unsigned char* raw0 = sm + 6 * G::BG;
-  auto rawC = [&](int b) { return reinterpret_cast<float*>(raw0 + (size_t)b * G::RAW); };
-  auto rawH = [&](int b) { return reinterpret_cast<float*>(raw0 + (size_t)b * G::RAW + G::RAWC); };
+  auto rawC = [&](int b) { return sm + (size_t)b * G::RAW; };
+  auto rawH = [&](int b) { return sm + (size_t)b * G::RAW + G::NBC * kBox; };
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, hf = warp >> 2;
   const int lr = q * 32 + lane, c0 = hf * HH;
-  float4* stage = reinterpret_cast<float4*>(raw0 + 2 * (size_t)G::RAW) + warp * 32 * tc::kStagePitch<NQ>;
+  float4* stage = reinterpret_cast<float4*>(bh_lo + G::BG) + warp * 32 * tc::kStagePitch<NQ>;
   const int LG = 2 * H * H;
   stage_gate_weights<H>(bz_hi, bz_lo, L);
   stage_gate_weights<H>(br_hi, br_lo, L + LG);
@@ -522,17 +530,17 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const float* __re
   float lz[HH], lrr[HH], lh[HH];
 #pragma unroll
   for (int j = 0; j < HH; ++j) { lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; }
-  auto issue = [&](int tile, int b) {                   // TMA row copies of tile into raw buffer b
+  auto issue = [&](int tile, int b) {                   // (thread 0) TMA boxes of tile into raw buffer b
     if (tile >= ntiles) return;
-    const int r0 = tile * 128, nv = min(128, V - r0);
-    if (threadIdx.x == 0) tc::mbar_expect_tx(&full[b], (uint32_t)nv * (H3 + H) * 4);
-    if (lr < nv) {
-      if (hf == 0) tc::bulk_g2s(rawC(b) + lr * G::PC, C + (int64_t)(r0 + lr) * H3, H3 * 4, &full[b]);
-      else tc::bulk_g2s(rawH(b) + lr * G::PH, Hp + (int64_t)(r0 + lr) * H, H * 4, &full[b]);
-    }
+    tc::mbar_expect_tx(&full[b], (uint32_t)(G::NBC + G::NBH) * kBox);
+#pragma unroll
+    for (int k = 0; k < G::NBC; ++k) tc::tma_load_2d(rawC(b) + k * kBox, &tmC, 32 * k, tile * 128, &full[b]);
+    tc::tma_load_2d(rawH(b), &tmH, 0, tile * 128, &full[b]);
   };
-  issue(blockIdx.x, 0);
-  issue(blockIdx.x + gridDim.x, 1);
+  if (threadIdx.x == 0) {
+    issue(blockIdx.x, 0);
+    issue(blockIdx.x + gridDim.x, 1);
+  }
   const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0);
   uint32_t mph = 0;
   int i = 0;
@@ -543,16 +551,14 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const float* __re
     float h[HH];
     {
       float t[HH];
-      const float* rc = rawC(b) + lr * G::PC;
-      raw_to_tmem<HH>(rc + c0, tq + c0, tq + 3 * H + c0, t);                    // C_z
-      raw_to_tmem<HH>(rc + H + c0, tq + H + c0, tq + 4 * H + c0, t);            // C_r
-      raw_to_tmem<HH>(rc + 2 * H + c0, tq + 6 * H + c0, tq + 7 * H + c0, t);    // C_h
-      raw_to_tmem<HH>(rawH(b) + lr * G::PH + c0, tq + 2 * H + c0, tq + 5 * H + c0, h);   // H
+      raw_to_tmem<HH>(rawC(b), lr, c0, tq + c0, tq + 3 * H + c0, t);                    // C_z
+      raw_to_tmem<HH>(rawC(b), lr, H + c0, tq + H + c0, tq + 4 * H + c0, t);            // C_r
+      raw_to_tmem<HH>(rawC(b), lr, 2 * H + c0, tq + 6 * H + c0, tq + 7 * H + c0, t);    // C_h
+      raw_to_tmem<HH>(rawH(b), lr, c0, tq + 2 * H + c0, tq + 5 * H + c0, h);            // H
     }
     tc::tmem_wait_st();
     tc::fence_before();
     __syncthreads();
-    issue(tile + 2 * gridDim.x, b);                    // raw buffer b is free
     if (threadIdx.x == 0) {
       tc::fence_after();
       const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
@@ -561,6 +567,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const float* __re
       mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, idesc, true);         // r: C_r part
       mma_ts_seg(tm + 9 * H, tm + 2 * H, tm + 5 * H, rh_, rl, 2 * H, H, H, idesc, false);    //    H part
       tc::commit(&mma_bar);
+      issue(tile + 2 * gridDim.x, b);                  // raw buffer b is free
     }
     tc::mbar_wait(&mma_bar, mph);
     mph ^= 1;
@@ -762,6 +769,244 @@ __global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_bwd(int V, const floa
   tc::fence_before();
   __syncthreads();
   if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
+}
+
+// ------------------------------------------------------------------ GRU backward, v2
+// Same data path as k_tc_gru_fwd2 (TMA boxes -> swizzled raw tile -> tensor
+// memory A operands; single raw buffer: the next tile is requested as soon as
+// the current one is in TMEM, so its loads overlap the four MMA phases):
+//   P1 z, r  (recompute, [C_z|H]·L_z, [C_r|H]·L_r)      P2 h ([C_h|RH]·L_h)
+//   P3 [dC_h|dRH] = da_h·L_hᵀ, [dC_z|dH_z] = da_z·L_zᵀ  P4 [dC_r|dH_r] = da_r·L_rᵀ
+// TMEM columns (units of H): P1/P2 as in k_tc_gru_fwd2; afterwards
+//   [0,H) da_h hi, [H,2H) lo, [2H,3H) da_z hi, [3H,4H) lo, [4H,6H) acc P3h,
+//   [6H,8H) acc P3z, [10H,11H) da_r hi, [11H,12H) lo, [8H,10H) acc P4.
+// Outputs dC' = n_dst ⊙ dC, dH_prev, da = [da_z|da_r|da_h], RH leave through
+// the per-warp shared stage (coalesced 64-byte row segments).
+template <int H>
+struct GruB2 {
+  static constexpr int H3 = 3 * H, HH = H / 2, NQ = HH / 4;
+  static constexpr int NBC = (H3 + 31) / 32, NBH = (H + 31) / 32;
+  static constexpr int RAW = (NBC + 2 * NBH) * kBox;                // C, H, G
+  static constexpr int BG = H * 2 * H * 4;
+  static constexpr int STAGE = 32 * tc::kStagePitch<NQ> * 16;
+  static constexpr int WOFF = RAW;
+  static constexpr int SMEM = WOFF + 12 * BG + 8 * STAGE + 1024;
+  static constexpr uint32_t TCOLS = 13 * H <= 256 ? 256 : 512;
+};
+
+template <int HH>
+__device__ __forceinline__ void tmem_st_split(uint32_t t_hi, uint32_t t_lo, const float (&v)[HH]) {
+  float lo[HH];
+#pragma unroll
+  for (int j = 0; j < HH; ++j) lo[j] = v[j] - tc::tf32_hi(v[j]);
+  if constexpr (HH == 16) {
+    tc::tmem_st16(t_hi, v);
+    tc::tmem_st16(t_lo, lo);
+  } else {
+    tc::tmem_st8(t_hi, v);
+    tc::tmem_st8(t_lo, lo);
+  }
+}
+
+// stage this thread's HH values (times s) as its row of the warp stage and flush to dst
+template <int HH>
+__device__ __forceinline__ void stage_flush(float4* stage, const float (&v)[HH], float s, float* dst, int64_t ld,
+                                            int row0, int nvalid) {
+  constexpr int NQ = HH / 4;
+  float4* srow = stage + (threadIdx.x & 31) * tc::kStagePitch<NQ>;
+#pragma unroll
+  for (int qq = 0; qq < NQ; ++qq)
+    srow[qq] = make_float4(s * v[4 * qq], s * v[4 * qq + 1], s * v[4 * qq + 2], s * v[4 * qq + 3]);
+  tc::flush_stage_rows<NQ>(stage, dst, ld, row0, nvalid);
+}
+
+template <int H>
+__global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_constant__ CUtensorMap tmC,
+                                                        const __grid_constant__ CUtensorMap tmH,
+                                                        const __grid_constant__ CUtensorMap tmG,
+                                                        const float* __restrict__ L, const float* __restrict__ l,
+                                                        const float* __restrict__ ndst, float* __restrict__ dCs,
+                                                        float* __restrict__ dHp, float* __restrict__ da,
+                                                        float* __restrict__ RHo) {
+  using G = GruB2<H>;
+  constexpr int H3 = G::H3, HH = G::HH, NQ = G::NQ;
+  extern __shared__ unsigned char sm_raw[];
+  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t full, mma_bar;
+  __shared__ uint32_t tslot;
+  unsigned char* w0 = sm + G::WOFF;
+  unsigned char* bz_hi = w0;              unsigned char* bz_lo = w0 + 1 * G::BG;
+  unsigned char* br_hi = w0 + 2 * G::BG;  unsigned char* br_lo = w0 + 3 * G::BG;
+  unsigned char* bh_hi = w0 + 4 * G::BG;  unsigned char* bh_lo = w0 + 5 * G::BG;
+  unsigned char* lz_hi = w0 + 6 * G::BG;  unsigned char* lz_lo = w0 + 7 * G::BG;
+  unsigned char* lr_hi = w0 + 8 * G::BG;  unsigned char* lr_lo = w0 + 9 * G::BG;
+  unsigned char* lh_hi = w0 + 10 * G::BG; unsigned char* lh_lo = w0 + 11 * G::BG;
+  unsigned char* rawC = sm;
+  unsigned char* rawH = sm + G::NBC * kBox;
+  unsigned char* rawG = sm + (G::NBC + G::NBH) * kBox;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, hf = warp >> 2;
+  const int lr = q * 32 + lane, c0 = hf * HH;
+  float4* stage = reinterpret_cast<float4*>(w0 + 12 * G::BG) + warp * 32 * tc::kStagePitch<NQ>;
+  const int LG = 2 * H * H;
+  stage_gate_weights<H>(bz_hi, bz_lo, L);
+  stage_gate_weights<H>(br_hi, br_lo, L + LG);
+  stage_gate_weights<H>(bh_hi, bh_lo, L + 2 * LG);
+  stage_plain<H>(lz_hi, lz_lo, L);
+  stage_plain<H>(lr_hi, lr_lo, L + LG);
+  stage_plain<H>(lh_hi, lh_lo, L + 2 * LG);
+  if (warp == 0) tc::tmem_alloc(&tslot, G::TCOLS);
+  if (threadIdx.x == 0) {
+    tc::mbar_init(&full, 1); tc::mbar_init(&mma_bar, 1);
+    tc::fence_mbar_init();
+  }
+  tc::fence_proxy_async();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  const uint32_t tq = tm + ((uint32_t)(q * 32) << 16);
+  const int ntiles = (V + 127) / 128;
+  auto issue = [&](int tile) {                          // (thread 0) TMA boxes of tile into the raw buffer
+    if (tile >= ntiles) return;
+    tc::mbar_expect_tx(&full, (uint32_t)(G::NBC + 2 * G::NBH) * kBox);
+#pragma unroll
+    for (int k = 0; k < G::NBC; ++k) tc::tma_load_2d(rawC + k * kBox, &tmC, 32 * k, tile * 128, &full);
+    tc::tma_load_2d(rawH, &tmH, 0, tile * 128, &full);
+    tc::tma_load_2d(rawG, &tmG, 0, tile * 128, &full);
+  };
+  if (threadIdx.x == 0) issue(blockIdx.x);
+  const uint32_t id_h = tc::idesc_tf32(128, H, 0, 0), id_2h = tc::idesc_tf32(128, 2 * H, 0, 0);
+  auto mma_wait = [&](uint32_t& ph) {
+    tc::mbar_wait(&mma_bar, ph);
+    ph ^= 1;
+    tc::fence_after();
+  };
+  auto sync_tmem = [&]() {                              // thread-written TMEM visible to the MMA issuer
+    tc::tmem_wait_st();
+    tc::fence_before();
+    __syncthreads();
+  };
+  uint32_t mph = 0;
+  int i = 0;
+  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+    const int r0 = tile * 128, nv = min(128, V - r0), wr0 = r0 + q * 32, wnv = nv - q * 32;
+    const int row = r0 + lr;
+    const float nd = row < V ? __ldg(ndst + row) : 0.f;
+    tc::mbar_wait(&full, i & 1);
+    float h[HH], g[HH];
+    {
+      float t[HH];
+      raw_to_tmem<HH>(rawC, lr, c0, tq + c0, tq + 3 * H + c0, t);                    // C_z
+      raw_to_tmem<HH>(rawC, lr, H + c0, tq + H + c0, tq + 4 * H + c0, t);            // C_r
+      raw_to_tmem<HH>(rawC, lr, 2 * H + c0, tq + 6 * H + c0, tq + 7 * H + c0, t);    // C_h
+      raw_to_tmem<HH>(rawH, lr, c0, tq + 2 * H + c0, tq + 5 * H + c0, h);            // H
+      const unsigned char* box = rawG + (c0 / 32) * kBox;
+#pragma unroll
+      for (int qq = 0; qq < HH / 4; ++qq) {
+        const float4 x = *reinterpret_cast<const float4*>(box + tc::swz128(lr, (c0 % 32) / 4 + qq));
+        g[4 * qq] = x.x; g[4 * qq + 1] = x.y; g[4 * qq + 2] = x.z; g[4 * qq + 3] = x.w;
+      }
+    }
+    sync_tmem();
+    if (threadIdx.x == 0) {                             // P1; then request the next tile
+      tc::fence_after();
+      const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
+      mma_ts_seg(tm + 8 * H, tm + 0, tm + 3 * H, zh, zl, 2 * H, 0, H, id_h, true);
+      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, id_h, false);
+      mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, id_h, true);
+      mma_ts_seg(tm + 9 * H, tm + 2 * H, tm + 5 * H, rh_, rl, 2 * H, H, H, id_h, false);
+      tc::commit(&mma_bar);
+      issue(tile + gridDim.x);
+    }
+    mma_wait(mph);
+    float z[HH], r[HH];
+    {
+      float az[HH], ar[HH], rh[HH];
+      tmem_row_load<HH>(tm + 8 * H, c0, az);
+      tmem_row_load<HH>(tm + 9 * H, c0, ar);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        z[j] = sigm(az[j] + __ldg(l + c0 + j));
+        r[j] = sigm(ar[j] + __ldg(l + H + c0 + j));
+        rh[j] = r[j] * h[j];
+      }
+      tmem_st_split<HH>(tq + 10 * H + c0, tq + 11 * H + c0, rh);
+      sync_tmem();
+      if (threadIdx.x == 0) {                           // P2
+        tc::fence_after();
+        const uint32_t hh_ = tc::smem_u32(bh_hi), hl = tc::smem_u32(bh_lo);
+        mma_ts_seg(tm + 12 * H, tm + 6 * H, tm + 7 * H, hh_, hl, 2 * H, 0, H, id_h, true);
+        mma_ts_seg(tm + 12 * H, tm + 10 * H, tm + 11 * H, hh_, hl, 2 * H, H, H, id_h, false);
+        tc::commit(&mma_bar);
+      }
+      stage_flush<HH>(stage, rh, 1.0f, RHo + c0, H, wr0, wnv);            // RH (for dL_h²), overlaps P2
+    }
+    mma_wait(mph);
+    float dh[HH];
+    {
+      float ah[HH], dah[HH], daz[HH];
+      tmem_row_load<HH>(tm + 12 * H, c0, ah);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        const float hh = tanhf(ah[j] + __ldg(l + 2 * H + c0 + j));
+        const float dZ = g[j] * (h[j] - hh), dHh = g[j] * (1.0f - z[j]);
+        dah[j] = dHh * (1.0f - hh * hh);
+        daz[j] = dZ * z[j] * (1.0f - z[j]);
+        dh[j] = g[j] * z[j];
+      }
+      // P1/P2 operands are consumed: reuse [0,4H) for da_h, da_z
+      tmem_st_split<HH>(tq + c0, tq + H + c0, dah);
+      tmem_st_split<HH>(tq + 2 * H + c0, tq + 3 * H + c0, daz);
+      sync_tmem();
+      if (threadIdx.x == 0) {                           // P3
+        tc::fence_after();
+        mma_ts_seg(tm + 4 * H, tm + 0, tm + H, tc::smem_u32(lh_hi), tc::smem_u32(lh_lo), H, 0, H, id_2h, true);
+        mma_ts_seg(tm + 6 * H, tm + 2 * H, tm + 3 * H, tc::smem_u32(lz_hi), tc::smem_u32(lz_lo), H, 0, H, id_2h, true);
+        tc::commit(&mma_bar);
+      }
+      stage_flush<HH>(stage, daz, 1.0f, da + c0, H3, wr0, wnv);            // da_z
+      stage_flush<HH>(stage, dah, 1.0f, da + 2 * H + c0, H3, wr0, wnv);    // da_h
+    }
+    mma_wait(mph);
+    {
+      float dch[HH], drh[HH], dar[HH];
+      tmem_row_load<HH>(tm + 4 * H, c0, dch);          // dC_h
+      tmem_row_load<HH>(tm + 5 * H, c0, drh);          // dRH
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        dh[j] += drh[j] * r[j];
+        dar[j] = drh[j] * h[j] * r[j] * (1.0f - r[j]);
+      }
+      tmem_st_split<HH>(tq + 10 * H + c0, tq + 11 * H + c0, dar);
+      sync_tmem();
+      if (threadIdx.x == 0) {                           // P4
+        tc::fence_after();
+        mma_ts_seg(tm + 8 * H, tm + 10 * H, tm + 11 * H, tc::smem_u32(lr_hi), tc::smem_u32(lr_lo), H, 0, H, id_2h, true);
+        tc::commit(&mma_bar);
+      }
+      stage_flush<HH>(stage, dch, nd, dCs + 2 * H + c0, H3, wr0, wnv);     // dC'_h
+      stage_flush<HH>(stage, dar, 1.0f, da + H + c0, H3, wr0, wnv);        // da_r
+      float dcz[HH], dhz[HH];
+      tmem_row_load<HH>(tm + 6 * H, c0, dcz);          // dC_z
+      tmem_row_load<HH>(tm + 7 * H, c0, dhz);          // dH_z
+#pragma unroll
+      for (int j = 0; j < HH; ++j) dh[j] += dhz[j];
+      stage_flush<HH>(stage, dcz, nd, dCs + c0, H3, wr0, wnv);             // dC'_z
+    }
+    mma_wait(mph);
+    {
+      float dcr[HH], dhr[HH];
+      tmem_row_load<HH>(tm + 8 * H, c0, dcr);          // dC_r
+      tmem_row_load<HH>(tm + 9 * H, c0, dhr);          // dH_r
+#pragma unroll
+      for (int j = 0; j < HH; ++j) dh[j] += dhr[j];
+      stage_flush<HH>(stage, dcr, nd, dCs + H + c0, H3, wr0, wnv);         // dC'_r
+      stage_flush<HH>(stage, dh, 1.0f, dHp + c0, H, wr0, wnv);             // dH_prev
+    }
+    tc::fence_before();
+    __syncthreads();                                   // TMEM / stage reuse by the next tile
+  }
+  if (warp == 0) tc::tmem_free(tm, G::TCOLS);
 }
 
 // ------------------------------------------------------------------ Σ_rows Aᵀ·B
@@ -989,12 +1234,15 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
                       cudaStream_t s) {
   const int ntiles = (V + 127) / 128;
   const int nb = std::min(ntiles, num_sms());
+  CUtensorMap tmC, tmH;
+  STG_TRY(make_tmap_f32(&tmC, C, (uint64_t)V, 3 * H, 3 * H, 32, 128));
+  STG_TRY(make_tmap_f32(&tmH, Hp, (uint64_t)V, H, H, 32, 128));
   if (H == 32) {
     STG_TRY(prep(k_tc_gru_fwd2<32>, GruF2<32>::SMEM));
-    k_tc_gru_fwd2<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, C, Hp, L, l, Hn);
+    k_tc_gru_fwd2<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, Hn);
   } else {
     STG_TRY(prep(k_tc_gru_fwd2<16>, GruF2<16>::SMEM));
-    k_tc_gru_fwd2<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, C, Hp, L, l, Hn);
+    k_tc_gru_fwd2<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, Hn);
   }
   count_launch();
   return check_launch("tc_gru_fwd");
@@ -1003,16 +1251,17 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
 stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float* G, const float* L, const float* l,
                       const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s) {
   const int ntiles = (V + 127) / 128;
+  const int nb = std::min(ntiles, num_sms());
+  CUtensorMap tmC, tmH, tmG;
+  STG_TRY(make_tmap_f32(&tmC, C, (uint64_t)V, 3 * H, 3 * H, 32, 128));
+  STG_TRY(make_tmap_f32(&tmH, Hp, (uint64_t)V, H, H, 32, 128));
+  STG_TRY(make_tmap_f32(&tmG, G, (uint64_t)V, H, H, 32, 128));
   if (H == 32) {
-    const size_t smem = 12 * GruSmem<32>::BG + 2 * GruSmem<32>::A1;
-    STG_TRY(prep(k_tc_gru_bwd<32>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_bwd<32>, smem, kGruThreads));
-    k_tc_gru_bwd<32><<<nb, kGruThreads, smem, s>>>(V, C, Hp, G, L, l, ndst, dCs, dHp, da, RH);
+    STG_TRY(prep(k_tc_gru_bwd2<32>, GruB2<32>::SMEM));
+    k_tc_gru_bwd2<32><<<nb, 256, GruB2<32>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, dCs, dHp, da, RH);
   } else {
-    const size_t smem = 12 * GruSmem<16>::BG + 2 * GruSmem<16>::A1;
-    STG_TRY(prep(k_tc_gru_bwd<16>, smem));
-    const int nb = std::min(ntiles, occupancy_blocks(k_tc_gru_bwd<16>, smem, kGruThreads));
-    k_tc_gru_bwd<16><<<nb, kGruThreads, smem, s>>>(V, C, Hp, G, L, l, ndst, dCs, dHp, da, RH);
+    STG_TRY(prep(k_tc_gru_bwd2<16>, GruB2<16>::SMEM));
+    k_tc_gru_bwd2<16><<<nb, 256, GruB2<16>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, dCs, dHp, da, RH);
   }
   count_launch();
   return check_launch("tc_gru_bwd");
