@@ -419,8 +419,9 @@ def stg_partition_rows(V: int, in_rowptr: torch.Tensor, world: int, stream=None)
 
 def stg_debug_tc_gemm(mode: int, A: torch.Tensor, B: torch.Tensor, stream=None) -> torch.Tensor:
     """mode 0: A[M,K]·B[K,N]; mode 1: Aᵀ·B with A[R,128], B[R,N] (tcgen05 3xTF32);
-    mode 2: as 0 with A in tensor memory; mode 3: one unsplit tf32 pass of A·B."""
-    if mode != 1:
+    mode 2: as 0 with A in tensor memory; mode 3: one unsplit tf32 pass of A·B;
+    mode 4: as 1 with TMA-loaded MN-major (SWIZZLE_128B_BASE32B) operands."""
+    if mode not in (1, 4):
         M, K = A.shape
         N = B.shape[1]
         C = torch.empty(M, N, device=A.device)
@@ -429,7 +430,7 @@ def stg_debug_tc_gemm(mode: int, A: torch.Tensor, B: torch.Tensor, stream=None) 
         R = A.shape[0]
         N = B.shape[1]
         C = torch.empty(128, N, device=A.device)
-        _check(_lib.stg_debug_tc_gemm(1, 128, N, 0, R, _ptr(A), _ptr(B), _ptr(C), _stream(stream)))
+        _check(_lib.stg_debug_tc_gemm(mode, 128, N, 0, R, _ptr(A), _ptr(B), _ptr(C), _stream(stream)))
     return C
 
 

@@ -88,9 +88,10 @@ int num_sms();
 
 // 2-D TMA descriptor of a row-major fp32 matrix [rows × cols] (row stride ld
 // elements, 16-byte aligned), box [box_rows × box_cols] with 128-byte swizzle
-// (box_cols·4 <= 128).  Encoded through the driver entry point (no libcuda link).
+// (box_cols·4 <= 128; atom32: 32-byte swizzle atoms = the UMMA MN-major
+// SWIZZLE_128B_BASE32B layout).  Encoded through the driver entry point.
 stg_status make_tmap_f32(CUtensorMap* out, const float* base, uint64_t rows, uint64_t cols, uint64_t ld,
-                         uint32_t box_cols, uint32_t box_rows);
+                         uint32_t box_cols, uint32_t box_rows, bool atom32 = false);
 
 // ---------------------------------------------------------------- profiler
 // Per-phase device time with CUDA events on the launching stream (bench.py and

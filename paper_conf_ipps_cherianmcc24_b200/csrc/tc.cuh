@@ -35,6 +35,19 @@ __device__ __forceinline__ uint64_t desc(uint32_t saddr, uint32_t lbo, uint32_t 
   return d;
 }
 
+// SM100 descriptor of an MN-major operand in the SWIZZLE_128B_BASE32B layout
+// (layout type 1): 128-byte rows of 32 tf32 along M/N, K = rows; atoms of 4
+// K-rows (SBO = 512 B apart along K), 32-element M/N chunks LBO bytes apart.
+__device__ __forceinline__ uint64_t desc_mn_sw128_32b(uint32_t saddr, uint32_t lbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)((512u >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)1 << 61;
+  return d;
+}
+
 // Instruction descriptor: kind::tf32, D fp32, A/B tf32, dense.
 __host__ __device__ constexpr uint32_t idesc_tf32(int M, int N, int a_mn, int b_mn) {
   return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |

@@ -8,6 +8,9 @@
 //   mode 3: ONE tf32 MMA on unsplit fp32 operands (A raw · B raw): the test
 //           compares it with truncated and rounded tf32 products to pin the
 //           hardware's fp32 -> tf32 input conversion
+//   mode 4: as mode 1 (Xᵀ·Y, X[R,128], Y[R,N]) with both operands loaded by 2-D
+//           TMA boxes (128 rows x 32 fp32) in the MN-major SWIZZLE_128B_BASE32B
+//           layout (k_tc_debug_mn: no transposition by threads; hi = raw)
 #include "common.cuh"
 #include "tc.cuh"
 
@@ -148,6 +151,76 @@ __global__ void __launch_bounds__(128) k_tc_debug(int mode, int M, int N, int K,
   (void)M;
 }
 
+// mode 4: D[128 x N] += Xᵀ Y over R rows in 128-row tiles, A/B MN-major (TMA).
+__global__ void __launch_bounds__(128) k_tc_debug_mn(int N, int R, const __grid_constant__ CUtensorMap tmX,
+                                                     const __grid_constant__ CUtensorMap tmY, float* __restrict__ C) {
+  extern __shared__ unsigned char sm_raw[];
+  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t full, mbar;
+  __shared__ uint32_t tslot;
+  constexpr int BOX = 128 * 32 * 4;
+  const int nby = N / 32;
+  unsigned char* xh = sm;                       // 4 boxes
+  unsigned char* xl = sm + 4 * BOX;
+  unsigned char* yh = sm + 8 * BOX;             // nby boxes
+  unsigned char* yl = yh + nby * BOX;
+  const int warp = threadIdx.x >> 5;
+  uint32_t ncols = 32;
+  while ((int)ncols < N) ncols <<= 1;
+  if (warp == 0) tc::tmem_alloc(&tslot, ncols);
+  if (threadIdx.x == 0) { tc::mbar_init(&full, 1); tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  const uint32_t idesc = tc::idesc_tf32(128, N, 1, 1);
+  for (int t = 0; t < R / 128; ++t) {
+    if (threadIdx.x == 0) {
+      tc::mbar_expect_tx(&full, (uint32_t)(4 + nby) * BOX);
+      for (int k = 0; k < 4; ++k) tc::tma_load_2d(xh + k * BOX, &tmX, 32 * k, 128 * t, &full);
+      for (int k = 0; k < nby; ++k) tc::tma_load_2d(yh + k * BOX, &tmY, 32 * k, 128 * t, &full);
+    }
+    tc::mbar_wait(&full, t & 1);
+    // lo = raw - trunc(raw), elementwise over the (identically laid out) boxes
+    for (int e = threadIdx.x; e < (4 + nby) * BOX / 16; e += 128) {
+      const int which = e < 4 * BOX / 16 ? 0 : 1;
+      const int o = which ? e - 4 * BOX / 16 : e;
+      const float4 v = reinterpret_cast<const float4*>(which ? yh : xh)[o];
+      reinterpret_cast<float4*>(which ? yl : xl)[o] =
+          make_float4(v.x - tc::tf32_hi(v.x), v.y - tc::tf32_hi(v.y), v.z - tc::tf32_hi(v.z), v.w - tc::tf32_hi(v.w));
+    }
+    tc::fence_proxy_async();
+    tc::fence_before();
+    __syncthreads();
+    tc::fence_after();
+    if (threadIdx.x == 0) {
+      for (int k = 0; k < 128; k += 8) {               // 8 K-rows (1024 B) per MMA
+        const uint32_t o = (uint32_t)k * 128;
+        const uint64_t ah = tc::desc_mn_sw128_32b(tc::smem_u32(xh) + o, BOX), al = tc::desc_mn_sw128_32b(tc::smem_u32(xl) + o, BOX);
+        const uint64_t bh = tc::desc_mn_sw128_32b(tc::smem_u32(yh) + o, BOX), bl = tc::desc_mn_sw128_32b(tc::smem_u32(yl) + o, BOX);
+        tc::mma_tf32(tm, al, bh, idesc, (t > 0 || k > 0) ? 1u : 0u);
+        tc::mma_tf32(tm, ah, bl, idesc, 1u);
+        tc::mma_tf32(tm, ah, bh, idesc, 1u);
+      }
+      tc::commit(&mbar);
+    }
+    tc::mbar_wait(&mbar, t & 1);
+    tc::fence_after();
+    __syncthreads();
+  }
+  const int r = warp * 32 + (threadIdx.x & 31);
+  for (int c = 0; c < N; c += 8) {
+    float v[8];
+    tc::tmem_ld8(tm + ((uint32_t)(warp * 32) << 16) + (uint32_t)c, v);
+    tc::tmem_wait_ld();
+#pragma unroll
+    for (int i = 0; i < 8; ++i) C[(int64_t)r * N + c + i] = v[i];
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 0) tc::tmem_free(tm, ncols);
+}
+
 }  // namespace
 }  // namespace stg
 
@@ -155,7 +228,18 @@ extern "C" stg_status stg_debug_tc_gemm(int32_t mode, int32_t M, int32_t N, int3
                                         const float* B, float* C, stg_stream_t stream) {
   using namespace stg;
   if (N % 16 || N < 16 || N > 256) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: N=%d", N);
-  if (mode < 0 || mode > 3) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: mode=%d", mode);
+  if (mode < 0 || mode > 4) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: mode=%d", mode);
+  if (mode == 4) {
+    if (R % 128 || N % 32) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: mode 4 needs R %% 128 == 0, N %% 32 == 0");
+    CUtensorMap tx, ty;
+    STG_TRY(make_tmap_f32(&tx, A, (uint64_t)R, 128, 128, 32, 128, true));
+    STG_TRY(make_tmap_f32(&ty, B, (uint64_t)R, (uint64_t)N, (uint64_t)N, 32, 128, true));
+    const size_t smem = (size_t)2 * (4 + N / 32) * 128 * 32 * 4 + 1024;
+    STG_CUDA(cudaFuncSetAttribute(k_tc_debug_mn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    k_tc_debug_mn<<<1, 128, smem, (cudaStream_t)stream>>>(N, R, tx, ty, C);
+    count_launch();
+    return check_launch("stg_debug_tc_gemm mode 4");
+  }
   if (mode != 1 && (M % 128 || K % 8 || K < 8 || K > 256)) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: M/K");
   if (mode == 2 && K > 128) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: K > 128 for TMEM A");
   if (mode == 1 && (R % 32 || R < 32)) return fail(STG_ERR_INVALID_ARG, "stg_debug_tc_gemm: R");

@@ -19,6 +19,7 @@
 #include <cstdlib>
 #include <map>
 #include <mutex>
+#include <vector>
 
 #include "common.cuh"
 #include "tc.cuh"
@@ -1126,6 +1127,168 @@ __global__ void __launch_bounds__(kAtbThreads, 1) k_tc_atb(const AtbArgs p) {
   if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
 }
 
+// ------------------------------------------------------------------ Σ_rows Aᵀ·B, v2 (TMA, MN-major)
+// D_a[128 x N] = Σ_r A_a[r,:]ᵀ B[r,:] for one or two A operands, both operands
+// loaded by 2-D TMA boxes (RT rows x 32 fp32) straight into the UMMA MN-major
+// SWIZZLE_128B_BASE32B layout (K = rows; pinned by tests/test_gpu_tc.py mode 4):
+// no transposition by threads; hi = the raw fp32 (hardware truncation) and
+// lo = x - trunc(x) is computed in place, elementwise, by 4 converter warps.
+// Each A operand is 4 feature boxes (M = 128): TMA boxes, an optional static
+// "ones" box (1.0 in feature 0 of every row: the Σ_rows term of dl) and zero
+// boxes.  Warp 0 issues the TMA, warp 1 the MMAs, warps 2-5 convert and run
+// the epilogue; a 2-stage ring overlaps loads, conversion and MMAs.  Each CTA
+// accumulates its tiles (grid-stride, fixed) in TMEM and writes its partial;
+// k_tc_sum_parts adds the partials in a fixed order (deterministic).
+constexpr int kAtbRT = 32;                        // rows per tile
+constexpr int kAtbBox = kAtbRT * 32 * 4;          // 4 KB per box
+constexpr int kAtbStages = 2;
+
+struct AtbSpec2 {
+  int V;
+  int na;                 // 1 or 2 A operands
+  int src_map[2][4];      // per A operand and feature box: tensor map 0..3, or -1 zero, -2 ones (m_ones)
+  int src_col[2][4];
+  int nb;                 // B boxes (N = 32 nb), from map b_map at columns 32 k
+  int b_map;
+  float* part;            // [gridDim][na][128][N]
+};
+
+template <int NB>
+__global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUtensorMap m0,
+                                                    const __grid_constant__ CUtensorMap m1,
+                                                    const __grid_constant__ CUtensorMap m2,
+                                                    const __grid_constant__ CUtensorMap m3,
+                                                    const __grid_constant__ CUtensorMap m_ones, const AtbSpec2 sp) {
+  constexpr int N = 32 * NB;
+  extern __shared__ unsigned char sm_raw[];
+  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t full[kAtbStages], conv[kAtbStages], empty[kAtbStages], done, init_bar;
+  __shared__ uint32_t tslot;
+  const int na = sp.na;
+  const int nbox = 4 * na + NB;                    // boxes per stage (A boxes, then B boxes)
+  const size_t half = (size_t)nbox * kAtbBox;      // hi region of a stage; lo follows
+  auto hi = [&](int st, int bx) { return sm + (size_t)st * 2 * half + (size_t)bx * kAtbBox; };
+  auto lo = [&](int st, int bx) { return sm + (size_t)st * 2 * half + half + (size_t)bx * kAtbBox; };
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const CUtensorMap* maps[4] = {&m0, &m1, &m2, &m3};
+  // zero every stage once (zero / ones slots are never written by the ring)
+  for (size_t e = threadIdx.x; e < (size_t)kAtbStages * 2 * half / 16; e += blockDim.x)
+    reinterpret_cast<float4*>(sm)[e] = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (warp == 1) tc::tmem_alloc(&tslot, na * N <= 128 ? 128 : 256);
+  if (threadIdx.x == 0) {
+    for (int st = 0; st < kAtbStages; ++st) {
+      tc::mbar_init(&full[st], 1); tc::mbar_init(&conv[st], 128); tc::mbar_init(&empty[st], 1);
+    }
+    tc::mbar_init(&done, 1); tc::mbar_init(&init_bar, 1);
+    tc::fence_mbar_init();
+  }
+  tc::fence_proxy_async();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  // "ones" boxes: TMA the ones tile (laid out by the hardware's own swizzle) into each stage
+  int n_ones = 0;
+  for (int a = 0; a < na; ++a)
+    for (int k = 0; k < 4; ++k) n_ones += sp.src_map[a][k] == -2;
+  if (n_ones) {
+    if (threadIdx.x == 0) {
+      tc::mbar_expect_tx(&init_bar, (uint32_t)(n_ones * kAtbStages * kAtbBox));
+      for (int st = 0; st < kAtbStages; ++st)
+        for (int a = 0; a < na; ++a)
+          for (int k = 0; k < 4; ++k)
+            if (sp.src_map[a][k] == -2) tc::tma_load_2d(hi(st, 4 * a + k), &m_ones, 0, 0, &init_bar);
+    }
+    tc::mbar_wait(&init_bar, 0);
+  }
+  const uint32_t tm = tslot;
+  const int ntiles = (sp.V + kAtbRT - 1) / kAtbRT;
+  int my_tiles = 0;
+  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) ++my_tiles;
+  if (warp == 0) {                                   // ---- TMA producer
+    if (lane == 0) {
+      int bytes = NB * kAtbBox;
+      for (int a = 0; a < na; ++a)
+        for (int k = 0; k < 4; ++k) bytes += sp.src_map[a][k] >= 0 ? kAtbBox : 0;
+      for (int i = 0; i < my_tiles; ++i) {
+        const int st = i % kAtbStages, kk = i / kAtbStages, r0 = (blockIdx.x + i * gridDim.x) * kAtbRT;
+        if (kk > 0) tc::mbar_wait(&empty[st], (kk - 1) & 1);
+        tc::mbar_expect_tx(&full[st], (uint32_t)bytes);
+        for (int a = 0; a < na; ++a)
+          for (int k = 0; k < 4; ++k)
+            if (sp.src_map[a][k] >= 0) tc::tma_load_2d(hi(st, 4 * a + k), maps[sp.src_map[a][k]], sp.src_col[a][k], r0, &full[st]);
+        for (int k = 0; k < NB; ++k) tc::tma_load_2d(hi(st, 4 * na + k), maps[sp.b_map], 32 * k, r0, &full[st]);
+      }
+    }
+  } else if (warp == 1) {                            // ---- MMA issuer
+    if (lane == 0) {
+      const uint32_t idesc = tc::idesc_tf32(128, N, 1, 1);
+      for (int i = 0; i < my_tiles; ++i) {
+        const int st = i % kAtbStages, kk = i / kAtbStages;
+        tc::mbar_wait(&conv[st], kk & 1);
+        tc::fence_after();
+        const uint32_t bh = tc::smem_u32(hi(st, 4 * na)), bl = tc::smem_u32(lo(st, 4 * na));
+        for (int a = 0; a < na; ++a) {
+          const uint32_t ah = tc::smem_u32(hi(st, 4 * a)), al = tc::smem_u32(lo(st, 4 * a));
+          for (int k = 0; k < kAtbRT; k += 8) {            // 8 K-rows (1024 B) per MMA
+            const uint32_t o = (uint32_t)k * 128;
+            const uint64_t dah = tc::desc_mn_sw128_32b(ah + o, kAtbBox), dal = tc::desc_mn_sw128_32b(al + o, kAtbBox);
+            const uint64_t dbh = tc::desc_mn_sw128_32b(bh + o, kAtbBox), dbl = tc::desc_mn_sw128_32b(bl + o, kAtbBox);
+            const uint32_t d = tm + a * N;
+            tc::mma_tf32(d, dal, dbh, idesc, (i > 0 || k > 0) ? 1u : 0u);
+            tc::mma_tf32(d, dah, dbl, idesc, 1u);
+            tc::mma_tf32(d, dah, dbh, idesc, 1u);
+          }
+        }
+        tc::commit(&empty[st]);
+      }
+      tc::commit(&done);
+    }
+  } else {                                           // ---- converters (warps 2-5), then epilogue
+    const int ct = threadIdx.x - 64;
+    for (int i = 0; i < my_tiles; ++i) {
+      const int st = i % kAtbStages;
+      tc::mbar_wait(&full[st], (i / kAtbStages) & 1);
+      for (int a = 0; a <= na; ++a) {
+        const int b0 = a < na ? 4 * a : 4 * na, nbx = a < na ? 4 : NB;
+        for (int bx = 0; bx < nbx; ++bx) {
+          if (a < na && sp.src_map[a][bx] < 0) continue;     // zero / ones: lo stays 0
+          const float4* src = reinterpret_cast<const float4*>(hi(st, b0 + bx));
+          float4* dst = reinterpret_cast<float4*>(lo(st, b0 + bx));
+#pragma unroll 4
+          for (int e = ct; e < kAtbBox / 16; e += 128) {
+            const float4 v = src[e];
+            dst[e] = make_float4(v.x - tc::tf32_hi(v.x), v.y - tc::tf32_hi(v.y), v.z - tc::tf32_hi(v.z),
+                                 v.w - tc::tf32_hi(v.w));
+          }
+        }
+      }
+      tc::fence_proxy_async();
+      tc::mbar_arrive(&conv[st]);
+    }
+    // epilogue: this warp reads TMEM lane quarter warp % 4
+    tc::mbar_wait(&done, 0);
+    tc::fence_after();
+    const int q = warp & 3, row = q * 32 + lane;
+    float* out = sp.part + (size_t)blockIdx.x * na * 128 * N;
+    for (int c = 0; c < na * N; c += 8) {
+      float v[8];
+      if (my_tiles == 0) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = 0.f;
+      } else {
+        tc::tmem_ld8(tm + ((uint32_t)(q * 32) << 16) + (uint32_t)c, v);
+        tc::tmem_wait_ld();
+      }
+      const int a = c / N, cc = c % N;
+#pragma unroll
+      for (int e = 0; e < 8; ++e) out[(size_t)a * 128 * N + (size_t)row * N + cc + e] = v[e];
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 1) tc::tmem_free(tm, na * N <= 128 ? 128 : 256);
+}
+
 // Fixed-order sum of the per-CTA partials: tot[e] = Σ_b part[b][e] (blocks of 16).
 __global__ void k_tc_sum_parts(const float* __restrict__ part, int nb, int n, float* __restrict__ tot) {
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
@@ -1140,29 +1303,32 @@ __global__ void k_tc_sum_parts(const float* __restrict__ part, int nb, int n, fl
   }
 }
 
-// Scatter the dL / dl / db pieces out of tot = [D1 (128 × 3H) | D2 (128 × 3H)]:
-//   D1 rows: C_z | C_r | C_h | H,  D2 rows: RH | ones;  columns da_z | da_r | da_h
-__global__ void k_dl_scatter(int H, const float* __restrict__ tot, const float* __restrict__ L,
-                             float* __restrict__ dL, float* __restrict__ dl, float* __restrict__ db) {
-  const int H3 = 3 * H, LG = 2 * H * H;
+// Scatter the dL / dl / db pieces out of tot = [D1 (128 × ldd) | D2 (128 × ldd)]
+// (row = A feature, column = da feature: da_z | da_r | da_h, ldd >= 3H):
+//   D1 rows: C_z | C_r | C_h (rows 0..3H) | H (rows hoff..hoff+H),
+//   D2 rows: RH (rows 0..H) | ones (row orow).
+__global__ void k_dl_scatter(int H, int hoff, int orow, int ldd, const float* __restrict__ tot,
+                             const float* __restrict__ L, float* __restrict__ dL, float* __restrict__ dl,
+                             float* __restrict__ db) {
+  const int LG = 2 * H * H;
   const float* D1 = tot;
-  const float* D2 = tot + 128 * H3;
+  const float* D2 = tot + 128 * ldd;
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < 6 * H * H + 6 * H; e += gridDim.x * blockDim.x) {
     if (e < 6 * H * H) {
       const int g = e / LG, rem = e % LG, i = rem / H, j = rem % H;
       float v;
-      if (i < H) v = D1[(g * H + i) * H3 + g * H + j];                 // C_gᵀ da_g
-      else if (g < 2) v = D1[(3 * H + i - H) * H3 + g * H + j];       // Hᵀ da_z, Hᵀ da_r
-      else v = D2[(i - H) * H3 + 2 * H + j];                          // RHᵀ da_h
+      if (i < H) v = D1[(g * H + i) * ldd + g * H + j];                // C_gᵀ da_g
+      else if (g < 2) v = D1[(hoff + i - H) * ldd + g * H + j];       // Hᵀ da_z, Hᵀ da_r
+      else v = D2[(i - H) * ldd + 2 * H + j];                         // RHᵀ da_h
       dL[e] += v;
     } else if (e < 6 * H * H + 3 * H) {
       const int c = e - 6 * H * H;
-      dl[c] += D2[H * H3 + c];                                        // ones row: Σ_rows da
+      dl[c] += D2[orow * ldd + c];                                    // ones row: Σ_rows da
     } else {
       const int c = e - 6 * H * H - 3 * H, g = c / H, i = c % H;      // db_g = dl_g · L_g¹ᵀ
       const float* Lg = L + (int64_t)g * LG;
       float s = 0.f;
-      for (int j = 0; j < H; ++j) s = fmaf(D2[H * H3 + g * H + j], Lg[i * H + j], s);
+      for (int j = 0; j < H; ++j) s = fmaf(D2[orow * ldd + g * H + j], Lg[i * H + j], s);
       db[c] += s;
     }
   }
@@ -1283,48 +1449,91 @@ static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
   return check_launch("tc_atb");
 }
 
-// dW[f][c] += Σ_v X[v,f]·dP[v,c]  via D = dPᵀ·X  ([3H pad 128] × roundup16(F)).
+template <int NB>
+static stg_status atb2_launch(const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb_out,
+                              cudaStream_t s) {
+  const int nbox = 4 * sp.na + NB;
+  const size_t smem = (size_t)kAtbStages * 2 * nbox * kAtbBox + 1024;
+  STG_CUDA(cudaFuncSetAttribute(k_tc_atb2<NB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int ntiles = (sp.V + kAtbRT - 1) / kAtbRT;
+  const int nb = std::max(1, std::min(ntiles, tc_atb_max_blocks()));
+  k_tc_atb2<NB><<<nb, 192, smem, s>>>(m[0], m[1], m[2], m[3], ones, sp);
+  count_launch();
+  *nb_out = nb;
+  return check_launch("tc_atb2");
+}
+
+static stg_status atb2_dispatch(int NB, const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb,
+                                cudaStream_t s) {
+  switch (NB) {
+    case 1: return atb2_launch<1>(m, ones, sp, nb, s);
+    case 2: return atb2_launch<2>(m, ones, sp, nb, s);
+    case 3: return atb2_launch<3>(m, ones, sp, nb, s);
+    case 4: return atb2_launch<4>(m, ones, sp, nb, s);
+    default: return fail(STG_ERR_INVALID_ARG, "atb2: %d B boxes", NB);
+  }
+}
+
+// the [kAtbRT x 32] "ones" tile (1.0 in column 0): the Σ_rows feature of dl
+static stg_status ones_map(CUtensorMap* out, cudaStream_t s) {
+  static float* d = nullptr;
+  if (!d) {
+    std::vector<float> h((size_t)kAtbRT * 32, 0.f);
+    for (int r = 0; r < kAtbRT; ++r) h[(size_t)r * 32] = 1.f;
+    if (cudaMalloc(&d, h.size() * sizeof(float)) != cudaSuccess) return fail(STG_ERR_NO_MEMORY, "ones tile");
+    STG_CUDA(cudaMemcpy(d, h.data(), h.size() * sizeof(float), cudaMemcpyHostToDevice));
+  }
+  (void)s;
+  return make_tmap_f32(out, d, kAtbRT, 32, 32, 32, kAtbRT, true);
+}
+
+// dW[f][c] += Σ_v X[v,f]·dP[v,c]  via D = dPᵀ·X  (M = 128 features of dP, N = 32·ceil(F/32)).
 // part: tc_atb_max_blocks() · 2 · 128 · 128 floats; tot: 2 · 128 · 128 floats.
 stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* tot, float* dW,
                  cudaStream_t s) {
-  AtbArgs a{};
-  a.V = V; a.A1 = dP; a.lda1 = 3 * H; a.FA1 = 3 * H; a.B = X; a.ldb = F; a.FB = F; a.part = part;
+  const int H3 = 3 * H, NB = (F + 31) / 32, N = 32 * NB;
+  CUtensorMap m[4], ones;
+  STG_TRY(make_tmap_f32(&m[0], dP, (uint64_t)V, H3, H3, 32, kAtbRT, true));
+  STG_TRY(make_tmap_f32(&m[1], X, (uint64_t)V, F, F, 32, kAtbRT, true));
+  m[2] = m[0]; m[3] = m[0];
+  STG_TRY(ones_map(&ones, s));
+  AtbSpec2 sp{};
+  sp.V = V; sp.na = 1; sp.nb = NB; sp.b_map = 1; sp.part = part;
+  for (int k = 0; k < 4; ++k) { sp.src_map[0][k] = 32 * k < H3 ? 0 : -1; sp.src_col[0][k] = 32 * k; }
   int nb = 0;
-  const int Np = (F + 15) / 16 * 16;
-  switch (Np) {
-    case 16: STG_TRY((atb<16, 1>(a, &nb, s))); break;
-    case 32: STG_TRY((atb<32, 1>(a, &nb, s))); break;
-    case 48: STG_TRY((atb<48, 1>(a, &nb, s))); break;
-    case 64: STG_TRY((atb<64, 1>(a, &nb, s))); break;
-    case 96: STG_TRY((atb<96, 1>(a, &nb, s))); break;
-    case 128: STG_TRY((atb<128, 1>(a, &nb, s))); break;
-    default: return fail(STG_ERR_INVALID_ARG, "tc_dw: F=%d", F);
-  }
-  const int n = 128 * Np;
+  STG_TRY(atb2_dispatch(NB, m, ones, sp, &nb, s));
+  const int n = 128 * N;
   k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
-  k_dw_scatter<<<(F * 3 * H + 255) / 256, 256, 0, s>>>(F, 3 * H, Np, tot, dW);
+  k_dw_scatter<<<(F * H3 + 255) / 256, 256, 0, s>>>(F, H3, N, tot, dW);
   count_launch(2);
   return check_launch("tc_dw");
 }
 
-// dL, dl, db from C, H, RH, da (see k_tc_gru_bwd) with ONE reduction kernel:
-//   D1 = [C_z|C_r|C_h|H]ᵀ·da,  D2 = [RH|1]ᵀ·da  (da = [da_z|da_r|da_h]).
+// dL, dl, db from C, H, RH, da (see k_tc_gru_bwd2) with ONE reduction kernel:
+//   D1 = [C_z|C_r|C_h | H]ᵀ·da  (C in feature boxes 0.., H at feature 32·ceil(3H/32)),
+//   D2 = [RH | ones]ᵀ·da        (RH features 0..H, the ones feature at 32).
 stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
                  float* tot, float* dL, float* dl, float* db, const float* L, cudaStream_t s) {
-  const int H3 = 3 * H;
-  AtbArgs a{};
-  a.V = V;
-  a.A1 = C; a.lda1 = H3; a.FA1 = H3;
-  a.A2 = Hp; a.lda2 = H; a.FA2 = H;
-  a.A3 = RH; a.lda3 = H; a.FA3 = H; a.ones = 1;
-  a.B = da; a.ldb = H3; a.FB = H3;
-  a.part = part;
+  const int H3 = 3 * H, NBC = (H3 + 31) / 32;
+  CUtensorMap m[4], ones;
+  STG_TRY(make_tmap_f32(&m[0], C, (uint64_t)V, H3, H3, 32, kAtbRT, true));
+  STG_TRY(make_tmap_f32(&m[1], Hp, (uint64_t)V, H, H, 32, kAtbRT, true));
+  STG_TRY(make_tmap_f32(&m[2], RH, (uint64_t)V, H, H, 32, kAtbRT, true));
+  STG_TRY(make_tmap_f32(&m[3], da, (uint64_t)V, H3, H3, 32, kAtbRT, true));
+  STG_TRY(ones_map(&ones, s));
+  AtbSpec2 sp{};
+  sp.V = V; sp.na = 2; sp.nb = NBC; sp.b_map = 3; sp.part = part;
+  for (int k = 0; k < 4; ++k) {
+    sp.src_map[0][k] = k < NBC ? 0 : (k == NBC ? 1 : -1);
+    sp.src_col[0][k] = k < NBC ? 32 * k : 0;
+    sp.src_map[1][k] = k == 0 ? 2 : (k == 1 ? -2 : -1);
+    sp.src_col[1][k] = 0;
+  }
   int nb = 0;
-  if (H == 32) STG_TRY((atb<96, 2>(a, &nb, s)));
-  else STG_TRY((atb<48, 2>(a, &nb, s)));
-  const int n = 2 * 128 * H3;
+  STG_TRY(atb2_dispatch(NBC, m, ones, sp, &nb, s));
+  const int N = 32 * NBC, n = 2 * 128 * N;
   k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
-  k_dl_scatter<<<(6 * H * H + 6 * H + 255) / 256, 256, 0, s>>>(H, tot, L, dL, dl, db);
+  k_dl_scatter<<<(6 * H * H + 6 * H + 255) / 256, 256, 0, s>>>(H, N, 32, N, tot, L, dL, dl, db);
   count_launch(2);
   return check_launch("tc_dl");
 }

@@ -68,3 +68,15 @@ def test_tf32_input_conversion(stg):
     e_rna = np.max(np.abs(C - _tf32_rna(A) @ _tf32_rna(B)) / cond)
     print("tf32 conversion: err vs truncation %.3g, vs round-nearest %.3g" % (e_trunc, e_rna))
     assert e_trunc < 1e-6 and e_rna > 1e-5, (e_trunc, e_rna)
+
+
+@pytest.mark.parametrize("R,N", [(128, 32), (512, 96), (1024, 64), (256, 32)])
+def test_tc_gemm_mn_major_tma(stg, R, N):
+    """Xᵀ·Y with both operands loaded by 2-D TMA boxes in the MN-major
+    SWIZZLE_128B_BASE32B layout (the reduction GEMMs dW / dL): no thread
+    transposition, hi = raw (truncation), lo computed in place."""
+    X = gen.uniform_pm1(9, R, R * 128).reshape(R, 128).astype(np.float64)
+    Y = gen.uniform_pm1(10, N, R * N).reshape(R, N).astype(np.float64)
+    C = stg.stg_debug_tc_gemm(4, to_gpu(X), to_gpu(Y)).cpu().numpy()
+    err = np.max(np.abs(C - X.T @ Y) / _cond(X.T, Y))
+    assert err < 2e-6, err
