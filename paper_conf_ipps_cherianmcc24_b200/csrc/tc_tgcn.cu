@@ -1133,52 +1133,52 @@ __global__ void __launch_bounds__(kAtbThreads, 1) k_tc_atb(const AtbArgs p) {
 // SWIZZLE_128B_BASE32B layout (K = rows; pinned by tests/test_gpu_tc.py mode 4):
 // no transposition by threads; hi = the raw fp32 (hardware truncation) and
 // lo = x - trunc(x) is computed in place, elementwise, by 4 converter warps.
-// Each A operand is 4 feature boxes (M = 128): TMA boxes, an optional static
-// "ones" box (1.0 in feature 0 of every row: the Σ_rows term of dl) and zero
-// boxes.  Warp 0 issues the TMA, warp 1 the MMAs, warps 2-5 convert and run
-// the epilogue; a 2-stage ring overlaps loads, conversion and MMAs.  Each CTA
-// accumulates its tiles (grid-stride, fixed) in TMEM and writes its partial;
-// k_tc_sum_parts adds the partials in a fixed order (deterministic).
-constexpr int kAtbRT = 32;                        // rows per tile
-constexpr int kAtbBox = kAtbRT * 32 * 4;          // 4 KB per box
-constexpr int kAtbStages = 2;
-
+// A stage is a row of box slots [A slots | B slots]; A operand a covers 4
+// consecutive slots from a_first[a] (M = 128 features, one 32-feature chunk per
+// slot): slots past an operand's real boxes hold the following boxes, so the
+// corresponding D rows are garbage that is never read (rows are independent).
+// A slot is a TMA box or the static "ones" box (1.0 in feature 0 of every row:
+// the Σ_rows term of dl).  Warp 0 issues the TMA, warp 1 the MMAs, warps 2-5
+// convert and run the epilogue; an S-stage ring overlaps loads, conversion and
+// MMAs.  Each CTA accumulates its tiles (grid-stride, fixed) in TMEM and
+// writes its partial; k_tc_sum_parts adds the partials in a fixed order.
 struct AtbSpec2 {
   int V;
   int na;                 // 1 or 2 A operands
-  int src_map[2][4];      // per A operand and feature box: tensor map 0..3, or -1 zero, -2 ones (m_ones)
-  int src_col[2][4];
+  int a_first[2];         // first slot of each A operand
+  int nsa;                // A slots in a stage (<= 8)
+  int src_map[8];         // A slot source: tensor map 0..3, or -2 = ones box
+  int src_col[8];
   int nb;                 // B boxes (N = 32 nb), from map b_map at columns 32 k
   int b_map;
   float* part;            // [gridDim][na][128][N]
 };
 
-template <int NB>
+template <int NB, int RT, int S>
 __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUtensorMap m0,
                                                     const __grid_constant__ CUtensorMap m1,
                                                     const __grid_constant__ CUtensorMap m2,
                                                     const __grid_constant__ CUtensorMap m3,
                                                     const __grid_constant__ CUtensorMap m_ones, const AtbSpec2 sp) {
   constexpr int N = 32 * NB;
+  constexpr int BOX = RT * 32 * 4;
   extern __shared__ unsigned char sm_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
-  __shared__ uint64_t full[kAtbStages], conv[kAtbStages], empty[kAtbStages], done, init_bar;
+  __shared__ uint64_t full[S], conv[S], empty[S], done, init_bar;
   __shared__ uint32_t tslot;
-  const int na = sp.na;
-  const int nbox = 4 * na + NB;                    // boxes per stage (A boxes, then B boxes)
-  const size_t half = (size_t)nbox * kAtbBox;      // hi region of a stage; lo follows
-  auto hi = [&](int st, int bx) { return sm + (size_t)st * 2 * half + (size_t)bx * kAtbBox; };
-  auto lo = [&](int st, int bx) { return sm + (size_t)st * 2 * half + half + (size_t)bx * kAtbBox; };
+  const int na = sp.na, nsa = sp.nsa;
+  const int nbox = nsa + NB;                       // box slots per stage
+  const size_t half = (size_t)nbox * BOX;          // hi region of a stage; lo follows
+  auto hi = [&](int st, int bx) { return sm + (size_t)st * 2 * half + (size_t)bx * BOX; };
+  auto lo = [&](int st, int bx) { return sm + (size_t)st * 2 * half + half + (size_t)bx * BOX; };
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const CUtensorMap* maps[4] = {&m0, &m1, &m2, &m3};
-  // zero every stage once (zero / ones slots are never written by the ring)
-  for (size_t e = threadIdx.x; e < (size_t)kAtbStages * 2 * half / 16; e += blockDim.x)
+  auto map_of = [&](int m) -> const CUtensorMap* { return m == 0 ? &m0 : (m == 1 ? &m1 : (m == 2 ? &m2 : &m3)); };
+  for (size_t e = threadIdx.x; e < (size_t)S * 2 * half / 16; e += blockDim.x)   // lo of the ones box stays 0
     reinterpret_cast<float4*>(sm)[e] = make_float4(0.f, 0.f, 0.f, 0.f);
-  if (warp == 1) tc::tmem_alloc(&tslot, na * N <= 128 ? 128 : 256);
+  const uint32_t tcols = na * N <= 128 ? 128 : 256;
+  if (warp == 1) tc::tmem_alloc(&tslot, tcols);
   if (threadIdx.x == 0) {
-    for (int st = 0; st < kAtbStages; ++st) {
-      tc::mbar_init(&full[st], 1); tc::mbar_init(&conv[st], 128); tc::mbar_init(&empty[st], 1);
-    }
+    for (int st = 0; st < S; ++st) { tc::mbar_init(&full[st], 1); tc::mbar_init(&conv[st], 128); tc::mbar_init(&empty[st], 1); }
     tc::mbar_init(&done, 1); tc::mbar_init(&init_bar, 1);
     tc::fence_mbar_init();
   }
@@ -1186,53 +1186,48 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
-  // "ones" boxes: TMA the ones tile (laid out by the hardware's own swizzle) into each stage
   int n_ones = 0;
-  for (int a = 0; a < na; ++a)
-    for (int k = 0; k < 4; ++k) n_ones += sp.src_map[a][k] == -2;
-  if (n_ones) {
+  for (int k = 0; k < nsa; ++k) n_ones += sp.src_map[k] == -2;
+  if (n_ones) {                                      // the ones box (hardware swizzle) into each stage
     if (threadIdx.x == 0) {
-      tc::mbar_expect_tx(&init_bar, (uint32_t)(n_ones * kAtbStages * kAtbBox));
-      for (int st = 0; st < kAtbStages; ++st)
-        for (int a = 0; a < na; ++a)
-          for (int k = 0; k < 4; ++k)
-            if (sp.src_map[a][k] == -2) tc::tma_load_2d(hi(st, 4 * a + k), &m_ones, 0, 0, &init_bar);
+      tc::mbar_expect_tx(&init_bar, (uint32_t)(n_ones * S * BOX));
+      for (int st = 0; st < S; ++st)
+        for (int k = 0; k < nsa; ++k)
+          if (sp.src_map[k] == -2) tc::tma_load_2d(hi(st, k), &m_ones, 0, 0, &init_bar);
     }
     tc::mbar_wait(&init_bar, 0);
   }
   const uint32_t tm = tslot;
-  const int ntiles = (sp.V + kAtbRT - 1) / kAtbRT;
+  const int ntiles = (sp.V + RT - 1) / RT;
   int my_tiles = 0;
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) ++my_tiles;
   if (warp == 0) {                                   // ---- TMA producer
     if (lane == 0) {
-      int bytes = NB * kAtbBox;
-      for (int a = 0; a < na; ++a)
-        for (int k = 0; k < 4; ++k) bytes += sp.src_map[a][k] >= 0 ? kAtbBox : 0;
+      int bytes = NB * BOX;
+      for (int k = 0; k < nsa; ++k) bytes += sp.src_map[k] >= 0 ? BOX : 0;
       for (int i = 0; i < my_tiles; ++i) {
-        const int st = i % kAtbStages, kk = i / kAtbStages, r0 = (blockIdx.x + i * gridDim.x) * kAtbRT;
+        const int st = i % S, kk = i / S, r0 = (blockIdx.x + i * gridDim.x) * RT;
         if (kk > 0) tc::mbar_wait(&empty[st], (kk - 1) & 1);
         tc::mbar_expect_tx(&full[st], (uint32_t)bytes);
-        for (int a = 0; a < na; ++a)
-          for (int k = 0; k < 4; ++k)
-            if (sp.src_map[a][k] >= 0) tc::tma_load_2d(hi(st, 4 * a + k), maps[sp.src_map[a][k]], sp.src_col[a][k], r0, &full[st]);
-        for (int k = 0; k < NB; ++k) tc::tma_load_2d(hi(st, 4 * na + k), maps[sp.b_map], 32 * k, r0, &full[st]);
+        for (int k = 0; k < nsa; ++k)
+          if (sp.src_map[k] >= 0) tc::tma_load_2d(hi(st, k), map_of(sp.src_map[k]), sp.src_col[k], r0, &full[st]);
+        for (int k = 0; k < NB; ++k) tc::tma_load_2d(hi(st, nsa + k), map_of(sp.b_map), 32 * k, r0, &full[st]);
       }
     }
   } else if (warp == 1) {                            // ---- MMA issuer
     if (lane == 0) {
       const uint32_t idesc = tc::idesc_tf32(128, N, 1, 1);
       for (int i = 0; i < my_tiles; ++i) {
-        const int st = i % kAtbStages, kk = i / kAtbStages;
+        const int st = i % S, kk = i / S;
         tc::mbar_wait(&conv[st], kk & 1);
         tc::fence_after();
-        const uint32_t bh = tc::smem_u32(hi(st, 4 * na)), bl = tc::smem_u32(lo(st, 4 * na));
+        const uint32_t bh = tc::smem_u32(hi(st, nsa)), bl = tc::smem_u32(lo(st, nsa));
         for (int a = 0; a < na; ++a) {
-          const uint32_t ah = tc::smem_u32(hi(st, 4 * a)), al = tc::smem_u32(lo(st, 4 * a));
-          for (int k = 0; k < kAtbRT; k += 8) {            // 8 K-rows (1024 B) per MMA
+          const uint32_t ah = tc::smem_u32(hi(st, sp.a_first[a])), al = tc::smem_u32(lo(st, sp.a_first[a]));
+          for (int k = 0; k < RT; k += 8) {                // 8 K-rows (1024 B) per MMA
             const uint32_t o = (uint32_t)k * 128;
-            const uint64_t dah = tc::desc_mn_sw128_32b(ah + o, kAtbBox), dal = tc::desc_mn_sw128_32b(al + o, kAtbBox);
-            const uint64_t dbh = tc::desc_mn_sw128_32b(bh + o, kAtbBox), dbl = tc::desc_mn_sw128_32b(bl + o, kAtbBox);
+            const uint64_t dah = tc::desc_mn_sw128_32b(ah + o, BOX), dal = tc::desc_mn_sw128_32b(al + o, BOX);
+            const uint64_t dbh = tc::desc_mn_sw128_32b(bh + o, BOX), dbl = tc::desc_mn_sw128_32b(bl + o, BOX);
             const uint32_t d = tm + a * N;
             tc::mma_tf32(d, dal, dbh, idesc, (i > 0 || k > 0) ? 1u : 0u);
             tc::mma_tf32(d, dah, dbl, idesc, 1u);
@@ -1246,20 +1241,17 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   } else {                                           // ---- converters (warps 2-5), then epilogue
     const int ct = threadIdx.x - 64;
     for (int i = 0; i < my_tiles; ++i) {
-      const int st = i % kAtbStages;
-      tc::mbar_wait(&full[st], (i / kAtbStages) & 1);
-      for (int a = 0; a <= na; ++a) {
-        const int b0 = a < na ? 4 * a : 4 * na, nbx = a < na ? 4 : NB;
-        for (int bx = 0; bx < nbx; ++bx) {
-          if (a < na && sp.src_map[a][bx] < 0) continue;     // zero / ones: lo stays 0
-          const float4* src = reinterpret_cast<const float4*>(hi(st, b0 + bx));
-          float4* dst = reinterpret_cast<float4*>(lo(st, b0 + bx));
-#pragma unroll 4
-          for (int e = ct; e < kAtbBox / 16; e += 128) {
-            const float4 v = src[e];
-            dst[e] = make_float4(v.x - tc::tf32_hi(v.x), v.y - tc::tf32_hi(v.y), v.z - tc::tf32_hi(v.z),
-                                 v.w - tc::tf32_hi(v.w));
-          }
+      const int st = i % S;
+      tc::mbar_wait(&full[st], (i / S) & 1);
+      for (int bx = 0; bx < nbox; ++bx) {
+        if (bx < nsa && sp.src_map[bx] < 0) continue;   // ones box: lo stays 0
+        const float4* src = reinterpret_cast<const float4*>(hi(st, bx));
+        float4* dst = reinterpret_cast<float4*>(lo(st, bx));
+#pragma unroll
+        for (int e = ct; e < BOX / 16; e += 128) {
+          const float4 v = src[e];
+          dst[e] = make_float4(v.x - tc::tf32_hi(v.x), v.y - tc::tf32_hi(v.y), v.z - tc::tf32_hi(v.z),
+                               v.w - tc::tf32_hi(v.w));
         }
       }
       tc::fence_proxy_async();
@@ -1286,7 +1278,7 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   }
   tc::fence_before();
   __syncthreads();
-  if (warp == 1) tc::tmem_free(tm, na * N <= 128 ? 128 : 256);
+  if (warp == 1) tc::tmem_free(tm, tcols);
 }
 
 // Fixed-order sum of the per-CTA partials: tot[e] = Σ_b part[b][e] (blocks of 16).
@@ -1449,57 +1441,71 @@ static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
   return check_launch("tc_atb");
 }
 
-template <int NB>
+template <int NB, int RT, int S>
 static stg_status atb2_launch(const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb_out,
                               cudaStream_t s) {
-  const int nbox = 4 * sp.na + NB;
-  const size_t smem = (size_t)kAtbStages * 2 * nbox * kAtbBox + 1024;
-  STG_CUDA(cudaFuncSetAttribute(k_tc_atb2<NB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const int ntiles = (sp.V + kAtbRT - 1) / kAtbRT;
+  const int nbox = sp.nsa + NB;
+  const size_t smem = (size_t)S * 2 * nbox * RT * 32 * 4 + 1024;
+  STG_CUDA(cudaFuncSetAttribute(k_tc_atb2<NB, RT, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int ntiles = (sp.V + RT - 1) / RT;
   const int nb = std::max(1, std::min(ntiles, tc_atb_max_blocks()));
-  k_tc_atb2<NB><<<nb, 192, smem, s>>>(m[0], m[1], m[2], m[3], ones, sp);
+  k_tc_atb2<NB, RT, S><<<nb, 192, smem, s>>>(m[0], m[1], m[2], m[3], ones, sp);
   count_launch();
   *nb_out = nb;
   return check_launch("tc_atb2");
 }
 
+// 32-row tiles; as many ring stages (4, 3 or 2) as fit in shared memory
+template <int NB>
+static stg_status atb2_stages(const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb,
+                              cudaStream_t s) {
+  constexpr int RT = 32;
+  const size_t stage = (size_t)2 * (sp.nsa + NB) * RT * 32 * 4;
+  const size_t cap = 220 * 1024;
+  if (4 * stage <= cap) return atb2_launch<NB, RT, 4>(m, ones, sp, nb, s);
+  if (3 * stage <= cap) return atb2_launch<NB, RT, 3>(m, ones, sp, nb, s);
+  return atb2_launch<NB, RT, 2>(m, ones, sp, nb, s);
+}
+
 static stg_status atb2_dispatch(int NB, const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb,
                                 cudaStream_t s) {
   switch (NB) {
-    case 1: return atb2_launch<1>(m, ones, sp, nb, s);
-    case 2: return atb2_launch<2>(m, ones, sp, nb, s);
-    case 3: return atb2_launch<3>(m, ones, sp, nb, s);
-    case 4: return atb2_launch<4>(m, ones, sp, nb, s);
+    case 1: return atb2_stages<1>(m, ones, sp, nb, s);
+    case 2: return atb2_stages<2>(m, ones, sp, nb, s);
+    case 3: return atb2_stages<3>(m, ones, sp, nb, s);
+    case 4: return atb2_stages<4>(m, ones, sp, nb, s);
     default: return fail(STG_ERR_INVALID_ARG, "atb2: %d B boxes", NB);
   }
 }
+constexpr int kAtbRT = 32;
 
-// the [kAtbRT x 32] "ones" tile (1.0 in column 0): the Σ_rows feature of dl
-static stg_status ones_map(CUtensorMap* out, cudaStream_t s) {
+// the [RT x 32] "ones" tile (1.0 in column 0): the Σ_rows feature of dl
+static stg_status ones_map(CUtensorMap* out, int RT, cudaStream_t s) {
   static float* d = nullptr;
+  constexpr int kMaxRT = 64;
   if (!d) {
-    std::vector<float> h((size_t)kAtbRT * 32, 0.f);
-    for (int r = 0; r < kAtbRT; ++r) h[(size_t)r * 32] = 1.f;
+    std::vector<float> h((size_t)kMaxRT * 32, 0.f);
+    for (int r = 0; r < kMaxRT; ++r) h[(size_t)r * 32] = 1.f;
     if (cudaMalloc(&d, h.size() * sizeof(float)) != cudaSuccess) return fail(STG_ERR_NO_MEMORY, "ones tile");
     STG_CUDA(cudaMemcpy(d, h.data(), h.size() * sizeof(float), cudaMemcpyHostToDevice));
   }
   (void)s;
-  return make_tmap_f32(out, d, kAtbRT, 32, 32, 32, kAtbRT, true);
+  return make_tmap_f32(out, d, RT, 32, 32, 32, RT, true);
 }
 
 // dW[f][c] += Σ_v X[v,f]·dP[v,c]  via D = dPᵀ·X  (M = 128 features of dP, N = 32·ceil(F/32)).
 // part: tc_atb_max_blocks() · 2 · 128 · 128 floats; tot: 2 · 128 · 128 floats.
 stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* tot, float* dW,
                  cudaStream_t s) {
-  const int H3 = 3 * H, NB = (F + 31) / 32, N = 32 * NB;
+  const int H3 = 3 * H, NB = (F + 31) / 32, N = 32 * NB, NA = (H3 + 31) / 32;
   CUtensorMap m[4], ones;
   STG_TRY(make_tmap_f32(&m[0], dP, (uint64_t)V, H3, H3, 32, kAtbRT, true));
   STG_TRY(make_tmap_f32(&m[1], X, (uint64_t)V, F, F, 32, kAtbRT, true));
   m[2] = m[0]; m[3] = m[0];
-  STG_TRY(ones_map(&ones, s));
+  STG_TRY(ones_map(&ones, kAtbRT, s));
   AtbSpec2 sp{};
-  sp.V = V; sp.na = 1; sp.nb = NB; sp.b_map = 1; sp.part = part;
-  for (int k = 0; k < 4; ++k) { sp.src_map[0][k] = 32 * k < H3 ? 0 : -1; sp.src_col[0][k] = 32 * k; }
+  sp.V = V; sp.na = 1; sp.a_first[0] = 0; sp.nsa = NA; sp.nb = NB; sp.b_map = 1; sp.part = part;
+  for (int k = 0; k < NA; ++k) { sp.src_map[k] = 0; sp.src_col[k] = 32 * k; }
   int nb = 0;
   STG_TRY(atb2_dispatch(NB, m, ones, sp, &nb, s));
   const int n = 128 * N;
@@ -1520,15 +1526,18 @@ stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH,
   STG_TRY(make_tmap_f32(&m[1], Hp, (uint64_t)V, H, H, 32, kAtbRT, true));
   STG_TRY(make_tmap_f32(&m[2], RH, (uint64_t)V, H, H, 32, kAtbRT, true));
   STG_TRY(make_tmap_f32(&m[3], da, (uint64_t)V, H3, H3, 32, kAtbRT, true));
-  STG_TRY(ones_map(&ones, s));
+  STG_TRY(ones_map(&ones, kAtbRT, s));
+  // slots: C boxes | H | RH | ones | da boxes;  A1 = [C.. | H] (H at feature 32·NBC), A2 = [RH | ones]
   AtbSpec2 sp{};
   sp.V = V; sp.na = 2; sp.nb = NBC; sp.b_map = 3; sp.part = part;
-  for (int k = 0; k < 4; ++k) {
-    sp.src_map[0][k] = k < NBC ? 0 : (k == NBC ? 1 : -1);
-    sp.src_col[0][k] = k < NBC ? 32 * k : 0;
-    sp.src_map[1][k] = k == 0 ? 2 : (k == 1 ? -2 : -1);
-    sp.src_col[1][k] = 0;
-  }
+  int k = 0;
+  for (; k < NBC; ++k) { sp.src_map[k] = 0; sp.src_col[k] = 32 * k; }
+  sp.src_map[k] = 1; sp.src_col[k] = 0; ++k;
+  sp.a_first[0] = 0;
+  sp.a_first[1] = k;
+  sp.src_map[k] = 2; sp.src_col[k] = 0; ++k;
+  sp.src_map[k] = -2; sp.src_col[k] = 0; ++k;
+  sp.nsa = k;
   int nb = 0;
   STG_TRY(atb2_dispatch(NBC, m, ones, sp, &nb, s));
   const int N = 32 * NBC, n = 2 * 128 * N;
