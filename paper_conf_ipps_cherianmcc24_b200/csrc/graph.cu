@@ -310,11 +310,17 @@ __device__ __forceinline__ int64_t lb_keys(const uint64_t* a, int64_t lo, int64_
 }
 
 // Surviving old edges move to new_rowptr[v] + i - (#dels < c) + (#adds < c).
+// Edge labels ("relabelled" after an update) follow the move:
+// the in-direction pass records emap[old position] = new position (-1 if
+// deleted); the out-direction pass sets eid_new[new out position] =
+// emap[eid_old[old out position]] — one lookup per edge instead of a search.
 __global__ void k_merge_old(const int32_t* __restrict__ orow, const int32_t* __restrict__ ocol,
                             const int32_t* __restrict__ orowptr, int64_t E_old,
                             const int32_t* __restrict__ nrowptr, const int4* __restrict__ touch,
                             const uint64_t* __restrict__ adds, const uint64_t* __restrict__ dels, int nb,
-                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol) {
+                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol, int32_t* __restrict__ emap_out,
+                            const int32_t* __restrict__ emap_in, const int32_t* __restrict__ eid_old,
+                            int32_t* __restrict__ eid_new) {
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < E_old; j += (int64_t)gridDim.x * blockDim.x) {
     int32_t v = orow[j], c = ocol[j];
     int4 t = touch[v];
@@ -322,20 +328,40 @@ __global__ void k_merge_old(const int32_t* __restrict__ orow, const int32_t* __r
     if (t.y != t.x || t.w != t.z) {
       uint64_t key = ((uint64_t)v << nb) | (uint64_t)c;
       int64_t dl = lb_keys(dels, t.z, t.w, key);
-      if (dl < t.w && dels[dl] == key) continue;  // deleted
+      if (dl < t.w && dels[dl] == key) {            // deleted
+        if (emap_out) emap_out[j] = -1;
+        continue;
+      }
       int64_t al = lb_keys(adds, t.x, t.y, key);
       pos += (al - t.x) - (dl - t.z);
     }
     nrow[pos] = v;
     ncol[pos] = c;
+    if (emap_out) emap_out[j] = (int32_t)pos;
+    if (eid_new) eid_new[pos] = emap_in[eid_old[j]];
   }
 }
 
+// in-CSR position of edge (u -> v) in the (new) in-CSR: rowptr[v] + lower_bound(col row v, u)
+__device__ __forceinline__ int32_t in_position(const int32_t* __restrict__ in_rowptr, const int32_t* __restrict__ in_col,
+                                               int32_t u, int32_t v) {
+  int32_t lo = in_rowptr[v], hi = in_rowptr[v + 1];
+  while (lo < hi) {
+    int32_t mid = (lo + hi) >> 1;
+    if (in_col[mid] < u) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
 // Added edge a of row v lands at new_rowptr[v] + (a - add_lo) + (#old < c) - (#dels < c).
+// Out-direction pass with labels: the label of an added out-edge (v -> c) is
+// searched in the new in-CSR (only the |A'| added edges).
 __global__ void k_merge_add(const uint64_t* __restrict__ adds, int64_t nadd, const uint64_t* __restrict__ dels,
                             int nb, const int32_t* __restrict__ ocol, const int32_t* __restrict__ orowptr,
                             const int32_t* __restrict__ nrowptr, const int4* __restrict__ touch,
-                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol) {
+                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol,
+                            const int32_t* __restrict__ in_rowptr_new, const int32_t* __restrict__ in_col_new,
+                            int32_t* __restrict__ eid_new) {
   const uint64_t mask = (uint64_t(1) << nb) - 1;
   for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < nadd; a += (int64_t)gridDim.x * blockDim.x) {
     uint64_t key = adds[a];
@@ -351,23 +377,35 @@ __global__ void k_merge_add(const uint64_t* __restrict__ adds, int64_t nadd, con
     int64_t pos = (int64_t)nrowptr[v] + (a - t.x) + (b - lo) - (dl - t.z);
     nrow[pos] = v;
     ncol[pos] = c;
+    if (eid_new) eid_new[pos] = in_position(in_rowptr_new, in_col_new, v, c);
   }
 }
 
+// Labels: `emap_out` (in-direction pass) records old -> new in-CSR positions;
+// `eid` (out-direction pass) carries {emap_in, eid_old, eid_new, new in-CSR}.
+struct EidPass {
+  const int32_t* emap_in = nullptr;
+  const int32_t* eid_old = nullptr;
+  int32_t* eid_new = nullptr;
+  const int32_t* in_rowptr_new = nullptr;
+  const int32_t* in_col_new = nullptr;
+};
+
 static stg_status apply_dir(int32_t V, int nb, const int32_t* orow, const int32_t* ocol, const int32_t* orowptr,
                             const int32_t* odeg, int64_t E_old, int32_t* nrow, int32_t* ncol, int32_t* nrowptr,
-                            int32_t* ndeg, const DirDelta& d, int4* touch, BuildWs& ws, cudaStream_t s) {
+                            int32_t* ndeg, const DirDelta& d, int4* touch, BuildWs& ws, cudaStream_t s,
+                            int32_t* emap_out, const EidPass& eid) {
   if (d.nadd) { k_touch_mark<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, nb, 0, touch); count_launch(); }
   if (d.ndel) { k_touch_mark<<<grid_for(d.ndel, 256), 256, 0, s>>>(d.del, d.ndel, nb, 1, touch); count_launch(); }
   STG_TRY(scan(NewDegIn{odeg, touch}, RowptrOut{nrowptr, ndeg}, V, ws.scan, s, nullptr, nrowptr + V));
   if (E_old) {
     k_merge_old<<<grid_for(E_old, 256), 256, 0, s>>>(orow, ocol, orowptr, E_old, nrowptr, touch, d.add, d.del, nb,
-                                                    nrow, ncol);
+                                                    nrow, ncol, emap_out, eid.emap_in, eid.eid_old, eid.eid_new);
     count_launch();
   }
   if (d.nadd) {
     k_merge_add<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, d.del, nb, ocol, orowptr, nrowptr, touch, nrow,
-                                                     ncol);
+                                                     ncol, eid.in_rowptr_new, eid.in_col_new, eid.eid_new);
     count_launch();
   }
   if (d.nadd) { k_touch_clear<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, nb, touch); count_launch(); }
@@ -378,17 +416,30 @@ static stg_status apply_dir(int32_t V, int nb, const int32_t* orow, const int32_
 stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
                        int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws, cudaStream_t s) {
   const int32_t V = src.V;
+  // labels are carried incrementally when the source snapshot has them
+  const bool carry = dst.edge_ids && src.edge_ids && src.E > 0;
+  int32_t* emap = nullptr;
+  if (carry) {
+    STG_TRY(ws.emap.alloc((size_t)src.E, s));
+    emap = ws.emap.p;
+  }
   STG_TRY(apply_dir(V, src.nb, src.in_row.p, src.in_col.p, src.in_rowptr.p, src.in_deg.p, src.E, dst.in_row.p,
-                    dst.in_col.p, dst.in_rowptr.p, dst.in_deg.p, in_dir, touch_in, ws, s));
+                    dst.in_col.p, dst.in_rowptr.p, dst.in_deg.p, in_dir, touch_in, ws, s, emap, EidPass{}));
+  EidPass ep;
+  if (carry) {
+    ep.emap_in = emap; ep.eid_old = src.out_eid.p; ep.eid_new = dst.out_eid.p;
+    ep.in_rowptr_new = dst.in_rowptr.p; ep.in_col_new = dst.in_col.p;
+  }
   STG_TRY(apply_dir(V, src.nb, src.out_row.p, src.out_col.p, src.out_rowptr.p, src.out_deg.p, src.E,
-                    dst.out_row.p, dst.out_col.p, dst.out_rowptr.p, dst.out_deg.p, out_dir, touch_out, ws, s));
+                    dst.out_row.p, dst.out_col.p, dst.out_rowptr.p, dst.out_deg.p, out_dir, touch_out, ws, s, nullptr,
+                    ep));
   dst.E = E_new;
   dst.t = t_new;
   k_norm<<<grid_for(V, 256), 256, 0, s>>>(dst.in_deg.p, dst.out_deg.p, V, dst.dgl_both, dst.norm_src.p,
                                          dst.norm_dst.p);
   count_launch();
   STG_TRY(build_ids_and_sched(dst, ws, s));
-  return build_out_eid(dst, s);
+  return carry ? check_launch("apply_delta") : build_out_eid(dst, s);
 }
 
 // ------------------------------------------------------------ static graph

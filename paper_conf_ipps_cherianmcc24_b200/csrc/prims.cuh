@@ -24,6 +24,7 @@ struct BuildWs {
   DArray<uint32_t> dkey, dkey_alt;
   DArray<int32_t> dval, dval_alt;
   DArray<int64_t> count;
+  DArray<int32_t> emap;        // delta apply: old in-CSR position -> new position (-1 = deleted)
 };
 
 namespace {

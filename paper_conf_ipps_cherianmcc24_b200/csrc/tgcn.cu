@@ -392,19 +392,30 @@ __global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t H, const flo
   }
 }
 
-__global__ void k_mse_reduce(int32_t nb, int32_t H, int32_t V, const double* __restrict__ lpart,
-                             const float* __restrict__ gpart, float* __restrict__ loss, float* __restrict__ dw_o,
-                             float* __restrict__ db_o) {
-  if (blockIdx.x == 0 && threadIdx.x == 0 && loss) {
-    double t = 0.0;
-    for (int b = 0; b < nb; ++b) t += lpart[b];
-    *loss += (float)(t / (double)V);
+// Fixed-order reduction of the per-block partials: block k < H sums column k
+// of gpart (dw_o), block H the db_o column, block H+1 the loss partials; each
+// thread sums a fixed strided subset, then a fixed shared-memory tree.
+__global__ void __launch_bounds__(256) k_mse_reduce(int32_t nb, int32_t H, int32_t V, const double* __restrict__ lpart,
+                                                    const float* __restrict__ gpart, float* __restrict__ loss,
+                                                    float* __restrict__ dw_o, float* __restrict__ db_o) {
+  __shared__ double sd[256];
+  const int k = blockIdx.x;
+  double t = 0.0;
+  if (k <= H) {
+    for (int b = threadIdx.x; b < nb; b += 256) t += (double)gpart[(int64_t)b * (H + 1) + k];
+  } else {
+    for (int b = threadIdx.x; b < nb; b += 256) t += lpart[b];
   }
-  for (int k = threadIdx.x; k < H + 1; k += blockDim.x) {
-    float t = 0.0f;
-    for (int b = 0; b < nb; ++b) t += gpart[(int64_t)b * (H + 1) + k];
-    if (k < H) { if (dw_o) dw_o[k] += t; }
-    else if (db_o) db_o[0] += t;
+  sd[threadIdx.x] = t;
+  __syncthreads();
+  for (int o = 128; o; o >>= 1) {
+    if (threadIdx.x < o) sd[threadIdx.x] += sd[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    if (k < H) { if (dw_o) dw_o[k] += (float)sd[0]; }
+    else if (k == H) { if (db_o) db_o[0] += (float)sd[0]; }
+    else if (loss) *loss += (float)(sd[0] / (double)V);
   }
 }
 
@@ -669,8 +680,8 @@ stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, c
     case 16: k_mse_head<16><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
     default: k_mse_head<32><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
   }
-  k_mse_reduce<<<1, 64, 0, s>>>(nb, H, V, ws.lpart.p, ws.gpart.p, loss_accum, want ? dw_o : nullptr,
-                                want ? db_o : nullptr);
+  k_mse_reduce<<<H + 2, 256, 0, s>>>(nb, H, V, ws.lpart.p, ws.gpart.p, loss_accum, want ? dw_o : nullptr,
+                                     want ? db_o : nullptr);
   count_launch(2);
   return check_launch("stg_mse_head");
 }
