@@ -379,7 +379,7 @@ def main():
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "k_aggregate (fwd in-CSR + bwd out-CSR, W=%d)" % Wagg,
+                         "kernel": "k_agg_stream + k_agg_hubs (fwd in-CSR + bwd out-CSR, W=%d)" % Wagg,
                          "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": agg_avg_s * 1e3,
                          "peak_source": peak_src},
             "phases_ms_per_step": {k: v[0] / nprof for k, v in prof.items()},
