@@ -379,6 +379,10 @@ def main():
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
+                         "dram_GBps_at_traffic": (traffic / agg_avg_s / 1e9) if traffic else None,
+                         "dram_frac_at_traffic": (traffic / agg_avg_s / 1e9 / peak) if traffic else None,
+                         "alg_bytes_model": "compulsory: 4E col + 4(V+1) rowptr + 4V node_ids + 4V row scale "
+                                            "+ 4VW (each source row once) + 4VW (output)",
                          "kernel": "k_agg_stream + k_agg_hubs (fwd in-CSR + bwd out-CSR, W=%d)" % Wagg,
                          "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": agg_avg_s * 1e3,
                          "peak_source": peak_src},
