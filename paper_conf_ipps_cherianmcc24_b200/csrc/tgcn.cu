@@ -9,6 +9,7 @@
 //                      the out-CSR (dP) → k_dw (Xᵀ·dP partials) → fixed-order
 //                      reduction.  No float atomics: deterministic run to run.
 #include <algorithm>
+#include <map>
 #include <mutex>
 #include <vector>
 
@@ -695,6 +696,35 @@ stg_status stg_sgd_update(float* p, float* g, int64_t n, float lr, stg_stream_t 
   return check_launch("stg_sgd_update");
 }
 
+namespace {
+// per-device side stream and sequence events of stg_tgcn_train_sequence
+cudaStream_t side_stream() {
+  static std::mutex mu;
+  static std::map<int, cudaStream_t> streams;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = streams.find(dev);
+  if (it != streams.end()) return it->second;
+  cudaStream_t s = nullptr;
+  cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+  return streams[dev] = s;
+}
+cudaEvent_t seq_event(int k) {
+  static std::mutex mu;
+  static std::map<std::pair<int, int>, cudaEvent_t> evs;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  auto key = std::make_pair(dev, k);
+  auto it = evs.find(key);
+  if (it != evs.end()) return it->second;
+  cudaEvent_t e = nullptr;
+  cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+  return evs[key] = e;
+}
+}  // namespace
+
 stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
                                    const stg_tgcn_params* p, const float* w_o, const float* b_o,
                                    const float* const* X, const float* const* Y, const float* H0, float* H_seq,
@@ -718,32 +748,72 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
   }
   const int32_t H = p->H;
   const size_t VH = (size_t)V * H;
+  cudaStream_t ms = (cudaStream_t)stream;
+  // Snapshot builds (Get-Graph / Get-Backward-Graph) of the NEXT timestamp run on a side
+  // stream while the current timestamp's TGCN step runs on `stream`: the build of t+1 writes
+  // the other slot of the snapshot pair, after the step that last read that slot (t-1) is
+  // done; step t+1 waits for its build.  (Streams instead of a tracing compiler.)
+  const bool overlap = dtdg != nullptr && S > 1;
+  cudaStream_t ss = overlap ? side_stream() : nullptr;
+  cudaEvent_t ev_done[2] = {nullptr, nullptr}, ev_built[2] = {nullptr, nullptr};
+  if (overlap) {
+    for (int k = 0; k < 2; ++k) { ev_done[k] = seq_event(2 * k); ev_built[k] = seq_event(2 * k + 1); }
+    STG_CUDA(cudaEventRecord(ev_done[1], ms));      // everything before this sequence (incl. Get-Graph(t0))
+  }
   std::vector<int32_t> graph_stack;
+  stg_csr_view views[2] = {view, view};
   // forward, Algorithm 1 lines 7-16
   for (int32_t i = 0; i < S; ++i) {
     const int32_t t = t0 + i;
     if (dtdg) {
-      if (i > 0) STG_TRY(stg_dtdg_get_snapshot(dtdg, t, stream, &view));   // Get-Graph (Alg. 2)
+      if (overlap) {
+        if (i + 1 < S) {                                                    // prefetch Get-Graph(t+1)
+          STG_CUDA(cudaStreamWaitEvent(ss, ev_done[(i + 1) & 1], 0));       // step t-1 (slot reuse) done
+          STG_TRY(stg_dtdg_get_snapshot(dtdg, t + 1, ss, &views[(i + 1) & 1]));
+          STG_CUDA(cudaEventRecord(ev_built[(i + 1) & 1], ss));
+        }
+        if (i > 0) STG_CUDA(cudaStreamWaitEvent(ms, ev_built[i & 1], 0));
+      } else if (i > 0) {
+        STG_TRY(stg_dtdg_get_snapshot(dtdg, t, stream, &views[i & 1]));    // Get-Graph (Alg. 2)
+      }
       graph_stack.push_back(t);                                             // graph-stack.push(t)
     }
+    const stg_csr_view& v = views[dtdg ? (i & 1) : 0];
     const float* Hp = i == 0 ? H0 : H_seq + (size_t)(i - 1) * VH;
-    STG_TRY(stg_tgcn_step(&view, p, X[i], Hp, H_seq + (size_t)i * VH, stack, stream));   // push + fwdprop
+    STG_TRY(stg_tgcn_step(&v, p, X[i], Hp, H_seq + (size_t)i * VH, stack, stream));   // push + fwdprop
     STG_TRY(stg_mse_head(V, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr, nullptr,
                          stream));                                          // loss += loss-fn(out)
+    if (overlap) STG_CUDA(cudaEventRecord(ev_done[i & 1], ms));
   }
   // backward in LIFO order, lines 18-25
   float* G = G_work;
   float* Gn = G_work + VH;
-  STG_CUDA(cudaMemsetAsync(G, 0, sizeof(float) * VH, (cudaStream_t)stream));
+  STG_CUDA(cudaMemsetAsync(G, 0, sizeof(float) * VH, ms));
+  stg_csr_view bviews[2] = {views[0], views[1]};
+  if (dtdg) {
+    const int32_t t = graph_stack.back();
+    STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, t, ss ? ss : ms, &bviews[(S - 1) & 1]));   // the forward head
+    if (overlap) STG_CUDA(cudaEventRecord(ev_built[(S - 1) & 1], ss));
+  }
   for (int32_t i = S - 1; i >= 0; --i) {
     if (dtdg) {
-      const int32_t t = graph_stack.back();
-      graph_stack.pop_back();
-      STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, t, stream, &view));     // Get-Backward-Graph
+      graph_stack.pop_back();                                               // graph-stack.pop()
+      if (overlap) {
+        if (i > 0) {                                                        // prefetch Get-Backward-Graph(t-1)
+          STG_CUDA(cudaStreamWaitEvent(ss, ev_done[(i + 1) & 1], 0));       // step t+1 (slot reuse) done
+          STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, graph_stack.back(), ss, &bviews[(i - 1) & 1]));
+          STG_CUDA(cudaEventRecord(ev_built[(i - 1) & 1], ss));
+        }
+        STG_CUDA(cudaStreamWaitEvent(ms, ev_built[i & 1], 0));
+      } else if (i < S - 1) {
+        STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, t0 + i, stream, &bviews[i & 1]));   // Get-Backward-Graph
+      }
     }
+    const stg_csr_view& v = bviews[dtdg ? (i & 1) : 0];
     // G = dℓ_t/dH_t + dH from step t+1
     STG_TRY(stg_mse_head(V, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, nullptr, G, 1, dw_o, db_o, stream));
-    STG_TRY(stg_tgcn_step_backward(&view, p, X[i], G, Gn, grads, stack, stream));   // pop + bwdprop
+    STG_TRY(stg_tgcn_step_backward(&v, p, X[i], G, Gn, grads, stack, stream));   // pop + bwdprop
+    if (overlap) STG_CUDA(cudaEventRecord(ev_done[i & 1], ms));
     std::swap(G, Gn);
   }
   return STG_OK;
