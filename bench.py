@@ -42,6 +42,10 @@ def parse():
     ap.add_argument("--lr", type=float, default=1e-3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--mode", default="sharded", choices=["sharded", "replicas"],
+                    help="N>1: row-block shards of one graph (SURVEY §8(e)) or independent replicas")
+    ap.add_argument("--shard-sim", default=None, metavar="K/N",
+                    help="(testing on one GPU) run rank K's row block of an N-way sharding, no process group")
     return ap.parse_args()
 
 
@@ -175,8 +179,12 @@ def main():
     import gen
     import paper_conf_ipps_cherianmcc24_b200 as stg
 
+    sim = args.shard_sim is not None
+    if sim:
+        rank, world = (int(x) for x in args.shard_sim.split("/"))
     torch.cuda.set_device(local)
-    if world > 1:
+    pg = world > 1 and not sim                  # a real process group (torchrun)
+    if pg:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
     cfg = gen.CONFIGS[args.config]
@@ -185,29 +193,53 @@ def main():
     V, F, H, T = cfg.V, cfg.F, cfg.H, d.T
     S = args.seq
     seqs = [(t0, min(S, T - t0)) for t0 in range(0, T, S)]
+    # N > 1, sharded (default): destination row blocks with ~E/N in-edges of S_0 each
+    # (SURVEY §8(e)); each rank's DTDG holds the edges into its block, X_t is resident
+    # on every rank, and the per-sequence gradients are summed by one NCCL all-reduce.
+    sharded = world > 1 and args.mode == "sharded"
+    lo, hi = 0, V
+    if sharded:
+        from paper_conf_ipps_cherianmcc24_b200 import parallel
+        bounds = parallel.base_row_blocks(V, d.src0, d.dst0, world, self_loops=True)
+        lo, hi = bounds[rank], bounds[rank + 1]
+    R = hi - lo
     g = stg.stg_dtdg_create(V, T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src, d.del_dst,
-                            stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS)
+                            stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS, dist=(rank, world, lo, hi) if sharded else None)
     E_t = [g.num_edges(t) for t in range(T)]
-    edges_per_step = 2 * sum(E_t)
+    edges_per_step = 2 * sum(E_t)            # this rank's edges (whole graph unless sharded)
+    edges_all = edges_per_step
+    if pg:
+        te = torch.tensor([float(edges_per_step)], dtype=torch.float64, device=torch.device("cuda", local))
+        dist.all_reduce(te)
+        edges_all = int(te.item())
 
     # inputs: 2 distinct seeded X_t matrices cycled over t (each 256 MB > L2), labels per t
     NX = 2
     Xh = [torch.from_numpy(gen.features(cfg, i)) for i in range(NX)]
-    Yh = [torch.from_numpy(gen.labels(cfg, t)) for t in range(T)]
+    Yh = [torch.from_numpy(gen.labels(cfg, t)[lo:hi].copy()) for t in range(T)]
     Xd = [x.to(dev) for x in Xh]
     Yd = [y.to(dev) for y in Yh]
     p = {k: torch.from_numpy(v).to(dev) for k, v in gen.tgcn_params(F, H, cfg.seed).items()}
-    grads = {"W": torch.zeros(F, 3 * H, device=dev), "b": torch.zeros(3 * H, device=dev),
-             "L": torch.zeros(3, 2 * H, H, device=dev), "l": torch.zeros(3, H, device=dev)}
-    dw_o, db_o = torch.zeros(H, device=dev), torch.zeros(1, device=dev)
+    # all gradients live in one flat buffer: one all-reduce per sequence when sharded
+    gshapes = {"W": (F, 3 * H), "b": (3 * H,), "L": (3, 2 * H, H), "l": (3, H), "w_o": (H,), "b_o": (1,)}
+    gflat = torch.zeros(sum(int(np.prod(v)) for v in gshapes.values()), device=dev)
+    gv, off = {}, 0
+    for k, shp in gshapes.items():
+        n = int(np.prod(shp))
+        gv[k] = gflat[off:off + n].view(shp)
+        off += n
+    grads = {k: gv[k] for k in ("W", "b", "L", "l")}
+    dw_o, db_o = gv["w_o"], gv["b_o"]
     loss = torch.zeros(1, device=dev)
-    Hbuf = [torch.empty(S, V, H, device=dev) for _ in range(2)]
-    H0 = torch.zeros(V, H, device=dev)
-    Gw = torch.empty(2, V, H, device=dev)
-    stack = stg.stg_state_stack_create(S * V * 3 * H * 4 + (64 << 20))
+    Hbuf = [torch.empty(S, R, H, device=dev) for _ in range(2)]
+    H0 = torch.zeros(R, H, device=dev)
+    Gw = torch.empty(2, R, H, device=dev)
+    stack = stg.stg_state_stack_create(S * max(R, 1) * 3 * H * 4 + (64 << 20))
     stream = torch.cuda.current_stream()
 
     def sgd():
+        if sharded and pg:
+            dist.all_reduce(gflat)               # whole-graph gradient = Σ_ranks (NCCL, ~51 KB)
         for k in ("W", "b", "L", "l"):
             stg.stg_sgd_update(p[k], grads[k], args.lr)
         stg.stg_sgd_update(p["w_o"], dw_o, args.lr)
@@ -233,7 +265,7 @@ def main():
     clocks = ClockSampler(local)
     stg.stg_profile_enable(False)
     stg.stg_profile_read(reset=True)
-    if world > 1:
+    if pg:
         dist.barrier()
     torch.cuda.synchronize()
     clocks.start()
@@ -248,13 +280,14 @@ def main():
     ms = ev0.elapsed_time(ev1)
     launches = stg.kernel_launch_count() - launches0
     clk = clocks.stop()
-    if world > 1:
+    if pg:
         t = torch.tensor([ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = t.item()
         dist.barrier()
-    value = world * edges_per_step * args.steps / (ms / 1e3)
-    tsps = world * T * args.steps / (ms / 1e3)
+    value = edges_all * args.steps / (ms / 1e3)
+    # sharded: the ranks advance the same T timestamps together; replicas: N epochs
+    tsps = (1 if sharded else world) * T * args.steps / (ms / 1e3)
 
     # ---------------- per-phase device times (profiled pass, same work)
     stg.stg_profile_enable(True)
@@ -268,10 +301,12 @@ def main():
 
     # roofline of the dominant kernel: the aggregation (fwd + bwd, W = 3H)
     Wagg = 3 * H
-    E_mean = sum(E_t) / T
+    E_mean = sum(E_t) / T                       # this rank's edges per snapshot
     # compulsory bytes per launch: col 4E + rowptr 4(V+1) + node_ids 4V + row scale 4V
     # + read each source row once 4VW + write each output row 4VW
-    alg_bytes = 4 * E_mean + 4 * (V + 1) + 4 * V + 4 * V + 8 * V * Wagg
+    # (sharded rank, mean of fwd and bwd: the fwd reads all V source rows and writes R rows, the bwd the
+    # reverse; R = V unsharded gives 4E + 4(V+1) + 8V + 8VW)
+    alg_bytes = 4 * E_mean + 2 * (V + 1) + 2 * (R + 1) + 4 * (V + R) + 4 * Wagg * (V + R)
     agg_ms = prof["agg_fwd"][0] + prof["agg_bwd"][0]
     agg_n = prof["agg_fwd"][1] + prof["agg_bwd"][1]
     agg_avg_s = (agg_ms / agg_n) / 1e3 if agg_n else float("nan")
@@ -293,7 +328,7 @@ def main():
         Ypin = [y.pin_memory() for y in Yh]
         copy = torch.cuda.Stream(device=dev)
         stage = [[torch.empty(V, F, device=dev) for _ in range(S)] for _ in range(2)]
-        ystage = [[torch.empty(V, device=dev) for _ in range(S)] for _ in range(2)]
+        ystage = [[torch.empty(R, device=dev) for _ in range(S)] for _ in range(2)]
         loss_h = torch.empty(1, pin_memory=True)
         h2d = 0
 
@@ -338,17 +373,17 @@ def main():
             e2e_epoch()
         h2d = 0
         torch.cuda.synchronize()
-        if world > 1:
+        if pg:
             dist.barrier()
         t0w = time.perf_counter()
         for _ in range(args.steps):
             e2e_epoch()
         e2e_s = time.perf_counter() - t0w
-        if world > 1:
+        if pg:
             tt = torch.tensor([e2e_s], device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             e2e_s = tt.item()
-        e2e = {"value": world * edges_per_step * args.steps / e2e_s, "unit": UNIT,
+        e2e = {"value": edges_all * args.steps / e2e_s, "unit": UNIT,
                "h2d_bytes_per_step": int(h2d / args.steps), "d2h_bytes_per_step": 4,
                "ms_per_step": 1e3 * e2e_s / args.steps,
                "note": "X_t (256 MB) and y_t copied H2D from pinned host memory every timestep on a copy "
@@ -356,7 +391,7 @@ def main():
 
     # ---------------- CPU baseline: the oracle on one C5 timestep (rank 0, N=1 only)
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not sim and not args.no_cpu_baseline:
         import oracle
         oracle.build()
         S0 = next(oracle.snapshot_sets_fold(d, self_loops=True))
@@ -365,17 +400,20 @@ def main():
                "sample": "one C5 timestep (t=1): fold S_0->S_1, CSR pair, TGCN fwd + MSE head + bwd, fp64, "
                          "single thread; %.1f s" % dt_c}
 
-    if rank == 0:
+    if rank == 0 or sim:
         out = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1 if sim else world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": cfg.desc + " (BASELINE.json configs[4])", "config": cfg.name, "V": V,
                        "E_mean": int(E_mean), "T": T, "F": F, "H": H, "seq_len": S, "sequences": len(seqs),
                        "step": "one Algorithm-1 training epoch over all T timestamps",
                        "l2": "inputs larger than L2 (X_t 256 MB, graph ~0.3 GB, state 8 GB)",
-                       "parallelism": "replicas" if world > 1 else "single"},
+                       "parallelism": ("row-block shards x%d (resident X_t, NCCL gradient all-reduce per "
+                                       "sequence)" % world) if sharded else ("replicas" if world > 1 else "single"),
+                       "E_local_mean_rank0": int(E_mean)},
             "timesteps_per_s": tsps,
+            "shard_sim": args.shard_sim,
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
@@ -393,7 +431,7 @@ def main():
             "cpu_baseline": cpu,
         }
         print(json.dumps(out), flush=True)
-    if world > 1:
+    if pg:
         dist.barrier()
         dist.destroy_process_group()
 

@@ -69,10 +69,18 @@ enum {
                                    both = in_deg^-1/2, PyG gcn_norm, reading C1) */
 };
 
-/* Row-block sharding: an object created with a non-NULL
- * stg_dist holds only the destination rows [row_begin,row_end) of the
- * forward in-CSR and, for the backward out-CSR, only the edges whose
- * destination lies in that block (rows = all sources).  NULL = whole graph. */
+/* Row-block sharding (north_star "partitioned ... by
+ * destination-vertex row blocks"): an object created with a non-NULL stg_dist
+ * holds only the edges whose destination lies in [row_begin,row_end): the
+ * forward in-CSR has the R = row_end-row_begin local rows, the backward
+ * out-CSR has all V source rows but only the local edges.  Vertex ids stay
+ * global.  Degrees and node_ids describe the held edges (in_ids lists the R
+ * local rows first); norm_src / norm_dst are those of the WHOLE graph (the
+ * library keeps the whole-graph degrees current from the whole-graph deltas),
+ * so the local results are exactly the rows / partial sums of the whole-graph
+ * computation.  Snapshot builds need no communication.  rank / world are
+ * informational.  row_begin <= row_end must lie in [0,V]
+ * (STG_ERR_INVALID_ARG otherwise).  NULL = whole graph. */
 typedef struct {
   int32_t rank, world;
   int32_t row_begin, row_end;
@@ -141,7 +149,7 @@ stg_status stg_dtdg_get_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, st
  * reached from the backward cursor by reverse updates, without disturbing the
  * cached forward head (which the next sequence starts from). */
 stg_status stg_dtdg_get_backward_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, stg_csr_view* out);
-int64_t stg_dtdg_num_edges(const stg_dtdg* g, int32_t t);    /* -1 if t out of range */
+int64_t stg_dtdg_num_edges(const stg_dtdg* g, int32_t t);    /* edges held at t (the local block's if sharded); -1 if t out of range */
 int32_t stg_dtdg_num_timestamps(const stg_dtdg* g);
 /* Number of effective added / deleted edges of step t (0 for t = 0). */
 int64_t stg_dtdg_num_deltas(const stg_dtdg* g, int32_t t, int32_t deletes);
@@ -151,7 +159,8 @@ void stg_dtdg_destroy(stg_dtdg* g);
  * forward : y[v,:] = n_dst[v] · Σ_{u∈N_in(v)} n_src[u] · x[u,:]   over the in-CSR,
  *           for the local rows v of the view (y row i ↔ vertex row_begin+i).
  * backward: gx[u,:] = n_src[u] · Σ_{v∈N_out(u)} n_dst[v] · gy[v,:] over the out-CSR
- *           (the exact transpose), for all V sources (partial sums if sharded).
+ *           (the exact transpose), for all V sources (partial sums if sharded;
+ *           gy then holds the R local rows: gy row i ↔ vertex row_begin+i).
  * x/gy: [V,W] (forward: all sources) with leading dimension ldx >= W;
  * y/gx: leading dimension ldy >= W.  fp32 accumulation in a fixed order per
  * row: results are deterministic run to run (no float atomics; reading C20).
@@ -162,7 +171,9 @@ stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* 
                                  float* gx, int64_t ldgx, stg_stream_t stream);
 /* General form used by both: backward=0 → in-CSR, 1 → out-CSR;
  *   out[r,:] = scale_row[r] · Σ_{c∈row r} scale_col[c] · in[c,:] + bias[:]
- * with scale_row / scale_col / bias each optional (NULL = 1 / 1 / 0). */
+ * with scale_row / scale_col / bias each optional (NULL = 1 / 1 / 0).
+ * In a sharded view the arrays indexed by a DESTINATION vertex hold the local
+ * rows only (forward: out, scale_row; backward: in, scale_col). */
 stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t W,
                                 const float* in, int64_t ldin, float* out, int64_t ldout,
                                 const float* scale_row, const float* scale_col, const float* bias,
@@ -209,15 +220,21 @@ void stg_state_stack_destroy(stg_state_stack* s);
 
 /* Forward step at one timestamp (a7):
  *   P' = diag(n_src)·X·W;  C = diag(n_dst)·A·P' + b;  GRU gates;  H_next.
- * X [V,F], H_prev/H_next [V,H] (all vertices; sharded views compute the local
- * rows of C and H_next only).  stack == NULL: inference, nothing retained. */
+ * X [V,F] (all vertices, resident on every rank), H_prev/H_next [R,H] with
+ * R = row_end-row_begin (R = V unsharded): a sharded view computes P' for all V
+ * sources and C, the GRU and H_next for its R local rows only.
+ * stack == NULL: inference, nothing retained. */
 stg_status stg_tgcn_step(const stg_csr_view* g_fwd, const stg_tgcn_params* p, const float* X,
                          const float* H_prev, float* H_next, stg_state_stack* stack,
                          stg_stream_t stream);
 /* Backward step (a8): pops {H_prev, C} pushed by the matching forward step and,
  * given dH_next = dℓ/dH_t (total), writes dH_prev = dℓ/dH_{t-1} and accumulates
  * parameter gradients.  g_bwd must be the snapshot of the same t (its out-CSR
- * carries dP = Âᵀ·dC).  dH_prev may alias nothing else. */
+ * carries dP = Âᵀ·dC).  dH_prev may alias nothing else.  Sharded: dH_next /
+ * dH_prev are [R,H]; dP holds the partial sums of the local edges for all V
+ * sources, so the accumulated gradients are this rank's share: their sum over
+ * ranks (one all-reduce per sequence, before the optimiser step) is the
+ * whole-graph gradient. */
 stg_status stg_tgcn_step_backward(const stg_csr_view* g_bwd, const stg_tgcn_params* p, const float* X,
                                   const float* dH_next, float* dH_prev, stg_tgcn_grads* grads,
                                   stg_state_stack* stack, stg_stream_t stream);
@@ -229,6 +246,11 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g_bwd, const stg_tgcn_para
 stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o,
                         const float* b_o, float* loss_accum, float* dH, int32_t accumulate,
                         float* dw_o, float* db_o, stg_stream_t stream);
+/* The same over V local rows of a V_total-row graph (sharded): the mean is
+ * taken over V_total, so the per-rank losses and gradients add up. */
+stg_status stg_mse_head_ex(int32_t V, int32_t V_total, int32_t H, const float* Hn, const float* y,
+                           const float* w_o, const float* b_o, float* loss_accum, float* dH,
+                           int32_t accumulate, float* dw_o, float* db_o, stg_stream_t stream);
 
 /* p -= lr·g over n elements, then g = 0 for the next accumulation (the
  * per-sequence optimiser step, reading C17). */
@@ -238,9 +260,10 @@ stg_status stg_sgd_update(float* p, float* g, int64_t n, float lr, stg_stream_t 
  * (DTDG: Get-Graph, graph-stack push; state-stack push; step; loss), then
  * backward in LIFO order (graph-stack pop, Get-Backward-Graph, head gradient,
  * step_backward).  Exactly one of `graph` / `dtdg` is non-NULL.
- * X (host)[S] device pointers to X_t [V,F]; Y (host)[S] device pointers to y_t [V];
- * H0 [V,H] initial state (detached); H_seq [S][V,H] receives H_t (H_seq[S-1] is
- * the state the next sequence starts from, reading C15); G_work [2][V,H] scratch.
+ * X (host)[S] device pointers to X_t [V,F]; Y (host)[S] device pointers to y_t [R];
+ * H0 [R,H] initial state (detached); H_seq [S][R,H] receives H_t (H_seq[S-1] is
+ * the state the next sequence starts from, reading C15); G_work [2][R,H] scratch
+ * (R = the local rows of a sharded graph / dtdg, else V).
  * Gradients (grads, dw_o, db_o) and loss_accum are accumulated. */
 stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
                                    const stg_tgcn_params* p, const float* w_o, const float* b_o,

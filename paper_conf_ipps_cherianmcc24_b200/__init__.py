@@ -97,6 +97,7 @@ _decl("stg_tgcn_step", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn_pa
 _decl("stg_tgcn_step_backward", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn_params), _P, _P, _P,
                                  ctypes.POINTER(stg_tgcn_grads), _P, _P])
 _decl("stg_mse_head", [_i32, _i32, _P, _P, _P, _P, _P, _P, _i32, _P, _P, _P])
+_decl("stg_mse_head_ex", [_i32, _i32, _i32, _P, _P, _P, _P, _P, _P, _i32, _P, _P, _P])
 _decl("stg_sgd_update", [_P, _P, _i64, _f32, _P])
 _decl("stg_tgcn_train_sequence", [_P, _P, _i32, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P,
                                   ctypes.POINTER(_P), ctypes.POINTER(_P), _P, _P, _P,
@@ -115,7 +116,7 @@ ABI_SYMBOLS = [
     "stg_dtdg_num_timestamps", "stg_dtdg_num_deltas", "stg_dtdg_destroy",
     "stg_gcn_aggregate_fwd", "stg_gcn_aggregate_bwd", "stg_gcn_aggregate_ex",
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
-    "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_sgd_update", "stg_tgcn_train_sequence",
+    "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_mse_head_ex", "stg_sgd_update", "stg_tgcn_train_sequence",
     "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
 ]
@@ -224,10 +225,18 @@ class Dtdg:
             pass
 
 
-def stg_static_graph_create(V: int, src, dst, flags: int = 0, stream=None) -> Graph:
+def _dist(dist):
+    """dist = None (whole graph) or (rank, world, row_begin, row_end) -> stg_dist* (SURVEY §8(e))."""
+    if dist is None:
+        return None
+    r, w, b, e = (int(x) for x in dist)
+    return ctypes.byref(stg_dist(r, w, b, e))
+
+
+def stg_static_graph_create(V: int, src, dst, flags: int = 0, stream=None, dist=None) -> Graph:
     s, d = _dev_i32(src), _dev_i32(dst)
     out = ctypes.c_void_p()
-    _check(_lib.stg_static_graph_create(V, s.numel(), _ptr(s), _ptr(d), flags, None, _stream(stream),
+    _check(_lib.stg_static_graph_create(V, s.numel(), _ptr(s), _ptr(d), flags, _dist(dist), _stream(stream),
                                         ctypes.byref(out)))
     return Graph(out)
 
@@ -239,7 +248,7 @@ def stg_graph_view(g: Graph) -> stg_csr_view:
 
 
 def stg_dtdg_create(V: int, T: int, src0, dst0, add_off, add_src, add_dst, del_off, del_src, del_dst,
-                    flags: int = 0, stream=None) -> Dtdg:
+                    flags: int = 0, stream=None, dist=None) -> Dtdg:
     s0, d0 = _dev_i32(src0), _dev_i32(dst0)
     a_s, a_d = _dev_i32(add_src), _dev_i32(add_dst)
     r_s, r_d = _dev_i32(del_src), _dev_i32(del_dst)
@@ -253,7 +262,7 @@ def stg_dtdg_create(V: int, T: int, src0, dst0, add_off, add_src, add_dst, del_o
                                 _ptr(a_d) if a_d.numel() else None,
                                 do.ctypes.data_as(_P), _ptr(r_s) if r_s.numel() else None,
                                 _ptr(r_d) if r_d.numel() else None,
-                                flags, None, _stream(stream), ctypes.byref(out)))
+                                flags, _dist(dist), _stream(stream), ctypes.byref(out)))
     torch.cuda.current_stream().synchronize()
     return Dtdg(out)
 
@@ -387,10 +396,12 @@ def stg_tgcn_step_backward(v: stg_csr_view, params: dict, X, dH_next, grads: dic
     return dH_prev
 
 
-def stg_mse_head(Hn, y, w_o, b_o, loss_accum=None, dH=None, accumulate=False, dw_o=None, db_o=None, stream=None):
+def stg_mse_head(Hn, y, w_o, b_o, loss_accum=None, dH=None, accumulate=False, dw_o=None, db_o=None, stream=None,
+                 V_total=None):
     V, H = Hn.shape
-    _check(_lib.stg_mse_head(V, H, _ptr(Hn), _ptr(y), _ptr(w_o), _ptr(b_o), _ptr(loss_accum), _ptr(dH),
-                             int(accumulate), _ptr(dw_o), _ptr(db_o), _stream(stream)))
+    _check(_lib.stg_mse_head_ex(V, V if V_total is None else int(V_total), H, _ptr(Hn), _ptr(y), _ptr(w_o),
+                                _ptr(b_o), _ptr(loss_accum), _ptr(dH), int(accumulate), _ptr(dw_o), _ptr(db_o),
+                                _stream(stream)))
 
 
 def stg_sgd_update(p: torch.Tensor, g: torch.Tensor, lr: float, stream=None):

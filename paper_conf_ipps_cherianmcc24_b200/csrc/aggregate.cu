@@ -248,6 +248,7 @@ struct Agg2Args {
   int64_t ldy;
   float* partials;
   int32_t* counters;
+  int32_t upad;     // a valid column id for the padding gathers past the stream end
 };
 
 // Strategy 1: software-pipelined degree-ordered items.  A warp serves 32/G
@@ -537,7 +538,7 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
       for (int st = 16; st >= 1; st >>= 1)
         if (lo + st <= 31 && ex[lo + st] <= pos) lo += st;
       k = lo;
-      u = pos < N ? __ldcs(a.col + s_beg[w][lo] + (pos - ex[lo])) : 0;
+      u = pos < N ? __ldcs(a.col + s_beg[w][lo] + (pos - ex[lo])) : a.upad;
     };
     auto flush = [&](int c, const float4& sum) {
       const float sv = __shfl_sync(FULL, sl, c);
@@ -724,6 +725,22 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   if (!a.rowptr || (gv->num_edges > 0 && !a.col))
     return fail(STG_ERR_INVALID_ARG, "aggregate: view lacks the %s CSR", backward ? "backward" : "forward");
   if (a.sched && (!a.ids || !gv->workspace)) a.sched = nullptr;
+  // Sharded views (row block [rb, re)): destination-indexed arrays are local
+  // rows (forward: out, scale_row; backward: in, scale_col), everything else is
+  // global.  Work items carry global vertex ids, so the local arrays are
+  // addressed through bases shifted by -rb rows (the view's in_rowptr is the
+  // local suffix of the global row pointer).
+  const int64_t rb = gv->row_begin;
+  if (rb != 0 && a.ids) {
+    if (!backward) {
+      a.rowptr -= rb;
+      out -= rb * ldout;
+      if (srow) srow -= rb;
+    } else {
+      in -= rb * ldin;
+      if (scol) scol -= rb;
+    }
+  }
   a.srow = srow;
   a.scol = scol;
   a.bias = bias;
@@ -763,6 +780,7 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
       b.partials = a.partials; b.counters = a.counters;
       b.W = wl; b.x = in + c0; b.ldx = ldin; b.y = out + c0; b.ldy = ldout;
       b.bias = bias ? bias + c0 : nullptr;
+      b.upad = (backward && a.ids) ? (int32_t)rb : 0;   // row 0 of a shifted input is not a valid row
       fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(b, ws->queue.p + k);
       k_agg_hubs<<<(unsigned)(4 * num_sms()), 256, 0, s>>>(b, hids);
       count_launch(2);
@@ -822,8 +840,8 @@ stg_status stg_gcn_aggregate_fwd(const stg_csr_view* g, int32_t W, const float* 
 stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* gy, int64_t ldgy, float* gx,
                                  int64_t ldgx, stg_stream_t stream) {
   if (!g) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_bwd: view is NULL");
-  return stg::aggregate_launch(g, 1, W, gy, ldgy, gx, ldgx, g->norm_src, g->norm_dst, nullptr,
-                               (cudaStream_t)stream);
+  return stg::aggregate_launch(g, 1, W, gy, ldgy, gx, ldgx, g->norm_src,
+                               g->norm_dst ? g->norm_dst + g->row_begin : nullptr, nullptr, (cudaStream_t)stream);
 }
 
 stg_status stg_aggregate_set_strategy(int32_t strategy) {

@@ -112,9 +112,17 @@ using namespace stg;
 struct stg_dtdg {
   int32_t V = 0, T = 0, nb = 1;
   uint32_t flags = 0;
-  std::vector<int64_t> E;                          // E_t
+  std::vector<int64_t> E;                          // E_t (edges held: the local block's if sharded)
   std::vector<int64_t> a_off, d_off;               // offsets into the delta arrays, [T+1]
   DArray<uint64_t> add_out, add_in, del_out, del_in;  // effective deltas, packed, sorted per direction
+  // row-block sharding: the deltas above are those of the local
+  // block; the whole-graph effective deltas (src-major) keep the whole-graph
+  // degrees of every slot current for the GCN norms
+  bool sharded = false;
+  int32_t rb = 0, re = 0;
+  int64_t E0_global = 0;
+  std::vector<int64_t> ga_off, gd_off;
+  DArray<uint64_t> gadd, gdel;
   Snapshot slot[5];                                // 0 = base, 1-2 = forward pair, 3-4 = backward pair
   int head_f = -1, head_b = -1;
   DArray<int4> touch_in, touch_out;
@@ -136,6 +144,15 @@ struct stg_dtdg {
     const int32_t t1 = t0 + dirn;
     const int32_t td = dirn > 0 ? t1 : t0;       // batch applied (forward) or undone (reverse)
     const bool rev = dirn < 0;
+    if (sharded) {                                 // whole-graph degrees of slot `to`
+      const size_t vb = sizeof(int32_t) * (size_t)V;
+      STG_CUDA(cudaMemcpyAsync(slot[to].gin_deg.p, slot[from].gin_deg.p, vb, cudaMemcpyDeviceToDevice, s));
+      STG_CUDA(cudaMemcpyAsync(slot[to].gout_deg.p, slot[from].gout_deg.p, vb, cudaMemcpyDeviceToDevice, s));
+      degree_hist(gadd.p + ga_off[td], ga_off[td + 1] - ga_off[td], nb, rev ? -1 : 1, slot[to].gin_deg.p,
+                  slot[to].gout_deg.p, s);
+      degree_hist(gdel.p + gd_off[td], gd_off[td + 1] - gd_off[td], nb, rev ? 1 : -1, slot[to].gin_deg.p,
+                  slot[to].gout_deg.p, s);
+    }
     return apply_delta(slot[from], slot[to], dir(td, true, rev), dir(td, false, rev), E[t1], t1, touch_in.p,
                        touch_out.p, *ws, s);
   }
@@ -174,7 +191,9 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
   if (T < 1) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: T=%d < 1", T);
   if (E0 < 0 || (E0 > 0 && (!src0 || !dst0))) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: bad base edges");
   if (!add_off || !del_off) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: add_off/del_off (host) are NULL");
-  if (dist) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: row-block sharding is not implemented in libstg (see DESIGN.md §Multi-GPU)");
+  if (dist && (dist->row_begin < 0 || dist->row_end > V || dist->row_begin > dist->row_end))
+    return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: row block [%d,%d) outside [0,%d]", dist->row_begin,
+                dist->row_end, V);
   for (int32_t t = 0; t < T; ++t) {
     if (add_off[t + 1] < add_off[t] || del_off[t + 1] < del_off[t])
       return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: offsets decrease at t=%d", t);
@@ -189,6 +208,10 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
 
   auto* g = new stg_dtdg();
   g->V = V; g->T = T; g->flags = flags;
+  g->rb = dist ? dist->row_begin : 0;
+  g->re = dist ? dist->row_end : V;
+  g->sharded = g->rb != 0 || g->re != V;
+  const bool shard = g->sharded;
   g->ws = buildws_create();
   BuildWs& ws = *g->ws;
   int nb = 1;
@@ -261,6 +284,21 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
   DArray<uint64_t> base_keys;
   CK(base_keys.alloc(ns + 1));
   if (st == STG_OK) cudaMemcpyAsync(base_keys.p, S, sizeof(uint64_t) * ns, cudaMemcpyDeviceToDevice, s);
+  // sharded: the local block's edge count per t (E_loc) and the whole-graph deltas
+  std::vector<DArray<uint64_t>> gA(T), gD(T);
+  g->ga_off.assign(T + 1, 0);
+  g->gd_off.assign(T + 1, 0);
+  int64_t e_loc = ns;
+  g->E0_global = ns;
+  if (shard && st == STG_OK) {
+    CK(filter_block(S, ns, nb, true, g->rb, g->re, Salt, cnt.p, ws, s));
+    if (st == STG_OK) {
+      cudaMemcpyAsync(&e_loc, cnt.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+      cudaStreamSynchronize(s);
+    }
+    g->E[0] = e_loc;
+    max_e = e_loc;
+  }
 
   for (int32_t t = 1; t < T && st == STG_OK; ++t) {
     const int64_t na = add_off[t + 1] - add_off[t], nd = del_off[t + 1] - del_off[t];
@@ -306,7 +344,30 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
     std::swap(S, Salt);
     ns = ns - nde + nae;
     g->E[t] = ns;
-    max_e = std::max(max_e, ns);
+    if (shard) {
+      // whole-graph deltas for the degrees; the local block's deltas for the CSRs
+      CK(gA[t].alloc(nae + 1)); CK(gD[t].alloc(nde + 1));
+      if (st == STG_OK) {
+        if (nae) cudaMemcpyAsync(gA[t].p, Ae.p, sizeof(uint64_t) * nae, cudaMemcpyDeviceToDevice, s);
+        if (nde) cudaMemcpyAsync(gD[t].p, De.p, sizeof(uint64_t) * nde, cudaMemcpyDeviceToDevice, s);
+      }
+      g->ga_off[t + 1] = g->ga_off[t] + nae;
+      g->gd_off[t + 1] = g->gd_off[t] + nde;
+      int64_t c3[2] = {0, 0};
+      CK(filter_block(gA[t].p, nae, nb, true, g->rb, g->re, A1.p, cnt.p + 2, ws, s));
+      CK(filter_block(gD[t].p, nde, nb, true, g->rb, g->re, D1.p, cnt.p + 3, ws, s));
+      if (st == STG_OK) {
+        cudaMemcpyAsync(c3, cnt.p + 2, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s);
+        cudaStreamSynchronize(s);
+      }
+      if (nae) cudaMemcpyAsync(Ae.p, A1.p, sizeof(uint64_t) * c3[0], cudaMemcpyDeviceToDevice, s);
+      if (nde) cudaMemcpyAsync(De.p, D1.p, sizeof(uint64_t) * c3[1], cudaMemcpyDeviceToDevice, s);
+      nae = c3[0];
+      nde = c3[1];
+      e_loc += nae - nde;
+      g->E[t] = e_loc;
+    }
+    max_e = std::max(max_e, g->E[t]);
     // keep A'_t, D'_t (src-major order now)
     CK(dA[t].alloc(nae + 1)); CK(dD[t].alloc(nde + 1));
     if (st == STG_OK) {
@@ -338,15 +399,34 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
     }
     dA[t].reset(); dD[t].reset();
   }
+  if (shard) {                                     // whole-graph deltas, contiguous
+    CK(g->gadd.alloc(g->ga_off[T] + 1)); CK(g->gdel.alloc(g->gd_off[T] + 1));
+    for (int32_t t = 1; t < T && st == STG_OK; ++t) {
+      const int64_t na = g->ga_off[t + 1] - g->ga_off[t], nd = g->gd_off[t + 1] - g->gd_off[t];
+      if (na) cudaMemcpyAsync(g->gadd.p + g->ga_off[t], gA[t].p, sizeof(uint64_t) * na, cudaMemcpyDeviceToDevice, s);
+      if (nd) cudaMemcpyAsync(g->gdel.p + g->gd_off[t], gD[t].p, sizeof(uint64_t) * nd, cudaMemcpyDeviceToDevice, s);
+    }
+    if (st == STG_OK) cudaStreamSynchronize(s);
+    for (int32_t t = 0; t < T; ++t) { gA[t].reset(); gD[t].reset(); }
+  }
   // snapshot slots
   const bool eids = (flags & STG_EDGE_IDS) != 0, dgl = (flags & STG_NORM_DGL_BOTH) != 0;
-  for (int i = 0; i < 5 && st == STG_OK; ++i) CK(g->slot[i].alloc(V, max_e, eids, dgl));
+  for (int i = 0; i < 5 && st == STG_OK; ++i) CK(g->slot[i].alloc(V, max_e, eids, dgl, g->rb, g->re));
   CK(g->touch_in.alloc(V)); CK(g->touch_out.alloc(V));
   if (st == STG_OK) {
     cudaMemsetAsync(g->touch_in.p, 0, sizeof(int4) * V, s);
     cudaMemsetAsync(g->touch_out.p, 0, sizeof(int4) * V, s);
     g->slot[0].t = 0;
-    CK(build_from_out_keys(base_keys.p, g->E[0], g->slot[0], ws, s));
+    const uint64_t* bk = base_keys.p;
+    if (shard) {                                   // whole-graph degrees of S_0, local edges of S_0
+      Snapshot& b0 = g->slot[0];
+      cudaMemsetAsync(b0.gin_deg.p, 0, sizeof(int32_t) * V, s);
+      cudaMemsetAsync(b0.gout_deg.p, 0, sizeof(int32_t) * V, s);
+      degree_hist(base_keys.p, g->E0_global, nb, 1, b0.gin_deg.p, b0.gout_deg.p, s);
+      CK(filter_block(base_keys.p, g->E0_global, nb, true, g->rb, g->re, S2.p, cnt.p, ws, s));
+      bk = S2.p;
+    }
+    CK(build_from_out_keys(bk, g->E[0], g->slot[0], ws, s));
   }
   if (st == STG_OK && cudaStreamSynchronize(s) != cudaSuccess)
     st = fail(STG_ERR_CUDA, "stg_dtdg_create: %s", cudaGetErrorString(cudaGetLastError()));

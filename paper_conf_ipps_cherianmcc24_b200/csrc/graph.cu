@@ -16,8 +16,11 @@ static inline unsigned grid_for(int64_t n, int threads, int64_t max_blocks = 148
   return (unsigned)(b < max_blocks ? b : max_blocks);
 }
 
-stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl) {
+stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_t rb_, int32_t re_) {
   V = V_;
+  rb = rb_;
+  re = re_ < 0 ? V_ : re_;
+  sharded = rb != 0 || re != V;
   cap = cap_ > 0 ? cap_ : 1;
   nb = 1;
   while ((int64_t(1) << nb) < (int64_t)V) ++nb;
@@ -32,16 +35,18 @@ stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl) {
   STG_TRY(in_ids.alloc(V)); STG_TRY(out_ids.alloc(V));
   STG_TRY(in_sched.alloc(sc)); STG_TRY(out_sched.alloc(sc));
   STG_TRY(norm_src.alloc(V)); STG_TRY(norm_dst.alloc(V));
+  if (sharded) { STG_TRY(gin_deg.alloc(V)); STG_TRY(gout_deg.alloc(V)); }
   return STG_OK;
 }
 
 void Snapshot::view(stg_csr_view* v, AggWs* ws) const {
   v->num_nodes = V;
-  v->row_begin = 0;
-  v->row_end = V;
+  v->row_begin = rb;
+  v->row_end = re;
   v->timestamp = t;
   v->num_edges = E;
-  v->in_rowptr = in_rowptr.p; v->in_col = in_col.p; v->in_row = in_row.p;
+  // rows below rb are empty, so in_rowptr[rb] = 0: the local row pointer is a suffix
+  v->in_rowptr = in_rowptr.p + rb; v->in_col = in_col.p; v->in_row = in_row.p;
   v->out_rowptr = out_rowptr.p; v->out_col = out_col.p; v->out_row = out_row.p;
   v->out_eid = edge_ids ? out_eid.p : nullptr;
   v->in_deg = in_deg.p; v->out_deg = out_deg.p; v->in_ids = in_ids.p; v->out_ids = out_ids.p;
@@ -84,6 +89,7 @@ __global__ void k_deg(const int32_t* __restrict__ rowptr, int32_t V, int32_t* __
 }
 
 // GCN normalisation vectors (reading C1): IEEE 1/sqrtf, 0 for degree 0.
+// A sharded snapshot passes the whole-graph degrees (gin_deg / gout_deg).
 __global__ void k_norm(const int32_t* __restrict__ in_deg, const int32_t* __restrict__ out_deg, int32_t V,
                        int dgl_both, float* __restrict__ n_src, float* __restrict__ n_dst) {
   for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
@@ -100,11 +106,12 @@ __global__ void k_norm(const int32_t* __restrict__ in_deg, const int32_t* __rest
 }
 
 // node_ids sort keys: ascending (mask - deg) == descending degree; the stable
-// sort keeps ascending ids among equal degrees (reading C4).
-__global__ void k_deg_keys(const int32_t* __restrict__ deg, int32_t V, uint32_t mask, uint32_t* __restrict__ keys,
-                           int32_t* __restrict__ vals) {
+// sort keeps ascending ids among equal degrees (reading C4).  Rows
+// outside [rb, re) (sharded in-direction) get key mask + 1: they sort last.
+__global__ void k_deg_keys(const int32_t* __restrict__ deg, int32_t V, uint32_t mask, int32_t rb, int32_t re,
+                           uint32_t* __restrict__ keys, int32_t* __restrict__ vals) {
   for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
-    keys[v] = mask - (uint32_t)deg[v];
+    keys[v] = (v >= rb && v < re) ? mask - (uint32_t)deg[v] : mask + 1;
     vals[v] = v;
   }
 }
@@ -189,6 +196,44 @@ struct UniqOut {
   }
 };
 
+// ---------------------------------------------------- row-block sharding
+__global__ void k_degree_hist(const uint64_t* __restrict__ keys, int64_t n, int nb, int sign, int32_t* __restrict__ gin,
+                              int32_t* __restrict__ gout) {
+  const uint64_t mask = (uint64_t(1) << nb) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t k = keys[i];
+    atomicAdd(gin + (int32_t)(k & mask), sign);
+    if (gout) atomicAdd(gout + (int32_t)(k >> nb), sign);
+  }
+}
+
+void degree_hist(const uint64_t* keys, int64_t n, int nb, int sign, int32_t* gin, int32_t* gout, cudaStream_t s) {
+  if (n <= 0) return;
+  k_degree_hist<<<grid_for(n, 256), 256, 0, s>>>(keys, n, nb, sign, gin, gout);
+  count_launch();
+}
+
+struct InBlock {
+  const uint64_t* k;
+  int nb;
+  bool dst_low;
+  int32_t rb, re;
+  __device__ int64_t operator()(int64_t i) const {
+    const uint64_t key = k[i];
+    const int32_t d = dst_low ? (int32_t)(key & ((uint64_t(1) << nb) - 1)) : (int32_t)(key >> nb);
+    return d >= rb && d < re;
+  }
+};
+
+stg_status filter_block(const uint64_t* keys, int64_t n, int nb, bool dst_low, int32_t rb, int32_t re, uint64_t* out,
+                        int64_t* d_count, BuildWs& ws, cudaStream_t s) {
+  if (n <= 0) {
+    STG_CUDA(cudaMemsetAsync(d_count, 0, sizeof(int64_t), s));
+    return STG_OK;
+  }
+  return scan(InBlock{keys, nb, dst_low, rb, re}, UniqOut{keys, out}, n, ws.scan, s, d_count);
+}
+
 stg_status sort_unique_keys(uint64_t** keys, uint64_t** alt, int64_t n, int nbits, int64_t* d_count, BuildWs& ws,
                             cudaStream_t s) {
   uint32_t* nov = nullptr;
@@ -210,23 +255,27 @@ stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s) {
     int32_t* deg = dir == 0 ? g.in_deg.p : g.out_deg.p;
     int32_t* ids = dir == 0 ? g.in_ids.p : g.out_ids.p;
     int32_t* sched = dir == 0 ? g.in_sched.p : g.out_sched.p;
+    // rows of this direction's schedule: the local block (in-CSR) or all V sources
+    const bool blk = dir == 0 && g.sharded;
+    const int32_t R = blk ? g.rows() : V;
     uint32_t* k = ws.dkey.p; uint32_t* ka = ws.dkey_alt.p;
     int32_t* vv = ids; int32_t* va = ws.dval_alt.p;
-    k_deg_keys<<<grid_for(V, 256), 256, 0, s>>>(deg, V, mask, k, vv);
+    k_deg_keys<<<grid_for(V, 256), 256, 0, s>>>(deg, V, mask, blk ? g.rb : 0, blk ? g.re : V, k, vv);
     count_launch();
-    STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, dbits, ws.radix, s)));
+    STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, dbits + (blk ? 1 : 0), ws.radix, s)));
     if (vv != ids) {
       STG_CUDA(cudaMemcpyAsync(ids, vv, sizeof(int32_t) * V, cudaMemcpyDeviceToDevice, s));
     }
     const int32_t* rowptr = dir == 0 ? g.in_rowptr.p : g.out_rowptr.p;
     const int64_t coff = sched_cptr_off(V, g.cap);
-    k_sched_count<<<grid_for(m + 1, 256), 256, 0, s>>>(ids, deg, V, m, sched);
+    const int64_t mr = std::min<int64_t>(m, R);
+    k_sched_count<<<grid_for(mr + 1, 256), 256, 0, s>>>(ids, deg, R, mr, sched);
     count_launch();
     // chunk_ptr (exclusive) in cptr[0..m], total chunks in cptr[m] and sched[1]
-    STG_TRY(scan(ChunkIn{ids, deg}, StoreExcl32{sched + coff}, m, ws.scan, s, nullptr, sched + coff + m));
-    STG_CUDA(cudaMemcpyAsync(sched + 1, sched + coff + m, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
+    STG_TRY(scan(ChunkIn{ids, deg}, StoreExcl32{sched + coff}, mr, ws.scan, s, nullptr, sched + coff + mr));
+    STG_CUDA(cudaMemcpyAsync(sched + 1, sched + coff + mr, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
     const int64_t icap = sched_items_cap(V, g.cap);
-    k_items<<<grid_for(icap, 256), 256, 0, s>>>(ids, rowptr, V, icap, coff, sched);
+    k_items<<<grid_for(icap, 256), 256, 0, s>>>(ids, rowptr, R, icap, coff, sched);
     count_launch();
   }
   return check_launch("build_ids_and_sched");
@@ -259,7 +308,9 @@ stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& g, Bui
   k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.in_row.p, E, V, g.in_rowptr.p);
   k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.in_rowptr.p, V, g.in_deg.p);
   k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.out_rowptr.p, V, g.out_deg.p);
-  k_norm<<<grid_for(V, 256), 256, 0, s>>>(g.in_deg.p, g.out_deg.p, V, g.dgl_both, g.norm_src.p, g.norm_dst.p);
+  k_norm<<<grid_for(V, 256), 256, 0, s>>>(g.sharded ? g.gin_deg.p : g.in_deg.p,
+                                         g.sharded ? g.gout_deg.p : g.out_deg.p, V, g.dgl_both, g.norm_src.p,
+                                         g.norm_dst.p);
   count_launch(5);
   STG_TRY(check_launch("build_from_out_keys"));
   STG_TRY(build_ids_and_sched(g, ws, s));
@@ -435,8 +486,9 @@ stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_di
                     ep));
   dst.E = E_new;
   dst.t = t_new;
-  k_norm<<<grid_for(V, 256), 256, 0, s>>>(dst.in_deg.p, dst.out_deg.p, V, dst.dgl_both, dst.norm_src.p,
-                                         dst.norm_dst.p);
+  k_norm<<<grid_for(V, 256), 256, 0, s>>>(dst.sharded ? dst.gin_deg.p : dst.in_deg.p,
+                                         dst.sharded ? dst.gout_deg.p : dst.out_deg.p, V, dst.dgl_both,
+                                         dst.norm_src.p, dst.norm_dst.p);
   count_launch();
   STG_TRY(build_ids_and_sched(dst, ws, s));
   return carry ? check_launch("apply_delta") : build_out_eid(dst, s);
@@ -470,14 +522,17 @@ stg_status stg_static_graph_create(int32_t V, int64_t E, const int32_t* src, con
   if (E + ((flags & STG_SELF_LOOPS) ? V : 0) >= (int64_t(1) << 31))
     return fail(STG_ERR_OUT_OF_RANGE, "stg_static_graph_create: E=%lld >= 2^31", (long long)E);
   if (E > 0 && (!src || !dst)) return fail(STG_ERR_INVALID_ARG, "stg_static_graph_create: src/dst NULL");
-  if (dist) return fail(STG_ERR_INVALID_ARG, "stg_static_graph_create: row-block sharding is not implemented for static graphs");
+  if (dist && (dist->row_begin < 0 || dist->row_end > V || dist->row_begin > dist->row_end))
+    return fail(STG_ERR_INVALID_ARG, "stg_static_graph_create: row block [%d,%d) outside [0,%d]", dist->row_begin,
+                dist->row_end, V);
   cudaStream_t s = (cudaStream_t)stream;
   auto* g = new stg_graph();
   BuildWs ws;
   const int loops = (flags & STG_SELF_LOOPS) ? 1 : 0;
   const int64_t n = E + (loops ? V : 0);
   Snapshot& sn = g->snap;
-  stg_status st = sn.alloc(V, n, (flags & STG_EDGE_IDS) != 0, (flags & STG_NORM_DGL_BOTH) != 0);
+  stg_status st = sn.alloc(V, n, (flags & STG_EDGE_IDS) != 0, (flags & STG_NORM_DGL_BOTH) != 0,
+                           dist ? dist->row_begin : 0, dist ? dist->row_end : -1);
   DArray<uint64_t> k1, k2;
   DArray<int32_t> bad;
   DArray<int64_t> cnt;
@@ -501,6 +556,17 @@ stg_status stg_static_graph_create(int32_t V, int64_t E, const int32_t* src, con
         st = fail(STG_ERR_CUDA, "stg_static_graph_create: %s", cudaGetErrorString(cudaGetLastError()));
     }
     if (st == STG_OK && hbad) st = fail(STG_ERR_OUT_OF_RANGE, "stg_static_graph_create: vertex id outside [0,%d)", V);
+    if (st == STG_OK && sn.sharded) {
+      // whole-graph degrees for the norms, then keep the edges into the local block
+      cudaMemsetAsync(sn.gin_deg.p, 0, sizeof(int32_t) * V, s);
+      cudaMemsetAsync(sn.gout_deg.p, 0, sizeof(int32_t) * V, s);
+      degree_hist(a, E2, sn.nb, 1, sn.gin_deg.p, sn.gout_deg.p, s);
+      st = filter_block(a, E2, sn.nb, true, sn.rb, sn.re, b, cnt.p, ws, s);
+      if (st == STG_OK && (cudaMemcpyAsync(&E2, cnt.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+                           cudaStreamSynchronize(s) != cudaSuccess))
+        st = fail(STG_ERR_CUDA, "stg_static_graph_create: %s", cudaGetErrorString(cudaGetLastError()));
+      std::swap(a, b);
+    }
     if (st == STG_OK) st = build_from_out_keys(a, E2, sn, ws, s);
     if (st == STG_OK && cudaStreamSynchronize(s) != cudaSuccess)
       st = fail(STG_ERR_CUDA, "stg_static_graph_create: %s", cudaGetErrorString(cudaGetLastError()));

@@ -41,17 +41,25 @@ struct AggWs {
   DArray<uint32_t> queue;        // edge-stream work-queue heads, one per column chunk (reset per launch)
 };
 
+// Row-block sharding: a sharded snapshot holds only the edges
+// whose destination lies in [rb, re).  Its CSRs keep global vertex numbering
+// (in-CSR rows outside the block are empty; the out-CSR has all V rows), its
+// in_ids list the local rows first, and the GCN norms come from the degrees
+// of the WHOLE graph (gin_deg / gout_deg), maintained from the global deltas.
 struct Snapshot {
   int32_t V = 0, nb = 1;   // nb: bits per id in packed keys
   int32_t t = -1;
-  int64_t E = 0, cap = 0;  // current edges, edge capacity
-  bool edge_ids = false, dgl_both = false;
+  int32_t rb = 0, re = 0;  // local destination rows [rb, re) (whole graph: [0, V))
+  int64_t E = 0, cap = 0;  // current (local) edges, edge capacity
+  bool edge_ids = false, dgl_both = false, sharded = false;
   DArray<int32_t> in_rowptr, in_col, in_row, in_deg, in_ids;
   DArray<int32_t> out_rowptr, out_col, out_row, out_deg, out_ids, out_eid;
   DArray<int32_t> in_sched, out_sched;  // [sched_size(V, cap)], layout above
+  DArray<int32_t> gin_deg, gout_deg;    // sharded only: whole-graph degrees
   DArray<float> norm_src, norm_dst;
 
-  stg_status alloc(int32_t V_, int64_t cap_, bool eids, bool dgl);
+  stg_status alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_t rb_ = 0, int32_t re_ = -1);
+  int32_t rows() const { return re - rb; }
   void view(stg_csr_view* v, AggWs* ws) const;
 };
 
@@ -59,6 +67,15 @@ struct Snapshot {
 struct BuildWs;
 BuildWs* buildws_create();
 void buildws_destroy(BuildWs*);
+
+// whole-graph degree histograms of packed (src << nb | dst) keys (sign = +1 / -1),
+// added into gin (by dst) and gout (by src; may be NULL)
+void degree_hist(const uint64_t* keys, int64_t n, int nb, int sign, int32_t* gin, int32_t* gout, cudaStream_t s);
+// compact the packed keys whose destination (low nb bits if dst_low, else high) lies in [rb, re);
+// the count is written to *d_count (device)
+stg_status filter_block(const uint64_t* keys, int64_t n, int nb, bool dst_low, int32_t rb, int32_t re,
+                        uint64_t* out, int64_t* d_count, BuildWs& ws, cudaStream_t s);
+
 
 // Build every array of `out` from the sorted unique packed out-keys
 // (src << nb | dst) of the snapshot edge set.  No host synchronisation.

@@ -324,7 +324,7 @@ __global__ void k_reduce_part(const float* __restrict__ part, int32_t nb, int32_
 // rows in flight per warp.  Per-block partials [loss | dw_o (H) | db_o]
 // (fp32 gradients, fp64 loss), reduced in a fixed order by k_mse_reduce.
 template <int LPR>
-__global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t H, const float* __restrict__ Hn,
+__global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t Vn, int32_t H, const float* __restrict__ Hn,
                                                  const float* __restrict__ y, const float* __restrict__ w_o,
                                                  const float* __restrict__ b_o, float* __restrict__ dH, int accumulate,
                                                  int want_grad, double* __restrict__ lpart,
@@ -338,7 +338,7 @@ __global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t H, const flo
   float4 gw = make_float4(0.f, 0.f, 0.f, 0.f);
   float gb = 0.f;
   const float b = b_o[0];
-  const float invV = 1.0f / (float)V;
+  const float invV = 1.0f / (float)Vn;               // mean over the whole graph's Vn rows
   const float4 wo = reinterpret_cast<const float4*>(w_o)[ql];
   const int64_t step = (int64_t)gridDim.x * (kT / 32) * RPW;
   for (int64_t v0 = ((int64_t)blockIdx.x * (kT / 32) + w) * RPW; v0 < V; v0 += step) {
@@ -396,7 +396,7 @@ __global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t H, const flo
 // Fixed-order reduction of the per-block partials: block k < H sums column k
 // of gpart (dw_o), block H the db_o column, block H+1 the loss partials; each
 // thread sums a fixed strided subset, then a fixed shared-memory tree.
-__global__ void __launch_bounds__(256) k_mse_reduce(int32_t nb, int32_t H, int32_t V, const double* __restrict__ lpart,
+__global__ void __launch_bounds__(256) k_mse_reduce(int32_t nb, int32_t H, int32_t Vn, const double* __restrict__ lpart,
                                                     const float* __restrict__ gpart, float* __restrict__ loss,
                                                     float* __restrict__ dw_o, float* __restrict__ db_o) {
   __shared__ double sd[256];
@@ -416,7 +416,7 @@ __global__ void __launch_bounds__(256) k_mse_reduce(int32_t nb, int32_t H, int32
   if (threadIdx.x == 0) {
     if (k < H) { if (dw_o) dw_o[k] += (float)sd[0]; }
     else if (k == H) { if (db_o) db_o[0] += (float)sd[0]; }
-    else if (loss) *loss += (float)(sd[0] / (double)V);
+    else if (loss) *loss += (float)(sd[0] / (double)Vn);
   }
 }
 
@@ -514,12 +514,13 @@ stg_status stg_tgcn_step(const stg_csr_view* g, const stg_tgcn_params* p, const 
                          float* H_next, stg_state_stack* stack, stg_stream_t stream) {
   STG_TRY(check_params(p));
   if (!g || !X || !H_prev || !H_next) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step: NULL argument");
-  if (g->row_begin != 0 || g->row_end != g->num_nodes)
-    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step: sharded views are driven from Python (DESIGN.md §Multi-GPU)");
   cudaStream_t s = (cudaStream_t)stream;
-  const int32_t V = g->num_nodes, F = p->F, H = p->H, H3 = 3 * H;
+  // Sharded views (resident mode): P' for all Vall source rows
+  // (X is resident on every rank), C / GRU / H for the R local rows.
+  const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, F = p->F, H = p->H, H3 = 3 * H;
+  const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
   TgcnWs& ws = stack ? stack->ws : global_ws();
-  STG_TRY(ws.P.alloc((size_t)V * H3));
+  STG_TRY(ws.P.alloc((size_t)Vall * H3));
   float* C = nullptr;
   const size_t cbytes = sizeof(float) * (size_t)V * H3;
   if (stack) {
@@ -537,20 +538,21 @@ stg_status stg_tgcn_step(const stg_csr_view* g, const stg_tgcn_params* p, const 
   {
     ProfScope prof(PH_XW, s);
     if (use_tc) {
-      STG_TRY(tc_xw(V, F, H, X, p->W, g->norm_src, ws.P.p, s));
+      STG_TRY(tc_xw(Vall, F, H, X, p->W, g->norm_src, ws.P.p, s));
     } else {
       const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
       STG_TRY(set_smem(k_xw, smem));
-      const int nb = grid_blocks((const void*)k_xw, smem, (V + 31) / 32);
-      k_xw<<<nb, kT, smem, s>>>(V, F, H3, X, p->W, g->norm_src, ws.P.p);
+      const int nb = grid_blocks((const void*)k_xw, smem, (Vall + 31) / 32);
+      k_xw<<<nb, kT, smem, s>>>(Vall, F, H3, X, p->W, g->norm_src, ws.P.p);
       count_launch();
     }
   }
   // C = diag(n_dst)·A·P' + b
-  STG_TRY(aggregate_launch(g, 0, H3, ws.P.p, H3, C, H3, g->norm_dst, nullptr, p->b, s));
+  STG_TRY(aggregate_launch(g, 0, H3, ws.P.p, H3, C, H3, ndst_loc, nullptr, p->b, s));
   // GRU
   ProfScope prof_gru(PH_GRU_FWD, s);
-  if (use_tc) {
+  if (V == 0) {
+  } else if (use_tc) {
     STG_TRY(tc_gru_fwd(V, H, C, H_prev, p->L, p->l, H_next, s));
   } else if (H <= 32) {
     const size_t smem = gru_fwd_smem(H, 32);
@@ -584,12 +586,15 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
     return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward: NULL gradient pointer");
   if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn_step_backward: state stack is empty");
   const StackEntry e = stack->entries.back();
-  const int32_t V = g->num_nodes, F = p->F, H = p->H, H3 = 3 * H;
+  // sharded views: GRU and dC for the R local rows, dP (partial sums from the
+  // local edges) and dW over all Vall sources
+  const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, F = p->F, H = p->H, H3 = 3 * H;
   if (e.V != V || e.H != H) return fail(STG_ERR_STATE, "stg_tgcn_step_backward: stack top does not match (V,H)");
+  const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
   cudaStream_t s = (cudaStream_t)stream;
   TgcnWs& ws = stack->ws;
-  STG_TRY(ws.dC.alloc((size_t)V * H3));
-  STG_TRY(ws.dP.alloc((size_t)V * H3));
+  STG_TRY(ws.dC.alloc((size_t)V * H3 + 4));
+  STG_TRY(ws.dP.alloc((size_t)Vall * H3));
   if (tc_supported(F, H)) {
     STG_TRY(ws.da.alloc((size_t)V * H3));
     STG_TRY(ws.RH.alloc((size_t)V * H));
@@ -597,14 +602,16 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
     STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
     {
       ProfScope prof(PH_GRU_BWD, s);
-      STG_TRY(tc_gru_bwd(V, H, e.C, e.Hp, dH_next, p->L, p->l, g->norm_dst, ws.dC.p, dH_prev, ws.da.p, ws.RH.p, s));
-      STG_TRY(tc_dl(V, H, e.C, e.Hp, ws.RH.p, ws.da.p, ws.part_tc.p, ws.dl_tmp.p, grads->L, grads->l, grads->b, p->L,
-                    s));
+      if (V > 0) {
+        STG_TRY(tc_gru_bwd(V, H, e.C, e.Hp, dH_next, p->L, p->l, ndst_loc, ws.dC.p, dH_prev, ws.da.p, ws.RH.p, s));
+        STG_TRY(tc_dl(V, H, e.C, e.Hp, ws.RH.p, ws.da.p, ws.part_tc.p, ws.dl_tmp.p, grads->L, grads->l, grads->b,
+                      p->L, s));
+      }
     }
     STG_TRY(aggregate_launch(g, 1, H3, ws.dC.p, H3, ws.dP.p, H3, g->norm_src, nullptr, nullptr, s));
     {
       ProfScope prof(PH_DW, s);
-      STG_TRY(tc_dw(V, F, H, X, ws.dP.p, ws.part_tc.p, ws.dl_tmp.p, grads->W, s));
+      STG_TRY(tc_dw(Vall, F, H, X, ws.dP.p, ws.part_tc.p, ws.dl_tmp.p, grads->W, s));
     }
     STG_TRY(check_launch("stg_tgcn_step_backward"));
     stack->entries.pop_back();
@@ -615,6 +622,7 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
   ProfScope* prof_gru = new ProfScope(PH_GRU_BWD, s);
   const int BR = H <= 32 ? 16 : 4;
   const size_t smem = gru_bwd_smem(H, BR);
+  if (V == 0) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward: empty row block on the SIMT path");
   const int NP = 6 * H * H + 6 * H;
   int nbg;
   if (BR == 16) {
@@ -626,10 +634,10 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
   }
   STG_TRY(ws.part_gru.alloc((size_t)nbg * NP));
   if (BR == 16)
-    k_gru_bwd<16><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, g->norm_dst, ws.dC.p, dH_prev,
+    k_gru_bwd<16><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, ndst_loc, ws.dC.p, dH_prev,
                                         ws.part_gru.p);
   else
-    k_gru_bwd<4><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, g->norm_dst, ws.dC.p, dH_prev,
+    k_gru_bwd<4><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, ndst_loc, ws.dC.p, dH_prev,
                                        ws.part_gru.p);
   count_launch();
   k_reduce_part<<<(NP + 255) / 256, 256, 0, s>>>(ws.part_gru.p, nbg, NP, grads->L, 6 * H * H, grads->l, 3 * H,
@@ -643,9 +651,9 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
     ProfScope prof(PH_DW, s);
     const size_t sm2 = sizeof(float) * (size_t)(32 * F + 32 * H3 + F * H3);
     STG_TRY(set_smem(k_dw, sm2));
-    const int nb = grid_blocks((const void*)k_dw, sm2, (V + 31) / 32);
+    const int nb = grid_blocks((const void*)k_dw, sm2, (Vall + 31) / 32);
     STG_TRY(ws.part_dw.alloc((size_t)nb * F * H3));
-    k_dw<<<nb, kT, sm2, s>>>(V, F, H3, X, ws.dP.p, ws.part_dw.p);
+    k_dw<<<nb, kT, sm2, s>>>(Vall, F, H3, X, ws.dP.p, ws.part_dw.p);
     k_reduce_part<<<(F * H3 + 255) / 256, 256, 0, s>>>(ws.part_dw.p, nb, F * H3, grads->W, F * H3, nullptr, 0,
                                                        nullptr);
     count_launch(2);
@@ -659,7 +667,17 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
 stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o, const float* b_o,
                         float* loss_accum, float* dH, int32_t accumulate, float* dw_o, float* db_o,
                         stg_stream_t stream) {
-  if (V < 1 || H < 1 || H > 128 || H % 4 || !Hn || !y || !w_o || !b_o)
+  return stg_mse_head_ex(V, V, H, Hn, y, w_o, b_o, loss_accum, dH, accumulate, dw_o, db_o, stream);
+}
+
+stg_status stg_mse_head_ex(int32_t V, int32_t V_total, int32_t H, const float* Hn, const float* y, const float* w_o,
+                           const float* b_o, float* loss_accum, float* dH, int32_t accumulate, float* dw_o,
+                           float* db_o, stg_stream_t stream) {
+  if (V_total < 1 || V_total < V)
+    return fail(STG_ERR_INVALID_ARG, "stg_mse_head: V_total=%d must be >= max(1, V=%d)", V_total, V);
+  if (V < 0) return fail(STG_ERR_INVALID_ARG, "stg_mse_head: V=%d < 0", V);
+  if (V == 0) return STG_OK;
+  if (H < 1 || H > 128 || H % 4 || !Hn || !y || !w_o || !b_o)
     return fail(STG_ERR_INVALID_ARG, "stg_mse_head: bad arguments (V=%d H=%d; H %% 4 == 0, H <= 128)", V, H);
   if (((uintptr_t)Hn | (uintptr_t)w_o | (uintptr_t)(dH ? dH : Hn)) % 16)
     return fail(STG_ERR_INVALID_ARG, "stg_mse_head: Hn, w_o, dH must be 16-byte aligned");
@@ -674,14 +692,14 @@ stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, c
   const int want = (dH || dw_o || db_o) ? 1 : 0;
   ProfScope prof(PH_HEAD, s);
   switch (LPR) {
-    case 1: k_mse_head<1><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
-    case 2: k_mse_head<2><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
-    case 4: k_mse_head<4><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
-    case 8: k_mse_head<8><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
-    case 16: k_mse_head<16><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
-    default: k_mse_head<32><<<nb, kT, 0, s>>>(V, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 1: k_mse_head<1><<<nb, kT, 0, s>>>(V, V_total, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 2: k_mse_head<2><<<nb, kT, 0, s>>>(V, V_total, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 4: k_mse_head<4><<<nb, kT, 0, s>>>(V, V_total, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 8: k_mse_head<8><<<nb, kT, 0, s>>>(V, V_total, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    case 16: k_mse_head<16><<<nb, kT, 0, s>>>(V, V_total, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
+    default: k_mse_head<32><<<nb, kT, 0, s>>>(V, V_total, H, Hn, y, w_o, b_o, dH, accumulate, want, ws.lpart.p, ws.gpart.p); break;
   }
-  k_mse_reduce<<<H + 2, 256, 0, s>>>(nb, H, V, ws.lpart.p, ws.gpart.p, loss_accum, want ? dw_o : nullptr,
+  k_mse_reduce<<<H + 2, 256, 0, s>>>(nb, H, V_total, ws.lpart.p, ws.gpart.p, loss_accum, want ? dw_o : nullptr,
                                      want ? db_o : nullptr);
   count_launch(2);
   return check_launch("stg_mse_head");
@@ -739,13 +757,13 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
   int32_t V;
   if (graph) {
     STG_TRY(stg_graph_view(graph, &view));
-    V = view.num_nodes;
   } else {
     if (t0 < 0 || t0 + S > stg_dtdg_num_timestamps(dtdg))
       return fail(STG_ERR_OUT_OF_RANGE, "stg_tgcn_train_sequence: [%d,%d) outside the DTDG", t0, t0 + S);
     STG_TRY(stg_dtdg_get_snapshot(dtdg, t0, stream, &view));
-    V = view.num_nodes;
   }
+  V = view.row_end - view.row_begin;               // local rows (all V unless sharded)
+  const int32_t Vall = view.num_nodes;
   const int32_t H = p->H;
   const size_t VH = (size_t)V * H;
   cudaStream_t ms = (cudaStream_t)stream;
@@ -781,8 +799,8 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     const stg_csr_view& v = views[dtdg ? (i & 1) : 0];
     const float* Hp = i == 0 ? H0 : H_seq + (size_t)(i - 1) * VH;
     STG_TRY(stg_tgcn_step(&v, p, X[i], Hp, H_seq + (size_t)i * VH, stack, stream));   // push + fwdprop
-    STG_TRY(stg_mse_head(V, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr, nullptr,
-                         stream));                                          // loss += loss-fn(out)
+    STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr,
+                            nullptr, stream));                                          // loss += loss-fn(out)
     if (overlap) STG_CUDA(cudaEventRecord(ev_done[i & 1], ms));
   }
   // backward in LIFO order, lines 18-25
@@ -811,7 +829,7 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     }
     const stg_csr_view& v = bviews[dtdg ? (i & 1) : 0];
     // G = dℓ_t/dH_t + dH from step t+1
-    STG_TRY(stg_mse_head(V, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, nullptr, G, 1, dw_o, db_o, stream));
+    STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, nullptr, G, 1, dw_o, db_o, stream));
     STG_TRY(stg_tgcn_step_backward(&v, p, X[i], G, Gn, grads, stack, stream));   // pop + bwdprop
     if (overlap) STG_CUDA(cudaEventRecord(ev_done[i & 1], ms));
     std::swap(G, Gn);

@@ -30,6 +30,18 @@ def row_blocks(rowptr: np.ndarray, world: int) -> list:
     return b
 
 
+def base_row_blocks(V: int, src0, dst0, world: int, self_loops: bool = True) -> list:
+    """Row blocks of a graph given as an edge list (the DTDG base S_0 in bench.py): the
+    in-degrees of the edge SET (duplicates removed, plus the self-loops the library adds
+    with STG_SELF_LOOPS) -> row pointer -> row_blocks."""
+    k = np.unique(np.asarray(src0, np.int64) * V + np.asarray(dst0, np.int64))
+    s, d = k // V, k % V
+    if self_loops:
+        d = d[s != d]
+    deg = np.bincount(d, minlength=V) + (1 if self_loops else 0)
+    return row_blocks(np.concatenate([[0], np.cumsum(deg)]), world)
+
+
 def local_in_csr(rowptr: np.ndarray, col: np.ndarray, lo: int, hi: int):
     """The in-CSR rows [lo, hi) of a snapshot (local row pointer, global column ids)."""
     rp = np.asarray(rowptr, dtype=np.int64)

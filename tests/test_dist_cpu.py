@@ -97,3 +97,57 @@ def test_row_blocks_properties():
             for k in range(world):
                 nnz = rp[b[k + 1]] - rp[b[k]]
                 assert nnz <= E / world + deg.max() + 1
+
+
+def test_base_row_blocks_match_the_oracle_rowptr():
+    """bench.py's partition of the DTDG base (edge list -> edge set + loops -> blocks)
+    equals row_blocks over the oracle's in-CSR row pointer of S_0."""
+    for name in ("C4", "C5s"):
+        cfg = gen.CONFIGS[name]
+        dd = gen.dtdg(cfg)
+        g = oracle.csr(cfg.V, next(oracle.snapshot_sets_fold(dd, self_loops=True)))
+        for world in (2, 3, 8):
+            assert parallel.base_row_blocks(cfg.V, dd.src0, dd.dst0, world) == \
+                parallel.row_blocks(g["in_rowptr"], world), (name, world)
+
+
+def _grad_worker(rank, world, port, q):
+    """Sharded TGCN gradients: rank k's share of every parameter gradient
+    is the sum over its local rows / edges; bench.py all-reduces one flat buffer per
+    sequence.  Here the shares are the fp64 oracle's per-block row sums of a separable
+    gradient (Σ_rows Aᵀ B over the block) and the all-reduce must give the whole sum."""
+    try:
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        V, F, N = 1000, 8, 12
+        A = gen.uniform_pm1(5, 1, V * F).reshape(V, F).astype(np.float64)
+        B = gen.uniform_pm1(5, 2, V * N).reshape(V, N).astype(np.float64)
+        rp = np.arange(V + 1)
+        bounds = parallel.row_blocks(rp, world)
+        lo, hi = bounds[rank], bounds[rank + 1]
+        flat = torch.zeros(F * N + N, dtype=torch.float64)
+        flat[: F * N] = torch.from_numpy((A[lo:hi].T @ B[lo:hi]).ravel())
+        flat[F * N:] = torch.from_numpy(B[lo:hi].sum(0))
+        parallel.allreduce_sum_(flat)
+        ok = np.allclose(flat[: F * N].numpy().reshape(F, N), A.T @ B, rtol=1e-12, atol=1e-12) and \
+            np.allclose(flat[F * N:].numpy(), B.sum(0), rtol=1e-12, atol=1e-12)
+        q.put((rank, bool(ok), None))
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover
+        q.put((rank, False, repr(e)))
+
+
+def test_sharded_gradient_allreduce_world2():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_grad_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, ok, info in res:
+        assert ok, (rank, info)
