@@ -283,7 +283,8 @@ stg_status stg_partition_rows(int32_t V, const int32_t* in_rowptr, int32_t world
  * around each phase (bench.py; the GNN vs graph-update split of Fig. 9,
  * P:L316/L345).  phase: 0 aggregation fwd, 1 aggregation bwd, 2 snapshot
  * build (Get-Graph / Get-Backward-Graph), 3 P' = X·W, 4 GRU fwd, 5 GRU bwd,
- * 6 dW, 7 head.  stg_profile_read synchronises on the recorded events and
+ * 6 dW, 7 head, 8 dL/dl/db reductions.  Phases launched on different streams
+ * may overlap.  stg_profile_read synchronises on the recorded events and
  * returns the accumulated milliseconds and count (reset != 0 clears them). */
 stg_status stg_profile_enable(int32_t on);
 stg_status stg_profile_read(int32_t phase, double* total_ms, int64_t* count, int32_t reset);

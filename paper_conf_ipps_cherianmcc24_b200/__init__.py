@@ -121,7 +121,7 @@ ABI_SYMBOLS = [
     "stg_aggregate_set_param",
 ]
 
-PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head"]
+PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head", "dl"]
 
 
 def stg_profile_enable(on: bool = True):

@@ -92,11 +92,16 @@ int num_sms();
 // SWIZZLE_128B_BASE32B layout).  Encoded through the driver entry point.
 stg_status make_tmap_f32(CUtensorMap* out, const float* base, uint64_t rows, uint64_t cols, uint64_t ld,
                          uint32_t box_cols, uint32_t box_rows, bool atom32 = false);
+// Output (store) map of the per-warp box stores: box [box_rows × box_cols] with
+// the swizzle whose span equals the box row (box_cols·4 = 32 or 64 bytes), see
+// tc::box_off.
+stg_status make_tmap_f32_store(CUtensorMap* out, float* base, uint64_t rows, uint64_t cols, uint64_t ld,
+                               uint32_t box_cols, uint32_t box_rows);
 
 // ---------------------------------------------------------------- profiler
 // Per-phase device time with CUDA events on the launching stream (bench.py and
 // the Fig. 9 breakdown).  Off by default; zero cost when off.
-enum Phase { PH_AGG_FWD = 0, PH_AGG_BWD, PH_SNAPSHOT, PH_XW, PH_GRU_FWD, PH_GRU_BWD, PH_DW, PH_HEAD, PH_COUNT };
+enum Phase { PH_AGG_FWD = 0, PH_AGG_BWD, PH_SNAPSHOT, PH_XW, PH_GRU_FWD, PH_GRU_BWD, PH_DW, PH_HEAD, PH_DL, PH_COUNT };
 bool prof_on();
 cudaEvent_t prof_event();
 void prof_push(int phase, cudaEvent_t a, cudaEvent_t b);

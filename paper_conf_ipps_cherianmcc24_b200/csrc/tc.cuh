@@ -397,5 +397,55 @@ __device__ __forceinline__ void mma_3xtf32_kmajor(uint32_t tmem_d, uint32_t a_hi
   }
 }
 
+// ---- per-warp TMA box stores (outputs leave asynchronously: no register
+// dependency, no LSU store queue).  A warp owns 32 consecutive rows; its box is
+// 32 rows x NCOL fp32 (NCOL*4 = 64 or 32 bytes), stored in shared memory in the
+// TMA SWIZZLE_64B / SWIZZLE_32B layout (16-byte chunk c of row r at
+// r*NCOL*4 + ((c ^ s(r)) << 4)), so the row-per-lane writes are conflict-free.
+template <int NCOL>
+__device__ __forceinline__ uint32_t box_off(int r, int c) {
+  static_assert(NCOL == 16 || NCOL == 8, "box of 64 or 32 bytes");
+  if constexpr (NCOL == 16) return (uint32_t)(r * 64 + ((c ^ ((r >> 1) & 3)) << 4));
+  else return (uint32_t)(r * 32 + ((c ^ ((r >> 2) & 1)) << 4));
+}
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, int c0, int r0, const void* src) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(c0), "r"(r0), "r"(smem_u32(src))
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// Double-buffered per-warp box store: buffers buf[0], buf[1] (each 32*NCOL*4
+// bytes, 1024-aligned); `slot` alternates 0/1 across calls of this warp.
+// Writes v*s (this lane's row) into the free buffer, then lane 0 issues the
+// TMA store of box (c0, r0).  Rows past the tensor end are clipped by TMA.
+template <int NCOL>
+__device__ __forceinline__ void warp_box_store(unsigned char* buf0, int& slot, const float (&v)[NCOL], float s,
+                                               const CUtensorMap* map, int c0, int r0) {
+  constexpr int BYTES = 32 * NCOL * 4;
+  const int lane = threadIdx.x & 31;
+  unsigned char* buf = buf0 + slot * BYTES;
+  if (lane == 0) bulk_wait_read<1>();           // the store that last used this buffer has read it
+  __syncwarp();
+#pragma unroll
+  for (int c = 0; c < NCOL / 4; ++c) {
+    const float4 x = make_float4(s * v[4 * c], s * v[4 * c + 1], s * v[4 * c + 2], s * v[4 * c + 3]);
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(buf + box_off<NCOL>(lane, c))),
+                 "f"(x.x), "f"(x.y), "f"(x.z), "f"(x.w)
+                 : "memory");
+  }
+  fence_proxy_async();
+  __syncwarp();
+  if (lane == 0) {
+    tma_store_2d(map, c0, r0, buf);
+    bulk_commit();
+  }
+  slot ^= 1;
+}
+
 }  // namespace tc
 }  // namespace stg

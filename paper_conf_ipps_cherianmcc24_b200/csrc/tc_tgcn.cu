@@ -449,9 +449,9 @@ struct GruF2 {
   static constexpr int NBC = (H3 + 31) / 32, NBH = (H + 31) / 32;   // boxes per C / H tile
   static constexpr int RAW = (NBC + NBH) * kBox;
   static constexpr int BG = H * 2 * H * 4;
-  static constexpr int STAGE = 32 * tc::kStagePitch<NQ> * 16;
+  static constexpr int OBUF = 2 * 32 * HH * 4;                     // per-warp output box buffers
   static constexpr int WOFF = 2 * RAW;                              // weights after the raw buffers
-  static constexpr int SMEM = WOFF + 6 * BG + 8 * STAGE + 1024;     // + alignment slack
+  static constexpr int SMEM = WOFF + 6 * BG + 8 * OBUF + 1024;      // + alignment slack
   static constexpr uint32_t TCOLS = 13 * H <= 256 ? 256 : 512;
 };
 
@@ -497,7 +497,7 @@ template <int H>
 __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_constant__ CUtensorMap tmC,
                                                         const __grid_constant__ CUtensorMap tmH,
                                                         const float* __restrict__ L, const float* __restrict__ l,
-                                                        float* __restrict__ Hn) {
+                                                        const __grid_constant__ CUtensorMap tmHn) {
   using G = GruF2<H>;
   constexpr int HH = G::HH, NQ = G::NQ;
   extern __shared__ unsigned char sm_raw[];
@@ -511,7 +511,8 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
   auto rawH = [&](int b) { return sm + (size_t)b * G::RAW + G::NBC * kBox; };
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, hf = warp >> 2;
   const int lr = q * 32 + lane, c0 = hf * HH;
-  float4* stage = reinterpret_cast<float4*>(bh_lo + G::BG) + warp * 32 * tc::kStagePitch<NQ>;
+  unsigned char* obuf = bh_lo + G::BG + warp * G::OBUF;          // this warp's two output box buffers
+  int oslot = 0;
   const int LG = 2 * H * H;
   stage_gate_weights<H>(bz_hi, bz_lo, L);
   stage_gate_weights<H>(br_hi, br_lo, L + LG);
@@ -546,7 +547,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
   uint32_t mph = 0;
   int i = 0;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
-    const int b = i & 1, r0 = tile * 128, nv = min(128, V - r0);
+    const int b = i & 1, r0 = tile * 128;
     tc::mbar_wait(&full[b], (i >> 1) & 1);
     // raw tile -> tensor-memory A operands; this thread's half of H stays in registers
     float h[HH];
@@ -601,24 +602,18 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
     mph ^= 1;
     tc::fence_after();
     {
-      float ah[HH];
+      float ah[HH], o[HH];
       tmem_row_load<HH>(tm + 12 * H, c0, ah);
-      float4* srow = stage + lane * tc::kStagePitch<NQ>;
 #pragma unroll
-      for (int qq = 0; qq < NQ; ++qq) {
-        float o[4];
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const int j = 4 * qq + e;
-          const float hh = tanhf(ah[j] + lh[j]);
-          o[e] = z[j] * h[j] + (1.0f - z[j]) * hh;
-        }
-        srow[qq] = make_float4(o[0], o[1], o[2], o[3]);
+      for (int j = 0; j < HH; ++j) {
+        const float hh = tanhf(ah[j] + lh[j]);
+        o[j] = z[j] * h[j] + (1.0f - z[j]) * hh;
       }
-      tc::flush_stage_rows<NQ>(stage, Hn + c0, H, r0 + q * 32, nv - q * 32);
+      tc::warp_box_store<HH>(obuf, oslot, o, 1.0f, &tmHn, c0, r0 + q * 32);    // H'
     }
     tc::fence_before();
   }
+  if (lane == 0) tc::bulk_wait_all();                // output boxes written before the CTA exits
   __syncthreads();
   if (warp == 0) tc::tmem_free(tm, G::TCOLS);
 }
@@ -789,9 +784,9 @@ struct GruB2 {
   static constexpr int NBC = (H3 + 31) / 32, NBH = (H + 31) / 32;
   static constexpr int RAW = (NBC + 2 * NBH) * kBox;                // C, H, G
   static constexpr int BG = H * 2 * H * 4;
-  static constexpr int STAGE = 32 * tc::kStagePitch<NQ> * 16;
+  static constexpr int OBUF = 2 * 32 * HH * 4;                     // per-warp output box buffers
   static constexpr int WOFF = RAW;
-  static constexpr int SMEM = WOFF + 12 * BG + 8 * STAGE + 1024;
+  static constexpr int SMEM = WOFF + 12 * BG + 8 * OBUF + 1024;
   static constexpr uint32_t TCOLS = 13 * H <= 256 ? 256 : 512;
 };
 
@@ -826,11 +821,13 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
                                                         const __grid_constant__ CUtensorMap tmH,
                                                         const __grid_constant__ CUtensorMap tmG,
                                                         const float* __restrict__ L, const float* __restrict__ l,
-                                                        const float* __restrict__ ndst, float* __restrict__ dCs,
-                                                        float* __restrict__ dHp, float* __restrict__ da,
-                                                        float* __restrict__ RHo) {
+                                                        const float* __restrict__ ndst,
+                                                        const __grid_constant__ CUtensorMap tmDC,
+                                                        const __grid_constant__ CUtensorMap tmDH,
+                                                        const __grid_constant__ CUtensorMap tmDA,
+                                                        const __grid_constant__ CUtensorMap tmRH) {
   using G = GruB2<H>;
-  constexpr int H3 = G::H3, HH = G::HH, NQ = G::NQ;
+  constexpr int H3 = G::H3, HH = G::HH;
   extern __shared__ unsigned char sm_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full, mma_bar;
@@ -847,7 +844,10 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
   unsigned char* rawG = sm + (G::NBC + G::NBH) * kBox;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, hf = warp >> 2;
   const int lr = q * 32 + lane, c0 = hf * HH;
-  float4* stage = reinterpret_cast<float4*>(w0 + 12 * G::BG) + warp * 32 * tc::kStagePitch<NQ>;
+  unsigned char* obuf = w0 + 12 * G::BG + warp * G::OBUF;       // this warp's two output box buffers
+  int oslot = 0;
+  __shared__ float s_l[3 * H];                                   // gate biases
+  for (int e = threadIdx.x; e < 3 * H; e += blockDim.x) s_l[e] = l[e];
   const int LG = 2 * H * H;
   stage_gate_weights<H>(bz_hi, bz_lo, L);
   stage_gate_weights<H>(br_hi, br_lo, L + LG);
@@ -890,7 +890,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
   uint32_t mph = 0;
   int i = 0;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
-    const int r0 = tile * 128, nv = min(128, V - r0), wr0 = r0 + q * 32, wnv = nv - q * 32;
+    const int r0 = tile * 128, wr0 = r0 + q * 32;
     const int row = r0 + lr;
     const float nd = row < V ? __ldg(ndst + row) : 0.f;
     tc::mbar_wait(&full, i & 1);
@@ -927,8 +927,8 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
       tmem_row_load<HH>(tm + 9 * H, c0, ar);
 #pragma unroll
       for (int j = 0; j < HH; ++j) {
-        z[j] = sigm(az[j] + __ldg(l + c0 + j));
-        r[j] = sigm(ar[j] + __ldg(l + H + c0 + j));
+        z[j] = sigm(az[j] + s_l[c0 + j]);
+        r[j] = sigm(ar[j] + s_l[H + c0 + j]);
         rh[j] = r[j] * h[j];
       }
       tmem_st_split<HH>(tq + 10 * H + c0, tq + 11 * H + c0, rh);
@@ -940,7 +940,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
         mma_ts_seg(tm + 12 * H, tm + 10 * H, tm + 11 * H, hh_, hl, 2 * H, H, H, id_h, false);
         tc::commit(&mma_bar);
       }
-      stage_flush<HH>(stage, rh, 1.0f, RHo + c0, H, wr0, wnv);            // RH (for dL_h²), overlaps P2
+      tc::warp_box_store<HH>(obuf, oslot, rh, 1.0f, &tmRH, c0, wr0);       // RH (for dL_h²), overlaps P2
     }
     mma_wait(mph);
     float dh[HH];
@@ -949,7 +949,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
       tmem_row_load<HH>(tm + 12 * H, c0, ah);
 #pragma unroll
       for (int j = 0; j < HH; ++j) {
-        const float hh = tanhf(ah[j] + __ldg(l + 2 * H + c0 + j));
+        const float hh = tanhf(ah[j] + s_l[2 * H + c0 + j]);
         const float dZ = g[j] * (h[j] - hh), dHh = g[j] * (1.0f - z[j]);
         dah[j] = dHh * (1.0f - hh * hh);
         daz[j] = dZ * z[j] * (1.0f - z[j]);
@@ -965,8 +965,8 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
         mma_ts_seg(tm + 6 * H, tm + 2 * H, tm + 3 * H, tc::smem_u32(lz_hi), tc::smem_u32(lz_lo), H, 0, H, id_2h, true);
         tc::commit(&mma_bar);
       }
-      stage_flush<HH>(stage, daz, 1.0f, da + c0, H3, wr0, wnv);            // da_z
-      stage_flush<HH>(stage, dah, 1.0f, da + 2 * H + c0, H3, wr0, wnv);    // da_h
+      tc::warp_box_store<HH>(obuf, oslot, daz, 1.0f, &tmDA, c0, wr0);      // da_z
+      tc::warp_box_store<HH>(obuf, oslot, dah, 1.0f, &tmDA, 2 * H + c0, wr0);   // da_h
     }
     mma_wait(mph);
     {
@@ -985,14 +985,14 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
         mma_ts_seg(tm + 8 * H, tm + 10 * H, tm + 11 * H, tc::smem_u32(lr_hi), tc::smem_u32(lr_lo), H, 0, H, id_2h, true);
         tc::commit(&mma_bar);
       }
-      stage_flush<HH>(stage, dch, nd, dCs + 2 * H + c0, H3, wr0, wnv);     // dC'_h
-      stage_flush<HH>(stage, dar, 1.0f, da + H + c0, H3, wr0, wnv);        // da_r
+      tc::warp_box_store<HH>(obuf, oslot, dch, nd, &tmDC, 2 * H + c0, wr0);     // dC'_h
+      tc::warp_box_store<HH>(obuf, oslot, dar, 1.0f, &tmDA, H + c0, wr0);  // da_r
       float dcz[HH], dhz[HH];
       tmem_row_load<HH>(tm + 6 * H, c0, dcz);          // dC_z
       tmem_row_load<HH>(tm + 7 * H, c0, dhz);          // dH_z
 #pragma unroll
       for (int j = 0; j < HH; ++j) dh[j] += dhz[j];
-      stage_flush<HH>(stage, dcz, nd, dCs + c0, H3, wr0, wnv);             // dC'_z
+      tc::warp_box_store<HH>(obuf, oslot, dcz, nd, &tmDC, c0, wr0);        // dC'_z
     }
     mma_wait(mph);
     {
@@ -1001,12 +1001,13 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
       tmem_row_load<HH>(tm + 9 * H, c0, dhr);          // dH_r
 #pragma unroll
       for (int j = 0; j < HH; ++j) dh[j] += dhr[j];
-      stage_flush<HH>(stage, dcr, nd, dCs + H + c0, H3, wr0, wnv);         // dC'_r
-      stage_flush<HH>(stage, dh, 1.0f, dHp + c0, H, wr0, wnv);             // dH_prev
+      tc::warp_box_store<HH>(obuf, oslot, dcr, nd, &tmDC, H + c0, wr0);    // dC'_r
+      tc::warp_box_store<HH>(obuf, oslot, dh, 1.0f, &tmDH, c0, wr0);       // dH_prev
     }
     tc::fence_before();
     __syncthreads();                                   // TMEM / stage reuse by the next tile
   }
+  if (lane == 0) tc::bulk_wait_all();                // output boxes written before the CTA exits
   if (warp == 0) tc::tmem_free(tm, G::TCOLS);
 }
 
@@ -1392,15 +1393,16 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
                       cudaStream_t s) {
   const int ntiles = (V + 127) / 128;
   const int nb = std::min(ntiles, num_sms());
-  CUtensorMap tmC, tmH;
+  CUtensorMap tmC, tmH, tmHn;
   STG_TRY(make_tmap_f32(&tmC, C, (uint64_t)V, 3 * H, 3 * H, 32, 128));
   STG_TRY(make_tmap_f32(&tmH, Hp, (uint64_t)V, H, H, 32, 128));
+  STG_TRY(make_tmap_f32_store(&tmHn, Hn, (uint64_t)V, H, H, (uint32_t)H / 2, 32));
   if (H == 32) {
     STG_TRY(prep(k_tc_gru_fwd2<32>, GruF2<32>::SMEM));
-    k_tc_gru_fwd2<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, Hn);
+    k_tc_gru_fwd2<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
   } else {
     STG_TRY(prep(k_tc_gru_fwd2<16>, GruF2<16>::SMEM));
-    k_tc_gru_fwd2<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, Hn);
+    k_tc_gru_fwd2<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
   }
   count_launch();
   return check_launch("tc_gru_fwd");
@@ -1410,16 +1412,21 @@ stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float
                       const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s) {
   const int ntiles = (V + 127) / 128;
   const int nb = std::min(ntiles, num_sms());
-  CUtensorMap tmC, tmH, tmG;
+  CUtensorMap tmC, tmH, tmG, tmDC, tmDH, tmDA, tmRH;
   STG_TRY(make_tmap_f32(&tmC, C, (uint64_t)V, 3 * H, 3 * H, 32, 128));
   STG_TRY(make_tmap_f32(&tmH, Hp, (uint64_t)V, H, H, 32, 128));
   STG_TRY(make_tmap_f32(&tmG, G, (uint64_t)V, H, H, 32, 128));
+  const uint32_t hh = (uint32_t)H / 2;                  // output boxes: 32 rows x H/2 columns per warp
+  STG_TRY(make_tmap_f32_store(&tmDC, dCs, (uint64_t)V, 3 * H, 3 * H, hh, 32));
+  STG_TRY(make_tmap_f32_store(&tmDH, dHp, (uint64_t)V, H, H, hh, 32));
+  STG_TRY(make_tmap_f32_store(&tmDA, da, (uint64_t)V, 3 * H, 3 * H, hh, 32));
+  STG_TRY(make_tmap_f32_store(&tmRH, RH, (uint64_t)V, H, H, hh, 32));
   if (H == 32) {
     STG_TRY(prep(k_tc_gru_bwd2<32>, GruB2<32>::SMEM));
-    k_tc_gru_bwd2<32><<<nb, 256, GruB2<32>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, dCs, dHp, da, RH);
+    k_tc_gru_bwd2<32><<<nb, 256, GruB2<32>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, tmDC, tmDH, tmDA, tmRH);
   } else {
     STG_TRY(prep(k_tc_gru_bwd2<16>, GruB2<16>::SMEM));
-    k_tc_gru_bwd2<16><<<nb, 256, GruB2<16>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, dCs, dHp, da, RH);
+    k_tc_gru_bwd2<16><<<nb, 256, GruB2<16>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, tmDC, tmDH, tmDA, tmRH);
   }
   count_launch();
   return check_launch("tc_gru_bwd");
@@ -1461,7 +1468,10 @@ static stg_status atb2_stages(const CUtensorMap* m, const CUtensorMap& ones, con
                               cudaStream_t s) {
   constexpr int RT = 32;
   const size_t stage = (size_t)2 * (sp.nsa + NB) * RT * 32 * 4;
-  const size_t cap = 220 * 1024;
+  static const size_t cap = [] {                    // ring budget (experiments: STG_ATB_SMEM_KB)
+    const char* v = getenv("STG_ATB_SMEM_KB");
+    return (size_t)(v ? atoi(v) : 220) * 1024;
+  }();
   if (4 * stage <= cap) return atb2_launch<NB, RT, 4>(m, ones, sp, nb, s);
   if (3 * stage <= cap) return atb2_launch<NB, RT, 3>(m, ones, sp, nb, s);
   return atb2_launch<NB, RT, 2>(m, ones, sp, nb, s);

@@ -489,6 +489,150 @@ static size_t gru_bwd_smem(int H, int BR) {
   return sizeof(float) * (6 * H * H + 3 * H + BR * 3 * H + 8 * BR * H + BR * 3 * H + 6 * H * H + 6 * H);
 }
 
+static size_t stack_bytes(int32_t V, int32_t H) {
+  return (sizeof(float) * (size_t)V * 3 * H + 255) & ~size_t(255);
+}
+
+// ---- the TGCN step in stream-explicit pieces (stg_tgcn_step runs them on one
+// stream; stg_tgcn_train_sequence pipelines them over several, see there).
+// Sharded views (resident mode): P' for all Vall source rows
+// (X is resident on every rank), C / GRU / H for the V = R local rows.
+
+// P' = diag(n_src)·X·W (all Vall rows) and C = diag(n_dst)·A·P' + b (local rows)
+static stg_status fwd_conv(const stg_csr_view* g, const stg_tgcn_params* p, const float* X, float* P, float* C,
+                           cudaStream_t s) {
+  const int32_t Vall = g->num_nodes, F = p->F, H = p->H, H3 = 3 * H;
+  {
+    ProfScope prof(PH_XW, s);
+    if (tc_supported(F, H)) {
+      STG_TRY(tc_xw(Vall, F, H, X, p->W, g->norm_src, P, s));
+    } else {
+      const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
+      STG_TRY(set_smem(k_xw, smem));
+      const int nb = grid_blocks((const void*)k_xw, smem, (Vall + 31) / 32);
+      k_xw<<<nb, kT, smem, s>>>(Vall, F, H3, X, p->W, g->norm_src, P);
+      count_launch();
+    }
+  }
+  const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
+  return aggregate_launch(g, 0, H3, P, H3, C, H3, ndst_loc, nullptr, p->b, s);
+}
+
+// GRU over V local rows: H_next from C and H_prev
+static stg_status fwd_gru(int32_t V, const stg_tgcn_params* p, const float* C, const float* H_prev, float* H_next,
+                          cudaStream_t s) {
+  const int32_t H = p->H;
+  ProfScope prof_gru(PH_GRU_FWD, s);
+  if (V == 0) return STG_OK;
+  if (tc_supported(p->F, H)) {
+    STG_TRY(tc_gru_fwd(V, H, C, H_prev, p->L, p->l, H_next, s));
+  } else if (H <= 32) {
+    const size_t smem = gru_fwd_smem(H, 32);
+    STG_TRY(set_smem(k_gru_fwd<32>, smem));
+    const int nb = grid_blocks((const void*)k_gru_fwd<32>, smem, (V + 31) / 32);
+    k_gru_fwd<32><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
+    count_launch();
+  } else {
+    const size_t smem = gru_fwd_smem(H, 16);
+    STG_TRY(set_smem(k_gru_fwd<16>, smem));
+    const int nb = grid_blocks((const void*)k_gru_fwd<16>, smem, (V + 15) / 16);
+    k_gru_fwd<16><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
+    count_launch();
+  }
+  return check_launch("tgcn fwd_gru");
+}
+
+// Backward buffers of one step (buffer set k of ws): dC' [V,3H], dP [Vall,3H],
+// and on the tensor-core path da [V,3H], RH [V,H]
+struct BwdBufs {
+  float *dC[2], *dP[2], *da[2], *RH[2];
+};
+
+static stg_status bwd_alloc(TgcnWs& ws, const stg_csr_view* g, const stg_tgcn_params* p, int nsets, BwdBufs* b) {
+  const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, H = p->H, H3 = 3 * H;
+  const size_t nC = ((size_t)V * H3 + 64) & ~size_t(63), nP = ((size_t)Vall * H3 + 64) & ~size_t(63);
+  const size_t nR = ((size_t)V * H + 64) & ~size_t(63);
+  STG_TRY(ws.dC.alloc(nC * nsets));
+  STG_TRY(ws.dP.alloc(nP * nsets));
+  const bool tc = tc_supported(p->F, H);
+  if (tc) {
+    STG_TRY(ws.da.alloc(nC * nsets));
+    STG_TRY(ws.RH.alloc(nR * nsets));
+    STG_TRY(ws.part_tc.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));
+    STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
+  }
+  for (int k = 0; k < 2; ++k) {
+    const int kk = k < nsets ? k : 0;
+    b->dC[k] = ws.dC.p + kk * nC;
+    b->dP[k] = ws.dP.p + kk * nP;
+    b->da[k] = tc ? ws.da.p + kk * nC : nullptr;
+    b->RH[k] = tc ? ws.RH.p + kk * nR : nullptr;
+  }
+  return STG_OK;
+}
+
+// GRU backward over the V local rows into buffer set 0 of `bb` (dC', da, RH)
+// and dH_prev.  SIMT path: also the dL, dl, db partials (fused in its kernel).
+static stg_status bwd_gru(const stg_csr_view* g, const stg_tgcn_params* p, const float* C, const float* Hp,
+                          const float* dH_next, float* dH_prev, stg_tgcn_grads* grads, TgcnWs& ws,
+                          const BwdBufs& bb, cudaStream_t s) {
+  const int32_t V = g->row_end - g->row_begin, H = p->H;
+  const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
+  ProfScope prof(PH_GRU_BWD, s);
+  if (V == 0) return STG_OK;
+  if (tc_supported(p->F, H))
+    return tc_gru_bwd(V, H, C, Hp, dH_next, p->L, p->l, ndst_loc, bb.dC[0], dH_prev, bb.da[0], bb.RH[0], s);
+  const int BR = H <= 32 ? 16 : 4;
+  const size_t smem = gru_bwd_smem(H, BR);
+  const int NP = 6 * H * H + 6 * H;
+  int nbg;
+  if (BR == 16) {
+    STG_TRY(set_smem(k_gru_bwd<16>, smem));
+    nbg = grid_blocks((const void*)k_gru_bwd<16>, smem, (V + 15) / 16);
+  } else {
+    STG_TRY(set_smem(k_gru_bwd<4>, smem));
+    nbg = grid_blocks((const void*)k_gru_bwd<4>, smem, (V + 3) / 4);
+  }
+  STG_TRY(ws.part_gru.alloc((size_t)nbg * NP));
+  if (BR == 16)
+    k_gru_bwd<16><<<nbg, kT, smem, s>>>(V, H, C, Hp, dH_next, p->L, p->l, ndst_loc, bb.dC[0], dH_prev,
+                                        ws.part_gru.p);
+  else
+    k_gru_bwd<4><<<nbg, kT, smem, s>>>(V, H, C, Hp, dH_next, p->L, p->l, ndst_loc, bb.dC[0], dH_prev,
+                                       ws.part_gru.p);
+  count_launch();
+  k_reduce_part<<<(NP + 255) / 256, 256, 0, s>>>(ws.part_gru.p, nbg, NP, grads->L, 6 * H * H, grads->l, 3 * H,
+                                                 grads->b);
+  count_launch();
+  return check_launch("tgcn bwd_gru");
+}
+
+// The parameter-gradient reductions of one step from buffer set 0 of `bb`:
+// dL, dl, db = Σ_rows [C|H]ᵀda, [RH|1]ᵀda (tensor-core path), dP = diag(n_src)·Aᵀ·dC'
+// over the out-CSR, dW += Xᵀ·dP.
+static stg_status bwd_grads(const stg_csr_view* g, const stg_tgcn_params* p, const float* X, const float* C,
+                            const float* Hp, stg_tgcn_grads* grads, TgcnWs& ws, const BwdBufs& bb, cudaStream_t s) {
+  const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, F = p->F, H = p->H, H3 = 3 * H;
+  const bool tc = tc_supported(F, H);
+  if (tc && V > 0) {
+    ProfScope prof(PH_DL, s);
+    STG_TRY(tc_dl(V, H, C, Hp, bb.RH[0], bb.da[0], ws.part_tc.p, ws.dl_tmp.p, grads->L, grads->l, grads->b, p->L,
+                  s));
+  }
+  STG_TRY(aggregate_launch(g, 1, H3, bb.dC[0], H3, bb.dP[0], H3, g->norm_src, nullptr, nullptr, s));
+  ProfScope prof(PH_DW, s);
+  if (tc) return tc_dw(Vall, F, H, X, bb.dP[0], ws.part_tc.p, ws.dl_tmp.p, grads->W, s);
+  const size_t sm2 = sizeof(float) * (size_t)(32 * F + 32 * H3 + F * H3);
+  STG_TRY(set_smem(k_dw, sm2));
+  const int nb = grid_blocks((const void*)k_dw, sm2, (Vall + 31) / 32);
+  STG_TRY(ws.part_dw.alloc((size_t)nb * F * H3));
+  k_dw<<<nb, kT, sm2, s>>>(Vall, F, H3, X, bb.dP[0], ws.part_dw.p);
+  k_reduce_part<<<(F * H3 + 255) / 256, 256, 0, s>>>(ws.part_dw.p, nb, F * H3, grads->W, F * H3, nullptr, 0,
+                                                     nullptr);
+  count_launch(2);
+  return check_launch("tgcn bwd_grads");
+}
+
 extern "C" {
 
 stg_status stg_state_stack_create(int64_t capacity_bytes, stg_state_stack** out) {
@@ -515,61 +659,23 @@ stg_status stg_tgcn_step(const stg_csr_view* g, const stg_tgcn_params* p, const 
   STG_TRY(check_params(p));
   if (!g || !X || !H_prev || !H_next) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step: NULL argument");
   cudaStream_t s = (cudaStream_t)stream;
-  // Sharded views (resident mode): P' for all Vall source rows
-  // (X is resident on every rank), C / GRU / H for the R local rows.
-  const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, F = p->F, H = p->H, H3 = 3 * H;
-  const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
+  const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, H = p->H, H3 = 3 * H;
   TgcnWs& ws = stack ? stack->ws : global_ws();
   STG_TRY(ws.P.alloc((size_t)Vall * H3));
   float* C = nullptr;
-  const size_t cbytes = sizeof(float) * (size_t)V * H3;
+  const size_t need = stack_bytes(V, H);
   if (stack) {
-    const size_t need = (cbytes + 255) & ~size_t(255);
     if (stack->top + need > stack->cap)
       return fail(STG_ERR_NO_MEMORY, "stg_tgcn_step: state stack full (%zu + %zu > %zu bytes)", stack->top, need,
                   stack->cap);
     C = reinterpret_cast<float*>(stack->arena.p + stack->top);
   } else {
-    STG_TRY(ws.dC.alloc((size_t)V * H3));
+    STG_TRY(ws.dC.alloc((size_t)V * H3 + 4));
     C = ws.dC.p;
   }
-  const bool use_tc = tc_supported(F, H);
-  // P' = diag(n_src)·X·W
-  {
-    ProfScope prof(PH_XW, s);
-    if (use_tc) {
-      STG_TRY(tc_xw(Vall, F, H, X, p->W, g->norm_src, ws.P.p, s));
-    } else {
-      const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
-      STG_TRY(set_smem(k_xw, smem));
-      const int nb = grid_blocks((const void*)k_xw, smem, (Vall + 31) / 32);
-      k_xw<<<nb, kT, smem, s>>>(Vall, F, H3, X, p->W, g->norm_src, ws.P.p);
-      count_launch();
-    }
-  }
-  // C = diag(n_dst)·A·P' + b
-  STG_TRY(aggregate_launch(g, 0, H3, ws.P.p, H3, C, H3, ndst_loc, nullptr, p->b, s));
-  // GRU
-  ProfScope prof_gru(PH_GRU_FWD, s);
-  if (V == 0) {
-  } else if (use_tc) {
-    STG_TRY(tc_gru_fwd(V, H, C, H_prev, p->L, p->l, H_next, s));
-  } else if (H <= 32) {
-    const size_t smem = gru_fwd_smem(H, 32);
-    STG_TRY(set_smem(k_gru_fwd<32>, smem));
-    const int nb = grid_blocks((const void*)k_gru_fwd<32>, smem, (V + 31) / 32);
-    k_gru_fwd<32><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
-    count_launch();
-  } else {
-    const size_t smem = gru_fwd_smem(H, 16);
-    STG_TRY(set_smem(k_gru_fwd<16>, smem));
-    const int nb = grid_blocks((const void*)k_gru_fwd<16>, smem, (V + 15) / 16);
-    k_gru_fwd<16><<<nb, kT, smem, s>>>(V, H, C, H_prev, p->L, p->l, H_next);
-    count_launch();
-  }
-  STG_TRY(check_launch("stg_tgcn_step"));
+  STG_TRY(fwd_conv(g, p, X, ws.P.p, C, s));
+  STG_TRY(fwd_gru(V, p, C, H_prev, H_next, s));
   if (stack) {
-    const size_t need = (cbytes + 255) & ~size_t(255);
     stack->entries.push_back(StackEntry{H_prev, C, V, H, need});
     stack->top += need;
   }
@@ -586,79 +692,13 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
     return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward: NULL gradient pointer");
   if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn_step_backward: state stack is empty");
   const StackEntry e = stack->entries.back();
-  // sharded views: GRU and dC for the R local rows, dP (partial sums from the
-  // local edges) and dW over all Vall sources
-  const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, F = p->F, H = p->H, H3 = 3 * H;
+  const int32_t V = g->row_end - g->row_begin, H = p->H;
   if (e.V != V || e.H != H) return fail(STG_ERR_STATE, "stg_tgcn_step_backward: stack top does not match (V,H)");
-  const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
   cudaStream_t s = (cudaStream_t)stream;
-  TgcnWs& ws = stack->ws;
-  STG_TRY(ws.dC.alloc((size_t)V * H3 + 4));
-  STG_TRY(ws.dP.alloc((size_t)Vall * H3));
-  if (tc_supported(F, H)) {
-    STG_TRY(ws.da.alloc((size_t)V * H3));
-    STG_TRY(ws.RH.alloc((size_t)V * H));
-    STG_TRY(ws.part_tc.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));
-    STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
-    {
-      ProfScope prof(PH_GRU_BWD, s);
-      if (V > 0) {
-        STG_TRY(tc_gru_bwd(V, H, e.C, e.Hp, dH_next, p->L, p->l, ndst_loc, ws.dC.p, dH_prev, ws.da.p, ws.RH.p, s));
-        STG_TRY(tc_dl(V, H, e.C, e.Hp, ws.RH.p, ws.da.p, ws.part_tc.p, ws.dl_tmp.p, grads->L, grads->l, grads->b,
-                      p->L, s));
-      }
-    }
-    STG_TRY(aggregate_launch(g, 1, H3, ws.dC.p, H3, ws.dP.p, H3, g->norm_src, nullptr, nullptr, s));
-    {
-      ProfScope prof(PH_DW, s);
-      STG_TRY(tc_dw(Vall, F, H, X, ws.dP.p, ws.part_tc.p, ws.dl_tmp.p, grads->W, s));
-    }
-    STG_TRY(check_launch("stg_tgcn_step_backward"));
-    stack->entries.pop_back();
-    stack->top -= e.bytes;
-    return STG_OK;
-  }
-  // GRU backward + partials of dL, dl, db
-  ProfScope* prof_gru = new ProfScope(PH_GRU_BWD, s);
-  const int BR = H <= 32 ? 16 : 4;
-  const size_t smem = gru_bwd_smem(H, BR);
-  if (V == 0) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward: empty row block on the SIMT path");
-  const int NP = 6 * H * H + 6 * H;
-  int nbg;
-  if (BR == 16) {
-    STG_TRY(set_smem(k_gru_bwd<16>, smem));
-    nbg = grid_blocks((const void*)k_gru_bwd<16>, smem, (V + 15) / 16);
-  } else {
-    STG_TRY(set_smem(k_gru_bwd<4>, smem));
-    nbg = grid_blocks((const void*)k_gru_bwd<4>, smem, (V + 3) / 4);
-  }
-  STG_TRY(ws.part_gru.alloc((size_t)nbg * NP));
-  if (BR == 16)
-    k_gru_bwd<16><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, ndst_loc, ws.dC.p, dH_prev,
-                                        ws.part_gru.p);
-  else
-    k_gru_bwd<4><<<nbg, kT, smem, s>>>(V, H, e.C, e.Hp, dH_next, p->L, p->l, ndst_loc, ws.dC.p, dH_prev,
-                                       ws.part_gru.p);
-  count_launch();
-  k_reduce_part<<<(NP + 255) / 256, 256, 0, s>>>(ws.part_gru.p, nbg, NP, grads->L, 6 * H * H, grads->l, 3 * H,
-                                                 grads->b);
-  count_launch();
-  delete prof_gru;
-  // dP = diag(n_src)·Aᵀ·(n_dst ⊙ dC) over the out-CSR
-  STG_TRY(aggregate_launch(g, 1, H3, ws.dC.p, H3, ws.dP.p, H3, g->norm_src, nullptr, nullptr, s));
-  // dW += Xᵀ·dP
-  {
-    ProfScope prof(PH_DW, s);
-    const size_t sm2 = sizeof(float) * (size_t)(32 * F + 32 * H3 + F * H3);
-    STG_TRY(set_smem(k_dw, sm2));
-    const int nb = grid_blocks((const void*)k_dw, sm2, (Vall + 31) / 32);
-    STG_TRY(ws.part_dw.alloc((size_t)nb * F * H3));
-    k_dw<<<nb, kT, sm2, s>>>(Vall, F, H3, X, ws.dP.p, ws.part_dw.p);
-    k_reduce_part<<<(F * H3 + 255) / 256, 256, 0, s>>>(ws.part_dw.p, nb, F * H3, grads->W, F * H3, nullptr, 0,
-                                                       nullptr);
-    count_launch(2);
-  }
-  STG_TRY(check_launch("stg_tgcn_step_backward"));
+  BwdBufs bb;
+  STG_TRY(bwd_alloc(stack->ws, g, p, 1, &bb));
+  STG_TRY(bwd_gru(g, p, e.C, e.Hp, dH_next, dH_prev, grads, stack->ws, bb, s));
+  STG_TRY(bwd_grads(g, p, X, e.C, e.Hp, grads, stack->ws, bb, s));
   stack->entries.pop_back();
   stack->top -= e.bytes;
   return STG_OK;
@@ -715,18 +755,20 @@ stg_status stg_sgd_update(float* p, float* g, int64_t n, float lr, stg_stream_t 
 }
 
 namespace {
-// per-device side stream and sequence events of stg_tgcn_train_sequence
-cudaStream_t side_stream() {
+// per-device side streams (0: snapshot builds, 1: the pipelined compute) and
+// sequence events of stg_tgcn_train_sequence
+cudaStream_t side_stream(int which) {
   static std::mutex mu;
-  static std::map<int, cudaStream_t> streams;
+  static std::map<std::pair<int, int>, cudaStream_t> streams;
   int dev = 0;
   cudaGetDevice(&dev);
   std::lock_guard<std::mutex> lk(mu);
-  auto it = streams.find(dev);
+  auto key = std::make_pair(dev, which);
+  auto it = streams.find(key);
   if (it != streams.end()) return it->second;
   cudaStream_t s = nullptr;
   cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
-  return streams[dev] = s;
+  return streams[key] = s;
 }
 cudaEvent_t seq_event(int k) {
   static std::mutex mu;
@@ -741,8 +783,28 @@ cudaEvent_t seq_event(int k) {
   cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
   return evs[key] = e;
 }
+bool pipeline_enabled() {
+  static const bool on = [] {
+    const char* v = getenv("STG_SEQ_PIPELINE");
+    return !(v && v[0] == '0');
+  }();
+  return on;
+}
 }  // namespace
 
+// Algorithm 1 for one sequence, scheduled over three streams (streams instead of
+// a tracing compiler).  Per timestamp the work splits into a GRU chain that
+// carries H (forward GRU + head; backward head + GRU) and H-independent work:
+//   forward : Get-Graph(t+1) [snapshot stream SS] -> P' = XW, C = ÂP'+b [aux A]
+//             -> GRU(t), head(t) [caller stream M]
+//   backward: Get-Backward-Graph(t-1) [SS]; head(t), GRU bwd(t) [M]
+//             -> dL/dl/db, dP = Âᵀ dC', dW [A]
+// so the X·W and aggregations of t+1 (forward) and the reductions, backward
+// aggregation and dW of t (backward) overlap the GRU chain.  Events order
+// every reuse: snapshot slot pairs (a build waits for the last reader of its
+// slot), the two backward buffer sets (GRU bwd(t) waits for the reductions of
+// t+2), and the stack arena (a new sequence starts after the old one joined).
+// Same arithmetic in the same order as the single-stream stg_tgcn_step path.
 stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
                                    const stg_tgcn_params* p, const float* w_o, const float* b_o,
                                    const float* const* X, const float* const* Y, const float* H0, float* H_seq,
@@ -752,9 +814,10 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence: exactly one of graph / dtdg must be given");
   if (S < 1 || !X || !Y || !H0 || !H_seq || !G_work || !stack)
     return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence: bad arguments");
+  if (!grads || !grads->W || !grads->b || !grads->L || !grads->l)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence: NULL gradient pointer");
   STG_TRY(check_params(p));
   stg_csr_view view;
-  int32_t V;
   if (graph) {
     STG_TRY(stg_graph_view(graph, &view));
   } else {
@@ -762,78 +825,98 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
       return fail(STG_ERR_OUT_OF_RANGE, "stg_tgcn_train_sequence: [%d,%d) outside the DTDG", t0, t0 + S);
     STG_TRY(stg_dtdg_get_snapshot(dtdg, t0, stream, &view));
   }
-  V = view.row_end - view.row_begin;               // local rows (all V unless sharded)
-  const int32_t Vall = view.num_nodes;
-  const int32_t H = p->H;
+  const int32_t V = view.row_end - view.row_begin;  // local rows (all V unless sharded)
+  const int32_t Vall = view.num_nodes, H = p->H;
   const size_t VH = (size_t)V * H;
   cudaStream_t ms = (cudaStream_t)stream;
-  // Snapshot builds (Get-Graph / Get-Backward-Graph) of the NEXT timestamp run on a side
-  // stream while the current timestamp's TGCN step runs on `stream`: the build of t+1 writes
-  // the other slot of the snapshot pair, after the step that last read that slot (t-1) is
-  // done; step t+1 waits for its build.  (Streams instead of a tracing compiler.)
-  const bool overlap = dtdg != nullptr && S > 1;
-  cudaStream_t ss = overlap ? side_stream() : nullptr;
-  cudaEvent_t ev_done[2] = {nullptr, nullptr}, ev_built[2] = {nullptr, nullptr};
-  if (overlap) {
-    for (int k = 0; k < 2; ++k) { ev_done[k] = seq_event(2 * k); ev_built[k] = seq_event(2 * k + 1); }
-    STG_CUDA(cudaEventRecord(ev_done[1], ms));      // everything before this sequence (incl. Get-Graph(t0))
+  const bool pipe = pipeline_enabled();
+  cudaStream_t as = pipe ? side_stream(1) : ms;
+  cudaStream_t ss = (dtdg && pipe) ? side_stream(0) : ms;
+  // every buffer is sized before any asynchronous use (grow-only reallocations
+  // would free memory another stream may still read)
+  TgcnWs& ws = stack->ws;
+  STG_TRY(ws.P.alloc((size_t)Vall * 3 * H));
+  BwdBufs bb;
+  STG_TRY(bwd_alloc(ws, &view, p, 2, &bb));
+  const size_t need = stack_bytes(V, H);
+  if (stack->top + (size_t)S * need > stack->cap)
+    return fail(STG_ERR_NO_MEMORY, "stg_tgcn_train_sequence: state stack too small (%zu + %d x %zu > %zu bytes)",
+                stack->top, S, need, stack->cap);
+  cudaEvent_t ev_start = seq_event(0), ev_conv[2] = {seq_event(1), seq_event(2)};
+  cudaEvent_t ev_built[2] = {seq_event(3), seq_event(4)}, ev_gru[2] = {seq_event(5), seq_event(6)};
+  cudaEvent_t ev_bdone[2] = {seq_event(7), seq_event(8)};
+  auto wait = [](cudaStream_t st, cudaEvent_t e, cudaStream_t rec) -> stg_status {
+    if (st != rec) STG_CUDA(cudaStreamWaitEvent(st, e, 0));
+    return STG_OK;
+  };
+  auto record = [](cudaEvent_t e, cudaStream_t st) -> stg_status {
+    STG_CUDA(cudaEventRecord(e, st));
+    return STG_OK;
+  };
+  if (pipe) {
+    STG_TRY(record(ev_start, ms));                       // Get-Graph(t0) and everything before
+    STG_TRY(wait(as, ev_start, ms));
+    if (ss != ms) STG_TRY(wait(ss, ev_start, ms));
   }
   std::vector<int32_t> graph_stack;
   stg_csr_view views[2] = {view, view};
-  // forward, Algorithm 1 lines 7-16
+  // ---- forward, Algorithm 1 lines 7-16
   for (int32_t i = 0; i < S; ++i) {
     const int32_t t = t0 + i;
-    if (dtdg) {
-      if (overlap) {
-        if (i + 1 < S) {                                                    // prefetch Get-Graph(t+1)
-          STG_CUDA(cudaStreamWaitEvent(ss, ev_done[(i + 1) & 1], 0));       // step t-1 (slot reuse) done
-          STG_TRY(stg_dtdg_get_snapshot(dtdg, t + 1, ss, &views[(i + 1) & 1]));
-          STG_CUDA(cudaEventRecord(ev_built[(i + 1) & 1], ss));
-        }
-        if (i > 0) STG_CUDA(cudaStreamWaitEvent(ms, ev_built[i & 1], 0));
-      } else if (i > 0) {
-        STG_TRY(stg_dtdg_get_snapshot(dtdg, t, stream, &views[i & 1]));    // Get-Graph (Alg. 2)
-      }
-      graph_stack.push_back(t);                                             // graph-stack.push(t)
+    const int k = dtdg ? (i & 1) : 0;
+    float* C = reinterpret_cast<float*>(stack->arena.p + stack->top);   // state-stack.push target
+    if (dtdg && i > 0) STG_TRY(wait(as, ev_built[i & 1], ss));
+    STG_TRY(fwd_conv(&views[k], p, X[i], ws.P.p, C, as));               // P', C (H-independent)
+    STG_TRY(record(ev_conv[i & 1], as));
+    if (dtdg && i + 1 < S) {                                            // prefetch Get-Graph(t+1)
+      if (i >= 1) STG_TRY(wait(ss, ev_conv[(i + 1) & 1], as));          // conv(t-1) done with that slot
+      STG_TRY(stg_dtdg_get_snapshot(dtdg, t + 1, ss, &views[(i + 1) & 1]));
+      STG_TRY(record(ev_built[(i + 1) & 1], ss));
     }
-    const stg_csr_view& v = views[dtdg ? (i & 1) : 0];
+    if (dtdg) graph_stack.push_back(t);                                 // graph-stack.push(t)
+    STG_TRY(wait(ms, ev_conv[i & 1], as));
     const float* Hp = i == 0 ? H0 : H_seq + (size_t)(i - 1) * VH;
-    STG_TRY(stg_tgcn_step(&v, p, X[i], Hp, H_seq + (size_t)i * VH, stack, stream));   // push + fwdprop
+    STG_TRY(fwd_gru(V, p, C, Hp, H_seq + (size_t)i * VH, ms));           // fwdprop
+    stack->entries.push_back(StackEntry{Hp, C, V, H, need});
+    stack->top += need;
     STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr,
-                            nullptr, stream));                                          // loss += loss-fn(out)
-    if (overlap) STG_CUDA(cudaEventRecord(ev_done[i & 1], ms));
+                            nullptr, stream));                          // loss += loss-fn(out)
   }
-  // backward in LIFO order, lines 18-25
+  // ---- backward in LIFO order, lines 18-25
   float* G = G_work;
   float* Gn = G_work + VH;
   STG_CUDA(cudaMemsetAsync(G, 0, sizeof(float) * VH, ms));
   stg_csr_view bviews[2] = {views[0], views[1]};
-  if (dtdg) {
-    const int32_t t = graph_stack.back();
-    STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, t, ss ? ss : ms, &bviews[(S - 1) & 1]));   // the forward head
-    if (overlap) STG_CUDA(cudaEventRecord(ev_built[(S - 1) & 1], ss));
-  }
+  if (dtdg) STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, graph_stack.back(), ms, &bviews[(S - 1) & 1]));  // the head
   for (int32_t i = S - 1; i >= 0; --i) {
+    const int b = i & 1;
     if (dtdg) {
-      graph_stack.pop_back();                                               // graph-stack.pop()
-      if (overlap) {
-        if (i > 0) {                                                        // prefetch Get-Backward-Graph(t-1)
-          STG_CUDA(cudaStreamWaitEvent(ss, ev_done[(i + 1) & 1], 0));       // step t+1 (slot reuse) done
-          STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, graph_stack.back(), ss, &bviews[(i - 1) & 1]));
-          STG_CUDA(cudaEventRecord(ev_built[(i - 1) & 1], ss));
-        }
-        STG_CUDA(cudaStreamWaitEvent(ms, ev_built[i & 1], 0));
-      } else if (i < S - 1) {
-        STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, t0 + i, stream, &bviews[i & 1]));   // Get-Backward-Graph
+      graph_stack.pop_back();                                           // graph-stack.pop()
+      if (i > 0) {                                                      // prefetch Get-Backward-Graph(t-1)
+        if (i + 1 <= S - 1) STG_TRY(wait(ss, ev_bdone[(i + 1) & 1], as));   // step t+1 done with that slot
+        STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, graph_stack.back(), ss, &bviews[(i - 1) & 1]));
+        STG_TRY(record(ev_built[(i - 1) & 1], ss));
       }
+      if (i < S - 1) STG_TRY(wait(ms, ev_built[i & 1], ss));
     }
+    if (i + 2 <= S - 1) STG_TRY(wait(ms, ev_bdone[b], as));             // buffer set b free (step t+2)
     const stg_csr_view& v = bviews[dtdg ? (i & 1) : 0];
     // G = dℓ_t/dH_t + dH from step t+1
     STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, nullptr, G, 1, dw_o, db_o, stream));
-    STG_TRY(stg_tgcn_step_backward(&v, p, X[i], G, Gn, grads, stack, stream));   // pop + bwdprop
-    if (overlap) STG_CUDA(cudaEventRecord(ev_done[i & 1], ms));
+    if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn_train_sequence: state stack underflow");
+    const StackEntry e = stack->entries.back();                         // state-stack.pop()
+    BwdBufs sb = bb;
+    sb.dC[0] = bb.dC[b]; sb.dP[0] = bb.dP[b]; sb.da[0] = bb.da[b]; sb.RH[0] = bb.RH[b];
+    STG_TRY(bwd_gru(&v, p, e.C, e.Hp, G, Gn, grads, ws, sb, ms));       // bwdprop: the H chain
+    STG_TRY(record(ev_gru[b], ms));
+    STG_TRY(wait(as, ev_gru[b], ms));
+    STG_TRY(bwd_grads(&v, p, X[i], e.C, e.Hp, grads, ws, sb, as));      // parameter gradients
+    STG_TRY(record(ev_bdone[b], as));
+    stack->entries.pop_back();
+    stack->top -= e.bytes;
     std::swap(G, Gn);
   }
+  for (int b = 0; b < 2 && b < S; ++b) STG_TRY(wait(ms, ev_bdone[b], as));   // join
   return STG_OK;
 }
 
