@@ -149,6 +149,22 @@ stg_status stg_dtdg_get_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, st
  * reached from the backward cursor by reverse updates, without disturbing the
  * cached forward head (which the next sequence starts from). */
 stg_status stg_dtdg_get_backward_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, stg_csr_view* out);
+/* Snapshot parts (stg_dtdg_get_snapshot_parts): a pass that needs one CSR
+ * direction asks for that one only — the forward in-CSR for Get-Graph, the
+ * reverse out-CSR for Get-Backward-Graph — and the library delta-merges only
+ * that direction per step.  A cached snapshot that lacks a requested
+ * direction gets it by a stable transpose of the one it has (Algorithm 3,
+ * P:L218-251, in the canonical order of reading C7).  Degrees and norms are
+ * always current (whole-graph degree histograms of the deltas). */
+enum { STG_PART_IN = 1u << 0, STG_PART_OUT = 1u << 1, STG_PART_EID = 1u << 2 /* implies both */ };
+/* Get-Graph (backward = 0) / Get-Backward-Graph (backward = 1) of the parts in
+ * `parts` (STG_PART_*; at least one direction).  The view's pointers of the
+ * parts not requested may be NULL (in_rowptr/in_col/in_row/in_ids/in_sched
+ * for the in-CSR, likewise out_*; out_eid unless STG_PART_EID).  Same
+ * validity and stream rules as stg_dtdg_get_snapshot, which equals
+ * parts = IN|OUT|EID (EID only with STG_EDGE_IDS). */
+stg_status stg_dtdg_get_snapshot_parts(stg_dtdg* g, int32_t t, int32_t backward, uint32_t parts,
+                                       stg_stream_t stream, stg_csr_view* out);
 int64_t stg_dtdg_num_edges(const stg_dtdg* g, int32_t t);    /* edges held at t (the local block's if sharded); -1 if t out of range */
 int32_t stg_dtdg_num_timestamps(const stg_dtdg* g);
 /* Number of effective added / deleted edges of step t (0 for t = 0). */

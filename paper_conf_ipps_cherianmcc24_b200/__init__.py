@@ -21,6 +21,7 @@ STG_SELF_LOOPS = 1 << 0
 STG_EDGE_IDS = 1 << 1
 STG_VALIDATE = 1 << 2
 STG_NORM_DGL_BOTH = 1 << 3
+STG_PART_IN, STG_PART_OUT, STG_PART_EID = 1 << 0, 1 << 1, 1 << 2
 
 STATUS = {0: "STG_OK", 1: "STG_ERR_INVALID_ARG", 2: "STG_ERR_OUT_OF_RANGE", 3: "STG_ERR_NO_MEMORY",
           4: "STG_ERR_CUDA", 5: "STG_ERR_NCCL", 6: "STG_ERR_STATE"}
@@ -83,6 +84,7 @@ _decl("stg_graph_destroy", [_P], None)
 _decl("stg_dtdg_create", [_i32, _i32, _i64, _P, _P, _P, _P, _P, _P, _P, _P, _u32, _P, _P, ctypes.POINTER(_P)])
 _decl("stg_dtdg_get_snapshot", [_P, _i32, _P, ctypes.POINTER(stg_csr_view)])
 _decl("stg_dtdg_get_backward_snapshot", [_P, _i32, _P, ctypes.POINTER(stg_csr_view)])
+_decl("stg_dtdg_get_snapshot_parts", [_P, _i32, _i32, _u32, _P, ctypes.POINTER(stg_csr_view)])
 _decl("stg_dtdg_num_edges", [_P, _i32], _i64)
 _decl("stg_dtdg_num_timestamps", [_P], _i32)
 _decl("stg_dtdg_num_deltas", [_P, _i32, _i32], _i64)
@@ -112,7 +114,8 @@ _decl("stg_profile_read", [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER
 ABI_SYMBOLS = [
     "stg_last_error", "stg_version", "stg_kernel_launch_count", "stg_set_allocator", "stg_memcpy",
     "stg_static_graph_create", "stg_graph_view", "stg_graph_destroy",
-    "stg_dtdg_create", "stg_dtdg_get_snapshot", "stg_dtdg_get_backward_snapshot", "stg_dtdg_num_edges",
+    "stg_dtdg_create", "stg_dtdg_get_snapshot", "stg_dtdg_get_backward_snapshot", "stg_dtdg_get_snapshot_parts",
+    "stg_dtdg_num_edges",
     "stg_dtdg_num_timestamps", "stg_dtdg_num_deltas", "stg_dtdg_destroy",
     "stg_gcn_aggregate_fwd", "stg_gcn_aggregate_bwd", "stg_gcn_aggregate_ex",
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
@@ -270,6 +273,13 @@ def stg_dtdg_create(V: int, T: int, src0, dst0, add_off, add_src, add_dst, del_o
 def stg_dtdg_get_snapshot(d: Dtdg, t: int, stream=None) -> stg_csr_view:
     v = stg_csr_view()
     _check(_lib.stg_dtdg_get_snapshot(d.handle, t, _stream(stream), ctypes.byref(v)))
+    return v
+
+
+def stg_dtdg_get_snapshot_parts(d: Dtdg, t: int, parts: int, backward: bool = False, stream=None) -> stg_csr_view:
+    """Get-Graph / Get-Backward-Graph of only the CSR parts in `parts` (STG_PART_*)."""
+    v = stg_csr_view()
+    _check(_lib.stg_dtdg_get_snapshot_parts(d.handle, t, int(backward), parts, _stream(stream), ctypes.byref(v)))
     return v
 
 

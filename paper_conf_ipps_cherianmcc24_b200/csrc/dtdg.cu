@@ -138,27 +138,30 @@ struct stg_dtdg {
     return DirDelta{D, nd, A, na};
   }
 
-  // one delta step from slot `from` (time t0) to slot `to` (time t0 ± 1)
-  stg_status step(int from, int to, int dirn, cudaStream_t s) {
+  // one delta step from slot `from` (time t0) to slot `to` (time t0 ± 1) of the
+  // CSR directions in `parts`; the whole-graph degrees (norms) always follow
+  stg_status step(int from, int to, int dirn, uint32_t parts, cudaStream_t s) {
     const int32_t t0 = slot[from].t;
     const int32_t t1 = t0 + dirn;
     const int32_t td = dirn > 0 ? t1 : t0;       // batch applied (forward) or undone (reverse)
     const bool rev = dirn < 0;
-    if (sharded) {                                 // whole-graph degrees of slot `to`
-      const size_t vb = sizeof(int32_t) * (size_t)V;
-      STG_CUDA(cudaMemcpyAsync(slot[to].gin_deg.p, slot[from].gin_deg.p, vb, cudaMemcpyDeviceToDevice, s));
-      STG_CUDA(cudaMemcpyAsync(slot[to].gout_deg.p, slot[from].gout_deg.p, vb, cudaMemcpyDeviceToDevice, s));
-      degree_hist(gadd.p + ga_off[td], ga_off[td + 1] - ga_off[td], nb, rev ? -1 : 1, slot[to].gin_deg.p,
-                  slot[to].gout_deg.p, s);
-      degree_hist(gdel.p + gd_off[td], gd_off[td + 1] - gd_off[td], nb, rev ? 1 : -1, slot[to].gin_deg.p,
-                  slot[to].gout_deg.p, s);
-    }
+    const uint64_t* ga = sharded ? gadd.p : add_out.p;
+    const uint64_t* gd = sharded ? gdel.p : del_out.p;
+    const std::vector<int64_t>& gao = sharded ? ga_off : a_off;
+    const std::vector<int64_t>& gdo = sharded ? gd_off : d_off;
+    const size_t vb = sizeof(int32_t) * (size_t)V;
+    STG_CUDA(cudaMemcpyAsync(slot[to].gin_deg.p, slot[from].gin_deg.p, vb, cudaMemcpyDeviceToDevice, s));
+    STG_CUDA(cudaMemcpyAsync(slot[to].gout_deg.p, slot[from].gout_deg.p, vb, cudaMemcpyDeviceToDevice, s));
+    degree_hist(ga + gao[td], gao[td + 1] - gao[td], nb, rev ? -1 : 1, slot[to].gin_deg.p, slot[to].gout_deg.p, s);
+    degree_hist(gd + gdo[td], gdo[td + 1] - gdo[td], nb, rev ? 1 : -1, slot[to].gin_deg.p, slot[to].gout_deg.p, s);
     return apply_delta(slot[from], slot[to], dir(td, true, rev), dir(td, false, rev), E[t1], t1, touch_in.p,
-                       touch_out.p, *ws, s);
+                       touch_out.p, *ws, s, parts & (PART_IN | PART_OUT));
   }
 
-  // walk from the best cached slot to t, writing into the pair {p0, p0+1}
-  stg_status walk(int32_t t, int p0, int& out, cudaStream_t s) {
+  // Walk from the best cached slot to t, writing into the pair {p0, p0+1}, for
+  // the CSR directions in `parts` (the starting slot is completed first by a
+  // transpose if it lacks one of them); labels (PART_EID) are added at the end.
+  stg_status walk(int32_t t, int p0, uint32_t parts, int& out, cudaStream_t s) {
     ProfScope prof(PH_SNAPSHOT, s);
     int cands[3] = {p0 == 1 ? head_f : head_b, p0 == 1 ? head_b : head_f, 0};
     int best = -1;
@@ -169,12 +172,43 @@ struct stg_dtdg {
       if (d < bd) { bd = d; best = c; }
     }
     int cur = best;
+    const uint32_t dirs = parts & (PART_IN | PART_OUT);
+    if (slot[cur].t != t || (slot[cur].parts & dirs) != dirs)
+      STG_TRY(complete_parts(slot[cur], dirs, *ws, s));
     while (slot[cur].t != t) {
       int to = (cur == p0) ? p0 + 1 : p0;
-      STG_TRY(step(cur, to, slot[cur].t < t ? 1 : -1, s));
+      STG_TRY(step(cur, to, slot[cur].t < t ? 1 : -1, dirs, s));
       cur = to;
     }
+    STG_TRY(complete_parts(slot[cur], parts, *ws, s));
     out = cur;
+    return STG_OK;
+  }
+
+  stg_status get(int32_t t, bool backward, uint32_t parts, cudaStream_t s, stg_csr_view* v) {
+    int idx = -1;
+    if (!backward) {
+      if (t == 0 && head_f < 0) {
+        idx = 0;
+        ProfScope prof(PH_SNAPSHOT, s);
+        STG_TRY(complete_parts(slot[0], parts, *ws, s));
+      } else {
+        STG_TRY(walk(t, 1, parts, idx, s));
+        if (idx == 1 || idx == 2) head_f = idx;  // a 0-step hit on base/backward slots leaves the head
+      }
+    } else {
+      if (head_f >= 0 && slot[head_f].t == t) idx = head_f;       // forward head is t itself
+      else if (head_b >= 0 && slot[head_b].t == t) idx = head_b;
+      else if (t == 0) idx = 0;
+      if (idx >= 0) {
+        ProfScope prof(PH_SNAPSHOT, s);
+        STG_TRY(complete_parts(slot[idx], parts, *ws, s));
+      } else {
+        STG_TRY(walk(t, 3, parts, idx, s));
+        if (idx >= 3) head_b = idx;
+      }
+    }
+    slot[idx].view(v, &agg);
     return STG_OK;
   }
 };
@@ -439,31 +473,25 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
 stg_status stg_dtdg_get_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, stg_csr_view* out) {
   if (!g || !out) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_get_snapshot: NULL argument");
   if (t < 0 || t >= g->T) return fail(STG_ERR_OUT_OF_RANGE, "stg_dtdg_get_snapshot: t=%d outside [0,%d)", t, g->T);
-  int idx = 0;
-  if (t == 0 && g->head_f < 0) {
-    idx = 0;
-  } else {
-    STG_TRY(g->walk(t, 1, idx, (cudaStream_t)stream));
-    if (idx == 1 || idx == 2) g->head_f = idx;  // a 0-step hit on base/backward slots leaves the head
-  }
-  g->slot[idx].view(out, &g->agg);
-  return STG_OK;
+  return g->get(t, false, PART_ALL, (cudaStream_t)stream, out);
 }
 
 stg_status stg_dtdg_get_backward_snapshot(stg_dtdg* g, int32_t t, stg_stream_t stream, stg_csr_view* out) {
   if (!g || !out) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_get_backward_snapshot: NULL argument");
   if (t < 0 || t >= g->T)
     return fail(STG_ERR_OUT_OF_RANGE, "stg_dtdg_get_backward_snapshot: t=%d outside [0,%d)", t, g->T);
-  int idx = -1;
-  if (g->head_f >= 0 && g->slot[g->head_f].t == t) idx = g->head_f;       // forward head is t itself
-  else if (g->head_b >= 0 && g->slot[g->head_b].t == t) idx = g->head_b;
-  else if (t == 0) idx = 0;
-  else {
-    STG_TRY(g->walk(t, 3, idx, (cudaStream_t)stream));
-    if (idx >= 3) g->head_b = idx;
-  }
-  g->slot[idx].view(out, &g->agg);
-  return STG_OK;
+  return g->get(t, true, PART_ALL, (cudaStream_t)stream, out);
+}
+
+stg_status stg_dtdg_get_snapshot_parts(stg_dtdg* g, int32_t t, int32_t backward, uint32_t parts,
+                                       stg_stream_t stream, stg_csr_view* out) {
+  if (!g || !out) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_get_snapshot_parts: NULL argument");
+  if (t < 0 || t >= g->T) return fail(STG_ERR_OUT_OF_RANGE, "stg_dtdg_get_snapshot_parts: t=%d outside [0,%d)", t, g->T);
+  if (!(parts & (STG_PART_IN | STG_PART_OUT)) || (parts & ~(uint32_t)(STG_PART_IN | STG_PART_OUT | STG_PART_EID)))
+    return fail(STG_ERR_INVALID_ARG, "stg_dtdg_get_snapshot_parts: parts=0x%x", parts);
+  uint32_t p = ((parts & STG_PART_IN) ? PART_IN : 0u) | ((parts & STG_PART_OUT) ? PART_OUT : 0u);
+  if (parts & STG_PART_EID) p = PART_ALL;          // labels tie both directions
+  return g->get(t, backward != 0, p, (cudaStream_t)stream, out);
 }
 
 int64_t stg_dtdg_num_edges(const stg_dtdg* g, int32_t t) {

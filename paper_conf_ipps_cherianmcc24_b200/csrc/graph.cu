@@ -35,7 +35,8 @@ stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_
   STG_TRY(in_ids.alloc(V)); STG_TRY(out_ids.alloc(V));
   STG_TRY(in_sched.alloc(sc)); STG_TRY(out_sched.alloc(sc));
   STG_TRY(norm_src.alloc(V)); STG_TRY(norm_dst.alloc(V));
-  if (sharded) { STG_TRY(gin_deg.alloc(V)); STG_TRY(gout_deg.alloc(V)); }
+  STG_TRY(gin_deg.alloc(V)); STG_TRY(gout_deg.alloc(V));
+  parts = 0;
   return STG_OK;
 }
 
@@ -45,13 +46,20 @@ void Snapshot::view(stg_csr_view* v, AggWs* ws) const {
   v->row_end = re;
   v->timestamp = t;
   v->num_edges = E;
-  // rows below rb are empty, so in_rowptr[rb] = 0: the local row pointer is a suffix
-  v->in_rowptr = in_rowptr.p + rb; v->in_col = in_col.p; v->in_row = in_row.p;
-  v->out_rowptr = out_rowptr.p; v->out_col = out_col.p; v->out_row = out_row.p;
-  v->out_eid = edge_ids ? out_eid.p : nullptr;
-  v->in_deg = in_deg.p; v->out_deg = out_deg.p; v->in_ids = in_ids.p; v->out_ids = out_ids.p;
+  // rows below rb are empty, so in_rowptr[rb] = 0: the local row pointer is a suffix.
+  // Parts this snapshot does not hold are NULL.
+  const bool hi = (parts & PART_IN) != 0, ho = (parts & PART_OUT) != 0;
+  v->in_rowptr = hi ? in_rowptr.p + rb : nullptr; v->in_col = hi ? in_col.p : nullptr;
+  v->in_row = hi ? in_row.p : nullptr;
+  v->out_rowptr = ho ? out_rowptr.p : nullptr; v->out_col = ho ? out_col.p : nullptr;
+  v->out_row = ho ? out_row.p : nullptr;
+  v->out_eid = (edge_ids && (parts & PART_EID)) ? out_eid.p : nullptr;
+  // degrees: whole-graph (always current) unless sharded, where they describe the held edges
+  v->in_deg = sharded ? (hi ? in_deg.p : nullptr) : gin_deg.p;
+  v->out_deg = sharded ? (ho ? out_deg.p : nullptr) : gout_deg.p;
+  v->in_ids = hi ? in_ids.p : nullptr; v->out_ids = ho ? out_ids.p : nullptr;
   v->norm_src = norm_src.p; v->norm_dst = norm_dst.p;
-  v->in_sched = in_sched.p; v->out_sched = out_sched.p;
+  v->in_sched = hi ? in_sched.p : nullptr; v->out_sched = ho ? out_sched.p : nullptr;
   v->workspace = ws;
 }
 
@@ -243,7 +251,7 @@ stg_status sort_unique_keys(uint64_t** keys, uint64_t** alt, int64_t n, int nbit
   return STG_OK;
 }
 
-stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s) {
+stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s, uint32_t parts) {
   const int32_t V = g.V;
   STG_TRY(ws.dkey.alloc(V)); STG_TRY(ws.dkey_alt.alloc(V));
   STG_TRY(ws.dval_alt.alloc(V));
@@ -252,6 +260,7 @@ stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s) {
   const uint32_t mask = (uint32_t)((uint64_t(1) << dbits) - 1);
   const int64_t m = std::min<int64_t>(V, sched_cap(g.cap));
   for (int dir = 0; dir < 2; ++dir) {
+    if (!(parts & (dir == 0 ? PART_IN : PART_OUT))) continue;
     int32_t* deg = dir == 0 ? g.in_deg.p : g.out_deg.p;
     int32_t* ids = dir == 0 ? g.in_ids.p : g.out_ids.p;
     int32_t* sched = dir == 0 ? g.in_sched.p : g.out_sched.p;
@@ -308,13 +317,95 @@ stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& g, Bui
   k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.in_row.p, E, V, g.in_rowptr.p);
   k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.in_rowptr.p, V, g.in_deg.p);
   k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.out_rowptr.p, V, g.out_deg.p);
-  k_norm<<<grid_for(V, 256), 256, 0, s>>>(g.sharded ? g.gin_deg.p : g.in_deg.p,
-                                         g.sharded ? g.gout_deg.p : g.out_deg.p, V, g.dgl_both, g.norm_src.p,
-                                         g.norm_dst.p);
-  count_launch(5);
+  count_launch(4);
+  if (!g.sharded) {                   // whole graph: the whole-graph degrees are the row lengths
+    STG_CUDA(cudaMemcpyAsync(g.gin_deg.p, g.in_deg.p, sizeof(int32_t) * V, cudaMemcpyDeviceToDevice, s));
+    STG_CUDA(cudaMemcpyAsync(g.gout_deg.p, g.out_deg.p, sizeof(int32_t) * V, cudaMemcpyDeviceToDevice, s));
+  }
+  build_norms(g, s);
   STG_TRY(check_launch("build_from_out_keys"));
   STG_TRY(build_ids_and_sched(g, ws, s));
+  g.parts = PART_IN | PART_OUT | (g.edge_ids ? PART_EID : 0u);
   return build_out_eid(g, s);
+}
+
+void build_norms(Snapshot& g, cudaStream_t s) {
+  k_norm<<<grid_for(g.V, 256), 256, 0, s>>>(g.gin_deg.p, g.gout_deg.p, g.V, g.dgl_both, g.norm_src.p, g.norm_dst.p);
+  count_launch();
+}
+
+// ------------------------------------------------------- transpose (Alg. 3)
+__global__ void k_iota(int32_t* __restrict__ a, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    a[i] = (int32_t)i;
+}
+// dst[i] = src[idx[i]]
+__global__ void k_gather_i32(const int32_t* __restrict__ src, const int32_t* __restrict__ idx, int64_t n,
+                             int32_t* __restrict__ dst) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = __ldg(src + __ldg(idx + i));
+}
+// dst[idx[i]] = i
+__global__ void k_scatter_pos(const int32_t* __restrict__ idx, int64_t n, int32_t* __restrict__ dst) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[idx[i]] = (int32_t)i;
+}
+
+// One direction from the other: a stable LSD radix sort of the edge positions
+// by the other endpoint.  The source CSR is sorted by (row, col), so sorting
+// its edges stably by col gives (col, row) order: the transpose in canonical
+// order (reading C3/C7); the sorted positions are the shared edge labels.
+stg_status complete_parts(Snapshot& g, uint32_t want, BuildWs& ws, cudaStream_t s) {
+  const bool need_in = (want & PART_IN) && !(g.parts & PART_IN);
+  const bool need_out = (want & PART_OUT) && !(g.parts & PART_OUT);
+  const bool need_eid = g.edge_ids && (want & PART_EID) && !(g.parts & PART_EID);
+  if (!need_in && !need_out && !need_eid) return STG_OK;
+  if (!(g.parts & (PART_IN | PART_OUT))) return fail(STG_ERR_STATE, "snapshot holds no CSR to transpose");
+  const int64_t E = g.E, En = E > 0 ? E : 1;
+  const int32_t V = g.V;
+  STG_TRY(ws.kalt.alloc(2 * (size_t)En));
+  uint32_t* k1 = reinterpret_cast<uint32_t*>(ws.kalt.p);
+  uint32_t* k2 = k1 + En;
+  int32_t* v1 = reinterpret_cast<int32_t*>(k2 + En);
+  int32_t* v2 = v1 + En;
+  const bool from_in = (g.parts & PART_IN) != 0;   // transpose in -> out (else out -> in)
+  const int32_t* key_src = from_in ? g.in_col.p : g.out_col.p;
+  if (E > 0) {
+    STG_CUDA(cudaMemcpyAsync(k1, key_src, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
+    k_iota<<<grid_for(E, 256), 256, 0, s>>>(v1, E);
+    count_launch();
+    uint32_t* kk = k1; uint32_t* ka = k2; int32_t* vv = v1; int32_t* va = v2;
+    STG_TRY((radix_sort<uint32_t, int32_t>(&kk, &ka, &vv, &va, E, 0, g.nb, ws.radix, s)));
+    k1 = kk; v1 = vv;
+  }
+  if (from_in) {
+    // out_row = sorted src, out_col = in_row[pos], out_eid = pos
+    if (E > 0) {
+      STG_CUDA(cudaMemcpyAsync(g.out_row.p, k1, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
+      k_gather_i32<<<grid_for(E, 256), 256, 0, s>>>(g.in_row.p, v1, E, g.out_col.p);
+      count_launch();
+      if (g.edge_ids) STG_CUDA(cudaMemcpyAsync(g.out_eid.p, v1, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
+    }
+    k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.out_row.p, E, V, g.out_rowptr.p);
+    k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.out_rowptr.p, V, g.out_deg.p);
+    count_launch(2);
+    STG_TRY(build_ids_and_sched(g, ws, s, PART_OUT));
+    g.parts |= PART_OUT | (g.edge_ids ? PART_EID : 0u);
+  } else {
+    // in_row = sorted dst, in_col = out_row[pos]; out_eid[pos] = in position
+    if (E > 0) {
+      STG_CUDA(cudaMemcpyAsync(g.in_row.p, k1, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
+      k_gather_i32<<<grid_for(E, 256), 256, 0, s>>>(g.out_row.p, v1, E, g.in_col.p);
+      count_launch();
+      if (g.edge_ids) { k_scatter_pos<<<grid_for(E, 256), 256, 0, s>>>(v1, E, g.out_eid.p); count_launch(); }
+    }
+    k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.in_row.p, E, V, g.in_rowptr.p);
+    k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.in_rowptr.p, V, g.in_deg.p);
+    count_launch(2);
+    STG_TRY(build_ids_and_sched(g, ws, s, PART_IN));
+    g.parts |= PART_IN | (g.edge_ids ? PART_EID : 0u);
+  }
+  return check_launch("complete_parts");
 }
 
 // -------------------------------------------------------------- delta apply
@@ -465,33 +556,41 @@ static stg_status apply_dir(int32_t V, int nb, const int32_t* orow, const int32_
 }
 
 stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
-                       int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws, cudaStream_t s) {
+                       int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws, cudaStream_t s,
+                       uint32_t parts) {
   const int32_t V = src.V;
-  // labels are carried incrementally when the source snapshot has them
-  const bool carry = dst.edge_ids && src.edge_ids && src.E > 0;
+  const bool do_in = (parts & PART_IN) != 0, do_out = (parts & PART_OUT) != 0;
+  if ((do_in && !(src.parts & PART_IN)) || (do_out && !(src.parts & PART_OUT)))
+    return fail(STG_ERR_STATE, "apply_delta: source snapshot lacks a requested direction");
+  // labels are carried incrementally when both directions and the source labels are there
+  const bool carry = dst.edge_ids && src.edge_ids && (src.parts & PART_EID) && do_in && do_out && src.E > 0;
   int32_t* emap = nullptr;
   if (carry) {
     STG_TRY(ws.emap.alloc((size_t)src.E, s));
     emap = ws.emap.p;
   }
-  STG_TRY(apply_dir(V, src.nb, src.in_row.p, src.in_col.p, src.in_rowptr.p, src.in_deg.p, src.E, dst.in_row.p,
-                    dst.in_col.p, dst.in_rowptr.p, dst.in_deg.p, in_dir, touch_in, ws, s, emap, EidPass{}));
+  if (do_in)
+    STG_TRY(apply_dir(V, src.nb, src.in_row.p, src.in_col.p, src.in_rowptr.p, src.in_deg.p, src.E, dst.in_row.p,
+                      dst.in_col.p, dst.in_rowptr.p, dst.in_deg.p, in_dir, touch_in, ws, s, emap, EidPass{}));
   EidPass ep;
   if (carry) {
     ep.emap_in = emap; ep.eid_old = src.out_eid.p; ep.eid_new = dst.out_eid.p;
     ep.in_rowptr_new = dst.in_rowptr.p; ep.in_col_new = dst.in_col.p;
   }
-  STG_TRY(apply_dir(V, src.nb, src.out_row.p, src.out_col.p, src.out_rowptr.p, src.out_deg.p, src.E,
-                    dst.out_row.p, dst.out_col.p, dst.out_rowptr.p, dst.out_deg.p, out_dir, touch_out, ws, s, nullptr,
-                    ep));
+  if (do_out)
+    STG_TRY(apply_dir(V, src.nb, src.out_row.p, src.out_col.p, src.out_rowptr.p, src.out_deg.p, src.E,
+                      dst.out_row.p, dst.out_col.p, dst.out_rowptr.p, dst.out_deg.p, out_dir, touch_out, ws, s,
+                      nullptr, ep));
   dst.E = E_new;
   dst.t = t_new;
-  k_norm<<<grid_for(V, 256), 256, 0, s>>>(dst.sharded ? dst.gin_deg.p : dst.in_deg.p,
-                                         dst.sharded ? dst.gout_deg.p : dst.out_deg.p, V, dst.dgl_both,
-                                         dst.norm_src.p, dst.norm_dst.p);
-  count_launch();
-  STG_TRY(build_ids_and_sched(dst, ws, s));
-  return carry ? check_launch("apply_delta") : build_out_eid(dst, s);
+  dst.parts = (do_in ? PART_IN : 0u) | (do_out ? PART_OUT : 0u);
+  build_norms(dst, s);
+  STG_TRY(build_ids_and_sched(dst, ws, s, dst.parts));
+  if (dst.edge_ids && do_in && do_out) {
+    if (!carry) STG_TRY(build_out_eid(dst, s));
+    dst.parts |= PART_EID;
+  }
+  return check_launch("apply_delta");
 }
 
 // ------------------------------------------------------------ static graph

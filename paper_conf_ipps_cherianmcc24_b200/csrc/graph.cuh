@@ -46,16 +46,22 @@ struct AggWs {
 // (in-CSR rows outside the block are empty; the out-CSR has all V rows), its
 // in_ids list the local rows first, and the GCN norms come from the degrees
 // of the WHOLE graph (gin_deg / gout_deg), maintained from the global deltas.
+// Parts of a snapshot (a DTDG builds only the direction a pass needs: the
+// forward in-CSR for Get-Graph, the reverse out-CSR for Get-Backward-Graph,
+// the other one by a transpose when asked for, Algorithm 3).
+enum : uint32_t { PART_IN = 1u, PART_OUT = 2u, PART_EID = 4u, PART_ALL = 7u };
+
 struct Snapshot {
   int32_t V = 0, nb = 1;   // nb: bits per id in packed keys
   int32_t t = -1;
   int32_t rb = 0, re = 0;  // local destination rows [rb, re) (whole graph: [0, V))
   int64_t E = 0, cap = 0;  // current (local) edges, edge capacity
   bool edge_ids = false, dgl_both = false, sharded = false;
+  uint32_t parts = 0;      // valid parts (PART_*); degrees and norms are always valid
   DArray<int32_t> in_rowptr, in_col, in_row, in_deg, in_ids;
   DArray<int32_t> out_rowptr, out_col, out_row, out_deg, out_ids, out_eid;
   DArray<int32_t> in_sched, out_sched;  // [sched_size(V, cap)], layout above
-  DArray<int32_t> gin_deg, gout_deg;    // sharded only: whole-graph degrees
+  DArray<int32_t> gin_deg, gout_deg;    // whole-graph degrees (the norms' source; maintained per step)
   DArray<float> norm_src, norm_dst;
 
   stg_status alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_t rb_ = 0, int32_t re_ = -1);
@@ -87,10 +93,16 @@ stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& out, B
 stg_status sort_unique_keys(uint64_t** keys, uint64_t** alt, int64_t n, int nbits, int64_t* d_count,
                             BuildWs& ws, cudaStream_t s);
 
-// Recompute degrees' dependents: node_ids (both directions) and the hub
-// schedules.  Needs deg arrays and rowptrs set.
-stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s);
+// Recompute degrees' dependents: node_ids and the hub schedules of the
+// directions in `parts`.  Needs the deg arrays and rowptrs of those parts.
+stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s, uint32_t parts = PART_IN | PART_OUT);
 stg_status build_out_eid(Snapshot& g, cudaStream_t s);
+// GCN norms from the whole-graph degrees gin_deg / gout_deg (reading C1)
+void build_norms(Snapshot& g, cudaStream_t s);
+// Complete the missing CSR direction(s) of `g` from the one it has by a stable
+// transpose (Algorithm 3, with the canonical order of reading C7),
+// plus node_ids, schedule and (edge_ids) the shared labels.  want: PART_* mask.
+stg_status complete_parts(Snapshot& g, uint32_t want, BuildWs& ws, cudaStream_t s);
 
 // Delta application (DTDG Get-Graph / Get-Backward-Graph step).  For one
 // direction: the sorted packed deltas (row << nb | col) of that direction.
@@ -100,9 +112,12 @@ struct DirDelta {
   const uint64_t* del;
   int64_t ndel;
 };
+// Applies the delta to the directions in `parts` (src must hold them; labels
+// are carried when both directions and src's labels are present).  The caller
+// has already updated dst's whole-graph degrees (gin_deg / gout_deg).
 stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
                        int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws,
-                       cudaStream_t s);
+                       cudaStream_t s, uint32_t parts = PART_ALL);
 
 }  // namespace stg
 

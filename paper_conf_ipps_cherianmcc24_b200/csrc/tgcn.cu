@@ -823,7 +823,7 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
   } else {
     if (t0 < 0 || t0 + S > stg_dtdg_num_timestamps(dtdg))
       return fail(STG_ERR_OUT_OF_RANGE, "stg_tgcn_train_sequence: [%d,%d) outside the DTDG", t0, t0 + S);
-    STG_TRY(stg_dtdg_get_snapshot(dtdg, t0, stream, &view));
+    STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, t0, 0, STG_PART_IN, stream, &view));
   }
   const int32_t V = view.row_end - view.row_begin;  // local rows (all V unless sharded)
   const int32_t Vall = view.num_nodes, H = p->H;
@@ -870,7 +870,7 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     STG_TRY(record(ev_conv[i & 1], as));
     if (dtdg && i + 1 < S) {                                            // prefetch Get-Graph(t+1)
       if (i >= 1) STG_TRY(wait(ss, ev_conv[(i + 1) & 1], as));          // conv(t-1) done with that slot
-      STG_TRY(stg_dtdg_get_snapshot(dtdg, t + 1, ss, &views[(i + 1) & 1]));
+      STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, t + 1, 0, STG_PART_IN, ss, &views[(i + 1) & 1]));
       STG_TRY(record(ev_built[(i + 1) & 1], ss));
     }
     if (dtdg) graph_stack.push_back(t);                                 // graph-stack.push(t)
@@ -887,14 +887,17 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
   float* Gn = G_work + VH;
   STG_CUDA(cudaMemsetAsync(G, 0, sizeof(float) * VH, ms));
   stg_csr_view bviews[2] = {views[0], views[1]};
-  if (dtdg) STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, graph_stack.back(), ms, &bviews[(S - 1) & 1]));  // the head
+  if (dtdg) {      // the forward head; its out-CSR by a transpose (Alg. 3), needed by the reductions only
+    STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, graph_stack.back(), 1, STG_PART_OUT, ss, &bviews[(S - 1) & 1]));
+    STG_TRY(record(ev_built[(S - 1) & 1], ss));
+  }
   for (int32_t i = S - 1; i >= 0; --i) {
     const int b = i & 1;
     if (dtdg) {
       graph_stack.pop_back();                                           // graph-stack.pop()
       if (i > 0) {                                                      // prefetch Get-Backward-Graph(t-1)
         if (i + 1 <= S - 1) STG_TRY(wait(ss, ev_bdone[(i + 1) & 1], as));   // step t+1 done with that slot
-        STG_TRY(stg_dtdg_get_backward_snapshot(dtdg, graph_stack.back(), ss, &bviews[(i - 1) & 1]));
+        STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, graph_stack.back(), 1, STG_PART_OUT, ss, &bviews[(i - 1) & 1]));
         STG_TRY(record(ev_built[(i - 1) & 1], ss));
       }
       if (i < S - 1) STG_TRY(wait(ms, ev_built[i & 1], ss));
@@ -910,6 +913,7 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     STG_TRY(bwd_gru(&v, p, e.C, e.Hp, G, Gn, grads, ws, sb, ms));       // bwdprop: the H chain
     STG_TRY(record(ev_gru[b], ms));
     STG_TRY(wait(as, ev_gru[b], ms));
+    if (dtdg) STG_TRY(wait(as, ev_built[i & 1], ss));                 // the out-CSR of t
     STG_TRY(bwd_grads(&v, p, X[i], e.C, e.Hp, grads, ws, sb, as));      // parameter gradients
     STG_TRY(record(ev_bdone[b], as));
     stack->entries.pop_back();

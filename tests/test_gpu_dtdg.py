@@ -142,3 +142,61 @@ def test_bad_arguments(stg):
     with pytest.raises(stg.StgError):
         stg.stg_dtdg_create(d.V, d.T, d.src0, d.dst0, bad_off, d.add_src, d.add_dst, d.del_off, d.del_src,
                             d.del_dst, 0)
+
+
+def _check_parts(a, ref, parts, tag):
+    """The directions in `parts` bit-exact; degrees (whole graph) and norms always."""
+    V = ref["V"]
+    if parts & 1:
+        for k in ("in_rowptr", "in_col", "in_ids"):
+            assert np.array_equal(a[k].cpu().numpy(), ref[k]), (tag, k)
+        assert np.array_equal(a["in_row"].cpu().numpy(), np.repeat(np.arange(V), np.diff(ref["in_rowptr"]))), tag
+    if parts & 2:
+        for k in ("out_rowptr", "out_col", "out_ids"):
+            assert np.array_equal(a[k].cpu().numpy(), ref[k]), (tag, k)
+    if parts & 4:
+        assert np.array_equal(a["out_eid"].cpu().numpy(), ref["out_eid"]), (tag, "out_eid")
+    for k in ("in_deg", "out_deg"):
+        assert np.array_equal(a[k].cpu().numpy(), ref[k]), (tag, k)
+    for k in ("norm_src", "norm_dst"):
+        np.testing.assert_allclose(a[k].cpu().numpy().astype(np.float64), ref[k], rtol=2.5e-7, atol=0,
+                                   err_msg=str((tag, k)))
+
+
+@pytest.mark.parametrize("loops", [False, True])
+def test_snapshot_parts_and_transpose(stg, dtdg_case, loops):
+    """Direction-only walks (the Algorithm-1 pattern of the TGCN driver: in-CSR forward,
+    out-CSR backward from a transposed head), then full views at random t that force
+    transposes in -> out and out -> in with labels."""
+    name, d, refs = dtdg_case
+    flags = stg.STG_EDGE_IDS | (stg.STG_SELF_LOOPS if loops else 0)
+    g = _create(stg, d, flags)
+    T, S = d.T, 5
+    IN, OUT, EID = stg.STG_PART_IN, stg.STG_PART_OUT, stg.STG_PART_EID
+    for t0 in range(0, T, S):
+        ts = list(range(t0, min(T, t0 + S)))
+        for t in ts:
+            v = stg.stg_dtdg_get_snapshot_parts(g, t, IN)      # other parts may be present (e.g. the base)
+            _check_parts(stg.view_arrays(v), refs[loops][t], IN, (name, "fin", t))
+        for t in reversed(ts):
+            v = stg.stg_dtdg_get_snapshot_parts(g, t, OUT, backward=True)
+            _check_parts(stg.view_arrays(v), refs[loops][t], OUT, (name, "bout", t))
+    rng = np.random.default_rng(3)
+    for _ in range(12):
+        t = int(rng.integers(0, T))
+        bwd = bool(rng.integers(0, 2))
+        parts = [IN, OUT, IN | OUT, IN | OUT | EID][int(rng.integers(0, 4))]
+        v = stg.stg_dtdg_get_snapshot_parts(g, t, parts, backward=bwd)
+        want = parts | ((IN | OUT) if parts & EID else 0)
+        _check_parts(stg.view_arrays(v), refs[loops][t], want, (name, "rand", t, bwd, parts))
+        full = stg.stg_dtdg_get_backward_snapshot(g, t) if bwd else stg.stg_dtdg_get_snapshot(g, t)
+        assert_graph_equal(stg.view_arrays(full), refs[loops][t], tag=(name, "full", t, bwd))
+
+
+def test_snapshot_parts_rejects_bad_mask(stg):
+    d = gen.dtdg(gen.CONFIGS["C5s"])
+    g = _create(stg, d, stg.STG_SELF_LOOPS)
+    for bad in (0, 8, stg.STG_PART_IN | 16):
+        with pytest.raises(stg.StgError) as e:
+            stg.stg_dtdg_get_snapshot_parts(g, 1, bad)
+        assert e.value.status == 1
