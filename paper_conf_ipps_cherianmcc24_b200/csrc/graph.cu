@@ -124,6 +124,44 @@ __global__ void k_deg_keys(const int32_t* __restrict__ deg, int32_t V, uint32_t 
   }
 }
 
+// Two-pass node_ids: the 16-bit key kSat - min(deg, kSat) (65535 for rows outside a
+// sharded block) sorts every vertex by
+// degree desc / id asc except that degrees >= kSat tie; those (at most
+// E / kSat, a short prefix of ids) are re-ranked by k_fix_saturated.
+constexpr int32_t kSat = 65534;
+constexpr int kSatMax = 4096;       // prefix the single-CTA fix handles (E < kSat * kSatMax)
+__global__ void k_deg_keys16(const int32_t* __restrict__ deg, int32_t V, int32_t rb, int32_t re,
+                             uint32_t* __restrict__ keys, int32_t* __restrict__ vals) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+    // rows outside [rb, re) (sharded in-direction) sort after every local row
+    keys[v] = (v >= rb && v < re) ? (uint32_t)(kSat - min(deg[v], kSat)) : 65535u;
+    vals[v] = v;
+  }
+}
+// ids[0, m) hold the saturated vertices (degree >= kSat, ascending id) followed
+// by others; rank the saturated ones by (degree desc, id asc) and rewrite them.
+__global__ void __launch_bounds__(1024) k_fix_saturated(int32_t* __restrict__ ids, const int32_t* __restrict__ deg,
+                                                        int32_t m) {
+  __shared__ int32_t sid[kSatMax], sdeg[kSatMax];
+  __shared__ int32_t nsat;
+  if (threadIdx.x == 0) nsat = 0;
+  __syncthreads();
+  for (int i = threadIdx.x; i < m; i += blockDim.x) {
+    const int32_t v = ids[i], d = deg[v];
+    sid[i] = v;
+    sdeg[i] = d;
+    if (d >= kSat) atomicMax(&nsat, i + 1);
+  }
+  __syncthreads();
+  const int n = nsat;
+  for (int i = threadIdx.x; i < n; i += blockDim.x) {
+    int r = 0;
+    for (int j = 0; j < n; ++j)
+      r += sdeg[j] > sdeg[i] || (sdeg[j] == sdeg[i] && sid[j] < sid[i]);
+    ids[r] = sid[i];
+  }
+}
+
 // sched[0] = number of hub rows (deg > kHubChunk) = length of that prefix of ids.
 __global__ void k_sched_count(const int32_t* __restrict__ ids, const int32_t* __restrict__ deg, int32_t V,
                               int64_t m, int32_t* __restrict__ sched) {
@@ -269,11 +307,23 @@ stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s, uint32_
     const int32_t R = blk ? g.rows() : V;
     uint32_t* k = ws.dkey.p; uint32_t* ka = ws.dkey_alt.p;
     int32_t* vv = ids; int32_t* va = ws.dval_alt.p;
-    k_deg_keys<<<grid_for(V, 256), 256, 0, s>>>(deg, V, mask, blk ? g.rb : 0, blk ? g.re : V, k, vv);
-    count_launch();
-    STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, dbits + (blk ? 1 : 0), ws.radix, s)));
+    const int64_t msat = std::min<int64_t>(V, g.cap / kSat + 1);   // bound on saturated vertices
+    const bool two_pass = dbits > 16 && msat <= kSatMax;
+    if (two_pass) {
+      k_deg_keys16<<<grid_for(V, 256), 256, 0, s>>>(deg, V, blk ? g.rb : 0, blk ? g.re : V, k, vv);
+      count_launch();
+      STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, 16, ws.radix, s)));   // two 8-bit digits
+    } else {
+      k_deg_keys<<<grid_for(V, 256), 256, 0, s>>>(deg, V, mask, blk ? g.rb : 0, blk ? g.re : V, k, vv);
+      count_launch();
+      STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, dbits + (blk ? 1 : 0), ws.radix, s)));
+    }
     if (vv != ids) {
       STG_CUDA(cudaMemcpyAsync(ids, vv, sizeof(int32_t) * V, cudaMemcpyDeviceToDevice, s));
+    }
+    if (two_pass) {
+      k_fix_saturated<<<1, 1024, 0, s>>>(ids, deg, (int32_t)msat);
+      count_launch();
     }
     const int32_t* rowptr = dir == 0 ? g.in_rowptr.p : g.out_rowptr.p;
     const int64_t coff = sched_cptr_off(V, g.cap);
@@ -456,31 +506,55 @@ __device__ __forceinline__ int64_t lb_keys(const uint64_t* a, int64_t lo, int64_
 // the in-direction pass records emap[old position] = new position (-1 if
 // deleted); the out-direction pass sets eid_new[new out position] =
 // emap[eid_old[old out position]] — one lookup per edge instead of a search.
-__global__ void k_merge_old(const int32_t* __restrict__ orow, const int32_t* __restrict__ ocol,
+__global__ void __launch_bounds__(256) k_merge_old(const int32_t* __restrict__ orow, const int32_t* __restrict__ ocol,
                             const int32_t* __restrict__ orowptr, int64_t E_old,
                             const int32_t* __restrict__ nrowptr, const int4* __restrict__ touch,
                             const uint64_t* __restrict__ adds, const uint64_t* __restrict__ dels, int nb,
                             int32_t* __restrict__ nrow, int32_t* __restrict__ ncol, int32_t* __restrict__ emap_out,
                             const int32_t* __restrict__ emap_in, const int32_t* __restrict__ eid_old,
                             int32_t* __restrict__ eid_new) {
-  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < E_old; j += (int64_t)gridDim.x * blockDim.x) {
-    int32_t v = orow[j], c = ocol[j];
-    int4 t = touch[v];
-    int64_t pos = (int64_t)nrowptr[v] + (j - orowptr[v]);
-    if (t.y != t.x || t.w != t.z) {
-      uint64_t key = ((uint64_t)v << nb) | (uint64_t)c;
-      int64_t dl = lb_keys(dels, t.z, t.w, key);
-      if (dl < t.w && dels[dl] == key) {            // deleted
-        if (emap_out) emap_out[j] = -1;
-        continue;
-      }
-      int64_t al = lb_keys(adds, t.x, t.y, key);
-      pos += (al - t.x) - (dl - t.z);
+  // 4 edges per thread per round (coalesced: edge k of the round is k*256 + tid of
+  // the block's 1024-edge tile), with all their row lookups issued before any use
+  constexpr int U = 4;
+  const int64_t tile_stride = (int64_t)gridDim.x * U * blockDim.x;
+  for (int64_t base = (int64_t)blockIdx.x * U * blockDim.x + threadIdx.x; base < E_old; base += tile_stride) {
+    int64_t j[U];
+    int32_t v[U], c[U];
+    bool ok[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      j[k] = base + (int64_t)k * blockDim.x;
+      ok[k] = j[k] < E_old;
+      v[k] = ok[k] ? __ldcs(orow + j[k]) : 0;
+      c[k] = ok[k] ? __ldcs(ocol + j[k]) : 0;
     }
-    nrow[pos] = v;
-    ncol[pos] = c;
-    if (emap_out) emap_out[j] = (int32_t)pos;
-    if (eid_new) eid_new[pos] = emap_in[eid_old[j]];
+    int4 t[U];
+    int32_t orp[U], nrp[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      t[k] = __ldg(touch + v[k]);
+      orp[k] = __ldg(orowptr + v[k]);
+      nrp[k] = __ldg(nrowptr + v[k]);
+    }
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      if (!ok[k]) continue;
+      int64_t pos = (int64_t)nrp[k] + (j[k] - orp[k]);
+      if (t[k].y != t[k].x || t[k].w != t[k].z) {
+        const uint64_t key = ((uint64_t)v[k] << nb) | (uint64_t)c[k];
+        const int64_t dl = lb_keys(dels, t[k].z, t[k].w, key);
+        if (dl < t[k].w && dels[dl] == key) {       // deleted
+          if (emap_out) emap_out[j[k]] = -1;
+          continue;
+        }
+        const int64_t al = lb_keys(adds, t[k].x, t[k].y, key);
+        pos += (al - t[k].x) - (dl - t[k].z);
+      }
+      nrow[pos] = v[k];
+      ncol[pos] = c[k];
+      if (emap_out) emap_out[j[k]] = (int32_t)pos;
+      if (eid_new) eid_new[pos] = emap_in[eid_old[j[k]]];
+    }
   }
 }
 
@@ -541,7 +615,7 @@ static stg_status apply_dir(int32_t V, int nb, const int32_t* orow, const int32_
   if (d.ndel) { k_touch_mark<<<grid_for(d.ndel, 256), 256, 0, s>>>(d.del, d.ndel, nb, 1, touch); count_launch(); }
   STG_TRY(scan(NewDegIn{odeg, touch}, RowptrOut{nrowptr, ndeg}, V, ws.scan, s, nullptr, nrowptr + V));
   if (E_old) {
-    k_merge_old<<<grid_for(E_old, 256), 256, 0, s>>>(orow, ocol, orowptr, E_old, nrowptr, touch, d.add, d.del, nb,
+    k_merge_old<<<grid_for(ceil_div(E_old, 4), 256), 256, 0, s>>>(orow, ocol, orowptr, E_old, nrowptr, touch, d.add, d.del, nb,
                                                     nrow, ncol, emap_out, eid.emap_in, eid.eid_old, eid.eid_new);
     count_launch();
   }

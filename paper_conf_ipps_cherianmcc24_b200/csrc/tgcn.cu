@@ -448,7 +448,7 @@ stg_status set_smem(K fn, size_t smem) {
 
 // Scratch used by the TGCN kernels (grow-only).
 struct TgcnWs {
-  DArray<float> P, dC, dP, part_gru, part_dw, gpart, da, RH, part_tc, dl_tmp;
+  DArray<float> P, dC, dP, part_gru, part_dw, gpart, da, RH, part_tc, dl_tmp, part_dl, dl_tmp2;
   DArray<double> lpart;
 };
 
@@ -560,6 +560,8 @@ static stg_status bwd_alloc(TgcnWs& ws, const stg_csr_view* g, const stg_tgcn_pa
     STG_TRY(ws.RH.alloc(nR * nsets));
     STG_TRY(ws.part_tc.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));
     STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
+    STG_TRY(ws.part_dl.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));   // dL scratch (own stream order)
+    STG_TRY(ws.dl_tmp2.alloc(2 * 128 * 128));
   }
   for (int k = 0; k < 2; ++k) {
     const int kk = k < nsets ? k : 0;
@@ -610,15 +612,21 @@ static stg_status bwd_gru(const stg_csr_view* g, const stg_tgcn_params* p, const
 // The parameter-gradient reductions of one step from buffer set 0 of `bb`:
 // dL, dl, db = Σ_rows [C|H]ᵀda, [RH|1]ᵀda (tensor-core path), dP = diag(n_src)·Aᵀ·dC'
 // over the out-CSR, dW += Xᵀ·dP.
+// dL, dl, db = Σ_rows [C|H]ᵀda, [RH|1]ᵀda (tensor-core path; the SIMT GRU kernel fuses them)
+static stg_status bwd_dl(const stg_csr_view* g, const stg_tgcn_params* p, const float* C, const float* Hp,
+                         stg_tgcn_grads* grads, TgcnWs& ws, const BwdBufs& bb, cudaStream_t s) {
+  const int32_t V = g->row_end - g->row_begin, H = p->H;
+  if (!tc_supported(p->F, H) || V == 0) return STG_OK;
+  ProfScope prof(PH_DL, s);
+  return tc_dl(V, H, C, Hp, bb.RH[0], bb.da[0], ws.part_dl.p, ws.dl_tmp2.p, grads->L, grads->l, grads->b, p->L, s);
+}
+
 static stg_status bwd_grads(const stg_csr_view* g, const stg_tgcn_params* p, const float* X, const float* C,
-                            const float* Hp, stg_tgcn_grads* grads, TgcnWs& ws, const BwdBufs& bb, cudaStream_t s) {
+                            const float* Hp, stg_tgcn_grads* grads, TgcnWs& ws, const BwdBufs& bb, cudaStream_t s,
+                            bool with_dl = true) {
   const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, F = p->F, H = p->H, H3 = 3 * H;
   const bool tc = tc_supported(F, H);
-  if (tc && V > 0) {
-    ProfScope prof(PH_DL, s);
-    STG_TRY(tc_dl(V, H, C, Hp, bb.RH[0], bb.da[0], ws.part_tc.p, ws.dl_tmp.p, grads->L, grads->l, grads->b, p->L,
-                  s));
-  }
+  if (with_dl) STG_TRY(bwd_dl(g, p, C, Hp, grads, ws, bb, s));
   STG_TRY(aggregate_launch(g, 1, H3, bb.dC[0], H3, bb.dP[0], H3, g->norm_src, nullptr, nullptr, s));
   ProfScope prof(PH_DW, s);
   if (tc) return tc_dw(Vall, F, H, X, bb.dP[0], ws.part_tc.p, ws.dl_tmp.p, grads->W, s);
@@ -783,6 +791,16 @@ cudaEvent_t seq_event(int k) {
   cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
   return evs[key] = e;
 }
+// where the dL/dl/db reductions run in the pipelined backward: 0 = with the other
+// reductions on the aux stream (default; measured 129.2 vs 131.6 ms/epoch for 1 =
+// after the GRU backward on the H-chain stream, profiles/r01_sched_sweep.jsonl)
+int dl_on_chain() {
+  static const int v = [] {
+    const char* e = getenv("STG_DL_STREAM");
+    return e ? atoi(e) : 0;
+  }();
+  return v;
+}
 bool pipeline_enabled() {
   static const bool on = [] {
     const char* v = getenv("STG_SEQ_PIPELINE");
@@ -912,9 +930,11 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     sb.dC[0] = bb.dC[b]; sb.dP[0] = bb.dP[b]; sb.da[0] = bb.da[b]; sb.RH[0] = bb.RH[b];
     STG_TRY(bwd_gru(&v, p, e.C, e.Hp, G, Gn, grads, ws, sb, ms));       // bwdprop: the H chain
     STG_TRY(record(ev_gru[b], ms));
+    const bool dl_chain = pipe && dl_on_chain();
+    if (dl_chain) STG_TRY(bwd_dl(&v, p, e.C, e.Hp, grads, ws, sb, ms));   // dL after the GRU, off the A stream
     STG_TRY(wait(as, ev_gru[b], ms));
     if (dtdg) STG_TRY(wait(as, ev_built[i & 1], ss));                 // the out-CSR of t
-    STG_TRY(bwd_grads(&v, p, X[i], e.C, e.Hp, grads, ws, sb, as));      // parameter gradients
+    STG_TRY(bwd_grads(&v, p, X[i], e.C, e.Hp, grads, ws, sb, as, !dl_chain));   // parameter gradients
     STG_TRY(record(ev_bdone[b], as));
     stack->entries.pop_back();
     stack->top -= e.bytes;

@@ -1,5 +1,5 @@
 #!/bin/bash
-# Epoch time of the C5 bench under scheduling knobs (pipelined sequence driver, atb2 ring budget).
+# Epoch time of the C5 bench under scheduling knobs (pipelined sequence driver).
 set -u
 run() {  # name, env...
   local name=$1; shift
@@ -12,8 +12,7 @@ print(json.dumps({"name": n, "ms_per_step": round(d["ms_per_step"], 2), "Gedges_
                   "phases": {k: round(v, 1) for k, v in d["phases_ms_per_step"].items()}}))
 PY
 }
-run serial STG_SEQ_PIPELINE=0
-run pipe STG_SEQ_PIPELINE=1
-run pipe_atb150 STG_SEQ_PIPELINE=1 STG_ATB_SMEM_KB=150
-run pipe_atb110 STG_SEQ_PIPELINE=1 STG_ATB_SMEM_KB=110
-run serial_atb150 STG_SEQ_PIPELINE=0 STG_ATB_SMEM_KB=150
+for cfg in "$@"; do
+  name=${cfg%%:*}; envs=${cfg#*:}
+  run "$name" $envs
+done
