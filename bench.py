@@ -44,6 +44,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="sharded", choices=["sharded", "replicas"],
                     help="N>1: row-block shards of one graph (SURVEY §8(e)) or independent replicas")
+    ap.add_argument("--graphs", type=int, default=-1,
+                    help="replay each epoch as one CUDA graph (1/0; default: on for static-temporal configs, "
+                         "whose tiny per-timestamp work is launch-bound, off for DTDGs)")
     ap.add_argument("--shard-sim", default=None, metavar="K/N",
                     help="(testing on one GPU) run rank K's row block of an N-way sharding, no process group")
     return ap.parse_args()
@@ -133,29 +136,68 @@ def oracle_timestep(cfg, d, t: int, S_prev):
     return 2 * g["E"], dt, S
 
 
+def oracle_timestep_static(cfg, g, t: int, reps: int = 1):
+    """The fp64 oracle on `reps` timesteps of a static-temporal config (the graph is
+    built once, outside the timing): TGCN forward, MSE head, TGCN backward."""
+    import gen
+    import oracle
+    X = gen.features(cfg, t % 2)
+    Y = gen.labels(cfg, t)
+    p = gen.tgcn_params(cfg.F, cfg.H, cfg.seed)
+    Hp = np.zeros((cfg.V, cfg.H))
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        f = oracle.tgcn_fwd(g, p, X, Hp)
+        grads = oracle.zero_grads(cfg.F, cfg.H)
+        _, dH = oracle.mse_head(f["Hn"], Y, p["w_o"], p["b_o"], grads)
+        oracle.tgcn_bwd(g, p, X, Hp, f, dH, grads)
+    return 2 * g["E"] * reps, time.perf_counter() - t0
+
+
+def static_reps(cfg) -> int:
+    """Timesteps per oracle sample: about 20 M edge-visits of work (seconds of CPU)."""
+    return max(1, int(2e7 // max(1, 2 * cfg.E)))
+
+
 def run_reference(args):
     import gen
     import oracle
     cfg = gen.CONFIGS[args.config]
-    d = gen.dtdg(cfg)
     oracle.build()
-    S = next(oracle.snapshot_sets_fold(d, self_loops=True))
     edges, secs = 0, 0.0
-    t = 1
-    for i in range(args.warmup + args.steps):
-        e, dt, S = oracle_timestep(cfg, d, t, S)
-        if i >= args.warmup:
-            edges += e
-            secs += dt
-        t = t + 1 if t + 1 < d.T else 1
-        if t == 1:
-            S = next(oracle.snapshot_sets_fold(d, self_loops=True))
-    value = edges / secs
-    sample = "per step: one C5 timestep (fold S_{t-1}->S_t, CSR pair, TGCN fwd + MSE head + bwd) in the fp64 oracle"
+    if cfg.kind == "static":
+        s_, d_ = gen.static_edges(cfg)
+        g = oracle.static_graph(cfg.V, s_, d_, self_loops=True)
+        reps = static_reps(cfg)
+        for i in range(args.warmup + args.steps):
+            e, dt = oracle_timestep_static(cfg, g, i, reps)
+            if i >= args.warmup:
+                edges += e
+                secs += dt
+        value = edges / secs
+        sample = ("per step: %d %s timesteps (TGCN fwd + MSE head + bwd on the static CSR) in the fp64 oracle"
+                  % (reps, cfg.name))
+        T = cfg.T
+    else:
+        d = gen.dtdg(cfg)
+        S = next(oracle.snapshot_sets_fold(d, self_loops=True))
+        t = 1
+        for i in range(args.warmup + args.steps):
+            e, dt, S = oracle_timestep(cfg, d, t, S)
+            if i >= args.warmup:
+                edges += e
+                secs += dt
+            t = t + 1 if t + 1 < d.T else 1
+            if t == 1:
+                S = next(oracle.snapshot_sets_fold(d, self_loops=True))
+        value = edges / secs
+        sample = ("per step: one %s timestep (fold S_{t-1}->S_t, CSR pair, TGCN fwd + MSE head + bwd) in the fp64 "
+                  "oracle" % cfg.name)
+        T = d.T
     out = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-           "config": {"workload": cfg.desc, "config": cfg.name, "V": cfg.V, "F": cfg.F, "H": cfg.H, "T": d.T,
+           "config": {"workload": cfg.desc, "config": cfg.name, "V": cfg.V, "F": cfg.F, "H": cfg.H, "T": T,
                       "sample": sample},
            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -188,9 +230,16 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
     cfg = gen.CONFIGS[args.config]
-    assert cfg.kind == "dtdg"
-    d = gen.dtdg(cfg)
-    V, F, H, T = cfg.V, cfg.F, cfg.H, d.T
+    static = cfg.kind == "static"
+    if static:
+        s_e, d_e = gen.static_edges(cfg)
+        d = None
+        T = cfg.T
+    else:
+        d = gen.dtdg(cfg)
+        s_e, d_e = d.src0, d.dst0
+        T = d.T
+    V, F, H = cfg.V, cfg.F, cfg.H
     S = args.seq
     seqs = [(t0, min(S, T - t0)) for t0 in range(0, T, S)]
     # N > 1, sharded (default): destination row blocks with ~E/N in-edges of S_0 each
@@ -200,12 +249,17 @@ def main():
     lo, hi = 0, V
     if sharded:
         from paper_conf_ipps_cherianmcc24_b200 import parallel
-        bounds = parallel.base_row_blocks(V, d.src0, d.dst0, world, self_loops=True)
+        bounds = parallel.base_row_blocks(V, s_e, d_e, world, self_loops=True)
         lo, hi = bounds[rank], bounds[rank + 1]
     R = hi - lo
-    g = stg.stg_dtdg_create(V, T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src, d.del_dst,
-                            stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS, dist=(rank, world, lo, hi) if sharded else None)
-    E_t = [g.num_edges(t) for t in range(T)]
+    dist_arg = (rank, world, lo, hi) if sharded else None
+    if static:
+        g = stg.stg_static_graph_create(V, s_e, d_e, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS, dist=dist_arg)
+        E_t = [g.view().num_edges] * T
+    else:
+        g = stg.stg_dtdg_create(V, T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                                d.del_dst, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS, dist=dist_arg)
+        E_t = [g.num_edges(t) for t in range(T)]
     edges_per_step = 2 * sum(E_t)            # this rank's edges (whole graph unless sharded)
     edges_all = edges_per_step
     if pg:
@@ -260,6 +314,20 @@ def main():
     for _ in range(args.warmup):
         epoch(Xdev, Ydev)
     torch.cuda.synchronize()
+    # CUDA graph of one whole epoch (static graphs: no host-side snapshot state), replayed
+    use_graphs = (args.graphs == 1) or (args.graphs < 0 and static and not pg)
+    cg = None
+    run_epoch = lambda: epoch(Xdev, Ydev)
+    launches_per_epoch = None
+    if use_graphs:
+        cg = torch.cuda.CUDAGraph()
+        l0 = stg.kernel_launch_count()
+        with torch.cuda.graph(cg, capture_error_mode="relaxed"):
+            epoch(Xdev, Ydev)
+        launches_per_epoch = stg.kernel_launch_count() - l0
+        cg.replay()
+        torch.cuda.synchronize()
+        run_epoch = cg.replay
 
     # ---------------- timed region (device-resident inputs)
     clocks = ClockSampler(local)
@@ -274,11 +342,13 @@ def main():
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
     for _ in range(args.steps):
-        epoch(Xdev, Ydev)
+        run_epoch()
     ev1.record(stream)
     torch.cuda.synchronize()
     ms = ev0.elapsed_time(ev1)
     launches = stg.kernel_launch_count() - launches0
+    if cg is not None:
+        launches = launches_per_epoch * args.steps       # graph replays launch the captured kernels
     clk = clocks.stop()
     if pg:
         t = torch.tensor([ms], device=dev)
@@ -394,21 +464,30 @@ def main():
     if rank == 0 and world == 1 and not sim and not args.no_cpu_baseline:
         import oracle
         oracle.build()
-        S0 = next(oracle.snapshot_sets_fold(d, self_loops=True))
-        e_c, dt_c, _ = oracle_timestep(cfg, d, 1, S0)
+        if static:
+            reps = static_reps(cfg)
+            e_c, dt_c = oracle_timestep_static(cfg, oracle.static_graph(V, s_e, d_e, self_loops=True), 1, reps)
+            smp = "%d %s timesteps: TGCN fwd + MSE head + bwd on the static CSR" % (reps, cfg.name)
+        else:
+            S0 = next(oracle.snapshot_sets_fold(d, self_loops=True))
+            e_c, dt_c, _ = oracle_timestep(cfg, d, 1, S0)
+            smp = "one %s timestep (t=1): fold S_0->S_1, CSR pair, TGCN fwd + MSE head + bwd" % cfg.name
         cpu = {"value": e_c / dt_c, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": "one C5 timestep (t=1): fold S_0->S_1, CSR pair, TGCN fwd + MSE head + bwd, fp64, "
-                         "single thread; %.1f s" % dt_c}
+               "sample": smp + ", fp64, single thread; %.1f s" % dt_c}
 
     if rank == 0 or sim:
         out = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1 if sim else world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": cfg.desc + " (BASELINE.json configs[4])", "config": cfg.name, "V": V,
+            "config": {"workload": cfg.desc + " (BASELINE.json configs[%d])" % ["C1", "C2", "C3", "C4", "C5"].index(
+                           cfg.name) if cfg.name in ("C1", "C2", "C3", "C4", "C5") else cfg.desc, "config": cfg.name,
+                       "V": V,
                        "E_mean": int(E_mean), "T": T, "F": F, "H": H, "seq_len": S, "sequences": len(seqs),
                        "step": "one Algorithm-1 training epoch over all T timestamps",
-                       "l2": "inputs larger than L2 (X_t 256 MB, graph ~0.3 GB, state 8 GB)",
+                       "l2": ("inputs larger than L2 (X_t 256 MB, graph ~0.3 GB, state 8 GB)" if cfg.name == "C5"
+                              else "working set fits in L2 (not flushed between epochs)"),
+                       "cuda_graph": cg is not None,
                        "parallelism": ("row-block shards x%d (resident X_t, NCCL gradient all-reduce per "
                                        "sequence)" % world) if sharded else ("replicas" if world > 1 else "single"),
                        "E_local_mean_rank0": int(E_mean)},

@@ -68,6 +68,27 @@ __device__ __forceinline__ void fma_v(float4& a, float s, const float4& b) {
 }
 __device__ __forceinline__ void fma_v(float& a, float s, const float& b) { a = fmaf(s, b, a); }
 __device__ __forceinline__ void add_v(float4& a, const float4& b) { a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w; }
+// Packed fp32x2 adds / fmas (FADD2 / FFMA2, sm_100): two IEEE round-to-nearest
+// operations per instruction, bit-identical to the scalar ones.
+__device__ __forceinline__ void add2_v(float4& a, const float4& b) {
+  unsigned long long a0, a1;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(a0) : "l"(*reinterpret_cast<const unsigned long long*>(&a.x)),
+      "l"(*reinterpret_cast<const unsigned long long*>(&b.x)));
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(a1) : "l"(*reinterpret_cast<const unsigned long long*>(&a.z)),
+      "l"(*reinterpret_cast<const unsigned long long*>(&b.z)));
+  *reinterpret_cast<unsigned long long*>(&a.x) = a0;
+  *reinterpret_cast<unsigned long long*>(&a.z) = a1;
+}
+__device__ __forceinline__ void fma2_v(float4& a, float s, const float4& b) {
+  const float2 ss = make_float2(s, s);
+  unsigned long long a0, a1;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(a0) : "l"(*reinterpret_cast<const unsigned long long*>(&ss)),
+      "l"(*reinterpret_cast<const unsigned long long*>(&b.x)), "l"(*reinterpret_cast<const unsigned long long*>(&a.x)));
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(a1) : "l"(*reinterpret_cast<const unsigned long long*>(&ss)),
+      "l"(*reinterpret_cast<const unsigned long long*>(&b.z)), "l"(*reinterpret_cast<const unsigned long long*>(&a.z)));
+  *reinterpret_cast<unsigned long long*>(&a.x) = a0;
+  *reinterpret_cast<unsigned long long*>(&a.z) = a1;
+}
 __device__ __forceinline__ void add_v(float& a, const float& b) { a += b; }
 __device__ __forceinline__ float4 scale_bias(float s, const float4& a, const float* bias, int c0) {
   float4 r;
@@ -249,6 +270,8 @@ struct Agg2Args {
   float* partials;
   int32_t* counters;
   int32_t upad;     // a valid column id for the padding gathers past the stream end
+  int32_t hgrp;     // edge stream: hub-chunk items per work group (<= 32)
+  int32_t lgrp;     // edge stream: light-row items per work group (<= 32)
 };
 
 // Strategy 1: software-pipelined degree-ordered items.  A warp serves 32/G
@@ -405,6 +428,7 @@ __global__ void __launch_bounds__(kAggThreads, 4) k_agg_items(const Agg2Args a) 
 // (deterministic: the tree shape depends only on the chunk count), written as
 // y[v] = s_v·Σ + bias.  Rows with more than 64 blocks run in rounds of 64.
 constexpr int kHubBlk = 16, kHubRound = 64;
+constexpr int kHubGroup = 8;     // hub-chunk items per edge-stream work group (at most)
 __global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_t* __restrict__ ids) {
   __shared__ float4 blk[kHubRound][32];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -482,17 +506,25 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t total = a.sched[3];
   const int4* items = reinterpret_cast<const int4*>(a.sched + kSchedHdr);
-  const uint32_t ngroups = (uint32_t)((total + 31) / 32);
+  // Work groups: hub chunks (<= 64 edges each) a.hgrp per group, light rows
+  // a.lgrp per group (host-chosen so that small graphs still spread over many
+  // warps), so no warp walks a long single group while others idle.
+  const int64_t n_chunks = a.sched[1];
+  const int64_t hg = a.hgrp, lg = a.lgrp;
+  const int64_t nhg = (n_chunks + hg - 1) / hg;
+  const uint32_t ngroups = (uint32_t)(nhg + (total - n_chunks + lg - 1) / lg);
+  auto gbase = [&](int64_t g) { return g < nhg ? g * hg : n_chunks + (g - nhg) * lg; };
+  auto gend = [&](int64_t g) { return g < nhg ? min((g + 1) * hg, n_chunks) : min(gbase(g) + lg, total); };
   const int nv = a.W >> 2;
   const bool lane_on = lane < nv;
   const float4* xl = reinterpret_cast<const float4*>(a.x) + (lane_on ? lane : nv - 1);
   const uint32_t ld4 = (uint32_t)(a.ldx >> 2);
   int32_t* ex = s_excl[w];
   auto fetch = [&](uint32_t g, int buf) {         // cp.async the 32 descriptors of group g
-    const int64_t it = (int64_t)g * 32 + lane;
+    const int64_t it = gbase(g) + lane;
     const uint32_t dst = (uint32_t)__cvta_generic_to_shared(&s_items[w][buf][lane]);
     const int4* src = items + (it < total ? it : 0);
-    const int bytes = (g < ngroups && it < total) ? 16 : 0;
+    const int bytes = (g < ngroups && it < gend(g)) ? 16 : 0;
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst), "l"(src), "r"(bytes) : "memory");
     asm volatile("cp.async.commit_group;\n" ::: "memory");
   };
@@ -510,7 +542,8 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
     __syncwarp();
     int4 m = s_items[w][buf][lane];
     buf ^= 1;
-    if ((int64_t)g_cur * 32 + lane >= total) m = make_int4(0, 0, 0, -2);
+    const int64_t ib = gbase(g_cur);
+    if (ib + lane >= gend(g_cur)) m = make_int4(0, 0, 0, -2);
     const int32_t nl = m.w > -2 ? m.z : 0;
     int32_t incl = nl;
 #pragma unroll
@@ -547,7 +580,7 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
         if (hub < 0)
           __stcs(reinterpret_cast<float4*>(a.y + (int64_t)s_v[w][c] * a.ldy) + lane, scale_bias(sv, sum, a.bias, 4 * lane));
         else
-          reinterpret_cast<float4*>(a.partials + ((int64_t)g_cur * 32 + c) * a.W)[lane] = sum;
+          reinterpret_cast<float4*>(a.partials + (ib + c) * a.W)[lane] = sum;
       }
     };
     int32_t u0, k0;
@@ -573,17 +606,26 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
           const uint32_t u = (uint32_t)__shfl_sync(FULL, uc, (j0 + d) & 31);
           v[d] = __ldg(xl + (size_t)u * ld4);
         }
+        const uint32_t mseg = (bm >> (j0 & 31)) & (D >= 32 ? 0xffffffffu : ((1u << D) - 1u));
+        if (mseg == 0) {                                // warp-uniform: no item starts in this group
+#pragma unroll
+          for (int d = 0; d < D; ++d) {
+            if (SCOL) fma2_v(acc, __shfl_sync(FULL, sc, (j0 + d) & 31), v[d]);
+            else add2_v(acc, v[d]);
+          }
+          continue;
+        }
 #pragma unroll
         for (int d = 0; d < D; ++d) {
           const float sj = SCOL ? __shfl_sync(FULL, sc, (j0 + d) & 31) : 1.0f;
-          if ((bm >> ((j0 + d) & 31)) & 1u) {
+          if ((mseg >> d) & 1u) {
             if (cur >= 0) flush(cur, acc);
             cur = __shfl_sync(FULL, kc, (j0 + d) & 31);
-            if (SCOL) { acc = make_float4(0.f, 0.f, 0.f, 0.f); fma_v(acc, sj, v[d]); }
+            if (SCOL) { acc = make_float4(0.f, 0.f, 0.f, 0.f); fma2_v(acc, sj, v[d]); }
             else acc = v[d];
           } else {
-            if (SCOL) fma_v(acc, sj, v[d]);
-            else add_v(acc, v[d]);
+            if (SCOL) fma2_v(acc, sj, v[d]);
+            else add2_v(acc, v[d]);
           }
         }
       }
@@ -771,7 +813,15 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     STG_TRY(ws->queue.alloc(nsplit, s));
     STG_CUDA(cudaMemsetAsync(ws->queue.p, 0, sizeof(uint32_t) * nsplit, s));
     const StreamFn fn = pick_stream(g_tune.d, g_tune.minb, scol != nullptr);
-    const int64_t blocks = std::min<int64_t>(occupancy_grid((const void*)fn), ceil_div(items_bound, 32 * 8) + 1);
+    // group sizes: ~max(256, E / (8 warps x #SM)) edges per group (all 32-item light
+    // groups at C5 scale; small graphs get small groups, hence many warps)
+    const int64_t target = std::max<int64_t>(256, gv->num_edges / (8 * (int64_t)num_sms()));
+    const int64_t avg = std::max<int64_t>(1, gv->num_edges / std::max<int32_t>(1, R));
+    int hgrp = kHubGroup, lgrp = 32;
+    while (hgrp > 2 && (int64_t)hgrp * kHubChunk > target) hgrp >>= 1;
+    while (lgrp > 4 && (int64_t)lgrp * avg > 2 * target) lgrp >>= 1;
+    const int64_t ngroups = ceil_div(chunks_bound, hgrp) + ceil_div(R, lgrp) + 1;   // bound on work groups
+    const int64_t blocks = std::min<int64_t>(occupancy_grid((const void*)fn), ceil_div(ngroups, 8) + 1);
     const int32_t* hids = backward ? gv->out_ids : gv->in_ids;
     for (int k = 0; k < nsplit; ++k) {
       const int32_t c0 = k * wsplit, wl = std::min(wsplit, W - c0);
@@ -781,6 +831,7 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
       b.W = wl; b.x = in + c0; b.ldx = ldin; b.y = out + c0; b.ldy = ldout;
       b.bias = bias ? bias + c0 : nullptr;
       b.upad = (backward && a.ids) ? (int32_t)rb : 0;   // row 0 of a shifted input is not a valid row
+      b.hgrp = hgrp; b.lgrp = lgrp;
       fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(b, ws->queue.p + k);
       k_agg_hubs<<<(unsigned)(4 * num_sms()), 256, 0, s>>>(b, hids);
       count_launch(2);
