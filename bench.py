@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--graphs", type=int, default=-1,
                     help="replay each epoch as one CUDA graph (1/0; default: on for static-temporal configs, "
                          "whose tiny per-timestamp work is launch-bound, off for DTDGs)")
+    ap.add_argument("--schedule", default="auto", choices=["auto", "batched", "per-step"],
+                    help="static graphs: sequence-batched (NEXT-1, default) or per-timestamp Algorithm-1 driver")
     ap.add_argument("--shard-sim", default=None, metavar="K/N",
                     help="(testing on one GPU) run rank K's row block of an N-way sharding, no process group")
     return ap.parse_args()
@@ -252,6 +254,7 @@ def main():
         bounds = parallel.base_row_blocks(V, s_e, d_e, world, self_loops=True)
         lo, hi = bounds[rank], bounds[rank + 1]
     R = hi - lo
+    batched = static and not sharded and (args.schedule in ("auto", "batched"))
     dist_arg = (rank, world, lo, hi) if sharded else None
     if static:
         g = stg.stg_static_graph_create(V, s_e, d_e, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS, dist=dist_arg)
@@ -303,9 +306,14 @@ def main():
         Hprev = H0
         for k, (t0, n) in enumerate(seqs):
             Hs = Hbuf[k % 2]
-            stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], [Xsrc(t) for t in range(t0, t0 + n)],
-                                        [Ysrc(t) for t in range(t0, t0 + n)], Hprev, Hs, Gw, grads, dw_o, db_o,
-                                        loss, stack)
+            if batched:
+                stg.stg_tgcn_train_sequence_batched(g, n, p, p["w_o"], p["b_o"], [Xsrc(t) for t in range(t0, t0 + n)],
+                                                    [Ysrc(t) for t in range(t0, t0 + n)], Hprev, Hs, grads, dw_o,
+                                                    db_o, loss, stack)
+            else:
+                stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], [Xsrc(t) for t in range(t0, t0 + n)],
+                                            [Ysrc(t) for t in range(t0, t0 + n)], Hprev, Hs, Gw, grads, dw_o, db_o,
+                                            loss, stack)
             sgd()
             Hprev = Hs[n - 1]
 
@@ -426,8 +434,12 @@ def main():
                 if k + 1 < len(seqs):
                     nxt = issue(k + 1) if True else None
                 Hs = Hbuf[k % 2]
-                stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], stage[k % 2][:n], ystage[k % 2][:n],
-                                            Hprev, Hs, Gw, grads, dw_o, db_o, loss, stack)
+                if batched:
+                    stg.stg_tgcn_train_sequence_batched(g, n, p, p["w_o"], p["b_o"], stage[k % 2][:n],
+                                                        ystage[k % 2][:n], Hprev, Hs, grads, dw_o, db_o, loss, stack)
+                else:
+                    stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], stage[k % 2][:n], ystage[k % 2][:n],
+                                                Hprev, Hs, Gw, grads, dw_o, db_o, loss, stack)
                 sgd()
                 ev = torch.cuda.Event()
                 ev.record(stream)
@@ -488,6 +500,7 @@ def main():
                        "l2": ("inputs larger than L2 (X_t 256 MB, graph ~0.3 GB, state 8 GB)" if cfg.name == "C5"
                               else "working set fits in L2 (not flushed between epochs)"),
                        "cuda_graph": cg is not None,
+                       "schedule": "sequence-batched (NEXT-1)" if batched else "per-timestamp Algorithm 1",
                        "parallelism": ("row-block shards x%d (resident X_t, NCCL gradient all-reduce per "
                                        "sequence)" % world) if sharded else ("replicas" if world > 1 else "single"),
                        "E_local_mean_rank0": int(E_mean)},

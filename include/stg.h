@@ -288,6 +288,23 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
                                    float* db_o, float* loss_accum, stg_state_stack* stack,
                                    stg_stream_t stream);
 
+/* Sequence-batched Algorithm 1 for a STATIC graph: the
+ * same forward, loss and gradients as stg_tgcn_train_sequence over t = 0..S-1
+ * (P:L120-171), scheduled per sequence.  Because C_t = Â(X_t W) + b does not
+ * depend on H (reading C13/C14), X_t W and the aggregation run once for all S
+ * timestamps (one SpMM of width S·3H over [V][S][3H] rows), the GRU recurrence
+ * and the MSE head run for all t inside one persistent row-tile kernel per
+ * direction, and dL/dl/db, dP = Âᵀ dC', dW reduce over all V·S (vertex, t)
+ * rows at once.  Requirements: unsharded graph, tensor-core shapes (H 16|32,
+ * F % 4 == 0, F <= 64), 1 <= S <= 64.  Arguments as stg_tgcn_train_sequence
+ * (X/Y (host)[S] device pointers, H0 [V,H], H_seq [S][V,H] receives H_t,
+ * gradients and loss accumulated); the stack only provides scratch. */
+stg_status stg_tgcn_train_sequence_batched(const stg_graph* graph, int32_t S, const stg_tgcn_params* p,
+                                           const float* w_o, const float* b_o, const float* const* X,
+                                           const float* const* Y, const float* H0, float* H_seq,
+                                           stg_tgcn_grads* grads, float* dw_o, float* db_o,
+                                           float* loss_accum, stg_state_stack* stack, stg_stream_t stream);
+
 /* ---- multi-GPU helpers ----
  * nnz-balanced destination row blocks: bounds (host)[world+1] with bounds[0]=0,
  * bounds[world]=V, block k ≈ E/world in-edges.  in_rowptr is a DEVICE [V+1]

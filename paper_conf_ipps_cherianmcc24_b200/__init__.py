@@ -104,6 +104,9 @@ _decl("stg_sgd_update", [_P, _P, _i64, _f32, _P])
 _decl("stg_tgcn_train_sequence", [_P, _P, _i32, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P,
                                   ctypes.POINTER(_P), ctypes.POINTER(_P), _P, _P, _P,
                                   ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P, _P])
+_decl("stg_tgcn_train_sequence_batched", [_P, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P, ctypes.POINTER(_P),
+                                          ctypes.POINTER(_P), _P, _P, ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P,
+                                          _P])
 _decl("stg_partition_rows", [_i32, _P, _i32, ctypes.POINTER(_i32), _P])
 _decl("stg_profile_enable", [_i32])
 _decl("stg_debug_tc_gemm", [_i32, _i32, _i32, _i32, _i32, _P, _P, _P, _P])
@@ -120,6 +123,7 @@ ABI_SYMBOLS = [
     "stg_gcn_aggregate_fwd", "stg_gcn_aggregate_bwd", "stg_gcn_aggregate_ex",
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
     "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_mse_head_ex", "stg_sgd_update", "stg_tgcn_train_sequence",
+    "stg_tgcn_train_sequence_batched",
     "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
 ]
@@ -416,6 +420,18 @@ def stg_mse_head(Hn, y, w_o, b_o, loss_accum=None, dH=None, accumulate=False, dw
 
 def stg_sgd_update(p: torch.Tensor, g: torch.Tensor, lr: float, stream=None):
     _check(_lib.stg_sgd_update(_ptr(p), _ptr(g), p.numel(), float(lr), _stream(stream)))
+
+
+def stg_tgcn_train_sequence_batched(graph, S: int, params: dict, w_o, b_o, Xs, Ys, H0, H_seq, grads: dict, dw_o,
+                                    db_o, loss_accum, stack: StateStack, stream=None):
+    """Sequence-batched Algorithm 1 over a static graph (NEXT-1): same maths, per-sequence kernels."""
+    P = make_params(params)
+    G = make_grads(grads)
+    xp = (_P * S)(*[x.data_ptr() for x in Xs])
+    yp = (_P * S)(*[y.data_ptr() for y in Ys])
+    _check(_lib.stg_tgcn_train_sequence_batched(graph.handle, S, ctypes.byref(P), _ptr(w_o), _ptr(b_o), xp, yp,
+                                                _ptr(H0), _ptr(H_seq), ctypes.byref(G), _ptr(dw_o), _ptr(db_o),
+                                                _ptr(loss_accum), stack.handle, _stream(stream)))
 
 
 def stg_tgcn_train_sequence(source, t0: int, S: int, params: dict, w_o, b_o, Xs, Ys, H0, H_seq, G_work,

@@ -272,6 +272,10 @@ struct Agg2Args {
   int32_t upad;     // a valid column id for the padding gathers past the stream end
   int32_t hgrp;     // edge stream: hub-chunk items per work group (<= 32)
   int32_t lgrp;     // edge stream: light-row items per work group (<= 32)
+  // column chunks run side by side (blockIdx.y = chunk): chunk k covers columns
+  // [k·wsplit, min((k+1)·wsplit, wtotal)) and its hub partials start at k·pstride
+  int32_t wsplit, wtotal;
+  int64_t pstride;
 };
 
 // Strategy 1: software-pipelined degree-ordered items.  A warp serves 32/G
@@ -435,7 +439,12 @@ __global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_
   const int32_t n_hub = a.sched[0];
   const int32_t* cptr = a.sched + a.sched[2];
   const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
-  const int nv = a.W >> 2;
+  const int c0y = blockIdx.y * a.wsplit;                       // this launch's column chunk
+  const int Wl = min(a.wsplit, a.wtotal - c0y);
+  float* const ybase = a.y + c0y;
+  const float* const bbase = a.bias ? a.bias + c0y : nullptr;
+  const float* const pbase = a.partials + (int64_t)blockIdx.y * a.pstride;
+  const int nv = Wl >> 2;
   const int c = lane < nv ? lane : nv - 1;
   // big hubs (more than one block of chunks) lead the schedule: n_big = first h
   // with cptr[h+1] - cptr[h] <= kHubBlk (chunk counts are non-increasing)
@@ -457,7 +466,7 @@ __global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_
         float4 p[kHubBlk];
 #pragma unroll
         for (int i = 0; i < kHubBlk; ++i)
-          p[i] = q0 + i < q1 ? __ldcg(reinterpret_cast<const float4*>(a.partials + (int64_t)(q0 + i) * a.W) + c) : z4;
+          p[i] = q0 + i < q1 ? __ldcg(reinterpret_cast<const float4*>(pbase + (int64_t)(q0 + i) * Wl) + c) : z4;
         float4 sb = p[0];
 #pragma unroll
         for (int i = 1; i < kHubBlk; ++i) add_v(sb, p[i]);
@@ -476,7 +485,7 @@ __global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_
     }
     if (warp == 0 && lane < nv) {
       const float sv = a.srow ? a.srow[v] : 1.0f;
-      __stcs(reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy) + lane, scale_bias(sv, tot, a.bias, 4 * lane));
+      __stcs(reinterpret_cast<float4*>(ybase + (int64_t)v * a.ldy) + lane, scale_bias(sv, tot, bbase, 4 * lane));
     }
   }
   // (2) hubs of <= 16 chunks: one warp each, all chunk partials loaded together
@@ -486,13 +495,13 @@ __global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_
     float4 p[kHubBlk];
 #pragma unroll
     for (int i = 0; i < kHubBlk; ++i)
-      p[i] = cb + i < ce ? __ldcg(reinterpret_cast<const float4*>(a.partials + (int64_t)(cb + i) * a.W) + c) : z4;
+      p[i] = cb + i < ce ? __ldcg(reinterpret_cast<const float4*>(pbase + (int64_t)(cb + i) * Wl) + c) : z4;
     float4 sb = p[0];
 #pragma unroll
     for (int i = 1; i < kHubBlk; ++i) add_v(sb, p[i]);
     if (lane < nv) {
       const float sv = a.srow ? a.srow[v] : 1.0f;
-      __stcs(reinterpret_cast<float4*>(a.y + (int64_t)v * a.ldy) + lane, scale_bias(sv, sb, a.bias, 4 * lane));
+      __stcs(reinterpret_cast<float4*>(ybase + (int64_t)v * a.ldy) + lane, scale_bias(sv, sb, bbase, 4 * lane));
     }
   }
 }
@@ -515,9 +524,15 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
   const uint32_t ngroups = (uint32_t)(nhg + (total - n_chunks + lg - 1) / lg);
   auto gbase = [&](int64_t g) { return g < nhg ? g * hg : n_chunks + (g - nhg) * lg; };
   auto gend = [&](int64_t g) { return g < nhg ? min((g + 1) * hg, n_chunks) : min(gbase(g) + lg, total); };
-  const int nv = a.W >> 2;
+  const int c0y = blockIdx.y * a.wsplit;                       // this launch's column chunk
+  const int Wl = min(a.wsplit, a.wtotal - c0y);
+  float* const ybase = a.y + c0y;
+  const float* const bbase = a.bias ? a.bias + c0y : nullptr;
+  float* const pbase = a.partials + (int64_t)blockIdx.y * a.pstride;
+  queue += blockIdx.y;
+  const int nv = Wl >> 2;
   const bool lane_on = lane < nv;
-  const float4* xl = reinterpret_cast<const float4*>(a.x) + (lane_on ? lane : nv - 1);
+  const float4* xl = reinterpret_cast<const float4*>(a.x + c0y) + (lane_on ? lane : nv - 1);
   const uint32_t ld4 = (uint32_t)(a.ldx >> 2);
   int32_t* ex = s_excl[w];
   auto fetch = [&](uint32_t g, int buf) {         // cp.async the 32 descriptors of group g
@@ -562,8 +577,8 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
     for (unsigned zm = zmask; zm; zm &= zm - 1) {      // rows without edges: y = bias
       const int32_t vz = s_v[w][__ffs(zm) - 1];
       if (lane_on)
-        __stcs(reinterpret_cast<float4*>(a.y + (int64_t)vz * a.ldy) + lane,
-               scale_bias(0.f, make_float4(0.f, 0.f, 0.f, 0.f), a.bias, 4 * lane));
+        __stcs(reinterpret_cast<float4*>(ybase + (int64_t)vz * a.ldy) + lane,
+               scale_bias(0.f, make_float4(0.f, 0.f, 0.f, 0.f), bbase, 4 * lane));
     }
     auto resolve = [&](int32_t pos, int32_t& u, int32_t& k) {
       int32_t lo = 0;
@@ -578,9 +593,9 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
       const int32_t hub = s_hub[w][c];
       if (lane_on) {
         if (hub < 0)
-          __stcs(reinterpret_cast<float4*>(a.y + (int64_t)s_v[w][c] * a.ldy) + lane, scale_bias(sv, sum, a.bias, 4 * lane));
+          __stcs(reinterpret_cast<float4*>(ybase + (int64_t)s_v[w][c] * a.ldy) + lane, scale_bias(sv, sum, bbase, 4 * lane));
         else
-          reinterpret_cast<float4*>(a.partials + (ib + c) * a.W)[lane] = sum;
+          reinterpret_cast<float4*>(pbase + (ib + c) * Wl)[lane] = sum;
       }
     };
     int32_t u0, k0;
@@ -812,6 +827,8 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   if (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128) {
     STG_TRY(ws->queue.alloc(nsplit, s));
     STG_CUDA(cudaMemsetAsync(ws->queue.p, 0, sizeof(uint32_t) * nsplit, s));
+    const int64_t pstride = chunks_bound * wsplit;               // the column chunks run concurrently
+    STG_TRY(ws->partials.alloc((size_t)(pstride * nsplit) + 4, s));
     const StreamFn fn = pick_stream(g_tune.d, g_tune.minb, scol != nullptr);
     // group sizes: ~max(256, E / (8 warps x #SM)) edges per group (all 32-item light
     // groups at C5 scale; small graphs get small groups, hence many warps)
@@ -823,19 +840,22 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     const int64_t ngroups = ceil_div(chunks_bound, hgrp) + ceil_div(R, lgrp) + 1;   // bound on work groups
     const int64_t blocks = std::min<int64_t>(occupancy_grid((const void*)fn), ceil_div(ngroups, 8) + 1);
     const int32_t* hids = backward ? gv->out_ids : gv->in_ids;
-    for (int k = 0; k < nsplit; ++k) {
-      const int32_t c0 = k * wsplit, wl = std::min(wsplit, W - c0);
-      Agg2Args b{};
-      b.sched = a.sched; b.col = a.col; b.srow = srow; b.scol = scol;
-      b.partials = a.partials; b.counters = a.counters;
-      b.W = wl; b.x = in + c0; b.ldx = ldin; b.y = out + c0; b.ldy = ldout;
-      b.bias = bias ? bias + c0 : nullptr;
-      b.upad = (backward && a.ids) ? (int32_t)rb : 0;   // row 0 of a shifted input is not a valid row
-      b.hgrp = hgrp; b.lgrp = lgrp;
-      fn<<<(unsigned)blocks, kAggThreads, 0, s>>>(b, ws->queue.p + k);
-      k_agg_hubs<<<(unsigned)(4 * num_sms()), 256, 0, s>>>(b, hids);
-      count_launch(2);
-    }
+    Agg2Args b{};
+    b.sched = a.sched; b.col = a.col; b.srow = srow; b.scol = scol;
+    b.partials = ws->partials.p; b.counters = a.counters;
+    b.W = wsplit; b.x = in; b.ldx = ldin; b.y = out; b.ldy = ldout;
+    b.bias = bias;
+    b.upad = (backward && a.ids) ? (int32_t)rb : 0;     // row 0 of a shifted input is not a valid row
+    b.hgrp = hgrp; b.lgrp = lgrp;
+    b.wsplit = wsplit; b.wtotal = W; b.pstride = pstride;
+    // one launch for all column chunks (gridDim.y): the chunks of a wide W (e.g. a
+    // sequence-batched S·3H) walk the graph side by side instead of one after another
+    const int64_t bx = nsplit > 1 ? std::max<int64_t>(1, std::min<int64_t>(blocks, ceil_div(occupancy_grid(
+                                                                               (const void*)fn), nsplit)))
+                                  : blocks;
+    fn<<<dim3((unsigned)bx, (unsigned)nsplit), kAggThreads, 0, s>>>(b, ws->queue.p);
+    k_agg_hubs<<<dim3((unsigned)std::max(1, 4 * num_sms() / nsplit), (unsigned)nsplit), 256, 0, s>>>(b, hids);
+    count_launch(2);
     return check_launch("aggregate_stream");
   }
   // strategy 1: pipelined items

@@ -157,6 +157,29 @@ stg_status make_tmap_f32_store(CUtensorMap* out, float* base, uint64_t rows, uin
   return STG_OK;
 }
 
+stg_status make_tmap_f32_store3(CUtensorMap* out, float* base, uint64_t planes, uint64_t rows, uint64_t cols,
+                                uint32_t box_cols, uint32_t box_rows) {
+  static PFN_encodeTiled fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess || !p)
+      return fail(STG_ERR_CUDA, "cuTensorMapEncodeTiled entry point unavailable");
+    fn = reinterpret_cast<PFN_encodeTiled>(p);
+  }
+  if ((box_cols * 4 != 64 && box_cols * 4 != 32) || (cols * 4) % 16 || ((uintptr_t)base) % 16)
+    return fail(STG_ERR_INVALID_ARG, "store map 3d: box of %u cols / alignment", box_cols);
+  const cuuint64_t dims[3] = {cols, rows, planes};
+  const cuuint64_t strides[2] = {cols * 4, rows * cols * 4};
+  const cuuint32_t box[3] = {box_cols, box_rows, 1};
+  const cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(out, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  box_cols * 4 == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B,
+                  CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(STG_ERR_CUDA, "cuTensorMapEncodeTiled (store 3d) failed (%d)", (int)r);
+  return STG_OK;
+}
+
 }  // namespace stg
 
 extern "C" {

@@ -97,6 +97,9 @@ stg_status make_tmap_f32(CUtensorMap* out, const float* base, uint64_t rows, uin
 // tc::box_off.
 stg_status make_tmap_f32_store(CUtensorMap* out, float* base, uint64_t rows, uint64_t cols, uint64_t ld,
                                uint32_t box_cols, uint32_t box_rows);
+// 3-D store map of a contiguous [planes][rows][cols] fp32 tensor, box [1][box_rows][box_cols]
+stg_status make_tmap_f32_store3(CUtensorMap* out, float* base, uint64_t planes, uint64_t rows, uint64_t cols,
+                                uint32_t box_cols, uint32_t box_rows);
 
 // ---------------------------------------------------------------- profiler
 // Per-phase device time with CUDA events on the launching stream (bench.py and

@@ -414,6 +414,12 @@ __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, int c0, int
                "r"(c0), "r"(r0), "r"(smem_u32(src))
                : "memory");
 }
+__device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, int c0, int r0, int z, const void* src) {
+  asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%1, %2, %3}], [%4];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(c0), "r"(r0), "r"(z), "r"(smem_u32(src))
+               : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
@@ -442,6 +448,29 @@ __device__ __forceinline__ void warp_box_store(unsigned char* buf0, int& slot, c
   __syncwarp();
   if (lane == 0) {
     tma_store_2d(map, c0, r0, buf);
+    bulk_commit();
+  }
+  slot ^= 1;
+}
+
+// the same into plane z of a 3-D tensor [Z][rows][cols] (rows past the plane end are clipped)
+template <int NCOL>
+__device__ __forceinline__ void warp_box_store3(unsigned char* buf0, int& slot, const float (&v)[NCOL],
+                                                const CUtensorMap* map, int c0, int r0, int z) {
+  constexpr int BYTES = 32 * NCOL * 4;
+  const int lane = threadIdx.x & 31;
+  unsigned char* buf = buf0 + slot * BYTES;
+  if (lane == 0) bulk_wait_read<1>();
+  __syncwarp();
+#pragma unroll
+  for (int c = 0; c < NCOL / 4; ++c)
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(buf + box_off<NCOL>(lane, c))),
+                 "f"(v[4 * c]), "f"(v[4 * c + 1]), "f"(v[4 * c + 2]), "f"(v[4 * c + 3])
+                 : "memory");
+  fence_proxy_async();
+  __syncwarp();
+  if (lane == 0) {
+    tma_store_3d(map, c0, r0, z, buf);
     bulk_commit();
   }
   slot ^= 1;

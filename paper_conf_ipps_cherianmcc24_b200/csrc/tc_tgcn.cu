@@ -172,7 +172,7 @@ template <int N>
 __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int Kp, const float* __restrict__ X,
                                                               const float* __restrict__ W,
                                                               const float* __restrict__ rs, float* __restrict__ P,
-                                                              int dbg) {
+                                                              int dbg, int rs_div) {
   extern __shared__ __align__(128) unsigned char sm[];
   __shared__ uint64_t full[kXwStages], empty[kXwStages], tfull[2], tempty[2];
   __shared__ uint32_t tslot;
@@ -236,7 +236,7 @@ __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int 
     for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
       const int b = i & 1, kb = i >> 1;
       const int row = tile * 128 + threadIdx.x;
-      const float sc = (rs && row < V) ? __ldg(rs + row) : 1.0f;
+      const float sc = (rs && row < V) ? __ldg(rs + row / rs_div) : 1.0f;   // row scale of vertex row / rs_div
       tc::mbar_wait(&tfull[b], kb & 1);
       tc::fence_after();
       // TMEM -> registers in 16-column pieces -> scaled row in this warp's stage
@@ -1335,6 +1335,452 @@ __global__ void k_dw_scatter(int F, int N3, int Np, const float* __restrict__ to
   }
 }
 
+// ------------------------------------------------------------------ sequence-batched GRU (NEXT-1)
+// Static graphs: C_t = Â(X_t W) + b does not depend on H, so a whole sequence's
+// aggregations run as ONE width-S·3H SpMM and the GRU recurrence, being
+// row-local, runs for all S timestamps inside one persistent kernel: a CTA
+// walks t = 0..S-1 (forward) or S-1..0 (backward) for each of its row tiles,
+// carrying H (forward) / dH (backward) in registers.  Layouts: C_all, dC'_all,
+// da_all [V][S][3H]; Hp_all [V][S][H] (slot t = H_{t-1}); RH_all [V][S][H];
+// H_seq [S][V][H] (the API's); Y_all [V][S].  The MSE head is fused: the
+// forward accumulates the loss, the backward the head gradient (G = dℓ_t/dH_t
+// + dH from t+1) and dw_o, db_o — per-CTA partials, reduced in a fixed order.
+template <int H>
+__device__ __forceinline__ float row_dot_relu(const float (&hv)[H / 2], const float* __restrict__ w, int c0) {
+  float d = 0.f;
+#pragma unroll
+  for (int j = 0; j < H / 2; ++j) d = fmaf(fmaxf(hv[j], 0.f), w[c0 + j], d);
+  return d;
+}
+
+template <int H>
+__global__ void __launch_bounds__(256, 1) k_tc_gru_seq_fwd(int V, int S, const __grid_constant__ CUtensorMap tmC,
+                                                           const __grid_constant__ CUtensorMap tmH0,
+                                                           const float* __restrict__ L, const float* __restrict__ l,
+                                                           const __grid_constant__ CUtensorMap tmHseq,
+                                                           const __grid_constant__ CUtensorMap tmHp,
+                                                           const float* __restrict__ Yall,
+                                                           const float* __restrict__ w_o,
+                                                           const float* __restrict__ b_o, double* __restrict__ lpart) {
+  using G = GruF2<H>;
+  constexpr int HH = G::HH, H3 = 3 * H;
+  constexpr int RAWC = G::NBC * kBox;                     // one C_t tile; two buffers, then H0, weights, obuf
+  extern __shared__ unsigned char sm_raw[];
+  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t full[2], h0bar, mma_bar;
+  __shared__ uint32_t tslot;
+  __shared__ float s_dot[2][128];
+  __shared__ double s_loss[8];
+  unsigned char* rawH0 = sm + 2 * RAWC;
+  unsigned char* bz_hi = rawH0 + kBox;  unsigned char* bz_lo = bz_hi + G::BG;
+  unsigned char* br_hi = bz_lo + G::BG; unsigned char* br_lo = br_hi + G::BG;
+  unsigned char* bh_hi = br_lo + G::BG; unsigned char* bh_lo = bh_hi + G::BG;
+  auto rawC = [&](int b) { return sm + (size_t)b * RAWC; };
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, hf = warp >> 2;
+  const int lr = q * 32 + lane, c0 = hf * HH;
+  unsigned char* obuf = bh_lo + G::BG + warp * G::OBUF;
+  int oslot = 0;
+  const int LG = 2 * H * H;
+  stage_gate_weights<H>(bz_hi, bz_lo, L);
+  stage_gate_weights<H>(br_hi, br_lo, L + LG);
+  stage_gate_weights<H>(bh_hi, bh_lo, L + 2 * LG);
+  if (warp == 0) tc::tmem_alloc(&tslot, G::TCOLS);
+  if (threadIdx.x == 0) {
+    tc::mbar_init(&full[0], 1); tc::mbar_init(&full[1], 1); tc::mbar_init(&h0bar, 1); tc::mbar_init(&mma_bar, 1);
+    tc::fence_mbar_init();
+  }
+  tc::fence_proxy_async();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  const uint32_t tq = tm + ((uint32_t)(q * 32) << 16);
+  const int ntiles = (V + 127) / 128;
+  float lz[HH], lrr[HH], lh[HH], wo[HH];
+#pragma unroll
+  for (int j = 0; j < HH; ++j) {
+    lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; wo[j] = w_o[c0 + j];
+  }
+  const float bo = b_o[0];
+  int my_tiles = 0;
+  for (int tl = blockIdx.x; tl < ntiles; tl += gridDim.x) ++my_tiles;
+  const int nitems = my_tiles * S;                         // item i = (tile i / S, t = i % S)
+  auto issue = [&](int i) {                                 // (thread 0) C_t boxes of item i (+ H0 at t = 0)
+    if (i >= nitems) return;
+    const int b = i & 1, tile = blockIdx.x + (i / S) * gridDim.x, t = i % S;
+    tc::mbar_expect_tx(&full[b], (uint32_t)G::NBC * kBox);
+#pragma unroll
+    for (int k = 0; k < G::NBC; ++k) tc::tma_load_2d(rawC(b) + k * kBox, &tmC, t * H3 + 32 * k, tile * 128, &full[b]);
+  };
+  auto issue_h0 = [&](int i) {                              // (thread 0) H0 box of the tile of item i
+    if (i >= nitems) return;
+    const int tile = blockIdx.x + (i / S) * gridDim.x;
+    tc::mbar_expect_tx(&h0bar, (uint32_t)kBox);
+    tc::tma_load_2d(rawH0, &tmH0, 0, tile * 128, &h0bar);
+  };
+  if (threadIdx.x == 0) { issue(0); issue(1); issue_h0(0); }
+  const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0);
+  uint32_t mph = 0, h0ph = 0;
+  double lacc = 0.0;
+  float h[HH];
+  for (int i = 0; i < nitems; ++i) {
+    const int b = i & 1, tile = blockIdx.x + (i / S) * gridDim.x, t = i % S, r0 = tile * 128;
+    const int row = r0 + lr;
+    tc::mbar_wait(&full[b], (i >> 1) & 1);
+    {
+      float tt[HH];
+      raw_to_tmem<HH>(rawC(b), lr, c0, tq + c0, tq + 3 * H + c0, tt);                    // C_z
+      raw_to_tmem<HH>(rawC(b), lr, H + c0, tq + H + c0, tq + 4 * H + c0, tt);            // C_r
+      raw_to_tmem<HH>(rawC(b), lr, 2 * H + c0, tq + 6 * H + c0, tq + 7 * H + c0, tt);    // C_h
+      if (t == 0) {                                                                      // H_{-1} = H0
+        tc::mbar_wait(&h0bar, h0ph);
+        h0ph ^= 1;
+        raw_to_tmem<HH>(rawH0, lr, c0, tq + 2 * H + c0, tq + 5 * H + c0, h);
+      } else {                                                                           // H_{t-1} from registers
+        tmem_st_split<HH>(tq + 2 * H + c0, tq + 5 * H + c0, h);
+      }
+    }
+    tc::warp_box_store<HH>(obuf, oslot, h, 1.0f, &tmHp, t * H + c0, r0 + q * 32);          // Hp_all slot t
+    tc::tmem_wait_st();
+    tc::fence_before();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      tc::fence_after();
+      const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
+      mma_ts_seg(tm + 8 * H, tm + 0, tm + 3 * H, zh, zl, 2 * H, 0, H, idesc, true);
+      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, idesc, false);
+      mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, idesc, true);
+      mma_ts_seg(tm + 9 * H, tm + 2 * H, tm + 5 * H, rh_, rl, 2 * H, H, H, idesc, false);
+      tc::commit(&mma_bar);
+      issue(i + 2);                                       // raw buffer b is in TMEM
+      if (t == 0) issue_h0(i + S);                        // the next tile's H0 (rawH0 consumed)
+    }
+    tc::mbar_wait(&mma_bar, mph);
+    mph ^= 1;
+    tc::fence_after();
+    float z[HH];
+    {
+      float az[HH], ar[HH], rh[HH], lo[HH];
+      tmem_row_load<HH>(tm + 8 * H, c0, az);
+      tmem_row_load<HH>(tm + 9 * H, c0, ar);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        z[j] = sigm(az[j] + lz[j]);
+        rh[j] = sigm(ar[j] + lrr[j]) * h[j];
+        lo[j] = rh[j] - tc::tf32_hi(rh[j]);
+      }
+      if constexpr (HH == 16) { tc::tmem_st16(tq + 10 * H + c0, rh); tc::tmem_st16(tq + 11 * H + c0, lo); }
+      else { tc::tmem_st8(tq + 10 * H + c0, rh); tc::tmem_st8(tq + 11 * H + c0, lo); }
+    }
+    tc::tmem_wait_st();
+    tc::fence_before();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      tc::fence_after();
+      const uint32_t hh_ = tc::smem_u32(bh_hi), hl = tc::smem_u32(bh_lo);
+      mma_ts_seg(tm + 12 * H, tm + 6 * H, tm + 7 * H, hh_, hl, 2 * H, 0, H, idesc, true);
+      mma_ts_seg(tm + 12 * H, tm + 10 * H, tm + 11 * H, hh_, hl, 2 * H, H, H, idesc, false);
+      tc::commit(&mma_bar);
+    }
+    tc::mbar_wait(&mma_bar, mph);
+    mph ^= 1;
+    tc::fence_after();
+    {
+      float ah[HH];
+      tmem_row_load<HH>(tm + 12 * H, c0, ah);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        const float hh = tanhf(ah[j] + lh[j]);
+        h[j] = z[j] * h[j] + (1.0f - z[j]) * hh;          // H_t
+      }
+    }
+    tc::warp_box_store3<HH>(obuf, oslot, h, &tmHseq, c0, r0 + q * 32, t);                // H_seq[t]
+    // fused head, forward: loss += (Σ_k ReLU(H_t)·w_o + b_o − y_t)² over the tile's rows
+    s_dot[hf][lr] = row_dot_relu<H>(h, wo, 0);
+    tc::fence_before();
+    __syncthreads();
+    if (hf == 0 && row < V) {
+      const float e = (s_dot[0][lr] + s_dot[1][lr] + bo) - Yall[(int64_t)row * S + t];
+      lacc += (double)e * (double)e;
+    }
+  }
+  // per-CTA loss partial (fixed order: lanes, then warps)
+#pragma unroll
+  for (int o = 16; o; o >>= 1) lacc += __shfl_xor_sync(0xffffffffu, lacc, o);
+  if (lane == 0) s_loss[warp] = lacc;
+  if (lane == 0) tc::bulk_wait_all();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double tot = 0.0;
+    for (int w = 0; w < 8; ++w) tot += s_loss[w];
+    lpart[blockIdx.x] = tot;
+  }
+  if (warp == 0) tc::tmem_free(tm, G::TCOLS);
+}
+
+template <int H>
+__global__ void __launch_bounds__(256, 1) k_tc_gru_seq_bwd(int V, int S, const __grid_constant__ CUtensorMap tmC,
+                                                           const __grid_constant__ CUtensorMap tmHp,
+                                                           const __grid_constant__ CUtensorMap tmHs,
+                                                           const float* __restrict__ L, const float* __restrict__ l,
+                                                           const float* __restrict__ ndst,
+                                                           const float* __restrict__ Yall,
+                                                           const float* __restrict__ w_o,
+                                                           const float* __restrict__ b_o, float inv_vn,
+                                                           const __grid_constant__ CUtensorMap tmDC,
+                                                           const __grid_constant__ CUtensorMap tmDA,
+                                                           const __grid_constant__ CUtensorMap tmRH,
+                                                           float* __restrict__ gpart) {
+  using G = GruB2<H>;
+  constexpr int H3 = G::H3, HH = G::HH;
+  extern __shared__ unsigned char sm_raw[];
+  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t full, mma_bar;
+  __shared__ uint32_t tslot;
+  __shared__ float s_l[3 * H];
+  __shared__ float s_dot[2][128];
+  __shared__ float s_g[4][H + 1];
+  unsigned char* w0 = sm + G::WOFF;
+  unsigned char* bz_hi = w0;              unsigned char* bz_lo = w0 + 1 * G::BG;
+  unsigned char* br_hi = w0 + 2 * G::BG;  unsigned char* br_lo = w0 + 3 * G::BG;
+  unsigned char* bh_hi = w0 + 4 * G::BG;  unsigned char* bh_lo = w0 + 5 * G::BG;
+  unsigned char* lz_hi = w0 + 6 * G::BG;  unsigned char* lz_lo = w0 + 7 * G::BG;
+  unsigned char* lr_hi = w0 + 8 * G::BG;  unsigned char* lr_lo = w0 + 9 * G::BG;
+  unsigned char* lh_hi = w0 + 10 * G::BG; unsigned char* lh_lo = w0 + 11 * G::BG;
+  unsigned char* rawC = sm;
+  unsigned char* rawH = sm + G::NBC * kBox;                 // H_{t-1}
+  unsigned char* rawT = sm + (G::NBC + G::NBH) * kBox;      // H_t (the head's input)
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, hf = warp >> 2;
+  const int lr = q * 32 + lane, c0 = hf * HH;
+  unsigned char* obuf = w0 + 12 * G::BG + warp * G::OBUF;
+  int oslot = 0;
+  for (int e = threadIdx.x; e < 3 * H; e += blockDim.x) s_l[e] = l[e];
+  const int LG = 2 * H * H;
+  stage_gate_weights<H>(bz_hi, bz_lo, L);
+  stage_gate_weights<H>(br_hi, br_lo, L + LG);
+  stage_gate_weights<H>(bh_hi, bh_lo, L + 2 * LG);
+  stage_plain<H>(lz_hi, lz_lo, L);
+  stage_plain<H>(lr_hi, lr_lo, L + LG);
+  stage_plain<H>(lh_hi, lh_lo, L + 2 * LG);
+  if (warp == 0) tc::tmem_alloc(&tslot, G::TCOLS);
+  if (threadIdx.x == 0) {
+    tc::mbar_init(&full, 1); tc::mbar_init(&mma_bar, 1);
+    tc::fence_mbar_init();
+  }
+  tc::fence_proxy_async();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  const uint32_t tq = tm + ((uint32_t)(q * 32) << 16);
+  const int ntiles = (V + 127) / 128;
+  float wo[HH];
+#pragma unroll
+  for (int j = 0; j < HH; ++j) wo[j] = w_o[c0 + j];
+  const float bo = b_o[0];
+  int my_tiles = 0;
+  for (int tl = blockIdx.x; tl < ntiles; tl += gridDim.x) ++my_tiles;
+  const int nitems = my_tiles * S;                         // item i = (tile i / S, t = S-1 - i % S)
+  auto issue = [&](int i) {
+    if (i >= nitems) return;
+    const int tile = blockIdx.x + (i / S) * gridDim.x, t = S - 1 - i % S;
+    tc::mbar_expect_tx(&full, (uint32_t)(G::NBC + 2 * G::NBH) * kBox);
+#pragma unroll
+    for (int k = 0; k < G::NBC; ++k) tc::tma_load_2d(rawC + k * kBox, &tmC, t * H3 + 32 * k, tile * 128, &full);
+    tc::tma_load_2d(rawH, &tmHp, t * H, tile * 128, &full);
+    tc::tma_load_2d(rawT, &tmHs, 0, t * V + tile * 128, &full);   // H_seq as [S·V, H]: rows past V are
+                                                                    // the next plane's, unused (gs = 0 there)
+  };
+  if (threadIdx.x == 0) issue(0);
+  const uint32_t id_h = tc::idesc_tf32(128, H, 0, 0), id_2h = tc::idesc_tf32(128, 2 * H, 0, 0);
+  auto mma_wait = [&](uint32_t& ph) {
+    tc::mbar_wait(&mma_bar, ph);
+    ph ^= 1;
+    tc::fence_after();
+  };
+  auto sync_tmem = [&]() {
+    tc::tmem_wait_st();
+    tc::fence_before();
+    __syncthreads();
+  };
+  uint32_t mph = 0;
+  float dh[HH];                                             // dℓ/dH_t flowing back from t+1
+  float gw[HH], gb = 0.f;                                   // head gradient partials (dw_o, db_o)
+#pragma unroll
+  for (int j = 0; j < HH; ++j) gw[j] = 0.f;
+  for (int i = 0; i < nitems; ++i) {
+    const int tile = blockIdx.x + (i / S) * gridDim.x, t = S - 1 - i % S;
+    const int r0 = tile * 128, wr0 = r0 + q * 32, row = r0 + lr;
+    if (t == S - 1) {
+#pragma unroll
+      for (int j = 0; j < HH; ++j) dh[j] = 0.f;
+    }
+    const float nd = row < V ? __ldg(ndst + row) : 0.f;
+    tc::mbar_wait(&full, i & 1);
+    float h[HH], g[HH];
+    {
+      float tt[HH], ht[HH];
+      raw_to_tmem<HH>(rawC, lr, c0, tq + c0, tq + 3 * H + c0, tt);                    // C_z
+      raw_to_tmem<HH>(rawC, lr, H + c0, tq + H + c0, tq + 4 * H + c0, tt);            // C_r
+      raw_to_tmem<HH>(rawC, lr, 2 * H + c0, tq + 6 * H + c0, tq + 7 * H + c0, tt);    // C_h
+      raw_to_tmem<HH>(rawH, lr, c0, tq + 2 * H + c0, tq + 5 * H + c0, h);            // H_{t-1}
+      const unsigned char* box = rawT + (c0 / 32) * kBox;
+#pragma unroll
+      for (int qq = 0; qq < HH / 4; ++qq) {
+        const float4 x = *reinterpret_cast<const float4*>(box + tc::swz128(lr, (c0 % 32) / 4 + qq));
+        ht[4 * qq] = x.x; ht[4 * qq + 1] = x.y; ht[4 * qq + 2] = x.z; ht[4 * qq + 3] = x.w;
+      }
+      // fused head, backward: gs = 2(ŷ − y)/V_total;  G = gs·w_o⊙[H_t > 0] + dH(t+1)
+      s_dot[hf][lr] = row_dot_relu<H>(ht, wo, 0);
+      sync_tmem();
+      const float yv = row < V ? Yall[(int64_t)row * S + t] : 0.f;
+      const float e = (s_dot[0][lr] + s_dot[1][lr] + bo) - yv;
+      const float gs = row < V ? 2.0f * e * inv_vn : 0.f;
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        const float r = fmaxf(ht[j], 0.f);
+        g[j] = (ht[j] > 0.f ? gs * wo[j] : 0.f) + dh[j];
+        gw[j] = fmaf(gs, r, gw[j]);
+      }
+      if (hf == 0) gb += gs;
+    }
+    if (threadIdx.x == 0) {                             // P1; then request the next item
+      tc::fence_after();
+      const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
+      mma_ts_seg(tm + 8 * H, tm + 0, tm + 3 * H, zh, zl, 2 * H, 0, H, id_h, true);
+      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, id_h, false);
+      mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, id_h, true);
+      mma_ts_seg(tm + 9 * H, tm + 2 * H, tm + 5 * H, rh_, rl, 2 * H, H, H, id_h, false);
+      tc::commit(&mma_bar);
+      issue(i + 1);
+    }
+    mma_wait(mph);
+    float z[HH], r[HH];
+    {
+      float az[HH], ar[HH], rh[HH];
+      tmem_row_load<HH>(tm + 8 * H, c0, az);
+      tmem_row_load<HH>(tm + 9 * H, c0, ar);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        z[j] = sigm(az[j] + s_l[c0 + j]);
+        r[j] = sigm(ar[j] + s_l[H + c0 + j]);
+        rh[j] = r[j] * h[j];
+      }
+      tmem_st_split<HH>(tq + 10 * H + c0, tq + 11 * H + c0, rh);
+      sync_tmem();
+      if (threadIdx.x == 0) {                           // P2
+        tc::fence_after();
+        const uint32_t hh_ = tc::smem_u32(bh_hi), hl = tc::smem_u32(bh_lo);
+        mma_ts_seg(tm + 12 * H, tm + 6 * H, tm + 7 * H, hh_, hl, 2 * H, 0, H, id_h, true);
+        mma_ts_seg(tm + 12 * H, tm + 10 * H, tm + 11 * H, hh_, hl, 2 * H, H, H, id_h, false);
+        tc::commit(&mma_bar);
+      }
+      tc::warp_box_store<HH>(obuf, oslot, rh, 1.0f, &tmRH, t * H + c0, wr0);          // RH_t
+    }
+    mma_wait(mph);
+    float dhn[HH];
+    {
+      float ah[HH], dah[HH], daz[HH];
+      tmem_row_load<HH>(tm + 12 * H, c0, ah);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        const float hh = tanhf(ah[j] + s_l[2 * H + c0 + j]);
+        const float dZ = g[j] * (h[j] - hh), dHh = g[j] * (1.0f - z[j]);
+        dah[j] = dHh * (1.0f - hh * hh);
+        daz[j] = dZ * z[j] * (1.0f - z[j]);
+        dhn[j] = g[j] * z[j];
+      }
+      tmem_st_split<HH>(tq + c0, tq + H + c0, dah);
+      tmem_st_split<HH>(tq + 2 * H + c0, tq + 3 * H + c0, daz);
+      sync_tmem();
+      if (threadIdx.x == 0) {                           // P3
+        tc::fence_after();
+        mma_ts_seg(tm + 4 * H, tm + 0, tm + H, tc::smem_u32(lh_hi), tc::smem_u32(lh_lo), H, 0, H, id_2h, true);
+        mma_ts_seg(tm + 6 * H, tm + 2 * H, tm + 3 * H, tc::smem_u32(lz_hi), tc::smem_u32(lz_lo), H, 0, H, id_2h, true);
+        tc::commit(&mma_bar);
+      }
+      tc::warp_box_store<HH>(obuf, oslot, daz, 1.0f, &tmDA, t * H3 + c0, wr0);         // da_z
+      tc::warp_box_store<HH>(obuf, oslot, dah, 1.0f, &tmDA, t * H3 + 2 * H + c0, wr0); // da_h
+    }
+    mma_wait(mph);
+    {
+      float dch[HH], drh[HH], dar[HH];
+      tmem_row_load<HH>(tm + 4 * H, c0, dch);
+      tmem_row_load<HH>(tm + 5 * H, c0, drh);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) {
+        dhn[j] += drh[j] * r[j];
+        dar[j] = drh[j] * h[j] * r[j] * (1.0f - r[j]);
+      }
+      tmem_st_split<HH>(tq + 10 * H + c0, tq + 11 * H + c0, dar);
+      sync_tmem();
+      if (threadIdx.x == 0) {                           // P4
+        tc::fence_after();
+        mma_ts_seg(tm + 8 * H, tm + 10 * H, tm + 11 * H, tc::smem_u32(lr_hi), tc::smem_u32(lr_lo), H, 0, H, id_2h, true);
+        tc::commit(&mma_bar);
+      }
+      tc::warp_box_store<HH>(obuf, oslot, dch, nd, &tmDC, t * H3 + 2 * H + c0, wr0);   // dC'_h
+      tc::warp_box_store<HH>(obuf, oslot, dar, 1.0f, &tmDA, t * H3 + H + c0, wr0);     // da_r
+      float dcz[HH], dhz[HH];
+      tmem_row_load<HH>(tm + 6 * H, c0, dcz);
+      tmem_row_load<HH>(tm + 7 * H, c0, dhz);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) dhn[j] += dhz[j];
+      tc::warp_box_store<HH>(obuf, oslot, dcz, nd, &tmDC, t * H3 + c0, wr0);          // dC'_z
+    }
+    mma_wait(mph);
+    {
+      float dcr[HH], dhr[HH];
+      tmem_row_load<HH>(tm + 8 * H, c0, dcr);
+      tmem_row_load<HH>(tm + 9 * H, c0, dhr);
+#pragma unroll
+      for (int j = 0; j < HH; ++j) dh[j] = dhn[j] + dhr[j];                           // dℓ/dH_{t-1}
+      tc::warp_box_store<HH>(obuf, oslot, dcr, nd, &tmDC, t * H3 + H + c0, wr0);      // dC'_r
+    }
+    tc::fence_before();
+    __syncthreads();
+  }
+  // head-gradient partials of this CTA: rows (lanes, then the 4 lane quarters) in a fixed order
+#pragma unroll
+  for (int j = 0; j < HH; ++j) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) gw[j] += __shfl_xor_sync(0xffffffffu, gw[j], o);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) gb += __shfl_xor_sync(0xffffffffu, gb, o);
+  for (int qq = 0; qq < 4; ++qq) {
+    if (q == qq && lane == 0) {
+#pragma unroll
+      for (int j = 0; j < HH; ++j) s_g[qq][c0 + j] = gw[j];
+      if (hf == 0) s_g[qq][H] = gb;
+    }
+  }
+  if (lane == 0) tc::bulk_wait_all();
+  __syncthreads();
+  for (int k = threadIdx.x; k <= H; k += blockDim.x)
+    gpart[(int64_t)blockIdx.x * (H + 1) + k] = ((s_g[0][k] + s_g[1][k]) + s_g[2][k]) + s_g[3][k];
+  if (warp == 0) tc::tmem_free(tm, G::TCOLS);
+}
+
+// fixed-order sum of the per-CTA partials of the fused head: loss (double, ÷ V_total),
+// dw_o [H], db_o [1]
+__global__ void k_seq_head_reduce(int nb, int H, const double* __restrict__ lpart, const float* __restrict__ gpart,
+                                  double inv_vn, float* __restrict__ loss, float* __restrict__ dw_o,
+                                  float* __restrict__ db_o) {
+  const int k = threadIdx.x;
+  if (lpart && k == 0 && loss) {
+    double t = 0.0;
+    for (int b = 0; b < nb; ++b) t += lpart[b];
+    *loss += (float)(t * inv_vn);
+  }
+  if (gpart && k <= H) {
+    float t = 0.f;
+    for (int b = 0; b < nb; ++b) t += gpart[(int64_t)b * (H + 1) + k];
+    if (k < H) { if (dw_o) dw_o[k] += t; }
+    else if (db_o) db_o[0] += t;
+  }
+}
+
 template <class K>
 int occupancy_blocks(K fn, size_t smem, int threads = kTcThreads) {
   int per_sm = 0;
@@ -1357,7 +1803,8 @@ stg_status prep(K fn, size_t smem) {
 bool tc_supported(int F, int H) { return (H == 16 || H == 32) && F % 4 == 0 && F <= 128 && F >= 4; }
 // part for tc_dw / tc_dl: tc_atb_max_blocks() · 2 · 128 · 128 floats; tot: 2 · 128 · 128
 
-stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s) {
+stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s,
+                 int rs_div) {
   const int N = 3 * H, Kp = (F + 7) / 8 * 8;
   const int ntiles = (V + 127) / 128;
   if (Kp <= 64) {                     // pipelined kernel (2-stage ring of 128 x Kp tiles + output stage)
@@ -1368,12 +1815,13 @@ stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const floa
     const int dbg = dv ? atoi(dv) : 0;
     if (H == 32) {
       STG_TRY(prep(k_tc_xw_pipe<96>, smem));
-      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg);
+      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div);
     } else {
       STG_TRY(prep(k_tc_xw_pipe<48>, smem));
-      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg);
+      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div);
     }
   } else {                            // 64 < F <= 128: one tile per CTA at a time
+    if (rs_div != 1) return fail(STG_ERR_INVALID_ARG, "tc_xw: row-scale divisor needs F <= 64");
     const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)2 * 128 * Kp * 4;
     if (H == 32) {
       STG_TRY(prep(k_tc_xw<96>, smem));
@@ -1555,6 +2003,74 @@ stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH,
   k_dl_scatter<<<(6 * H * H + 6 * H + 255) / 256, 256, 0, s>>>(H, N, 32, N, tot, L, dL, dl, db);
   count_launch(2);
   return check_launch("tc_dl");
+}
+
+}  // namespace stg
+
+namespace stg {
+
+// ---- sequence-batched GRU launchers (NEXT-1; layouts in the kernels' comment)
+stg_status tc_gru_seq_fwd(int V, int S, int H, const float* C_all, const float* H0, const float* L, const float* l,
+                          float* H_seq, float* Hp_all, const float* Y_all, const float* w_o, const float* b_o,
+                          double* lpart, int* nb_out, cudaStream_t s) {
+  const int ntiles = (V + 127) / 128;
+  const int nb = std::min(ntiles, num_sms());
+  const uint32_t hh = (uint32_t)H / 2;
+  CUtensorMap tmC, tmH0, tmHs, tmHp;
+  STG_TRY(make_tmap_f32(&tmC, C_all, (uint64_t)V, (uint64_t)S * 3 * H, (uint64_t)S * 3 * H, 32, 128));
+  STG_TRY(make_tmap_f32(&tmH0, H0, (uint64_t)V, H, H, 32, 128));
+  STG_TRY(make_tmap_f32_store3(&tmHs, H_seq, (uint64_t)S, (uint64_t)V, H, hh, 32));
+  STG_TRY(make_tmap_f32_store(&tmHp, Hp_all, (uint64_t)V, (uint64_t)S * H, (uint64_t)S * H, hh, 32));
+  if (H == 32) {
+    using G = GruF2<32>;
+    const size_t smem = 2 * G::NBC * kBox + kBox + 6 * G::BG + 8 * G::OBUF + 1024;
+    STG_TRY(prep(k_tc_gru_seq_fwd<32>, smem));
+    k_tc_gru_seq_fwd<32><<<nb, 256, smem, s>>>(V, S, tmC, tmH0, L, l, tmHs, tmHp, Y_all, w_o, b_o, lpart);
+  } else {
+    using G = GruF2<16>;
+    const size_t smem = 2 * G::NBC * kBox + kBox + 6 * G::BG + 8 * G::OBUF + 1024;
+    STG_TRY(prep(k_tc_gru_seq_fwd<16>, smem));
+    k_tc_gru_seq_fwd<16><<<nb, 256, smem, s>>>(V, S, tmC, tmH0, L, l, tmHs, tmHp, Y_all, w_o, b_o, lpart);
+  }
+  count_launch();
+  *nb_out = nb;
+  return check_launch("tc_gru_seq_fwd");
+}
+
+stg_status tc_gru_seq_bwd(int V, int S, int H, const float* C_all, const float* Hp_all, const float* H_seq,
+                          const float* L, const float* l, const float* ndst, const float* Y_all, const float* w_o,
+                          const float* b_o, float inv_vn, float* dC_all, float* da_all, float* RH_all, float* gpart,
+                          int* nb_out, cudaStream_t s) {
+  const int ntiles = (V + 127) / 128;
+  const int nb = std::min(ntiles, num_sms());
+  const uint32_t hh = (uint32_t)H / 2;
+  const uint64_t H3S = (uint64_t)S * 3 * H;
+  CUtensorMap tmC, tmHp, tmHs, tmDC, tmDA, tmRH;
+  STG_TRY(make_tmap_f32(&tmC, C_all, (uint64_t)V, H3S, H3S, 32, 128));
+  STG_TRY(make_tmap_f32(&tmHp, Hp_all, (uint64_t)V, (uint64_t)S * H, (uint64_t)S * H, 32, 128));
+  STG_TRY(make_tmap_f32(&tmHs, H_seq, (uint64_t)S * V, H, H, 32, 128));
+  STG_TRY(make_tmap_f32_store(&tmDC, dC_all, (uint64_t)V, H3S, H3S, hh, 32));
+  STG_TRY(make_tmap_f32_store(&tmDA, da_all, (uint64_t)V, H3S, H3S, hh, 32));
+  STG_TRY(make_tmap_f32_store(&tmRH, RH_all, (uint64_t)V, (uint64_t)S * H, (uint64_t)S * H, hh, 32));
+  if (H == 32) {
+    STG_TRY(prep(k_tc_gru_seq_bwd<32>, GruB2<32>::SMEM));
+    k_tc_gru_seq_bwd<32><<<nb, 256, GruB2<32>::SMEM, s>>>(V, S, tmC, tmHp, tmHs, L, l, ndst, Y_all, w_o, b_o, inv_vn,
+                                                          tmDC, tmDA, tmRH, gpart);
+  } else {
+    STG_TRY(prep(k_tc_gru_seq_bwd<16>, GruB2<16>::SMEM));
+    k_tc_gru_seq_bwd<16><<<nb, 256, GruB2<16>::SMEM, s>>>(V, S, tmC, tmHp, tmHs, L, l, ndst, Y_all, w_o, b_o, inv_vn,
+                                                          tmDC, tmDA, tmRH, gpart);
+  }
+  count_launch();
+  *nb_out = nb;
+  return check_launch("tc_gru_seq_bwd");
+}
+
+stg_status tc_seq_head_reduce(int nb, int H, const double* lpart, const float* gpart, double inv_vn, float* loss,
+                              float* dw_o, float* db_o, cudaStream_t s) {
+  k_seq_head_reduce<<<1, 128, 0, s>>>(nb, H, lpart, gpart, inv_vn, loss, dw_o, db_o);
+  count_launch();
+  return check_launch("tc_seq_head_reduce");
 }
 
 }  // namespace stg

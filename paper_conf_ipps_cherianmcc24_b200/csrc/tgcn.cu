@@ -18,7 +18,17 @@
 namespace stg {
 bool tc_supported(int F, int H);
 int tc_atb_max_blocks();
-stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s);
+stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s,
+                 int rs_div = 1);
+stg_status tc_gru_seq_fwd(int V, int S, int H, const float* C_all, const float* H0, const float* L, const float* l,
+                          float* H_seq, float* Hp_all, const float* Y_all, const float* w_o, const float* b_o,
+                          double* lpart, int* nb_out, cudaStream_t s);
+stg_status tc_gru_seq_bwd(int V, int S, int H, const float* C_all, const float* Hp_all, const float* H_seq,
+                          const float* L, const float* l, const float* ndst, const float* Y_all, const float* w_o,
+                          const float* b_o, float inv_vn, float* dC_all, float* da_all, float* RH_all, float* gpart,
+                          int* nb_out, cudaStream_t s);
+stg_status tc_seq_head_reduce(int nb, int H, const double* lpart, const float* gpart, double inv_vn, float* loss,
+                              float* dw_o, float* db_o, cudaStream_t s);
 stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float* L, const float* l, float* Hn,
                       cudaStream_t s);
 stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float* G, const float* L, const float* l,
@@ -427,6 +437,26 @@ __global__ void k_sgd(float* __restrict__ p, float* __restrict__ g, int64_t n, f
   }
 }
 
+// Sequence-batched layouts: X_all[v][t][:] = X_t[v][:], Y_all[v][t] = y_t[v], b_all[t][:] = b
+constexpr int kSeqMax = 64;
+struct SeqPtrs {
+  const float* x[kSeqMax];
+  const float* y[kSeqMax];
+};
+__global__ void k_seq_gather(const SeqPtrs ptrs, int S, int V, int F, const float* __restrict__ b, int H3,
+                             float* __restrict__ X_all, float* __restrict__ Y_all, float* __restrict__ b_all) {
+  const int64_t nx = (int64_t)V * S * F;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nx; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = e / ((int64_t)S * F);
+    const int t = (int)((e / F) % S), f = (int)(e % F);
+    X_all[e] = __ldg(ptrs.x[t] + v * F + f);
+  }
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < (int64_t)V * S;
+       e += (int64_t)gridDim.x * blockDim.x)
+    Y_all[e] = __ldg(ptrs.y[e % S] + e / S);
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < S * H3; e += gridDim.x * blockDim.x) b_all[e] = b[e % H3];
+}
+
 int grid_blocks(const void* fn, size_t smem, int64_t tiles) {
   int per_sm = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kT, smem) != cudaSuccess || per_sm < 1) {
@@ -450,6 +480,9 @@ stg_status set_smem(K fn, size_t smem) {
 struct TgcnWs {
   DArray<float> P, dC, dP, part_gru, part_dw, gpart, da, RH, part_tc, dl_tmp, part_dl, dl_tmp2;
   DArray<double> lpart;
+  // sequence-batched path: X_all, Y_all, b_all, then [V][S][·] activations and the head partials
+  DArray<float> sX, sY, sb, sP, sC, sHp, sdC, sdP, sda, sRH, sgpart;
+  DArray<double> slpart;
 };
 
 }  // namespace stg
@@ -942,6 +975,78 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
   }
   for (int b = 0; b < 2 && b < S; ++b) STG_TRY(wait(ms, ev_bdone[b], as));   // join
   return STG_OK;
+}
+
+// Sequence-batched Algorithm 1 over a STATIC graph: the
+// same model and gradients as stg_tgcn_train_sequence, scheduled per sequence
+// instead of per timestamp (see k_tc_gru_seq_fwd).  10 kernel launches per
+// sequence instead of ~17 per timestamp.
+stg_status stg_tgcn_train_sequence_batched(const stg_graph* graph, int32_t S, const stg_tgcn_params* p,
+                                           const float* w_o, const float* b_o, const float* const* X,
+                                           const float* const* Y, const float* H0, float* H_seq,
+                                           stg_tgcn_grads* grads, float* dw_o, float* db_o, float* loss_accum,
+                                           stg_state_stack* stack, stg_stream_t stream) {
+  if (!graph || S < 1 || !X || !Y || !H0 || !H_seq || !stack || !w_o || !b_o)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_batched: bad arguments");
+  if (S > kSeqMax) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_batched: S=%d > %d", S, kSeqMax);
+  if (!grads || !grads->W || !grads->b || !grads->L || !grads->l)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_batched: NULL gradient pointer");
+  STG_TRY(check_params(p));
+  const int32_t F = p->F, H = p->H, H3 = 3 * H;
+  if (!tc_supported(F, H) || F > 64)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_batched: needs the tensor-core path (H 16|32, F%%4, F<=64)");
+  stg_csr_view view;
+  STG_TRY(stg_graph_view(graph, &view));
+  if (view.row_begin != 0 || view.row_end != view.num_nodes)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_batched: sharded graphs use the per-step driver");
+  const int32_t V = view.num_nodes;
+  const size_t VS = (size_t)V * S;
+  cudaStream_t s = (cudaStream_t)stream;
+  TgcnWs& ws = stack->ws;
+  const int nbmax = num_sms();
+  STG_TRY(ws.sX.alloc(VS * F)); STG_TRY(ws.sY.alloc(VS)); STG_TRY(ws.sb.alloc((size_t)S * H3));
+  STG_TRY(ws.sP.alloc(VS * H3)); STG_TRY(ws.sC.alloc(VS * H3)); STG_TRY(ws.sHp.alloc(VS * H));
+  STG_TRY(ws.sdC.alloc(VS * H3)); STG_TRY(ws.sdP.alloc(VS * H3)); STG_TRY(ws.sda.alloc(VS * H3));
+  STG_TRY(ws.sRH.alloc(VS * H)); STG_TRY(ws.slpart.alloc(nbmax)); STG_TRY(ws.sgpart.alloc((size_t)nbmax * (H + 1)));
+  STG_TRY(ws.part_tc.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));
+  STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
+  SeqPtrs ptrs{};
+  for (int t = 0; t < S; ++t) {
+    if (!X[t] || !Y[t]) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_batched: NULL X/Y at %d", t);
+    ptrs.x[t] = X[t];
+    ptrs.y[t] = Y[t];
+  }
+  k_seq_gather<<<(unsigned)std::min<int64_t>(ceil_div((int64_t)VS * F, 256), 4096), 256, 0, s>>>(
+      ptrs, S, V, F, p->b, H3, ws.sX.p, ws.sY.p, ws.sb.p);
+  count_launch();
+  {
+    ProfScope prof(PH_XW, s);                        // P'_all = diag(n_src)·X_all·W over V·S rows
+    STG_TRY(tc_xw(V * S, F, H, ws.sX.p, p->W, view.norm_src, ws.sP.p, s, S));
+  }
+  // C_all = Â·P'_all + b: one aggregation of width S·3H for the whole sequence
+  STG_TRY(aggregate_launch(&view, 0, S * H3, ws.sP.p, S * H3, ws.sC.p, S * H3, view.norm_dst, nullptr, ws.sb.p, s));
+  int nb1 = 0, nb2 = 0;
+  {
+    ProfScope prof(PH_GRU_FWD, s);                   // GRU over t = 0..S-1 + loss
+    STG_TRY(tc_gru_seq_fwd(V, S, H, ws.sC.p, H0, p->L, p->l, H_seq, ws.sHp.p, ws.sY.p, w_o, b_o, ws.slpart.p, &nb1,
+                           s));
+    STG_TRY(tc_seq_head_reduce(nb1, H, ws.slpart.p, nullptr, 1.0 / V, loss_accum, nullptr, nullptr, s));
+  }
+  {
+    ProfScope prof(PH_GRU_BWD, s);                   // GRU backward over t = S-1..0 + head gradient
+    STG_TRY(tc_gru_seq_bwd(V, S, H, ws.sC.p, ws.sHp.p, H_seq, p->L, p->l, view.norm_dst, ws.sY.p, w_o, b_o,
+                           1.0f / (float)V, ws.sdC.p, ws.sda.p, ws.sRH.p, ws.sgpart.p, &nb2, s));
+    STG_TRY(tc_seq_head_reduce(nb2, H, nullptr, ws.sgpart.p, 0.0, nullptr, dw_o, db_o, s));
+  }
+  {
+    ProfScope prof(PH_DL, s);                        // dL, dl, db over all V·S (row, t) pairs
+    STG_TRY(tc_dl(V * S, H, ws.sC.p, ws.sHp.p, ws.sRH.p, ws.sda.p, ws.part_tc.p, ws.dl_tmp.p, grads->L, grads->l,
+                  grads->b, p->L, s));
+  }
+  // dP_all = diag(n_src)·Âᵀ·dC'_all (width S·3H), dW += X_allᵀ·dP_all
+  STG_TRY(aggregate_launch(&view, 1, S * H3, ws.sdC.p, S * H3, ws.sdP.p, S * H3, view.norm_src, nullptr, nullptr, s));
+  ProfScope prof(PH_DW, s);
+  return tc_dw(V * S, F, H, ws.sX.p, ws.sdP.p, ws.part_tc.p, ws.dl_tmp.p, grads->W, s);
 }
 
 }  // extern "C"

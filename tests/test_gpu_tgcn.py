@@ -182,3 +182,53 @@ def test_sgd_update(stg):
     stg.stg_sgd_update(p, g, 0.5)
     assert torch.equal(p, torch.arange(10, dtype=torch.float32, device="cuda") - 0.5)
     assert torch.count_nonzero(g) == 0
+
+
+def _run_batched(stg, g, cfg, pg, Xs, Ys, H0, S):
+    V, H, F = cfg.V, pg["L"].shape[2], cfg.F
+    grads = _zero_grads(F, H)
+    dw, db, loss = torch.zeros(H, device="cuda"), torch.zeros(1, device="cuda"), torch.zeros(1, device="cuda")
+    Hseq = torch.empty(S, V, H, device="cuda")
+    stack = stg.stg_state_stack_create(1 << 20)
+    stg.stg_tgcn_train_sequence_batched(g, S, pg, pg["w_o"], pg["b_o"], Xs, Ys, H0, Hseq, grads, dw, db, loss, stack)
+    torch.cuda.synchronize()
+    return loss.item(), grads, dw, db, Hseq
+
+
+@pytest.mark.parametrize("name,S", [("C1", 16), ("C2", 8), ("C3", 5), ("C6", 3), ("C2", 1)])
+def test_train_sequence_batched_static(stg, name, S):
+    """NEXT-1 (sequence-batched schedule) against the fp64 oracle's Algorithm 1 and
+    against the per-timestamp GPU driver: same losses, states and gradients."""
+    cfg = gen.CONFIGS[name]
+    s, d = gen.static_edges(cfg)
+    g = stg.stg_static_graph_create(cfg.V, s, d, stg.STG_SELF_LOOPS)
+    ref = oracle.static_graph(cfg.V, s, d, self_loops=True)
+    p, pg = _params(cfg.F, cfg.H, 3)
+    Xs = [gen.features(cfg, 40 + i) for i in range(S)]
+    Ys = [gen.labels(cfg, 40 + i) for i in range(S)]
+    H0 = gen.uniform_pm1(9, 9, cfg.V * cfg.H).reshape(cfg.V, cfg.H)
+    Xg, Yg = [to_gpu(x) for x in Xs], [to_gpu(y) for y in Ys]
+    loss, grads, dw, db, Hseq = _run_batched(stg, g, cfg, pg, Xg, Yg, to_gpu(H0), S)
+    rl, rg, rH = oracle.train_sequence([ref] * S, [ref] * S, p, Xs, Ys, H0)
+    assert abs(loss - rl) <= 1e-5 * abs(rl), (loss, rl)
+    assert np.max(np.abs(Hseq[-1].cpu().numpy() - rH)) <= H_TOL
+    for k in ("W", "b", "L", "l"):
+        assert _normwise(grads[k].cpu().numpy(), rg[k]) <= g_tol(cfg.V * S), k
+    assert _normwise(dw.cpu().numpy(), rg["w_o"]) <= g_tol(cfg.V * S)
+    assert _normwise(db.cpu().numpy(), rg["b_o"]) <= g_tol(cfg.V * S)
+    # the per-timestamp driver on the same inputs: identical H_t (same per-row arithmetic)
+    l2, g2, dw2, db2, H2 = _run_sequence(stg, g, cfg, pg, Xg, Yg, to_gpu(H0), S, 0)
+    assert np.max(np.abs(Hseq.cpu().numpy() - H2.cpu().numpy())) <= 1e-6
+    assert abs(loss - l2) <= 1e-6 * abs(l2)
+
+
+def test_train_sequence_batched_rejects(stg):
+    cfg = gen.CONFIGS["C2"]
+    s, d = gen.static_edges(cfg)
+    g = stg.stg_static_graph_create(cfg.V, s, d, stg.STG_SELF_LOOPS)
+    p, pg = _params(cfg.F, cfg.H, 3)
+    X = [to_gpu(gen.features(cfg, 0))] * 65
+    Y = [to_gpu(gen.labels(cfg, 0))] * 65
+    with pytest.raises(stg.StgError) as e:
+        _run_batched(stg, g, cfg, pg, X, Y, torch.zeros(cfg.V, cfg.H, device="cuda"), 65)
+    assert e.value.status == 1
