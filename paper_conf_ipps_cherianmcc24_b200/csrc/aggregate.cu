@@ -805,7 +805,8 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
                     ((uintptr_t)in % 16 == 0) && ((uintptr_t)out % 16 == 0);
   // column split: launches of <= 512 columns (strategies 0/1) or <= 128 (strategy 2)
   const int32_t cmax = vec4 ? 512 : 128;
-  const int64_t chunks_bound = a.sched ? (gv->num_edges / kHubChunk) + 2 : 0;
+  // hub chunks: <= E/64 full chunks plus one partial chunk per hub row (<= sched_cap(E) hub rows)
+  const int64_t chunks_bound = a.sched ? (gv->num_edges / kHubChunk) + sched_cap(gv->num_edges) + 2 : 0;
   AggWs* ws = static_cast<AggWs*>(gv->workspace);
   if (a.sched) {
     STG_TRY(ws->partials.alloc((size_t)chunks_bound * std::min(W, cmax) + 4, s));
