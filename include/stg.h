@@ -312,6 +312,89 @@ stg_status stg_tgcn_train_sequence_batched(const stg_graph* graph, int32_t S, co
 stg_status stg_partition_rows(int32_t V, const int32_t* in_rowptr, int32_t world, int32_t* bounds,
                               stg_stream_t stream);
 
+/* ---- sharded mode over peer memory (SURVEY §8(e) "sharded mode"; north_star
+ * "partitioned ... by destination-vertex row blocks, with ... all-gather over
+ * NVLink of the source feature/hidden rows each timestep") ----
+ * Every rank owns the rows of its block of a [V,W] row matrix (P' = diag(n_src)XW,
+ * or any feature/hidden rows).  Instead of copying the whole matrix to every rank
+ * and then aggregating, the aggregation kernel loads each neighbour row directly
+ * from its OWNER's buffer (NVLink peer loads of CUDA-IPC-mapped memory), so the
+ * exchange is fused into the gather, tile by tile, with no staging copy.
+ * Ordering across ranks is the caller's: the owners' writes must be complete
+ * (e.g. a stream-ordered NCCL all-reduce of one element, or a host barrier after a
+ * synchronize) before a rank gathers, and a buffer is rewritten only after every
+ * reader finished (double-buffer per timestep).
+ *
+ * A row table: block k (0 <= k < world <= STG_MAX_PEERS) holds the rows
+ * [bounds[k], bounds[k+1]) of the matrix, block-local row 0 = vertex bounds[k],
+ * leading dimension ld (floats, % 4 == 0), base 16-byte aligned.  bounds (host)
+ * [world+1], non-decreasing, bounds[0] = 0, bounds[world] = V; blocks (host)
+ * [world] DEVICE pointers valid on the calling device (local, or opened with
+ * stg_peer_open).  A NULL block is allowed only when the block is empty. */
+#define STG_MAX_PEERS 8
+typedef struct {
+  int32_t world;
+  const int32_t* bounds;
+  const float* const* blocks;
+  int64_t ld;
+} stg_peer_rows;
+
+/* CUDA IPC handle of a peer-visible allocation (opaque, 64 bytes). */
+typedef struct { unsigned char reserved[64]; } stg_ipc_handle;
+/* Allocates `bytes` of device memory that other processes may map
+ * (cudaMalloc'd, not pooled) and returns its IPC handle.  Free with stg_peer_free. */
+stg_status stg_peer_alloc(int64_t bytes, void** dptr, stg_ipc_handle* handle);
+stg_status stg_peer_free(void* dptr);
+/* Maps another process's allocation (same or peer device, peer access enabled
+ * lazily over NVLink).  STG_ERR_CUDA if the handle was created in this process. */
+stg_status stg_peer_open(const stg_ipc_handle* handle, void** dptr);
+stg_status stg_peer_close(void* dptr);
+
+/* All-gather of row blocks over peer loads: full[u,:] = row u of its owner's block,
+ * for all u in [0,V), W columns; full has leading dimension ldf >= W.  (The
+ * explicit form of the exchange, for consumers other than the fused gather.) */
+stg_status stg_allgather_rows(const stg_peer_rows* src, int32_t W, float* full, int64_t ldf,
+                              stg_stream_t stream);
+
+/* Fused forward aggregation over peer memory: as stg_gcn_aggregate_ex with
+ * backward = 0, but each source row in[c,:] is read from its owner's block of `x`
+ * (x->bounds must cover the view's num_nodes).  Width 4 <= W <= 512, W % 4 == 0,
+ * and the view must carry the library schedule (views of library objects do). */
+stg_status stg_gcn_aggregate_peer(const stg_csr_view* g, int32_t W, const stg_peer_rows* x,
+                                  float* out, int64_t ldout, const float* scale_row,
+                                  const float* scale_col, const float* bias, stg_stream_t stream);
+
+/* Reduce-scatter over peer loads: for the rows u of `rank`'s block
+ * [bounds[rank], bounds[rank+1]), out[u - bounds[rank], :] = Σ_{q=0..world-1}
+ * partials[q][u, :] summed in rank order q = 0, 1, ... (deterministic).
+ * partials (host)[world] device pointers to every rank's FULL [V, ld] buffer. */
+stg_status stg_reduce_scatter_rows(int32_t world, const int32_t* bounds, const float* const* partials,
+                                   int64_t ld, int32_t rank, int32_t W, float* out, int64_t ldout,
+                                   stg_stream_t stream);
+
+/* The TGCN step in sharded mode (X row-sharded, nothing replicated):
+ *   stg_tgcn_project      P'_loc = diag(n_src[rows]) · X_loc · W for the R local rows
+ *                         (X_loc [R,F], P_loc [R,3H]);
+ *   stg_tgcn_step_peer    C = diag(n_dst)·A·P' + b with P' gathered from the owners
+ *                         (stg_gcn_aggregate_peer), GRU, H_next; pushes {H_prev, C};
+ *   stg_tgcn_step_backward_peer  pops, GRU backward, dL/dl/db, and the partial
+ *                         dP_part = diag(n_src)·Aᵀ_loc·dC' [V,3H] of the local edges
+ *                         for all V sources (no dW);
+ *   stg_reduce_scatter_rows  dP_loc = Σ_ranks dP_part over the owner's rows;
+ *   stg_tgcn_dw           dW += X_locᵀ · dP_loc.
+ * The per-rank gradients add up to the whole-graph gradient (all-reduce per
+ * sequence, as in resident mode). */
+stg_status stg_tgcn_project(const stg_csr_view* g, const stg_tgcn_params* p, const float* X_loc,
+                            float* P_loc, stg_stream_t stream);
+stg_status stg_tgcn_step_peer(const stg_csr_view* g_fwd, const stg_tgcn_params* p, const stg_peer_rows* P,
+                              const float* H_prev, float* H_next, stg_state_stack* stack,
+                              stg_stream_t stream);
+stg_status stg_tgcn_step_backward_peer(const stg_csr_view* g_bwd, const stg_tgcn_params* p,
+                                       const float* dH_next, float* dH_prev, stg_tgcn_grads* grads,
+                                       float* dP_part, stg_state_stack* stack, stg_stream_t stream);
+stg_status stg_tgcn_dw(const stg_tgcn_params* p, int32_t R, const float* X_loc, const float* dP_loc,
+                       stg_tgcn_grads* grads, stg_state_stack* stack, stg_stream_t stream);
+
 /* Per-phase device timing with CUDA events recorded on the launching stream
  * around each phase (bench.py; the GNN vs graph-update split of Fig. 9,
  * P:L316/L345).  phase: 0 aggregation fwd, 1 aggregation bwd, 2 snapshot

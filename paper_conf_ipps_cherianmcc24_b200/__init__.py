@@ -56,6 +56,17 @@ class stg_csr_view(ctypes.Structure):
                 ("workspace", _P)]
 
 
+STG_MAX_PEERS = 8
+
+
+class stg_peer_rows(ctypes.Structure):
+    _fields_ = [("world", _i32), ("bounds", ctypes.POINTER(_i32)), ("blocks", ctypes.POINTER(_P)), ("ld", _i64)]
+
+
+class stg_ipc_handle(ctypes.Structure):
+    _fields_ = [("reserved", ctypes.c_ubyte * 64)]
+
+
 class stg_tgcn_params(ctypes.Structure):
     _fields_ = [("F", _i32), ("H", _i32), ("W", _P), ("b", _P), ("L", _P), ("l", _P)]
 
@@ -113,6 +124,20 @@ _decl("stg_debug_tc_gemm", [_i32, _i32, _i32, _i32, _i32, _P, _P, _P, _P])
 _decl("stg_aggregate_set_strategy", [_i32])
 _decl("stg_aggregate_set_param", [_i32, _i64])
 _decl("stg_profile_read", [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64), _i32])
+_decl("stg_peer_alloc", [_i64, ctypes.POINTER(_P), ctypes.POINTER(stg_ipc_handle)])
+_decl("stg_peer_free", [_P])
+_decl("stg_peer_open", [ctypes.POINTER(stg_ipc_handle), ctypes.POINTER(_P)])
+_decl("stg_peer_close", [_P])
+_decl("stg_allgather_rows", [ctypes.POINTER(stg_peer_rows), _i32, _P, _i64, _P])
+_decl("stg_gcn_aggregate_peer", [ctypes.POINTER(stg_csr_view), _i32, ctypes.POINTER(stg_peer_rows), _P, _i64, _P, _P,
+                                 _P, _P])
+_decl("stg_reduce_scatter_rows", [_i32, ctypes.POINTER(_i32), ctypes.POINTER(_P), _i64, _i32, _i32, _P, _i64, _P])
+_decl("stg_tgcn_project", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn_params), _P, _P, _P])
+_decl("stg_tgcn_step_peer", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn_params),
+                             ctypes.POINTER(stg_peer_rows), _P, _P, _P, _P])
+_decl("stg_tgcn_step_backward_peer", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn_params), _P, _P,
+                                      ctypes.POINTER(stg_tgcn_grads), _P, _P, _P])
+_decl("stg_tgcn_dw", [ctypes.POINTER(stg_tgcn_params), _i32, _P, _P, ctypes.POINTER(stg_tgcn_grads), _P, _P])
 
 ABI_SYMBOLS = [
     "stg_last_error", "stg_version", "stg_kernel_launch_count", "stg_set_allocator", "stg_memcpy",
@@ -126,6 +151,9 @@ ABI_SYMBOLS = [
     "stg_tgcn_train_sequence_batched",
     "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
+    "stg_peer_alloc", "stg_peer_free", "stg_peer_open", "stg_peer_close", "stg_allgather_rows",
+    "stg_gcn_aggregate_peer", "stg_reduce_scatter_rows", "stg_tgcn_project", "stg_tgcn_step_peer",
+    "stg_tgcn_step_backward_peer", "stg_tgcn_dw",
 ]
 
 PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head", "dl"]
@@ -482,3 +510,118 @@ AGG_ROWS_IN_FLIGHT, AGG_MIN_BLOCKS, AGG_STREAM_WMIN = 0, 1, 2
 def stg_aggregate_set_param(key: int, value: int):
     """Edge-stream tunables (include/stg.h): 0 rows in flight, 1 min blocks/SM, 2 min width."""
     _check(_lib.stg_aggregate_set_param(int(key), int(value)))
+
+
+# ---------------------------------------------------------------- sharded mode (peer memory)
+class PeerBuffer:
+    """A CUDA-IPC-visible fp32 [rows, cols] buffer owned by libstg (stg_peer_alloc),
+    exposed to torch through __cuda_array_interface__ (no copy)."""
+
+    def __init__(self, rows: int, cols: int):
+        self.rows, self.cols = int(rows), int(cols)
+        self.handle = stg_ipc_handle()
+        p = ctypes.c_void_p()
+        _check(_lib.stg_peer_alloc(max(1, self.rows * self.cols * 4), ctypes.byref(p), ctypes.byref(self.handle)))
+        self.ptr = p.value
+        self.__cuda_array_interface__ = {"shape": (self.rows, self.cols), "typestr": "<f4",
+                                         "data": (self.ptr, False), "version": 2, "strides": None}
+        self.tensor = torch.as_tensor(self, device="cuda")
+
+    def handle_bytes(self) -> bytes:
+        return bytes(self.handle.reserved)
+
+    def close(self):
+        if self.ptr:
+            self.tensor = None
+            _lib.stg_peer_free(ctypes.c_void_p(self.ptr))
+            self.ptr = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def stg_peer_open(handle: bytes) -> int:
+    """Map another process's PeerBuffer (its handle_bytes()); returns the device pointer."""
+    h = stg_ipc_handle()
+    ctypes.memmove(h.reserved, handle, 64)
+    p = ctypes.c_void_p()
+    _check(_lib.stg_peer_open(ctypes.byref(h), ctypes.byref(p)))
+    return p.value
+
+
+def stg_peer_close(ptr: int):
+    _check(_lib.stg_peer_close(ctypes.c_void_p(ptr)))
+
+
+class PeerRows:
+    """stg_peer_rows: block k = rows [bounds[k], bounds[k+1]) at device pointer ptrs[k] (ld floats)."""
+
+    def __init__(self, bounds, ptrs, ld: int):
+        world = len(bounds) - 1
+        if len(ptrs) != world or not 1 <= world <= STG_MAX_PEERS:
+            raise StgError(1, "PeerRows: need 1 <= world <= %d blocks" % STG_MAX_PEERS)
+        self._b = (_i32 * (world + 1))(*[int(x) for x in bounds])
+        self._p = (_P * world)(*[int(p) if p else None for p in ptrs])
+        self.c = stg_peer_rows(world, self._b, self._p, int(ld))
+
+
+def _row_ptr(t):
+    return t.data_ptr() if isinstance(t, torch.Tensor) else int(t)
+
+
+def stg_allgather_rows(rows: PeerRows, W: int, full: torch.Tensor, stream=None) -> torch.Tensor:
+    _check(_lib.stg_allgather_rows(ctypes.byref(rows.c), int(W), _ptr(full), full.stride(0), _stream(stream)))
+    return full
+
+
+def stg_gcn_aggregate_peer(v: stg_csr_view, rows: PeerRows, W: int, out: torch.Tensor = None, scale_row=None,
+                           scale_col=None, bias=None, stream=None) -> torch.Tensor:
+    if out is None:
+        out = torch.empty((v.row_end - v.row_begin, W), dtype=torch.float32, device="cuda")
+    _check(_lib.stg_gcn_aggregate_peer(ctypes.byref(v), int(W), ctypes.byref(rows.c), _ptr(out), out.stride(0),
+                                       _ptr(scale_row), _ptr(scale_col), _ptr(bias), _stream(stream)))
+    return out
+
+
+def stg_reduce_scatter_rows(bounds, partials, ld: int, rank: int, W: int, out: torch.Tensor, stream=None):
+    world = len(bounds) - 1
+    b = (_i32 * (world + 1))(*[int(x) for x in bounds])
+    pp = (_P * world)(*[_row_ptr(p) for p in partials])
+    _check(_lib.stg_reduce_scatter_rows(world, b, pp, int(ld), int(rank), int(W), _ptr(out), out.stride(0),
+                                        _stream(stream)))
+    return out
+
+
+def stg_tgcn_project(v: stg_csr_view, params: dict, X_loc, P_loc, stream=None):
+    P = make_params(params)
+    _check(_lib.stg_tgcn_project(ctypes.byref(v), ctypes.byref(P), _ptr(X_loc), ctypes.c_void_p(_row_ptr(P_loc)),
+                                 _stream(stream)))
+
+
+def stg_tgcn_step_peer(v: stg_csr_view, params: dict, rows: PeerRows, H_prev, H_next, stack: StateStack = None,
+                       stream=None):
+    P = make_params(params)
+    _check(_lib.stg_tgcn_step_peer(ctypes.byref(v), ctypes.byref(P), ctypes.byref(rows.c), _ptr(H_prev),
+                                   _ptr(H_next), stack.handle if stack else None, _stream(stream)))
+    return H_next
+
+
+def stg_tgcn_step_backward_peer(v: stg_csr_view, params: dict, dH_next, dH_prev, grads: dict, dP_part,
+                                stack: StateStack, stream=None):
+    P = make_params(params)
+    G = make_grads(grads)
+    _check(_lib.stg_tgcn_step_backward_peer(ctypes.byref(v), ctypes.byref(P), _ptr(dH_next), _ptr(dH_prev),
+                                            ctypes.byref(G), ctypes.c_void_p(_row_ptr(dP_part)), stack.handle,
+                                            _stream(stream)))
+    return dH_prev
+
+
+def stg_tgcn_dw(params: dict, X_loc, dP_loc, grads: dict, stack: StateStack, stream=None):
+    P = make_params(params)
+    G = make_grads(grads)
+    R = X_loc.shape[0]
+    _check(_lib.stg_tgcn_dw(ctypes.byref(P), int(R), _ptr(X_loc), ctypes.c_void_p(_row_ptr(dP_loc)),
+                            ctypes.byref(G), stack.handle, _stream(stream)))

@@ -276,6 +276,11 @@ struct Agg2Args {
   // [k·wsplit, min((k+1)·wsplit, wtotal)) and its hub partials start at k·pstride
   int32_t wsplit, wtotal;
   int64_t pstride;
+  // sharded mode (stg_gcn_aggregate_peer): source row u lives in block k with
+  // pbnd[k] <= u < pbnd[k+1] (pbnd[k] = INT_MAX past the last block), at
+  // pbase[k] + u·ldx (the block base shifted back by pbnd[k] rows)
+  const float* pbase[STG_MAX_PEERS];
+  int32_t pbnd[STG_MAX_PEERS];
 };
 
 // Strategy 1: software-pipelined degree-ordered items.  A warp serves 32/G
@@ -506,13 +511,22 @@ __global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_
   }
 }
 
-template <int D, int MINB, bool SCOL>
+template <int D, int MINB, bool SCOL, bool PEER>
 __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args a, uint32_t* __restrict__ queue) {
   constexpr int NW = kAggThreads / 32;
   __shared__ __align__(16) int4 s_items[NW][2][32];
   __shared__ int32_t s_excl[NW][32], s_v[NW][32], s_beg[NW][32], s_hub[NW][32];
+  __shared__ const float* s_pbase[STG_MAX_PEERS];
+  __shared__ int32_t s_pbnd[STG_MAX_PEERS];
   const unsigned FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  if (PEER) {
+    if (threadIdx.x < STG_MAX_PEERS) {
+      s_pbase[threadIdx.x] = a.pbase[threadIdx.x];
+      s_pbnd[threadIdx.x] = a.pbnd[threadIdx.x];
+    }
+    __syncthreads();
+  }
   const int64_t total = a.sched[3];
   const int4* items = reinterpret_cast<const int4*>(a.sched + kSchedHdr);
   // Work groups: hub chunks (<= 64 edges each) a.hgrp per group, light rows
@@ -532,8 +546,18 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
   queue += blockIdx.y;
   const int nv = Wl >> 2;
   const bool lane_on = lane < nv;
-  const float4* xl = reinterpret_cast<const float4*>(a.x + c0y) + (lane_on ? lane : nv - 1);
+  const int lanec = lane_on ? lane : nv - 1;
+  const float4* xl = reinterpret_cast<const float4*>(a.x + c0y) + lanec;
   const uint32_t ld4 = (uint32_t)(a.ldx >> 2);
+  // sharded mode: the float4 offset of source row u's column chunk in its owner's
+  // block (resolved once per edge by the lane that loads the column id)
+  auto peer_row = [&](int32_t u) -> unsigned long long {
+    int k = 0;
+#pragma unroll
+    for (int i = 1; i < STG_MAX_PEERS; ++i) k += (u >= s_pbnd[i]) ? 1 : 0;
+    return reinterpret_cast<unsigned long long>(reinterpret_cast<const float4*>(s_pbase[k] + c0y) +
+                                                (size_t)(uint32_t)u * ld4);
+  };
   int32_t* ex = s_excl[w];
   auto fetch = [&](uint32_t g, int buf) {         // cp.async the 32 descriptors of group g
     const int64_t it = gbase(g) + lane;
@@ -613,13 +637,19 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
       float sc = 1.0f;
       if (SCOL && lane < nb) sc = __ldg(a.scol + u0);
       const int32_t uc = u0;
+      const unsigned long long ua = PEER ? peer_row(u0) : 0ull;
       if (b0 + 32 < N) resolve(b0 + 32 + lane, u0, k0);  // next batch in flight
       for (int32_t j0 = 0; j0 < nb; j0 += D) {
         float4 v[D];
 #pragma unroll
         for (int d = 0; d < D; ++d) {
-          const uint32_t u = (uint32_t)__shfl_sync(FULL, uc, (j0 + d) & 31);
-          v[d] = __ldg(xl + (size_t)u * ld4);
+          if (PEER) {          // NVLink peer (or local) load from the owner's block
+            const unsigned long long r = __shfl_sync(FULL, ua, (j0 + d) & 31);
+            v[d] = __ldg(reinterpret_cast<const float4*>(r) + lanec);
+          } else {
+            const uint32_t u = (uint32_t)__shfl_sync(FULL, uc, (j0 + d) & 31);
+            v[d] = __ldg(xl + (size_t)u * ld4);
+          }
         }
         const uint32_t mseg = (bm >> (j0 & 31)) & (D >= 32 ? 0xffffffffu : ((1u << D) - 1u));
         if (mseg == 0) {                                // warp-uniform: no item starts in this group
@@ -680,10 +710,13 @@ ItemsFn pick_items(int g, int vpl) {
 using StreamFn = void (*)(const Agg2Args, uint32_t*);
 StreamFn pick_stream(int d, int minb, bool scol) {
 #define STG_STREAM(DD, MB) \
-  if (d == DD && minb == MB) return scol ? k_agg_stream<DD, MB, true> : k_agg_stream<DD, MB, false>;
+  if (d == DD && minb == MB) return scol ? k_agg_stream<DD, MB, true, false> : k_agg_stream<DD, MB, false, false>;
   STG_STREAM(4, 6) STG_STREAM(8, 4) STG_STREAM(16, 2) STG_STREAM(16, 3)
 #undef STG_STREAM
-  return scol ? k_agg_stream<16, 3, true> : k_agg_stream<16, 3, false>;
+  return scol ? k_agg_stream<16, 3, true, false> : k_agg_stream<16, 3, false, false>;
+}
+StreamFn pick_stream_peer(bool scol) {
+  return scol ? k_agg_stream<16, 3, true, true> : k_agg_stream<16, 3, false, true>;
 }
 
 using KernelFn = void (*)(const AggArgs);
@@ -764,15 +797,42 @@ static void lane_groups(int nv, int vpl_max, int* g, int* vpl) {
   *vpl = (nv + gg - 1) / gg;
 }
 
+// Sharded mode (stg_gcn_aggregate_peer): the source rows come from the owners'
+// blocks of `peers` (in / ldin are ignored); only the edge-stream kernel serves it.
 stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
                             float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
-                            cudaStream_t s) {
+                            cudaStream_t s, const stg_peer_rows* peers) {
   if (!gv) return fail(STG_ERR_INVALID_ARG, "aggregate: view is NULL");
   if (W < 1) return fail(STG_ERR_INVALID_ARG, "aggregate: W=%d < 1", W);
+  int32_t peer_pad = 0;
+  if (peers) {
+    if (backward) return fail(STG_ERR_INVALID_ARG, "aggregate_peer: forward direction only");
+    if (peers->world < 1 || peers->world > STG_MAX_PEERS || !peers->bounds || !peers->blocks)
+      return fail(STG_ERR_INVALID_ARG, "aggregate_peer: world must be in [1,%d] with bounds and blocks", STG_MAX_PEERS);
+    if (W % 4 || W > 512 || peers->ld < W || peers->ld % 4)
+      return fail(STG_ERR_INVALID_ARG, "aggregate_peer: need W %% 4 == 0, W <= 512, ld >= W, ld %% 4 == 0");
+    const int32_t* bd = peers->bounds;
+    if (bd[0] != 0 || bd[peers->world] != gv->num_nodes)
+      return fail(STG_ERR_INVALID_ARG, "aggregate_peer: bounds must span [0, V=%d)", gv->num_nodes);
+    peer_pad = -1;
+    for (int k = 0; k < peers->world; ++k) {
+      if (bd[k + 1] < bd[k]) return fail(STG_ERR_INVALID_ARG, "aggregate_peer: bounds decrease at %d", k);
+      if (bd[k + 1] > bd[k]) {
+        if (!peers->blocks[k] || (uintptr_t)peers->blocks[k] % 16)
+          return fail(STG_ERR_INVALID_ARG, "aggregate_peer: block %d is NULL or not 16-byte aligned", k);
+        if (peer_pad < 0) peer_pad = bd[k];
+      }
+    }
+    if (peer_pad < 0) peer_pad = 0;
+    if (!gv->in_sched || !gv->in_ids || !gv->workspace)
+      return fail(STG_ERR_INVALID_ARG, "aggregate_peer: the view lacks the library schedule");
+    in = peers->blocks[0] ? peers->blocks[0] : reinterpret_cast<const float*>(16);   // alignment checks only
+    ldin = peers->ld;
+  }
   if (ldin < W || ldout < W) return fail(STG_ERR_INVALID_ARG, "aggregate: leading dimension < W");
-  if (!in || !out) return fail(STG_ERR_INVALID_ARG, "aggregate: NULL input/output");
   const int32_t R = backward ? gv->num_nodes : gv->row_end - gv->row_begin;
-  if (R <= 0) return STG_OK;
+  if (R <= 0) return STG_OK;                     // an empty row block: nothing to write
+  if (!in || !out) return fail(STG_ERR_INVALID_ARG, "aggregate: NULL input/output");
   AggArgs a{};
   a.R = R;
   a.rowptr = backward ? gv->out_rowptr : gv->in_rowptr;
@@ -825,12 +885,14 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   // strategy 2: edge stream, in near-equal column chunks of <= 128 columns
   const int nsplit = (int)ceil_div(W, 128);
   const int32_t wsplit = (int32_t)(ceil_div(ceil_div(W, 4), nsplit) * 4);
-  if (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128) {
+  if (peers && !(vec4 && a.sched && wsplit <= 128))
+    return fail(STG_ERR_INVALID_ARG, "aggregate_peer: output must be 16-byte aligned with ldout %% 4 == 0");
+  if (peers || (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128)) {
     STG_TRY(ws->queue.alloc(nsplit, s));
     STG_CUDA(cudaMemsetAsync(ws->queue.p, 0, sizeof(uint32_t) * nsplit, s));
     const int64_t pstride = chunks_bound * wsplit;               // the column chunks run concurrently
     STG_TRY(ws->partials.alloc((size_t)(pstride * nsplit) + 4, s));
-    const StreamFn fn = pick_stream(g_tune.d, g_tune.minb, scol != nullptr);
+    const StreamFn fn = peers ? pick_stream_peer(scol != nullptr) : pick_stream(g_tune.d, g_tune.minb, scol != nullptr);
     // group sizes: ~max(256, E / (8 warps x #SM)) edges per group (all 32-item light
     // groups at C5 scale; small graphs get small groups, hence many warps)
     const int64_t target = std::max<int64_t>(256, gv->num_edges / (8 * (int64_t)num_sms()));
@@ -849,6 +911,21 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     b.upad = (backward && a.ids) ? (int32_t)rb : 0;     // row 0 of a shifted input is not a valid row
     b.hgrp = hgrp; b.lgrp = lgrp;
     b.wsplit = wsplit; b.wtotal = W; b.pstride = pstride;
+    for (int k = 0; k < STG_MAX_PEERS; ++k) {
+      b.pbnd[k] = INT32_MAX;
+      b.pbase[k] = nullptr;
+    }
+    if (peers) {
+      b.upad = peer_pad;
+      for (int k = 0; k < peers->world; ++k) {
+        b.pbnd[k] = k == 0 ? 0 : peers->bounds[k];
+        // block k base shifted back by bounds[k] rows: row u is at pbase[k] + u·ld
+        b.pbase[k] = reinterpret_cast<const float*>(reinterpret_cast<uintptr_t>(peers->blocks[k]) -
+                                                    (uintptr_t)((int64_t)peers->bounds[k] * peers->ld * 4));
+      }
+      // empty blocks: never selected (rows of an empty block k belong to the next
+      // non-empty block, pbnd is non-decreasing so the count skips them)
+    }
     // one launch for all column chunks (gridDim.y): the chunks of a wide W (e.g. a
     // sequence-batched S·3H) walk the graph side by side instead of one after another
     const int64_t bx = nsplit > 1 ? std::max<int64_t>(1, std::min<int64_t>(blocks, ceil_div(occupancy_grid(
@@ -914,6 +991,13 @@ stg_status stg_gcn_aggregate_bwd(const stg_csr_view* g, int32_t W, const float* 
   if (!g) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_bwd: view is NULL");
   return stg::aggregate_launch(g, 1, W, gy, ldgy, gx, ldgx, g->norm_src,
                                g->norm_dst ? g->norm_dst + g->row_begin : nullptr, nullptr, (cudaStream_t)stream);
+}
+
+stg_status stg_gcn_aggregate_peer(const stg_csr_view* g, int32_t W, const stg_peer_rows* x, float* out,
+                                  int64_t ldout, const float* scale_row, const float* scale_col, const float* bias,
+                                  stg_stream_t stream) {
+  if (!x) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_peer: row table is NULL");
+  return stg::aggregate_launch(g, 0, W, nullptr, 0, out, ldout, scale_row, scale_col, bias, (cudaStream_t)stream, x);
 }
 
 stg_status stg_aggregate_set_strategy(int32_t strategy) {

@@ -37,9 +37,6 @@ stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* pa
                  cudaStream_t s);
 stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
                  float* tot, float* dL, float* dl, float* db, const float* L, cudaStream_t s);
-stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
-                            float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
-                            cudaStream_t s);
 }
 
 namespace stg {
@@ -531,22 +528,26 @@ static size_t stack_bytes(int32_t V, int32_t H) {
 // Sharded views (resident mode): P' for all Vall source rows
 // (X is resident on every rank), C / GRU / H for the V = R local rows.
 
+// P'[i] = n[i]·X[i]·W over n_rows rows (n = NULL: unscaled)
+static stg_status project_rows(int32_t n_rows, const stg_tgcn_params* p, const float* X, const float* n, float* P,
+                               cudaStream_t s) {
+  const int32_t F = p->F, H = p->H, H3 = 3 * H;
+  ProfScope prof(PH_XW, s);
+  if (n_rows == 0) return STG_OK;
+  if (tc_supported(F, H)) return tc_xw(n_rows, F, H, X, p->W, n, P, s);
+  const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
+  STG_TRY(set_smem(k_xw, smem));
+  const int nb = grid_blocks((const void*)k_xw, smem, (n_rows + 31) / 32);
+  k_xw<<<nb, kT, smem, s>>>(n_rows, F, H3, X, p->W, n, P);
+  count_launch();
+  return check_launch("tgcn project");
+}
+
 // P' = diag(n_src)·X·W (all Vall rows) and C = diag(n_dst)·A·P' + b (local rows)
 static stg_status fwd_conv(const stg_csr_view* g, const stg_tgcn_params* p, const float* X, float* P, float* C,
                            cudaStream_t s) {
-  const int32_t Vall = g->num_nodes, F = p->F, H = p->H, H3 = 3 * H;
-  {
-    ProfScope prof(PH_XW, s);
-    if (tc_supported(F, H)) {
-      STG_TRY(tc_xw(Vall, F, H, X, p->W, g->norm_src, P, s));
-    } else {
-      const size_t smem = sizeof(float) * (size_t)(F * H3 + 32 * F);
-      STG_TRY(set_smem(k_xw, smem));
-      const int nb = grid_blocks((const void*)k_xw, smem, (Vall + 31) / 32);
-      k_xw<<<nb, kT, smem, s>>>(Vall, F, H3, X, p->W, g->norm_src, P);
-      count_launch();
-    }
-  }
+  const int32_t Vall = g->num_nodes, H3 = 3 * p->H;
+  STG_TRY(project_rows(Vall, p, X, g->norm_src, P, s));
   const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
   return aggregate_launch(g, 0, H3, P, H3, C, H3, ndst_loc, nullptr, p->b, s);
 }
@@ -743,6 +744,94 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
   stack->entries.pop_back();
   stack->top -= e.bytes;
   return STG_OK;
+}
+
+// ---- sharded mode over peer memory (include/stg.h): P' of the local rows only,
+// the aggregation gathers P' rows from their owners, the backward leaves
+// partial dP rows for every source that stg_reduce_scatter_rows sums per owner.
+stg_status stg_tgcn_project(const stg_csr_view* g, const stg_tgcn_params* p, const float* X_loc, float* P_loc,
+                            stg_stream_t stream) {
+  STG_TRY(check_params(p));
+  if (!g || !X_loc || !P_loc) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_project: NULL argument");
+  const int32_t R = g->row_end - g->row_begin;
+  return project_rows(R, p, X_loc, g->norm_src ? g->norm_src + g->row_begin : nullptr, P_loc, (cudaStream_t)stream);
+}
+
+stg_status stg_tgcn_step_peer(const stg_csr_view* g, const stg_tgcn_params* p, const stg_peer_rows* P,
+                              const float* H_prev, float* H_next, stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_params(p));
+  if (!g || !P || !H_prev || !H_next) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_peer: NULL argument");
+  cudaStream_t s = (cudaStream_t)stream;
+  const int32_t V = g->row_end - g->row_begin, H = p->H, H3 = 3 * H;
+  TgcnWs& ws = stack ? stack->ws : global_ws();
+  float* C = nullptr;
+  const size_t need = stack_bytes(V, H);
+  if (stack) {
+    if (stack->top + need > stack->cap)
+      return fail(STG_ERR_NO_MEMORY, "stg_tgcn_step_peer: state stack full (%zu + %zu > %zu bytes)", stack->top,
+                  need, stack->cap);
+    C = reinterpret_cast<float*>(stack->arena.p + stack->top);
+  } else {
+    STG_TRY(ws.dC.alloc((size_t)V * H3 + 4));
+    C = ws.dC.p;
+  }
+  const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
+  STG_TRY(aggregate_launch(g, 0, H3, nullptr, 0, C, H3, ndst_loc, nullptr, p->b, s, P));
+  STG_TRY(fwd_gru(V, p, C, H_prev, H_next, s));
+  if (stack) {
+    stack->entries.push_back(StackEntry{H_prev, C, V, H, need});
+    stack->top += need;
+  }
+  return STG_OK;
+}
+
+stg_status stg_tgcn_step_backward_peer(const stg_csr_view* g, const stg_tgcn_params* p, const float* dH_next,
+                                       float* dH_prev, stg_tgcn_grads* grads, float* dP_part, stg_state_stack* stack,
+                                       stg_stream_t stream) {
+  STG_TRY(check_params(p));
+  if (!g || !dH_next || !dH_prev || !grads || !stack || !dP_part)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward_peer: NULL argument");
+  if (!grads->W || !grads->b || !grads->L || !grads->l)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_step_backward_peer: NULL gradient pointer");
+  if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn_step_backward_peer: state stack is empty");
+  const StackEntry e = stack->entries.back();
+  const int32_t V = g->row_end - g->row_begin, H = p->H, H3 = 3 * H;
+  if (e.V != V || e.H != H) return fail(STG_ERR_STATE, "stg_tgcn_step_backward_peer: stack top does not match (V,H)");
+  cudaStream_t s = (cudaStream_t)stream;
+  BwdBufs bb;
+  STG_TRY(bwd_alloc(stack->ws, g, p, 1, &bb));
+  STG_TRY(bwd_gru(g, p, e.C, e.Hp, dH_next, dH_prev, grads, stack->ws, bb, s));
+  STG_TRY(bwd_dl(g, p, e.C, e.Hp, grads, stack->ws, bb, s));
+  STG_TRY(aggregate_launch(g, 1, H3, bb.dC[0], H3, dP_part, H3, g->norm_src, nullptr, nullptr, s));
+  stack->entries.pop_back();
+  stack->top -= e.bytes;
+  return STG_OK;
+}
+
+stg_status stg_tgcn_dw(const stg_tgcn_params* p, int32_t R, const float* X_loc, const float* dP_loc,
+                       stg_tgcn_grads* grads, stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_params(p));
+  if (R < 0 || (R > 0 && (!X_loc || !dP_loc)) || !grads || !grads->W || !stack)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_dw: bad arguments");
+  if (R == 0) return STG_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  const int32_t F = p->F, H = p->H, H3 = 3 * H;
+  TgcnWs& ws = stack->ws;
+  ProfScope prof(PH_DW, s);
+  if (tc_supported(F, H)) {
+    STG_TRY(ws.part_tc.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));
+    STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
+    return tc_dw(R, F, H, X_loc, dP_loc, ws.part_tc.p, ws.dl_tmp.p, grads->W, s);
+  }
+  const size_t sm2 = sizeof(float) * (size_t)(32 * F + 32 * H3 + F * H3);
+  STG_TRY(set_smem(k_dw, sm2));
+  const int nb = grid_blocks((const void*)k_dw, sm2, (R + 31) / 32);
+  STG_TRY(ws.part_dw.alloc((size_t)nb * F * H3));
+  k_dw<<<nb, kT, sm2, s>>>(R, F, H3, X_loc, dP_loc, ws.part_dw.p);
+  k_reduce_part<<<(F * H3 + 255) / 256, 256, 0, s>>>(ws.part_dw.p, nb, F * H3, grads->W, F * H3, nullptr, 0,
+                                                     nullptr);
+  count_launch(2);
+  return check_launch("stg_tgcn_dw");
 }
 
 stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o, const float* b_o,

@@ -76,3 +76,110 @@ def allgather_rows(local: torch.Tensor, bounds: list, group=None) -> torch.Tenso
 def allreduce_sum_(t: torch.Tensor, group=None) -> torch.Tensor:
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
     return t
+
+
+# ---------------------------------------------------------------- sharded mode over peer memory
+def stream_barrier(device=None):
+    """Cross-rank ordering point for the peer buffers (include/stg.h): with NCCL a
+    one-element all-reduce on the current stream (stream-ordered, no host sync);
+    with gloo (CPU tests, ranks sharing one GPU) a device synchronize + barrier."""
+    if dist.get_backend() == "nccl":
+        t = torch.zeros(1, device=device or torch.device("cuda", torch.cuda.current_device()))
+        dist.all_reduce(t)
+    else:
+        torch.cuda.synchronize()
+        dist.barrier()
+
+
+class PeerGroup:
+    """One IPC-shared fp32 row matrix over the ranks of the default process group:
+    this rank's PeerBuffer ([rows, cols]; rows = its block, or V with full=True)
+    plus every peer's buffer mapped into this process (stg_peer_open)."""
+
+    def __init__(self, bounds, cols: int, full: bool = False):
+        from paper_conf_ipps_cherianmcc24_b200 import PeerBuffer, PeerRows, stg_peer_open
+        self.rank, self.world = dist.get_rank(), dist.get_world_size()
+        self.bounds = list(bounds)
+        rows = self.bounds[-1] if full else self.bounds[self.rank + 1] - self.bounds[self.rank]
+        self.buf = PeerBuffer(rows, cols)
+        handles = [None] * self.world
+        dist.all_gather_object(handles, self.buf.handle_bytes())
+        self._opened = []
+        self.ptrs = []
+        for k, h in enumerate(handles):
+            if k == self.rank:
+                self.ptrs.append(self.buf.ptr)
+            else:
+                p = stg_peer_open(h)
+                self._opened.append(p)
+                self.ptrs.append(p)
+        self.rows = PeerRows(self.bounds, self.ptrs, cols)
+
+    @property
+    def tensor(self) -> torch.Tensor:
+        return self.buf.tensor
+
+    def close(self):
+        from paper_conf_ipps_cherianmcc24_b200 import stg_peer_close
+        for p in self._opened:
+            stg_peer_close(p)
+        self._opened = []
+        self.buf.close()
+
+
+class PeerTGCN:
+    """Algorithm 1 for one rank in sharded mode: X is row-sharded,
+    P' = diag(n_src)XW is computed for the local rows only and gathered from the
+    owners inside the aggregation (stg_tgcn_step_peer); the backward's partial
+    dP of the local edges is reduce-scattered to the owners over peer loads
+    (stg_reduce_scatter_rows) before dW += X_locᵀ dP_loc.  Two buffers per
+    exchanged matrix alternate per timestep, so one stream barrier per exchange
+    orders every write after the previous readers."""
+
+    def __init__(self, stg, bounds, V: int, F: int, H: int, S: int):
+        self.stg = stg
+        self.bounds = list(bounds)
+        self.rank = dist.get_rank()
+        self.V, self.F, self.H, self.S = V, F, H, S
+        self.R = self.bounds[self.rank + 1] - self.bounds[self.rank]
+        self.P = [PeerGroup(self.bounds, 3 * H) for _ in range(2)]
+        self.dP = [PeerGroup(self.bounds, 3 * H, full=True) for _ in range(2)]
+        self.dP_loc = torch.empty(max(self.R, 1), 3 * H, device="cuda")
+        self.G = torch.empty(2, max(self.R, 1), H, device="cuda")
+        self.stack = stg.stg_state_stack_create(S * max(self.R, 1) * 3 * H * 4 + (1 << 20))
+
+    def train_sequence(self, source, t0, params, w_o, b_o, X_loc, Y_loc, H0, H_seq, grads, dw_o, db_o, loss,
+                       barrier=stream_barrier):
+        stg, S, R, H = self.stg, len(X_loc), self.R, self.H
+        dyn = isinstance(source, stg.Dtdg)
+
+        def view(t, backward):
+            if not dyn:
+                return source.view()
+            part = stg.STG_PART_OUT if backward else stg.STG_PART_IN
+            return stg.stg_dtdg_get_snapshot_parts(source, t, part, backward=backward)
+
+        for i in range(S):                                     # forward, lines 7-16
+            v = view(t0 + i, False)
+            buf = self.P[i & 1]
+            stg.stg_tgcn_project(v, params, X_loc[i], buf.buf.ptr)
+            barrier()                                          # every owner's P' rows written
+            Hp = H0 if i == 0 else H_seq[i - 1]
+            stg.stg_tgcn_step_peer(v, params, buf.rows, Hp, H_seq[i], self.stack)
+            stg.stg_mse_head(H_seq[i], Y_loc[i], w_o, b_o, loss_accum=loss, V_total=self.V)
+        G, Gn = self.G[0][:R], self.G[1][:R]
+        G.zero_()
+        for i in range(S - 1, -1, -1):                         # backward, lines 18-25
+            v = view(t0 + i, True)
+            stg.stg_mse_head(H_seq[i], Y_loc[i], w_o, b_o, dH=G, accumulate=True, dw_o=dw_o, db_o=db_o,
+                             V_total=self.V)
+            dpg = self.dP[i & 1]
+            stg.stg_tgcn_step_backward_peer(v, params, G, Gn, grads, dpg.buf.ptr, self.stack)
+            barrier()                                          # every rank's partial dP written
+            stg.stg_reduce_scatter_rows(self.bounds, dpg.ptrs, 3 * H, self.rank, 3 * H, self.dP_loc[:R])
+            stg.stg_tgcn_dw(params, X_loc[i], self.dP_loc[:R], grads, self.stack)
+            G, Gn = Gn, G
+
+    def close(self):
+        for g in self.P + self.dP:
+            g.close()
