@@ -42,8 +42,11 @@ def parse():
     ap.add_argument("--lr", type=float, default=1e-3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--mode", default="sharded", choices=["sharded", "replicas"],
-                    help="N>1: row-block shards of one graph (SURVEY §8(e)) or independent replicas")
+    ap.add_argument("--mode", default="sharded", choices=["sharded", "peer", "replicas"],
+                    help="N>1: row-block shards of one graph with X_t resident on every rank (SURVEY §8(e) "
+                         "resident mode, default), row-block shards with X_t row-sharded and P' rows gathered "
+                         "from their owners over NVLink peer memory (sharded mode; also runs at N=1), or "
+                         "independent replicas")
     ap.add_argument("--graphs", type=int, default=-1,
                     help="replay each epoch as one CUDA graph (1/0; default: on for static-temporal configs, "
                          "whose tiny per-timestamp work is launch-bound, off for DTDGs)")
@@ -228,8 +231,15 @@ def main():
         rank, world = (int(x) for x in args.shard_sim.split("/"))
     torch.cuda.set_device(local)
     pg = world > 1 and not sim                  # a real process group (torchrun)
+    peer = args.mode == "peer" and not sim
     if pg:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif peer:                                  # N=1 sharded mode: a one-rank group for the peer plumbing
+        import socket
+        with socket.socket() as sk:
+            sk.bind(("127.0.0.1", 0))
+            port = sk.getsockname()[1]
+        dist.init_process_group("gloo", init_method="tcp://127.0.0.1:%d" % port, rank=0, world_size=1)
     dev = torch.device("cuda", local)
     cfg = gen.CONFIGS[args.config]
     static = cfg.kind == "static"
@@ -247,14 +257,19 @@ def main():
     # N > 1, sharded (default): destination row blocks with ~E/N in-edges of S_0 each
     # (SURVEY §8(e)); each rank's DTDG holds the edges into its block, X_t is resident
     # on every rank, and the per-sequence gradients are summed by one NCCL all-reduce.
-    sharded = world > 1 and args.mode == "sharded"
+    sharded = (world > 1 and args.mode == "sharded") or peer
     lo, hi = 0, V
+    bounds = [0, V]
     if sharded:
         from paper_conf_ipps_cherianmcc24_b200 import parallel
         bounds = parallel.base_row_blocks(V, s_e, d_e, world, self_loops=True)
         lo, hi = bounds[rank], bounds[rank + 1]
     R = hi - lo
     batched = static and not sharded and (args.schedule in ("auto", "batched"))
+    peer_drv = None
+    if peer:
+        from paper_conf_ipps_cherianmcc24_b200 import parallel
+        peer_drv = parallel.PeerTGCN(stg, bounds, V, F, H, S)
     dist_arg = (rank, world, lo, hi) if sharded else None
     if static:
         g = stg.stg_static_graph_create(V, s_e, d_e, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS, dist=dist_arg)
@@ -272,7 +287,9 @@ def main():
 
     # inputs: 2 distinct seeded X_t matrices cycled over t (each 256 MB > L2), labels per t
     NX = 2
-    Xh = [torch.from_numpy(gen.features(cfg, i)) for i in range(NX)]
+    # (sharded mode: every rank holds only its rows of X_t)
+    Xh = [torch.from_numpy(gen.features(cfg, i)[lo:hi].copy() if peer else gen.features(cfg, i))
+          for i in range(NX)]
     Yh = [torch.from_numpy(gen.labels(cfg, t)[lo:hi].copy()) for t in range(T)]
     Xd = [x.to(dev) for x in Xh]
     Yd = [y.to(dev) for y in Yh]
@@ -306,7 +323,10 @@ def main():
         Hprev = H0
         for k, (t0, n) in enumerate(seqs):
             Hs = Hbuf[k % 2]
-            if batched:
+            if peer:
+                peer_drv.train_sequence(g, t0, p, p["w_o"], p["b_o"], [Xsrc(t) for t in range(t0, t0 + n)],
+                                        [Ysrc(t) for t in range(t0, t0 + n)], Hprev, Hs, grads, dw_o, db_o, loss)
+            elif batched:
                 stg.stg_tgcn_train_sequence_batched(g, n, p, p["w_o"], p["b_o"], [Xsrc(t) for t in range(t0, t0 + n)],
                                                     [Ysrc(t) for t in range(t0, t0 + n)], Hprev, Hs, grads, dw_o,
                                                     db_o, loss, stack)
@@ -405,7 +425,7 @@ def main():
         Xpin = [x.pin_memory() for x in Xh]
         Ypin = [y.pin_memory() for y in Yh]
         copy = torch.cuda.Stream(device=dev)
-        stage = [[torch.empty(V, F, device=dev) for _ in range(S)] for _ in range(2)]
+        stage = [[torch.empty(R if peer else V, F, device=dev) for _ in range(S)] for _ in range(2)]
         ystage = [[torch.empty(R, device=dev) for _ in range(S)] for _ in range(2)]
         loss_h = torch.empty(1, pin_memory=True)
         h2d = 0
@@ -434,7 +454,10 @@ def main():
                 if k + 1 < len(seqs):
                     nxt = issue(k + 1) if True else None
                 Hs = Hbuf[k % 2]
-                if batched:
+                if peer:
+                    peer_drv.train_sequence(g, t0, p, p["w_o"], p["b_o"], stage[k % 2][:n], ystage[k % 2][:n],
+                                            Hprev, Hs, grads, dw_o, db_o, loss)
+                elif batched:
                     stg.stg_tgcn_train_sequence_batched(g, n, p, p["w_o"], p["b_o"], stage[k % 2][:n],
                                                         ystage[k % 2][:n], Hprev, Hs, grads, dw_o, db_o, loss, stack)
                 else:
@@ -468,7 +491,7 @@ def main():
         e2e = {"value": edges_all * args.steps / e2e_s, "unit": UNIT,
                "h2d_bytes_per_step": int(h2d / args.steps), "d2h_bytes_per_step": 4,
                "ms_per_step": 1e3 * e2e_s / args.steps,
-               "note": "X_t (256 MB) and y_t copied H2D from pinned host memory every timestep on a copy "
+               "note": "X_t (this rank's rows in sharded mode) and y_t copied H2D from pinned host memory every timestep on a copy "
                        "stream overlapped with the previous sequence; loss read back every epoch"}
 
     # ---------------- CPU baseline: the oracle on one C5 timestep (rank 0, N=1 only)
@@ -501,8 +524,11 @@ def main():
                               else "working set fits in L2 (not flushed between epochs)"),
                        "cuda_graph": cg is not None,
                        "schedule": "sequence-batched (NEXT-1)" if batched else "per-timestamp Algorithm 1",
-                       "parallelism": ("row-block shards x%d (resident X_t, NCCL gradient all-reduce per "
-                                       "sequence)" % world) if sharded else ("replicas" if world > 1 else "single"),
+                       "parallelism": ("row-block shards x%d, sharded mode: X_t row-sharded, P' gathered from "
+                                       "its owners over CUDA-IPC peer memory inside the aggregation, partial dP "
+                                       "reduce-scattered over peer loads" % world) if peer else
+                                      (("row-block shards x%d (resident X_t, NCCL gradient all-reduce per "
+                                        "sequence)" % world) if sharded else ("replicas" if world > 1 else "single")),
                        "E_local_mean_rank0": int(E_mean)},
             "timesteps_per_s": tsps,
             "shard_sim": args.shard_sim,
@@ -523,7 +549,12 @@ def main():
             "cpu_baseline": cpu,
         }
         print(json.dumps(out), flush=True)
-    if pg:
+    if peer_drv is not None:
+        torch.cuda.synchronize()
+        if pg:
+            dist.barrier()
+        peer_drv.close()
+    if pg or peer:
         dist.barrier()
         dist.destroy_process_group()
 

@@ -83,6 +83,8 @@ def stream_barrier(device=None):
     """Cross-rank ordering point for the peer buffers (include/stg.h): with NCCL a
     one-element all-reduce on the current stream (stream-ordered, no host sync);
     with gloo (CPU tests, ranks sharing one GPU) a device synchronize + barrier."""
+    if dist.get_world_size() == 1:                # no peers: stream order suffices
+        return
     if dist.get_backend() == "nccl":
         t = torch.zeros(1, device=device or torch.device("cuda", torch.cuda.current_device()))
         dist.all_reduce(t)
