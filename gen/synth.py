@@ -331,3 +331,8 @@ def tgcn_params(F: int, H: int, seed: int, scale: float = 1.0):
         "w_o": u(904, H, H),
         "b_o": u(905, 1, H),
     }
+
+
+def edge_weights(seed: int, n: int, lo: float = 0.5, hi: float = 2.0, stream: int = 40) -> np.ndarray:
+    """n seeded positive edge weights in [lo, hi) (NEXT-4 inputs), multiples of 2^-24 scaled."""
+    return (lo + (hi - lo) * uniform_01(seed, stream, n)).astype(np.float32)

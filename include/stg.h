@@ -195,6 +195,26 @@ stg_status stg_gcn_aggregate_ex(const stg_csr_view* g, int32_t backward, int32_t
                                 const float* scale_row, const float* scale_col, const float* bias,
                                 stg_stream_t stream);
 
+/* Edge-weighted aggregation (features "of nodes and edges",
+ * P:L50; shared edge labels):
+ *   out[r,:] = scale_row[r] · Σ_{j ∈ row r} w_j · scale_col[c_j] · in[c_j,:] + bias[:]
+ * where w_j is the weight of the EDGE at position j: ew is indexed by the edge
+ * label = in-CSR position (reading C6), so the forward reads ew[j] and the
+ * backward (out-CSR) reads ew[out_eid[j]] — the transpose uses the same weights
+ * without a permuted copy.  ew [E] fp32 device array in in-CSR order.  The backward
+ * needs a view with out_eid (STG_EDGE_IDS).  Float4 path only: W % 4 == 0,
+ * W <= 512, 16-byte aligned rows, a library view (STG_ERR_INVALID_ARG otherwise).
+ * Other conventions as stg_gcn_aggregate_ex. */
+stg_status stg_gcn_aggregate_weighted(const stg_csr_view* g, int32_t backward, int32_t W, const float* ew,
+                                      const float* in, int64_t ldin, float* out, int64_t ldout,
+                                      const float* scale_row, const float* scale_col, const float* bias,
+                                      stg_stream_t stream);
+/* Weighted GCN normalisation (PyG gcn_norm with edge weights; reading C21):
+ * norm[i] = (Σ_{j ∈ in-row i} ew[j])^-1/2, 0 if the sum is <= 0, for the R local rows
+ * of the view (R = V unsharded; the symmetric norm uses it for both n_src and n_dst).
+ * Per-row sums in fp64 (fixed order), result rounded to fp32. */
+stg_status stg_gcn_weighted_norm(const stg_csr_view* g, const float* ew, float* norm, stg_stream_t stream);
+
 /* Work decomposition of the aggregation (process-wide; every strategy is
  * deterministic, uses no float atomics, and keeps each fp32 chain <= 64 terms).
  * The snapshot schedule lists rows in node_ids order (degree presort,

@@ -49,6 +49,10 @@ def lib():
         _lib.orc_csr_build.argtypes = [i32, i64, P, i32] + [P] * 11
         _lib.orc_aggregate.restype = None
         _lib.orc_aggregate.argtypes = [i32, P, P, P, P, i32, P, P]
+        _lib.orc_aggregate_edges.restype = None
+        _lib.orc_aggregate_edges.argtypes = [i32, i64, P, P, P, P, i32, i32, P, P]
+        _lib.orc_weighted_norm.restype = None
+        _lib.orc_weighted_norm.argtypes = [i32, i64, P, P, P]
         _lib.orc_set_apply.restype = i64
         _lib.orc_set_apply.argtypes = [P, i64, P, i64, P, i64, P]
         _lib.orc_window_set.restype = i64
@@ -143,6 +147,30 @@ def aggregate_bwd(g: dict, gy) -> np.ndarray:
 def aggregate_scale(g: dict, x, bwd: bool = False) -> np.ndarray:
     """Same aggregation over |x| — the per-element condition scale s_i of reading C19."""
     return (aggregate_bwd if bwd else aggregate_fwd)(g, np.abs(np.asarray(x, np.float64)))
+
+
+def aggregate_edges(V: int, S, w, nrow, ncol, x, backward: bool = False) -> np.ndarray:
+    """Edge-weighted aggregation over the edge set S with per-edge weights w
+    (aligned with the sorted keys S): forward y_v = Σ_{(u,v)∈S} n[v]·w·n[u]·x_u,
+    backward the transpose (NEXT-4)."""
+    S, w = _c(S, np.uint64), _c(w, np.float64)
+    x = _c(x, np.float64)
+    W = x.shape[1]
+    nrow = _c(nrow, np.float64)
+    ncol_p = None if ncol is None else _c(ncol, np.float64)
+    y = np.zeros((V, W), np.float64)
+    lib().orc_aggregate_edges(V, S.size, _p(S if S.size else np.zeros(1, np.uint64)),
+                              _p(w if w.size else np.zeros(1)), _p(nrow), None if ncol_p is None else _p(ncol_p),
+                              int(backward), W, _p(x), _p(y))
+    return y
+
+
+def weighted_norm(V: int, S, w) -> np.ndarray:
+    S, w = _c(S, np.uint64), _c(w, np.float64)
+    out = np.zeros(max(V, 1), np.float64)
+    lib().orc_weighted_norm(V, S.size, _p(S if S.size else np.zeros(1, np.uint64)), _p(w if w.size else np.zeros(1)),
+                            _p(out))
+    return out[:V]
 
 
 # ------------------------------------------------------------------ snapshots

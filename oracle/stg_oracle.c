@@ -160,6 +160,35 @@ void orc_aggregate(int32_t R, const int32_t* rowptr, const int32_t* col,
 }
 
 /* ---------------------------------------------------------------------------
+ * Edge-weighted aggregation (edge features; the
+ * weights PyG-T's TGCN passes to its GCN, reading C21), written over the edge
+ * SET itself (no CSR, no labels): S sorted unique keys (src,dst), w[k] = the
+ * weight of edge S[k].
+ *   forward : y[v,:]  += n[v] * w(u,v) * n[u] * x[u,:]   for every (u,v) in S
+ *   backward: gx[u,:] += n[u] * w(u,v) * n[v] * gy[v,:]  for every (u,v) in S
+ * (nrow = the scale of the output vertex, ncol = the scale of the input vertex;
+ * ncol may be NULL = 1).  y has V rows and is overwritten.  fp64.
+ * ------------------------------------------------------------------------- */
+void orc_aggregate_edges(int32_t V, int64_t n, const uint64_t* S, const double* w, const double* nrow,
+                         const double* ncol, int32_t backward, int32_t W, const double* x, double* y) {
+  for (int64_t i = 0; i < (int64_t)V * W; ++i) y[i] = 0.0;
+  for (int64_t k = 0; k < n; ++k) {
+    int32_t u = ksrc(S[k]), v = kdst(S[k]);
+    int32_t o = backward ? u : v, in = backward ? v : u;      /* output row, input row */
+    double c = nrow[o] * w[k] * (ncol ? ncol[in] : 1.0);
+    for (int32_t j = 0; j < W; ++j) y[(int64_t)o * W + j] += c * x[(int64_t)in * W + j];
+  }
+}
+
+/* Weighted GCN normalisation (PyG gcn_norm with edge weights):
+ * deg[v] = sum_{(u,v) in S} w(u,v);  norm[v] = deg^-1/2, 0 if deg <= 0. */
+void orc_weighted_norm(int32_t V, int64_t n, const uint64_t* S, const double* w, double* norm) {
+  for (int32_t v = 0; v < V; ++v) norm[v] = 0.0;
+  for (int64_t k = 0; k < n; ++k) norm[kdst(S[k])] += w[k];
+  for (int32_t v = 0; v < V; ++v) norm[v] = norm[v] > 0.0 ? 1.0 / sqrt(norm[v]) : 0.0;
+}
+
+/* ---------------------------------------------------------------------------
  * DTDG snapshots (base graph + list of edge additions/deletions).
  * S_t = (S_{t-1} \ D_t) ∪ A_t.  S sorted unique; A, D arbitrary multisets.
  * out capacity: n + na.  Returns |S_t|.

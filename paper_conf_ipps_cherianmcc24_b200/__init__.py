@@ -124,6 +124,9 @@ _decl("stg_debug_tc_gemm", [_i32, _i32, _i32, _i32, _i32, _P, _P, _P, _P])
 _decl("stg_aggregate_set_strategy", [_i32])
 _decl("stg_aggregate_set_param", [_i32, _i64])
 _decl("stg_profile_read", [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64), _i32])
+_decl("stg_gcn_aggregate_weighted", [ctypes.POINTER(stg_csr_view), _i32, _i32, _P, _P, _i64, _P, _i64, _P, _P, _P,
+                                     _P])
+_decl("stg_gcn_weighted_norm", [ctypes.POINTER(stg_csr_view), _P, _P, _P])
 _decl("stg_peer_alloc", [_i64, ctypes.POINTER(_P), ctypes.POINTER(stg_ipc_handle)])
 _decl("stg_peer_free", [_P])
 _decl("stg_peer_open", [ctypes.POINTER(stg_ipc_handle), ctypes.POINTER(_P)])
@@ -151,6 +154,7 @@ ABI_SYMBOLS = [
     "stg_tgcn_train_sequence_batched",
     "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
+    "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm",
     "stg_peer_alloc", "stg_peer_free", "stg_peer_open", "stg_peer_close", "stg_allgather_rows",
     "stg_gcn_aggregate_peer", "stg_reduce_scatter_rows", "stg_tgcn_project", "stg_tgcn_step_peer",
     "stg_tgcn_step_backward_peer", "stg_tgcn_dw",
@@ -380,6 +384,25 @@ def stg_gcn_aggregate_ex(v: stg_csr_view, backward: bool, x: torch.Tensor, out: 
     _check(_lib.stg_gcn_aggregate_ex(ctypes.byref(v), int(backward), W, _ptr(x), x.stride(0), _ptr(out),
                                      out.stride(0), _ptr(scale_row), _ptr(scale_col), _ptr(bias), _stream(stream)))
     return out
+
+
+def stg_gcn_aggregate_weighted(v: stg_csr_view, backward: bool, ew: torch.Tensor, x: torch.Tensor,
+                               out: torch.Tensor = None, scale_row=None, scale_col=None, bias=None, stream=None):
+    """Edge-weighted aggregation; ew [E] in in-CSR order (edge label = in-CSR position)."""
+    W = x.shape[1]
+    rows = v.num_nodes if backward else v.row_end - v.row_begin
+    out = _out2d(x, rows, W, out)
+    _check(_lib.stg_gcn_aggregate_weighted(ctypes.byref(v), int(backward), W, _ptr(ew), _ptr(x), x.stride(0),
+                                           _ptr(out), out.stride(0), _ptr(scale_row), _ptr(scale_col), _ptr(bias),
+                                           _stream(stream)))
+    return out
+
+
+def stg_gcn_weighted_norm(v: stg_csr_view, ew: torch.Tensor, norm: torch.Tensor = None, stream=None):
+    if norm is None:
+        norm = torch.empty(v.row_end - v.row_begin, dtype=torch.float32, device="cuda")
+    _check(_lib.stg_gcn_weighted_norm(ctypes.byref(v), _ptr(ew), _ptr(norm), _stream(stream)))
+    return norm
 
 
 # ---------------------------------------------------------------- TGCN

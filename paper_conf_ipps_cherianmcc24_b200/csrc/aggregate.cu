@@ -281,6 +281,12 @@ struct Agg2Args {
   // pbase[k] + u·ldx (the block base shifted back by pbnd[k] rows)
   const float* pbase[STG_MAX_PEERS];
   int32_t pbnd[STG_MAX_PEERS];
+  // edge weights (stg_gcn_aggregate_weighted): the weight of
+  // the edge at CSR position e is ew[eid ? eid[e] : e] (ew in in-CSR order, the
+  // shared edge labels P:L197; the out-CSR reaches it through out_eid).  Only the
+  // SCOL instantiation reads them.
+  const float* ew;
+  const int32_t* eid;
 };
 
 // Strategy 1: software-pipelined degree-ordered items.  A warp serves 32/G
@@ -604,13 +610,14 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
         __stcs(reinterpret_cast<float4*>(ybase + (int64_t)vz * a.ldy) + lane,
                scale_bias(0.f, make_float4(0.f, 0.f, 0.f, 0.f), bbase, 4 * lane));
     }
-    auto resolve = [&](int32_t pos, int32_t& u, int32_t& k) {
+    auto resolve = [&](int32_t pos, int32_t& u, int32_t& k, int32_t& e) {
       int32_t lo = 0;
 #pragma unroll
       for (int st = 16; st >= 1; st >>= 1)
         if (lo + st <= 31 && ex[lo + st] <= pos) lo += st;
       k = lo;
-      u = pos < N ? __ldcs(a.col + s_beg[w][lo] + (pos - ex[lo])) : a.upad;
+      e = s_beg[w][lo] + (pos - ex[lo]);
+      u = pos < N ? __ldcs(a.col + e) : a.upad;
     };
     auto flush = [&](int c, const float4& sum) {
       const float sv = __shfl_sync(FULL, sl, c);
@@ -622,8 +629,8 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
           reinterpret_cast<float4*>(pbase + (ib + c) * Wl)[lane] = sum;
       }
     };
-    int32_t u0, k0;
-    resolve(lane, u0, k0);
+    int32_t u0, k0, e0;
+    resolve(lane, u0, k0, e0);
     int cur = -1;
     float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
     for (int32_t b0 = 0; b0 < N; b0 += 32) {
@@ -635,10 +642,13 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
       const int32_t kc = lane < nb ? k0 : -1;
       const uint32_t bm = __ballot_sync(FULL, lane <= nb && (lane == 0 ? kc != cur : (lane == nb || kc != kp)));
       float sc = 1.0f;
-      if (SCOL && lane < nb) sc = __ldg(a.scol + u0);
+      if (SCOL && lane < nb) {
+        sc = a.scol ? __ldg(a.scol + u0) : 1.0f;
+        if (a.ew) sc *= __ldg(a.ew + (a.eid ? __ldg(a.eid + e0) : e0));
+      }
       const int32_t uc = u0;
       const unsigned long long ua = PEER ? peer_row(u0) : 0ull;
-      if (b0 + 32 < N) resolve(b0 + 32 + lane, u0, k0);  // next batch in flight
+      if (b0 + 32 < N) resolve(b0 + 32 + lane, u0, k0, e0);  // next batch in flight
       for (int32_t j0 = 0; j0 < nb; j0 += D) {
         float4 v[D];
 #pragma unroll
@@ -679,6 +689,24 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
     __syncwarp();
   }
   asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+}
+
+// Weighted GCN normalisation (PyG gcn_norm with edge weights, reading C21 / NEXT-4):
+// deg_w[v] = Σ_{j ∈ in-row v} ew[j], norm[v] = deg_w^-1/2 (0 if deg_w <= 0).  One
+// warp per row; lane-strided fp64 partial sums and a fixed shuffle tree, so the
+// fp32 result is the correctly rounded norm of a (nearly) exact sum, run to run.
+__global__ void __launch_bounds__(256) k_weighted_norm(const int32_t* __restrict__ rowptr, int32_t R,
+                                                       const float* __restrict__ ew, float* __restrict__ norm) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < R; v += nw) {
+    const int32_t b = rowptr[v], e = rowptr[v + 1];
+    double acc = 0.0;
+    for (int32_t j = b + lane; j < e; j += 32) acc += (double)__ldg(ew + j);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) norm[v] = acc > 0.0 ? (float)(1.0 / sqrt(acc)) : 0.0f;
+  }
 }
 
 using ItemsFn = void (*)(const Agg2Args);
@@ -801,8 +829,10 @@ static void lane_groups(int nv, int vpl_max, int* g, int* vpl) {
 // blocks of `peers` (in / ldin are ignored); only the edge-stream kernel serves it.
 stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
                             float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
-                            cudaStream_t s, const stg_peer_rows* peers) {
+                            cudaStream_t s, const stg_peer_rows* peers, const float* ew) {
   if (!gv) return fail(STG_ERR_INVALID_ARG, "aggregate: view is NULL");
+  if (ew && backward && !gv->out_eid)
+    return fail(STG_ERR_INVALID_ARG, "aggregate_weighted: the backward needs the edge labels (STG_EDGE_IDS)");
   if (W < 1) return fail(STG_ERR_INVALID_ARG, "aggregate: W=%d < 1", W);
   int32_t peer_pad = 0;
   if (peers) {
@@ -887,12 +917,16 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   const int32_t wsplit = (int32_t)(ceil_div(ceil_div(W, 4), nsplit) * 4);
   if (peers && !(vec4 && a.sched && wsplit <= 128))
     return fail(STG_ERR_INVALID_ARG, "aggregate_peer: output must be 16-byte aligned with ldout %% 4 == 0");
-  if (peers || (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128)) {
+  if (ew && !(vec4 && a.sched && wsplit <= 128))
+    return fail(STG_ERR_INVALID_ARG, "aggregate_weighted: needs W %% 4 == 0, W <= 512, 16-byte aligned rows "
+                "and a library view (schedule)");
+  if (peers || ew || (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128)) {
     STG_TRY(ws->queue.alloc(nsplit, s));
     STG_CUDA(cudaMemsetAsync(ws->queue.p, 0, sizeof(uint32_t) * nsplit, s));
     const int64_t pstride = chunks_bound * wsplit;               // the column chunks run concurrently
     STG_TRY(ws->partials.alloc((size_t)(pstride * nsplit) + 4, s));
-    const StreamFn fn = peers ? pick_stream_peer(scol != nullptr) : pick_stream(g_tune.d, g_tune.minb, scol != nullptr);
+    const bool per_edge = scol != nullptr || ew != nullptr;
+    const StreamFn fn = peers ? pick_stream_peer(per_edge) : pick_stream(g_tune.d, g_tune.minb, per_edge);
     // group sizes: ~max(256, E / (8 warps x #SM)) edges per group (all 32-item light
     // groups at C5 scale; small graphs get small groups, hence many warps)
     const int64_t target = std::max<int64_t>(256, gv->num_edges / (8 * (int64_t)num_sms()));
@@ -911,6 +945,8 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     b.upad = (backward && a.ids) ? (int32_t)rb : 0;     // row 0 of a shifted input is not a valid row
     b.hgrp = hgrp; b.lgrp = lgrp;
     b.wsplit = wsplit; b.wtotal = W; b.pstride = pstride;
+    b.ew = ew;
+    b.eid = (ew && backward) ? gv->out_eid : nullptr;
     for (int k = 0; k < STG_MAX_PEERS; ++k) {
       b.pbnd[k] = INT32_MAX;
       b.pbase[k] = nullptr;
@@ -998,6 +1034,28 @@ stg_status stg_gcn_aggregate_peer(const stg_csr_view* g, int32_t W, const stg_pe
                                   stg_stream_t stream) {
   if (!x) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_peer: row table is NULL");
   return stg::aggregate_launch(g, 0, W, nullptr, 0, out, ldout, scale_row, scale_col, bias, (cudaStream_t)stream, x);
+}
+
+stg_status stg_gcn_aggregate_weighted(const stg_csr_view* g, int32_t backward, int32_t W, const float* ew,
+                                      const float* in, int64_t ldin, float* out, int64_t ldout,
+                                      const float* scale_row, const float* scale_col, const float* bias,
+                                      stg_stream_t stream) {
+  if (!g) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_weighted: view is NULL");
+  if (!ew && g->num_edges > 0) return stg::fail(STG_ERR_INVALID_ARG, "stg_gcn_aggregate_weighted: ew is NULL");
+  return stg::aggregate_launch(g, backward, W, in, ldin, out, ldout, scale_row, scale_col, bias, (cudaStream_t)stream,
+                               nullptr, ew ? ew : nullptr);
+}
+
+stg_status stg_gcn_weighted_norm(const stg_csr_view* g, const float* ew, float* norm, stg_stream_t stream) {
+  using stg::fail;
+  if (!g || !norm || (!ew && g->num_edges > 0)) return fail(STG_ERR_INVALID_ARG, "stg_gcn_weighted_norm: NULL argument");
+  if (!g->in_rowptr) return fail(STG_ERR_INVALID_ARG, "stg_gcn_weighted_norm: view lacks the forward CSR");
+  const int32_t R = g->row_end - g->row_begin;
+  if (R <= 0) return STG_OK;
+  const unsigned blocks = (unsigned)std::min<int64_t>(stg::ceil_div(R, 8), (int64_t)stg::num_sms() * 16);
+  stg::k_weighted_norm<<<blocks, 256, 0, (cudaStream_t)stream>>>(g->in_rowptr, R, ew, norm);
+  stg::count_launch();
+  return stg::check_launch("stg_gcn_weighted_norm");
 }
 
 stg_status stg_aggregate_set_strategy(int32_t strategy) {

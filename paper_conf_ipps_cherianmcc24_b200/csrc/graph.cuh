@@ -38,7 +38,7 @@ inline int64_t sched_size(int64_t V, int64_t E) {
 // sharded-mode gather from the owners' row blocks (stg_gcn_aggregate_peer).
 stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, const float* in, int64_t ldin,
                             float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
-                            cudaStream_t s, const stg_peer_rows* peers = nullptr);
+                            cudaStream_t s, const stg_peer_rows* peers = nullptr, const float* ew = nullptr);
 
 struct AggWs {
   DArray<float> partials;
