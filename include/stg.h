@@ -65,8 +65,12 @@ enum {
   STG_VALIDATE = 1u << 2,       /* DTDG: reject ill-formed batches (duplicate adds, adds of
                                    present edges, deletes of absent edges) instead of
                                    normalising them (reading C9) */
-  STG_NORM_DGL_BOTH = 1u << 3   /* n_src = out_deg^-1/2, n_dst = in_deg^-1/2 (default:
+  STG_NORM_DGL_BOTH = 1u << 3,  /* n_src = out_deg^-1/2, n_dst = in_deg^-1/2 (default:
                                    both = in_deg^-1/2, PyG gcn_norm, reading C1) */
+  STG_NAIVE = 1u << 4           /* DTDG NaiveGraph mode:
+                                   materialise every snapshot S_0..S_{T-1} at create
+                                   (memory ∝ Σ_t |E_t|); Get-Graph / Get-Backward-Graph
+                                   are lookups.  Unsharded only. */
 };
 
 /* Row-block sharding (north_star "partitioned ... by
@@ -169,6 +173,10 @@ int64_t stg_dtdg_num_edges(const stg_dtdg* g, int32_t t);    /* edges held at t 
 int32_t stg_dtdg_num_timestamps(const stg_dtdg* g);
 /* Number of effective added / deleted edges of step t (0 for t = 0). */
 int64_t stg_dtdg_num_deltas(const stg_dtdg* g, int32_t t, int32_t deletes);
+/* Device bytes held by a DTDG (the Table III / Fig. 8 memory comparison):
+ * the normalised delta arrays, the snapshot cache (Alg. 2 slots, scratch), and the
+ * snapshots materialised by STG_NAIVE (0 otherwise). */
+stg_status stg_dtdg_memory(const stg_dtdg* g, int64_t* deltas, int64_t* cache, int64_t* materialised);
 void stg_dtdg_destroy(stg_dtdg* g);
 
 /* ---- GCN aggregation (north_star) ----

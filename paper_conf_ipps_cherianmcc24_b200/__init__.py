@@ -21,6 +21,7 @@ STG_SELF_LOOPS = 1 << 0
 STG_EDGE_IDS = 1 << 1
 STG_VALIDATE = 1 << 2
 STG_NORM_DGL_BOTH = 1 << 3
+STG_NAIVE = 1 << 4
 STG_PART_IN, STG_PART_OUT, STG_PART_EID = 1 << 0, 1 << 1, 1 << 2
 
 STATUS = {0: "STG_OK", 1: "STG_ERR_INVALID_ARG", 2: "STG_ERR_OUT_OF_RANGE", 3: "STG_ERR_NO_MEMORY",
@@ -100,6 +101,7 @@ _decl("stg_dtdg_num_edges", [_P, _i32], _i64)
 _decl("stg_dtdg_num_timestamps", [_P], _i32)
 _decl("stg_dtdg_num_deltas", [_P, _i32, _i32], _i64)
 _decl("stg_dtdg_destroy", [_P], None)
+_decl("stg_dtdg_memory", [_P, ctypes.POINTER(_i64), ctypes.POINTER(_i64), ctypes.POINTER(_i64)])
 _decl("stg_gcn_aggregate_fwd", [ctypes.POINTER(stg_csr_view), _i32, _P, _i64, _P, _i64, _P])
 _decl("stg_gcn_aggregate_bwd", [ctypes.POINTER(stg_csr_view), _i32, _P, _i64, _P, _i64, _P])
 _decl("stg_gcn_aggregate_ex", [ctypes.POINTER(stg_csr_view), _i32, _i32, _P, _i64, _P, _i64, _P, _P, _P, _P])
@@ -147,7 +149,7 @@ ABI_SYMBOLS = [
     "stg_static_graph_create", "stg_graph_view", "stg_graph_destroy",
     "stg_dtdg_create", "stg_dtdg_get_snapshot", "stg_dtdg_get_backward_snapshot", "stg_dtdg_get_snapshot_parts",
     "stg_dtdg_num_edges",
-    "stg_dtdg_num_timestamps", "stg_dtdg_num_deltas", "stg_dtdg_destroy",
+    "stg_dtdg_num_timestamps", "stg_dtdg_num_deltas", "stg_dtdg_destroy", "stg_dtdg_memory",
     "stg_gcn_aggregate_fwd", "stg_gcn_aggregate_bwd", "stg_gcn_aggregate_ex",
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
     "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_mse_head_ex", "stg_sgd_update", "stg_tgcn_train_sequence",
@@ -251,6 +253,12 @@ class Dtdg:
 
     def num_deltas(self, t: int, deletes: bool) -> int:
         return int(_lib.stg_dtdg_num_deltas(self.handle, t, int(deletes)))
+
+    def memory(self) -> dict:
+        """Device bytes: normalised deltas, snapshot cache, materialised snapshots (STG_NAIVE)."""
+        a, b, c = _i64(0), _i64(0), _i64(0)
+        _check(_lib.stg_dtdg_memory(self.handle, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
+        return {"deltas": a.value, "cache": b.value, "materialised": c.value}
 
     def close(self):
         if self.handle:

@@ -7,6 +7,8 @@
 // step is exactly reversible and every E_t is known without a host sync.
 #include <vector>
 
+#include <memory>
+
 #include "graph.cuh"
 #include "prims.cuh"
 
@@ -124,6 +126,9 @@ struct stg_dtdg {
   std::vector<int64_t> ga_off, gd_off;
   DArray<uint64_t> gadd, gdel;
   Snapshot slot[5];                                // 0 = base, 1-2 = forward pair, 3-4 = backward pair
+  // NaiveGraph mode (STG_NAIVE): every snapshot
+  // materialised at create, Get-Graph is a lookup
+  std::vector<std::unique_ptr<Snapshot>> naive;
   int head_f = -1, head_b = -1;
   DArray<int4> touch_in, touch_out;
   BuildWs* ws = nullptr;
@@ -141,7 +146,10 @@ struct stg_dtdg {
   // one delta step from slot `from` (time t0) to slot `to` (time t0 ± 1) of the
   // CSR directions in `parts`; the whole-graph degrees (norms) always follow
   stg_status step(int from, int to, int dirn, uint32_t parts, cudaStream_t s) {
-    const int32_t t0 = slot[from].t;
+    return step_snap(slot[from], slot[to], dirn, parts, s);
+  }
+  stg_status step_snap(const Snapshot& sf, Snapshot& st, int dirn, uint32_t parts, cudaStream_t s) {
+    const int32_t t0 = sf.t;
     const int32_t t1 = t0 + dirn;
     const int32_t td = dirn > 0 ? t1 : t0;       // batch applied (forward) or undone (reverse)
     const bool rev = dirn < 0;
@@ -150,11 +158,11 @@ struct stg_dtdg {
     const std::vector<int64_t>& gao = sharded ? ga_off : a_off;
     const std::vector<int64_t>& gdo = sharded ? gd_off : d_off;
     const size_t vb = sizeof(int32_t) * (size_t)V;
-    STG_CUDA(cudaMemcpyAsync(slot[to].gin_deg.p, slot[from].gin_deg.p, vb, cudaMemcpyDeviceToDevice, s));
-    STG_CUDA(cudaMemcpyAsync(slot[to].gout_deg.p, slot[from].gout_deg.p, vb, cudaMemcpyDeviceToDevice, s));
-    degree_hist(ga + gao[td], gao[td + 1] - gao[td], nb, rev ? -1 : 1, slot[to].gin_deg.p, slot[to].gout_deg.p, s);
-    degree_hist(gd + gdo[td], gdo[td + 1] - gdo[td], nb, rev ? 1 : -1, slot[to].gin_deg.p, slot[to].gout_deg.p, s);
-    return apply_delta(slot[from], slot[to], dir(td, true, rev), dir(td, false, rev), E[t1], t1, touch_in.p,
+    STG_CUDA(cudaMemcpyAsync(st.gin_deg.p, sf.gin_deg.p, vb, cudaMemcpyDeviceToDevice, s));
+    STG_CUDA(cudaMemcpyAsync(st.gout_deg.p, sf.gout_deg.p, vb, cudaMemcpyDeviceToDevice, s));
+    degree_hist(ga + gao[td], gao[td + 1] - gao[td], nb, rev ? -1 : 1, st.gin_deg.p, st.gout_deg.p, s);
+    degree_hist(gd + gdo[td], gdo[td + 1] - gdo[td], nb, rev ? 1 : -1, st.gin_deg.p, st.gout_deg.p, s);
+    return apply_delta(sf, st, dir(td, true, rev), dir(td, false, rev), E[t1], t1, touch_in.p,
                        touch_out.p, *ws, s, parts & (PART_IN | PART_OUT));
   }
 
@@ -186,6 +194,10 @@ struct stg_dtdg {
   }
 
   stg_status get(int32_t t, bool backward, uint32_t parts, cudaStream_t s, stg_csr_view* v) {
+    if (!naive.empty()) {                          // NaiveGraph: every part of every t is stored
+      naive[t]->view(v, &agg);
+      return STG_OK;
+    }
     int idx = -1;
     if (!backward) {
       if (t == 0 && head_f < 0) {
@@ -236,6 +248,8 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
     return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: batch 0 must be empty (S_0 is the base)");
   if ((add_off[T] > add_off[0] && (!add_src || !add_dst)) || (del_off[T] > del_off[0] && (!del_src || !del_dst)))
     return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: NULL delta arrays");
+  if ((flags & STG_NAIVE) && dist && (dist->row_begin != 0 || dist->row_end != V))
+    return fail(STG_ERR_INVALID_ARG, "stg_dtdg_create: STG_NAIVE is for unsharded graphs");
   const int loops = (flags & STG_SELF_LOOPS) ? 1 : 0;
   if (E0 + (loops ? V : 0) >= (int64_t(1) << 31)) return fail(STG_ERR_OUT_OF_RANGE, "stg_dtdg_create: E0 >= 2^31");
   cudaStream_t s = (cudaStream_t)stream;
@@ -462,6 +476,24 @@ stg_status stg_dtdg_create(int32_t V, int32_t T, int64_t E0, const int32_t* src0
     }
     CK(build_from_out_keys(bk, g->E[0], g->slot[0], ws, s));
   }
+  // NaiveGraph mode: materialise S_0 .. S_{T-1} (both CSRs, labels, schedules) by
+  // walking the deltas forward once
+  if (st == STG_OK && (flags & STG_NAIVE)) {
+    g->naive.resize(T);
+    for (int32_t t = 0; t < T && st == STG_OK; ++t) {
+      g->naive[t].reset(new Snapshot());
+      Snapshot& sn = *g->naive[t];
+      CK(sn.alloc(V, std::max<int64_t>(g->E[t], 1), eids, dgl, g->rb, g->re));
+      if (st != STG_OK) break;
+      if (t == 0) {
+        sn.t = 0;
+        CK(build_from_out_keys(base_keys.p, g->E[0], sn, ws, s));
+      } else {
+        CK(g->step_snap(*g->naive[t - 1], sn, 1, PART_IN | PART_OUT, s));
+        CK(complete_parts(sn, PART_ALL, ws, s));
+      }
+    }
+  }
   if (st == STG_OK && cudaStreamSynchronize(s) != cudaSuccess)
     st = fail(STG_ERR_CUDA, "stg_dtdg_create: %s", cudaGetErrorString(cudaGetLastError()));
 #undef CK
@@ -504,6 +536,21 @@ int32_t stg_dtdg_num_timestamps(const stg_dtdg* g) { return g ? g->T : -1; }
 int64_t stg_dtdg_num_deltas(const stg_dtdg* g, int32_t t, int32_t deletes) {
   if (!g || t < 0 || t >= g->T) return -1;
   return deletes ? g->d_off[t + 1] - g->d_off[t] : g->a_off[t + 1] - g->a_off[t];
+}
+
+stg_status stg_dtdg_memory(const stg_dtdg* g, int64_t* deltas, int64_t* cache, int64_t* materialised) {
+  if (!g || !deltas || !cache || !materialised) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_memory: NULL argument");
+  const DArray<uint64_t>* d[] = {&g->add_out, &g->add_in, &g->del_out, &g->del_in, &g->gadd, &g->gdel};
+  int64_t b = 0;
+  for (const auto* a : d) b += (int64_t)(a->n * sizeof(uint64_t));
+  *deltas = b;
+  b = (int64_t)((g->touch_in.n + g->touch_out.n) * sizeof(int4));
+  for (const auto& sl : g->slot) b += (int64_t)sl.bytes();
+  *cache = b;
+  b = 0;
+  for (const auto& sn : g->naive) b += (int64_t)sn->bytes();
+  *materialised = b;
+  return STG_OK;
 }
 
 void stg_dtdg_destroy(stg_dtdg* g) {

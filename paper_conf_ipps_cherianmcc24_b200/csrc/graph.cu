@@ -40,6 +40,14 @@ stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_
   return STG_OK;
 }
 
+size_t Snapshot::bytes() const {
+  const DArray<int32_t>* ia[] = {&in_rowptr, &in_col, &in_row, &in_deg, &in_ids, &out_rowptr, &out_col, &out_row,
+                                 &out_deg, &out_ids, &out_eid, &in_sched, &out_sched, &gin_deg, &gout_deg};
+  size_t b = 0;
+  for (const auto* a : ia) b += a->n * sizeof(int32_t);
+  return b + (norm_src.n + norm_dst.n) * sizeof(float);
+}
+
 void Snapshot::view(stg_csr_view* v, AggWs* ws) const {
   v->num_nodes = V;
   v->row_begin = rb;

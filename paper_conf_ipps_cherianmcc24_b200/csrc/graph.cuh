@@ -72,6 +72,7 @@ struct Snapshot {
 
   stg_status alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_t rb_ = 0, int32_t re_ = -1);
   int32_t rows() const { return re - rb; }
+  size_t bytes() const;   // device bytes held
   void view(stg_csr_view* v, AggWs* ws) const;
 };
 
