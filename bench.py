@@ -52,6 +52,9 @@ def parse():
                          "whose tiny per-timestamp work is launch-bound, off for DTDGs)")
     ap.add_argument("--schedule", default="auto", choices=["auto", "batched", "per-step"],
                     help="static graphs: sequence-batched (NEXT-1, default) or per-timestamp Algorithm-1 driver")
+    ap.add_argument("--naive", action="store_true",
+                    help="DTDG configs: NaiveGraph mode (every snapshot materialised at create, P:L202-204; "
+                         "Table III's time/memory trade-off against the default on-demand snapshots)")
     ap.add_argument("--shard-sim", default=None, metavar="K/N",
                     help="(testing on one GPU) run rank K's row block of an N-way sharding, no process group")
     return ap.parse_args()
@@ -276,7 +279,8 @@ def main():
         E_t = [g.view().num_edges] * T
     else:
         g = stg.stg_dtdg_create(V, T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
-                                d.del_dst, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS, dist=dist_arg)
+                                d.del_dst, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS |
+                                (stg.STG_NAIVE if args.naive else 0), dist=dist_arg)
         E_t = [g.num_edges(t) for t in range(T)]
     edges_per_step = 2 * sum(E_t)            # this rank's edges (whole graph unless sharded)
     edges_all = edges_per_step
@@ -531,6 +535,9 @@ def main():
                                         "sequence)" % world) if sharded else ("replicas" if world > 1 else "single")),
                        "E_local_mean_rank0": int(E_mean)},
             "timesteps_per_s": tsps,
+            "graph_memory_bytes": None if static else g.memory(),
+            "snapshots": None if static else ("materialised (NaiveGraph, STG_NAIVE)" if args.naive
+                                              else "on demand from base + deltas (Algorithm 2 cache)"),
             "shard_sim": args.shard_sim,
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

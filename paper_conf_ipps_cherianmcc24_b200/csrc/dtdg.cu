@@ -538,6 +538,14 @@ int64_t stg_dtdg_num_deltas(const stg_dtdg* g, int32_t t, int32_t deletes) {
   return deletes ? g->d_off[t + 1] - g->d_off[t] : g->a_off[t + 1] - g->a_off[t];
 }
 
+}  // extern "C"
+
+namespace stg {
+bool dtdg_materialised(const stg_dtdg* g) { return g && !g->naive.empty(); }
+}  // namespace stg
+
+extern "C" {
+
 stg_status stg_dtdg_memory(const stg_dtdg* g, int64_t* deltas, int64_t* cache, int64_t* materialised) {
   if (!g || !deltas || !cache || !materialised) return fail(STG_ERR_INVALID_ARG, "stg_dtdg_memory: NULL argument");
   const DArray<uint64_t>* d[] = {&g->add_out, &g->add_in, &g->del_out, &g->del_in, &g->gadd, &g->gdel};

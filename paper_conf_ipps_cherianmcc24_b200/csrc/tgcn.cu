@@ -16,6 +16,7 @@
 #include "graph.cuh"
 
 namespace stg {
+bool dtdg_materialised(const stg_dtdg* g);
 bool tc_supported(int F, int H);
 int tc_atb_max_blocks();
 stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s,
@@ -930,6 +931,15 @@ bool pipeline_enabled() {
   }();
   return on;
 }
+// compute on an aux stream beside the H chain (1, default) or on the caller's
+// stream with only the snapshot builds overlapped (0)
+bool aux_stream_enabled() {
+  static const bool on = [] {
+    const char* v = getenv("STG_AUX_STREAM");
+    return !(v && v[0] == '0');
+  }();
+  return on;
+}
 }  // namespace
 
 // Algorithm 1 for one sequence, scheduled over three streams (streams instead of
@@ -970,7 +980,18 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
   const size_t VH = (size_t)V * H;
   cudaStream_t ms = (cudaStream_t)stream;
   const bool pipe = pipeline_enabled();
-  cudaStream_t as = pipe ? side_stream(1) : ms;
+  // With every snapshot materialised (STG_NAIVE) there are no builds to hide: HBM-bound
+  // steps (P' larger than L2) then run faster one at a time (C5: 112.6 vs 140.6 ms per
+  // epoch), L2-resident ones still gain from the overlap (C4: 10.9 vs 11.9 ms;
+  // profiles/r01_table3_naive_vs_ondemand.jsonl)
+  static const int l2_bytes = [] {
+    int dev = 0, b = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&b, cudaDevAttrL2CacheSize, dev);
+    return b;
+  }();
+  const bool hbm_bound = (double)Vall * 3 * H * sizeof(float) > (double)l2_bytes;
+  cudaStream_t as = (pipe && aux_stream_enabled() && !(dtdg_materialised(dtdg) && hbm_bound)) ? side_stream(1) : ms;
   cudaStream_t ss = (dtdg && pipe) ? side_stream(0) : ms;
   // every buffer is sized before any asynchronous use (grow-only reallocations
   // would free memory another stream may still read)
