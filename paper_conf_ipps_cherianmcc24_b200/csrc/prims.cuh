@@ -136,7 +136,7 @@ stg_status scan(In in, Out out, int64_t n, ScanWs& ws, cudaStream_t s, int64_t* 
 // ------------------------------------------------------------- radix sort
 constexpr int kRadixThreads = 256;
 constexpr int kRadixWarps = kRadixThreads / 32;
-constexpr int kRadixIPT = 16;                                // items per lane
+constexpr int kRadixIPT = 8;                                 // items per lane
 constexpr int kRadixWarpItems = 32 * kRadixIPT;              // 512
 constexpr int kRadixTile = kRadixWarpItems * kRadixWarps;    // 4096
 constexpr int kRadixBits = 8;
@@ -149,9 +149,14 @@ __global__ void __launch_bounds__(kRadixThreads) k_radix_hist(const K* __restric
   for (int d = threadIdx.x; d < kRadixDigits; d += kRadixThreads) h[d] = 0;
   __syncthreads();
   const int64_t base = (int64_t)blockIdx.x * kRadixTile;
+  const int lane = threadIdx.x & 31;
+  // warp-aggregated: one shared atomic per distinct digit per warp (skewed keys such
+  // as vertex degrees would otherwise serialise on a few counters)
   for (int k = threadIdx.x; k < kRadixTile; k += kRadixThreads) {
-    int64_t i = base + k;
-    if (i < n) atomicAdd(&h[(int)((keys[i] >> shift) & (kRadixDigits - 1))], 1);
+    const int64_t i = base + k;
+    const int d = i < n ? (int)((keys[i] >> shift) & (kRadixDigits - 1)) : kRadixDigits + lane;
+    const unsigned peers = __match_any_sync(0xffffffffu, d);
+    if (d < kRadixDigits && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&h[d], __popc(peers));
   }
   __syncthreads();
   for (int d = threadIdx.x; d < kRadixDigits; d += kRadixThreads) counts[(int64_t)d * ntiles + blockIdx.x] = h[d];
