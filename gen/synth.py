@@ -336,3 +336,16 @@ def tgcn_params(F: int, H: int, seed: int, scale: float = 1.0):
 def edge_weights(seed: int, n: int, lo: float = 0.5, hi: float = 2.0, stream: int = 40) -> np.ndarray:
     """n seeded positive edge weights in [lo, hi) (NEXT-4 inputs), multiples of 2^-24 scaled."""
     return (lo + (hi - lo) * uniform_01(seed, stream, n)).astype(np.float32)
+
+
+def tgcn2_params(F: int, H: int, seed: int, scale: float = 1.0):
+    """Original T-GCN cell parameters (NEXT-2): Wg [F+H, 2H] (r | u), bg [2H], Wc [F+H, H],
+    bc [H], U[±1/sqrt(fan_in)], plus the surrogate head w_o [H], b_o [1]."""
+    K = F + H
+    a = scale / np.sqrt(K)
+
+    def u(stream, n, bound):
+        return (uniform_pm1(seed, stream, n) * np.float32(bound)).astype(np.float32)
+    return {"Wg": u(81, K * 2 * H, a).reshape(K, 2 * H), "bg": u(82, 2 * H, a),
+            "Wc": u(83, K * H, a).reshape(K, H), "bc": u(84, H, a),
+            "w_o": u(85, H, scale / np.sqrt(H)), "b_o": u(86, 1, scale / np.sqrt(H))}

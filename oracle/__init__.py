@@ -63,6 +63,10 @@ def lib():
         _lib.orc_tgcn_fwd.argtypes = [i32, i32, i32] + [P] * 15
         _lib.orc_tgcn_bwd.restype = None
         _lib.orc_tgcn_bwd.argtypes = [i32, i32, i32] + [P] * 17
+        _lib.orc_tgcn2_fwd.restype = None
+        _lib.orc_tgcn2_fwd.argtypes = [i32, i32, i32] + [P] * 14
+        _lib.orc_tgcn2_bwd.restype = None
+        _lib.orc_tgcn2_bwd.argtypes = [i32, i32, i32] + [P] * 19
         _lib.orc_mse_head.restype = ctypes.c_double
         _lib.orc_mse_head.argtypes = [i32, i32, P, P, P, ctypes.c_double, P, P, P]
     return _lib
@@ -306,4 +310,68 @@ def train_sequence(graphs_fwd, graphs_bwd, p: dict, Xs, Ys, H0):
         Hp, f = stack.pop()
         G = f["dH_head"] + Gnext
         Gnext = tgcn_bwd(graphs_bwd[i], p, Xs[i], Hp, f, G, grads)
+    return loss, grads, Hc
+
+
+# ------------------------------------------------------ original T-GCN (NEXT-2)
+def tgcn2_fwd(g: dict, p: dict, X, Hp) -> dict:
+    """Original T-GCN cell (GCN over [X, H], aggregate-first as written; NEXT-2)."""
+    V, F = X.shape
+    H = Hp.shape[1]
+    X, Hp = _c(X, np.float64), _c(Hp, np.float64)
+    Wg, bg, Wc, bc = (_c(p[k], np.float64) for k in ("Wg", "bg", "Wc", "bc"))
+    out = {k: np.zeros((V, H), np.float64) for k in ("R", "U", "Cc", "Hn")}
+    ns, nd = _c(g["norm_src"], np.float64), _c(g["norm_dst"], np.float64)
+    col = g["in_col"] if g["in_col"].size else np.zeros(1, np.int32)
+    lib().orc_tgcn2_fwd(V, F, H, _p(_c(g["in_rowptr"], np.int32)), _p(_c(col, np.int32)), _p(ns), _p(nd),
+                        _p(X), _p(Hp), _p(Wg), _p(bg), _p(Wc), _p(bc),
+                        _p(out["R"]), _p(out["U"]), _p(out["Cc"]), _p(out["Hn"]))
+    return out
+
+
+def zero_grads2(F: int, H: int) -> dict:
+    return {"Wg": np.zeros((F + H, 2 * H)), "bg": np.zeros(2 * H), "Wc": np.zeros((F + H, H)),
+            "bc": np.zeros(H), "w_o": np.zeros(H), "b_o": np.zeros(1)}
+
+
+def tgcn2_bwd(g: dict, p: dict, X, Hp, fwd: dict, G, grads: dict) -> np.ndarray:
+    """Accumulates into grads (float64 arrays); returns dH_{t-1}."""
+    V, F = X.shape
+    H = Hp.shape[1]
+    X, Hp, G = _c(X, np.float64), _c(Hp, np.float64), _c(G, np.float64)
+    dHp = np.zeros((V, H), np.float64)
+    ns, nd = _c(g["norm_src"], np.float64), _c(g["norm_dst"], np.float64)
+    icol = g["in_col"] if g["in_col"].size else np.zeros(1, np.int32)
+    ocol = g["out_col"] if g["out_col"].size else np.zeros(1, np.int32)
+    for k in ("Wg", "bg", "Wc", "bc"):
+        assert grads[k].dtype == np.float64 and grads[k].flags.c_contiguous
+    lib().orc_tgcn2_bwd(V, F, H, _p(_c(g["in_rowptr"], np.int32)), _p(_c(icol, np.int32)),
+                        _p(_c(g["out_rowptr"], np.int32)), _p(_c(ocol, np.int32)), _p(ns), _p(nd),
+                        _p(X), _p(Hp), _p(_c(p["Wg"], np.float64)), _p(_c(p["Wc"], np.float64)),
+                        _p(_c(fwd["R"], np.float64)), _p(_c(fwd["U"], np.float64)), _p(_c(fwd["Cc"], np.float64)),
+                        _p(G), _p(dHp), _p(grads["Wg"]), _p(grads["bg"]), _p(grads["Wc"]), _p(grads["bc"]))
+    return dHp
+
+
+def train_sequence2(graphs, p: dict, Xs, Ys, H0):
+    """Algorithm 1 for one sequence with the original T-GCN cell (NEXT-2), fp64.
+    Returns (sum of losses, grads, H_last)."""
+    S = len(Xs)
+    F = Xs[0].shape[1]
+    H = H0.shape[1]
+    grads = zero_grads2(F, H)
+    stack = []
+    Hc = np.asarray(H0, np.float64)
+    loss = 0.0
+    for i in range(S):
+        f = tgcn2_fwd(graphs[i], p, Xs[i], Hc)
+        stack.append((Hc, f))
+        l_i, _ = mse_head(f["Hn"], Ys[i], p["w_o"], p["b_o"], {"w_o": np.zeros(H), "b_o": np.zeros(1)})
+        loss += l_i
+        Hc = f["Hn"]
+    dH = np.zeros_like(Hc)
+    for i in range(S - 1, -1, -1):
+        Hp, f = stack.pop()
+        _, dh_head = mse_head(f["Hn"], Ys[i], p["w_o"], p["b_o"], grads)
+        dH = tgcn2_bwd(graphs[i], p, Xs[i], Hp, f, dH + dh_head, grads)
     return loss, grads, Hc

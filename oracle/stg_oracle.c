@@ -405,3 +405,133 @@ double orc_mse_head(int32_t V, int32_t H, const double* Hn, const double* y,
   }
   return loss / (double)V;
 }
+
+/* ---------------------------------------------------------------------------
+ * Original T-GCN cell (the model the paper cites for TGCN,
+ * P:L58, whose graph convolution acts on the concatenation [X, H] — reading C13
+ * alternative).  Written in the order of that formulation (aggregate first):
+ *   XH  = [X | H]                      [V, F+H]
+ *   G   = (Â·XH)·Wg + bg               Wg [F+H, 2H] (columns r | u)
+ *   r   = σ(G[:, :H]),  u = σ(G[:, H:])
+ *   XR  = [X | r⊙H]
+ *   Cc  = tanh((Â·XR)·Wc + bc)         Wc [F+H, H]
+ *   H'  = u⊙H + (1−u)⊙Cc
+ * Â_vu = n_dst[v]·n_src[u] over the in-CSR (the same GCN normalisation, C1).
+ * Outputs R, U, Cc, Hn [V,H].  fp64, row-major.
+ * ------------------------------------------------------------------------- */
+static void cat_rows(int32_t V, int32_t F, int32_t H, const double* X, const double* Hm, const double* mul,
+                     double* out) {
+  for (int32_t v = 0; v < V; ++v) {
+    for (int32_t f = 0; f < F; ++f) out[(int64_t)v * (F + H) + f] = X[(int64_t)v * F + f];
+    for (int32_t j = 0; j < H; ++j)
+      out[(int64_t)v * (F + H) + F + j] = Hm[(int64_t)v * H + j] * (mul ? mul[(int64_t)v * H + j] : 1.0);
+  }
+}
+
+static void matmul(int32_t V, int32_t K, int32_t N, const double* A, const double* W, const double* bias,
+                   double* out) {
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t c = 0; c < N; ++c) {
+      double s = bias ? bias[c] : 0.0;
+      for (int32_t k = 0; k < K; ++k) s += A[(int64_t)v * K + k] * W[(int64_t)k * N + c];
+      out[(int64_t)v * N + c] = s;
+    }
+}
+
+void orc_tgcn2_fwd(int32_t V, int32_t F, int32_t H, const int32_t* in_rowptr, const int32_t* in_col,
+                   const double* n_src, const double* n_dst, const double* X, const double* Hp,
+                   const double* Wg, const double* bg, const double* Wc, const double* bc,
+                   double* R, double* U, double* Cc, double* Hn) {
+  const int32_t K = F + H;
+  double* cat = (double*)malloc(sizeof(double) * ((size_t)V * K + 1));
+  double* agg = (double*)malloc(sizeof(double) * ((size_t)V * K + 1));
+  double* G = (double*)malloc(sizeof(double) * ((size_t)V * 2 * H + 1));
+  cat_rows(V, F, H, X, Hp, NULL, cat);
+  orc_aggregate(V, in_rowptr, in_col, n_dst, n_src, K, cat, agg);
+  matmul(V, K, 2 * H, agg, Wg, bg, G);
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t j = 0; j < H; ++j) {
+      R[(int64_t)v * H + j] = sigm(G[(int64_t)v * 2 * H + j]);
+      U[(int64_t)v * H + j] = sigm(G[(int64_t)v * 2 * H + H + j]);
+    }
+  cat_rows(V, F, H, X, Hp, R, cat);
+  orc_aggregate(V, in_rowptr, in_col, n_dst, n_src, K, cat, agg);
+  matmul(V, K, H, agg, Wc, bc, Cc);
+  for (int64_t i = 0; i < (int64_t)V * H; ++i) {
+    Cc[i] = tanh(Cc[i]);
+    Hn[i] = U[i] * Hp[i] + (1.0 - U[i]) * Cc[i];
+  }
+  free(cat); free(agg); free(G);
+}
+
+/* Backward of orc_tgcn2_fwd by the chain rule, given G = dℓ/dH' (total):
+ *   du = G⊙(H−Cc); dCc = G⊙(1−u); dH = G⊙u
+ *   dzc = dCc⊙(1−Cc²);  dWc += (Â·XR)ᵀ dzc;  dbc += 1ᵀdzc
+ *   dXR = Âᵀ·(dzc·Wcᵀ);  d(r⊙H) = dXR[:, F:];  dr = d(r⊙H)⊙H;  dH += d(r⊙H)⊙r
+ *   dzg = [dr⊙r(1−r) | du⊙u(1−u)];  dWg += (Â·XH)ᵀ dzg;  dbg += 1ᵀdzg
+ *   dXH = Âᵀ·(dzg·Wgᵀ);  dH += dXH[:, F:]
+ * Âᵀ runs over the out-CSR (rows = sources; ncol = n_dst of the destinations).
+ * Gradients accumulate (+=); dHp is overwritten. */
+void orc_tgcn2_bwd(int32_t V, int32_t F, int32_t H, const int32_t* in_rowptr, const int32_t* in_col,
+                   const int32_t* out_rowptr, const int32_t* out_col, const double* n_src, const double* n_dst,
+                   const double* X, const double* Hp, const double* Wg, const double* Wc, const double* R,
+                   const double* U, const double* Cc, const double* Gd, double* dHp, double* dWg, double* dbg,
+                   double* dWc, double* dbc) {
+  const int32_t K = F + H, H2 = 2 * H;
+  double* cat = (double*)malloc(sizeof(double) * ((size_t)V * K + 1));
+  double* agg = (double*)malloc(sizeof(double) * ((size_t)V * K + 1));
+  double* dz = (double*)calloc((size_t)V * H2 + 1, sizeof(double));
+  double* dcat = (double*)malloc(sizeof(double) * ((size_t)V * K + 1));
+  double* dxr = (double*)malloc(sizeof(double) * ((size_t)V * K + 1));
+  double* du = (double*)malloc(sizeof(double) * ((size_t)V * H + 1));
+  for (int64_t i = 0; i < (int64_t)V * H; ++i) {
+    du[i] = Gd[i] * (Hp[i] - Cc[i]);
+    dz[i] = Gd[i] * (1.0 - U[i]) * (1.0 - Cc[i] * Cc[i]);      /* dzc, [V,H] */
+    dHp[i] = Gd[i] * U[i];
+  }
+  /* candidate: dWc, dbc, dXR */
+  cat_rows(V, F, H, X, Hp, R, cat);
+  orc_aggregate(V, in_rowptr, in_col, n_dst, n_src, K, cat, agg);
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t c = 0; c < H; ++c) {
+      const double d = dz[(int64_t)v * H + c];
+      dbc[c] += d;
+      for (int32_t k = 0; k < K; ++k) dWc[(int64_t)k * H + c] += agg[(int64_t)v * K + k] * d;
+    }
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t k = 0; k < K; ++k) {
+      double s = 0.0;
+      for (int32_t c = 0; c < H; ++c) s += dz[(int64_t)v * H + c] * Wc[(int64_t)k * H + c];
+      dcat[(int64_t)v * K + k] = s;
+    }
+  orc_aggregate(V, out_rowptr, out_col, n_src, n_dst, K, dcat, dxr);
+  double* dzg = (double*)calloc((size_t)V * H2 + 1, sizeof(double));
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t j = 0; j < H; ++j) {
+      const int64_t i = (int64_t)v * H + j;
+      const double drh = dxr[(int64_t)v * K + F + j];
+      const double dr = drh * Hp[i];
+      dHp[i] += drh * R[i];
+      dzg[(int64_t)v * H2 + j] = dr * R[i] * (1.0 - R[i]);
+      dzg[(int64_t)v * H2 + H + j] = du[i] * U[i] * (1.0 - U[i]);
+    }
+  /* gates: dWg, dbg, dXH */
+  cat_rows(V, F, H, X, Hp, NULL, cat);
+  orc_aggregate(V, in_rowptr, in_col, n_dst, n_src, K, cat, agg);
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t c = 0; c < H2; ++c) {
+      const double d = dzg[(int64_t)v * H2 + c];
+      dbg[c] += d;
+      for (int32_t k = 0; k < K; ++k) dWg[(int64_t)k * H2 + c] += agg[(int64_t)v * K + k] * d;
+    }
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t k = 0; k < K; ++k) {
+      double s = 0.0;
+      for (int32_t c = 0; c < H2; ++c) s += dzg[(int64_t)v * H2 + c] * Wg[(int64_t)k * H2 + c];
+      dcat[(int64_t)v * K + k] = s;
+    }
+  orc_aggregate(V, out_rowptr, out_col, n_src, n_dst, K, dcat, dxr);
+  for (int32_t v = 0; v < V; ++v)
+    for (int32_t j = 0; j < H; ++j) dHp[(int64_t)v * H + j] += dxr[(int64_t)v * K + F + j];
+  free(cat); free(agg); free(dz); free(dcat); free(dxr); free(du); free(dzg);
+}
