@@ -283,6 +283,27 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g_bwd, const stg_tgcn_para
                                   const float* dH_next, float* dH_prev, stg_tgcn_grads* grads,
                                   stg_state_stack* stack, stg_stream_t stream);
 
+/* ---- original T-GCN cell (the model cited at P:L58, whose
+ * graph convolution acts on [X, H]; oracle orc_tgcn2_fwd/bwd):
+ *   [r | u] = σ(Â([X, H]·Wg) + bg),  c = tanh(Â([X, r⊙H]·Wc) + bc),  H' = u⊙H + (1−u)⊙c
+ * Wg [F+H, 2H] (columns r | u), bg [2H], Wc [F+H, H], bc [H]; X [V,F], H [V,H].
+ * Two aggregations per step (widths 2H and H) sit on the recurrent path; the
+ * backward runs two over the out-CSR.  Unsharded views; H in {4,8,16,32,64}.
+ * The state stack saves [r | u | c] per step (H_prev by reference, as stg_tgcn_step);
+ * gradients accumulate (+=), dH_prev is overwritten. */
+typedef struct {
+  int32_t F, H;
+  const float *Wg, *bg, *Wc, *bc;
+} stg_tgcn2_params;
+typedef struct {
+  float *Wg, *bg, *Wc, *bc;
+} stg_tgcn2_grads;
+stg_status stg_tgcn2_step(const stg_csr_view* g, const stg_tgcn2_params* p, const float* X, const float* H_prev,
+                          float* H_next, stg_state_stack* stack, stg_stream_t stream);
+stg_status stg_tgcn2_step_backward(const stg_csr_view* g, const stg_tgcn2_params* p, const float* X,
+                                   const float* dH_next, float* dH_prev, stg_tgcn2_grads* grads,
+                                   stg_state_stack* stack, stg_stream_t stream);
+
 /* Surrogate MSE head (timing only; A15): ŷ_v = Σ_k ReLU(H_vk)·w_o[k] + b_o[0],
  *   ℓ = mean_v (ŷ_v − y_v)².
  * loss_accum (device scalar, may be NULL) += ℓ.  If dH != NULL: dH (+)= dℓ/dH

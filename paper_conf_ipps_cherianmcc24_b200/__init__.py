@@ -76,6 +76,14 @@ class stg_tgcn_grads(ctypes.Structure):
     _fields_ = [("W", _P), ("b", _P), ("L", _P), ("l", _P)]
 
 
+class stg_tgcn2_params(ctypes.Structure):
+    _fields_ = [("F", _i32), ("H", _i32), ("Wg", _P), ("bg", _P), ("Wc", _P), ("bc", _P)]
+
+
+class stg_tgcn2_grads(ctypes.Structure):
+    _fields_ = [("Wg", _P), ("bg", _P), ("Wc", _P), ("bc", _P)]
+
+
 _lib = ctypes.CDLL(LIB_PATH)
 
 
@@ -129,6 +137,9 @@ _decl("stg_profile_read", [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER
 _decl("stg_gcn_aggregate_weighted", [ctypes.POINTER(stg_csr_view), _i32, _i32, _P, _P, _i64, _P, _i64, _P, _P, _P,
                                      _P])
 _decl("stg_gcn_weighted_norm", [ctypes.POINTER(stg_csr_view), _P, _P, _P])
+_decl("stg_tgcn2_step", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn2_params), _P, _P, _P, _P, _P])
+_decl("stg_tgcn2_step_backward", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn2_params), _P, _P, _P,
+                                  ctypes.POINTER(stg_tgcn2_grads), _P, _P])
 _decl("stg_peer_alloc", [_i64, ctypes.POINTER(_P), ctypes.POINTER(stg_ipc_handle)])
 _decl("stg_peer_free", [_P])
 _decl("stg_peer_open", [ctypes.POINTER(stg_ipc_handle), ctypes.POINTER(_P)])
@@ -156,7 +167,7 @@ ABI_SYMBOLS = [
     "stg_tgcn_train_sequence_batched",
     "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
-    "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm",
+    "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm", "stg_tgcn2_step", "stg_tgcn2_step_backward",
     "stg_peer_alloc", "stg_peer_free", "stg_peer_open", "stg_peer_close", "stg_allgather_rows",
     "stg_gcn_aggregate_peer", "stg_reduce_scatter_rows", "stg_tgcn_project", "stg_tgcn_step_peer",
     "stg_tgcn_step_backward_peer", "stg_tgcn_dw",
@@ -466,6 +477,33 @@ def stg_tgcn_step_backward(v: stg_csr_view, params: dict, X, dH_next, grads: dic
     G = make_grads(grads)
     _check(_lib.stg_tgcn_step_backward(ctypes.byref(v), ctypes.byref(P), _ptr(X), _ptr(dH_next), _ptr(dH_prev),
                                        ctypes.byref(G), stack.handle, _stream(stream)))
+    return dH_prev
+
+
+def make_params2(p: dict) -> stg_tgcn2_params:
+    K, H2 = p["Wg"].shape
+    H = H2 // 2
+    return stg_tgcn2_params(K - H, H, _ptr(p["Wg"]), _ptr(p["bg"]), _ptr(p["Wc"]), _ptr(p["bc"]))
+
+
+def stg_tgcn2_step(v: stg_csr_view, params: dict, X, H_prev, H_next=None, stack: StateStack = None, stream=None):
+    """Original T-GCN cell (NEXT-2): GCN over [X, H]."""
+    if H_next is None:
+        H_next = torch.empty_like(H_prev)
+    P = make_params2(params)
+    _check(_lib.stg_tgcn2_step(ctypes.byref(v), ctypes.byref(P), _ptr(X), _ptr(H_prev), _ptr(H_next),
+                               stack.handle if stack else None, _stream(stream)))
+    return H_next
+
+
+def stg_tgcn2_step_backward(v: stg_csr_view, params: dict, X, dH_next, grads: dict, stack: StateStack,
+                            dH_prev=None, stream=None):
+    if dH_prev is None:
+        dH_prev = torch.empty_like(dH_next)
+    P = make_params2(params)
+    G = stg_tgcn2_grads(_ptr(grads["Wg"]), _ptr(grads["bg"]), _ptr(grads["Wc"]), _ptr(grads["bc"]))
+    _check(_lib.stg_tgcn2_step_backward(ctypes.byref(v), ctypes.byref(P), _ptr(X), _ptr(dH_next), _ptr(dH_prev),
+                                        ctypes.byref(G), stack.handle, _stream(stream)))
     return dH_prev
 
 

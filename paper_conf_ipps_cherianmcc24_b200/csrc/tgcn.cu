@@ -455,6 +455,188 @@ __global__ void k_seq_gather(const SeqPtrs ptrs, int S, int V, int F, const floa
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < S * H3; e += gridDim.x * blockDim.x) b_all[e] = b[e % H3];
 }
 
+// ---------------------------------------------------------------- original T-GCN (NEXT-2)
+// The cell convolves [X, H] (orc_tgcn2_fwd): per timestep two
+// linear-first graph convolutions Â([X,H]Wg) + bg (width 2H) and Â([X, r⊙H]Wc) + bc
+// (width H) around the gates.  SIMT kernels: the dense parts are small (K = F+H,
+// N <= 2H) and the aggregations run in the library's aggregation kernels.
+
+// out[r, c] (+)= rs[r] · Σ_k A[r, k] · W(k, c) with A = [A1 (K1 cols) | A2 (K2 cols)]
+// and W(k, c) = W[k·sk + c·sn] (a transposed slice is just other strides).  32-row
+// tiles in shared memory; a thread computes 4 consecutive columns of one row.
+__global__ void __launch_bounds__(kT) k_cat_mm(int32_t V, const float* __restrict__ A1, int32_t K1, int64_t ld1,
+                                               const float* __restrict__ A2, int32_t K2, int64_t ld2,
+                                               const float* __restrict__ W, int64_t sk, int64_t sn, int32_t N,
+                                               const float* __restrict__ rs, float* __restrict__ out, int64_t ldo,
+                                               int accumulate) {
+  extern __shared__ float sm[];
+  constexpr int BR = 32;
+  const int K = K1 + K2, KP = K + 1;
+  float* sW = sm;                 // [K][N]
+  float* sA = sm + K * N;         // [BR][K+1]
+  for (int i = threadIdx.x; i < K * N; i += kT) sW[i] = W[(int64_t)(i / N) * sk + (int64_t)(i % N) * sn];
+  const int NG = N / 4;
+  const int64_t ntiles = (V + BR - 1) / BR;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * BR;
+    __syncthreads();
+    for (int i = threadIdx.x; i < BR * K; i += kT) {
+      const int r = i / K, k = i % K;
+      const int64_t row = r0 + r;
+      float v = 0.0f;
+      if (row < V) v = k < K1 ? A1[row * ld1 + k] : A2[row * ld2 + (k - K1)];
+      sA[r * KP + k] = v;
+    }
+    __syncthreads();
+    for (int o = threadIdx.x; o < BR * NG; o += kT) {
+      const int r = o / NG, c = 4 * (o % NG);
+      const int64_t row = r0 + r;
+      if (row >= V) continue;
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      const float* ar = sA + r * KP;
+      for (int k = 0; k < K; ++k) {
+        const float a = ar[k];
+        const float4 w = *reinterpret_cast<const float4*>(sW + k * N + c);
+        acc.x = fmaf(a, w.x, acc.x); acc.y = fmaf(a, w.y, acc.y);
+        acc.z = fmaf(a, w.z, acc.z); acc.w = fmaf(a, w.w, acc.w);
+      }
+      const float sc = rs ? rs[row] : 1.0f;
+      float* o4 = out + row * ldo + c;
+      if (accumulate) {
+        o4[0] += sc * acc.x; o4[1] += sc * acc.y; o4[2] += sc * acc.z; o4[3] += sc * acc.w;
+      } else {
+        o4[0] = sc * acc.x; o4[1] = sc * acc.y; o4[2] = sc * acc.z; o4[3] = sc * acc.w;
+      }
+    }
+  }
+}
+
+// part[b][k][c] = Σ_{rows of block b} A[r, k] · B[r, c], A = [A1 | A2]; B [V, N] (ld N).
+// Fixed row order per block; k_reduce_part adds the block partials in a fixed order.
+__global__ void __launch_bounds__(kT) k_cat_atb(int32_t V, const float* __restrict__ A1, int32_t K1,
+                                                const float* __restrict__ A2, int32_t K2,
+                                                const float* __restrict__ B, int32_t N, float* __restrict__ part) {
+  extern __shared__ float sm[];
+  constexpr int BR = 32;
+  const int K = K1 + K2;
+  float* sA = sm;                 // [BR][K]
+  float* sB = sA + BR * K;        // [BR][N]
+  float* sAcc = sB + BR * N;      // [K][N]
+  for (int i = threadIdx.x; i < K * N; i += kT) sAcc[i] = 0.0f;
+  const int NG = N / 4;
+  const int64_t ntiles = (V + BR - 1) / BR;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * BR;
+    __syncthreads();
+    for (int i = threadIdx.x; i < BR * K; i += kT) {
+      const int r = i / K, k = i % K;
+      const int64_t row = r0 + r;
+      sA[i] = row < V ? (k < K1 ? A1[row * K1 + k] : A2[row * K2 + (k - K1)]) : 0.0f;
+    }
+    for (int i = threadIdx.x; i < BR * N; i += kT) {
+      const int64_t row = r0 + i / N;
+      sB[i] = row < V ? B[row * N + i % N] : 0.0f;
+    }
+    __syncthreads();
+    const int nrows = (int)(V - r0 < BR ? V - r0 : BR);
+    for (int e = threadIdx.x; e < K * NG; e += kT) {
+      const int k = e / NG, c = 4 * (e % NG);
+      float4 acc = *reinterpret_cast<float4*>(sAcc + k * N + c);
+      for (int r = 0; r < nrows; ++r) {
+        const float a = sA[r * K + k];
+        const float4 b = *reinterpret_cast<const float4*>(sB + r * N + c);
+        acc.x = fmaf(a, b.x, acc.x); acc.y = fmaf(a, b.y, acc.y);
+        acc.z = fmaf(a, b.z, acc.z); acc.w = fmaf(a, b.w, acc.w);
+      }
+      *reinterpret_cast<float4*>(sAcc + k * N + c) = acc;
+    }
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < K * N; e += kT) part[(int64_t)blockIdx.x * K * N + e] = sAcc[e];
+}
+
+// part[b][c] = Σ_{rows of block b} D[r, c] (fixed order: thread slices, then a fixed tree)
+__global__ void __launch_bounds__(kT) k_colsum_part(int32_t V, const float* __restrict__ D, int32_t N,
+                                                    float* __restrict__ part) {
+  __shared__ float red[kT];
+  const int slices = kT / N;                       // N divides kT (N = H or 2H, powers of two)
+  const int c = threadIdx.x % N, sl = threadIdx.x / N;
+  float acc = 0.0f;
+  if (sl < slices)
+    for (int64_t r = (int64_t)blockIdx.x * slices + sl; r < V; r += (int64_t)gridDim.x * slices)
+      acc += D[r * N + c];
+  red[threadIdx.x] = acc;
+  __syncthreads();
+  if (threadIdx.x < N) {
+    float t = 0.0f;
+    for (int q = 0; q < slices; ++q) t += red[q * N + threadIdx.x];
+    part[(int64_t)blockIdx.x * N + threadIdx.x] = t;
+  }
+}
+
+__device__ __forceinline__ float t2_sig(float a) { return 1.0f / (1.0f + expf(-a)); }
+
+// r = σ(A[:, :H]), u = σ(A[:, H:]) -> RUC[:, 0:H), [H:2H); rH = r ⊙ Hp
+__global__ void k_t2_gates(int32_t V, int32_t H, const float* __restrict__ A, const float* __restrict__ Hp,
+                           float* __restrict__ RUC, float* __restrict__ rH) {
+  const int64_t n = (int64_t)V * H;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = i / H;
+    const int j = (int)(i % H);
+    const float r = t2_sig(A[v * 2 * H + j]), u = t2_sig(A[v * 2 * H + H + j]);
+    RUC[v * 3 * H + j] = r;
+    RUC[v * 3 * H + H + j] = u;
+    rH[i] = r * Hp[i];
+  }
+}
+
+// c = tanh(A) -> RUC[:, 2H:3H);  H' = u ⊙ Hp + (1 − u) ⊙ c
+__global__ void k_t2_cand(int32_t V, int32_t H, const float* __restrict__ A, const float* __restrict__ Hp,
+                          float* __restrict__ RUC, float* __restrict__ Hn) {
+  const int64_t n = (int64_t)V * H;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = i / H;
+    const int j = (int)(i % H);
+    const float c = tanhf(A[i]);
+    const float u = RUC[v * 3 * H + H + j];
+    RUC[v * 3 * H + 2 * H + j] = c;
+    Hn[i] = u * Hp[i] + (1.0f - u) * c;
+  }
+}
+
+// du = G ⊙ (Hp − c); dAc = G ⊙ (1 − u) ⊙ (1 − c²); dHp = G ⊙ u; rH = r ⊙ Hp
+__global__ void k_t2_cand_bwd(int32_t V, int32_t H, const float* __restrict__ G, const float* __restrict__ Hp,
+                              const float* __restrict__ RUC, float* __restrict__ dAc, float* __restrict__ du,
+                              float* __restrict__ dHp, float* __restrict__ rH) {
+  const int64_t n = (int64_t)V * H;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = i / H;
+    const int j = (int)(i % H);
+    const float r = RUC[v * 3 * H + j], u = RUC[v * 3 * H + H + j], c = RUC[v * 3 * H + 2 * H + j];
+    const float g = G[i], h = Hp[i];
+    du[i] = g * (h - c);
+    dAc[i] = g * (1.0f - u) * (1.0f - c * c);
+    dHp[i] = g * u;
+    rH[i] = r * h;
+  }
+}
+
+// dr = d(rH) ⊙ Hp;  dHp += d(rH) ⊙ r;  dAg = [dr ⊙ r(1−r) | du ⊙ u(1−u)]
+__global__ void k_t2_gate_bwd(int32_t V, int32_t H, const float* __restrict__ drH, const float* __restrict__ Hp,
+                              const float* __restrict__ RUC, const float* __restrict__ du, float* __restrict__ dHp,
+                              float* __restrict__ dAg) {
+  const int64_t n = (int64_t)V * H;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = i / H;
+    const int j = (int)(i % H);
+    const float r = RUC[v * 3 * H + j], u = RUC[v * 3 * H + H + j];
+    const float d = drH[i];
+    dHp[i] += d * r;
+    dAg[v * 2 * H + j] = d * Hp[i] * r * (1.0f - r);
+    dAg[v * 2 * H + H + j] = du[i] * u * (1.0f - u);
+  }
+}
+
 int grid_blocks(const void* fn, size_t smem, int64_t tiles) {
   int per_sm = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kT, smem) != cudaSuccess || per_sm < 1) {
@@ -481,6 +663,8 @@ struct TgcnWs {
   // sequence-batched path: X_all, Y_all, b_all, then [V][S][·] activations and the head partials
   DArray<float> sX, sY, sb, sP, sC, sHp, sdC, sdP, sda, sRH, sgpart;
   DArray<double> slpart;
+  // original T-GCN (NEXT-2) scratch
+  DArray<float> t2z, t2a, t2b, t2c, t2d, t2part;
 };
 
 }  // namespace stg
@@ -833,6 +1017,138 @@ stg_status stg_tgcn_dw(const stg_tgcn_params* p, int32_t R, const float* X_loc, 
                                                      nullptr);
   count_launch(2);
   return check_launch("stg_tgcn_dw");
+}
+
+// ---- original T-GCN (NEXT-2) host side
+static stg_status t2_mm(int32_t V, const float* A1, int32_t K1, int64_t ld1, const float* A2, int32_t K2, int64_t ld2,
+                        const float* W, int64_t sk, int64_t sn, int32_t N, const float* rs, float* out, int64_t ldo,
+                        bool accumulate, cudaStream_t s) {
+  if (V == 0) return STG_OK;
+  const int K = K1 + K2;
+  const size_t smem = sizeof(float) * ((size_t)K * N + 32 * (size_t)(K + 1));
+  STG_TRY(set_smem(k_cat_mm, smem));
+  const int nb = grid_blocks((const void*)k_cat_mm, smem, (V + 31) / 32);
+  k_cat_mm<<<nb, kT, smem, s>>>(V, A1, K1, ld1, A2, K2, ld2, W, sk, sn, N, rs, out, ldo, accumulate ? 1 : 0);
+  count_launch();
+  return check_launch("tgcn2 mm");
+}
+
+// grad[K][N] += [A1 | A2]ᵀ B   (fixed-order partials)
+static stg_status t2_atb(int32_t V, const float* A1, int32_t K1, const float* A2, int32_t K2, const float* B,
+                         int32_t N, float* grad, TgcnWs& ws, cudaStream_t s) {
+  if (V == 0) return STG_OK;
+  const int K = K1 + K2;
+  const size_t smem = sizeof(float) * (32 * (size_t)K + 32 * (size_t)N + (size_t)K * N);
+  STG_TRY(set_smem(k_cat_atb, smem));
+  const int nb = grid_blocks((const void*)k_cat_atb, smem, (V + 31) / 32);
+  STG_TRY(ws.t2part.alloc((size_t)nb * K * N));
+  k_cat_atb<<<nb, kT, smem, s>>>(V, A1, K1, A2, K2, B, N, ws.t2part.p);
+  k_reduce_part<<<(K * N + 255) / 256, 256, 0, s>>>(ws.t2part.p, nb, K * N, grad, K * N, nullptr, 0, nullptr);
+  count_launch(2);
+  return check_launch("tgcn2 atb");
+}
+
+static stg_status t2_colsum(int32_t V, const float* D, int32_t N, float* grad, TgcnWs& ws, cudaStream_t s) {
+  if (V == 0) return STG_OK;
+  const int nb = (int)std::min<int64_t>((V + 63) / 64, (int64_t)num_sms() * 4);
+  STG_TRY(ws.t2part.alloc((size_t)nb * N));
+  k_colsum_part<<<nb, kT, 0, s>>>(V, D, N, ws.t2part.p);
+  k_reduce_part<<<(N + 255) / 256, 256, 0, s>>>(ws.t2part.p, nb, N, grad, N, nullptr, 0, nullptr);
+  count_launch(2);
+  return check_launch("tgcn2 colsum");
+}
+
+static unsigned t2_grid(int64_t n) { return (unsigned)std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 16); }
+
+static stg_status check_tgcn2(const stg_csr_view* g, const stg_tgcn2_params* p) {
+  if (!g || !p || !p->Wg || !p->bg || !p->Wc || !p->bc) return fail(STG_ERR_INVALID_ARG, "tgcn2: NULL argument");
+  if (p->F < 1 || p->H < 4 || p->H > 64 || p->H % 4 || (p->H & (p->H - 1)))
+    return fail(STG_ERR_INVALID_ARG, "tgcn2: need F >= 1 and H in {4, 8, 16, 32, 64} (H=%d)", p->H);
+  if ((size_t)(p->F + p->H) * 2 * p->H * 4 + 32 * (size_t)(p->F + p->H + 1) * 4 > 200 * 1024)
+    return fail(STG_ERR_INVALID_ARG, "tgcn2: F+H=%d too large for the shared-memory weights", p->F + p->H);
+  if (g->row_begin != 0 || g->row_end != g->num_nodes)
+    return fail(STG_ERR_INVALID_ARG, "tgcn2: sharded views are not supported");
+  return STG_OK;
+}
+
+static stg_status t2_ws(TgcnWs& ws, int32_t V, int32_t H) {
+  const size_t n2 = (size_t)V * 2 * H + 4, n1 = (size_t)V * H + 4;
+  STG_TRY(ws.t2z.alloc(n2)); STG_TRY(ws.t2a.alloc(n2)); STG_TRY(ws.t2b.alloc(n1));
+  STG_TRY(ws.t2c.alloc(n1)); STG_TRY(ws.t2d.alloc(n1));
+  return STG_OK;
+}
+
+stg_status stg_tgcn2_step(const stg_csr_view* g, const stg_tgcn2_params* p, const float* X, const float* H_prev,
+                          float* H_next, stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_tgcn2(g, p));
+  if (!X || !H_prev || !H_next) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_step: NULL argument");
+  cudaStream_t s = (cudaStream_t)stream;
+  const int32_t V = g->num_nodes, F = p->F, H = p->H, H2 = 2 * H;
+  TgcnWs& ws = stack ? stack->ws : global_ws();
+  STG_TRY(t2_ws(ws, V, H));
+  float* RUC = nullptr;                                   // [V,3H]: r | u | c, the saved state
+  const size_t need = stack_bytes(V, H);
+  if (stack) {
+    if (stack->top + need > stack->cap)
+      return fail(STG_ERR_NO_MEMORY, "stg_tgcn2_step: state stack full (%zu + %zu > %zu bytes)", stack->top, need,
+                  stack->cap);
+    RUC = reinterpret_cast<float*>(stack->arena.p + stack->top);
+  } else {
+    STG_TRY(ws.dC.alloc((size_t)V * 3 * H + 4));
+    RUC = ws.dC.p;
+  }
+  float *Z = ws.t2z.p, *A = ws.t2a.p, *rH = ws.t2b.p;
+  // gates: A = Â([X, H]·Wg) + bg  (P'-style: rows pre-scaled by n_src, n_dst per output row)
+  STG_TRY(t2_mm(V, X, F, F, H_prev, H, H, p->Wg, H2, 1, H2, g->norm_src, Z, H2, false, s));
+  STG_TRY(aggregate_launch(g, 0, H2, Z, H2, A, H2, g->norm_dst, nullptr, p->bg, s));
+  k_t2_gates<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, A, H_prev, RUC, rH);
+  count_launch();
+  // candidate: A = Â([X, r⊙H]·Wc) + bc
+  STG_TRY(t2_mm(V, X, F, F, rH, H, H, p->Wc, H, 1, H, g->norm_src, Z, H, false, s));
+  STG_TRY(aggregate_launch(g, 0, H, Z, H, A, H, g->norm_dst, nullptr, p->bc, s));
+  k_t2_cand<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, A, H_prev, RUC, H_next);
+  count_launch();
+  if (stack) {
+    stack->entries.push_back(StackEntry{H_prev, RUC, V, H, need});
+    stack->top += need;
+  }
+  return check_launch("stg_tgcn2_step");
+}
+
+stg_status stg_tgcn2_step_backward(const stg_csr_view* g, const stg_tgcn2_params* p, const float* X,
+                                   const float* dH_next, float* dH_prev, stg_tgcn2_grads* grads,
+                                   stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_tgcn2(g, p));
+  if (!X || !dH_next || !dH_prev || !grads || !stack || !grads->Wg || !grads->bg || !grads->Wc || !grads->bc)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_step_backward: NULL argument");
+  if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn2_step_backward: state stack is empty");
+  const StackEntry e = stack->entries.back();
+  const int32_t V = g->num_nodes, F = p->F, H = p->H, H2 = 2 * H;
+  if (e.V != V || e.H != H) return fail(STG_ERR_STATE, "stg_tgcn2_step_backward: stack top does not match (V,H)");
+  if (!g->out_rowptr) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_step_backward: view lacks the backward CSR");
+  cudaStream_t s = (cudaStream_t)stream;
+  TgcnWs& ws = stack->ws;
+  STG_TRY(t2_ws(ws, V, H));
+  const float* RUC = e.C;
+  const float* Hp = e.Hp;
+  float *dAg = ws.t2z.p, *Y = ws.t2a.p, *rH = ws.t2b.p, *D1 = ws.t2c.p, *du = ws.t2d.p;
+  k_t2_cand_bwd<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, dH_next, Hp, RUC, D1, du, dH_prev, rH);
+  count_launch();
+  // candidate convolution: dbc, dY = Âᵀ dAc, dWc += [X, r⊙H]ᵀ dY, d(r⊙H) = dY · Wc[F:, :]ᵀ
+  STG_TRY(t2_colsum(V, D1, H, grads->bc, ws, s));
+  STG_TRY(aggregate_launch(g, 1, H, D1, H, Y, H, g->norm_src, g->norm_dst, nullptr, s));
+  STG_TRY(t2_atb(V, X, F, rH, H, Y, H, grads->Wc, ws, s));
+  STG_TRY(t2_mm(V, Y, H, H, nullptr, 0, 0, p->Wc + (size_t)F * H, 1, H, H, nullptr, D1, H, false, s));
+  k_t2_gate_bwd<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, D1, Hp, RUC, du, dH_prev, dAg);
+  count_launch();
+  // gate convolution: dbg, dY = Âᵀ dAg, dWg += [X, H]ᵀ dY, dH += dY · Wg[F:, :]ᵀ
+  STG_TRY(t2_colsum(V, dAg, H2, grads->bg, ws, s));
+  STG_TRY(aggregate_launch(g, 1, H2, dAg, H2, Y, H2, g->norm_src, g->norm_dst, nullptr, s));
+  STG_TRY(t2_atb(V, X, F, Hp, H, Y, H2, grads->Wg, ws, s));
+  STG_TRY(t2_mm(V, Y, H2, H2, nullptr, 0, 0, p->Wg + (size_t)F * H2, 1, H2, H, nullptr, dH_prev, H, true, s));
+  stack->entries.pop_back();
+  stack->top -= e.bytes;
+  return check_launch("stg_tgcn2_step_backward");
 }
 
 stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o, const float* b_o,
