@@ -232,11 +232,18 @@ def main():
     sim = args.shard_sim is not None
     if sim:
         rank, world = (int(x) for x in args.shard_sim.split("/"))
+    # STG_BENCH_BACKEND=gloo: functional check of the N > 1 flow with every rank on the
+    # GPUs that exist (ranks share a device when there are fewer GPUs than ranks)
+    backend = os.environ.get("STG_BENCH_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     pg = world > 1 and not sim                  # a real process group (torchrun)
     peer = args.mode == "peer" and not sim
     if pg:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     elif peer:                                  # N=1 sharded mode: a one-rank group for the peer plumbing
         import socket
         with socket.socket() as sk:
