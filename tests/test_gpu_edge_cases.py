@@ -1,0 +1,114 @@
+"""Degenerate and boundary cases of the hot path (③: empty / ragged inputs, maximum
+sizes, the method's degenerate cases), each against the oracle or a closed form:
+* a DTDG with T = 1 (the base only) and one whose snapshot becomes EMPTY (every
+  edge deleted, no self-loops) and is rebuilt afterwards;
+* aggregation and a TGCN step on the empty snapshot (Â = 0, so C = b);
+* a one-vertex graph (V = 1) through graph build, aggregation and a TGCN step;
+* size limits: E >= 2^31 and V >= 2^30 rejected with STG_ERR_OUT_OF_RANGE before
+  any device work."""
+import ctypes
+
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from helpers import assert_graph_equal, to_gpu
+
+pytestmark = pytest.mark.gpu
+
+
+def _dtdg(stg, V, T, s0, d0, adds, dels, flags):
+    """adds/dels: list over t of (src, dst) lists; batch 0 empty."""
+    def pack(b):
+        off = [0]
+        ss, dd = [], []
+        for (s, d) in b:
+            ss += list(s)
+            dd += list(d)
+            off.append(len(ss))
+        return np.array(off, np.int64), np.array(ss, np.int32), np.array(dd, np.int32)
+    ao, a_s, a_d = pack(adds)
+    do, d_s, d_d = pack(dels)
+    return stg.stg_dtdg_create(V, T, s0, d0, ao, a_s, a_d, do, d_s, d_d, flags)
+
+
+def _oracle_sets(V, s0, d0, adds, dels):
+    S = oracle.edge_set(V, s0, d0)
+    out = [S]
+    for t in range(1, len(adds)):
+        A = oracle.keys(*adds[t]) if len(adds[t][0]) else np.zeros(0, np.uint64)
+        D = oracle.keys(*dels[t]) if len(dels[t][0]) else np.zeros(0, np.uint64)
+        S = oracle.set_apply(S, D, A)
+        out.append(S)
+    return out
+
+
+def test_dtdg_single_timestamp(stg):
+    V = 50
+    s, d = gen.random_edges(3, V, 120, loops=False)
+    g = _dtdg(stg, V, 1, s, d, [([], [])], [([], [])], stg.STG_EDGE_IDS)
+    ref = oracle.csr(V, oracle.edge_set(V, s, d))
+    assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_snapshot(g, 0)), ref, tag="T=1 fwd")
+    assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_backward_snapshot(g, 0)), ref, tag="T=1 bwd")
+
+
+def test_dtdg_snapshot_becomes_empty(stg):
+    V = 40
+    s, d = gen.random_edges(5, V, 90, loops=False)
+    S0 = oracle.edge_set(V, s, d)
+    us, ud = oracle.unkey(S0)
+    adds = [([], []), ([], []), (list(us[:30]), list(ud[:30]))]
+    dels = [([], []), (list(us), list(ud)), ([], [])]
+    g = _dtdg(stg, V, 3, s, d, adds, dels, stg.STG_EDGE_IDS)
+    sets = _oracle_sets(V, s, d, adds, dels)
+    assert sets[1].size == 0 and g.num_edges(1) == 0
+    for t in (0, 1, 2, 1, 0):
+        v = stg.stg_dtdg_get_snapshot(g, t)
+        assert_graph_equal(stg.view_arrays(v), oracle.csr(V, sets[t]), tag=("empty walk", t))
+    v = stg.stg_dtdg_get_backward_snapshot(g, 1)
+    assert_graph_equal(stg.view_arrays(v), oracle.csr(V, sets[1]), tag="empty bwd")
+    # aggregation over the empty snapshot: every row has degree 0 -> norm 0 -> y = 0
+    x = to_gpu(gen.uniform_pm1(1, 80, V * 64).reshape(V, 64))
+    assert torch.count_nonzero(stg.stg_gcn_aggregate_fwd(v, x)) == 0
+    assert torch.count_nonzero(stg.stg_gcn_aggregate_bwd(v, x)) == 0
+    # a TGCN step on it: Â = 0, so C = b and the GRU sees only the bias (oracle)
+    F, H = 8, 32
+    p = gen.tgcn_params(F, H, 2)
+    pg = {k: torch.from_numpy(val).cuda() for k, val in p.items()}
+    X = gen.uniform_pm1(2, 81, V * F).reshape(V, F)
+    Hp = gen.uniform_pm1(2, 82, V * H).reshape(V, H)
+    Hn = stg.stg_tgcn_step(stg.stg_dtdg_get_snapshot(g, 1), pg, torch.from_numpy(X).cuda(),
+                           torch.from_numpy(Hp).cuda())
+    ref = oracle.tgcn_fwd(oracle.csr(V, sets[1]), p, X, Hp)
+    assert np.max(np.abs(Hn.cpu().numpy() - ref["Hn"])) <= 2e-5
+
+
+def test_single_vertex_graph(stg):
+    g = stg.stg_static_graph_create(1, [0], [0], stg.STG_EDGE_IDS)
+    ref = oracle.static_graph(1, [0], [0])
+    assert_graph_equal(stg.view_arrays(g.view()), ref, tag="V=1")
+    x = to_gpu(np.array([[1.0, -2.0, 3.0, 0.5]], np.float32))
+    y = stg.stg_gcn_aggregate_fwd(g.view(), x)
+    assert torch.equal(y, x)                                  # Â = [1]: y = x exactly
+    F, H = 4, 16
+    p = gen.tgcn_params(F, H, 9)
+    pg = {k: torch.from_numpy(val).cuda() for k, val in p.items()}
+    X = gen.uniform_pm1(9, 83, F).reshape(1, F)
+    Hp = gen.uniform_pm1(9, 84, H).reshape(1, H)
+    Hn = stg.stg_tgcn_step(g.view(), pg, torch.from_numpy(X).cuda(), torch.from_numpy(Hp).cuda())
+    assert np.max(np.abs(Hn.cpu().numpy() - oracle.tgcn_fwd(ref, p, X, Hp)["Hn"])) <= 2e-5
+
+
+def test_size_limits_rejected(stg):
+    lib = stg._lib
+    out = ctypes.c_void_p()
+    dummy = ctypes.c_void_p(16)
+    st = lib.stg_static_graph_create(1000, 1 << 31, dummy, dummy, 0, None, None, ctypes.byref(out))
+    assert st == 2 and not out.value                          # STG_ERR_OUT_OF_RANGE
+    st = lib.stg_static_graph_create(1 << 30, 10, dummy, dummy, 0, None, None, ctypes.byref(out))
+    assert st == 2
+    st = lib.stg_static_graph_create((1 << 31) - 2, (1 << 31) - 1 - 10, dummy, dummy, stg.STG_SELF_LOOPS, None,
+                                     None, ctypes.byref(out))
+    assert st == 2
