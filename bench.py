@@ -112,6 +112,12 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
+def workload_name(cfg) -> str:
+    """The config.workload string both arms print (the BASELINE.json config it is shaped on)."""
+    names = ["C1", "C2", "C3", "C4", "C5"]
+    return cfg.desc + (" (BASELINE.json configs[%d])" % names.index(cfg.name) if cfg.name in names else "")
+
+
 def measured_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -205,7 +211,7 @@ def run_reference(args):
     out = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-           "config": {"workload": cfg.desc, "config": cfg.name, "V": cfg.V, "F": cfg.F, "H": cfg.H, "T": T,
+           "config": {"workload": workload_name(cfg), "config": cfg.name, "V": cfg.V, "F": cfg.F, "H": cfg.H, "T": T,
                       "sample": sample},
            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -526,8 +532,7 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1 if sim else world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": cfg.desc + " (BASELINE.json configs[%d])" % ["C1", "C2", "C3", "C4", "C5"].index(
-                           cfg.name) if cfg.name in ("C1", "C2", "C3", "C4", "C5") else cfg.desc, "config": cfg.name,
+            "config": {"workload": workload_name(cfg), "config": cfg.name,
                        "V": V,
                        "E_mean": int(E_mean), "T": T, "F": F, "H": H, "seq_len": S, "sequences": len(seqs),
                        "step": "one Algorithm-1 training epoch over all T timestamps",
