@@ -337,6 +337,19 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
                                    float* db_o, float* loss_accum, stg_state_stack* stack,
                                    stg_stream_t stream);
 
+/* The same with per-timestamp input readiness: xy_ready (host)[S] holds a cudaEvent_t
+ * (as stg_event_t) per timestamp, recorded after X[i] and Y[i] were written (e.g. by
+ * a host->device copy on another stream), or NULL entries / a NULL array.  The step
+ * of timestamp i waits for its event only, so a sequence starts computing as soon as
+ * its first inputs have landed while later ones are still being copied (e2e). */
+typedef void* stg_event_t;
+stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
+                                      const stg_tgcn_params* p, const float* w_o, const float* b_o,
+                                      const float* const* X, const float* const* Y, const float* H0,
+                                      float* H_seq, float* G_work, stg_tgcn_grads* grads, float* dw_o,
+                                      float* db_o, float* loss_accum, stg_state_stack* stack,
+                                      const stg_event_t* xy_ready, stg_stream_t stream);
+
 /* Sequence-batched Algorithm 1 for a STATIC graph: the
  * same forward, loss and gradients as stg_tgcn_train_sequence over t = 0..S-1
  * (P:L120-171), scheduled per sequence.  Because C_t = Â(X_t W) + b does not

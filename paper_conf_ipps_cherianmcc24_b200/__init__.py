@@ -125,6 +125,9 @@ _decl("stg_sgd_update", [_P, _P, _i64, _f32, _P])
 _decl("stg_tgcn_train_sequence", [_P, _P, _i32, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P,
                                   ctypes.POINTER(_P), ctypes.POINTER(_P), _P, _P, _P,
                                   ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P, _P])
+_decl("stg_tgcn_train_sequence_ev", [_P, _P, _i32, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P,
+                                     ctypes.POINTER(_P), ctypes.POINTER(_P), _P, _P, _P,
+                                     ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P, ctypes.POINTER(_P), _P])
 _decl("stg_tgcn_train_sequence_batched", [_P, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P, ctypes.POINTER(_P),
                                           ctypes.POINTER(_P), _P, _P, ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P,
                                           _P])
@@ -164,7 +167,7 @@ ABI_SYMBOLS = [
     "stg_gcn_aggregate_fwd", "stg_gcn_aggregate_bwd", "stg_gcn_aggregate_ex",
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
     "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_mse_head_ex", "stg_sgd_update", "stg_tgcn_train_sequence",
-    "stg_tgcn_train_sequence_batched",
+    "stg_tgcn_train_sequence_batched", "stg_tgcn_train_sequence_ev",
     "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
     "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm", "stg_tgcn2_step", "stg_tgcn2_step_backward",
@@ -532,17 +535,21 @@ def stg_tgcn_train_sequence_batched(graph, S: int, params: dict, w_o, b_o, Xs, Y
 
 
 def stg_tgcn_train_sequence(source, t0: int, S: int, params: dict, w_o, b_o, Xs, Ys, H0, H_seq, G_work,
-                            grads: dict, dw_o, db_o, loss_accum, stack: StateStack, stream=None):
-    """Algorithm 1 over one sequence; `source` is a Graph or a Dtdg."""
+                            grads: dict, dw_o, db_o, loss_accum, stack: StateStack, stream=None, xy_ready=None):
+    """Algorithm 1 over one sequence; `source` is a Graph or a Dtdg.  xy_ready: optional list of
+    torch.cuda.Event, one per timestamp, recorded after X_t / y_t were written."""
     P = make_params(params)
     G = make_grads(grads)
     xp = (_P * S)(*[x.data_ptr() for x in Xs])
     yp = (_P * S)(*[y.data_ptr() for y in Ys])
     graph = source.handle if isinstance(source, Graph) else None
     dtdg = source.handle if isinstance(source, Dtdg) else None
-    _check(_lib.stg_tgcn_train_sequence(graph, dtdg, t0, S, ctypes.byref(P), _ptr(w_o), _ptr(b_o), xp, yp,
-                                        _ptr(H0), _ptr(H_seq), _ptr(G_work), ctypes.byref(G), _ptr(dw_o),
-                                        _ptr(db_o), _ptr(loss_accum), stack.handle, _stream(stream)))
+    ev = None
+    if xy_ready is not None:
+        ev = (_P * S)(*[e.cuda_event if e is not None else None for e in xy_ready])
+    _check(_lib.stg_tgcn_train_sequence_ev(graph, dtdg, t0, S, ctypes.byref(P), _ptr(w_o), _ptr(b_o), xp, yp,
+                                           _ptr(H0), _ptr(H_seq), _ptr(G_work), ctypes.byref(G), _ptr(dw_o),
+                                           _ptr(db_o), _ptr(loss_accum), stack.handle, ev, _stream(stream)))
 
 
 def stg_partition_rows(V: int, in_rowptr: torch.Tensor, world: int, stream=None) -> list:

@@ -1276,6 +1276,16 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
                                    const float* const* X, const float* const* Y, const float* H0, float* H_seq,
                                    float* G_work, stg_tgcn_grads* grads, float* dw_o, float* db_o,
                                    float* loss_accum, stg_state_stack* stack, stg_stream_t stream) {
+  return stg_tgcn_train_sequence_ev(graph, dtdg, t0, S, p, w_o, b_o, X, Y, H0, H_seq, G_work, grads, dw_o, db_o,
+                                    loss_accum, stack, nullptr, stream);
+}
+
+stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
+                                      const stg_tgcn_params* p, const float* w_o, const float* b_o,
+                                      const float* const* X, const float* const* Y, const float* H0, float* H_seq,
+                                      float* G_work, stg_tgcn_grads* grads, float* dw_o, float* db_o,
+                                      float* loss_accum, stg_state_stack* stack, const stg_event_t* xy_ready,
+                                      stg_stream_t stream) {
   if ((graph == nullptr) == (dtdg == nullptr))
     return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence: exactly one of graph / dtdg must be given");
   if (S < 1 || !X || !Y || !H0 || !H_seq || !G_work || !stack)
@@ -1343,6 +1353,7 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     const int k = dtdg ? (i & 1) : 0;
     float* C = reinterpret_cast<float*>(stack->arena.p + stack->top);   // state-stack.push target
     if (dtdg && i > 0) STG_TRY(wait(as, ev_built[i & 1], ss));
+    if (xy_ready && xy_ready[i]) STG_CUDA(cudaStreamWaitEvent(as, (cudaEvent_t)xy_ready[i], 0));   // X_t landed
     STG_TRY(fwd_conv(&views[k], p, X[i], ws.P.p, C, as));               // P', C (H-independent)
     STG_TRY(record(ev_conv[i & 1], as));
     if (dtdg && i + 1 < S) {                                            // prefetch Get-Graph(t+1)
@@ -1356,6 +1367,7 @@ stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32
     STG_TRY(fwd_gru(V, p, C, Hp, H_seq + (size_t)i * VH, ms));           // fwdprop
     stack->entries.push_back(StackEntry{Hp, C, V, H, need});
     stack->top += need;
+    if (xy_ready && xy_ready[i] && ms != as) STG_CUDA(cudaStreamWaitEvent(ms, (cudaEvent_t)xy_ready[i], 0));
     STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr,
                             nullptr, stream));                          // loss += loss-fn(out)
   }
