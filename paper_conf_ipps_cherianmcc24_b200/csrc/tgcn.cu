@@ -349,11 +349,30 @@ __global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t Vn, int32_t 
   const float invV = 1.0f / (float)Vn;               // mean over the whole graph's Vn rows
   const float4 wo = reinterpret_cast<const float4*>(w_o)[ql];
   const int64_t step = (int64_t)gridDim.x * (kT / 32) * RPW;
-  for (int64_t v0 = ((int64_t)blockIdx.x * (kT / 32) + w) * RPW; v0 < V; v0 += step) {
+  // U row steps per iteration with all their loads issued first (memory-level
+  // parallelism); the steps are then processed in order, so every accumulation
+  // keeps the one-step-at-a-time order
+  constexpr int U = 4;
+  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int64_t vb = ((int64_t)blockIdx.x * (kT / 32) + w) * RPW; vb < V; vb += U * step) {
+    float4 hu[U], du[U];
+    float yu[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t v = vb + u * step + rl;
+      const bool ok = v < V;
+      hu[u] = ok ? reinterpret_cast<const float4*>(Hn + v * H)[ql] : z4;
+      yu[u] = (ok && ql == 0) ? y[v] : 0.f;
+      du[u] = (ok && want_grad && dH && accumulate) ? reinterpret_cast<const float4*>(dH + v * H)[ql] : z4;
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+    const int64_t v0 = vb + u * step;
+    if (v0 >= V) break;                            // warp-uniform
     const int64_t v = v0 + rl;
     const bool ok = v < V;
-    float4 h = ok ? reinterpret_cast<const float4*>(Hn + v * H)[ql] : make_float4(0.f, 0.f, 0.f, 0.f);
-    const float yv = (ok && ql == 0) ? y[v] : 0.f;
+    const float4 h = hu[u];
+    const float yv = yu[u];
     float4 r = make_float4(fmaxf(h.x, 0.f), fmaxf(h.y, 0.f), fmaxf(h.z, 0.f), fmaxf(h.w, 0.f));
     float s = r.x * wo.x + r.y * wo.y + r.z * wo.z + r.w * wo.w;
 #pragma unroll
@@ -368,13 +387,14 @@ __global__ void __launch_bounds__(kT) k_mse_head(int32_t V, int32_t Vn, int32_t 
                                h.w > 0.f ? g * wo.w : 0.f);
         float4* dp = reinterpret_cast<float4*>(dH + v * H) + ql;
         if (accumulate) {
-          float4 o = *dp;
+          const float4 o = du[u];
           d.x += o.x; d.y += o.y; d.z += o.z; d.w += o.w;
         }
         *dp = d;
       }
       gw.x = fmaf(g, r.x, gw.x); gw.y = fmaf(g, r.y, gw.y); gw.z = fmaf(g, r.z, gw.z); gw.w = fmaf(g, r.w, gw.w);
       if (ql == 0) gb += g;
+    }
     }
   }
   // fixed-order reduction: over the RPW row slots of the warp, then over warps
