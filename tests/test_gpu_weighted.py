@@ -97,3 +97,40 @@ def test_weighted_rejects_bad_args(stg):
         stg.stg_gcn_aggregate_weighted(v, True, ew, x)
     with pytest.raises(stg.StgError):                       # W % 4
         stg.stg_gcn_aggregate_weighted(v, False, ew, torch.zeros(cfg.V, 6, device="cuda"))
+
+
+def test_weighted_sharded_blocks(stg):
+    """Row-block sharded views: each rank's weights in ITS in-CSR order; the
+    forward rows equal the whole-graph rows, the backward partials sum to the oracle."""
+    from paper_conf_ipps_cherianmcc24_b200 import parallel
+    cfg = gen.CONFIGS["C2"]
+    s, d = gen.static_edges(cfg)
+    V, W, world = cfg.V, 64, 3
+    S = oracle.edge_set(V, s, d, self_loops=True)
+    w = gen.edge_weights(11, S.size).astype(np.float64)
+    flags = stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS
+    gfull = stg.stg_static_graph_create(V, s, d, flags)
+    af = stg.view_arrays(gfull.view())
+    ew_full = to_gpu(_in_csr_weights(S, w, af["in_rowptr"].cpu().numpy(), af["in_col"].cpu().numpy()))
+    n = stg.stg_gcn_weighted_norm(gfull.view(), ew_full)
+    n_ref = oracle.weighted_norm(V, S, w)
+    x = gen.uniform_pm1(5, 90, V * W).reshape(V, W).astype(np.float64)
+    y_full = stg.stg_gcn_aggregate_weighted(gfull.view(), False, ew_full, to_gpu(x), scale_row=n, scale_col=n)
+    b = parallel.base_row_blocks(V, s, d, world)
+    gx_sum = np.zeros((V, W))
+    for k in range(world):
+        lo, hi = b[k], b[k + 1]
+        g = stg.stg_static_graph_create(V, s, d, flags, dist=(k, world, lo, hi))
+        v = g.view()
+        a = stg.view_arrays(v)
+        rows = np.repeat(np.arange(lo, hi), np.diff(a["in_rowptr"].cpu().numpy()))
+        keys = oracle.keys(a["in_col"].cpu().numpy(), rows)
+        ew = to_gpu(np.asarray(w)[np.searchsorted(S, keys)])
+        y = stg.stg_gcn_aggregate_weighted(v, False, ew, to_gpu(x), scale_row=n[lo:hi].contiguous(), scale_col=n)
+        assert torch.equal(y, y_full[lo:hi]), k
+        gx = stg.stg_gcn_aggregate_weighted(v, True, ew, to_gpu(x[lo:hi]), scale_row=n,
+                                            scale_col=n[lo:hi].contiguous())
+        gx_sum += gx.cpu().numpy()
+    ref = oracle.aggregate_edges(V, S, w, n_ref, n_ref, x, backward=True)
+    sc = oracle.aggregate_edges(V, S, w, n_ref, n_ref, np.abs(x), backward=True)
+    assert cond_err(gx_sum, ref, sc) <= 1e-5
