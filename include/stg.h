@@ -457,6 +457,29 @@ stg_status stg_tgcn_step_backward_peer(const stg_csr_view* g_bwd, const stg_tgcn
 stg_status stg_tgcn_dw(const stg_tgcn_params* p, int32_t R, const float* X_loc, const float* dP_loc,
                        stg_tgcn_grads* grads, stg_state_stack* stack, stg_stream_t stream);
 
+/* The original T-GCN cell in sharded mode over peer memory: both convolutions gather
+ * rows that carry H from their owners (north_star "all-gather ... of the source
+ * feature/hidden rows each timestep"), so the hidden state crosses ranks every
+ * step.  Each call runs one phase; the caller puts a cross-rank barrier between
+ * phases (parallel.PeerTGCN2).  R = local rows of the sharded view.
+ *   fwd phase 0: Z_loc [R,2H] = n_src ⊙ [X_loc, H_loc]·Wg   (this rank's block of Zg)
+ *       phase 1: gates from Â·Zg (rows gathered through Z) + bg; Z_loc [R,H] = n_src ⊙ [X_loc, r⊙H]·Wc
+ *       phase 2: c from Â·Zc (rows gathered through Z) + bc; H_next [R,H]; state pushed
+ *   bwd phase 0: candidate backward, dbc; part_out [V,H] = partial Âᵀ dA_c of the local edges
+ *       phase 1: dY_c = Σ_ranks parts (stg_reduce_scatter_rows), dWc, gate backward, dbg;
+ *                part_out [V,2H] = partial Âᵀ dA_g
+ *       phase 2: dY_g = Σ_ranks parts, dWg, dH_prev += dY_g·Wg[F:]ᵀ; state popped
+ * parts (host)[world] = every rank's part_out of the previous phase.  Gradients are this
+ * rank's share (sum over ranks = whole-graph gradient). */
+stg_status stg_tgcn2_peer_fwd(int32_t phase, const stg_csr_view* g, const stg_tgcn2_params* p, const float* X_loc,
+                              const float* H_loc, const stg_peer_rows* Z, float* Z_loc, float* H_next,
+                              stg_state_stack* stack, stg_stream_t stream);
+stg_status stg_tgcn2_peer_bwd(int32_t phase, const stg_csr_view* g, const stg_tgcn2_params* p, const float* X_loc,
+                              const float* dH_next, float* dH_prev, stg_tgcn2_grads* grads, int32_t rank,
+                              int32_t world, const int32_t* bounds, const float* const* parts, float* part_out,
+                              stg_state_stack* stack, stg_stream_t stream);
+
+
 /* Per-phase device timing with CUDA events recorded on the launching stream
  * around each phase (bench.py; the GNN vs graph-update split of Fig. 9,
  * P:L316/L345).  phase: 0 aggregation fwd, 1 aggregation bwd, 2 snapshot

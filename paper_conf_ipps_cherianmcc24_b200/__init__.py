@@ -143,6 +143,11 @@ _decl("stg_gcn_weighted_norm", [ctypes.POINTER(stg_csr_view), _P, _P, _P])
 _decl("stg_tgcn2_step", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn2_params), _P, _P, _P, _P, _P])
 _decl("stg_tgcn2_step_backward", [ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn2_params), _P, _P, _P,
                                   ctypes.POINTER(stg_tgcn2_grads), _P, _P])
+_decl("stg_tgcn2_peer_fwd", [_i32, ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn2_params), _P, _P,
+                             ctypes.POINTER(stg_peer_rows), _P, _P, _P, _P])
+_decl("stg_tgcn2_peer_bwd", [_i32, ctypes.POINTER(stg_csr_view), ctypes.POINTER(stg_tgcn2_params), _P, _P, _P,
+                             ctypes.POINTER(stg_tgcn2_grads), _i32, _i32, ctypes.POINTER(_i32), ctypes.POINTER(_P), _P,
+                             _P, _P])
 _decl("stg_peer_alloc", [_i64, ctypes.POINTER(_P), ctypes.POINTER(stg_ipc_handle)])
 _decl("stg_peer_free", [_P])
 _decl("stg_peer_open", [ctypes.POINTER(stg_ipc_handle), ctypes.POINTER(_P)])
@@ -173,7 +178,7 @@ ABI_SYMBOLS = [
     "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm", "stg_tgcn2_step", "stg_tgcn2_step_backward",
     "stg_peer_alloc", "stg_peer_free", "stg_peer_open", "stg_peer_close", "stg_allgather_rows",
     "stg_gcn_aggregate_peer", "stg_reduce_scatter_rows", "stg_tgcn_project", "stg_tgcn_step_peer",
-    "stg_tgcn_step_backward_peer", "stg_tgcn_dw",
+    "stg_tgcn_step_backward_peer", "stg_tgcn_dw", "stg_tgcn2_peer_fwd", "stg_tgcn2_peer_bwd",
 ]
 
 PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head", "dl"]
@@ -701,3 +706,28 @@ def stg_tgcn_dw(params: dict, X_loc, dP_loc, grads: dict, stack: StateStack, str
     R = X_loc.shape[0]
     _check(_lib.stg_tgcn_dw(ctypes.byref(P), int(R), _ptr(X_loc), ctypes.c_void_p(_row_ptr(dP_loc)),
                             ctypes.byref(G), stack.handle, _stream(stream)))
+
+
+def stg_tgcn2_peer_fwd(phase: int, v: stg_csr_view, params: dict, X_loc, H_loc, rows: PeerRows = None, Z_loc=None,
+                       H_next=None, stack: StateStack = None, stream=None):
+    """One phase of the sharded original T-GCN forward (include/stg.h)."""
+    P = make_params2(params)
+    _check(_lib.stg_tgcn2_peer_fwd(int(phase), ctypes.byref(v), ctypes.byref(P), _ptr(X_loc), _ptr(H_loc),
+                                   ctypes.byref(rows.c) if rows is not None else None,
+                                   ctypes.c_void_p(_row_ptr(Z_loc)) if Z_loc is not None else None,
+                                   _ptr(H_next) if H_next is not None else None, stack.handle, _stream(stream)))
+
+
+def stg_tgcn2_peer_bwd(phase: int, v: stg_csr_view, params: dict, X_loc, dH_next, dH_prev, grads: dict, rank: int,
+                       bounds, parts, part_out, stack: StateStack, stream=None):
+    """One phase of the sharded original T-GCN backward (include/stg.h)."""
+    P = make_params2(params)
+    G = stg_tgcn2_grads(_ptr(grads["Wg"]), _ptr(grads["bg"]), _ptr(grads["Wc"]), _ptr(grads["bc"]))
+    world = len(bounds) - 1
+    b = (_i32 * (world + 1))(*[int(x) for x in bounds])
+    pp = (_P * world)(*[_row_ptr(x) for x in parts]) if parts is not None else None
+    _check(_lib.stg_tgcn2_peer_bwd(int(phase), ctypes.byref(v), ctypes.byref(P), _ptr(X_loc),
+                                   _ptr(dH_next) if dH_next is not None else None, _ptr(dH_prev), ctypes.byref(G),
+                                   int(rank), world, b, pp,
+                                   ctypes.c_void_p(_row_ptr(part_out)) if part_out is not None else None,
+                                   stack.handle, _stream(stream)))

@@ -1171,6 +1171,112 @@ stg_status stg_tgcn2_step_backward(const stg_csr_view* g, const stg_tgcn2_params
   return check_launch("stg_tgcn2_step_backward");
 }
 
+// ---- original T-GCN in sharded mode over peer memory (NEXT-2 x §8(e)): both
+// convolutions gather their source rows — which carry H — from the owners' blocks,
+// so hidden-state rows cross ranks every timestep.  Phases are separated by the
+// caller's cross-rank barrier (parallel.PeerTGCN2).
+static stg_status check_tgcn2_peer(const stg_csr_view* g, const stg_tgcn2_params* p) {
+  if (!g || !p || !p->Wg || !p->bg || !p->Wc || !p->bc) return fail(STG_ERR_INVALID_ARG, "tgcn2_peer: NULL argument");
+  if (p->F < 1 || p->H < 4 || p->H > 64 || p->H % 4 || (p->H & (p->H - 1)))
+    return fail(STG_ERR_INVALID_ARG, "tgcn2_peer: need F >= 1 and H in {4, 8, 16, 32, 64} (H=%d)", p->H);
+  if ((size_t)(p->F + p->H) * 2 * p->H * 4 + 32 * (size_t)(p->F + p->H + 1) * 4 > 200 * 1024)
+    return fail(STG_ERR_INVALID_ARG, "tgcn2_peer: F+H=%d too large for the shared-memory weights", p->F + p->H);
+  return STG_OK;
+}
+
+stg_status stg_tgcn2_peer_fwd(int32_t phase, const stg_csr_view* g, const stg_tgcn2_params* p, const float* X_loc,
+                              const float* H_loc, const stg_peer_rows* Z, float* Z_loc, float* H_next,
+                              stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_tgcn2_peer(g, p));
+  if (!X_loc || !H_loc || !stack || phase < 0 || phase > 2)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_fwd: bad arguments (phase %d)", phase);
+  cudaStream_t s = (cudaStream_t)stream;
+  const int32_t R = g->row_end - g->row_begin, F = p->F, H = p->H, H2 = 2 * H;
+  const float* ns_loc = g->norm_src ? g->norm_src + g->row_begin : nullptr;
+  const float* nd_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
+  TgcnWs& ws = stack->ws;
+  STG_TRY(t2_ws(ws, R > 0 ? R : 1, H));
+  const size_t need = stack_bytes(R, H);
+  if (stack->top + need > stack->cap) return fail(STG_ERR_NO_MEMORY, "stg_tgcn2_peer_fwd: state stack full");
+  float* RUC = reinterpret_cast<float*>(stack->arena.p + stack->top);   // pushed at phase 2
+  if (phase == 0) {                          // Zg rows of this block -> the peer buffer
+    if (!Z_loc && R > 0) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_fwd: Z_loc is NULL");
+    return t2_mm(R, X_loc, F, F, H_loc, H, H, p->Wg, H2, 1, H2, ns_loc, Z_loc, H2, false, s);
+  }
+  if (!Z) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_fwd: row table is NULL");
+  float* A = ws.t2a.p;
+  if (phase == 1) {                          // gates from the gathered Zg, then this block's Zc
+    if (R == 0) return STG_OK;
+    if (!Z_loc) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_fwd: Z_loc is NULL");
+    STG_TRY(aggregate_launch(g, 0, H2, nullptr, 0, A, H2, nd_loc, nullptr, p->bg, s, Z));
+    k_t2_gates<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, A, H_loc, RUC, ws.t2b.p);
+    count_launch();
+    return t2_mm(R, X_loc, F, F, ws.t2b.p, H, H, p->Wc, H, 1, H, ns_loc, Z_loc, H, false, s);
+  }
+  if (!H_next && R > 0) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_fwd: H_next is NULL");
+  if (R > 0) {                               // candidate from the gathered Zc, H_next; push
+    STG_TRY(aggregate_launch(g, 0, H, nullptr, 0, A, H, nd_loc, nullptr, p->bc, s, Z));
+    k_t2_cand<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, A, H_loc, RUC, H_next);
+    count_launch();
+  }
+  stack->entries.push_back(StackEntry{H_loc, RUC, R, H, need});
+  stack->top += need;
+  return check_launch("stg_tgcn2_peer_fwd");
+}
+
+stg_status stg_tgcn2_peer_bwd(int32_t phase, const stg_csr_view* g, const stg_tgcn2_params* p, const float* X_loc,
+                              const float* dH_next, float* dH_prev, stg_tgcn2_grads* grads, int32_t rank,
+                              int32_t world, const int32_t* bounds, const float* const* parts, float* part_out,
+                              stg_state_stack* stack, stg_stream_t stream) {
+  STG_TRY(check_tgcn2_peer(g, p));
+  if (!X_loc || !dH_prev || !grads || !grads->Wg || !grads->bg || !grads->Wc || !grads->bc || !stack || phase < 0 ||
+      phase > 2)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_bwd: bad arguments (phase %d)", phase);
+  if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn2_peer_bwd: state stack is empty");
+  const StackEntry e = stack->entries.back();
+  const int32_t V = g->num_nodes, R = g->row_end - g->row_begin, F = p->F, H = p->H, H2 = 2 * H;
+  if (e.V != R || e.H != H) return fail(STG_ERR_STATE, "stg_tgcn2_peer_bwd: stack top does not match (R,H)");
+  cudaStream_t s = (cudaStream_t)stream;
+  TgcnWs& ws = stack->ws;
+  STG_TRY(t2_ws(ws, R > 0 ? R : 1, H));
+  const float* nd_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
+  const float* RUC = e.C;
+  const float* Hp = e.Hp;
+  float *dAg = ws.t2z.p, *Yl = ws.t2a.p, *rH = ws.t2b.p, *D1 = ws.t2c.p, *du = ws.t2d.p;
+  if (phase == 0) {                          // candidate backward; partial dY_c of the local edges for all V
+    if (!dH_next || !part_out) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_bwd: NULL dH_next / part_out");
+    if (R > 0) {
+      k_t2_cand_bwd<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, dH_next, Hp, RUC, D1, du, dH_prev, rH);
+      count_launch();
+      STG_TRY(t2_colsum(R, D1, H, grads->bc, ws, s));
+    }
+    return aggregate_launch(g, 1, H, D1, H, part_out, H, g->norm_src, nd_loc, nullptr, s);
+  }
+  if (!parts || !bounds || world < 1 || rank < 0 || rank >= world)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_bwd: bad peer arguments");
+  if (phase == 1) {                          // reduce-scatter dY_c; dWc, d(r⊙H), gate backward; partial dY_g
+    if (!part_out) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_bwd: part_out is NULL");
+    if (R > 0) {
+      STG_TRY(stg_reduce_scatter_rows(world, bounds, parts, H, rank, H, Yl, H, stream));
+      STG_TRY(t2_atb(R, X_loc, F, rH, H, Yl, H, grads->Wc, ws, s));
+      STG_TRY(t2_mm(R, Yl, H, H, nullptr, 0, 0, p->Wc + (size_t)F * H, 1, H, H, nullptr, D1, H, false, s));
+      k_t2_gate_bwd<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, D1, Hp, RUC, du, dH_prev, dAg);
+      count_launch();
+      STG_TRY(t2_colsum(R, dAg, H2, grads->bg, ws, s));
+    }
+    (void)V;
+    return aggregate_launch(g, 1, H2, dAg, H2, part_out, H2, g->norm_src, nd_loc, nullptr, s);
+  }
+  if (R > 0) {                               // reduce-scatter dY_g; dWg, dH; pop
+    STG_TRY(stg_reduce_scatter_rows(world, bounds, parts, H2, rank, H2, Yl, H2, stream));
+    STG_TRY(t2_atb(R, X_loc, F, Hp, H, Yl, H2, grads->Wg, ws, s));
+    STG_TRY(t2_mm(R, Yl, H2, H2, nullptr, 0, 0, p->Wg + (size_t)F * H2, 1, H2, H, nullptr, dH_prev, H, true, s));
+  }
+  stack->entries.pop_back();
+  stack->top -= e.bytes;
+  return check_launch("stg_tgcn2_peer_bwd");
+}
+
 stg_status stg_mse_head(int32_t V, int32_t H, const float* Hn, const float* y, const float* w_o, const float* b_o,
                         float* loss_accum, float* dH, int32_t accumulate, float* dw_o, float* db_o,
                         stg_stream_t stream) {

@@ -185,3 +185,65 @@ class PeerTGCN:
     def close(self):
         for g in self.P + self.dP:
             g.close()
+
+
+class PeerTGCN2:
+    """Algorithm 1 for one rank with the ORIGINAL T-GCN cell in sharded mode (NEXT-2):
+    the gate and candidate convolutions gather rows that carry H from their owners,
+    so hidden-state rows cross ranks every timestep (stg_tgcn2_peer_fwd / _bwd, one
+    stream barrier between phases).  Buffers alternate by timestep as in PeerTGCN."""
+
+    def __init__(self, stg, bounds, V: int, F: int, H: int, S: int):
+        self.stg = stg
+        self.bounds = list(bounds)
+        self.rank = dist.get_rank()
+        self.V, self.F, self.H = V, F, H
+        self.R = self.bounds[self.rank + 1] - self.bounds[self.rank]
+        self.Zg = [PeerGroup(self.bounds, 2 * H) for _ in range(2)]
+        self.Zc = [PeerGroup(self.bounds, H) for _ in range(2)]
+        self.Dc = [PeerGroup(self.bounds, H, full=True) for _ in range(2)]
+        self.Dg = [PeerGroup(self.bounds, 2 * H, full=True) for _ in range(2)]
+        self.G = torch.empty(2, max(self.R, 1), H, device="cuda")
+        self.stack = stg.stg_state_stack_create(S * max(self.R, 1) * 3 * H * 4 + (1 << 20))
+
+    def train_sequence(self, source, t0, params, w_o, b_o, X_loc, Y_loc, H0, H_seq, grads, dw_o, db_o, loss,
+                       barrier=stream_barrier):
+        stg, S, R = self.stg, len(X_loc), self.R
+        dyn = isinstance(source, stg.Dtdg)
+
+        def view(t, backward):
+            if not dyn:
+                return source.view()
+            part = stg.STG_PART_OUT if backward else stg.STG_PART_IN
+            return stg.stg_dtdg_get_snapshot_parts(source, t, part, backward=backward)
+
+        for i in range(S):
+            v = view(t0 + i, False)
+            Hp = H0 if i == 0 else H_seq[i - 1]
+            zg, zc = self.Zg[i & 1], self.Zc[i & 1]
+            stg.stg_tgcn2_peer_fwd(0, v, params, X_loc[i], Hp, Z_loc=zg.buf.ptr, stack=self.stack)
+            barrier()                                          # every owner's Zg rows written
+            stg.stg_tgcn2_peer_fwd(1, v, params, X_loc[i], Hp, rows=zg.rows, Z_loc=zc.buf.ptr, stack=self.stack)
+            barrier()                                          # every owner's Zc rows written
+            stg.stg_tgcn2_peer_fwd(2, v, params, X_loc[i], Hp, rows=zc.rows, H_next=H_seq[i], stack=self.stack)
+            stg.stg_mse_head(H_seq[i], Y_loc[i], w_o, b_o, loss_accum=loss, V_total=self.V)
+        G, Gn = self.G[0][:R], self.G[1][:R]
+        G.zero_()
+        for i in range(S - 1, -1, -1):
+            v = view(t0 + i, True)
+            stg.stg_mse_head(H_seq[i], Y_loc[i], w_o, b_o, dH=G, accumulate=True, dw_o=dw_o, db_o=db_o,
+                             V_total=self.V)
+            dc, dg = self.Dc[i & 1], self.Dg[i & 1]
+            stg.stg_tgcn2_peer_bwd(0, v, params, X_loc[i], G, Gn, grads, self.rank, self.bounds, None, dc.buf.ptr,
+                                   self.stack)
+            barrier()                                          # every rank's partial dY_c written
+            stg.stg_tgcn2_peer_bwd(1, v, params, X_loc[i], None, Gn, grads, self.rank, self.bounds, dc.ptrs,
+                                   dg.buf.ptr, self.stack)
+            barrier()                                          # every rank's partial dY_g written
+            stg.stg_tgcn2_peer_bwd(2, v, params, X_loc[i], None, Gn, grads, self.rank, self.bounds, dg.ptrs, None,
+                                   self.stack)
+            G, Gn = Gn, G
+
+    def close(self):
+        for g in self.Zg + self.Zc + self.Dc + self.Dg:
+            g.close()

@@ -106,3 +106,140 @@ def test_tgcn2_sequence_over_dtdg(stg):
     gd = dict(grads)
     gd["w_o"], gd["b_o"] = dw, db
     _check(gd, rg, V * S, keys=("Wg", "bg", "Wc", "bc", "w_o", "b_o"))
+
+
+def test_tgcn2_sharded_peer_simulated_ranks(stg):
+    """Sharded original T-GCN (hidden-state rows cross ranks every step): three ranks of a
+    DTDG interleaved phase by phase in one process (every block its own allocation);
+    the rows of H_t match the oracle and the summed loss / gradients match the
+    whole-graph oracle sequence."""
+    from paper_conf_ipps_cherianmcc24_b200 import parallel
+    cfg = gen.CONFIGS["C5s"]
+    dd = gen.dtdg(cfg)
+    V, F, H, S, world = cfg.V, cfg.F, cfg.H, 3, 3
+    p = gen.tgcn2_params(F, H, 6)
+    pg = {k: torch.from_numpy(v).cuda() for k, v in p.items()}
+    Xs = [gen.features(cfg, t) for t in range(S)]
+    Ys = [gen.labels(cfg, t) for t in range(S)]
+    b = parallel.base_row_blocks(V, dd.src0, dd.dst0, world)
+    ranks = []
+    for k in range(world):
+        lo, hi = b[k], b[k + 1]
+        R = hi - lo
+        r = {"lo": lo, "hi": hi, "R": R, "grads": _zero2(F, H)}
+        r["g"] = stg.stg_dtdg_create(V, dd.T, dd.src0, dd.dst0, dd.add_off, dd.add_src, dd.add_dst, dd.del_off,
+                                     dd.del_src, dd.del_dst, stg.STG_SELF_LOOPS, dist=(k, world, lo, hi))
+        r["dw"], r["db"], r["loss"] = (torch.zeros(H, device="cuda"), torch.zeros(1, device="cuda"),
+                                       torch.zeros(1, device="cuda"))
+        r["Hs"] = [torch.zeros(R, H, device="cuda")] + [torch.empty(R, H, device="cuda") for _ in range(S)]
+        r["X"] = [torch.from_numpy(x[lo:hi].copy()).cuda() for x in Xs]
+        r["Y"] = [torch.from_numpy(y[lo:hi].copy()).cuda() for y in Ys]
+        r["Zg"] = torch.empty(max(R, 1), 2 * H, device="cuda")
+        r["Zc"] = torch.empty(max(R, 1), H, device="cuda")
+        r["Dc"] = torch.empty(V, H, device="cuda")
+        r["Dg"] = torch.empty(V, 2 * H, device="cuda")
+        r["G"] = [torch.zeros(R, H, device="cuda"), torch.empty(R, H, device="cuda")]
+        r["st"] = stg.stg_state_stack_create(S * max(R, 1) * 3 * H * 4 + (1 << 20))
+        ranks.append(r)
+    for i in range(S):
+        vs = [stg.stg_dtdg_get_snapshot_parts(r["g"], i, stg.STG_PART_IN) for r in ranks]
+        for r, v in zip(ranks, vs):
+            stg.stg_tgcn2_peer_fwd(0, v, pg, r["X"][i], r["Hs"][i], Z_loc=r["Zg"], stack=r["st"])
+        tg = stg.PeerRows(b, [r["Zg"].data_ptr() for r in ranks], 2 * H)
+        for r, v in zip(ranks, vs):
+            stg.stg_tgcn2_peer_fwd(1, v, pg, r["X"][i], r["Hs"][i], rows=tg, Z_loc=r["Zc"], stack=r["st"])
+        tc = stg.PeerRows(b, [r["Zc"].data_ptr() for r in ranks], H)
+        for r, v in zip(ranks, vs):
+            stg.stg_tgcn2_peer_fwd(2, v, pg, r["X"][i], r["Hs"][i], rows=tc, H_next=r["Hs"][i + 1], stack=r["st"])
+            stg.stg_mse_head(r["Hs"][i + 1], r["Y"][i], pg["w_o"], pg["b_o"], loss_accum=r["loss"], V_total=V)
+    for i in range(S - 1, -1, -1):
+        vs = [stg.stg_dtdg_get_snapshot_parts(r["g"], i, stg.STG_PART_OUT, backward=True) for r in ranks]
+        for r, v in zip(ranks, vs):
+            G, Gn = r["G"]
+            stg.stg_mse_head(r["Hs"][i + 1], r["Y"][i], pg["w_o"], pg["b_o"], dH=G, accumulate=True, dw_o=r["dw"],
+                             db_o=r["db"], V_total=V)
+            stg.stg_tgcn2_peer_bwd(0, v, pg, r["X"][i], G, Gn, r["grads"], 0, b, None, r["Dc"], r["st"])
+        for k, (r, v) in enumerate(zip(ranks, vs)):
+            stg.stg_tgcn2_peer_bwd(1, v, pg, r["X"][i], None, r["G"][1], r["grads"], k, b,
+                                   [q["Dc"] for q in ranks], r["Dg"], r["st"])
+        for k, (r, v) in enumerate(zip(ranks, vs)):
+            stg.stg_tgcn2_peer_bwd(2, v, pg, r["X"][i], None, r["G"][1], r["grads"], k, b,
+                                   [q["Dg"] for q in ranks], None, r["st"])
+            r["G"] = [r["G"][1], r["G"][0]]
+    torch.cuda.synchronize()
+    sets = list(oracle.snapshot_sets_fold(dd, self_loops=True))
+    rl, rg, rH = oracle.train_sequence2([oracle.csr(V, sets[t]) for t in range(S)], p, Xs, Ys, np.zeros((V, H)))
+    l_sum, g_sum = 0.0, None
+    for r in ranks:
+        np.testing.assert_allclose(r["Hs"][-1].cpu().numpy(), rH[r["lo"]:r["hi"]], rtol=0, atol=2e-5)
+        l_sum += r["loss"].item()
+        gk = {n: t.cpu().numpy().astype(np.float64) for n, t in r["grads"].items()}
+        gk.update(w_o=r["dw"].cpu().numpy().astype(np.float64), b_o=r["db"].cpu().numpy().astype(np.float64))
+        g_sum = gk if g_sum is None else {n: g_sum[n] + gk[n] for n in g_sum}
+    assert abs(l_sum - rl) <= 1e-5 * abs(rl), (l_sum, rl)
+    _check(g_sum, rg, V * S, keys=("Wg", "bg", "Wc", "bc", "w_o", "b_o"))
+
+
+def _ipc_worker2(rank, world, port, outdir):
+    import os
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import torch.distributed as dist
+    import paper_conf_ipps_cherianmcc24_b200 as stg
+    from paper_conf_ipps_cherianmcc24_b200 import parallel
+    dist.init_process_group("gloo", init_method="tcp://127.0.0.1:%d" % port, rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    cfg = gen.CONFIGS["C5s"]
+    dd = gen.dtdg(cfg)
+    V, F, H, S = cfg.V, cfg.F, cfg.H, 2
+    b = parallel.base_row_blocks(V, dd.src0, dd.dst0, world)
+    lo, hi = b[rank], b[rank + 1]
+    R = hi - lo
+    g = stg.stg_dtdg_create(V, dd.T, dd.src0, dd.dst0, dd.add_off, dd.add_src, dd.add_dst, dd.del_off, dd.del_src,
+                            dd.del_dst, stg.STG_SELF_LOOPS, dist=(rank, world, lo, hi))
+    p = {k: torch.from_numpy(v).cuda() for k, v in gen.tgcn2_params(F, H, 6).items()}
+    grads = _zero2(F, H)
+    dw, db, loss = torch.zeros(H, device="cuda"), torch.zeros(1, device="cuda"), torch.zeros(1, device="cuda")
+    drv = parallel.PeerTGCN2(stg, b, V, F, H, S)
+    X = [torch.from_numpy(gen.features(cfg, t)[lo:hi].copy()).cuda() for t in range(S)]
+    Y = [torch.from_numpy(gen.labels(cfg, t)[lo:hi].copy()).cuda() for t in range(S)]
+    Hs = torch.empty(S, R, H, device="cuda")
+    drv.train_sequence(g, 0, p, p["w_o"], p["b_o"], X, Y, torch.zeros(R, H, device="cuda"), Hs, grads, dw, db, loss)
+    torch.cuda.synchronize()
+    out = {n: t.cpu().numpy() for n, t in grads.items()}
+    out.update(w_o=dw.cpu().numpy(), b_o=db.cpu().numpy(), loss=loss.cpu().numpy(), H=Hs[-1].cpu().numpy(),
+               lo=np.array(lo), hi=np.array(hi))
+    np.savez(os.path.join(outdir, "rank%d.npz" % rank), **out)
+    parallel.stream_barrier()
+    drv.close()
+    dist.destroy_process_group()
+
+
+def test_tgcn2_sharded_peer_two_processes(stg, tmp_path):
+    import os
+    import socket
+    import torch.multiprocessing as mp
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    world = 2
+    mp.start_processes(_ipc_worker2, args=(world, port, str(tmp_path)), nprocs=world, join=True,
+                       start_method="spawn")
+    cfg = gen.CONFIGS["C5s"]
+    dd = gen.dtdg(cfg)
+    V, H, S = cfg.V, cfg.H, 2
+    p = gen.tgcn2_params(cfg.F, H, 6)
+    sets = list(oracle.snapshot_sets_fold(dd, self_loops=True))
+    rl, rg, rH = oracle.train_sequence2([oracle.csr(V, sets[t]) for t in range(S)], p,
+                                        [gen.features(cfg, t) for t in range(S)],
+                                        [gen.labels(cfg, t) for t in range(S)], np.zeros((V, H)))
+    l_sum, g_sum = 0.0, None
+    for r in range(world):
+        z = np.load(os.path.join(str(tmp_path), "rank%d.npz" % r))
+        lo, hi = int(z["lo"]), int(z["hi"])
+        np.testing.assert_allclose(z["H"], rH[lo:hi], rtol=0, atol=2e-5)
+        l_sum += float(z["loss"][0])
+        gk = {n: z[n].astype(np.float64) for n in ("Wg", "bg", "Wc", "bc", "w_o", "b_o")}
+        g_sum = gk if g_sum is None else {n: g_sum[n] + gk[n] for n in g_sum}
+    assert abs(l_sum - rl) <= 1e-5 * abs(rl), (l_sum, rl)
+    _check(g_sum, rg, V * S, keys=("Wg", "bg", "Wc", "bc", "w_o", "b_o"))
