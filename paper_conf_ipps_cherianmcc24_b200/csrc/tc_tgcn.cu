@@ -2010,32 +2010,35 @@ stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH,
 namespace stg {
 
 // ---- sequence-batched GRU launchers (NEXT-1; layouts in the kernels' comment)
-// ---- sequence GRU for tiny graphs (V <= kSmallV): one CTA, fp32 SIMT, every row of the
-// graph in shared memory.  A 128-row tensor-core tile would be mostly padding and each
-// of its MMA phases a full round trip; here a timestep is a few block-wide phases of
-// 2H-term dot products.  Same outputs, layouts and fused head as the tcgen05 kernels.
-constexpr int kSmallV = 128, kSmallT = 512;
+// ---- sequence GRU for small graphs (V <= kSmallMaxV): fp32 SIMT, a CTA owns RB rows
+// (the recurrence is row-local) and stages its rows' whole-sequence inputs in shared
+// memory once.  A 128-row tcgen05 tile would be mostly padding for C1 (V = 20), and
+// each of its MMA phases is a full round trip; here a timestep is a few block-wide
+// phases of 2H-term dot products.  Same outputs, layouts and fused head as the
+// tcgen05 kernels; per-CTA head partials (nb = number of CTAs).
+constexpr int kSmallT = 512, kSmallMaxV = 128;   // measured: beyond one tile the tcgen05 kernels win (C2, C3)
 
 template <int H>
-__global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, const float* __restrict__ C_all,
+__global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, int RB, const float* __restrict__ C_all,
                                                            const float* __restrict__ H0, const float* __restrict__ L,
                                                            const float* __restrict__ l, float* __restrict__ H_seq,
                                                            float* __restrict__ Hp_all, const float* __restrict__ Yall,
                                                            const float* __restrict__ w_o,
                                                            const float* __restrict__ b_o, double* __restrict__ lpart) {
   extern __shared__ float sm[];
-  const int VH = V * H, H3 = 3 * H, LG = 2 * H * H;
+  const int r0 = blockIdx.x * RB, Vl = min(RB, V - r0);
+  const int VH = Vl * H, H3 = 3 * H, LG = 2 * H * H;
   float* sL = sm;                  // [3][2H][H]
-  float* sh = sL + 3 * LG;         // H_{t-1} [V][H]
-  float* sz = sh + VH;             // z
-  float* srh = sz + VH;            // r ⊙ h
-  float* sn = srh + VH;            // H_t
-  float* sC = sn + VH;             // C_all [V][S][3H], staged once
-  __shared__ double sloss[kSmallV];
-  for (int e = threadIdx.x; e < V * S * H3; e += kSmallT) sC[e] = C_all[e];
+  float* sh = sL + 3 * LG;         // H_{t-1} [Vl][H]
+  float* sz = sh + RB * H;         // z
+  float* srh = sz + RB * H;        // r ⊙ h
+  float* sn = srh + RB * H;        // H_t
+  float* sC = sn + RB * H;         // this CTA's rows of C_all [Vl][S][3H]
+  __shared__ double sloss[kSmallT];
+  for (int e = threadIdx.x; e < Vl * S * H3; e += kSmallT) sC[e] = C_all[(int64_t)r0 * S * H3 + e];
   for (int e = threadIdx.x; e < 3 * LG; e += kSmallT) sL[e] = L[e];
-  for (int e = threadIdx.x; e < VH; e += kSmallT) sh[e] = H0[e];
-  for (int v = threadIdx.x; v < V; v += kSmallT) sloss[v] = 0.0;
+  for (int e = threadIdx.x; e < VH; e += kSmallT) sh[e] = H0[(int64_t)r0 * H + e];
+  for (int v = threadIdx.x; v < Vl; v += kSmallT) sloss[v] = 0.0;
   const float* Lz = sL; const float* Lr = sL + LG; const float* Lh = sL + 2 * LG;
   const float bo = b_o[0];
   __syncthreads();
@@ -2057,7 +2060,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, const f
       }
       sz[e] = 1.0f / (1.0f + expf(-az));
       srh[e] = hv[j] / (1.0f + expf(-ar));
-      Hp_all[((int64_t)v * S + t) * H + j] = hv[j];
+      Hp_all[((int64_t)(r0 + v) * S + t) * H + j] = hv[j];
     }
     __syncthreads();
     for (int e = threadIdx.x; e < VH; e += kSmallT) {          // candidate, H_t
@@ -2071,14 +2074,14 @@ __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, const f
       const float z = sz[e], hh = tanhf(ah);
       const float hn = z * sh[e] + (1.0f - z) * hh;
       sn[e] = hn;
-      H_seq[((int64_t)t * V + v) * H + j] = hn;
+      H_seq[((int64_t)t * V + r0 + v) * H + j] = hn;
     }
     __syncthreads();
-    for (int v = threadIdx.x; v < V; v += kSmallT) {            // fused head: loss of row v at t
+    for (int v = threadIdx.x; v < Vl; v += kSmallT) {           // fused head: loss of row v at t
       float d = 0.f;
 #pragma unroll
       for (int j = 0; j < H; ++j) d = fmaf(fmaxf(sn[v * H + j], 0.f), w_o[j], d);
-      const float e = (d + bo) - Yall[(int64_t)v * S + t];
+      const float e = (d + bo) - Yall[(int64_t)(r0 + v) * S + t];
       sloss[v] += (double)e * (double)e;
     }
     for (int e = threadIdx.x; e < VH; e += kSmallT) sh[e] = sn[e];
@@ -2086,13 +2089,13 @@ __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, const f
   }
   if (threadIdx.x == 0) {
     double tot = 0.0;
-    for (int v = 0; v < V; ++v) tot += sloss[v];
-    lpart[0] = tot;
+    for (int v = 0; v < Vl; ++v) tot += sloss[v];
+    lpart[blockIdx.x] = tot;
   }
 }
 
 template <int H>
-__global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, const float* __restrict__ C_all,
+__global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB, const float* __restrict__ C_all,
                                                            const float* __restrict__ Hp_all,
                                                            const float* __restrict__ H_seq,
                                                            const float* __restrict__ L, const float* __restrict__ l,
@@ -2103,24 +2106,29 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, const f
                                                            float* __restrict__ dC_all, float* __restrict__ da_all,
                                                            float* __restrict__ RH_all, float* __restrict__ gpart) {
   extern __shared__ float sm[];
-  const int VH = V * H, H3 = 3 * H, LG = 2 * H * H;
+  const int r0 = blockIdx.x * RB, Vl = min(RB, V - r0);
+  const int VH = Vl * H, H3 = 3 * H, LG = 2 * H * H, RH = RB * H;
   float* sL = sm;                  // [3][2H][H]
   float* sdh = sL + 3 * LG;        // dℓ/dH_t flowing back from t+1
-  float* sg = sdh + VH;            // G
-  float* sz = sg + VH;
-  float* sr = sz + VH;
-  float* srh = sr + VH;
-  float* sdaz = srh + VH;
-  float* sdah = sdaz + VH;
-  float* sdar = sdah + VH;
-  float* sdhn = sdar + VH;
-  float* sC = sdhn + VH;                    // C_all [V][S][3H]
-  float* sHp = sC + (size_t)V * S * H3;     // Hp_all [V][S][H]
-  float* sHs = sHp + (size_t)V * S * H;     // H_seq [S][V][H]
-  __shared__ float sgs[kSmallV];
-  __shared__ float sgw[kSmallV + 1];
-  for (int e = threadIdx.x; e < V * S * H3; e += kSmallT) sC[e] = C_all[e];
-  for (int e = threadIdx.x; e < V * S * H; e += kSmallT) { sHp[e] = Hp_all[e]; sHs[e] = H_seq[e]; }
+  float* sg = sdh + RH;            // G
+  float* sz = sg + RH;
+  float* sr = sz + RH;
+  float* srh = sr + RH;
+  float* sdaz = srh + RH;
+  float* sdah = sdaz + RH;
+  float* sdar = sdah + RH;
+  float* sdhn = sdar + RH;
+  float* sC = sdhn + RH;                     // [Vl][S][3H]
+  float* sHp = sC + (size_t)RB * S * H3;     // [Vl][S][H]
+  float* sHs = sHp + (size_t)RB * S * H;     // [S][Vl][H]
+  __shared__ float sgs[kSmallT];
+  __shared__ float sgw[65];
+  for (int e = threadIdx.x; e < Vl * S * H3; e += kSmallT) sC[e] = C_all[(int64_t)r0 * S * H3 + e];
+  for (int e = threadIdx.x; e < Vl * S * H; e += kSmallT) {
+    sHp[e] = Hp_all[(int64_t)r0 * S * H + e];
+    const int t = e / VH, rem = e % VH;
+    sHs[e] = H_seq[((int64_t)t * V + r0) * H + rem];
+  }
   for (int e = threadIdx.x; e < 3 * LG; e += kSmallT) sL[e] = L[e];
   for (int e = threadIdx.x; e < VH; e += kSmallT) sdh[e] = 0.f;
   for (int j = threadIdx.x; j <= H; j += kSmallT) sgw[j] = 0.f;
@@ -2128,24 +2136,24 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, const f
   const float bo = b_o[0];
   __syncthreads();
   for (int t = S - 1; t >= 0; --t) {
-    for (int v = threadIdx.x; v < V; v += kSmallT) {            // head gradient scale of row v
-      const float* ht = sHs + ((int64_t)t * V + v) * H;
+    for (int v = threadIdx.x; v < Vl; v += kSmallT) {           // head gradient scale of row v
+      const float* ht = sHs + ((int64_t)t * Vl + v) * H;
       float d = 0.f;
 #pragma unroll
       for (int j = 0; j < H; ++j) d = fmaf(fmaxf(ht[j], 0.f), w_o[j], d);
-      sgs[v] = 2.0f * ((d + bo) - Yall[(int64_t)v * S + t]) * inv_vn;
+      sgs[v] = 2.0f * ((d + bo) - Yall[(int64_t)(r0 + v) * S + t]) * inv_vn;
     }
     __syncthreads();
     if (threadIdx.x <= H) {                                     // dw_o, db_o partials (rows in order)
       const int j = threadIdx.x;
       float acc = sgw[j];
-      for (int v = 0; v < V; ++v)
-        acc += j < H ? sgs[v] * fmaxf(sHs[((int64_t)t * V + v) * H + j], 0.f) : sgs[v];
+      for (int v = 0; v < Vl; ++v)
+        acc += j < H ? sgs[v] * fmaxf(sHs[((int64_t)t * Vl + v) * H + j], 0.f) : sgs[v];
       sgw[j] = acc;
     }
     for (int e = threadIdx.x; e < VH; e += kSmallT) {          // G, z, r, r⊙h
       const int v = e / H, j = e % H;
-      const float ht = sHs[((int64_t)t * V + v) * H + j];
+      const float ht = sHs[((int64_t)t * Vl + v) * H + j];
       sg[e] = (ht > 0.f ? sgs[v] * w_o[j] : 0.f) + sdh[e];
       const float* c = sC + ((int64_t)v * S + t) * H3;
       const float* hv = sHp + ((int64_t)v * S + t) * H;
@@ -2164,7 +2172,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, const f
       sz[e] = z;
       sr[e] = r;
       srh[e] = r * hv[j];
-      RH_all[((int64_t)v * S + t) * H + j] = r * hv[j];
+      RH_all[((int64_t)(r0 + v) * S + t) * H + j] = r * hv[j];
     }
     __syncthreads();
     for (int e = threadIdx.x; e < VH; e += kSmallT) {          // candidate; da_z, da_h
@@ -2182,7 +2190,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, const f
       sdah[e] = dah;
       sdaz[e] = daz;
       sdhn[e] = g * z;
-      float* da = da_all + ((int64_t)v * S + t) * H3;
+      float* da = da_all + ((int64_t)(r0 + v) * S + t) * H3;
       da[j] = daz;
       da[2 * H + j] = dah;
     }
@@ -2202,11 +2210,11 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, const f
       const float dar = drh * h * r * (1.0f - r);
       sdar[e] = dar;
       sdhn[e] += drh * r + dhz;
-      const float nd = ndst[v];
-      float* dc = dC_all + ((int64_t)v * S + t) * H3;
+      const float nd = ndst[r0 + v];
+      float* dc = dC_all + ((int64_t)(r0 + v) * S + t) * H3;
       dc[i] = nd * dcz;
       dc[2 * H + i] = nd * dch;
-      da_all[((int64_t)v * S + t) * H3 + H + i] = dar;
+      da_all[((int64_t)(r0 + v) * S + t) * H3 + H + i] = dar;
     }
     __syncthreads();
     for (int e = threadIdx.x; e < VH; e += kSmallT) {          // dC_r, dH_r; dℓ/dH_{t-1}
@@ -2218,39 +2226,46 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, const f
         dcr = fmaf(a, Lr[i * H + j], dcr);
         dhr = fmaf(a, Lr[(H + i) * H + j], dhr);
       }
-      dC_all[((int64_t)v * S + t) * H3 + H + i] = ndst[v] * dcr;
+      dC_all[((int64_t)(r0 + v) * S + t) * H3 + H + i] = ndst[r0 + v] * dcr;
       sdh[e] = sdhn[e] + dhr;
     }
     __syncthreads();
   }
-  for (int j = threadIdx.x; j <= H; j += kSmallT) gpart[j] = sgw[j];
+  for (int j = threadIdx.x; j <= H; j += kSmallT) gpart[(int64_t)blockIdx.x * (H + 1) + j] = sgw[j];
 }
 
-static size_t small_fwd_smem(int V, int S, int H) {
-  return sizeof(float) * (6 * (size_t)H * H + 4 * (size_t)V * H + (size_t)V * S * 3 * H);
+static size_t small_fwd_smem(int RB, int S, int H) {
+  return sizeof(float) * (6 * (size_t)H * H + 4 * (size_t)RB * H + (size_t)RB * S * 3 * H);
 }
-static size_t small_bwd_smem(int V, int S, int H) {
-  return sizeof(float) * (6 * (size_t)H * H + 9 * (size_t)V * H + (size_t)V * S * 5 * H);
+static size_t small_bwd_smem(int RB, int S, int H) {
+  return sizeof(float) * (6 * (size_t)H * H + 9 * (size_t)RB * H + (size_t)RB * S * 5 * H);
 }
-// the one-CTA path stages the whole sequence's inputs in shared memory
-static bool small_seq(int V, int S, int H) {
-  return V <= kSmallV && (H == 16 || H == 32) && small_bwd_smem(V, S, H) <= 200 * 1024;
+// rows per CTA of the small-graph path: as many as fit the staged sequence (<= 200 KB)
+// and the thread block (RB·H <= kSmallT); 0 = use the tensor-core kernels
+static int small_rows(int V, int S, int H) {
+  if (V > kSmallMaxV || (H != 16 && H != 32)) return 0;
+  int rb = kSmallT / H;
+  while (rb > 0 && small_bwd_smem(rb, S, H) > 200 * 1024) --rb;
+  if (rb < 4) return 0;
+  if ((V + rb - 1) / rb > num_sms()) return 0;     // the head partials hold one slot per SM
+  return rb >= V ? V : rb;
 }
 
 stg_status tc_gru_seq_fwd(int V, int S, int H, const float* C_all, const float* H0, const float* L, const float* l,
                           float* H_seq, float* Hp_all, const float* Y_all, const float* w_o, const float* b_o,
                           double* lpart, int* nb_out, cudaStream_t s) {
-  if (small_seq(V, S, H)) {
-    const size_t smem = small_fwd_smem(V, S, H);
+  if (const int rb = small_rows(V, S, H)) {
+    const size_t smem = small_fwd_smem(rb, S, H);
+    const int nb = (V + rb - 1) / rb;
     if (H == 32) {
       STG_TRY(prep(k_seq_fwd_small<32>, smem));
-      k_seq_fwd_small<32><<<1, kSmallT, smem, s>>>(V, S, C_all, H0, L, l, H_seq, Hp_all, Y_all, w_o, b_o, lpart);
+      k_seq_fwd_small<32><<<nb, kSmallT, smem, s>>>(V, S, rb, C_all, H0, L, l, H_seq, Hp_all, Y_all, w_o, b_o, lpart);
     } else {
       STG_TRY(prep(k_seq_fwd_small<16>, smem));
-      k_seq_fwd_small<16><<<1, kSmallT, smem, s>>>(V, S, C_all, H0, L, l, H_seq, Hp_all, Y_all, w_o, b_o, lpart);
+      k_seq_fwd_small<16><<<nb, kSmallT, smem, s>>>(V, S, rb, C_all, H0, L, l, H_seq, Hp_all, Y_all, w_o, b_o, lpart);
     }
     count_launch();
-    *nb_out = 1;
+    *nb_out = nb;
     return check_launch("seq_fwd_small");
   }
   const int ntiles = (V + 127) / 128;
@@ -2281,19 +2296,20 @@ stg_status tc_gru_seq_bwd(int V, int S, int H, const float* C_all, const float* 
                           const float* L, const float* l, const float* ndst, const float* Y_all, const float* w_o,
                           const float* b_o, float inv_vn, float* dC_all, float* da_all, float* RH_all, float* gpart,
                           int* nb_out, cudaStream_t s) {
-  if (small_seq(V, S, H)) {
-    const size_t smem = small_bwd_smem(V, S, H);
+  if (const int rb = small_rows(V, S, H)) {
+    const size_t smem = small_bwd_smem(rb, S, H);
+    const int nb = (V + rb - 1) / rb;
     if (H == 32) {
       STG_TRY(prep(k_seq_bwd_small<32>, smem));
-      k_seq_bwd_small<32><<<1, kSmallT, smem, s>>>(V, S, C_all, Hp_all, H_seq, L, l, ndst, Y_all, w_o, b_o, inv_vn,
-                                                   dC_all, da_all, RH_all, gpart);
+      k_seq_bwd_small<32><<<nb, kSmallT, smem, s>>>(V, S, rb, C_all, Hp_all, H_seq, L, l, ndst, Y_all, w_o, b_o,
+                                                    inv_vn, dC_all, da_all, RH_all, gpart);
     } else {
       STG_TRY(prep(k_seq_bwd_small<16>, smem));
-      k_seq_bwd_small<16><<<1, kSmallT, smem, s>>>(V, S, C_all, Hp_all, H_seq, L, l, ndst, Y_all, w_o, b_o, inv_vn,
-                                                   dC_all, da_all, RH_all, gpart);
+      k_seq_bwd_small<16><<<nb, kSmallT, smem, s>>>(V, S, rb, C_all, Hp_all, H_seq, L, l, ndst, Y_all, w_o, b_o,
+                                                    inv_vn, dC_all, da_all, RH_all, gpart);
     }
     count_launch();
-    *nb_out = 1;
+    *nb_out = nb;
     return check_launch("seq_bwd_small");
   }
   const int ntiles = (V + 127) / 128;

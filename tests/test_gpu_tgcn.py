@@ -232,3 +232,28 @@ def test_train_sequence_batched_rejects(stg):
     with pytest.raises(stg.StgError) as e:
         _run_batched(stg, g, cfg, pg, X, Y, torch.zeros(cfg.V, cfg.H, device="cuda"), 65)
     assert e.value.status == 1
+
+
+@pytest.mark.parametrize("V,H,S", [(100, 16, 16), (128, 32, 4), (47, 32, 9)])
+def test_train_sequence_batched_small_graph_row_blocks(stg, V, H, S):
+    """The one-CTA-per-row-block SIMT recurrence of small graphs (V <= 128; several
+    CTAs when V·H exceeds one block) against the fp64 oracle sequence."""
+    from types import SimpleNamespace
+    F = 8
+    s, d = gen.random_edges(V, V, 4 * V, loops=False)
+    cfg = SimpleNamespace(V=V, F=F, H=H)
+    g = stg.stg_static_graph_create(V, s, d, stg.STG_SELF_LOOPS)
+    ref = oracle.static_graph(V, s, d, self_loops=True)
+    p, pg = _params(F, H, 5)
+    Xs = [gen.uniform_pm1(60 + i, 61, V * F).reshape(V, F) for i in range(S)]
+    Ys = [gen.uniform_pm1(70 + i, 71, V) for i in range(S)]
+    H0 = gen.uniform_pm1(8, 8, V * H).reshape(V, H)
+    loss, grads, dw, db, Hseq = _run_batched(stg, g, cfg, pg, [to_gpu(x) for x in Xs], [to_gpu(y) for y in Ys],
+                                             to_gpu(H0), S)
+    rl, rg, rH = oracle.train_sequence([ref] * S, [ref] * S, p, Xs, Ys, H0)
+    assert abs(loss - rl) <= 1e-5 * abs(rl), (loss, rl)
+    assert np.max(np.abs(Hseq[-1].cpu().numpy() - rH)) <= H_TOL
+    for k in ("W", "b", "L", "l"):
+        assert _normwise(grads[k].cpu().numpy(), rg[k]) <= g_tol(V * S), k
+    assert _normwise(dw.cpu().numpy(), rg["w_o"]) <= g_tol(V * S)
+    assert _normwise(db.cpu().numpy(), rg["b_o"]) <= g_tol(V * S)
