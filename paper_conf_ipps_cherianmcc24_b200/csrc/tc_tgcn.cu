@@ -2016,7 +2016,21 @@ namespace stg {
 // each of its MMA phases is a full round trip; here a timestep is a few block-wide
 // phases of 2H-term dot products.  Same outputs, layouts and fused head as the
 // tcgen05 kernels; per-CTA head partials (nb = number of CTAs).
-constexpr int kSmallT = 512, kSmallMaxV = 128;   // measured: beyond one tile the tcgen05 kernels win (C2, C3)
+constexpr int kSmallT = 512, kSmallMaxV = 4096;
+
+// block-wide copy of n floats (n % 4 == 0, 16-byte aligned) with several loads in flight
+__device__ __forceinline__ void stage_f4(float* __restrict__ dst, const float* __restrict__ src, int n) {
+  const float4* s4 = reinterpret_cast<const float4*>(src);
+  float4* d4 = reinterpret_cast<float4*>(dst);
+  const int n4 = n >> 2;
+  int e = threadIdx.x;
+  for (; e + 3 * kSmallT < n4; e += 4 * kSmallT) {
+    const float4 a = __ldg(s4 + e), b = __ldg(s4 + e + kSmallT), c = __ldg(s4 + e + 2 * kSmallT),
+                 d = __ldg(s4 + e + 3 * kSmallT);
+    d4[e] = a; d4[e + kSmallT] = b; d4[e + 2 * kSmallT] = c; d4[e + 3 * kSmallT] = d;
+  }
+  for (; e < n4; e += kSmallT) d4[e] = __ldg(s4 + e);
+}
 
 template <int H>
 __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, int RB, const float* __restrict__ C_all,
@@ -2035,9 +2049,14 @@ __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, int RB,
   float* sn = srh + RB * H;        // H_t
   float* sC = sn + RB * H;         // this CTA's rows of C_all [Vl][S][3H]
   __shared__ double sloss[kSmallT];
-  for (int e = threadIdx.x; e < Vl * S * H3; e += kSmallT) sC[e] = C_all[(int64_t)r0 * S * H3 + e];
-  for (int e = threadIdx.x; e < 3 * LG; e += kSmallT) sL[e] = L[e];
-  for (int e = threadIdx.x; e < VH; e += kSmallT) sh[e] = H0[(int64_t)r0 * H + e];
+  __shared__ float sl[3 * H], swo[H];
+  float* sY = sC + (size_t)RB * S * H3;      // [Vl][S]
+  stage_f4(sC, C_all + (int64_t)r0 * S * H3, Vl * S * H3);
+  for (int e = threadIdx.x; e < Vl * S; e += kSmallT) sY[e] = Yall[(int64_t)r0 * S + e];
+  for (int e = threadIdx.x; e < 3 * H; e += kSmallT) sl[e] = l[e];
+  for (int e = threadIdx.x; e < H; e += kSmallT) swo[e] = w_o[e];
+  stage_f4(sL, L, 3 * LG);
+  stage_f4(sh, H0 + (int64_t)r0 * H, VH);
   for (int v = threadIdx.x; v < Vl; v += kSmallT) sloss[v] = 0.0;
   const float* Lz = sL; const float* Lr = sL + LG; const float* Lh = sL + 2 * LG;
   const float bo = b_o[0];
@@ -2047,7 +2066,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, int RB,
       const int v = e / H, j = e % H;
       const float* c = sC + ((int64_t)v * S + t) * H3;
       const float* hv = sh + v * H;
-      float az = l[j], ar = l[H + j];
+      float az = sl[j], ar = sl[H + j];
 #pragma unroll
       for (int i = 0; i < H; ++i) {
         az = fmaf(c[i], Lz[i * H + j], az);
@@ -2066,7 +2085,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, int RB,
     for (int e = threadIdx.x; e < VH; e += kSmallT) {          // candidate, H_t
       const int v = e / H, j = e % H;
       const float* c = sC + ((int64_t)v * S + t) * H3 + 2 * H;
-      float ah = l[2 * H + j];
+      float ah = sl[2 * H + j];
 #pragma unroll
       for (int i = 0; i < H; ++i) ah = fmaf(c[i], Lh[i * H + j], ah);
 #pragma unroll
@@ -2080,8 +2099,8 @@ __global__ void __launch_bounds__(kSmallT) k_seq_fwd_small(int V, int S, int RB,
     for (int v = threadIdx.x; v < Vl; v += kSmallT) {           // fused head: loss of row v at t
       float d = 0.f;
 #pragma unroll
-      for (int j = 0; j < H; ++j) d = fmaf(fmaxf(sn[v * H + j], 0.f), w_o[j], d);
-      const float e = (d + bo) - Yall[(int64_t)(r0 + v) * S + t];
+      for (int j = 0; j < H; ++j) d = fmaf(fmaxf(sn[v * H + j], 0.f), swo[j], d);
+      const float e = (d + bo) - sY[v * S + t];
       sloss[v] += (double)e * (double)e;
     }
     for (int e = threadIdx.x; e < VH; e += kSmallT) sh[e] = sn[e];
@@ -2123,13 +2142,16 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB,
   float* sHs = sHp + (size_t)RB * S * H;     // [S][Vl][H]
   __shared__ float sgs[kSmallT];
   __shared__ float sgw[65];
-  for (int e = threadIdx.x; e < Vl * S * H3; e += kSmallT) sC[e] = C_all[(int64_t)r0 * S * H3 + e];
-  for (int e = threadIdx.x; e < Vl * S * H; e += kSmallT) {
-    sHp[e] = Hp_all[(int64_t)r0 * S * H + e];
-    const int t = e / VH, rem = e % VH;
-    sHs[e] = H_seq[((int64_t)t * V + r0) * H + rem];
-  }
-  for (int e = threadIdx.x; e < 3 * LG; e += kSmallT) sL[e] = L[e];
+  __shared__ float sl[3 * H], swo[H], snd[kSmallT];
+  float* sY = sHs + (size_t)RB * S * H;      // [Vl][S]
+  for (int e = threadIdx.x; e < Vl * S; e += kSmallT) sY[e] = Yall[(int64_t)r0 * S + e];
+  for (int e = threadIdx.x; e < 3 * H; e += kSmallT) sl[e] = l[e];
+  for (int e = threadIdx.x; e < H; e += kSmallT) swo[e] = w_o[e];
+  for (int v = threadIdx.x; v < Vl; v += kSmallT) snd[v] = ndst[r0 + v];
+  stage_f4(sC, C_all + (int64_t)r0 * S * H3, Vl * S * H3);
+  stage_f4(sHp, Hp_all + (int64_t)r0 * S * H, Vl * S * H);
+  for (int t = 0; t < S; ++t) stage_f4(sHs + (size_t)t * VH, H_seq + ((int64_t)t * V + r0) * H, VH);
+  stage_f4(sL, L, 3 * LG);
   for (int e = threadIdx.x; e < VH; e += kSmallT) sdh[e] = 0.f;
   for (int j = threadIdx.x; j <= H; j += kSmallT) sgw[j] = 0.f;
   const float* Lz = sL; const float* Lr = sL + LG; const float* Lh = sL + 2 * LG;
@@ -2140,8 +2162,8 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB,
       const float* ht = sHs + ((int64_t)t * Vl + v) * H;
       float d = 0.f;
 #pragma unroll
-      for (int j = 0; j < H; ++j) d = fmaf(fmaxf(ht[j], 0.f), w_o[j], d);
-      sgs[v] = 2.0f * ((d + bo) - Yall[(int64_t)(r0 + v) * S + t]) * inv_vn;
+      for (int j = 0; j < H; ++j) d = fmaf(fmaxf(ht[j], 0.f), swo[j], d);
+      sgs[v] = 2.0f * ((d + bo) - sY[v * S + t]) * inv_vn;
     }
     __syncthreads();
     if (threadIdx.x <= H) {                                     // dw_o, db_o partials (rows in order)
@@ -2154,10 +2176,10 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB,
     for (int e = threadIdx.x; e < VH; e += kSmallT) {          // G, z, r, r⊙h
       const int v = e / H, j = e % H;
       const float ht = sHs[((int64_t)t * Vl + v) * H + j];
-      sg[e] = (ht > 0.f ? sgs[v] * w_o[j] : 0.f) + sdh[e];
+      sg[e] = (ht > 0.f ? sgs[v] * swo[j] : 0.f) + sdh[e];
       const float* c = sC + ((int64_t)v * S + t) * H3;
       const float* hv = sHp + ((int64_t)v * S + t) * H;
-      float az = l[j], ar = l[H + j];
+      float az = sl[j], ar = sl[H + j];
 #pragma unroll
       for (int i = 0; i < H; ++i) {
         az = fmaf(c[i], Lz[i * H + j], az);
@@ -2178,7 +2200,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB,
     for (int e = threadIdx.x; e < VH; e += kSmallT) {          // candidate; da_z, da_h
       const int v = e / H, j = e % H;
       const float* c = sC + ((int64_t)v * S + t) * H3 + 2 * H;
-      float ah = l[2 * H + j];
+      float ah = sl[2 * H + j];
 #pragma unroll
       for (int i = 0; i < H; ++i) ah = fmaf(c[i], Lh[i * H + j], ah);
 #pragma unroll
@@ -2210,7 +2232,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB,
       const float dar = drh * h * r * (1.0f - r);
       sdar[e] = dar;
       sdhn[e] += drh * r + dhz;
-      const float nd = ndst[r0 + v];
+      const float nd = snd[v];
       float* dc = dC_all + ((int64_t)(r0 + v) * S + t) * H3;
       dc[i] = nd * dcz;
       dc[2 * H + i] = nd * dch;
@@ -2226,7 +2248,7 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB,
         dcr = fmaf(a, Lr[i * H + j], dcr);
         dhr = fmaf(a, Lr[(H + i) * H + j], dhr);
       }
-      dC_all[((int64_t)(r0 + v) * S + t) * H3 + H + i] = ndst[r0 + v] * dcr;
+      dC_all[((int64_t)(r0 + v) * S + t) * H3 + H + i] = snd[v] * dcr;
       sdh[e] = sdhn[e] + dhr;
     }
     __syncthreads();
@@ -2235,19 +2257,29 @@ __global__ void __launch_bounds__(kSmallT) k_seq_bwd_small(int V, int S, int RB,
 }
 
 static size_t small_fwd_smem(int RB, int S, int H) {
-  return sizeof(float) * (6 * (size_t)H * H + 4 * (size_t)RB * H + (size_t)RB * S * 3 * H);
+  return sizeof(float) * (6 * (size_t)H * H + 4 * (size_t)RB * H + (size_t)RB * S * (3 * H + 1));
 }
 static size_t small_bwd_smem(int RB, int S, int H) {
-  return sizeof(float) * (6 * (size_t)H * H + 9 * (size_t)RB * H + (size_t)RB * S * 5 * H);
+  return sizeof(float) * (6 * (size_t)H * H + 9 * (size_t)RB * H + (size_t)RB * S * (5 * H + 1));
 }
 // rows per CTA of the small-graph path: as many as fit the staged sequence (<= 200 KB)
 // and the thread block (RB·H <= kSmallT); 0 = use the tensor-core kernels
 static int small_rows(int V, int S, int H) {
   if (V > kSmallMaxV || (H != 16 && H != 32)) return 0;
-  int rb = kSmallT / H;
+  // about two warps of (row, column) work per CTA: a timestep is a chain of dependent
+  // block-wide phases, so few rows per CTA spread over many SMs beat one full block
+  // (C1: 4 rows/CTA 4.64 ms vs 20 rows/CTA 6.10 ms per epoch)
+  int rb = 64 / H;
   while (rb > 0 && small_bwd_smem(rb, S, H) > 200 * 1024) --rb;
-  if (rb < 4) return 0;
-  if ((V + rb - 1) / rb > num_sms()) return 0;     // the head partials hold one slot per SM
+  if (rb < 1) return 0;
+  static const int forced = [] {                   // experiments: STG_SMALL_RB=rows per CTA
+    const char* e = getenv("STG_SMALL_RB");
+    return e ? atoi(e) : 0;
+  }();
+  if (forced > 0 && forced < rb) rb = forced;
+  // beyond about two waves of CTAs the tcgen05 tiles win (measured: C3, V = 319, 160 CTAs:
+  // 404 vs 505 ms per epoch; C2, V = 1068, 534 CTAs: 24.8 vs 21.7 ms)
+  if ((V + rb - 1) / rb > 2 * num_sms()) return 0;
   return rb >= V ? V : rb;
 }
 

@@ -1567,7 +1567,7 @@ stg_status stg_tgcn_train_sequence_batched(const stg_graph* graph, int32_t S, co
   const size_t VS = (size_t)V * S;
   cudaStream_t s = (cudaStream_t)stream;
   TgcnWs& ws = stack->ws;
-  const int nbmax = num_sms();
+  const int nbmax = std::max(num_sms(), V);          // head partials: one per CTA (<= V for the small-graph kernels)
   STG_TRY(ws.sX.alloc(VS * F)); STG_TRY(ws.sY.alloc(VS)); STG_TRY(ws.sb.alloc((size_t)S * H3));
   STG_TRY(ws.sP.alloc(VS * H3)); STG_TRY(ws.sC.alloc(VS * H3)); STG_TRY(ws.sHp.alloc(VS * H));
   STG_TRY(ws.sdC.alloc(VS * H3)); STG_TRY(ws.sdP.alloc(VS * H3)); STG_TRY(ws.sda.alloc(VS * H3));
