@@ -2262,24 +2262,21 @@ static size_t small_fwd_smem(int RB, int S, int H) {
 static size_t small_bwd_smem(int RB, int S, int H) {
   return sizeof(float) * (6 * (size_t)H * H + 9 * (size_t)RB * H + (size_t)RB * S * (5 * H + 1));
 }
-// rows per CTA of the small-graph path: as many as fit the staged sequence (<= 200 KB)
-// and the thread block (RB·H <= kSmallT); 0 = use the tensor-core kernels
+// Rows per CTA of the small-graph path (0 = use the tcgen05 kernels).  A timestep is a
+// latency chain of block-wide phases, so the rows are spread over one wave of CTAs with
+// as few rows per CTA as that allows (at least 64/H, about two warps of (row, column)
+// work).  Measured per epoch: C1 (V = 20) 4 rows 4.6 ms vs 20 rows 6.1 ms vs tcgen05
+// 7.1 ms; C3 (V = 319) 4 rows 364 ms, 2 rows 404 ms, tcgen05 505 ms; C2 (V = 1068) 8 rows
+// 19.3 ms vs tcgen05 21.7 ms, 2 rows (534 CTAs) 24.8 ms.  Beyond one wave of at most
+// kSmallT/H rows per CTA (or the shared-memory budget) the tcgen05 tiles take over.
 static int small_rows(int V, int S, int H) {
   if (V > kSmallMaxV || (H != 16 && H != 32)) return 0;
-  // about two warps of (row, column) work per CTA: a timestep is a chain of dependent
-  // block-wide phases, so few rows per CTA spread over many SMs beat one full block
-  // (C1: 4 rows/CTA 4.64 ms vs 20 rows/CTA 6.10 ms per epoch)
-  int rb = 64 / H;
-  while (rb > 0 && small_bwd_smem(rb, S, H) > 200 * 1024) --rb;
-  if (rb < 1) return 0;
   static const int forced = [] {                   // experiments: STG_SMALL_RB=rows per CTA
     const char* e = getenv("STG_SMALL_RB");
     return e ? atoi(e) : 0;
   }();
-  if (forced > 0 && forced < rb) rb = forced;
-  // beyond about two waves of CTAs the tcgen05 tiles win (measured: C3, V = 319, 160 CTAs:
-  // 404 vs 505 ms per epoch; C2, V = 1068, 534 CTAs: 24.8 vs 21.7 ms)
-  if ((V + rb - 1) / rb > 2 * num_sms()) return 0;
+  int rb = forced > 0 ? forced : std::max(64 / H, (V + num_sms() - 1) / num_sms());
+  if (rb * H > kSmallT || small_bwd_smem(rb, S, H) > 200 * 1024) return 0;
   return rb >= V ? V : rb;
 }
 
