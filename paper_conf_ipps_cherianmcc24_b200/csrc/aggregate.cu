@@ -535,15 +535,26 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
   }
   const int64_t total = a.sched[3];
   const int4* items = reinterpret_cast<const int4*>(a.sched + kSchedHdr);
-  // Work groups: hub chunks (<= 64 edges each) a.hgrp per group, light rows
-  // a.lgrp per group (host-chosen so that small graphs still spread over many
-  // warps), so no warp walks a long single group while others idle.
+  // Work groups: hub chunks (<= 64 edges each) a.hgrp per group; then the light
+  // rows (degree order) in three tiers — n > kTierB: 4 per group, n > kTierC: 16,
+  // the rest a.lgrp (host-chosen so that small graphs still spread over many
+  // warps) — so no warp walks a long group of the heaviest light rows while
+  // others idle (<= 256 edges per group outside the hubs).
   const int64_t n_chunks = a.sched[1];
+  const int64_t tb = a.sched[4], tc = a.sched[5];
   const int64_t hg = a.hgrp, lg = a.lgrp;
+  constexpr int64_t ga = 4, gb = 16;
   const int64_t nhg = (n_chunks + hg - 1) / hg;
-  const uint32_t ngroups = (uint32_t)(nhg + (total - n_chunks + lg - 1) / lg);
-  auto gbase = [&](int64_t g) { return g < nhg ? g * hg : n_chunks + (g - nhg) * lg; };
-  auto gend = [&](int64_t g) { return g < nhg ? min((g + 1) * hg, n_chunks) : min(gbase(g) + lg, total); };
+  const int64_t nga = nhg + (tb - n_chunks + ga - 1) / ga;          // groups before tier B
+  const int64_t ngb = nga + (tc - tb + gb - 1) / gb;                // groups before tier C
+  const uint32_t ngroups = (uint32_t)(ngb + (total - tc + lg - 1) / lg);
+  auto gbase = [&](int64_t g) {
+    return g < nhg ? g * hg : (g < nga ? n_chunks + (g - nhg) * ga : (g < ngb ? tb + (g - nga) * gb : tc + (g - ngb) * lg));
+  };
+  auto gend = [&](int64_t g) {
+    return g < nhg ? min((g + 1) * hg, n_chunks)
+                   : (g < nga ? min(gbase(g) + ga, tb) : (g < ngb ? min(gbase(g) + gb, tc) : min(gbase(g) + lg, total)));
+  };
   const int c0y = blockIdx.y * a.wsplit;                       // this launch's column chunk
   const int Wl = min(a.wsplit, a.wtotal - c0y);
   float* const ybase = a.y + c0y;
@@ -920,7 +931,12 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
   if (ew && !(vec4 && a.sched && wsplit <= 128))
     return fail(STG_ERR_INVALID_ARG, "aggregate_weighted: needs W %% 4 == 0, W <= 512, 16-byte aligned rows "
                 "and a library view (schedule)");
-  if (peers || ew || (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128)) {
+  // below ~1M edges a single-launch-width aggregation is latency-bound and the
+  // pipelined row items (strategy 1) finish first (measured at W = 96: C4 0.024 vs
+  // 0.036 ms, C2 0.016 vs 0.030 ms); wide (column-chunked) launches keep the stream
+  const bool small_narrow = gv->num_edges < (int64_t(1) << 20) && nsplit == 1;
+  if (peers || ew ||
+      (vec4 && g_strategy == 2 && a.sched && wsplit > 4 * (g_tune.wmin / 4) && wsplit <= 128 && !small_narrow)) {
     STG_TRY(ws->queue.alloc(nsplit, s));
     STG_CUDA(cudaMemsetAsync(ws->queue.p, 0, sizeof(uint32_t) * nsplit, s));
     const int64_t pstride = chunks_bound * wsplit;               // the column chunks run concurrently
@@ -934,7 +950,7 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     int hgrp = kHubGroup, lgrp = 32;
     while (hgrp > 2 && (int64_t)hgrp * kHubChunk > target) hgrp >>= 1;
     while (lgrp > 4 && (int64_t)lgrp * avg > 2 * target) lgrp >>= 1;
-    const int64_t ngroups = ceil_div(chunks_bound, hgrp) + ceil_div(R, lgrp) + 1;   // bound on work groups
+    const int64_t ngroups = ceil_div(chunks_bound, hgrp) + ceil_div(R, 4) + 3;       // bound on work groups
     const int64_t blocks = std::min<int64_t>(occupancy_grid((const void*)fn), ceil_div(ngroups, 8) + 1);
     const int32_t* hids = backward ? gv->out_ids : gv->in_ids;
     Agg2Args b{};

@@ -201,12 +201,26 @@ __global__ void k_items(const int32_t* __restrict__ ids, const int32_t* __restri
     } else {
       const int32_t v = ids[n_hub + (i - n_chunks)];
       const int32_t rb = rowptr[v];
-      items[i] = make_int4(v, rb, rowptr[v + 1] - rb, -1);
+      const int32_t n = rowptr[v + 1] - rb;
+      items[i] = make_int4(v, rb, n, -1);
+      // tier boundaries: light items are in non-increasing n (degree order)
+      int32_t np = INT32_MAX;
+      if (i > n_chunks) {
+        const int32_t vp = ids[n_hub + (i - 1 - n_chunks)];
+        np = rowptr[vp + 1] - rowptr[vp];
+      }
+      if (np > kTierB && n <= kTierB) sched[4] = (int32_t)i;
+      if (np > kTierC && n <= kTierC) sched[5] = (int32_t)i;
+      if (i == total - 1) {                          // tiers that reach the end are empty
+        if (n > kTierB) sched[4] = (int32_t)total;
+        if (n > kTierC) sched[5] = (int32_t)total;
+      }
     }
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     sched[2] = (int32_t)coff;
     sched[3] = (int32_t)total;
+    if (total == n_chunks) { sched[4] = (int32_t)total; sched[5] = (int32_t)total; }
   }
 }
 

@@ -22,10 +22,16 @@ inline int64_t sched_cap(int64_t E) { return E / (kHubChunk + 1) + 2; }
 //   sched[1] = n_chunks total hub chunks
 //   sched[2] = cptr_off offset (in int32) of cptr[0..n_hub] (exclusive chunk prefix)
 //   sched[3] = n_items  = n_chunks + V - n_hub
-//   sched[4 ..]         = items, int4 {v, beg, n, hub} in node_ids order: hub
+//   sched[4] = first item of the light rows with n <= kTierB (items are in degree order)
+//   sched[5] = first item of the light rows with n <= kTierC
+//   sched[6], sched[7]  unused (items stay 16-byte aligned)
+//   sched[8 ..]         = items, int4 {v, beg, n, hub} in node_ids order: hub
 //                         chunks first (hub = index into ids / cptr), then the
 //                         light rows (hub = -1).  n <= kHubChunk.
-constexpr int64_t kSchedHdr = 4;
+constexpr int64_t kSchedHdr = 8;
+// light-row tiers of the edge-stream work groups (aggregate.cu): rows with more edges go
+// in smaller groups so that no warp walks a long group of the heaviest light rows
+constexpr int32_t kTierB = 16, kTierC = 4;
 inline int64_t sched_items_cap(int64_t V, int64_t E) { return V + E / kHubChunk + 2; }
 inline int64_t sched_cptr_off(int64_t V, int64_t E) { return kSchedHdr + 4 * sched_items_cap(V, E); }
 inline int64_t sched_size(int64_t V, int64_t E) {

@@ -23,10 +23,15 @@ ap.add_argument("--only", default=None, help="run only configs whose name contai
 a = ap.parse_args()
 
 cfg = gen.CONFIGS[a.config]
-d = gen.dtdg(cfg)
-g = stg.stg_dtdg_create(cfg.V, d.T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src, d.del_dst,
-                        stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS)
-v = stg.stg_dtdg_get_snapshot(g, a.t)
+if cfg.kind == "static":
+    s_e, d_e = gen.static_edges(cfg)
+    g = stg.stg_static_graph_create(cfg.V, s_e, d_e, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS)
+    v = g.view()
+else:
+    d = gen.dtdg(cfg)
+    g = stg.stg_dtdg_create(cfg.V, d.T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                            d.del_dst, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS)
+    v = stg.stg_dtdg_get_snapshot(g, a.t)
 V, E, W = v.num_nodes, v.num_edges, a.W
 torch.manual_seed(0)
 x = torch.rand(V, W, device="cuda") * 2 - 1
