@@ -172,7 +172,8 @@ template <int N>
 __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int Kp, const float* __restrict__ X,
                                                               const float* __restrict__ W,
                                                               const float* __restrict__ rs, float* __restrict__ P,
-                                                              int dbg, int rs_div) {
+                                                              int dbg, int rs_div,
+                                                              const __grid_constant__ CUtensorMap tmP, int box) {
   extern __shared__ __align__(128) unsigned char sm[];
   __shared__ uint64_t full[kXwStages], empty[kXwStages], tfull[2], tempty[2];
   __shared__ uint32_t tslot;
@@ -230,7 +231,7 @@ __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int 
         tc::commit(&tfull[st]);
       }
     }
-  } else if (warp < 4) {                             // ---- epilogue
+  } else if (warp < 4 && !box) {                     // ---- epilogue (staged row stores)
     float4* stage = ostage + warp * 32 * tc::kStagePitch<NQ>;
     int i = 0;
     for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
@@ -259,6 +260,30 @@ __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int 
         __syncwarp();
       }
     }
+  } else if (warp < 4 && box) {                      // ---- epilogue, TMA box stores
+    unsigned char* obuf = reinterpret_cast<unsigned char*>(
+        (reinterpret_cast<uintptr_t>(abase + (size_t)kXwStages * 2 * ABYTES) + 1023) & ~uintptr_t(1023)) + warp * 4096;
+    int oslot = 0;
+    int i = 0;
+    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+      const int b = i & 1, kb = i >> 1;
+      const int row = tile * 128 + threadIdx.x;
+      const float sc = (rs && row < V) ? __ldg(rs + row / rs_div) : 1.0f;
+      tc::mbar_wait(&tfull[b], kb & 1);
+      tc::fence_after();
+      const int wr0 = tile * 128 + warp * 32;
+#pragma unroll
+      for (int c0 = 0; c0 < N; c0 += 16) {               // TMEM -> registers -> swizzled box -> TMA store
+        float v[16];
+        tmem_row_load<16>(tm + b * NC, c0, v);
+        if (c0 + 16 >= N) {                               // accumulator b fully read: release it early
+          tc::fence_before();
+          tc::mbar_arrive(&tempty[b]);
+        }
+        tc::warp_box_store<16>(obuf, oslot, v, sc, &tmP, c0, wr0);
+      }
+    }
+    if ((threadIdx.x & 31) == 0) tc::bulk_wait_all();  // output boxes written before the CTA exits
   }
   tc::fence_before();
   __syncthreads();
@@ -1809,16 +1834,22 @@ stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const floa
   const int ntiles = (V + 127) / 128;
   if (Kp <= 64) {                     // pipelined kernel (2-stage ring of 128 x Kp tiles + output stage)
     const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)kXwStages * 2 * 128 * Kp * 4 +
-                        (size_t)128 * (N / 4 + 1 + ((N / 4) & 1)) * 16;
+                        std::max<size_t>((size_t)128 * (N / 4 + 1 + ((N / 4) & 1)) * 16, 4 * 4096 + 1024);
     const int nb = std::min(ntiles, num_sms());
     const char* dv = getenv("STG_XW_DEBUG");       // timing experiments only: skip parts of the pipeline
     const int dbg = dv ? atoi(dv) : 0;
+    static const int box = [] {                    // epilogue: TMA box stores (1) or staged row stores (0)
+      const char* e = getenv("STG_XW_BOXSTORE");
+      return e ? atoi(e) : 1;
+    }();
+    CUtensorMap tmP;
+    STG_TRY(make_tmap_f32_store(&tmP, P, (uint64_t)V, (uint64_t)N, (uint64_t)N, 16, 32));
     if (H == 32) {
       STG_TRY(prep(k_tc_xw_pipe<96>, smem));
-      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div);
+      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div, tmP, box);
     } else {
       STG_TRY(prep(k_tc_xw_pipe<48>, smem));
-      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div);
+      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div, tmP, box);
     }
   } else {                            // 64 < F <= 128: one tile per CTA at a time
     if (rs_div != 1) return fail(STG_ERR_INVALID_ARG, "tc_xw: row-scale divisor needs F <= 64");
