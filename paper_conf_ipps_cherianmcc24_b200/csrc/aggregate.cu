@@ -808,8 +808,11 @@ int max_blocks_for(KernelFn fn) {
 // Work decomposition (stg_aggregate_set_strategy) and strategy-2 tunables.
 static int g_strategy = 2;
 struct AggTune {
-  int d = 16;        // rows in flight per warp (stream kernel)
-  int minb = 3;      // min resident blocks per SM (register budget of the stream kernel)
+  // rows in flight per warp and min resident blocks per SM (register budget) of the
+  // stream kernel: with the light-row tiers balancing the groups, 48 warps x 4 rows beat
+  // 24 x 16 (C5 W = 96: 0.443 vs 0.477 ms; W = 64: 0.357 vs 0.418 ms)
+  int d = 4;
+  int minb = 6;
   int wmin = 32;     // stream kernel for wmin < W_launch <= 128
 };
 static AggTune g_tune;

@@ -69,7 +69,7 @@ configs = [("s0", 0, {}), ("s1", 1, {})]
 for d, mb in ((4, 6), (8, 4), (16, 2), (16, 3)):
     configs.append(("s2 d%d minb%d" % (d, mb), 2, {0: d, 1: mb}))
 configs.append(("s2 d16 minb3 wmin64", 2, {0: 16, 1: 3, 2: 64}))
-defaults = {0: 16, 1: 3, 2: 32}
+defaults = {0: 4, 1: 6, 2: 32}
 if a.only:
     configs = [c for c in configs if a.only in c[0]]
 for name, strat, params in configs:
