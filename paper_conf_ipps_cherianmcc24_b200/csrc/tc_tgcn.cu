@@ -1165,8 +1165,9 @@ __global__ void __launch_bounds__(kAtbThreads, 1) k_tc_atb(const AtbArgs p) {
 // corresponding D rows are garbage that is never read (rows are independent).
 // A slot is a TMA box or the static "ones" box (1.0 in feature 0 of every row:
 // the Σ_rows term of dl).  Warp 0 issues the TMA, warp 1 the MMAs, warps 2-5
-// convert and run the epilogue; an S-stage ring overlaps loads, conversion and
-// MMAs.  Each CTA accumulates its tiles (grid-stride, fixed) in TMEM and
+// convert and run the epilogue.  The raw (hi) boxes sit in an S-stage TMA ring;
+// lo is written into a separate 2-slot ring (a tile is converted just before its
+// MMAs), so the shared memory goes to loads in flight rather than to lo copies.  Each CTA accumulates its tiles (grid-stride, fixed) in TMEM and
 // writes its partial; k_tc_sum_parts adds the partials in a fixed order.
 struct AtbSpec2 {
   int V;
@@ -1190,21 +1191,22 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   constexpr int BOX = RT * 32 * 4;
   extern __shared__ unsigned char sm_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
-  __shared__ uint64_t full[S], conv[S], empty[S], done, init_bar;
+  __shared__ uint64_t full[S], empty[S], conv[2], lfree[2], done, init_bar;
   __shared__ uint32_t tslot;
   const int na = sp.na, nsa = sp.nsa;
   const int nbox = nsa + NB;                       // box slots per stage
-  const size_t half = (size_t)nbox * BOX;          // hi region of a stage; lo follows
-  auto hi = [&](int st, int bx) { return sm + (size_t)st * 2 * half + (size_t)bx * BOX; };
-  auto lo = [&](int st, int bx) { return sm + (size_t)st * 2 * half + half + (size_t)bx * BOX; };
+  const size_t half = (size_t)nbox * BOX;          // one stage (hi ring) or one lo slot
+  auto hi = [&](int st, int bx) { return sm + (size_t)st * half + (size_t)bx * BOX; };
+  auto lo = [&](int ls, int bx) { return sm + (size_t)(S + ls) * half + (size_t)bx * BOX; };
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   auto map_of = [&](int m) -> const CUtensorMap* { return m == 0 ? &m0 : (m == 1 ? &m1 : (m == 2 ? &m2 : &m3)); };
-  for (size_t e = threadIdx.x; e < (size_t)S * 2 * half / 16; e += blockDim.x)   // lo of the ones box stays 0
+  for (size_t e = threadIdx.x; e < (size_t)(S + 2) * half / 16; e += blockDim.x)   // lo of the ones box stays 0
     reinterpret_cast<float4*>(sm)[e] = make_float4(0.f, 0.f, 0.f, 0.f);
   const uint32_t tcols = na * N <= 128 ? 128 : 256;
   if (warp == 1) tc::tmem_alloc(&tslot, tcols);
   if (threadIdx.x == 0) {
-    for (int st = 0; st < S; ++st) { tc::mbar_init(&full[st], 1); tc::mbar_init(&conv[st], 128); tc::mbar_init(&empty[st], 1); }
+    for (int st = 0; st < S; ++st) { tc::mbar_init(&full[st], 1); tc::mbar_init(&empty[st], 1); }
+    for (int ls = 0; ls < 2; ++ls) { tc::mbar_init(&conv[ls], 128); tc::mbar_init(&lfree[ls], 1); }
     tc::mbar_init(&done, 1); tc::mbar_init(&init_bar, 1);
     tc::fence_mbar_init();
   }
@@ -1244,12 +1246,12 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
     if (lane == 0) {
       const uint32_t idesc = tc::idesc_tf32(128, N, 1, 1);
       for (int i = 0; i < my_tiles; ++i) {
-        const int st = i % S, kk = i / S;
-        tc::mbar_wait(&conv[st], kk & 1);
+        const int st = i % S, ls = i & 1;
+        tc::mbar_wait(&conv[ls], (i >> 1) & 1);
         tc::fence_after();
-        const uint32_t bh = tc::smem_u32(hi(st, nsa)), bl = tc::smem_u32(lo(st, nsa));
+        const uint32_t bh = tc::smem_u32(hi(st, nsa)), bl = tc::smem_u32(lo(ls, nsa));
         for (int a = 0; a < na; ++a) {
-          const uint32_t ah = tc::smem_u32(hi(st, sp.a_first[a])), al = tc::smem_u32(lo(st, sp.a_first[a]));
+          const uint32_t ah = tc::smem_u32(hi(st, sp.a_first[a])), al = tc::smem_u32(lo(ls, sp.a_first[a]));
           for (int k = 0; k < RT; k += 8) {                // 8 K-rows (1024 B) per MMA
             const uint32_t o = (uint32_t)k * 128;
             const uint64_t dah = tc::desc_mn_sw128_32b(ah + o, BOX), dal = tc::desc_mn_sw128_32b(al + o, BOX);
@@ -1261,18 +1263,20 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
           }
         }
         tc::commit(&empty[st]);
+        tc::commit(&lfree[ls]);
       }
       tc::commit(&done);
     }
   } else {                                           // ---- converters (warps 2-5), then epilogue
     const int ct = threadIdx.x - 64;
     for (int i = 0; i < my_tiles; ++i) {
-      const int st = i % S;
+      const int st = i % S, ls = i & 1;
       tc::mbar_wait(&full[st], (i / S) & 1);
+      if (i >= 2) tc::mbar_wait(&lfree[ls], ((i >> 1) - 1) & 1);   // MMAs of tile i-2 done with slot ls
       for (int bx = 0; bx < nbox; ++bx) {
         if (bx < nsa && sp.src_map[bx] < 0) continue;   // ones box: lo stays 0
         const float4* src = reinterpret_cast<const float4*>(hi(st, bx));
-        float4* dst = reinterpret_cast<float4*>(lo(st, bx));
+        float4* dst = reinterpret_cast<float4*>(lo(ls, bx));
 #pragma unroll
         for (int e = ct; e < BOX / 16; e += 128) {
           const float4 v = src[e];
@@ -1281,7 +1285,7 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
         }
       }
       tc::fence_proxy_async();
-      tc::mbar_arrive(&conv[st]);
+      tc::mbar_arrive(&conv[ls]);
     }
     // epilogue: this warp reads TMEM lane quarter warp % 4
     tc::mbar_wait(&done, 0);
@@ -1911,7 +1915,7 @@ stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float
   return check_launch("tc_gru_bwd");
 }
 
-int tc_atb_max_blocks() { return num_sms(); }
+int tc_atb_max_blocks() { return 2 * num_sms(); }   // k_tc_atb2 may run 2 CTAs per SM
 
 template <int N, int NA>
 static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
@@ -1919,7 +1923,7 @@ static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
   const size_t smem = 2 * (size_t)STAGE;
   STG_CUDA(cudaFuncSetAttribute(k_tc_atb<N, NA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int ntiles = (args.V + kRK - 1) / kRK;
-  int nb = std::min(ntiles, tc_atb_max_blocks());
+  int nb = std::min(ntiles, num_sms());
   if (nb < 1) nb = 1;
   k_tc_atb<N, NA><<<nb, kAtbThreads, smem, s>>>(args);
   count_launch();
@@ -1929,12 +1933,12 @@ static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
 
 template <int NB, int RT, int S>
 static stg_status atb2_launch(const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb_out,
-                              cudaStream_t s) {
+                              cudaStream_t s, int ctas_per_sm = 1) {
   const int nbox = sp.nsa + NB;
-  const size_t smem = (size_t)S * 2 * nbox * RT * 32 * 4 + 1024;
+  const size_t smem = (size_t)(S + 2) * nbox * RT * 32 * 4 + 1024;   // S hi stages + 2 lo slots
   STG_CUDA(cudaFuncSetAttribute(k_tc_atb2<NB, RT, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int ntiles = (sp.V + RT - 1) / RT;
-  const int nb = std::max(1, std::min(ntiles, tc_atb_max_blocks()));
+  const int nb = std::max(1, std::min(ntiles, ctas_per_sm * num_sms()));
   k_tc_atb2<NB, RT, S><<<nb, 192, smem, s>>>(m[0], m[1], m[2], m[3], ones, sp);
   count_launch();
   *nb_out = nb;
@@ -1948,15 +1952,19 @@ template <int NB>
 static stg_status atb2_stages(const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb,
                               cudaStream_t s) {
   constexpr int RT = kAtbRT;
-  const size_t stage = (size_t)2 * (sp.nsa + NB) * RT * 32 * 4;
+  const size_t stage = (size_t)(sp.nsa + NB) * RT * 32 * 4;   // one hi stage = one lo slot
   static const size_t cap = [] {                    // ring budget (experiments: STG_ATB_SMEM_KB)
     const char* v = getenv("STG_ATB_SMEM_KB");
     return (size_t)(v ? atoi(v) : 220) * 1024;
   }();
-  if (8 * stage <= cap) return atb2_launch<NB, RT, 8>(m, ones, sp, nb, s);
-  if (6 * stage <= cap) return atb2_launch<NB, RT, 6>(m, ones, sp, nb, s);
-  if (4 * stage <= cap) return atb2_launch<NB, RT, 4>(m, ones, sp, nb, s);
-  if (3 * stage <= cap) return atb2_launch<NB, RT, 3>(m, ones, sp, nb, s);
+  static const int two = [] {                      // 2 CTAs per SM when 3 hi stages fit twice
+    const char* v = getenv("STG_ATB_CTAS");
+    return v ? atoi(v) == 2 : 1;
+  }();
+  if (two && 5 * stage <= 108 * 1024) return atb2_launch<NB, RT, 3>(m, ones, sp, nb, s, 2);
+  // measured on C5: deeper rings than 4 hi stages did not help (dW 10.9 ms/epoch at 4, 12.9 at 8)
+  if (6 * stage <= cap) return atb2_launch<NB, RT, 4>(m, ones, sp, nb, s);
+  if (5 * stage <= cap) return atb2_launch<NB, RT, 3>(m, ones, sp, nb, s);
   return atb2_launch<NB, RT, 2>(m, ones, sp, nb, s);
 }
 
