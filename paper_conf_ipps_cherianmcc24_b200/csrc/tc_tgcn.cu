@@ -1181,7 +1181,7 @@ struct AtbSpec2 {
   float* part;            // [gridDim][na][128][N]
 };
 
-template <int NB, int RT, int S>
+template <int NB, int RT, int S, int L = 2>
 __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUtensorMap m0,
                                                     const __grid_constant__ CUtensorMap m1,
                                                     const __grid_constant__ CUtensorMap m2,
@@ -1191,7 +1191,7 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   constexpr int BOX = RT * 32 * 4;
   extern __shared__ unsigned char sm_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
-  __shared__ uint64_t full[S], empty[S], conv[2], lfree[2], done, init_bar;
+  __shared__ uint64_t full[S], empty[S], conv[L], lfree[L], done, init_bar;
   __shared__ uint32_t tslot;
   const int na = sp.na, nsa = sp.nsa;
   const int nbox = nsa + NB;                       // box slots per stage
@@ -1200,13 +1200,13 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   auto lo = [&](int ls, int bx) { return sm + (size_t)(S + ls) * half + (size_t)bx * BOX; };
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   auto map_of = [&](int m) -> const CUtensorMap* { return m == 0 ? &m0 : (m == 1 ? &m1 : (m == 2 ? &m2 : &m3)); };
-  for (size_t e = threadIdx.x; e < (size_t)(S + 2) * half / 16; e += blockDim.x)   // lo of the ones box stays 0
+  for (size_t e = threadIdx.x; e < (size_t)(S + L) * half / 16; e += blockDim.x)   // lo of the ones box stays 0
     reinterpret_cast<float4*>(sm)[e] = make_float4(0.f, 0.f, 0.f, 0.f);
   const uint32_t tcols = na * N <= 128 ? 128 : 256;
   if (warp == 1) tc::tmem_alloc(&tslot, tcols);
   if (threadIdx.x == 0) {
     for (int st = 0; st < S; ++st) { tc::mbar_init(&full[st], 1); tc::mbar_init(&empty[st], 1); }
-    for (int ls = 0; ls < 2; ++ls) { tc::mbar_init(&conv[ls], 128); tc::mbar_init(&lfree[ls], 1); }
+    for (int ls = 0; ls < L; ++ls) { tc::mbar_init(&conv[ls], 128); tc::mbar_init(&lfree[ls], 1); }
     tc::mbar_init(&done, 1); tc::mbar_init(&init_bar, 1);
     tc::fence_mbar_init();
   }
@@ -1246,8 +1246,8 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
     if (lane == 0) {
       const uint32_t idesc = tc::idesc_tf32(128, N, 1, 1);
       for (int i = 0; i < my_tiles; ++i) {
-        const int st = i % S, ls = i & 1;
-        tc::mbar_wait(&conv[ls], (i >> 1) & 1);
+        const int st = i % S, ls = i % L;
+        tc::mbar_wait(&conv[ls], (i / L) & 1);
         tc::fence_after();
         const uint32_t bh = tc::smem_u32(hi(st, nsa)), bl = tc::smem_u32(lo(ls, nsa));
         for (int a = 0; a < na; ++a) {
@@ -1270,9 +1270,9 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   } else {                                           // ---- converters (warps 2-5), then epilogue
     const int ct = threadIdx.x - 64;
     for (int i = 0; i < my_tiles; ++i) {
-      const int st = i % S, ls = i & 1;
+      const int st = i % S, ls = i % L;
       tc::mbar_wait(&full[st], (i / S) & 1);
-      if (i >= 2) tc::mbar_wait(&lfree[ls], ((i >> 1) - 1) & 1);   // MMAs of tile i-2 done with slot ls
+      if (i >= L) tc::mbar_wait(&lfree[ls], ((i / L) - 1) & 1);   // MMAs of tile i-L done with slot ls
       for (int bx = 0; bx < nbox; ++bx) {
         if (bx < nsa && sp.src_map[bx] < 0) continue;   // ones box: lo stays 0
         const float4* src = reinterpret_cast<const float4*>(hi(st, bx));
@@ -1931,15 +1931,15 @@ static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
   return check_launch("tc_atb");
 }
 
-template <int NB, int RT, int S>
+template <int NB, int RT, int S, int L = 2>
 static stg_status atb2_launch(const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb_out,
                               cudaStream_t s, int ctas_per_sm = 1) {
   const int nbox = sp.nsa + NB;
-  const size_t smem = (size_t)(S + 2) * nbox * RT * 32 * 4 + 1024;   // S hi stages + 2 lo slots
-  STG_CUDA(cudaFuncSetAttribute(k_tc_atb2<NB, RT, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const size_t smem = (size_t)(S + L) * nbox * RT * 32 * 4 + 1024;   // S hi stages + L lo slots
+  STG_CUDA(cudaFuncSetAttribute(k_tc_atb2<NB, RT, S, L>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int ntiles = (sp.V + RT - 1) / RT;
   const int nb = std::max(1, std::min(ntiles, ctas_per_sm * num_sms()));
-  k_tc_atb2<NB, RT, S><<<nb, 192, smem, s>>>(m[0], m[1], m[2], m[3], ones, sp);
+  k_tc_atb2<NB, RT, S, L><<<nb, 192, smem, s>>>(m[0], m[1], m[2], m[3], ones, sp);
   count_launch();
   *nb_out = nb;
   return check_launch("tc_atb2");
@@ -1961,7 +1961,12 @@ static stg_status atb2_stages(const CUtensorMap* m, const CUtensorMap& ones, con
     const char* v = getenv("STG_ATB_CTAS");
     return v ? atoi(v) == 2 : 1;
   }();
+  static const int l1 = [] {                       // 2 CTAs x (2 hi stages + 1 lo slot): dL 19.0 -> 20.1 ms, off
+    const char* v = getenv("STG_ATB_L1");
+    return v ? atoi(v) : 0;
+  }();
   if (two && 5 * stage <= 108 * 1024) return atb2_launch<NB, RT, 3>(m, ones, sp, nb, s, 2);
+  if (two && l1 && 3 * stage <= 108 * 1024) return atb2_launch<NB, RT, 2, 1>(m, ones, sp, nb, s, 2);
   // measured on C5: deeper rings than 4 hi stages did not help (dW 10.9 ms/epoch at 4, 12.9 at 8)
   if (6 * stage <= cap) return atb2_launch<NB, RT, 4>(m, ones, sp, nb, s);
   if (5 * stage <= cap) return atb2_launch<NB, RT, 3>(m, ones, sp, nb, s);
