@@ -502,7 +502,7 @@ __device__ __forceinline__ void raw_to_tmem(const unsigned char* tile, int r, in
   const int c16 = (col % 32) / 4;
 #pragma unroll
   for (int q = 0; q < HH / 4; ++q) {
-    const float4 x = *reinterpret_cast<const float4*>(box + tc::swz128(r, c16 + q));
+    const float4 x = tc::lds128(tc::smem_u32(box) + tc::swz128(r, c16 + q));
     v[4 * q] = x.x; v[4 * q + 1] = x.y; v[4 * q + 2] = x.z; v[4 * q + 3] = x.w;
   }
   float lo[HH];
@@ -929,7 +929,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
       const unsigned char* box = rawG + (c0 / 32) * kBox;
 #pragma unroll
       for (int qq = 0; qq < HH / 4; ++qq) {
-        const float4 x = *reinterpret_cast<const float4*>(box + tc::swz128(lr, (c0 % 32) / 4 + qq));
+        const float4 x = tc::lds128(tc::smem_u32(box) + tc::swz128(lr, (c0 % 32) / 4 + qq));
         g[4 * qq] = x.x; g[4 * qq + 1] = x.y; g[4 * qq + 2] = x.z; g[4 * qq + 3] = x.w;
       }
     }
@@ -1215,7 +1215,9 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   __syncthreads();
   tc::fence_after();
   int n_ones = 0;
-  for (int k = 0; k < nsa; ++k) n_ones += sp.src_map[k] == -2;
+  uint32_t ones_mask = 0;
+  for (int k = 0; k < nsa; ++k)
+    if (sp.src_map[k] < 0) { n_ones += sp.src_map[k] == -2; ones_mask |= 1u << k; }
   if (n_ones) {                                      // the ones box (hardware swizzle) into each stage
     if (threadIdx.x == 0) {
       tc::mbar_expect_tx(&init_bar, (uint32_t)(n_ones * S * BOX));
@@ -1273,15 +1275,21 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
       const int st = i % S, ls = i % L;
       tc::mbar_wait(&full[st], (i / S) & 1);
       if (i >= L) tc::mbar_wait(&lfree[ls], ((i / L) - 1) & 1);   // MMAs of tile i-L done with slot ls
-      for (int bx = 0; bx < nbox; ++bx) {
-        if (bx < nsa && sp.src_map[bx] < 0) continue;   // ones box: lo stays 0
-        const float4* src = reinterpret_cast<const float4*>(hi(st, bx));
-        float4* dst = reinterpret_cast<float4*>(lo(ls, bx));
+      // the stage's boxes are contiguous: 8 shared loads in flight per thread, then the lo stores
+      const uint32_t hb = tc::smem_u32(hi(st, 0)), lb = tc::smem_u32(lo(ls, 0));
+      constexpr int B4 = BOX / 16;                    // float4 per box
+      for (int e0 = ct; e0 < nbox * B4; e0 += 8 * 128) {
+        float4 v[8];
 #pragma unroll
-        for (int e = ct; e < BOX / 16; e += 128) {
-          const float4 v = src[e];
-          dst[e] = make_float4(v.x - tc::tf32_hi(v.x), v.y - tc::tf32_hi(v.y), v.z - tc::tf32_hi(v.z),
-                               v.w - tc::tf32_hi(v.w));
+        for (int j = 0; j < 8; ++j)
+          if (e0 + 128 * j < nbox * B4) v[j] = tc::lds128(hb + 16u * (uint32_t)(e0 + 128 * j));
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int e = e0 + 128 * j;
+          if (e < nbox * B4 && !((ones_mask >> (e / B4)) & 1u))   // ones box: lo stays 0
+            tc::sts128(lb + 16u * (uint32_t)e,
+                       make_float4(v[j].x - tc::tf32_hi(v[j].x), v[j].y - tc::tf32_hi(v[j].y),
+                                   v[j].z - tc::tf32_hi(v[j].z), v[j].w - tc::tf32_hi(v[j].w)));
         }
       }
       tc::fence_proxy_async();
@@ -1656,7 +1664,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_seq_bwd(int V, int S, const _
       const unsigned char* box = rawT + (c0 / 32) * kBox;
 #pragma unroll
       for (int qq = 0; qq < HH / 4; ++qq) {
-        const float4 x = *reinterpret_cast<const float4*>(box + tc::swz128(lr, (c0 % 32) / 4 + qq));
+        const float4 x = tc::lds128(tc::smem_u32(box) + tc::swz128(lr, (c0 % 32) / 4 + qq));
         ht[4 * qq] = x.x; ht[4 * qq + 1] = x.y; ht[4 * qq + 2] = x.z; ht[4 * qq + 3] = x.w;
       }
       // fused head, backward: gs = 2(ŷ − y)/V_total;  G = gs·w_o⊙[H_t > 0] + dH(t+1)
