@@ -1468,6 +1468,37 @@ __global__ void k_tc_sum_parts(const float* __restrict__ part, int nb, int n, fl
   }
 }
 
+// The same sum in the same order, parallel over the 16-partial groups: a block owns 32
+// consecutive elements; warp y forms the group sums j = y, y+8, ... (coalesced rows of
+// 32), then lane row 0 adds them in group order — bit-identical to k_tc_sum_parts.
+constexpr int kSumMaxGroups = 64;                  // nb <= 1024
+__global__ void __launch_bounds__(256) k_tc_sum_parts2(const float* __restrict__ part, int nb, int n,
+                                                       float* __restrict__ tot) {
+  __shared__ float blk[kSumMaxGroups][33];
+  const int x = threadIdx.x & 31, y = threadIdx.x >> 5;
+  const int e = blockIdx.x * 32 + x;
+  const int ng = (nb + 15) / 16;
+  for (int j = y; j < ng; j += 8) {
+    float b = 0.f;
+    if (e < n) {
+      const int b0 = 16 * j, b1 = min(b0 + 16, nb);
+      float v[16];
+#pragma unroll
+      for (int k = 0; k < 16; ++k) v[k] = (b0 + k < b1) ? __ldg(part + (int64_t)(b0 + k) * n + e) : 0.f;
+#pragma unroll
+      for (int k = 0; k < 16; ++k)
+        if (b0 + k < b1) b += v[k];
+    }
+    blk[j][x] = b;
+  }
+  __syncthreads();
+  if (y == 0 && e < n) {
+    float t = 0.f;
+    for (int j = 0; j < ng; ++j) t += blk[j][x];
+    tot[e] = t;
+  }
+}
+
 // Scatter the dL / dl / db pieces out of tot = [D1 (128 × ldd) | D2 (128 × ldd)]
 // (row = A feature, column = da feature: da_z | da_r | da_h, ldd >= 3H):
 //   D1 rows: C_z | C_r | C_h (rows 0..3H) | H (rows hoff..hoff+H),
@@ -2167,7 +2198,8 @@ stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* pa
   int nb = 0;
   STG_TRY(atb2_dispatch(NB, m, ones, sp, &nb, s));
   const int n = 128 * N;
-  k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
+  if (nb <= 16 * kSumMaxGroups) k_tc_sum_parts2<<<(n + 31) / 32, 256, 0, s>>>(part, nb, n, tot);
+  else k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
   k_dw_scatter<<<(F * H3 + 255) / 256, 256, 0, s>>>(F, H3, N, tot, dW);
   count_launch(2);
   return check_launch("tc_dw");
@@ -2199,7 +2231,8 @@ stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH,
   int nb = 0;
   STG_TRY(atb2_dispatch(NBC, m, ones, sp, &nb, s));
   const int N = 32 * NBC, n = 2 * 128 * N;
-  k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
+  if (nb <= 16 * kSumMaxGroups) k_tc_sum_parts2<<<(n + 31) / 32, 256, 0, s>>>(part, nb, n, tot);
+  else k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
   k_dl_scatter<<<(6 * H * H + 6 * H + 255) / 256, 256, 0, s>>>(H, N, 32, N, tot, L, dL, dl, db);
   count_launch(2);
   return check_launch("tc_dl");
