@@ -237,10 +237,14 @@ stg_status stg_gcn_weighted_norm(const stg_csr_view* g, const float* ew, float* 
  *     caller-built views without a schedule). */
 stg_status stg_aggregate_set_strategy(int32_t strategy);
 /* Tunables of strategy 2 (STG_ERR_INVALID_ARG for a bad key/value):
- * key 0: neighbour rows in flight per warp, 4 | 8 | 16 (default 16);
- * key 1: minimum resident blocks per SM (register budget), 2..6 (default 3;
+ * key 0: neighbour rows in flight per warp, 4 | 8 | 16 (default 4);
+ * key 1: minimum resident blocks per SM (register budget), 2..6 (default 6;
  *        supported pairs (rows, blocks): (4,6) (8,4) (16,2) (16,3));
- * key 2: 32 | 64 (default 32): strategy 2 serves launch widths above this. */
+ * key 2: 32 | 64 (default 32): strategy 2 serves launch widths above this;
+ * key 3: source-row cache hints 0..4 (default 0 = none; with (4,6) only):
+ *        1 = rows u < hotk L2 evict_last, others L1 no_allocate + L2 evict_first,
+ *        2 = others only, 3 = hot only, 4 = 1 without the L1 no_allocate;
+ * key 4: hotk, the hot prefix length of the source order (rows). */
 stg_status stg_aggregate_set_param(int32_t key, int64_t value);
 
 /* ---- TGCN (GCN + GRU; reading C13-C15) ----
@@ -496,6 +500,15 @@ stg_status stg_profile_read(int32_t phase, double* total_ms, int64_t* count, int
  * N % 16 == 0, 16 <= N <= 256.  Row-major fp32 device arrays. */
 stg_status stg_debug_tc_gemm(int32_t mode, int32_t M, int32_t N, int32_t K, int32_t R, const float* A,
                              const float* B, float* C, stg_stream_t stream);
+
+/* Diagnostic: the fixed-order sum tot[e] = Σ_b part[b·n + e] of the Σ AᵀB
+ * reductions (per-CTA partials part[nb][n], added in blocks of 16 in block
+ * order, then over the blocks in order).  variant 0: one thread per element;
+ * variant 1: parallel over the 16-partial blocks (nb <= 1024).  Both give the
+ * same bits (tests/test_gpu_tc.py).  Device arrays; STG_ERR_INVALID_ARG for
+ * nb < 1, n < 1 or an unknown variant. */
+stg_status stg_debug_sum_parts(const float* part, int32_t nb, int32_t n, float* tot, int32_t variant,
+                               stg_stream_t stream);
 
 /* Stream-ordered byte copy (kind: 0 device->device, 1 host->device,
  * 2 device->host); lets bindings read borrowed view arrays. */

@@ -134,6 +134,7 @@ _decl("stg_tgcn_train_sequence_batched", [_P, _i32, ctypes.POINTER(stg_tgcn_para
 _decl("stg_partition_rows", [_i32, _P, _i32, ctypes.POINTER(_i32), _P])
 _decl("stg_profile_enable", [_i32])
 _decl("stg_debug_tc_gemm", [_i32, _i32, _i32, _i32, _i32, _P, _P, _P, _P])
+_decl("stg_debug_sum_parts", [_P, _i32, _i32, _P, _i32, _P])
 _decl("stg_aggregate_set_strategy", [_i32])
 _decl("stg_aggregate_set_param", [_i32, _i64])
 _decl("stg_profile_read", [_i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64), _i32])
@@ -173,7 +174,7 @@ ABI_SYMBOLS = [
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
     "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_mse_head_ex", "stg_sgd_update", "stg_tgcn_train_sequence",
     "stg_tgcn_train_sequence_batched", "stg_tgcn_train_sequence_ev",
-    "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_aggregate_set_strategy",
+    "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_debug_sum_parts", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
     "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm", "stg_tgcn2_step", "stg_tgcn2_step_backward",
     "stg_peer_alloc", "stg_peer_free", "stg_peer_open", "stg_peer_close", "stg_allgather_rows",
@@ -210,14 +211,23 @@ def _stream(stream=None):
     return ctypes.c_void_p(stream.cuda_stream)
 
 
-def _ptr(t):
+def _ptr(t, dt=torch.float32):
+    """Device pointer of a contiguous CUDA tensor of dtype `dt` (float32 features
+    and parameters, int32 ids): anything else would reach the kernels as raw bytes."""
     if t is None:
         return None
     if not t.is_cuda:
         raise StgError(1, "expected a CUDA tensor")
     if not t.is_contiguous():
         raise StgError(1, "expected a contiguous tensor")
+    if t.dtype != dt:
+        raise StgError(1, "expected a %s tensor, got %s" % (dt, t.dtype))
     return ctypes.c_void_p(t.data_ptr())
+
+
+def _ptrs(ts):
+    """Host array of device pointers of float32 CUDA tensors (per-timestamp inputs)."""
+    return (_P * len(ts))(*[_ptr(t).value for t in ts])
 
 
 def _dev_i32(a):
@@ -299,10 +309,21 @@ def _dist(dist):
     return ctypes.byref(stg_dist(r, w, b, e))
 
 
+def _order_inputs(stream, *ts):
+    """The id arrays were staged on the current stream: order the library's stream
+    after those copies and keep the caching allocator from reusing them early."""
+    if stream is None or stream == torch.cuda.current_stream():
+        return
+    stream.wait_stream(torch.cuda.current_stream())
+    for t in ts:
+        t.record_stream(stream)
+
+
 def stg_static_graph_create(V: int, src, dst, flags: int = 0, stream=None, dist=None) -> Graph:
     s, d = _dev_i32(src), _dev_i32(dst)
+    _order_inputs(stream, s, d)
     out = ctypes.c_void_p()
-    _check(_lib.stg_static_graph_create(V, s.numel(), _ptr(s), _ptr(d), flags, _dist(dist), _stream(stream),
+    _check(_lib.stg_static_graph_create(V, s.numel(), _ptr(s, torch.int32), _ptr(d, torch.int32), flags, _dist(dist), _stream(stream),
                                         ctypes.byref(out)))
     return Graph(out)
 
@@ -318,16 +339,17 @@ def stg_dtdg_create(V: int, T: int, src0, dst0, add_off, add_src, add_dst, del_o
     s0, d0 = _dev_i32(src0), _dev_i32(dst0)
     a_s, a_d = _dev_i32(add_src), _dev_i32(add_dst)
     r_s, r_d = _dev_i32(del_src), _dev_i32(del_dst)
+    _order_inputs(stream, s0, d0, a_s, a_d, r_s, r_d)
     ao = np.ascontiguousarray(add_off, dtype=np.int64)
     do = np.ascontiguousarray(del_off, dtype=np.int64)
     if ao.size != T + 1 or do.size != T + 1:
         raise StgError(1, "offset arrays must have T+1 entries")
     out = ctypes.c_void_p()
-    _check(_lib.stg_dtdg_create(V, T, s0.numel(), _ptr(s0), _ptr(d0),
-                                ao.ctypes.data_as(_P), _ptr(a_s) if a_s.numel() else None,
-                                _ptr(a_d) if a_d.numel() else None,
-                                do.ctypes.data_as(_P), _ptr(r_s) if r_s.numel() else None,
-                                _ptr(r_d) if r_d.numel() else None,
+    _check(_lib.stg_dtdg_create(V, T, s0.numel(), _ptr(s0, torch.int32), _ptr(d0, torch.int32),
+                                ao.ctypes.data_as(_P), _ptr(a_s, torch.int32) if a_s.numel() else None,
+                                _ptr(a_d, torch.int32) if a_d.numel() else None,
+                                do.ctypes.data_as(_P), _ptr(r_s, torch.int32) if r_s.numel() else None,
+                                _ptr(r_d, torch.int32) if r_d.numel() else None,
                                 flags, _dist(dist), _stream(stream), ctypes.byref(out)))
     torch.cuda.current_stream().synchronize()
     return Dtdg(out)
@@ -532,8 +554,8 @@ def stg_tgcn_train_sequence_batched(graph, S: int, params: dict, w_o, b_o, Xs, Y
     """Sequence-batched Algorithm 1 over a static graph (NEXT-1): same maths, per-sequence kernels."""
     P = make_params(params)
     G = make_grads(grads)
-    xp = (_P * S)(*[x.data_ptr() for x in Xs])
-    yp = (_P * S)(*[y.data_ptr() for y in Ys])
+    xp = _ptrs(Xs)
+    yp = _ptrs(Ys)
     _check(_lib.stg_tgcn_train_sequence_batched(graph.handle, S, ctypes.byref(P), _ptr(w_o), _ptr(b_o), xp, yp,
                                                 _ptr(H0), _ptr(H_seq), ctypes.byref(G), _ptr(dw_o), _ptr(db_o),
                                                 _ptr(loss_accum), stack.handle, _stream(stream)))
@@ -545,8 +567,8 @@ def stg_tgcn_train_sequence(source, t0: int, S: int, params: dict, w_o, b_o, Xs,
     torch.cuda.Event, one per timestamp, recorded after X_t / y_t were written."""
     P = make_params(params)
     G = make_grads(grads)
-    xp = (_P * S)(*[x.data_ptr() for x in Xs])
-    yp = (_P * S)(*[y.data_ptr() for y in Ys])
+    xp = _ptrs(Xs)
+    yp = _ptrs(Ys)
     graph = source.handle if isinstance(source, Graph) else None
     dtdg = source.handle if isinstance(source, Dtdg) else None
     ev = None
@@ -559,7 +581,7 @@ def stg_tgcn_train_sequence(source, t0: int, S: int, params: dict, w_o, b_o, Xs,
 
 def stg_partition_rows(V: int, in_rowptr: torch.Tensor, world: int, stream=None) -> list:
     b = (_i32 * (world + 1))()
-    _check(_lib.stg_partition_rows(V, _ptr(in_rowptr), world, b, _stream(stream)))
+    _check(_lib.stg_partition_rows(V, _ptr(in_rowptr, torch.int32), world, b, _stream(stream)))
     return list(b)
 
 
@@ -578,6 +600,14 @@ def stg_debug_tc_gemm(mode: int, A: torch.Tensor, B: torch.Tensor, stream=None) 
         C = torch.empty(128, N, device=A.device)
         _check(_lib.stg_debug_tc_gemm(mode, 128, N, 0, R, _ptr(A), _ptr(B), _ptr(C), _stream(stream)))
     return C
+
+
+def stg_debug_sum_parts(part: torch.Tensor, variant: int, stream=None) -> torch.Tensor:
+    """Fixed-order Σ over the rows of part [nb, n] (the Σ AᵀB partial sums): variant 0 serial, 1 parallel."""
+    nb, n = part.shape
+    tot = torch.empty(n, device=part.device)
+    _check(_lib.stg_debug_sum_parts(_ptr(part), nb, n, _ptr(tot), int(variant), _stream(stream)))
+    return tot
 
 
 def stg_aggregate_set_strategy(strategy: int):

@@ -3,6 +3,9 @@
 #pragma once
 
 #include <algorithm>
+#include <memory>
+#include <mutex>
+#include <vector>
 
 #include "common.cuh"
 
@@ -46,11 +49,25 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
                             float* out, int64_t ldout, const float* srow, const float* scol, const float* bias,
                             cudaStream_t s, const stg_peer_rows* peers = nullptr, const float* ew = nullptr);
 
-struct AggWs {
+struct AggScratch {
   DArray<float> partials;
   DArray<int32_t> counters;
   int64_t counters_n = 0;
   DArray<uint32_t> queue;        // edge-stream work-queue heads, one per column chunk (reset per launch)
+};
+// One scratch area per stream that has aggregated over the object: calls on
+// different streams never share a work queue, partials or counters (each call
+// is ordered only on its own stream, include/stg.h).
+struct AggWs {
+  std::mutex mu;
+  std::vector<std::pair<cudaStream_t, std::unique_ptr<AggScratch>>> per;
+  AggScratch* get(cudaStream_t s) {
+    std::lock_guard<std::mutex> lk(mu);
+    for (auto& e : per)
+      if (e.first == s) return e.second.get();
+    per.emplace_back(s, std::make_unique<AggScratch>());
+    return per.back().second.get();
+  }
 };
 
 // Row-block sharding: a sharded snapshot holds only the edges

@@ -2,17 +2,17 @@
 // 3xTF32 for fp32-class accuracy, accumulators in TMEM).  Each kernel is a
 // persistent loop over 128-row tiles (one row per thread in the epilogue):
 //
-//   k_tc_xw      P' = diag(n_src)·X·W                  (K = F, N = 3H)
-//   k_tc_gru_fwd a_z = [C_z|H]·L_z, a_r = [C_r|H]·L_r   (MMA, K = 2H, N = H each)
-//                Z, R = σ(·+l);  RH = R⊙H  staged in smem
-//                a_h = [C_h|RH]·L_h → Ĥ = tanh, H' = Z⊙H + (1−Z)⊙Ĥ
-//   k_tc_gru_bwd recompute a_z, a_r, a_h (as above), then
-//                [dC_h|dRH] = da_h·L_hᵀ, [dC_z|dH_z] = da_z·L_zᵀ, [dC_r|dH_r] = da_r·L_rᵀ
-//                (MMA, K = H, N = 2H each) and the elementwise chain rule;
-//                writes dC' = n_dst⊙dC, dH_prev, and da = [da_z|da_r|da_h], RH
-//                for the parameter-gradient reduction
-//   k_tc_atb     D = Σ_rows A[r,:]ᵀ·B[r,:] with A, B staged transposed (K = rows),
-//                per-CTA partials, fixed-order reduction → dW, dL, dl.
+//   k_tc_xw_pipe  P' = diag(n_src)·X·W                  (K = F, N = 3H; k_tc_xw for 64 < F <= 128)
+//   k_tc_gru_fwd2 a_z = [C_z|H]·L_z, a_r = [C_r|H]·L_r   (MMA, K = 2H, N = H each)
+//                 Z, R = σ(·+l);  RH = R⊙H
+//                 a_h = [C_h|RH]·L_h → Ĥ = tanh, H' = Z⊙H + (1−Z)⊙Ĥ
+//   k_tc_gru_bwd2 recompute a_z, a_r, a_h (as above), then
+//                 [dC_h|dRH] = da_h·L_hᵀ, [dC_z|dH_z] = da_z·L_zᵀ, [dC_r|dH_r] = da_r·L_rᵀ
+//                 (MMA, K = H, N = 2H each) and the elementwise chain rule;
+//                 writes dC' = n_dst⊙dC, dH_prev, and da = [da_z|da_r|da_h], RH
+//                 for the parameter-gradient reduction
+//   k_tc_atb2     D = Σ_rows A[r,:]ᵀ·B[r,:] with A, B loaded by TMA in the MN-major
+//                 layout (K = rows), per-CTA partials, fixed-order reduction → dW, dL, dl.
 //
 // The equations are those of SURVEY §8(c) (readings C13-C15).
 #include <algorithm>
@@ -172,8 +172,8 @@ template <int N>
 __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int Kp, const float* __restrict__ X,
                                                               const float* __restrict__ W,
                                                               const float* __restrict__ rs, float* __restrict__ P,
-                                                              int dbg, int rs_div,
-                                                              const __grid_constant__ CUtensorMap tmP, int box) {
+                                                              int rs_div,
+                                                              const __grid_constant__ CUtensorMap tmP) {
   extern __shared__ __align__(128) unsigned char sm[];
   __shared__ uint64_t full[kXwStages], empty[kXwStages], tfull[2], tempty[2];
   __shared__ uint32_t tslot;
@@ -206,14 +206,14 @@ __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int 
     const int grp = (warp - 4) >> 2, tid = threadIdx.x - 128 - 128 * grp;
     float4 v[16];
     int tile = blockIdx.x + grp * gridDim.x;
-    if (tile < ntiles && !(dbg & 4)) tc::grp_load<16>(v, X + (int64_t)tile * 128 * F, F, V - tile * 128, 128, F, 0, tid, 128);
+    if (tile < ntiles) tc::grp_load<16>(v, X + (int64_t)tile * 128 * F, F, V - tile * 128, 128, F, 0, tid, 128);
     for (int k = 0; tile < ntiles; tile += 2 * gridDim.x, ++k) {
       if (k > 0) tc::mbar_wait(&empty[grp], (k - 1) & 1);
-      if (!(dbg & 8)) tc::grp_store<16>(v, ahi(grp), alo(grp), 128, F, 0, Kp, tid, 128);
+      tc::grp_store<16>(v, ahi(grp), alo(grp), 128, F, 0, Kp, tid, 128);
       tc::fence_proxy_async();
       tc::mbar_arrive(&full[grp]);
       const int nt = tile + 2 * gridDim.x;
-      if (nt < ntiles && !(dbg & 4)) tc::grp_load<16>(v, X + (int64_t)nt * 128 * F, F, V - nt * 128, 128, F, 0, tid, 128);
+      if (nt < ntiles) tc::grp_load<16>(v, X + (int64_t)nt * 128 * F, F, V - nt * 128, 128, F, 0, tid, 128);
     }
   } else if (warp == 12) {                           // ---- MMA issuer
     if ((threadIdx.x & 31) == 0) {
@@ -224,43 +224,13 @@ __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int 
         tc::mbar_wait(&full[st], k & 1);
         if (k > 0) tc::mbar_wait(&tempty[st], (k - 1) & 1);
         tc::fence_after();
-        if (!(dbg & 2))
-          mma_seg(tm + st * NC, tc::smem_u32(ahi(st)), tc::smem_u32(alo(st)), Kp, 0, tc::smem_u32(bhi),
+        mma_seg(tm + st * NC, tc::smem_u32(ahi(st)), tc::smem_u32(alo(st)), Kp, 0, tc::smem_u32(bhi),
                   tc::smem_u32(blo), Kp, 0, Kp, idesc, true);
         tc::commit(&empty[st]);
         tc::commit(&tfull[st]);
       }
     }
-  } else if (warp < 4 && !box) {                     // ---- epilogue (staged row stores)
-    float4* stage = ostage + warp * 32 * tc::kStagePitch<NQ>;
-    int i = 0;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
-      const int b = i & 1, kb = i >> 1;
-      const int row = tile * 128 + threadIdx.x;
-      const float sc = (rs && row < V) ? __ldg(rs + row / rs_div) : 1.0f;   // row scale of vertex row / rs_div
-      tc::mbar_wait(&tfull[b], kb & 1);
-      tc::fence_after();
-      // TMEM -> registers in 16-column pieces -> scaled row in this warp's stage
-      const int lane = threadIdx.x & 31;
-#pragma unroll
-      for (int c0 = 0; c0 < N; c0 += 16) {
-        float v[16];
-        tmem_row_load<16>(tm + b * NC, c0, v);
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          stage[lane * tc::kStagePitch<NQ> + c0 / 4 + q] =
-              make_float4(sc * v[4 * q], sc * v[4 * q + 1], sc * v[4 * q + 2], sc * v[4 * q + 3]);
-      }
-      tc::fence_before();
-      tc::mbar_arrive(&tempty[b]);
-      if (!(dbg & 1)) {
-        const int wr0 = tile * 128 + warp * 32;
-        tc::flush_stage_rows<NQ>(stage, P, N, wr0, V - wr0);
-      } else {
-        __syncwarp();
-      }
-    }
-  } else if (warp < 4 && box) {                      // ---- epilogue, TMA box stores
+  } else if (warp < 4) {                             // ---- epilogue, TMA box stores
     unsigned char* obuf = reinterpret_cast<unsigned char*>(
         (reinterpret_cast<uintptr_t>(abase + (size_t)kXwStages * 2 * ABYTES) + 1023) & ~uintptr_t(1023)) + warp * 4096;
     int oslot = 0;
@@ -333,126 +303,11 @@ __device__ __forceinline__ void issue_zr(uint32_t tm, unsigned char* ahi, unsign
   mma_seg(tm + H, a_h, a_l, 3 * H, 2 * H, tc::smem_u32(br_hi), tc::smem_u32(br_lo), 2 * H, H, H, idesc, false);
 }
 
-// Writes RH (row-local, into columns [H, 2H) of the width-2H A2 tile).
-template <int H>
-__device__ __forceinline__ void stage_row_vec(unsigned char* hi, unsigned char* lo, int r, int k0, int K,
-                                              const float* v) {
-#pragma unroll
-  for (int q = 0; q < H / 4; ++q)
-    tc::st_split4(hi, lo, r, k0 / 4 + q, K, make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]));
-}
-
 // ------------------------------------------------------------------ GRU forward
 // 256 threads: thread t owns tile row (w % 4)·32 + lane (its TMEM lane) and the
 // column half (w / 4) of every H-wide quantity.  All GRU epilogue math is
 // column-local; the column mixing happens in the MMAs.
 constexpr int kGruThreads = 256;
-
-template <int N>
-__device__ __forceinline__ void ld_half(const float* __restrict__ src, bool ok, float (&v)[N]) {
-#pragma unroll
-  for (int q = 0; q < N / 4; ++q) {
-    float4 x = ok ? __ldg(reinterpret_cast<const float4*>(src) + q) : make_float4(0.f, 0.f, 0.f, 0.f);
-    v[4 * q] = x.x; v[4 * q + 1] = x.y; v[4 * q + 2] = x.z; v[4 * q + 3] = x.w;
-  }
-}
-template <int N>
-__device__ __forceinline__ void st_half(float* dst, const float (&v)[N], float scale = 1.0f) {
-#pragma unroll
-  for (int q = 0; q < N / 4; ++q)
-    reinterpret_cast<float4*>(dst)[q] =
-        make_float4(scale * v[4 * q], scale * v[4 * q + 1], scale * v[4 * q + 2], scale * v[4 * q + 3]);
-}
-template <int N>
-__device__ __forceinline__ void stage_half(unsigned char* hi, unsigned char* lo, int r, int k0, int K,
-                                           const float (&v)[N]) {
-#pragma unroll
-  for (int q = 0; q < N / 4; ++q)
-    tc::st_split4(hi, lo, r, k0 / 4 + q, K, make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]));
-}
-
-template <int H>
-__global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_fwd(int V, const float* __restrict__ C,
-                                                               const float* __restrict__ Hp,
-                                                               const float* __restrict__ L,
-                                                               const float* __restrict__ l, float* __restrict__ Hn) {
-  extern __shared__ __align__(128) unsigned char sm[];
-  __shared__ uint64_t mbar;
-  __shared__ uint32_t tslot;
-  constexpr int BG = GruSmem<H>::BG, A1 = GruSmem<H>::A1, H3 = 3 * H, HH = H / 2;
-  unsigned char* bz_hi = sm;               unsigned char* bz_lo = bz_hi + BG;
-  unsigned char* br_hi = bz_lo + BG;       unsigned char* br_lo = br_hi + BG;
-  unsigned char* bh_hi = br_lo + BG;       unsigned char* bh_lo = bh_hi + BG;
-  unsigned char* ahi = bh_lo + BG;         unsigned char* alo = ahi + A1;
-  const int LG = 2 * H * H;
-  stage_gate_weights<H>(bz_hi, bz_lo, L);
-  stage_gate_weights<H>(br_hi, br_lo, L + LG);
-  stage_gate_weights<H>(bh_hi, bh_lo, L + 2 * LG);
-  if ((threadIdx.x >> 5) == 0) tc::tmem_alloc(&tslot, 128);
-  if (threadIdx.x == 0) { tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  const uint32_t tm = tslot;
-  uint32_t phase = 0;
-  const int ntiles = (V + 127) / 128;
-  const int w = threadIdx.x >> 5, lr = (w & 3) * 32 + (threadIdx.x & 31), c0 = (w >> 2) * HH;
-  float lz[HH], lrr[HH], lh[HH];
-#pragma unroll
-  for (int j = 0; j < HH; ++j) { lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; }
-  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int r0 = tile * 128, nv = V - r0, row = r0 + lr;
-    const bool ok = row < V;
-    float h[HH];
-    ld_half<HH>(Hp + (int64_t)row * H + c0, ok, h);          // in flight during staging + MMA
-    tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, 2 * H, 0, 0, H3);
-    tc::stage_rows(ahi, alo, Hp + (int64_t)r0 * H, H, nv, 128, H, 0, 2 * H, H3);
-    sync_mma_operands();
-    if (threadIdx.x == 0) {
-      issue_zr<H>(tm, ahi, alo, bz_hi, bz_lo, br_hi, br_lo);
-      tc::commit(&mbar);
-    }
-    wait_mma(&mbar, phase);
-    float z[HH], rh[HH];
-    {
-      float az[HH], ar[HH];
-      tmem_row_load<HH>(tm, c0, az);
-      tmem_row_load<HH>(tm, H + c0, ar);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) {
-        z[j] = sigm(az[j] + lz[j]);
-        rh[j] = sigm(ar[j] + lrr[j]) * h[j];
-      }
-    }
-    // A2 = [C_h | RH] (width 2H) reuses the A1 storage (MMA on A1 has completed)
-    tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, H, 2 * H, 0, 2 * H);
-    stage_half<HH>(ahi, alo, lr, H + c0, 2 * H, rh);
-    sync_mma_operands();
-    if (threadIdx.x == 0) {
-      const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0);
-      mma_seg(tm + 2 * H, tc::smem_u32(ahi), tc::smem_u32(alo), 2 * H, 0, tc::smem_u32(bh_hi), tc::smem_u32(bh_lo),
-              2 * H, 0, 2 * H, idesc, true);
-      tc::commit(&mbar);
-    }
-    wait_mma(&mbar, phase);
-    {
-      float ah[HH], o[HH];
-      tmem_row_load<HH>(tm, 2 * H + c0, ah);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) {
-        const float hh = tanhf(ah[j] + lh[j]);
-        o[j] = z[j] * h[j] + (1.0f - z[j]) * hh;
-      }
-      if (ok) st_half<HH>(Hn + (int64_t)row * H + c0, o);
-    }
-    tc::fence_before();
-    __syncthreads();
-    tc::fence_after();
-  }
-  tc::fence_before();
-  __syncthreads();
-  if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, 128);
-}
 
 // ------------------------------------------------------------------ GRU forward, v2
 // One persistent CTA per SM, 8 warps; thread = (tile row = TMEM lane, column
@@ -778,155 +633,6 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd3(int V, const __grid_cons
   if (warp == 0) tc::tmem_free(tslot, 512);
 }
 
-// ------------------------------------------------------------------ GRU backward
-template <int H>
-__global__ void __launch_bounds__(kGruThreads, 1) k_tc_gru_bwd(int V, const float* __restrict__ C,
-                                                               const float* __restrict__ Hp,
-                                                               const float* __restrict__ G,
-                                                               const float* __restrict__ L,
-                                                               const float* __restrict__ l,
-                                                               const float* __restrict__ ndst,
-                                                               float* __restrict__ dCs, float* __restrict__ dHp,
-                                                               float* __restrict__ da, float* __restrict__ RHo) {
-  extern __shared__ __align__(128) unsigned char sm[];
-  __shared__ uint64_t mbar;
-  __shared__ uint32_t tslot;
-  constexpr int BG = GruSmem<H>::BG, A1 = GruSmem<H>::A1, H3 = 3 * H, HH = H / 2;
-  unsigned char* bz_hi = sm;               unsigned char* bz_lo = bz_hi + BG;
-  unsigned char* br_hi = bz_lo + BG;       unsigned char* br_lo = br_hi + BG;
-  unsigned char* bh_hi = br_lo + BG;       unsigned char* bh_lo = bh_hi + BG;
-  unsigned char* lz_hi = bh_lo + BG;       unsigned char* lz_lo = lz_hi + BG;
-  unsigned char* lr_hi = lz_lo + BG;       unsigned char* lr_lo = lr_hi + BG;
-  unsigned char* lh_hi = lr_lo + BG;       unsigned char* lh_lo = lh_hi + BG;
-  unsigned char* ahi = lh_lo + BG;         unsigned char* alo = ahi + A1;
-  const int LG = 2 * H * H;
-  stage_gate_weights<H>(bz_hi, bz_lo, L);
-  stage_gate_weights<H>(br_hi, br_lo, L + LG);
-  stage_gate_weights<H>(bh_hi, bh_lo, L + 2 * LG);
-  stage_plain<H>(lz_hi, lz_lo, L);
-  stage_plain<H>(lr_hi, lr_lo, L + LG);
-  stage_plain<H>(lh_hi, lh_lo, L + 2 * LG);
-  // TMEM columns: Dz [0,H), Dr [H,2H), Dh [2H,3H), D3 [4H,6H), D4z [6H,8H), D4r [8H,10H)
-  constexpr uint32_t NC = 10 * H <= 256 ? 256 : 512;
-  if ((threadIdx.x >> 5) == 0) tc::tmem_alloc(&tslot, NC);
-  if (threadIdx.x == 0) { tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  const uint32_t tm = tslot;
-  uint32_t phase = 0;
-  const int ntiles = (V + 127) / 128;
-  const int w = threadIdx.x >> 5, lr = (w & 3) * 32 + (threadIdx.x & 31), c0 = (w >> 2) * HH;
-  const uint32_t id_h = tc::idesc_tf32(128, H, 0, 0), id_2h = tc::idesc_tf32(128, 2 * H, 0, 0);
-  float lz[HH], lrr[HH], lh[HH];
-#pragma unroll
-  for (int j = 0; j < HH; ++j) { lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; }
-  unsigned char* a3h = ahi;                      unsigned char* a3l = alo;
-  unsigned char* a4zh = ahi + 128 * H * 4;       unsigned char* a4zl = alo + 128 * H * 4;
-  unsigned char* a4rh = ahi + 2 * 128 * H * 4;   unsigned char* a4rl = alo + 2 * 128 * H * 4;
-  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int r0 = tile * 128, nv = V - r0, row = r0 + lr;
-    const bool ok = row < V;
-    float h[HH], g[HH];
-    ld_half<HH>(Hp + (int64_t)row * H + c0, ok, h);           // in flight during staging + MMA
-    ld_half<HH>(G + (int64_t)row * H + c0, ok, g);
-    const float nd = ok ? __ldg(ndst + row) : 0.f;
-    tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, 2 * H, 0, 0, H3);
-    tc::stage_rows(ahi, alo, Hp + (int64_t)r0 * H, H, nv, 128, H, 0, 2 * H, H3);
-    sync_mma_operands();
-    if (threadIdx.x == 0) {
-      issue_zr<H>(tm, ahi, alo, bz_hi, bz_lo, br_hi, br_lo);
-      tc::commit(&mbar);
-    }
-    wait_mma(&mbar, phase);
-    float z[HH], r[HH], dh[HH];
-    {
-      float az[HH], ar[HH];
-      tmem_row_load<HH>(tm, c0, az);
-      tmem_row_load<HH>(tm, H + c0, ar);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) {
-        z[j] = sigm(az[j] + lz[j]);
-        r[j] = sigm(ar[j] + lrr[j]);
-        dh[j] = r[j] * h[j];                         // RH for now
-      }
-    }
-    tc::stage_rows(ahi, alo, C + (int64_t)r0 * H3, H3, nv, 128, H, 2 * H, 0, 2 * H);
-    stage_half<HH>(ahi, alo, lr, H + c0, 2 * H, dh);
-    if (ok) st_half<HH>(RHo + (int64_t)row * H + c0, dh);
-    sync_mma_operands();
-    if (threadIdx.x == 0) {
-      mma_seg(tm + 2 * H, tc::smem_u32(ahi), tc::smem_u32(alo), 2 * H, 0, tc::smem_u32(bh_hi), tc::smem_u32(bh_lo),
-              2 * H, 0, 2 * H, id_h, true);
-      tc::commit(&mbar);
-    }
-    wait_mma(&mbar, phase);
-    {
-      float ah[HH], dah[HH], daz[HH];
-      tmem_row_load<HH>(tm, 2 * H + c0, ah);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) {
-        const float hh = tanhf(ah[j] + lh[j]);
-        const float dZ = g[j] * (h[j] - hh), dHh = g[j] * (1.0f - z[j]);
-        dah[j] = dHh * (1.0f - hh * hh);
-        daz[j] = dZ * z[j] * (1.0f - z[j]);
-        dh[j] = g[j] * z[j];
-      }
-      stage_half<HH>(a3h, a3l, lr, c0, H, dah);
-      stage_half<HH>(a4zh, a4zl, lr, c0, H, daz);
-      if (ok) {
-        st_half<HH>(da + (int64_t)row * H3 + c0, daz);
-        st_half<HH>(da + (int64_t)row * H3 + 2 * H + c0, dah);
-      }
-    }
-    sync_mma_operands();
-    if (threadIdx.x == 0) {
-      mma_seg(tm + 4 * H, tc::smem_u32(a3h), tc::smem_u32(a3l), H, 0, tc::smem_u32(lh_hi), tc::smem_u32(lh_lo), H, 0,
-              H, id_2h, true);
-      mma_seg(tm + 6 * H, tc::smem_u32(a4zh), tc::smem_u32(a4zl), H, 0, tc::smem_u32(lz_hi), tc::smem_u32(lz_lo), H,
-              0, H, id_2h, true);
-      tc::commit(&mbar);
-    }
-    wait_mma(&mbar, phase);
-    {
-      float dch[HH], drh[HH], dar[HH];
-      tmem_row_load<HH>(tm, 4 * H + c0, dch);          // dC_h
-      tmem_row_load<HH>(tm, 5 * H + c0, drh);          // dRH
-      if (ok) st_half<HH>(dCs + (int64_t)row * H3 + 2 * H + c0, dch, nd);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) {
-        dh[j] += drh[j] * r[j];
-        dar[j] = drh[j] * h[j] * r[j] * (1.0f - r[j]);
-      }
-      stage_half<HH>(a4rh, a4rl, lr, c0, H, dar);
-      if (ok) st_half<HH>(da + (int64_t)row * H3 + H + c0, dar);
-    }
-    sync_mma_operands();
-    if (threadIdx.x == 0) {
-      mma_seg(tm + 8 * H, tc::smem_u32(a4rh), tc::smem_u32(a4rl), H, 0, tc::smem_u32(lr_hi), tc::smem_u32(lr_lo), H,
-              0, H, id_2h, true);
-      tc::commit(&mbar);
-    }
-    wait_mma(&mbar, phase);
-#pragma unroll
-    for (int half = 0; half < 2; ++half) {               // [dC_z | dH_z], then [dC_r | dH_r]
-      float dc[HH], dx[HH];
-      tmem_row_load<HH>(tm, (6 + 2 * half) * H + c0, dc);
-      tmem_row_load<HH>(tm, (7 + 2 * half) * H + c0, dx);
-      if (ok) st_half<HH>(dCs + (int64_t)row * H3 + half * H + c0, dc, nd);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) dh[j] += dx[j];
-    }
-    if (ok) st_half<HH>(dHp + (int64_t)row * H + c0, dh);
-    tc::fence_before();
-    __syncthreads();
-    tc::fence_after();
-  }
-  tc::fence_before();
-  __syncthreads();
-  if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
-}
-
 // ------------------------------------------------------------------ GRU backward, v2
 // Same data path as k_tc_gru_fwd2 (TMA boxes -> swizzled raw tile -> tensor
 // memory A operands; single raw buffer: the next tile is requested as soon as
@@ -1169,123 +875,6 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
   }
   if (lane == 0) tc::bulk_wait_all();                // output boxes written before the CTA exits
   if (warp == 0) tc::tmem_free(tm, G::TCOLS);
-}
-
-// ------------------------------------------------------------------ Σ_rows Aᵀ·B
-// D_a = Σ_rows A_a[r,:]ᵀ·B[r,:] for NA (1 or 2) A operands sharing one B.
-//   A_0 = [A1 (FA1 cols) | A2 (FA2 cols)], A_1 = [A3 (FA3 cols) | ones (opt.)],
-// each padded to 128 feature rows (M = 128), B = [B (FB cols)] padded to N.
-// Tiles of kRK rows are staged TRANSPOSED (K = rows) by all 16 warps into one
-// of two operand stages while the tensor core consumes the other (mbarrier
-// per stage).  Per-CTA partials [NA][128 × N] go to part[blockIdx.x].
-constexpr int kRK = 32;
-constexpr int kAtbThreads = 512;
-
-struct AtbArgs {
-  int V;
-  const float* A1; int64_t lda1; int FA1;
-  const float* A2; int64_t lda2; int FA2;
-  const float* A3; int64_t lda3; int FA3; int ones;
-  const float* B; int64_t ldb; int FB;
-  float* part;
-};
-
-template <int N, int NA>
-__global__ void __launch_bounds__(kAtbThreads, 1) k_tc_atb(const AtbArgs p) {
-  extern __shared__ __align__(128) unsigned char sm[];
-  __shared__ uint64_t mbar[2];
-  __shared__ uint32_t tslot;
-  constexpr int ABYTES = 128 / 8 * (kRK / 4) * 144, BBYTES = N / 8 * (kRK / 4) * 144;   // padded layout
-  constexpr int STAGE = NA * 2 * ABYTES + 2 * BBYTES;
-  constexpr uint32_t NC = NA * N <= 32 ? 32 : (NA * N <= 64 ? 64 : (NA * N <= 128 ? 128 : (NA * N <= 256 ? 256 : 512)));
-  auto ahi = [&](int st, int a) { return sm + st * STAGE + a * 2 * ABYTES; };
-  auto alo = [&](int st, int a) { return sm + st * STAGE + a * 2 * ABYTES + ABYTES; };
-  auto bhi = [&](int st) { return sm + st * STAGE + NA * 2 * ABYTES; };
-  auto blo = [&](int st) { return sm + st * STAGE + NA * 2 * ABYTES + BBYTES; };
-  const int FA0 = p.FA1 + p.FA2, FAx = p.FA3 + (p.ones ? 1 : 0);
-  // zero the padding feature rows of both stages once (ones row: 1.0 per valid row, set per tile)
-  for (int st = 0; st < 2; ++st) {
-    for (int e = threadIdx.x; e < 128 * kRK; e += kAtbThreads) {
-      const int f = e / kRK, k = e % kRK;
-      const uint32_t off = tc::tmaj_off(f, k, kRK);
-      if (f >= FA0) { *reinterpret_cast<float*>(ahi(st, 0) + off) = 0.f; *reinterpret_cast<float*>(alo(st, 0) + off) = 0.f; }
-      if (NA > 1 && f >= p.FA3) { *reinterpret_cast<float*>(ahi(st, 1) + off) = 0.f; *reinterpret_cast<float*>(alo(st, 1) + off) = 0.f; }
-    }
-    for (int e = threadIdx.x; e < (N - p.FB) * kRK; e += kAtbThreads) {
-      const int f = p.FB + e / kRK, k = e % kRK;
-      *reinterpret_cast<float*>(bhi(st) + tc::tmaj_off(f, k, kRK)) = 0.f;
-      *reinterpret_cast<float*>(blo(st) + tc::tmaj_off(f, k, kRK)) = 0.f;
-    }
-  }
-  if ((threadIdx.x >> 5) == 0) tc::tmem_alloc(&tslot, NC);
-  if (threadIdx.x == 0) {
-    tc::mbar_init(&mbar[0], 1);
-    tc::mbar_init(&mbar[1], 1);
-    tc::fence_mbar_init();
-  }
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  const uint32_t tm = tslot;
-  uint32_t phase[2] = {0u, 0u};
-  bool pending[2] = {false, false};
-  const uint32_t idesc = tc::idesc_tf32(128, N, 0, 0);
-  const int ntiles = (p.V + kRK - 1) / kRK;
-  int it = 0;
-  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++it) {
-    const int st = it & 1;
-    if (pending[st]) {                      // the MMAs that read this stage must be done
-      tc::mbar_wait(&mbar[st], phase[st]);
-      phase[st] ^= 1u;
-      pending[st] = false;
-    }
-    const int r0 = tile * kRK, nv = p.V - r0;
-    tc::stage_rows_T(ahi(st, 0), alo(st, 0), p.A1 + (int64_t)r0 * p.lda1, p.lda1, nv, p.FA1, 0, 0, kRK);
-    if (p.FA2) tc::stage_rows_T(ahi(st, 0), alo(st, 0), p.A2 + (int64_t)r0 * p.lda2, p.lda2, nv, p.FA2, 0, p.FA1, kRK);
-    if (NA > 1) {
-      tc::stage_rows_T(ahi(st, 1), alo(st, 1), p.A3 + (int64_t)r0 * p.lda3, p.lda3, nv, p.FA3, 0, 0, kRK);
-      if (p.ones)
-        for (int k = threadIdx.x; k < kRK; k += kAtbThreads)
-          *reinterpret_cast<float*>(ahi(st, 1) + tc::tmaj_off(p.FA3, k, kRK)) = k < nv ? 1.0f : 0.0f;
-    }
-    tc::stage_rows_T(bhi(st), blo(st), p.B + (int64_t)r0 * p.ldb, p.ldb, nv, p.FB, 0, 0, kRK);
-    sync_mma_operands();
-    if (threadIdx.x == 0) {
-      const bool first = it == 0;
-      mma_T(tm, tc::smem_u32(ahi(st, 0)), tc::smem_u32(alo(st, 0)), tc::smem_u32(bhi(st)), tc::smem_u32(blo(st)), kRK,
-            idesc, first);
-      if (NA > 1)
-        mma_T(tm + N, tc::smem_u32(ahi(st, 1)), tc::smem_u32(alo(st, 1)), tc::smem_u32(bhi(st)),
-              tc::smem_u32(blo(st)), kRK, idesc, first);
-      tc::commit(&mbar[st]);
-    }
-    pending[st] = true;
-  }
-  for (int st = 0; st < 2; ++st)
-    if (pending[st]) { tc::mbar_wait(&mbar[st], phase[st]); phase[st] ^= 1u; }
-  tc::fence_after();
-  (void)FAx;
-  // epilogue: warp w reads TMEM lane quarter (w % 4), column block (w / 4) of 4
-  const int w = threadIdx.x >> 5, q = w & 3, cb = w >> 2;
-  const int row = q * 32 + (threadIdx.x & 31);
-  constexpr int TOT = NA * N;                           // 8-column groups interleaved over the 4 warp groups
-  float* out = p.part + (int64_t)blockIdx.x * NA * 128 * N;
-  for (int c = cb * 8; c < TOT; c += 32) {
-    float v[8];
-    if (it == 0) {
-#pragma unroll
-      for (int i = 0; i < 8; ++i) v[i] = 0.f;
-    } else {
-      tc::tmem_ld8(tm + ((uint32_t)(q * 32) << 16) + (uint32_t)c, v);
-      tc::tmem_wait_ld();
-    }
-    const int a = c / N, cc = c % N;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) out[(int64_t)a * 128 * N + (int64_t)row * N + cc + i] = v[i];
-  }
-  tc::fence_before();
-  __syncthreads();
-  if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
 }
 
 // ------------------------------------------------------------------ Σ_rows Aᵀ·B, v2 (TMA, MN-major)
@@ -2014,20 +1603,14 @@ stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const floa
     const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)kXwStages * 2 * 128 * Kp * 4 +
                         std::max<size_t>((size_t)128 * (N / 4 + 1 + ((N / 4) & 1)) * 16, 4 * 4096 + 1024);
     const int nb = std::min(ntiles, num_sms());
-    const char* dv = getenv("STG_XW_DEBUG");       // timing experiments only: skip parts of the pipeline
-    const int dbg = dv ? atoi(dv) : 0;
-    static const int box = [] {                    // epilogue: TMA box stores (1) or staged row stores (0)
-      const char* e = getenv("STG_XW_BOXSTORE");
-      return e ? atoi(e) : 1;
-    }();
     CUtensorMap tmP;
     STG_TRY(make_tmap_f32_store(&tmP, P, (uint64_t)V, (uint64_t)N, (uint64_t)N, 16, 32));
     if (H == 32) {
       STG_TRY(prep(k_tc_xw_pipe<96>, smem));
-      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div, tmP, box);
+      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, rs_div, tmP);
     } else {
       STG_TRY(prep(k_tc_xw_pipe<48>, smem));
-      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, dbg, rs_div, tmP, box);
+      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, rs_div, tmP);
     }
   } else {                            // 64 < F <= 128: one tile per CTA at a time
     if (rs_div != 1) return fail(STG_ERR_INVALID_ARG, "tc_xw: row-scale divisor needs F <= 64");
@@ -2101,20 +1684,6 @@ stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float
 
 int tc_atb_max_blocks() { return 2 * num_sms(); }   // k_tc_atb2 may run 2 CTAs per SM
 
-template <int N, int NA>
-static stg_status atb(const AtbArgs& args, int* nb_out, cudaStream_t s) {
-  constexpr int STAGE = NA * 2 * (128 / 8) * (kRK / 4) * 144 + 2 * (N / 8) * (kRK / 4) * 144;
-  const size_t smem = 2 * (size_t)STAGE;
-  STG_CUDA(cudaFuncSetAttribute(k_tc_atb<N, NA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const int ntiles = (args.V + kRK - 1) / kRK;
-  int nb = std::min(ntiles, num_sms());
-  if (nb < 1) nb = 1;
-  k_tc_atb<N, NA><<<nb, kAtbThreads, smem, s>>>(args);
-  count_launch();
-  *nb_out = nb;
-  return check_launch("tc_atb");
-}
-
 template <int NB, int RT, int S, int L = 2>
 static stg_status atb2_launch(const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb_out,
                               cudaStream_t s, int ctas_per_sm = 1) {
@@ -2168,18 +1737,19 @@ static stg_status atb2_dispatch(int NB, const CUtensorMap* m, const CUtensorMap&
   }
 }
 
-// the [RT x 32] "ones" tile (1.0 in column 0): the Σ_rows feature of dl
+// the [RT x 32] "ones" tile (1.0 in column 0): the Σ_rows feature of dl.  A
+// statically initialised device global (one instance per device's module), so
+// no allocation or copy happens at run time (safe inside stream capture, on any
+// device, from any thread).
+constexpr int kOnesMaxRT = 64;
+__device__ __align__(128) float g_ones_tile[kOnesMaxRT][32] = {{1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}, {1.f}};
+
 static stg_status ones_map(CUtensorMap* out, int RT, cudaStream_t s) {
-  static float* d = nullptr;
-  constexpr int kMaxRT = 64;
-  if (!d) {
-    std::vector<float> h((size_t)kMaxRT * 32, 0.f);
-    for (int r = 0; r < kMaxRT; ++r) h[(size_t)r * 32] = 1.f;
-    if (cudaMalloc(&d, h.size() * sizeof(float)) != cudaSuccess) return fail(STG_ERR_NO_MEMORY, "ones tile");
-    STG_CUDA(cudaMemcpy(d, h.data(), h.size() * sizeof(float), cudaMemcpyHostToDevice));
-  }
   (void)s;
-  return make_tmap_f32(out, d, RT, 32, 32, 32, RT, true);
+  if (RT > kOnesMaxRT) return fail(STG_ERR_INVALID_ARG, "ones tile: %d rows > %d", RT, kOnesMaxRT);
+  void* d = nullptr;
+  STG_CUDA(cudaGetSymbolAddress(&d, g_ones_tile));
+  return make_tmap_f32(out, static_cast<const float*>(d), RT, 32, 32, 32, RT, true);
 }
 
 // dW[f][c] += Σ_v X[v,f]·dP[v,c]  via D = dPᵀ·X  (M = 128 features of dP, N = 32·ceil(F/32)).
@@ -2607,3 +2177,23 @@ stg_status tc_seq_head_reduce(int nb, int H, const double* lpart, const float* g
 }
 
 }  // namespace stg
+
+// Diagnostic entry point (tests only): the fixed-order partial sum of the Σ AᵀB
+// reductions in either implementation (0 = serial per element, 1 = parallel over
+// the 16-partial groups, nb <= 1024), so a test can check that they agree bit for bit.
+extern "C" stg_status stg_debug_sum_parts(const float* part, int32_t nb, int32_t n, float* tot, int32_t variant,
+                                          stg_stream_t stream) {
+  using namespace stg;
+  if (!part || !tot || nb < 1 || n < 1) return fail(STG_ERR_INVALID_ARG, "stg_debug_sum_parts: nb=%d n=%d", nb, n);
+  cudaStream_t s = (cudaStream_t)stream;
+  if (variant == 1) {
+    if (nb > 16 * kSumMaxGroups) return fail(STG_ERR_INVALID_ARG, "stg_debug_sum_parts: nb=%d > %d", nb, 16 * kSumMaxGroups);
+    k_tc_sum_parts2<<<(n + 31) / 32, 256, 0, s>>>(part, nb, n, tot);
+  } else if (variant == 0) {
+    k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
+  } else {
+    return fail(STG_ERR_INVALID_ARG, "stg_debug_sum_parts: variant %d", variant);
+  }
+  count_launch();
+  return check_launch("stg_debug_sum_parts");
+}

@@ -112,3 +112,39 @@ def test_size_limits_rejected(stg):
     st = lib.stg_static_graph_create((1 << 31) - 2, (1 << 31) - 1 - 10, dummy, dummy, stg.STG_SELF_LOOPS, None,
                                      None, ctypes.byref(out))
     assert st == 2
+
+
+def test_two_streams_on_one_graph(stg):
+    """Aggregations of one graph on two streams at once (per-stream
+    scratch): every result equals the single-stream result bit for bit."""
+    cfg = gen.CONFIGS["C4"]
+    d = gen.dtdg(cfg)
+    g = stg.stg_dtdg_create(d.V, d.T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                            d.del_dst, stg.STG_SELF_LOOPS)
+    v = stg.stg_dtdg_get_snapshot(g, 1)
+    torch.cuda.synchronize()
+    xs = [to_gpu(gen.uniform_pm1(5 + i, 7, cfg.V * 96).reshape(cfg.V, 96)) for i in range(2)]
+    want = [stg.stg_gcn_aggregate_fwd(v, x).clone() for x in xs]
+    torch.cuda.synchronize()
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    outs = [[torch.empty(cfg.V, 96, device="cuda") for _ in range(8)] for _ in range(2)]
+    for k in range(8):
+        for i in range(2):
+            with torch.cuda.stream(streams[i]):
+                stg.stg_gcn_aggregate_fwd(v, xs[i], outs[i][k], stream=streams[i])
+    torch.cuda.synchronize()
+    for i in range(2):
+        for k in range(8):
+            assert torch.equal(outs[i][k], want[i]), (i, k)
+
+
+def test_wrong_dtype_rejected(stg):
+    """float64 / int64 tensors are refused at the binding (they would reach the
+    fp32 / int32 kernels as raw bytes)."""
+    cfg = gen.CONFIGS["C2"]
+    s, d = gen.static_edges(cfg)
+    g = stg.stg_static_graph_create(cfg.V, s, d, stg.STG_SELF_LOOPS)
+    x = torch.zeros(cfg.V, 8, dtype=torch.float64, device="cuda")
+    with pytest.raises(stg.StgError) as e:
+        stg.stg_gcn_aggregate_fwd(g.view(), x)
+    assert e.value.status == 1

@@ -80,3 +80,24 @@ def test_tc_gemm_mn_major_tma(stg, R, N):
     C = stg.stg_debug_tc_gemm(4, to_gpu(X), to_gpu(Y)).cpu().numpy()
     err = np.max(np.abs(C - X.T @ Y) / _cond(X.T, Y))
     assert err < 2e-6, err
+
+
+@pytest.mark.parametrize("nb", [1, 15, 17, 148, 296, 1024])
+@pytest.mark.parametrize("n", [1, 100, 4103])
+def test_sum_parts_parallel_is_bit_identical(stg, nb, n):
+    """k_tc_sum_parts2 (parallel over 16-partial groups) == k_tc_sum_parts (serial)
+    bit for bit, and both == the fp32 sum in the documented order (blocks of 16 in
+    order, then the block sums in order)."""
+    rng = np.random.default_rng(nb * 7919 + n)
+    part = rng.standard_normal((nb, n)).astype(np.float32) * np.float32(1e3) ** rng.integers(-1, 2, (nb, n))
+    pg = to_gpu(part)
+    a = stg.stg_debug_sum_parts(pg, 0).cpu().numpy()
+    b = stg.stg_debug_sum_parts(pg, 1).cpu().numpy()
+    assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
+    want = np.zeros(n, np.float32)
+    for b0 in range(0, nb, 16):
+        blk = np.zeros(n, np.float32)
+        for k in range(b0, min(b0 + 16, nb)):
+            blk = (blk + part[k]).astype(np.float32)
+        want = (want + blk).astype(np.float32)
+    assert np.array_equal(a.view(np.uint32), want.view(np.uint32))

@@ -332,3 +332,21 @@ def test_sequence_bptt_and_head_finite_differences():
     fun = lambda: oracle.train_sequence(gs, gs, p, Xs, Ys, H0)[0]
     for k in ("W", "b", "L", "l", "w_o", "b_o"):
         _fd_check(fun, p[k], grads[k], n=8)
+
+
+def test_mse_head_hand_derived_golden():
+    """orc_mse_head's LOSS VALUE and gradients against hand-derived closed forms
+    (tests/golden/mse_head_hand.json): pins the surrogate's definition itself
+    (mean, not sum; ReLU before w_o; b_o outside the ReLU), which the finite
+    difference tests cannot (they only check the gradient against the loss)."""
+    import json
+    import os
+    spec = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "mse_head_hand.json")))
+    for c in spec["cases"]:
+        Hn = np.array(c["H"], np.float64)
+        grads = {"w_o": np.zeros(Hn.shape[1]), "b_o": np.zeros(1)}
+        loss, dH = oracle.mse_head(Hn, np.array(c["y"]), np.array(c["w_o"]), c["b_o"], grads)
+        assert loss == pytest.approx(c["loss"], rel=1e-15, abs=1e-15), c["name"]
+        np.testing.assert_allclose(dH, np.array(c["dH"]), rtol=1e-15, atol=1e-15, err_msg=c["name"])
+        np.testing.assert_allclose(grads["w_o"], np.array(c["dw_o"]), rtol=1e-15, atol=1e-15, err_msg=c["name"])
+        assert grads["b_o"][0] == pytest.approx(c["db_o"], rel=1e-15, abs=1e-15), c["name"]
