@@ -55,6 +55,10 @@ def parse():
     ap.add_argument("--naive", action="store_true",
                     help="DTDG configs: NaiveGraph mode (every snapshot materialised at create, P:L202-204; "
                          "Table III's time/memory trade-off against the default on-demand snapshots)")
+    ap.add_argument("--order", default="linear-first", choices=["linear-first", "aggregate-first"],
+                    help="graph-convolution order (reading C14): linear-first Â(XW)+b, the headline (forward over "
+                         "the in-CSR at width 3H, backward over the out-CSR), or aggregate-first (ÂX)W+b (SURVEY "
+                         "§8(f) NEXT-1: forward at width F, no backward aggregation or backward snapshots)")
     ap.add_argument("--shard-sim", default=None, metavar="K/N",
                     help="(testing on one GPU) run rank K's row block of an N-way sharding, no process group")
     return ap.parse_args()
@@ -173,11 +177,26 @@ def static_reps(cfg) -> int:
     return max(1, int(2e7 // max(1, 2 * cfg.E)))
 
 
+def host_info() -> dict:
+    """nproc and the CPU model of the box the oracle baseline ran on."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.startswith("Model name:"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
 def run_reference(args):
     import gen
     import oracle
     cfg = gen.CONFIGS[args.config]
     oracle.build()
+    threads = oracle.use_openmp(True)          # the oracle on ALL host cores (its OpenMP build)
     edges, secs = 0, 0.0
     if cfg.kind == "static":
         s_, d_ = gen.static_edges(cfg)
@@ -213,7 +232,9 @@ def run_reference(args):
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
            "config": {"workload": workload_name(cfg), "config": cfg.name, "V": cfg.V, "F": cfg.F, "H": cfg.H, "T": T,
                       "sample": sample},
-           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                            "sample": sample + " (OpenMP build of the same oracle source, %d threads)" % threads,
+                            "host": host_info()},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
@@ -295,7 +316,11 @@ def main():
                                 d.del_dst, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS |
                                 (stg.STG_NAIVE if args.naive else 0), dist=dist_arg)
         E_t = [g.num_edges(t) for t in range(T)]
-    edges_per_step = 2 * sum(E_t)            # this rank's edges (whole graph unless sharded)
+    agg_first = args.order == "aggregate-first"
+    stg.stg_set_conv_order(1 if agg_first else 0)
+    # aggregated edges per epoch: every snapshot forward and backward (linear-first), forward only
+    # (aggregate-first: the backward needs no aggregation)
+    edges_per_step = (1 if agg_first else 2) * sum(E_t)   # this rank's edges (whole graph unless sharded)
     edges_all = edges_per_step
     if pg:
         te = torch.tensor([float(edges_per_step)], dtype=torch.float64, device=torch.device("cuda", local))
@@ -325,7 +350,7 @@ def main():
     Hbuf = [torch.empty(S, R, H, device=dev) for _ in range(2)]
     H0 = torch.zeros(R, H, device=dev)
     Gw = torch.empty(2, R, H, device=dev)
-    stack = stg.stg_state_stack_create(S * max(R, 1) * 3 * H * 4 + (64 << 20))
+    stack = stg.stg_state_stack_create(S * max(R, 1) * (3 * H + (F if agg_first else 0)) * 4 + (64 << 20))
     stream = torch.cuda.current_stream()
 
     def sgd():
@@ -376,8 +401,12 @@ def main():
 
     # ---------------- timed region (device-resident inputs)
     clocks = ClockSampler(local)
-    stg.stg_profile_enable(False)
+    # per-phase CUDA events are recorded during the timed region itself (on the stream
+    # each phase is launched on): they give the aggregation's average launch time for
+    # the roofline; the pipelined phases overlap, so the phase SPLIT comes from a
+    # single-stream pass below
     stg.stg_profile_read(reset=True)
+    stg.stg_profile_enable(True)
     if pg:
         dist.barrier()
     torch.cuda.synchronize()
@@ -392,6 +421,8 @@ def main():
     torch.cuda.synchronize()
     ms = ev0.elapsed_time(ev1)
     launches = stg.kernel_launch_count() - launches0
+    prof_timed = stg.stg_profile_read(reset=True)
+    stg.stg_profile_enable(False)
     if cg is not None:
         launches = launches_per_epoch * args.steps       # graph replays launch the captured kernels
     clk = clocks.stop()
@@ -404,37 +435,74 @@ def main():
     # sharded: the ranks advance the same T timestamps together; replicas: N epochs
     tsps = (1 if sharded else world) * T * args.steps / (ms / 1e3)
 
-    # ---------------- per-phase device times (profiled pass, same work)
-    stg.stg_profile_enable(True)
+    # ---------------- per-phase device times: single-stream pass (same work, one kernel after another)
+    nprof = max(1, min(args.steps, 2))
+    stg.stg_set_pipeline(False)
     stg.stg_profile_read(reset=True)
-    for _ in range(max(1, min(args.steps, 2))):
+    stg.stg_profile_enable(True)
+    e0s, e1s = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0s.record(stream)
+    for _ in range(nprof):
         epoch(Xdev, Ydev)
+    e1s.record(stream)
     torch.cuda.synchronize()
+    ms_single = e0s.elapsed_time(e1s) / nprof
     prof = stg.stg_profile_read(reset=True)
     stg.stg_profile_enable(False)
-    nprof = max(1, min(args.steps, 2))
+    stg.stg_set_pipeline(True)
+    sub = {k: prof.pop(k) for k in ("snap_step", "snap_transpose")}
 
-    # roofline of the dominant kernel: the aggregation (fwd + bwd, W = 3H)
-    Wagg = 3 * H
+    # roofline of the dominant kernel: the aggregation (fwd + bwd, W = 3H), timed in the timed region
+    Wagg = F if agg_first else 3 * H
     E_mean = sum(E_t) / T                       # this rank's edges per snapshot
     # compulsory bytes per launch: col 4E + rowptr 4(V+1) + node_ids 4V + row scale 4V
     # + read each source row once 4VW + write each output row 4VW
     # (sharded rank, mean of fwd and bwd: the fwd reads all V source rows and writes R rows, the bwd the
     # reverse; R = V unsharded gives 4E + 4(V+1) + 8V + 8VW)
     alg_bytes = 4 * E_mean + 2 * (V + 1) + 2 * (R + 1) + 4 * (V + R) + 4 * Wagg * (V + R)
-    agg_ms = prof["agg_fwd"][0] + prof["agg_bwd"][0]
-    agg_n = prof["agg_fwd"][1] + prof["agg_bwd"][1]
-    agg_avg_s = (agg_ms / agg_n) / 1e3 if agg_n else float("nan")
+    f_ms, f_n = prof_timed["agg_fwd"]
+    b_ms, b_n = prof_timed["agg_bwd"]
+    agg_avg_s = ((f_ms + b_ms) / (f_n + b_n)) / 1e3 if (f_n + b_n) else float("nan")
+    agg_fwd_s = (f_ms / f_n) / 1e3 if f_n else float("nan")
+    agg_bwd_s = (b_ms / b_n) / 1e3 if b_n else float("nan")
     peak, peak_src = measured_peaks()
     achieved = alg_bytes / agg_avg_s / 1e9
-    traffic = None
+    traffic, traffic_src = None, None
     tp = os.path.join(ROOT, "profiles", "agg_traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get("bytes_per_launch")
+            tj = json.load(open(tp))
+            traffic, traffic_src = tj.get("bytes_per_launch"), tj.get("source")
         except Exception:
             traffic = None
     step_ms_prof = sum(v[0] for v in prof.values()) / nprof
+    # snapshot builder roofline: compulsory bytes of ONE delta step of ONE CSR
+    # direction, unsharded: read/write col (4E each), rowptr (4(V+1) each), the whole-graph
+    # in/out degrees (read + write 4V each), node_ids (read deg 4V, write ids 4V), norms (8V),
+    # schedule items (16 B per row) and the sorted deltas (8 B per key, read by the merge and
+    # by the degree histogram: 16 B per delta)
+    snap_rl = None
+    if not static and sub["snap_step"][1]:
+        nd = [g.num_deltas(t, False) + g.num_deltas(t, True) for t in range(1, T)]
+        d_mean = sum(nd) / max(1, len(nd))
+        sbytes = 8 * E_mean + 8 * (V + 1) + 16 * V + 8 * V + 8 * V + 16 * V + 16 * d_mean
+        st_s = sub["snap_step"][0] / sub["snap_step"][1] / 1e3
+        snap_rl = {"bound": "hbm", "achieved": sbytes / st_s / 1e9, "peak": peak, "unit": "GB/s",
+                   "frac": sbytes / st_s / 1e9 / peak, "alg_bytes_per_step": sbytes,
+                   "avg_step_us": st_s * 1e6, "steps_per_epoch": sub["snap_step"][1] / nprof,
+                   "transposes_per_epoch": sub["snap_transpose"][1] / nprof,
+                   "avg_transpose_us": (1e3 * sub["snap_transpose"][0] / sub["snap_transpose"][1]
+                                        if sub["snap_transpose"][1] else None),
+                   "bytes_model": "one delta step of one CSR direction: 8E col + 8(V+1) rowptr + 16V degrees "
+                                  "+ 8V node_ids + 8V norms + 16V schedule items + 16|delta|",
+                   "timing": "CUDA events around each delta step in the single-stream pass"}
+    tensor_pipe = None
+    tpp = os.path.join(ROOT, "profiles", "tensor_pipe.json")
+    if os.path.exists(tpp):
+        try:
+            tensor_pipe = json.load(open(tpp))
+        except Exception:
+            tensor_pipe = None
 
     # ---------------- end-to-end through the public API with host buffers
     e2e = None
@@ -516,21 +584,29 @@ def main():
                        "a step waits only for its own inputs) from pinned host memory every timestep on a copy "
                        "stream overlapped with the previous sequence; loss read back every epoch"}
 
-    # ---------------- CPU baseline: the oracle on one C5 timestep (rank 0, N=1 only)
+    # ---------------- CPU baseline: the oracle on one C5 timestep, 1 core and all cores (rank 0, N=1 only)
     cpu = None
     if rank == 0 and world == 1 and not sim and not args.no_cpu_baseline:
         import oracle
         oracle.build()
-        if static:
-            reps = static_reps(cfg)
-            e_c, dt_c = oracle_timestep_static(cfg, oracle.static_graph(V, s_e, d_e, self_loops=True), 1, reps)
-            smp = "%d %s timesteps: TGCN fwd + MSE head + bwd on the static CSR" % (reps, cfg.name)
-        else:
-            S0 = next(oracle.snapshot_sets_fold(d, self_loops=True))
-            e_c, dt_c, _ = oracle_timestep(cfg, d, 1, S0)
-            smp = "one %s timestep (t=1): fold S_0->S_1, CSR pair, TGCN fwd + MSE head + bwd" % cfg.name
-        cpu = {"value": e_c / dt_c, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": smp + ", fp64, single thread; %.1f s" % dt_c}
+        res = {}
+        for omp in (False, True):
+            thr = oracle.use_openmp(omp)
+            if static:
+                reps = static_reps(cfg)
+                e_c, dt_c = oracle_timestep_static(cfg, oracle.static_graph(V, s_e, d_e, self_loops=True), 1, reps)
+                smp = "%d %s timesteps: TGCN fwd + MSE head + bwd on the static CSR" % (reps, cfg.name)
+            else:
+                S0 = next(oracle.snapshot_sets_fold(d, self_loops=True))
+                e_c, dt_c, _ = oracle_timestep(cfg, d, 1, S0)
+                smp = "one %s timestep (t=1): fold S_0->S_1, CSR pair, TGCN fwd + MSE head + bwd" % cfg.name
+            res[omp] = (e_c / dt_c, thr, dt_c)
+        oracle.use_openmp(False)
+        cpu = {"value": res[True][0], "unit": UNIT, "cores": res[True][1], "kind": "oracle",
+               "sample": smp + ", fp64; all cores: the OpenMP build of the same oracle source (row loops "
+                               "split over %d threads), %.1f s" % (res[True][1], res[True][2]),
+               "single_core": {"value": res[False][0], "unit": UNIT, "cores": 1, "seconds": res[False][2]},
+               "host": host_info()}
 
     if rank == 0 or sim:
         out = {
@@ -544,6 +620,8 @@ def main():
                        "l2": ("inputs larger than L2 (X_t 256 MB, graph ~0.3 GB, state 8 GB)" if cfg.name == "C5"
                               else "working set fits in L2 (not flushed between epochs)"),
                        "cuda_graph": cg is not None,
+                       "conv_order": args.order + (" (Â(XW)+b, headline)" if not agg_first else
+                                                   " ((ÂX)W+b, NEXT-1: value counts forward aggregations only)"),
                        "schedule": "sequence-batched (NEXT-1)" if batched else "per-timestamp Algorithm 1",
                        "parallelism": ("row-block shards x%d, sharded mode: X_t row-sharded, P' gathered from "
                                        "its owners over CUDA-IPC peer memory inside the aggregation, partial dP "
@@ -565,9 +643,24 @@ def main():
                                             "+ 4VW (each source row once) + 4VW (output)",
                          "kernel": "k_agg_stream + k_agg_hubs (fwd in-CSR + bwd out-CSR, W=%d)" % Wagg,
                          "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": agg_avg_s * 1e3,
-                         "peak_source": peak_src},
+                         "avg_fwd_ms": agg_fwd_s * 1e3, "avg_bwd_ms": agg_bwd_s * 1e3,
+                         "launches_timed": f_n + b_n,
+                         "timing": "CUDA events around every aggregation launch on its stream, over the timed region",
+                         "traffic_source": traffic_src, "peak_source": peak_src},
+            "aggregation_edges_per_s": (2 * E_mean / (agg_fwd_s + agg_bwd_s)) if f_n and b_n else None,
+            "aggregation_metric": "SURVEY §8(d): 2E / (t_fwd + t_bwd) at W = 3H for one snapshot (mean E_t), "
+                                  "launch times from the timed region",
+            "snapshot_roofline": snap_rl,
+            "tensor_pipe": tensor_pipe,
+            "single_stream_ms_per_step": ms_single,
             "phases_ms_per_step": {k: v[0] / nprof for k, v in prof.items()},
             "phase_share": {k: (v[0] / nprof) / step_ms_prof for k, v in prof.items()} if step_ms_prof else None,
+            "fig9_split": ({"gnn": 1.0 - (prof["snapshot"][0] / nprof) / step_ms_prof,
+                            "graph_update": (prof["snapshot"][0] / nprof) / step_ms_prof}
+                           if step_ms_prof and not static else None),
+            "phases_note": "phases from a single-stream pass of the same epoch (stg_set_pipeline(0)): no overlap, "
+                           "so the shares are the exact Fig. 9 split (P:L316, L345); the timed region runs the "
+                           "three-stream pipeline",
             "clocks": clk,
             "e2e": e2e,
             "cpu_baseline": cpu,

@@ -49,10 +49,15 @@ int32_t stg_version(void);
 /* Number of device kernels this library launched since load (all threads). */
 int64_t stg_kernel_launch_count(void);
 
-/* Optional allocator hook (e.g. PyTorch's caching allocator).  alloc returns a
- * device pointer of >= bytes (256-byte aligned) or NULL; free releases it.
- * Both are called from the host thread that calls into the library.  Passing
- * NULL restores cudaMalloc/cudaFree.  Must be set before objects are created. */
+/* Optional allocator hook (the Python binding installs PyTorch's caching
+ * allocator at import; env STG_TORCH_ALLOCATOR=0 keeps cudaMalloc).  Every
+ * library-owned device buffer (graph / DTDG snapshot slots and deltas, state
+ * stack arena, scratch) then comes from alloc: bytes >= requested, 256-byte
+ * aligned, or NULL (the call fails with STG_ERR_NO_MEMORY).  A block is
+ * returned to the free function it was allocated with (after a device
+ * synchronisation, cudaFree's ordering), so the hook may be changed at any
+ * time.  Called from the host thread that calls into the library.  Passing
+ * NULL, NULL restores cudaMalloc/cudaFree. */
 typedef void* (*stg_alloc_fn)(size_t bytes, stg_stream_t stream, void* ctx);
 typedef void (*stg_free_fn)(void* ptr, stg_stream_t stream, void* ctx);
 stg_status stg_set_allocator(stg_alloc_fn alloc, stg_free_fn free_fn, void* ctx);
@@ -94,10 +99,9 @@ typedef struct {
  * or, for a DTDG, until the next stg_dtdg_get_* call on it.  Layout (Fig. 3,
  * P:L183-185):
  *   forward CSR  : in_rowptr[R+1] (R = row_end-row_begin, local rows),
- *                  in_col[E] = source ids ascending within a row,
- *                  in_row[E] = the destination id of every in-edge (COO)
- *   backward CSR : out_rowptr[V+1], out_col[E] = destination ids ascending,
- *                  out_row[E] = the source id of every out-edge (COO)
+ *                  in_col[E] = source ids ascending within a row
+ *   backward CSR : out_rowptr[V+1], out_col[E] = destination ids ascending
+ *   (no COO row arrays are kept: a row's edges are [rowptr[r], rowptr[r+1]))
  *   out_eid[E]   : in-CSR position of out-edge j (shared edge label), or NULL
  *   in_deg/out_deg[V], in_ids/out_ids[V] = vertices by degree desc, id asc
  *   norm_src/norm_dst[V] fp32 GCN normalisation vectors (reading C1)
@@ -109,8 +113,8 @@ typedef struct {
   int32_t row_begin, row_end;
   int32_t timestamp;            /* -1 for a static graph */
   int64_t num_edges;            /* edges held by this view (local edges if sharded) */
-  const int32_t *in_rowptr, *in_col, *in_row;
-  const int32_t *out_rowptr, *out_col, *out_row;
+  const int32_t *in_rowptr, *in_col;
+  const int32_t *out_rowptr, *out_col;
   const int32_t *out_eid;
   const int32_t *in_deg, *out_deg, *in_ids, *out_ids;
   const float *norm_src, *norm_dst;
@@ -163,7 +167,7 @@ stg_status stg_dtdg_get_backward_snapshot(stg_dtdg* g, int32_t t, stg_stream_t s
 enum { STG_PART_IN = 1u << 0, STG_PART_OUT = 1u << 1, STG_PART_EID = 1u << 2 /* implies both */ };
 /* Get-Graph (backward = 0) / Get-Backward-Graph (backward = 1) of the parts in
  * `parts` (STG_PART_*; at least one direction).  The view's pointers of the
- * parts not requested may be NULL (in_rowptr/in_col/in_row/in_ids/in_sched
+ * parts not requested may be NULL (in_rowptr/in_col/in_ids/in_sched
  * for the in-CSR, likewise out_*; out_eid unless STG_PART_EID).  Same
  * validity and stream rules as stg_dtdg_get_snapshot, which equals
  * parts = IN|OUT|EID (EID only with STG_EDGE_IDS). */
@@ -240,11 +244,7 @@ stg_status stg_aggregate_set_strategy(int32_t strategy);
  * key 0: neighbour rows in flight per warp, 4 | 8 | 16 (default 4);
  * key 1: minimum resident blocks per SM (register budget), 2..6 (default 6;
  *        supported pairs (rows, blocks): (4,6) (8,4) (16,2) (16,3));
- * key 2: 32 | 64 (default 32): strategy 2 serves launch widths above this;
- * key 3: source-row cache hints 0..4 (default 0 = none; with (4,6) only):
- *        1 = rows u < hotk L2 evict_last, others L1 no_allocate + L2 evict_first,
- *        2 = others only, 3 = hot only, 4 = 1 without the L1 no_allocate;
- * key 4: hotk, the hot prefix length of the source order (rows). */
+ * key 2: 32 | 64 (default 32): strategy 2 serves launch widths above this. */
 stg_status stg_aggregate_set_param(int32_t key, int64_t value);
 
 /* ---- TGCN (GCN + GRU; reading C13-C15) ----
@@ -488,11 +488,34 @@ stg_status stg_tgcn2_peer_bwd(int32_t phase, const stg_csr_view* g, const stg_tg
  * around each phase (bench.py; the GNN vs graph-update split of Fig. 9,
  * P:L316/L345).  phase: 0 aggregation fwd, 1 aggregation bwd, 2 snapshot
  * build (Get-Graph / Get-Backward-Graph), 3 P' = X·W, 4 GRU fwd, 5 GRU bwd,
- * 6 dW, 7 head, 8 dL/dl/db reductions.  Phases launched on different streams
- * may overlap.  stg_profile_read synchronises on the recorded events and
- * returns the accumulated milliseconds and count (reset != 0 clears them). */
+ * 6 dW, 7 head, 8 dL/dl/db reductions; sub-phases of 2: 9 one delta step of
+ * one CSR direction (Algorithm 2's update), 10 one transpose (Algorithm 3).
+ * Phases launched on different streams may overlap (stg_set_pipeline(0)
+ * serialises a training sequence for an exact split).  stg_profile_read
+ * synchronises on the recorded events and returns the accumulated
+ * milliseconds and count (reset != 0 clears them). */
 stg_status stg_profile_enable(int32_t on);
 stg_status stg_profile_read(int32_t phase, double* total_ms, int64_t* count, int32_t reset);
+
+/* Schedule of stg_tgcn_train_sequence(_ev): 1 (default; env STG_SEQ_PIPELINE=0
+ * sets 0 at load) = the three-stream pipeline (snapshot builds and the
+ * H-independent work overlap the GRU chain); 0 = everything on the caller's
+ * stream, one kernel after another (same arithmetic, same results; used to
+ * measure the per-phase split). */
+stg_status stg_set_pipeline(int32_t on);
+
+/* Order of the graph convolution in the TGCN step (reading C14; SURVEY §8(f)
+ * NEXT-1): 0 (default) = linear-first C = Â(XW) + b — the forward aggregates
+ * P' = n_src ⊙ XW (width 3H) over the in-CSR and the backward aggregates dC'
+ * over the out-CSR (dP = Âᵀ dC, dW = Xᵀ dP); 1 = aggregate-first C = (ÂX)W + b —
+ * the forward aggregates X (width F) and keeps ÂX on the state stack, the
+ * backward needs no graph (dW = (ÂX)ᵀ dC), so a DTDG sequence builds no
+ * backward snapshots.  Same model, same gradients up to rounding.  Order 1
+ * needs the tensor-core path (H in {16, 32}, F <= 64, F % 4 == 0) and is used
+ * by stg_tgcn_step / _backward and stg_tgcn_train_sequence(_ev); the state
+ * stack then needs V·(3H + F)·4 bytes per step.  STG_ERR_INVALID_ARG for
+ * another value. */
+stg_status stg_set_conv_order(int32_t order);
 
 /* Diagnostic tcgen05 3xTF32 GEMM (tests pin the UMMA conventions with it):
  * mode 0: C[M,N] = A[M,K]·B[K,N] (M % 128 == 0, K % 8 == 0, K <= 256);

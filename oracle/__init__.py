@@ -24,23 +24,48 @@ _SRC = os.path.join(_HERE, "stg_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 
-def build(force: bool = False) -> str:
-    """Compile stg_oracle.c with plain gcc -O2 (no fast-math)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        tmp = _LIB + ".tmp%d" % os.getpid()
-        subprocess.check_call(["gcc", "-O2", "-std=c99", "-fPIC", "-shared", "-fno-fast-math",
-                               "-o", tmp, _SRC, "-lm"])
-        os.replace(tmp, _LIB)
-    return _LIB
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")
 
 
-_lib = None
+def build(force: bool = False, omp: bool = False) -> str:
+    """Compile stg_oracle.c with plain gcc -O2 (no fast-math).  omp=True builds the
+    SAME source with -fopenmp (liboracle_omp.so): its `#pragma omp` lines split the
+    row loops over threads — used only to time the all-core CPU baseline
+    (bench.py); every parity test runs the plain single-thread build."""
+    out = _LIB_OMP if omp else _LIB
+    if force or not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(_SRC):
+        tmp = out + ".tmp%d" % os.getpid()
+        subprocess.check_call(["gcc", "-O2", "-std=c99", "-fPIC", "-shared", "-fno-fast-math"] +
+                              (["-fopenmp"] if omp else []) + ["-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, out)
+    if not omp:
+        build(force, omp=True)
+    return out
+
+
+_libs = {}
+_mode = {"omp": False}
+
+
+def use_openmp(on: bool) -> int:
+    """Route the oracle calls to the OpenMP timing build (True) or the plain build
+    (False).  Returns the thread count the OpenMP runtime will use."""
+    _mode["omp"] = bool(on)
+    if not on:
+        return 1
+    lib()
+    try:
+        gomp = ctypes.CDLL("libgomp.so.1")
+        return int(gomp.omp_get_max_threads())
+    except OSError:
+        return os.cpu_count() or 1
 
 
 def lib():
-    global _lib
-    if _lib is None:
-        _lib = ctypes.CDLL(build())
+    omp = _mode["omp"]
+    if omp not in _libs:
+        _lib = ctypes.CDLL(build(omp=omp) if omp else build())
+        _libs[omp] = _lib
         P = ctypes.c_void_p
         i32, i64 = ctypes.c_int32, ctypes.c_int64
         _lib.orc_edge_set.restype = i64
@@ -69,7 +94,7 @@ def lib():
         _lib.orc_tgcn2_bwd.argtypes = [i32, i32, i32] + [P] * 19
         _lib.orc_mse_head.restype = ctypes.c_double
         _lib.orc_mse_head.argtypes = [i32, i32, P, P, P, ctypes.c_double, P, P, P]
-    return _lib
+    return _libs[omp]
 
 
 def _p(a: np.ndarray):

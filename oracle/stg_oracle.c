@@ -147,6 +147,9 @@ void orc_csr_build(int32_t V, int64_t n, const uint64_t* S, int32_t dgl_both,
 void orc_aggregate(int32_t R, const int32_t* rowptr, const int32_t* col,
                    const double* nrow, const double* ncol, int32_t W,
                    const double* x, double* y) {
+#ifdef _OPENMP
+#pragma omp parallel for schedule(dynamic, 1024)
+#endif
   for (int32_t v = 0; v < R; ++v) {
     double* yv = y + (int64_t)v * W;
     for (int32_t k = 0; k < W; ++k) yv[k] = 0.0;
@@ -263,6 +266,9 @@ void orc_tgcn_fwd(int32_t V, int32_t F, int32_t H,
                   double* C, double* Z, double* R, double* Hh, double* Hn) {
   const int32_t H3 = 3 * H;
   double* P = (double*)calloc((size_t)V * H3 + 1, sizeof(double));
+#ifdef _OPENMP
+#pragma omp parallel for schedule(static)
+#endif
   for (int32_t v = 0; v < V; ++v)
     for (int32_t c = 0; c < H3; ++c) {
       double s = 0.0;
@@ -273,6 +279,9 @@ void orc_tgcn_fwd(int32_t V, int32_t F, int32_t H,
   for (int64_t i = 0; i < (int64_t)V * H3; ++i) C[i] += b[i % H3];
   free(P);
   const double* Lz = L;  const double* Lr = L + 2 * H * H;  const double* Lh = L + 4 * H * H;
+#ifdef _OPENMP
+#pragma omp parallel for schedule(static)
+#endif
   for (int32_t v = 0; v < V; ++v) {
     const double* cz = C + (int64_t)v * H3;  const double* cr = cz + H;  const double* ch = cz + 2 * H;
     const double* hv = Hp + (int64_t)v * H;
@@ -320,14 +329,24 @@ void orc_tgcn_bwd(int32_t V, int32_t F, int32_t H,
                   double* dHp, double* dW, double* db, double* dL, double* dl) {
   const int32_t H3 = 3 * H;
   const double* Lz = L;  const double* Lr = L + 2 * H * H;  const double* Lh = L + 4 * H * H;
-  double* dLz = dL;  double* dLr = dL + 2 * H * H;  double* dLh = dL + 4 * H * H;
   double* dC = (double*)calloc((size_t)V * H3 + 1, sizeof(double));
+  /* (the OpenMP timing build, bench.py's all-core baseline, gives every thread its
+   * own row scratch and reduces dL / dl over threads; the plain build runs the
+   * loop below as written, rows in ascending order) */
+#ifdef _OPENMP
+#pragma omp parallel
+#endif
+  {
   double* dah = (double*)malloc(sizeof(double) * (size_t)(H + 1));
   double* dar = (double*)malloc(sizeof(double) * (size_t)(H + 1));
   double* daz = (double*)malloc(sizeof(double) * (size_t)(H + 1));
   double* dR = (double*)malloc(sizeof(double) * (size_t)(H + 1));
   double* dRH = (double*)malloc(sizeof(double) * (size_t)(H + 1));
+#ifdef _OPENMP
+#pragma omp for schedule(static) reduction(+ : dL[:6 * H * H], dl[:3 * H])
+#endif
   for (int32_t v = 0; v < V; ++v) {
+    double* dLz = dL;  double* dLr = dL + 2 * H * H;  double* dLh = dL + 4 * H * H;
     const double* g = G + (int64_t)v * H;  const double* hv = Hp + (int64_t)v * H;
     const double* z = Z + (int64_t)v * H;  const double* r = R + (int64_t)v * H;
     const double* hh = Hh + (int64_t)v * H;
@@ -371,15 +390,20 @@ void orc_tgcn_bwd(int32_t V, int32_t F, int32_t H,
       }
     for (int32_t j = 0; j < H; ++j) { dl[j] += daz[j]; dl[H + j] += dar[j]; dl[2 * H + j] += dah[j]; }
   }
+  free(dah); free(dar); free(daz); free(dR); free(dRH);
+  }
   for (int64_t i = 0; i < (int64_t)V * H3; ++i) db[i % H3] += dC[i];
   double* dP = (double*)calloc((size_t)V * H3 + 1, sizeof(double));
   orc_aggregate(V, out_rowptr, out_col, n_src, n_dst, H3, dC, dP);   /* Âᵀ·dC */
+#ifdef _OPENMP
+#pragma omp parallel for schedule(static) reduction(+ : dW[:F * H3])
+#endif
   for (int32_t v = 0; v < V; ++v)
     for (int32_t f = 0; f < F; ++f) {
       double xv = X[(int64_t)v * F + f];
       for (int32_t c = 0; c < H3; ++c) dW[(int64_t)f * H3 + c] += xv * dP[(int64_t)v * H3 + c];
     }
-  free(dP); free(dC); free(dah); free(dar); free(daz); free(dR); free(dRH);
+  free(dP); free(dC);
 }
 
 /* ---------------------------------------------------------------------------

@@ -8,8 +8,10 @@ on a non-OK status.
 """
 from __future__ import annotations
 
+import atexit
 import ctypes
 import os
+import sys
 
 import numpy as np
 import torch
@@ -48,8 +50,8 @@ class stg_dist(ctypes.Structure):
 class stg_csr_view(ctypes.Structure):
     _fields_ = [("num_nodes", _i32), ("row_begin", _i32), ("row_end", _i32), ("timestamp", _i32),
                 ("num_edges", _i64),
-                ("in_rowptr", _P), ("in_col", _P), ("in_row", _P),
-                ("out_rowptr", _P), ("out_col", _P), ("out_row", _P),
+                ("in_rowptr", _P), ("in_col", _P),
+                ("out_rowptr", _P), ("out_col", _P),
                 ("out_eid", _P),
                 ("in_deg", _P), ("out_deg", _P), ("in_ids", _P), ("out_ids", _P),
                 ("norm_src", _P), ("norm_dst", _P),
@@ -133,6 +135,8 @@ _decl("stg_tgcn_train_sequence_batched", [_P, _i32, ctypes.POINTER(stg_tgcn_para
                                           _P])
 _decl("stg_partition_rows", [_i32, _P, _i32, ctypes.POINTER(_i32), _P])
 _decl("stg_profile_enable", [_i32])
+_decl("stg_set_pipeline", [_i32])
+_decl("stg_set_conv_order", [_i32])
 _decl("stg_debug_tc_gemm", [_i32, _i32, _i32, _i32, _i32, _P, _P, _P, _P])
 _decl("stg_debug_sum_parts", [_P, _i32, _i32, _P, _i32, _P])
 _decl("stg_aggregate_set_strategy", [_i32])
@@ -174,7 +178,7 @@ ABI_SYMBOLS = [
     "stg_state_stack_create", "stg_state_stack_depth", "stg_state_stack_destroy",
     "stg_tgcn_step", "stg_tgcn_step_backward", "stg_mse_head", "stg_mse_head_ex", "stg_sgd_update", "stg_tgcn_train_sequence",
     "stg_tgcn_train_sequence_batched", "stg_tgcn_train_sequence_ev",
-    "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_debug_sum_parts", "stg_aggregate_set_strategy",
+    "stg_partition_rows", "stg_profile_enable", "stg_profile_read", "stg_debug_tc_gemm", "stg_debug_sum_parts", "stg_set_pipeline", "stg_set_conv_order", "stg_aggregate_set_strategy",
     "stg_aggregate_set_param",
     "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm", "stg_tgcn2_step", "stg_tgcn2_step_backward",
     "stg_peer_alloc", "stg_peer_free", "stg_peer_open", "stg_peer_close", "stg_allgather_rows",
@@ -182,7 +186,66 @@ ABI_SYMBOLS = [
     "stg_tgcn_step_backward_peer", "stg_tgcn_dw", "stg_tgcn2_peer_fwd", "stg_tgcn2_peer_bwd",
 ]
 
-PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head", "dl"]
+# ---------------------------------------------------------------- allocator hook
+# Library-owned device memory (snapshot slots, deltas, state stack, scratch) from
+# PyTorch's caching allocator (include/stg.h stg_set_allocator), so torch's memory
+# statistics cover it and freed blocks return to torch's pool.
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+_lib.stg_set_allocator.argtypes = [_ALLOC_FN, _FREE_FN, ctypes.c_void_p]
+_lib.stg_set_allocator.restype = _i32
+_hook_stats = {"alloc": 0, "free": 0, "bytes": 0}
+_exiting = [False]
+# at interpreter exit, objects still alive are left to the process teardown: their
+# blocks belong to torch's allocator, which must not be called back during finalisation
+atexit.register(lambda: _exiting.__setitem__(0, True))
+
+
+def _torch_alloc(nbytes, stream, ctx):
+    try:
+        p = torch.cuda.caching_allocator_alloc(int(nbytes), device=torch.cuda.current_device(),
+                                               stream=int(stream or 0))
+    except Exception:                      # out of memory: the library reports STG_ERR_NO_MEMORY
+        return None
+    _hook_stats["alloc"] += 1
+    _hook_stats["bytes"] += int(nbytes)
+    return p
+
+
+def _torch_free(ptr, stream, ctx):
+    _hook_stats["free"] += 1
+    torch.cuda.caching_allocator_delete(int(ptr))
+
+
+_hooks = (_ALLOC_FN(_torch_alloc), _FREE_FN(_torch_free))
+
+
+def use_torch_allocator(on: bool = True):
+    """Route libstg's device allocations through torch's caching allocator (default at
+    import unless STG_TORCH_ALLOCATOR=0), or back to cudaMalloc (on=False)."""
+    if on:
+        _check(_lib.stg_set_allocator(_hooks[0], _hooks[1], None))
+    else:
+        _check(_lib.stg_set_allocator(_ALLOC_FN(0), _FREE_FN(0), None))
+
+
+def allocator_stats() -> dict:
+    """Calls of the torch allocator hook so far (alloc / free counts, bytes requested)."""
+    return dict(_hook_stats)
+
+
+PHASES = ["agg_fwd", "agg_bwd", "snapshot", "xw", "gru_fwd", "gru_bwd", "dw", "head", "dl", "snap_step",
+          "snap_transpose"]
+
+
+def stg_set_pipeline(on: bool):
+    """Training-sequence schedule: True = three-stream pipeline, False = one stream (exact phase split)."""
+    _check(_lib.stg_set_pipeline(int(bool(on))))
+
+
+def stg_set_conv_order(order: int):
+    """0 = linear-first Â(XW) + b (default), 1 = aggregate-first (ÂX)W + b (NEXT-1)."""
+    _check(_lib.stg_set_conv_order(int(order)))
 
 
 def stg_profile_enable(on: bool = True):
@@ -261,6 +324,8 @@ class Graph:
             self.handle = None
 
     def __del__(self):
+        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+            return
         try:
             self.close()
         except Exception:
@@ -295,6 +360,8 @@ class Dtdg:
             self.handle = None
 
     def __del__(self):
+        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+            return
         try:
             self.close()
         except Exception:
@@ -378,8 +445,8 @@ def view_arrays(v: stg_csr_view, stream=None) -> dict:
     """Copies of the view's arrays as CUDA tensors (for tests / inspection)."""
     V, E = v.num_nodes, v.num_edges
     R = v.row_end - v.row_begin
-    spec = {"in_rowptr": (R + 1, torch.int32), "in_col": (E, torch.int32), "in_row": (E, torch.int32),
-            "out_rowptr": (V + 1, torch.int32), "out_col": (E, torch.int32), "out_row": (E, torch.int32),
+    spec = {"in_rowptr": (R + 1, torch.int32), "in_col": (E, torch.int32),
+            "out_rowptr": (V + 1, torch.int32), "out_col": (E, torch.int32),
             "out_eid": (E, torch.int32), "in_deg": (V, torch.int32), "out_deg": (V, torch.int32),
             "in_ids": (V, torch.int32), "out_ids": (V, torch.int32), "norm_src": (V, torch.float32),
             "norm_dst": (V, torch.float32)}
@@ -399,6 +466,12 @@ def view_arrays(v: stg_csr_view, stream=None) -> dict:
             hdr = torch.empty(2, dtype=torch.int32, device="cuda")
             _check(_lib.stg_memcpy(ctypes.c_void_p(hdr.data_ptr()), ctypes.c_void_p(p), 8, 0, _stream(stream)))
             out[k] = hdr
+    # COO row ids implied by the row pointers (derived here; the library keeps none)
+    for k, rp, base in (("in_row", "in_rowptr", v.row_begin), ("out_row", "out_rowptr", 0)):
+        if rp in out:
+            n = out[rp].numel() - 1
+            out[k] = torch.repeat_interleave(torch.arange(base, base + n, device="cuda", dtype=torch.int32),
+                                             torch.diff(out[rp]).long())
     return out
 
 
@@ -471,6 +544,8 @@ class StateStack:
             self.handle = None
 
     def __del__(self):
+        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+            return
         try:
             self.close()
         except Exception:
@@ -648,6 +723,8 @@ class PeerBuffer:
             self.ptr = None
 
     def __del__(self):
+        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+            return
         try:
             self.close()
         except Exception:
@@ -761,3 +838,7 @@ def stg_tgcn2_peer_bwd(phase: int, v: stg_csr_view, params: dict, X_loc, dH_next
                                    int(rank), world, b, pp,
                                    ctypes.c_void_p(_row_ptr(part_out)) if part_out is not None else None,
                                    stack.handle, _stream(stream)))
+
+
+if os.environ.get("STG_TORCH_ALLOCATOR", "1") != "0" and torch.cuda.is_available():
+    use_torch_allocator(True)

@@ -287,24 +287,7 @@ struct Agg2Args {
   // SCOL instantiation reads them.
   const float* ew;
   const int32_t* eid;
-  // source-row cache hints (HINT > 0): rows u < hotk are the hot prefix of a
-  // hot-first source order (L2 evict_last), the rest stream through (L1
-  // no_allocate, L2 evict_first)
-  int32_t hotk;
 };
-
-__device__ __forceinline__ float4 ld_hint(const float4* p, uint64_t pol) {
-  float4 v;
-  asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
-  return v;
-}
-__device__ __forceinline__ float4 ld_hint_na(const float4* p, uint64_t pol) {
-  float4 v;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
-  return v;
-}
 
 // Strategy 1: software-pipelined degree-ordered items.  A warp serves 32/G
 // items at once (G lanes × VPL float4 per row) and runs a three-stage pipeline
@@ -534,7 +517,7 @@ __global__ void __launch_bounds__(256) k_agg_hubs(const Agg2Args a, const int32_
   }
 }
 
-template <int D, int MINB, bool SCOL, bool PEER, int HINT = 0>
+template <int D, int MINB, bool SCOL, bool PEER>
 __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args a, uint32_t* __restrict__ queue) {
   constexpr int NW = kAggThreads / 32;
   __shared__ __align__(16) int4 s_items[NW][2][32];
@@ -543,11 +526,6 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
   __shared__ int32_t s_pbnd[STG_MAX_PEERS];
   const unsigned FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  uint64_t pol_first = 0, pol_last = 0;
-  if (HINT) {
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_first));
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
-  }
   if (PEER) {
     if (threadIdx.x < STG_MAX_PEERS) {
       s_pbase[threadIdx.x] = a.pbase[threadIdx.x];
@@ -691,12 +669,7 @@ __global__ void __launch_bounds__(kAggThreads, MINB) k_agg_stream(const Agg2Args
             v[d] = __ldg(reinterpret_cast<const float4*>(r) + lanec);
           } else {
             const uint32_t u = (uint32_t)__shfl_sync(FULL, uc, (j0 + d) & 31);
-            const float4* xp = xl + (size_t)u * ld4;
-            if (HINT == 0) v[d] = __ldg(xp);
-            else if (HINT == 1) v[d] = (int32_t)u < a.hotk ? ld_hint(xp, pol_last) : ld_hint_na(xp, pol_first);
-            else if (HINT == 2) v[d] = (int32_t)u < a.hotk ? __ldg(xp) : ld_hint_na(xp, pol_first);
-            else if (HINT == 3) v[d] = (int32_t)u < a.hotk ? ld_hint(xp, pol_last) : __ldg(xp);
-            else v[d] = (int32_t)u < a.hotk ? ld_hint(xp, pol_last) : ld_hint(xp, pol_first);
+            v[d] = __ldg(xl + (size_t)u * ld4);
           }
         }
         const uint32_t mseg = (bm >> (j0 & 31)) & (D >= 32 ? 0xffffffffu : ((1u << D) - 1u));
@@ -774,15 +747,7 @@ ItemsFn pick_items(int g, int vpl) {
 }
 
 using StreamFn = void (*)(const Agg2Args, uint32_t*);
-StreamFn pick_stream(int d, int minb, bool scol, int hint) {
-  if (hint > 0 && !scol && d == 4 && minb == 6) {
-    switch (hint) {
-      case 1: return k_agg_stream<4, 6, false, false, 1>;
-      case 2: return k_agg_stream<4, 6, false, false, 2>;
-      case 3: return k_agg_stream<4, 6, false, false, 3>;
-      default: return k_agg_stream<4, 6, false, false, 4>;
-    }
-  }
+StreamFn pick_stream(int d, int minb, bool scol) {
 #define STG_STREAM(DD, MB) \
   if (d == DD && minb == MB) return scol ? k_agg_stream<DD, MB, true, false> : k_agg_stream<DD, MB, false, false>;
   STG_STREAM(4, 6) STG_STREAM(8, 4) STG_STREAM(16, 2) STG_STREAM(16, 3)
@@ -849,8 +814,6 @@ struct AggTune {
   int d = 4;
   int minb = 6;
   int wmin = 32;     // stream kernel for wmin < W_launch <= 128
-  int hint = 0;      // source-row cache hints (0 = off; see Agg2Args::hotk)
-  int32_t hotk = 0;
 };
 static AggTune g_tune;
 
@@ -982,7 +945,7 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     const int64_t pstride = chunks_bound * wsplit;               // the column chunks run concurrently
     STG_TRY(ws->partials.alloc((size_t)(pstride * nsplit) + 4, s));
     const bool per_edge = scol != nullptr || ew != nullptr;
-    const StreamFn fn = peers ? pick_stream_peer(per_edge) : pick_stream(g_tune.d, g_tune.minb, per_edge, g_tune.hint);
+    const StreamFn fn = peers ? pick_stream_peer(per_edge) : pick_stream(g_tune.d, g_tune.minb, per_edge);
     // group sizes: ~max(256, E / (8 warps x #SM)) edges per group (all 32-item light
     // groups at C5 scale; small graphs get small groups, hence many warps)
     const int64_t target = std::max<int64_t>(256, gv->num_edges / (8 * (int64_t)num_sms()));
@@ -1003,7 +966,6 @@ stg_status aggregate_launch(const stg_csr_view* gv, int backward, int32_t W, con
     b.wsplit = wsplit; b.wtotal = W; b.pstride = pstride;
     b.ew = ew;
     b.eid = (ew && backward) ? gv->out_eid : nullptr;
-    b.hotk = g_tune.hotk;
     for (int k = 0; k < STG_MAX_PEERS; ++k) {
       b.pbnd[k] = INT32_MAX;
       b.pbase[k] = nullptr;
@@ -1135,14 +1097,7 @@ stg_status stg_aggregate_set_param(int32_t key, int64_t value) {
       if (value != 32 && value != 64) break;
       stg::g_tune.wmin = (int)value;
       return STG_OK;
-    case 3:
-      if (value < 0 || value > 4) break;
-      stg::g_tune.hint = (int)value;
-      return STG_OK;
-    case 4:
-      if (value < 0 || value > INT32_MAX) break;
-      stg::g_tune.hotk = (int32_t)value;
-      return STG_OK;
+
     default:
       break;
   }

@@ -1,4 +1,7 @@
 // common.cu — error strings, allocator hook, launch counter.
+#include <mutex>
+#include <unordered_map>
+
 #include "common.cuh"
 
 #include <mutex>
@@ -43,8 +46,31 @@ stg_status check_launch(const char* what) {
   return STG_OK;
 }
 
+// Blocks from the allocator hook remember the free function they came from, so
+// a block outlives a later stg_set_allocator call safely.
+struct HookBlock {
+  stg_free_fn free_fn;
+  void* ctx;
+};
+static std::mutex g_hook_mu;
+static std::unordered_map<void*, HookBlock> g_hook_blocks;
+
 void* dmalloc(size_t bytes, cudaStream_t s) {
-  if (g_alloc) return g_alloc(bytes, (stg_stream_t)s, g_ctx);
+  stg_alloc_fn a;
+  stg_free_fn f;
+  void* ctx;
+  {
+    std::lock_guard<std::mutex> lk(g_hook_mu);
+    a = g_alloc; f = g_free; ctx = g_ctx;
+  }
+  if (a) {
+    void* p = a(bytes, (stg_stream_t)s, ctx);
+    if (p) {
+      std::lock_guard<std::mutex> lk(g_hook_mu);
+      g_hook_blocks[p] = HookBlock{f, ctx};
+    }
+    return p;
+  }
   void* p = nullptr;
   if (cudaMalloc(&p, bytes) != cudaSuccess) {
     cudaGetLastError();
@@ -55,7 +81,22 @@ void* dmalloc(size_t bytes, cudaStream_t s) {
 
 void dfree(void* p, cudaStream_t s) {
   if (!p) return;
-  if (g_free) { g_free(p, (stg_stream_t)s, g_ctx); return; }
+  HookBlock hb{nullptr, nullptr};
+  {
+    std::lock_guard<std::mutex> lk(g_hook_mu);
+    auto it = g_hook_blocks.find(p);
+    if (it != g_hook_blocks.end()) {
+      hb = it->second;
+      g_hook_blocks.erase(it);
+    }
+  }
+  if (hb.free_fn) {
+    // cudaFree's ordering: no kernel of any stream may still use the block when
+    // it returns to the caller's pool
+    cudaDeviceSynchronize();
+    hb.free_fn(p, (stg_stream_t)s, hb.ctx);
+    return;
+  }
   cudaFree(p);
 }
 
@@ -219,6 +260,7 @@ int64_t stg_kernel_launch_count(void) { return stg::g_launches.load(); }
 stg_status stg_set_allocator(stg_alloc_fn alloc, stg_free_fn free_fn, void* ctx) {
   if ((alloc == nullptr) != (free_fn == nullptr))
     return stg::fail(STG_ERR_INVALID_ARG, "stg_set_allocator: alloc and free must both be set or both NULL");
+  std::lock_guard<std::mutex> lk(stg::g_hook_mu);
   stg::g_alloc = alloc;
   stg::g_free = free_fn;
   stg::g_ctx = ctx;

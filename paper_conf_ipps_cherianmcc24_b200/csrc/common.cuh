@@ -101,10 +101,25 @@ stg_status make_tmap_f32_store(CUtensorMap* out, float* base, uint64_t rows, uin
 stg_status make_tmap_f32_store3(CUtensorMap* out, float* base, uint64_t planes, uint64_t rows, uint64_t cols,
                                 uint32_t box_cols, uint32_t box_rows);
 
+// The timing surrogate head fused into the GRU kernels (per-step Algorithm-1
+// driver): forward y_t, w_o, b_o, 1/V_total; per-CTA partials of Σ e² (lpart),
+// Σ g·ReLU(H') and Σ g (gpart [nb][H+1]); per row hg = {g, bits(H' > 0)} for
+// the backward, which adds dℓ/dH' = g·w_o ⊙ [H' > 0] to its upstream gradient.
+struct HeadArgs {
+  const float* y;
+  const float* w_o;
+  const float* b_o;
+  float inv_v;
+  double* lpart;
+  float* gpart;
+  float2* hg;
+};
+
 // ---------------------------------------------------------------- profiler
 // Per-phase device time with CUDA events on the launching stream (bench.py and
 // the Fig. 9 breakdown).  Off by default; zero cost when off.
-enum Phase { PH_AGG_FWD = 0, PH_AGG_BWD, PH_SNAPSHOT, PH_XW, PH_GRU_FWD, PH_GRU_BWD, PH_DW, PH_HEAD, PH_DL, PH_COUNT };
+enum Phase { PH_AGG_FWD = 0, PH_AGG_BWD, PH_SNAPSHOT, PH_XW, PH_GRU_FWD, PH_GRU_BWD, PH_DW, PH_HEAD, PH_DL,
+             PH_SNAP_STEP, PH_SNAP_XPOSE, PH_COUNT };   // (the last two are sub-phases of PH_SNAPSHOT)
 bool prof_on();
 cudaEvent_t prof_event();
 void prof_push(int phase, cudaEvent_t a, cudaEvent_t b);

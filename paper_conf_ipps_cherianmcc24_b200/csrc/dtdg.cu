@@ -149,6 +149,7 @@ struct stg_dtdg {
     return step_snap(slot[from], slot[to], dirn, parts, s);
   }
   stg_status step_snap(const Snapshot& sf, Snapshot& st, int dirn, uint32_t parts, cudaStream_t s) {
+    ProfScope prof(PH_SNAP_STEP, s);
     const int32_t t0 = sf.t;
     const int32_t t1 = t0 + dirn;
     const int32_t td = dirn > 0 ? t1 : t0;       // batch applied (forward) or undone (reverse)
@@ -160,8 +161,8 @@ struct stg_dtdg {
     const size_t vb = sizeof(int32_t) * (size_t)V;
     STG_CUDA(cudaMemcpyAsync(st.gin_deg.p, sf.gin_deg.p, vb, cudaMemcpyDeviceToDevice, s));
     STG_CUDA(cudaMemcpyAsync(st.gout_deg.p, sf.gout_deg.p, vb, cudaMemcpyDeviceToDevice, s));
-    degree_hist(ga + gao[td], gao[td + 1] - gao[td], nb, rev ? -1 : 1, st.gin_deg.p, st.gout_deg.p, s);
-    degree_hist(gd + gdo[td], gdo[td + 1] - gdo[td], nb, rev ? 1 : -1, st.gin_deg.p, st.gout_deg.p, s);
+    STG_TRY(degree_hist2(DirDelta{ga + gao[td], gao[td + 1] - gao[td], gd + gdo[td], gdo[td + 1] - gdo[td]}, nb,
+                         rev ? -1 : 1, st.gin_deg.p, st.gout_deg.p, s));
     return apply_delta(sf, st, dir(td, true, rev), dir(td, false, rev), E[t1], t1, touch_in.p,
                        touch_out.p, *ws, s, parts & (PART_IN | PART_OUT));
   }

@@ -28,8 +28,8 @@ stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_
   dgl_both = dgl;
   const int64_t sc = sched_size(V, cap);
   STG_TRY(in_rowptr.alloc(V + 1)); STG_TRY(out_rowptr.alloc(V + 1));
-  STG_TRY(in_col.alloc(cap)); STG_TRY(in_row.alloc(cap));
-  STG_TRY(out_col.alloc(cap)); STG_TRY(out_row.alloc(cap));
+  STG_TRY(in_col.alloc(cap));
+  STG_TRY(out_col.alloc(cap));
   if (eids) STG_TRY(out_eid.alloc(cap));
   STG_TRY(in_deg.alloc(V)); STG_TRY(out_deg.alloc(V));
   STG_TRY(in_ids.alloc(V)); STG_TRY(out_ids.alloc(V));
@@ -41,7 +41,7 @@ stg_status Snapshot::alloc(int32_t V_, int64_t cap_, bool eids, bool dgl, int32_
 }
 
 size_t Snapshot::bytes() const {
-  const DArray<int32_t>* ia[] = {&in_rowptr, &in_col, &in_row, &in_deg, &in_ids, &out_rowptr, &out_col, &out_row,
+  const DArray<int32_t>* ia[] = {&in_rowptr, &in_col, &in_deg, &in_ids, &out_rowptr, &out_col,
                                  &out_deg, &out_ids, &out_eid, &in_sched, &out_sched, &gin_deg, &gout_deg};
   size_t b = 0;
   for (const auto* a : ia) b += a->n * sizeof(int32_t);
@@ -58,9 +58,7 @@ void Snapshot::view(stg_csr_view* v, AggWs* ws) const {
   // Parts this snapshot does not hold are NULL.
   const bool hi = (parts & PART_IN) != 0, ho = (parts & PART_OUT) != 0;
   v->in_rowptr = hi ? in_rowptr.p + rb : nullptr; v->in_col = hi ? in_col.p : nullptr;
-  v->in_row = hi ? in_row.p : nullptr;
   v->out_rowptr = ho ? out_rowptr.p : nullptr; v->out_col = ho ? out_col.p : nullptr;
-  v->out_row = ho ? out_row.p : nullptr;
   v->out_eid = (edge_ids && (parts & PART_EID)) ? out_eid.p : nullptr;
   // degrees: whole-graph (always current) unless sharded, where they describe the held edges
   v->in_deg = sharded ? (hi ? in_deg.p : nullptr) : gin_deg.p;
@@ -104,6 +102,26 @@ __global__ void k_deg(const int32_t* __restrict__ rowptr, int32_t V, int32_t* __
     deg[v] = rowptr[v + 1] - rowptr[v];
 }
 
+// COO row ids of a CSR: rows[j] = r for rowptr[r] <= j < rowptr[r+1]: a thread per
+// row, rows of more than 32 edges written by the whole warp
+__global__ void k_expand_rows(const int32_t* __restrict__ rowptr, int32_t V, int32_t* __restrict__ rows) {
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x + threadIdx.x - lane; base < V; base += stride) {
+    const int64_t r = base + lane;
+    int32_t b = 0, e = 0;
+    if (r < V) { b = rowptr[r]; e = rowptr[r + 1]; }
+    const bool big = e - b > 32;
+    if (!big)
+      for (int32_t j = b; j < e; ++j) rows[j] = (int32_t)r;
+    for (unsigned m = __ballot_sync(0xffffffffu, big); m; m &= m - 1) {
+      const int src = __ffs(m) - 1;
+      const int32_t bb = __shfl_sync(0xffffffffu, b, src), ee = __shfl_sync(0xffffffffu, e, src);
+      for (int32_t j = bb + lane; j < ee; j += 32) rows[j] = (int32_t)(base + src);
+    }
+  }
+}
+
 // GCN normalisation vectors (reading C1): IEEE 1/sqrtf, 0 for degree 0.
 // A sharded snapshot passes the whole-graph degrees (gin_deg / gout_deg).
 __global__ void k_norm(const int32_t* __restrict__ in_deg, const int32_t* __restrict__ out_deg, int32_t V,
@@ -120,122 +138,6 @@ __global__ void k_norm(const int32_t* __restrict__ in_deg, const int32_t* __rest
     }
   }
 }
-
-// node_ids sort keys: ascending (mask - deg) == descending degree; the stable
-// sort keeps ascending ids among equal degrees (reading C4).  Rows
-// outside [rb, re) (sharded in-direction) get key mask + 1: they sort last.
-__global__ void k_deg_keys(const int32_t* __restrict__ deg, int32_t V, uint32_t mask, int32_t rb, int32_t re,
-                           uint32_t* __restrict__ keys, int32_t* __restrict__ vals) {
-  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
-    keys[v] = (v >= rb && v < re) ? mask - (uint32_t)deg[v] : mask + 1;
-    vals[v] = v;
-  }
-}
-
-// Two-pass node_ids: the 16-bit key kSat - min(deg, kSat) (65535 for rows outside a
-// sharded block) sorts every vertex by
-// degree desc / id asc except that degrees >= kSat tie; those (at most
-// E / kSat, a short prefix of ids) are re-ranked by k_fix_saturated.
-constexpr int32_t kSat = 65534;
-constexpr int kSatMax = 4096;       // prefix the single-CTA fix handles (E < kSat * kSatMax)
-__global__ void k_deg_keys16(const int32_t* __restrict__ deg, int32_t V, int32_t rb, int32_t re,
-                             uint32_t* __restrict__ keys, int32_t* __restrict__ vals) {
-  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
-    // rows outside [rb, re) (sharded in-direction) sort after every local row
-    keys[v] = (v >= rb && v < re) ? (uint32_t)(kSat - min(deg[v], kSat)) : 65535u;
-    vals[v] = v;
-  }
-}
-// ids[0, m) hold the saturated vertices (degree >= kSat, ascending id) followed
-// by others; rank the saturated ones by (degree desc, id asc) and rewrite them.
-__global__ void __launch_bounds__(1024) k_fix_saturated(int32_t* __restrict__ ids, const int32_t* __restrict__ deg,
-                                                        int32_t m) {
-  __shared__ int32_t sid[kSatMax], sdeg[kSatMax];
-  __shared__ int32_t nsat;
-  if (threadIdx.x == 0) nsat = 0;
-  __syncthreads();
-  for (int i = threadIdx.x; i < m; i += blockDim.x) {
-    const int32_t v = ids[i], d = deg[v];
-    sid[i] = v;
-    sdeg[i] = d;
-    if (d >= kSat) atomicMax(&nsat, i + 1);
-  }
-  __syncthreads();
-  const int n = nsat;
-  for (int i = threadIdx.x; i < n; i += blockDim.x) {
-    int r = 0;
-    for (int j = 0; j < n; ++j)
-      r += sdeg[j] > sdeg[i] || (sdeg[j] == sdeg[i] && sid[j] < sid[i]);
-    ids[r] = sid[i];
-  }
-}
-
-// sched[0] = number of hub rows (deg > kHubChunk) = length of that prefix of ids.
-__global__ void k_sched_count(const int32_t* __restrict__ ids, const int32_t* __restrict__ deg, int32_t V,
-                              int64_t m, int32_t* __restrict__ sched) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= m; i += (int64_t)gridDim.x * blockDim.x) {
-    int32_t dprev = i == 0 ? INT32_MAX : deg[ids[i - 1]];
-    int32_t dcur = i >= V ? 0 : deg[ids[i]];
-    if (dprev > kHubChunk && dcur <= kHubChunk) sched[0] = (int32_t)i;
-  }
-}
-
-// Work items in node_ids order (layout in graph.cuh): hub chunks, then light rows.
-__global__ void k_items(const int32_t* __restrict__ ids, const int32_t* __restrict__ rowptr, int32_t V,
-                        int64_t cap_items, int64_t coff, int32_t* __restrict__ sched) {
-  const int32_t n_hub = sched[0], n_chunks = sched[1];
-  const int32_t* cptr = sched + coff;
-  const int64_t total = (int64_t)n_chunks + V - n_hub;
-  int4* items = reinterpret_cast<int4*>(sched + kSchedHdr);
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total && i < cap_items;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    if (i < n_chunks) {
-      int32_t lo = 0, hi = n_hub;      // largest h with cptr[h] <= i
-      while (lo < hi) {
-        int32_t mid = (lo + hi + 1) >> 1;
-        if (cptr[mid] <= i) lo = mid; else hi = mid - 1;
-      }
-      const int32_t v = ids[lo], rb = rowptr[v], re = rowptr[v + 1];
-      const int32_t beg = rb + (int32_t)(i - cptr[lo]) * kHubChunk;
-      items[i] = make_int4(v, beg, min(kHubChunk, re - beg), lo);
-    } else {
-      const int32_t v = ids[n_hub + (i - n_chunks)];
-      const int32_t rb = rowptr[v];
-      const int32_t n = rowptr[v + 1] - rb;
-      items[i] = make_int4(v, rb, n, -1);
-      // tier boundaries: light items are in non-increasing n (degree order)
-      int32_t np = INT32_MAX;
-      if (i > n_chunks) {
-        const int32_t vp = ids[n_hub + (i - 1 - n_chunks)];
-        np = rowptr[vp + 1] - rowptr[vp];
-      }
-      if (np > kTierB && n <= kTierB) sched[4] = (int32_t)i;
-      if (np > kTierC && n <= kTierC) sched[5] = (int32_t)i;
-      if (i == total - 1) {                          // tiers that reach the end are empty
-        if (n > kTierB) sched[4] = (int32_t)total;
-        if (n > kTierC) sched[5] = (int32_t)total;
-      }
-    }
-  }
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    sched[2] = (int32_t)coff;
-    sched[3] = (int32_t)total;
-    if (total == n_chunks) { sched[4] = (int32_t)total; sched[5] = (int32_t)total; }
-  }
-}
-
-struct ChunkIn {
-  const int32_t* ids;
-  const int32_t* deg;
-  __device__ int64_t operator()(int64_t i) const {
-    int32_t d = deg[ids[i]];
-    return d > kHubChunk ? (d + kHubChunk - 1) / kHubChunk : 0;
-  }
-};
-struct StoreExcl32 {
-  int32_t* o;
-  __device__ void operator()(int64_t i, int64_t ex, int64_t) const { o[i] = (int32_t)ex; }
-};
 
 // shared edge labels: out_eid[j] = in-CSR position of out-edge j = (u -> v)
 __global__ void k_out_eid(const int32_t* __restrict__ out_row, const int32_t* __restrict__ out_col, int64_t E,
@@ -312,61 +214,23 @@ stg_status sort_unique_keys(uint64_t** keys, uint64_t** alt, int64_t n, int nbit
 }
 
 stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s, uint32_t parts) {
-  const int32_t V = g.V;
-  STG_TRY(ws.dkey.alloc(V)); STG_TRY(ws.dkey_alt.alloc(V));
-  STG_TRY(ws.dval_alt.alloc(V));
-  // degrees are bounded by V (edge sets have no multi-edges)
-  const int dbits = bits_for(V);
-  const uint32_t mask = (uint32_t)((uint64_t(1) << dbits) - 1);
-  const int64_t m = std::min<int64_t>(V, sched_cap(g.cap));
   for (int dir = 0; dir < 2; ++dir) {
     if (!(parts & (dir == 0 ? PART_IN : PART_OUT))) continue;
-    int32_t* deg = dir == 0 ? g.in_deg.p : g.out_deg.p;
-    int32_t* ids = dir == 0 ? g.in_ids.p : g.out_ids.p;
-    int32_t* sched = dir == 0 ? g.in_sched.p : g.out_sched.p;
     // rows of this direction's schedule: the local block (in-CSR) or all V sources
     const bool blk = dir == 0 && g.sharded;
-    const int32_t R = blk ? g.rows() : V;
-    uint32_t* k = ws.dkey.p; uint32_t* ka = ws.dkey_alt.p;
-    int32_t* vv = ids; int32_t* va = ws.dval_alt.p;
-    const int64_t msat = std::min<int64_t>(V, g.cap / kSat + 1);   // bound on saturated vertices
-    const bool two_pass = dbits > 16 && msat <= kSatMax;
-    if (two_pass) {
-      k_deg_keys16<<<grid_for(V, 256), 256, 0, s>>>(deg, V, blk ? g.rb : 0, blk ? g.re : V, k, vv);
-      count_launch();
-      STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, 16, ws.radix, s)));   // two 8-bit digits
-    } else {
-      k_deg_keys<<<grid_for(V, 256), 256, 0, s>>>(deg, V, mask, blk ? g.rb : 0, blk ? g.re : V, k, vv);
-      count_launch();
-      STG_TRY((radix_sort<uint32_t, int32_t>(&k, &ka, &vv, &va, V, 0, dbits + (blk ? 1 : 0), ws.radix, s)));
-    }
-    if (vv != ids) {
-      STG_CUDA(cudaMemcpyAsync(ids, vv, sizeof(int32_t) * V, cudaMemcpyDeviceToDevice, s));
-    }
-    if (two_pass) {
-      k_fix_saturated<<<1, 1024, 0, s>>>(ids, deg, (int32_t)msat);
-      count_launch();
-    }
-    const int32_t* rowptr = dir == 0 ? g.in_rowptr.p : g.out_rowptr.p;
-    const int64_t coff = sched_cptr_off(V, g.cap);
-    const int64_t mr = std::min<int64_t>(m, R);
-    k_sched_count<<<grid_for(mr + 1, 256), 256, 0, s>>>(ids, deg, R, mr, sched);
-    count_launch();
-    // chunk_ptr (exclusive) in cptr[0..m], total chunks in cptr[m] and sched[1]
-    STG_TRY(scan(ChunkIn{ids, deg}, StoreExcl32{sched + coff}, mr, ws.scan, s, nullptr, sched + coff + mr));
-    STG_CUDA(cudaMemcpyAsync(sched + 1, sched + coff + mr, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
-    const int64_t icap = sched_items_cap(V, g.cap);
-    k_items<<<grid_for(icap, 256), 256, 0, s>>>(ids, rowptr, R, icap, coff, sched);
-    count_launch();
+    STG_TRY(ids_sched_build(dir == 0 ? g.in_deg.p : g.out_deg.p, dir == 0 ? g.in_rowptr.p : g.out_rowptr.p, g.V,
+                            blk ? g.rows() : g.V, blk ? g.rb : 0, blk ? g.re : g.V, dir == 0 ? g.in_ids.p : g.out_ids.p,
+                            dir == 0 ? g.in_sched.p : g.out_sched.p, g.cap, ws, s));
   }
   return check_launch("build_ids_and_sched");
 }
 
-stg_status build_out_eid(Snapshot& g, cudaStream_t s) {
-  if (!g.edge_ids) return STG_OK;
-  k_out_eid<<<grid_for(g.E, 256), 256, 0, s>>>(g.out_row.p, g.out_col.p, g.E, g.in_rowptr.p, g.in_col.p,
-                                              g.out_eid.p);
-  count_launch();
+stg_status build_out_eid(Snapshot& g, BuildWs& ws, cudaStream_t s) {
+  if (!g.edge_ids || g.E <= 0) return STG_OK;
+  STG_TRY(ws.rows.alloc((size_t)g.E, s));
+  k_expand_rows<<<grid_for(g.V, 256), 256, 0, s>>>(g.out_rowptr.p, g.V, ws.rows.p);
+  k_out_eid<<<grid_for(g.E, 256), 256, 0, s>>>(ws.rows.p, g.out_col.p, g.E, g.in_rowptr.p, g.in_col.p, g.out_eid.p);
+  count_launch(2);
   return check_launch("out_eid");
 }
 
@@ -374,8 +238,9 @@ stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& g, Bui
   const int32_t V = g.V;
   g.E = E;
   // backward CSR (rows = src): keys are already (src, dst)-sorted
-  k_unpack<<<grid_for(E, 256), 256, 0, s>>>(keys, E, g.nb, g.out_row.p, g.out_col.p);
-  k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.out_row.p, E, V, g.out_rowptr.p);
+  STG_TRY(ws.rows.alloc((size_t)(E > 0 ? E : 1), s));
+  k_unpack<<<grid_for(E, 256), 256, 0, s>>>(keys, E, g.nb, ws.rows.p, g.out_col.p);
+  k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(ws.rows.p, E, V, g.out_rowptr.p);
   count_launch(2);
   // forward CSR (rows = dst): re-key as (dst, src) and sort (the transpose)
   STG_TRY(ws.kalt.alloc(2 * (size_t)(E > 0 ? E : 1)));
@@ -385,8 +250,8 @@ stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& g, Bui
   count_launch();
   uint32_t* nov = nullptr;
   STG_TRY((radix_sort<uint64_t, uint32_t>(&a, &b, nullptr, &nov, E, 0, 2 * g.nb, ws.radix, s)));
-  k_unpack<<<grid_for(E, 256), 256, 0, s>>>(a, E, g.nb, g.in_row.p, g.in_col.p);
-  k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.in_row.p, E, V, g.in_rowptr.p);
+  k_unpack<<<grid_for(E, 256), 256, 0, s>>>(a, E, g.nb, ws.rows.p, g.in_col.p);
+  k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(ws.rows.p, E, V, g.in_rowptr.p);
   k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.in_rowptr.p, V, g.in_deg.p);
   k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.out_rowptr.p, V, g.out_deg.p);
   count_launch(4);
@@ -398,7 +263,7 @@ stg_status build_from_out_keys(const uint64_t* keys, int64_t E, Snapshot& g, Bui
   STG_TRY(check_launch("build_from_out_keys"));
   STG_TRY(build_ids_and_sched(g, ws, s));
   g.parts = PART_IN | PART_OUT | (g.edge_ids ? PART_EID : 0u);
-  return build_out_eid(g, s);
+  return build_out_eid(g, ws, s);
 }
 
 void build_norms(Snapshot& g, cudaStream_t s) {
@@ -433,6 +298,7 @@ stg_status complete_parts(Snapshot& g, uint32_t want, BuildWs& ws, cudaStream_t 
   const bool need_eid = g.edge_ids && (want & PART_EID) && !(g.parts & PART_EID);
   if (!need_in && !need_out && !need_eid) return STG_OK;
   if (!(g.parts & (PART_IN | PART_OUT))) return fail(STG_ERR_STATE, "snapshot holds no CSR to transpose");
+  ProfScope prof(PH_SNAP_XPOSE, s);
   const int64_t E = g.E, En = E > 0 ? E : 1;
   const int32_t V = g.V;
   STG_TRY(ws.kalt.alloc(2 * (size_t)En));
@@ -442,6 +308,11 @@ stg_status complete_parts(Snapshot& g, uint32_t want, BuildWs& ws, cudaStream_t 
   int32_t* v2 = v1 + En;
   const bool from_in = (g.parts & PART_IN) != 0;   // transpose in -> out (else out -> in)
   const int32_t* key_src = from_in ? g.in_col.p : g.out_col.p;
+  // the source direction's COO rows (the other endpoint of every edge)
+  STG_TRY(ws.rows.alloc((size_t)En, s));
+  int32_t* rows = ws.rows.p;
+  k_expand_rows<<<grid_for(V, 256), 256, 0, s>>>(from_in ? g.in_rowptr.p : g.out_rowptr.p, V, rows);
+  count_launch();
   if (E > 0) {
     STG_CUDA(cudaMemcpyAsync(k1, key_src, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
     k_iota<<<grid_for(E, 256), 256, 0, s>>>(v1, E);
@@ -451,27 +322,25 @@ stg_status complete_parts(Snapshot& g, uint32_t want, BuildWs& ws, cudaStream_t 
     k1 = kk; v1 = vv;
   }
   if (from_in) {
-    // out_row = sorted src, out_col = in_row[pos], out_eid = pos
+    // out rows = sorted src (k1), out_col = in row of pos, out_eid = pos
     if (E > 0) {
-      STG_CUDA(cudaMemcpyAsync(g.out_row.p, k1, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
-      k_gather_i32<<<grid_for(E, 256), 256, 0, s>>>(g.in_row.p, v1, E, g.out_col.p);
+      k_gather_i32<<<grid_for(E, 256), 256, 0, s>>>(rows, v1, E, g.out_col.p);
       count_launch();
       if (g.edge_ids) STG_CUDA(cudaMemcpyAsync(g.out_eid.p, v1, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
     }
-    k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.out_row.p, E, V, g.out_rowptr.p);
+    k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(reinterpret_cast<const int32_t*>(k1), E, V, g.out_rowptr.p);
     k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.out_rowptr.p, V, g.out_deg.p);
     count_launch(2);
     STG_TRY(build_ids_and_sched(g, ws, s, PART_OUT));
     g.parts |= PART_OUT | (g.edge_ids ? PART_EID : 0u);
   } else {
-    // in_row = sorted dst, in_col = out_row[pos]; out_eid[pos] = in position
+    // in rows = sorted dst (k1), in_col = out row of pos; out_eid[pos] = in position
     if (E > 0) {
-      STG_CUDA(cudaMemcpyAsync(g.in_row.p, k1, sizeof(int32_t) * E, cudaMemcpyDeviceToDevice, s));
-      k_gather_i32<<<grid_for(E, 256), 256, 0, s>>>(g.out_row.p, v1, E, g.in_col.p);
+      k_gather_i32<<<grid_for(E, 256), 256, 0, s>>>(rows, v1, E, g.in_col.p);
       count_launch();
       if (g.edge_ids) { k_scatter_pos<<<grid_for(E, 256), 256, 0, s>>>(v1, E, g.out_eid.p); count_launch(); }
     }
-    k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(g.in_row.p, E, V, g.in_rowptr.p);
+    k_rowptr<<<grid_for(E + 1, 256), 256, 0, s>>>(reinterpret_cast<const int32_t*>(k1), E, V, g.in_rowptr.p);
     k_deg<<<grid_for(V, 256), 256, 0, s>>>(g.in_rowptr.p, V, g.in_deg.p);
     count_launch(2);
     STG_TRY(build_ids_and_sched(g, ws, s, PART_IN));
@@ -481,184 +350,16 @@ stg_status complete_parts(Snapshot& g, uint32_t want, BuildWs& ws, cudaStream_t 
 }
 
 // -------------------------------------------------------------- delta apply
-// touch[row] = {add_lo, add_hi, del_lo, del_hi} into the sorted delta lists.
-__global__ void k_touch_mark(const uint64_t* __restrict__ d, int64_t n, int nb, int comp, int4* __restrict__ touch) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    int32_t r = (int32_t)(d[i] >> nb);
-    bool first = i == 0 || (int32_t)(d[i - 1] >> nb) != r;
-    bool last = i == n - 1 || (int32_t)(d[i + 1] >> nb) != r;
-    int* t = reinterpret_cast<int*>(touch + r);
-    if (first) t[2 * comp] = (int)i;
-    if (last) t[2 * comp + 1] = (int)(i + 1);
-  }
-}
-
-__global__ void k_touch_clear(const uint64_t* __restrict__ d, int64_t n, int nb, int4* __restrict__ touch) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    touch[(int32_t)(d[i] >> nb)] = make_int4(0, 0, 0, 0);
-}
-
-struct NewDegIn {
-  const int32_t* deg;
-  const int4* touch;
-  __device__ int64_t operator()(int64_t v) const {
-    int4 t = touch[v];
-    return deg[v] + (t.y - t.x) - (t.w - t.z);
-  }
-};
-struct RowptrOut {
-  int32_t* rowptr;
-  int32_t* deg;
-  __device__ void operator()(int64_t v, int64_t ex, int64_t d) const {
-    rowptr[v] = (int32_t)ex;
-    deg[v] = (int32_t)d;
-  }
-};
-
-__device__ __forceinline__ int64_t lb_keys(const uint64_t* a, int64_t lo, int64_t hi, uint64_t k) {
-  while (lo < hi) {
-    int64_t mid = (lo + hi) >> 1;
-    if (a[mid] < k) lo = mid + 1; else hi = mid;
-  }
-  return lo;
-}
-
-// Surviving old edges move to new_rowptr[v] + i - (#dels < c) + (#adds < c).
-// Edge labels ("relabelled" after an update) follow the move:
-// the in-direction pass records emap[old position] = new position (-1 if
-// deleted); the out-direction pass sets eid_new[new out position] =
-// emap[eid_old[old out position]] — one lookup per edge instead of a search.
-__global__ void __launch_bounds__(256) k_merge_old(const int32_t* __restrict__ orow, const int32_t* __restrict__ ocol,
-                            const int32_t* __restrict__ orowptr, int64_t E_old,
-                            const int32_t* __restrict__ nrowptr, const int4* __restrict__ touch,
-                            const uint64_t* __restrict__ adds, const uint64_t* __restrict__ dels, int nb,
-                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol, int32_t* __restrict__ emap_out,
-                            const int32_t* __restrict__ emap_in, const int32_t* __restrict__ eid_old,
-                            int32_t* __restrict__ eid_new) {
-  // 4 edges per thread per round (coalesced: edge k of the round is k*256 + tid of
-  // the block's 1024-edge tile), with all their row lookups issued before any use
-  constexpr int U = 4;
-  const int64_t tile_stride = (int64_t)gridDim.x * U * blockDim.x;
-  for (int64_t base = (int64_t)blockIdx.x * U * blockDim.x + threadIdx.x; base < E_old; base += tile_stride) {
-    int64_t j[U];
-    int32_t v[U], c[U];
-    bool ok[U];
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-      j[k] = base + (int64_t)k * blockDim.x;
-      ok[k] = j[k] < E_old;
-      v[k] = ok[k] ? __ldcs(orow + j[k]) : 0;
-      c[k] = ok[k] ? __ldcs(ocol + j[k]) : 0;
-    }
-    int4 t[U];
-    int32_t orp[U], nrp[U];
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-      t[k] = __ldg(touch + v[k]);
-      orp[k] = __ldg(orowptr + v[k]);
-      nrp[k] = __ldg(nrowptr + v[k]);
-    }
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-      if (!ok[k]) continue;
-      int64_t pos = (int64_t)nrp[k] + (j[k] - orp[k]);
-      if (t[k].y != t[k].x || t[k].w != t[k].z) {
-        const uint64_t key = ((uint64_t)v[k] << nb) | (uint64_t)c[k];
-        const int64_t dl = lb_keys(dels, t[k].z, t[k].w, key);
-        if (dl < t[k].w && dels[dl] == key) {       // deleted
-          if (emap_out) emap_out[j[k]] = -1;
-          continue;
-        }
-        const int64_t al = lb_keys(adds, t[k].x, t[k].y, key);
-        pos += (al - t[k].x) - (dl - t[k].z);
-      }
-      nrow[pos] = v[k];
-      ncol[pos] = c[k];
-      if (emap_out) emap_out[j[k]] = (int32_t)pos;
-      if (eid_new) eid_new[pos] = emap_in[eid_old[j[k]]];
-    }
-  }
-}
-
-// in-CSR position of edge (u -> v) in the (new) in-CSR: rowptr[v] + lower_bound(col row v, u)
-__device__ __forceinline__ int32_t in_position(const int32_t* __restrict__ in_rowptr, const int32_t* __restrict__ in_col,
-                                               int32_t u, int32_t v) {
-  int32_t lo = in_rowptr[v], hi = in_rowptr[v + 1];
-  while (lo < hi) {
-    int32_t mid = (lo + hi) >> 1;
-    if (in_col[mid] < u) lo = mid + 1; else hi = mid;
-  }
-  return lo;
-}
-
-// Added edge a of row v lands at new_rowptr[v] + (a - add_lo) + (#old < c) - (#dels < c).
-// Out-direction pass with labels: the label of an added out-edge (v -> c) is
-// searched in the new in-CSR (only the |A'| added edges).
-__global__ void k_merge_add(const uint64_t* __restrict__ adds, int64_t nadd, const uint64_t* __restrict__ dels,
-                            int nb, const int32_t* __restrict__ ocol, const int32_t* __restrict__ orowptr,
-                            const int32_t* __restrict__ nrowptr, const int4* __restrict__ touch,
-                            int32_t* __restrict__ nrow, int32_t* __restrict__ ncol,
-                            const int32_t* __restrict__ in_rowptr_new, const int32_t* __restrict__ in_col_new,
-                            int32_t* __restrict__ eid_new) {
-  const uint64_t mask = (uint64_t(1) << nb) - 1;
-  for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < nadd; a += (int64_t)gridDim.x * blockDim.x) {
-    uint64_t key = adds[a];
-    int32_t v = (int32_t)(key >> nb), c = (int32_t)(key & mask);
-    int4 t = touch[v];
-    int32_t lo = orowptr[v], hi = orowptr[v + 1];
-    int32_t b = lo, e = hi;
-    while (b < e) {
-      int32_t mid = (b + e) >> 1;
-      if (ocol[mid] < c) b = mid + 1; else e = mid;
-    }
-    int64_t dl = lb_keys(dels, t.z, t.w, key);
-    int64_t pos = (int64_t)nrowptr[v] + (a - t.x) + (b - lo) - (dl - t.z);
-    nrow[pos] = v;
-    ncol[pos] = c;
-    if (eid_new) eid_new[pos] = in_position(in_rowptr_new, in_col_new, v, c);
-  }
-}
-
-// Labels: `emap_out` (in-direction pass) records old -> new in-CSR positions;
-// `eid` (out-direction pass) carries {emap_in, eid_old, eid_new, new in-CSR}.
-struct EidPass {
-  const int32_t* emap_in = nullptr;
-  const int32_t* eid_old = nullptr;
-  int32_t* eid_new = nullptr;
-  const int32_t* in_rowptr_new = nullptr;
-  const int32_t* in_col_new = nullptr;
-};
-
-static stg_status apply_dir(int32_t V, int nb, const int32_t* orow, const int32_t* ocol, const int32_t* orowptr,
-                            const int32_t* odeg, int64_t E_old, int32_t* nrow, int32_t* ncol, int32_t* nrowptr,
-                            int32_t* ndeg, const DirDelta& d, int4* touch, BuildWs& ws, cudaStream_t s,
-                            int32_t* emap_out, const EidPass& eid) {
-  if (d.nadd) { k_touch_mark<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, nb, 0, touch); count_launch(); }
-  if (d.ndel) { k_touch_mark<<<grid_for(d.ndel, 256), 256, 0, s>>>(d.del, d.ndel, nb, 1, touch); count_launch(); }
-  STG_TRY(scan(NewDegIn{odeg, touch}, RowptrOut{nrowptr, ndeg}, V, ws.scan, s, nullptr, nrowptr + V));
-  if (E_old) {
-    k_merge_old<<<grid_for(ceil_div(E_old, 4), 256), 256, 0, s>>>(orow, ocol, orowptr, E_old, nrowptr, touch, d.add, d.del, nb,
-                                                    nrow, ncol, emap_out, eid.emap_in, eid.eid_old, eid.eid_new);
-    count_launch();
-  }
-  if (d.nadd) {
-    k_merge_add<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, d.del, nb, ocol, orowptr, nrowptr, touch, nrow,
-                                                     ncol, eid.in_rowptr_new, eid.in_col_new, eid.eid_new);
-    count_launch();
-  }
-  if (d.nadd) { k_touch_clear<<<grid_for(d.nadd, 256), 256, 0, s>>>(d.add, d.nadd, nb, touch); count_launch(); }
-  if (d.ndel) { k_touch_clear<<<grid_for(d.ndel, 256), 256, 0, s>>>(d.del, d.ndel, nb, touch); count_launch(); }
-  return check_launch("apply_dir");
-}
-
+// (the per-direction kernels are in snapshot.cu)
 stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
                        int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws, cudaStream_t s,
                        uint32_t parts) {
-  const int32_t V = src.V;
   const bool do_in = (parts & PART_IN) != 0, do_out = (parts & PART_OUT) != 0;
   if ((do_in && !(src.parts & PART_IN)) || (do_out && !(src.parts & PART_OUT)))
     return fail(STG_ERR_STATE, "apply_delta: source snapshot lacks a requested direction");
-  // labels are carried incrementally when both directions and the source labels are there
+  // labels are carried incrementally when both directions and the source labels are there:
+  // the in-direction pass records old -> new in-CSR positions (emap), the out-direction
+  // pass looks every surviving out-edge's label up through it
   const bool carry = dst.edge_ids && src.edge_ids && (src.parts & PART_EID) && do_in && do_out && src.E > 0;
   int32_t* emap = nullptr;
   if (carry) {
@@ -666,24 +367,17 @@ stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_di
     emap = ws.emap.p;
   }
   if (do_in)
-    STG_TRY(apply_dir(V, src.nb, src.in_row.p, src.in_col.p, src.in_rowptr.p, src.in_deg.p, src.E, dst.in_row.p,
-                      dst.in_col.p, dst.in_rowptr.p, dst.in_deg.p, in_dir, touch_in, ws, s, emap, EidPass{}));
-  EidPass ep;
-  if (carry) {
-    ep.emap_in = emap; ep.eid_old = src.out_eid.p; ep.eid_new = dst.out_eid.p;
-    ep.in_rowptr_new = dst.in_rowptr.p; ep.in_col_new = dst.in_col.p;
-  }
+    STG_TRY(apply_dir2(src, dst, true, in_dir, touch_in, ws, s, true, emap, nullptr, nullptr, nullptr, nullptr,
+                       nullptr));
   if (do_out)
-    STG_TRY(apply_dir(V, src.nb, src.out_row.p, src.out_col.p, src.out_rowptr.p, src.out_deg.p, src.E,
-                      dst.out_row.p, dst.out_col.p, dst.out_rowptr.p, dst.out_deg.p, out_dir, touch_out, ws, s,
-                      nullptr, ep));
+    STG_TRY(apply_dir2(src, dst, false, out_dir, touch_out, ws, s, !do_in, nullptr, carry ? emap : nullptr,
+                       carry ? src.out_eid.p : nullptr, carry ? dst.out_eid.p : nullptr,
+                       carry ? dst.in_rowptr.p : nullptr, carry ? dst.in_col.p : nullptr));
   dst.E = E_new;
   dst.t = t_new;
   dst.parts = (do_in ? PART_IN : 0u) | (do_out ? PART_OUT : 0u);
-  build_norms(dst, s);
-  STG_TRY(build_ids_and_sched(dst, ws, s, dst.parts));
   if (dst.edge_ids && do_in && do_out) {
-    if (!carry) STG_TRY(build_out_eid(dst, s));
+    if (!carry) STG_TRY(build_out_eid(dst, ws, s));
     dst.parts |= PART_EID;
   }
   return check_launch("apply_delta");

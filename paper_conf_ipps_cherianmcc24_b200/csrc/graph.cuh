@@ -87,8 +87,8 @@ struct Snapshot {
   int64_t E = 0, cap = 0;  // current (local) edges, edge capacity
   bool edge_ids = false, dgl_both = false, sharded = false;
   uint32_t parts = 0;      // valid parts (PART_*); degrees and norms are always valid
-  DArray<int32_t> in_rowptr, in_col, in_row, in_deg, in_ids;
-  DArray<int32_t> out_rowptr, out_col, out_row, out_deg, out_ids, out_eid;
+  DArray<int32_t> in_rowptr, in_col, in_deg, in_ids;
+  DArray<int32_t> out_rowptr, out_col, out_deg, out_ids, out_eid;
   DArray<int32_t> in_sched, out_sched;  // [sched_size(V, cap)], layout above
   DArray<int32_t> gin_deg, gout_deg;    // whole-graph degrees (the norms' source; maintained per step)
   DArray<float> norm_src, norm_dst;
@@ -126,7 +126,7 @@ stg_status sort_unique_keys(uint64_t** keys, uint64_t** alt, int64_t n, int nbit
 // Recompute degrees' dependents: node_ids and the hub schedules of the
 // directions in `parts`.  Needs the deg arrays and rowptrs of those parts.
 stg_status build_ids_and_sched(Snapshot& g, BuildWs& ws, cudaStream_t s, uint32_t parts = PART_IN | PART_OUT);
-stg_status build_out_eid(Snapshot& g, cudaStream_t s);
+stg_status build_out_eid(Snapshot& g, BuildWs& ws, cudaStream_t s);
 // GCN norms from the whole-graph degrees gin_deg / gout_deg (reading C1)
 void build_norms(Snapshot& g, cudaStream_t s);
 // Complete the missing CSR direction(s) of `g` from the one it has by a stable
@@ -142,6 +142,18 @@ struct DirDelta {
   const uint64_t* del;
   int64_t ndel;
 };
+// snapshot.cu: node_ids (degree desc, id asc) and the schedule of one CSR
+// direction by a counting sort (rows outside [rb, re) sort last; R = rows in it)
+stg_status ids_sched_build(const int32_t* deg, const int32_t* rowptr, int32_t V, int32_t R, int32_t rb, int32_t re,
+                           int32_t* ids, int32_t* sched, int64_t cap, BuildWs& ws, cudaStream_t s);
+// whole-graph degree histogram of one delta batch (adds +sign, deletes -sign)
+stg_status degree_hist2(const DirDelta& d, int nb, int sign, int32_t* gin, int32_t* gout, cudaStream_t s);
+// one delta step of one CSR direction of src into dst (rowptr, col, degrees,
+// node_ids, schedule; the GCN norms too if `norms`); labels as in apply_delta
+stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const DirDelta& d, int4* touch, BuildWs& ws,
+                      cudaStream_t s, bool norms, int32_t* emap_out, const int32_t* emap_in, const int32_t* eid_old,
+                      int32_t* eid_new, const int32_t* in_rowptr_new, const int32_t* in_col_new);
+
 // Applies the delta to the directions in `parts` (src must hold them; labels
 // are carried when both directions and src's labels are present).  The caller
 // has already updated dst's whole-graph degrees (gin_deg / gout_deg).

@@ -173,7 +173,8 @@ __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int 
                                                               const float* __restrict__ W,
                                                               const float* __restrict__ rs, float* __restrict__ P,
                                                               int rs_div,
-                                                              const __grid_constant__ CUtensorMap tmP) {
+                                                              const __grid_constant__ CUtensorMap tmP,
+                                                              const float* __restrict__ bias) {
   extern __shared__ __align__(128) unsigned char sm[];
   __shared__ uint64_t full[kXwStages], empty[kXwStages], tfull[2], tempty[2];
   __shared__ uint32_t tslot;
@@ -250,7 +251,13 @@ __global__ void __launch_bounds__(kXwThreads, 1) k_tc_xw_pipe(int V, int F, int 
           tc::fence_before();
           tc::mbar_arrive(&tempty[b]);
         }
-        tc::warp_box_store<16>(obuf, oslot, v, sc, &tmP, c0, wr0);
+        if (bias) {                                       // C = (ÂX)·W + b (aggregate-first order, NEXT-1)
+#pragma unroll
+          for (int j = 0; j < 16; ++j) v[j] = __fadd_rn(__fmul_rn(v[j], sc), __ldg(bias + c0 + j));
+          tc::warp_box_store<16>(obuf, oslot, v, 1.0f, &tmP, c0, wr0);
+        } else {
+          tc::warp_box_store<16>(obuf, oslot, v, sc, &tmP, c0, wr0);
+        }
       }
     }
     if ((threadIdx.x & 31) == 0) tc::bulk_wait_all();  // output boxes written before the CTA exits
@@ -373,13 +380,18 @@ __device__ __forceinline__ void raw_to_tmem(const unsigned char* tile, int r, in
   }
 }
 
-template <int H>
+template <int H, bool HEAD>
 __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_constant__ CUtensorMap tmC,
                                                         const __grid_constant__ CUtensorMap tmH,
                                                         const float* __restrict__ L, const float* __restrict__ l,
-                                                        const __grid_constant__ CUtensorMap tmHn) {
+                                                        const __grid_constant__ CUtensorMap tmHn,
+                                                        const HeadArgs hd) {
   using G = GruF2<H>;
   constexpr int HH = G::HH, NQ = G::NQ;
+  __shared__ float s_dot[2][128];
+  __shared__ uint32_t s_mk[2][128];
+  __shared__ float s_red[8][HH + 1];
+  __shared__ double s_l[8];
   extern __shared__ unsigned char sm_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full[2], mma_bar;
@@ -412,6 +424,15 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
   float lz[HH], lrr[HH], lh[HH];
 #pragma unroll
   for (int j = 0; j < HH; ++j) { lz[j] = l[c0 + j]; lrr[j] = l[H + c0 + j]; lh[j] = l[2 * H + c0 + j]; }
+  // fused surrogate head (HEAD): per-thread partials of Σ e², Σ g·ReLU(H'), Σ g
+  float wo[HEAD ? HH : 1], gw[HEAD ? HH : 1];
+  float bo = 0.f, gb = 0.f;
+  double lacc = 0.0;
+  if (HEAD) {
+#pragma unroll
+    for (int j = 0; j < HH; ++j) { wo[j] = hd.w_o[c0 + j]; gw[j] = 0.f; }
+    bo = hd.b_o[0];
+  }
   auto issue = [&](int tile, int b) {                   // (thread 0) TMA boxes of tile into raw buffer b
     if (tile >= ntiles) return;
     tc::mbar_expect_tx(&full[b], (uint32_t)(G::NBC + G::NBH) * kBox);
@@ -490,10 +511,67 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
         o[j] = z[j] * h[j] + (1.0f - z[j]) * hh;
       }
       tc::warp_box_store<HH>(obuf, oslot, o, 1.0f, &tmHn, c0, r0 + q * 32);    // H'
+      if (HEAD) {        // ŷ = ReLU(H')·w_o + b_o, e = ŷ − y, g = 2e / V_total (the head's dℓ/dŷ)
+        float dot = 0.f;
+        uint32_t mk = 0;
+#pragma unroll
+        for (int j = 0; j < HH; ++j) {
+          dot = fmaf(fmaxf(o[j], 0.f), wo[j], dot);
+          mk |= (o[j] > 0.f ? 1u : 0u) << j;
+        }
+        s_dot[hf][lr] = dot;
+        s_mk[hf][lr] = mk << c0;
+        __syncthreads();
+        const int row = r0 + lr;
+        if (row < V) {
+          const float e = (s_dot[0][lr] + s_dot[1][lr] + bo) - __ldg(hd.y + row);
+          const float g = 2.0f * e * hd.inv_v;
+          if (hf == 0) {
+            lacc += (double)e * (double)e;
+            gb += g;
+            hd.hg[row] = make_float2(g, __uint_as_float(s_mk[0][lr] | s_mk[1][lr]));
+          }
+#pragma unroll
+          for (int j = 0; j < HH; ++j) gw[j] = fmaf(g, fmaxf(o[j], 0.f), gw[j]);
+        }
+        __syncthreads();                               // s_dot / s_mk reused by the next tile
+      }
     }
     tc::fence_before();
   }
   if (lane == 0) tc::bulk_wait_all();                // output boxes written before the CTA exits
+  if (HEAD) {        // fixed-order CTA partials: lanes (xor tree), then the 4 row-quarter warps in order
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+#pragma unroll
+      for (int j = 0; j < HH; ++j) gw[j] += __shfl_xor_sync(0xffffffffu, gw[j], o);
+      gb += __shfl_xor_sync(0xffffffffu, gb, o);
+      lacc += __shfl_xor_sync(0xffffffffu, lacc, o);
+    }
+    if (lane == 0) {
+#pragma unroll
+      for (int j = 0; j < HH; ++j) s_red[warp][j] = gw[j];
+      s_red[warp][HH] = gb;
+      s_l[warp] = lacc;
+    }
+    __syncthreads();
+    if (threadIdx.x <= H) {
+      const int k = threadIdx.x;
+      float t = 0.f;
+      if (k < H) {
+        const int h2 = k / HH, jj = k % HH;
+        for (int qq = 0; qq < 4; ++qq) t += s_red[h2 * 4 + qq][jj];
+      } else {
+        for (int qq = 0; qq < 4; ++qq) t += s_red[qq][HH];      // hf == 0 warps carry Σ g
+      }
+      hd.gpart[(int64_t)blockIdx.x * (H + 1) + k] = t;
+    }
+    if (threadIdx.x == 0) {
+      double t = 0.0;
+      for (int qq = 0; qq < 4; ++qq) t += s_l[qq];
+      hd.lpart[blockIdx.x] = t;
+    }
+  }
   __syncthreads();
   if (warp == 0) tc::tmem_free(tm, G::TCOLS);
 }
@@ -682,7 +760,7 @@ __device__ __forceinline__ void stage_flush(float4* stage, const float (&v)[HH],
   tc::flush_stage_rows<NQ>(stage, dst, ld, row0, nvalid);
 }
 
-template <int H>
+template <int H, bool HEADG>
 __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_constant__ CUtensorMap tmC,
                                                         const __grid_constant__ CUtensorMap tmH,
                                                         const __grid_constant__ CUtensorMap tmG,
@@ -691,7 +769,8 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
                                                         const __grid_constant__ CUtensorMap tmDC,
                                                         const __grid_constant__ CUtensorMap tmDH,
                                                         const __grid_constant__ CUtensorMap tmDA,
-                                                        const __grid_constant__ CUtensorMap tmRH) {
+                                                        const __grid_constant__ CUtensorMap tmRH,
+                                                        const float2* __restrict__ hg, const float* __restrict__ w_o) {
   using G = GruB2<H>;
   constexpr int H3 = G::H3, HH = G::HH;
   extern __shared__ unsigned char sm_raw[];
@@ -758,7 +837,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
     const int r0 = tile * 128, wr0 = r0 + q * 32;
     const int row = r0 + lr;
-    const float nd = row < V ? __ldg(ndst + row) : 0.f;
+    const float nd = row < V ? (ndst ? __ldg(ndst + row) : 1.0f) : 0.f;   // (NULL: dC unscaled, aggregate-first)
     tc::mbar_wait(&full, i & 1);
     float h[HH], g[HH];
     {
@@ -772,6 +851,13 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
       for (int qq = 0; qq < HH / 4; ++qq) {
         const float4 x = tc::lds128(tc::smem_u32(box) + tc::swz128(lr, (c0 % 32) / 4 + qq));
         g[4 * qq] = x.x; g[4 * qq + 1] = x.y; g[4 * qq + 2] = x.z; g[4 * qq + 3] = x.w;
+      }
+      if (HEADG && row < V) {            // G = dH from step t+1 + the head's g·w_o ⊙ [H' > 0]
+        const float2 hv = __ldg(hg + row);
+        const uint32_t mk = __float_as_uint(hv.y) >> c0;
+#pragma unroll
+        for (int j = 0; j < HH; ++j)
+          if ((mk >> j) & 1u) g[j] = __fadd_rn(g[j], __fmul_rn(hv.x, __ldg(w_o + c0 + j)));
       }
     }
     sync_tmem();
@@ -1407,7 +1493,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_seq_bwd(int V, int S, const _
 #pragma unroll
       for (int j = 0; j < HH; ++j) dh[j] = 0.f;
     }
-    const float nd = row < V ? __ldg(ndst + row) : 0.f;
+    const float nd = row < V ? (ndst ? __ldg(ndst + row) : 1.0f) : 0.f;   // (NULL: dC unscaled, aggregate-first)
     tc::mbar_wait(&full, i & 1);
     float h[HH], g[HH];
     {
@@ -1596,7 +1682,7 @@ bool tc_supported(int F, int H) { return (H == 16 || H == 32) && F % 4 == 0 && F
 // part for tc_dw / tc_dl: tc_atb_max_blocks() · 2 · 128 · 128 floats; tot: 2 · 128 · 128
 
 stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s,
-                 int rs_div) {
+                 int rs_div, const float* bias) {
   const int N = 3 * H, Kp = (F + 7) / 8 * 8;
   const int ntiles = (V + 127) / 128;
   if (Kp <= 64) {                     // pipelined kernel (2-stage ring of 128 x Kp tiles + output stage)
@@ -1607,13 +1693,14 @@ stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const floa
     STG_TRY(make_tmap_f32_store(&tmP, P, (uint64_t)V, (uint64_t)N, (uint64_t)N, 16, 32));
     if (H == 32) {
       STG_TRY(prep(k_tc_xw_pipe<96>, smem));
-      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, rs_div, tmP);
+      k_tc_xw_pipe<96><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, rs_div, tmP, bias);
     } else {
       STG_TRY(prep(k_tc_xw_pipe<48>, smem));
-      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, rs_div, tmP);
+      k_tc_xw_pipe<48><<<nb, kXwThreads, smem, s>>>(V, F, Kp, X, W, rs, P, rs_div, tmP, bias);
     }
   } else {                            // 64 < F <= 128: one tile per CTA at a time
     if (rs_div != 1) return fail(STG_ERR_INVALID_ARG, "tc_xw: row-scale divisor needs F <= 64");
+    if (bias) return fail(STG_ERR_INVALID_ARG, "tc_xw: a bias needs F <= 64");
     const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)2 * 128 * Kp * 4;
     if (H == 32) {
       STG_TRY(prep(k_tc_xw<96>, smem));
@@ -1629,8 +1716,10 @@ stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const floa
   return check_launch("tc_xw");
 }
 
+int tc_gru_blocks(int V) { return std::max(1, std::min((V + 127) / 128, num_sms())); }
+
 stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float* L, const float* l, float* Hn,
-                      cudaStream_t s) {
+                      cudaStream_t s, const HeadArgs* head) {
   const int ntiles = (V + 127) / 128;
   const int nb = std::min(ntiles, num_sms());
   CUtensorMap tmC, tmH, tmHn;
@@ -1641,25 +1730,34 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
     const char* v = getenv("STG_GRU_FWD3");         // measured neutral on C5 (12.3 ms/epoch both)
     return v ? atoi(v) : 0;
   }();
-  if (pp && H == 32) {
+  if (head) {                                      // fused surrogate head
+    if (H == 32) {
+      STG_TRY(prep(k_tc_gru_fwd2<32, true>, GruF2<32>::SMEM));
+      k_tc_gru_fwd2<32, true><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn, *head);
+    } else {
+      STG_TRY(prep(k_tc_gru_fwd2<16, true>, GruF2<16>::SMEM));
+      k_tc_gru_fwd2<16, true><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn, *head);
+    }
+  } else if (pp && H == 32) {
     STG_TRY(prep(k_tc_gru_fwd3<32>, GruF2<32>::SMEM));
     k_tc_gru_fwd3<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
   } else if (pp) {
     STG_TRY(prep(k_tc_gru_fwd3<16>, GruF2<16>::SMEM));
     k_tc_gru_fwd3<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
   } else if (H == 32) {
-    STG_TRY(prep(k_tc_gru_fwd2<32>, GruF2<32>::SMEM));
-    k_tc_gru_fwd2<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
+    STG_TRY(prep(k_tc_gru_fwd2<32, false>, GruF2<32>::SMEM));
+    k_tc_gru_fwd2<32, false><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn, HeadArgs{});
   } else {
-    STG_TRY(prep(k_tc_gru_fwd2<16>, GruF2<16>::SMEM));
-    k_tc_gru_fwd2<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
+    STG_TRY(prep(k_tc_gru_fwd2<16, false>, GruF2<16>::SMEM));
+    k_tc_gru_fwd2<16, false><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn, HeadArgs{});
   }
   count_launch();
   return check_launch("tc_gru_fwd");
 }
 
 stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float* G, const float* L, const float* l,
-                      const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s) {
+                      const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s,
+                      const float2* hg, const float* w_o) {
   const int ntiles = (V + 127) / 128;
   const int nb = std::min(ntiles, num_sms());
   CUtensorMap tmC, tmH, tmG, tmDC, tmDH, tmDA, tmRH;
@@ -1671,13 +1769,18 @@ stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float
   STG_TRY(make_tmap_f32_store(&tmDH, dHp, (uint64_t)V, H, H, hh, 32));
   STG_TRY(make_tmap_f32_store(&tmDA, da, (uint64_t)V, 3 * H, 3 * H, hh, 32));
   STG_TRY(make_tmap_f32_store(&tmRH, RH, (uint64_t)V, H, H, hh, 32));
+#define STG_GRU_BWD(HV, HD)                                                                                  \
+  do {                                                                                                       \
+    STG_TRY(prep(k_tc_gru_bwd2<HV, HD>, GruB2<HV>::SMEM));                                                    \
+    k_tc_gru_bwd2<HV, HD><<<nb, 256, GruB2<HV>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, tmDC, tmDH, tmDA, tmRH, \
+                                                           hg, w_o);                                          \
+  } while (0)
   if (H == 32) {
-    STG_TRY(prep(k_tc_gru_bwd2<32>, GruB2<32>::SMEM));
-    k_tc_gru_bwd2<32><<<nb, 256, GruB2<32>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, tmDC, tmDH, tmDA, tmRH);
+    if (hg) STG_GRU_BWD(32, true); else STG_GRU_BWD(32, false);
   } else {
-    STG_TRY(prep(k_tc_gru_bwd2<16>, GruB2<16>::SMEM));
-    k_tc_gru_bwd2<16><<<nb, 256, GruB2<16>::SMEM, s>>>(V, tmC, tmH, tmG, L, l, ndst, tmDC, tmDH, tmDA, tmRH);
+    if (hg) STG_GRU_BWD(16, true); else STG_GRU_BWD(16, false);
   }
+#undef STG_GRU_BWD
   count_launch();
   return check_launch("tc_gru_bwd");
 }

@@ -9,6 +9,7 @@
 //                      the out-CSR (dP) → k_dw (Xᵀ·dP partials) → fixed-order
 //                      reduction.  No float atomics: deterministic run to run.
 #include <algorithm>
+#include <atomic>
 #include <map>
 #include <mutex>
 #include <vector>
@@ -20,7 +21,7 @@ bool dtdg_materialised(const stg_dtdg* g);
 bool tc_supported(int F, int H);
 int tc_atb_max_blocks();
 stg_status tc_xw(int V, int F, int H, const float* X, const float* W, const float* rs, float* P, cudaStream_t s,
-                 int rs_div = 1);
+                 int rs_div = 1, const float* bias = nullptr);
 stg_status tc_gru_seq_fwd(int V, int S, int H, const float* C_all, const float* H0, const float* L, const float* l,
                           float* H_seq, float* Hp_all, const float* Y_all, const float* w_o, const float* b_o,
                           double* lpart, int* nb_out, cudaStream_t s);
@@ -31,9 +32,11 @@ stg_status tc_gru_seq_bwd(int V, int S, int H, const float* C_all, const float* 
 stg_status tc_seq_head_reduce(int nb, int H, const double* lpart, const float* gpart, double inv_vn, float* loss,
                               float* dw_o, float* db_o, cudaStream_t s);
 stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float* L, const float* l, float* Hn,
-                      cudaStream_t s);
+                      cudaStream_t s, const HeadArgs* head = nullptr);
 stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float* G, const float* L, const float* l,
-                      const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s);
+                      const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s,
+                      const float2* hg = nullptr, const float* w_o = nullptr);
+int tc_gru_blocks(int V);
 stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* tot, float* dW,
                  cudaStream_t s);
 stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
@@ -685,6 +688,11 @@ struct TgcnWs {
   DArray<double> slpart;
   // original T-GCN (NEXT-2) scratch
   DArray<float> t2z, t2a, t2b, t2c, t2d, t2part;
+  // per-step driver with the surrogate head fused into the GRU kernels: per-row
+  // {g, ReLU mask} of every timestamp of the sequence, per-CTA head partials
+  DArray<float2> hg;
+  DArray<float> hd_gpart;
+  DArray<double> hd_lpart;
 };
 
 }  // namespace stg
@@ -696,6 +704,7 @@ struct StackEntry {
   float* C;
   int32_t V, H;
   size_t bytes;
+  float* A = nullptr;     // aggregate-first: ÂX of the step (NULL: linear-first)
 };
 
 struct stg_state_stack {
@@ -724,8 +733,27 @@ static size_t gru_bwd_smem(int H, int BR) {
   return sizeof(float) * (6 * H * H + 3 * H + BR * 3 * H + 8 * BR * H + BR * 3 * H + 6 * H * H + 6 * H);
 }
 
-static size_t stack_bytes(int32_t V, int32_t H) {
-  return (sizeof(float) * (size_t)V * 3 * H + 255) & ~size_t(255);
+// Convolution order (reading C14 / SURVEY §8(f) NEXT-1): 0 = linear-first
+// C = Â(XW) + b (the default: P' = n_src ⊙ XW is aggregated forward, dP = Âᵀ dC'
+// backward over the out-CSR); 1 = aggregate-first C = (ÂX)W + b (X is aggregated
+// at width F, dW = (ÂX)ᵀ dC, no backward aggregation).  Same model and gradients.
+std::atomic<int> g_conv_order{0};
+bool agg_first() { return g_conv_order.load(std::memory_order_relaxed) != 0; }
+
+static size_t stack_bytes(int32_t V, int32_t H, int32_t F = 0) {
+  const size_t c = (sizeof(float) * (size_t)V * 3 * H + 255) & ~size_t(255);
+  return c + (F > 0 ? (sizeof(float) * (size_t)V * F + 255) & ~size_t(255) : 0);
+}
+// the aggregate-first state: A = ÂX after C in the same stack slot
+static float* stack_A(float* C, int32_t V, int32_t H) {
+  return reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(C) +
+                                  ((sizeof(float) * (size_t)V * 3 * H + 255) & ~size_t(255)));
+}
+static stg_status check_agg_first(const stg_tgcn_params* p) {
+  if (!tc_supported(p->F, p->H) || p->F > 64)
+    return fail(STG_ERR_INVALID_ARG, "aggregate-first order needs the tensor-core path (H in {16,32}, F <= 64, "
+                "F %% 4 == 0); F=%d H=%d", p->F, p->H);
+  return STG_OK;
 }
 
 // ---- the TGCN step in stream-explicit pieces (stg_tgcn_step runs them on one
@@ -748,23 +776,33 @@ static stg_status project_rows(int32_t n_rows, const stg_tgcn_params* p, const f
   return check_launch("tgcn project");
 }
 
-// P' = diag(n_src)·X·W (all Vall rows) and C = diag(n_dst)·A·P' + b (local rows)
+// P' = diag(n_src)·X·W (all Vall rows) and C = diag(n_dst)·A·P' + b (local rows);
+// aggregate-first (A != NULL): A = ÂX (local rows, width F), C = A·W + b
 static stg_status fwd_conv(const stg_csr_view* g, const stg_tgcn_params* p, const float* X, float* P, float* C,
-                           cudaStream_t s) {
+                           cudaStream_t s, float* A = nullptr) {
   const int32_t Vall = g->num_nodes, H3 = 3 * p->H;
+  if (A) {
+    const int32_t V = g->row_end - g->row_begin, F = p->F;
+    const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
+    STG_TRY(aggregate_launch(g, 0, F, X, F, A, F, ndst_loc, g->norm_src, nullptr, s));
+    ProfScope prof(PH_XW, s);
+    if (V == 0) return STG_OK;
+    return tc_xw(V, F, p->H, A, p->W, nullptr, C, s, 1, p->b);
+  }
   STG_TRY(project_rows(Vall, p, X, g->norm_src, P, s));
   const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
   return aggregate_launch(g, 0, H3, P, H3, C, H3, ndst_loc, nullptr, p->b, s);
 }
 
-// GRU over V local rows: H_next from C and H_prev
+// GRU over V local rows: H_next from C and H_prev (tensor-core path: with the
+// surrogate head fused if `head` is given)
 static stg_status fwd_gru(int32_t V, const stg_tgcn_params* p, const float* C, const float* H_prev, float* H_next,
-                          cudaStream_t s) {
+                          cudaStream_t s, const HeadArgs* head = nullptr) {
   const int32_t H = p->H;
   ProfScope prof_gru(PH_GRU_FWD, s);
   if (V == 0) return STG_OK;
   if (tc_supported(p->F, H)) {
-    STG_TRY(tc_gru_fwd(V, H, C, H_prev, p->L, p->l, H_next, s));
+    STG_TRY(tc_gru_fwd(V, H, C, H_prev, p->L, p->l, H_next, s, head));
   } else if (H <= 32) {
     const size_t smem = gru_fwd_smem(H, 32);
     STG_TRY(set_smem(k_gru_fwd<32>, smem));
@@ -816,13 +854,14 @@ static stg_status bwd_alloc(TgcnWs& ws, const stg_csr_view* g, const stg_tgcn_pa
 // and dH_prev.  SIMT path: also the dL, dl, db partials (fused in its kernel).
 static stg_status bwd_gru(const stg_csr_view* g, const stg_tgcn_params* p, const float* C, const float* Hp,
                           const float* dH_next, float* dH_prev, stg_tgcn_grads* grads, TgcnWs& ws,
-                          const BwdBufs& bb, cudaStream_t s) {
+                          const BwdBufs& bb, cudaStream_t s, const float2* hg = nullptr, const float* w_o = nullptr) {
   const int32_t V = g->row_end - g->row_begin, H = p->H;
   const float* ndst_loc = g->norm_dst ? g->norm_dst + g->row_begin : nullptr;
   ProfScope prof(PH_GRU_BWD, s);
   if (V == 0) return STG_OK;
   if (tc_supported(p->F, H))
-    return tc_gru_bwd(V, H, C, Hp, dH_next, p->L, p->l, ndst_loc, bb.dC[0], dH_prev, bb.da[0], bb.RH[0], s);
+    return tc_gru_bwd(V, H, C, Hp, dH_next, p->L, p->l, ndst_loc, bb.dC[0], dH_prev, bb.da[0], bb.RH[0], s, hg,
+                      w_o);
   const int BR = H <= 32 ? 16 : 4;
   const size_t smem = gru_bwd_smem(H, BR);
   const int NP = 6 * H * H + 6 * H;
@@ -862,10 +901,15 @@ static stg_status bwd_dl(const stg_csr_view* g, const stg_tgcn_params* p, const 
 
 static stg_status bwd_grads(const stg_csr_view* g, const stg_tgcn_params* p, const float* X, const float* C,
                             const float* Hp, stg_tgcn_grads* grads, TgcnWs& ws, const BwdBufs& bb, cudaStream_t s,
-                            bool with_dl = true) {
+                            bool with_dl = true, const float* A = nullptr) {
   const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, F = p->F, H = p->H, H3 = 3 * H;
   const bool tc = tc_supported(F, H);
   if (with_dl) STG_TRY(bwd_dl(g, p, C, Hp, grads, ws, bb, s));
+  if (A) {                                   // aggregate-first: dW += (ÂX)ᵀ dC over the local rows
+    ProfScope prof(PH_DW, s);
+    if (V == 0) return STG_OK;
+    return tc_dw(V, F, H, A, bb.dC[0], ws.part_tc.p, ws.dl_tmp.p, grads->W, s);
+  }
   STG_TRY(aggregate_launch(g, 1, H3, bb.dC[0], H3, bb.dP[0], H3, g->norm_src, nullptr, nullptr, s));
   ProfScope prof(PH_DW, s);
   if (tc) return tc_dw(Vall, F, H, X, bb.dP[0], ws.part_tc.p, ws.dl_tmp.p, grads->W, s);
@@ -908,22 +952,25 @@ stg_status stg_tgcn_step(const stg_csr_view* g, const stg_tgcn_params* p, const 
   cudaStream_t s = (cudaStream_t)stream;
   const int32_t Vall = g->num_nodes, V = g->row_end - g->row_begin, H = p->H, H3 = 3 * H;
   TgcnWs& ws = stack ? stack->ws : global_ws();
-  STG_TRY(ws.P.alloc((size_t)Vall * H3));
+  const bool af = agg_first();
+  if (af) STG_TRY(check_agg_first(p));
+  if (!af) STG_TRY(ws.P.alloc((size_t)Vall * H3));
   float* C = nullptr;
-  const size_t need = stack_bytes(V, H);
+  const size_t need = stack_bytes(V, H, af ? p->F : 0);
   if (stack) {
     if (stack->top + need > stack->cap)
       return fail(STG_ERR_NO_MEMORY, "stg_tgcn_step: state stack full (%zu + %zu > %zu bytes)", stack->top, need,
                   stack->cap);
     C = reinterpret_cast<float*>(stack->arena.p + stack->top);
   } else {
-    STG_TRY(ws.dC.alloc((size_t)V * H3 + 4));
+    STG_TRY(ws.dC.alloc(need / sizeof(float) + 4));
     C = ws.dC.p;
   }
-  STG_TRY(fwd_conv(g, p, X, ws.P.p, C, s));
+  float* A = af ? stack_A(C, V, H) : nullptr;
+  STG_TRY(fwd_conv(g, p, X, ws.P.p, C, s, A));
   STG_TRY(fwd_gru(V, p, C, H_prev, H_next, s));
   if (stack) {
-    stack->entries.push_back(StackEntry{H_prev, C, V, H, need});
+    stack->entries.push_back(StackEntry{H_prev, C, V, H, need, A});
     stack->top += need;
   }
   return STG_OK;
@@ -944,8 +991,15 @@ stg_status stg_tgcn_step_backward(const stg_csr_view* g, const stg_tgcn_params* 
   cudaStream_t s = (cudaStream_t)stream;
   BwdBufs bb;
   STG_TRY(bwd_alloc(stack->ws, g, p, 1, &bb));
-  STG_TRY(bwd_gru(g, p, e.C, e.Hp, dH_next, dH_prev, grads, stack->ws, bb, s));
-  STG_TRY(bwd_grads(g, p, X, e.C, e.Hp, grads, stack->ws, bb, s));
+  if (e.A) {                              // aggregate-first: dC unscaled, no backward aggregation
+    stg_csr_view gv = *g;
+    gv.norm_dst = nullptr;
+    STG_TRY(bwd_gru(&gv, p, e.C, e.Hp, dH_next, dH_prev, grads, stack->ws, bb, s));
+    STG_TRY(bwd_grads(g, p, X, e.C, e.Hp, grads, stack->ws, bb, s, true, e.A));
+  } else {
+    STG_TRY(bwd_gru(g, p, e.C, e.Hp, dH_next, dH_prev, grads, stack->ws, bb, s));
+    STG_TRY(bwd_grads(g, p, X, e.C, e.Hp, grads, stack->ws, bb, s));
+  }
   stack->entries.pop_back();
   stack->top -= e.bytes;
   return STG_OK;
@@ -1366,13 +1420,11 @@ int dl_on_chain() {
   }();
   return v;
 }
-bool pipeline_enabled() {
-  static const bool on = [] {
-    const char* v = getenv("STG_SEQ_PIPELINE");
-    return !(v && v[0] == '0');
-  }();
-  return on;
-}
+std::atomic<int> g_pipeline{[] {
+  const char* v = getenv("STG_SEQ_PIPELINE");
+  return (v && v[0] == '0') ? 0 : 1;
+}()};
+bool pipeline_enabled() { return g_pipeline.load(std::memory_order_relaxed) != 0; }
 // compute on an aux stream beside the H chain (1, default) or on the caller's
 // stream with only the snapshot builds overlapped (0)
 bool aux_stream_enabled() {
@@ -1397,6 +1449,17 @@ bool aux_stream_enabled() {
 // slot), the two backward buffer sets (GRU bwd(t) waits for the reductions of
 // t+2), and the stack arena (a new sequence starts after the old one joined).
 // Same arithmetic in the same order as the single-stream stg_tgcn_step path.
+stg_status stg_set_conv_order(int32_t order) {
+  if (order != 0 && order != 1) return fail(STG_ERR_INVALID_ARG, "stg_set_conv_order: %d (0 or 1)", order);
+  g_conv_order.store(order, std::memory_order_relaxed);
+  return STG_OK;
+}
+
+stg_status stg_set_pipeline(int32_t on) {
+  g_pipeline.store(on ? 1 : 0, std::memory_order_relaxed);
+  return STG_OK;
+}
+
 stg_status stg_tgcn_train_sequence(const stg_graph* graph, stg_dtdg* dtdg, int32_t t0, int32_t S,
                                    const stg_tgcn_params* p, const float* w_o, const float* b_o,
                                    const float* const* X, const float* const* Y, const float* H0, float* H_seq,
@@ -1432,6 +1495,10 @@ stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, in
   const size_t VH = (size_t)V * H;
   cudaStream_t ms = (cudaStream_t)stream;
   const bool pipe = pipeline_enabled();
+  const bool af = agg_first();                      // aggregate-first order: no backward graph needed
+  if (af) STG_TRY(check_agg_first(p));
+  stg_csr_view view_af = view;                      // (its dims only; dC stays unscaled)
+  view_af.norm_dst = nullptr;
   // With every snapshot materialised (STG_NAIVE) there are no builds to hide: HBM-bound
   // steps (P' larger than L2) then run faster one at a time (C5: 112.6 vs 140.6 ms per
   // epoch), L2-resident ones still gain from the overlap (C4: 10.9 vs 11.9 ms;
@@ -1451,7 +1518,16 @@ stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, in
   STG_TRY(ws.P.alloc((size_t)Vall * 3 * H));
   BwdBufs bb;
   STG_TRY(bwd_alloc(ws, &view, p, 2, &bb));
-  const size_t need = stack_bytes(V, H);
+  // the surrogate head runs inside the tensor-core GRU kernels (forward: loss, dw_o,
+  // db_o and each row's {g, ReLU mask}; backward: adds g·w_o ⊙ mask to G)
+  const bool fuse_head = tc_supported(p->F, H) && V > 0;
+  const int nbh = fuse_head ? tc_gru_blocks(V) : 0;
+  if (fuse_head) {
+    STG_TRY(ws.hg.alloc((size_t)S * V));
+    STG_TRY(ws.hd_lpart.alloc((size_t)nbh));
+    STG_TRY(ws.hd_gpart.alloc((size_t)nbh * (H + 1)));
+  }
+  const size_t need = stack_bytes(V, H, af ? p->F : 0);
   if (stack->top + (size_t)S * need > stack->cap)
     return fail(STG_ERR_NO_MEMORY, "stg_tgcn_train_sequence: state stack too small (%zu + %d x %zu > %zu bytes)",
                 stack->top, S, need, stack->cap);
@@ -1480,7 +1556,8 @@ stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, in
     float* C = reinterpret_cast<float*>(stack->arena.p + stack->top);   // state-stack.push target
     if (dtdg && i > 0) STG_TRY(wait(as, ev_built[i & 1], ss));
     if (xy_ready && xy_ready[i]) STG_CUDA(cudaStreamWaitEvent(as, (cudaEvent_t)xy_ready[i], 0));   // X_t landed
-    STG_TRY(fwd_conv(&views[k], p, X[i], ws.P.p, C, as));               // P', C (H-independent)
+    float* A = af ? stack_A(C, V, H) : nullptr;
+    STG_TRY(fwd_conv(&views[k], p, X[i], ws.P.p, C, as, A));            // P', C (H-independent)
     STG_TRY(record(ev_conv[i & 1], as));
     if (dtdg && i + 1 < S) {                                            // prefetch Get-Graph(t+1)
       if (i >= 1) STG_TRY(wait(ss, ev_conv[(i + 1) & 1], as));          // conv(t-1) done with that slot
@@ -1490,26 +1567,35 @@ stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, in
     if (dtdg) graph_stack.push_back(t);                                 // graph-stack.push(t)
     STG_TRY(wait(ms, ev_conv[i & 1], as));
     const float* Hp = i == 0 ? H0 : H_seq + (size_t)(i - 1) * VH;
-    STG_TRY(fwd_gru(V, p, C, Hp, H_seq + (size_t)i * VH, ms));           // fwdprop
-    stack->entries.push_back(StackEntry{Hp, C, V, H, need});
-    stack->top += need;
     if (xy_ready && xy_ready[i] && ms != as) STG_CUDA(cudaStreamWaitEvent(ms, (cudaEvent_t)xy_ready[i], 0));
-    STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr,
-                            nullptr, stream));                          // loss += loss-fn(out)
+    if (fuse_head) {                                                    // fwdprop + loss += loss-fn(out)
+      const HeadArgs ha{Y[i], w_o, b_o, 1.0f / (float)Vall, ws.hd_lpart.p, ws.hd_gpart.p, ws.hg.p + (size_t)i * V};
+      STG_TRY(fwd_gru(V, p, C, Hp, H_seq + (size_t)i * VH, ms, &ha));
+      ProfScope prof_h(PH_HEAD, ms);
+      STG_TRY(tc_seq_head_reduce(nbh, H, ws.hd_lpart.p, ws.hd_gpart.p, 1.0 / (double)Vall, loss_accum, dw_o, db_o,
+                                 ms));
+    } else {
+      STG_TRY(fwd_gru(V, p, C, Hp, H_seq + (size_t)i * VH, ms));         // fwdprop
+      STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, loss_accum, nullptr, 0, nullptr,
+                              nullptr, stream));                        // loss += loss-fn(out)
+    }
+    stack->entries.push_back(StackEntry{Hp, C, V, H, need, A});
+    stack->top += need;
   }
   // ---- backward in LIFO order, lines 18-25
   float* G = G_work;
   float* Gn = G_work + VH;
   STG_CUDA(cudaMemsetAsync(G, 0, sizeof(float) * VH, ms));
   stg_csr_view bviews[2] = {views[0], views[1]};
-  if (dtdg) {      // the forward head; its out-CSR by a transpose (Alg. 3), needed by the reductions only
+  const bool bgraph = dtdg && !af;   // aggregate-first: the backward needs no graph (dW = (ÂX)ᵀ dC)
+  if (bgraph) {    // the forward head; its out-CSR by a transpose (Alg. 3), needed by the reductions only
     STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, graph_stack.back(), 1, STG_PART_OUT, ss, &bviews[(S - 1) & 1]));
     STG_TRY(record(ev_built[(S - 1) & 1], ss));
   }
   for (int32_t i = S - 1; i >= 0; --i) {
     const int b = i & 1;
-    if (dtdg) {
-      graph_stack.pop_back();                                           // graph-stack.pop()
+    if (dtdg) graph_stack.pop_back();                                   // graph-stack.pop()
+    if (bgraph) {
       if (i > 0) {                                                      // prefetch Get-Backward-Graph(t-1)
         if (i + 1 <= S - 1) STG_TRY(wait(ss, ev_bdone[(i + 1) & 1], as));   // step t+1 done with that slot
         STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, graph_stack.back(), 1, STG_PART_OUT, ss, &bviews[(i - 1) & 1]));
@@ -1518,20 +1604,23 @@ stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, in
       if (i < S - 1) STG_TRY(wait(ms, ev_built[i & 1], ss));
     }
     if (i + 2 <= S - 1) STG_TRY(wait(ms, ev_bdone[b], as));             // buffer set b free (step t+2)
-    const stg_csr_view& v = bviews[dtdg ? (i & 1) : 0];
-    // G = dℓ_t/dH_t + dH from step t+1
-    STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, nullptr, G, 1, dw_o, db_o, stream));
+    const stg_csr_view& v = af ? view_af : bviews[dtdg ? (i & 1) : 0];
+    // G = dℓ_t/dH_t + dH from step t+1 (fused head: the GRU backward adds dℓ_t/dH_t)
+    if (!fuse_head)
+      STG_TRY(stg_mse_head_ex(V, Vall, H, H_seq + (size_t)i * VH, Y[i], w_o, b_o, nullptr, G, 1, dw_o, db_o,
+                              stream));
     if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn_train_sequence: state stack underflow");
     const StackEntry e = stack->entries.back();                         // state-stack.pop()
     BwdBufs sb = bb;
     sb.dC[0] = bb.dC[b]; sb.dP[0] = bb.dP[b]; sb.da[0] = bb.da[b]; sb.RH[0] = bb.RH[b];
-    STG_TRY(bwd_gru(&v, p, e.C, e.Hp, G, Gn, grads, ws, sb, ms));       // bwdprop: the H chain
+    STG_TRY(bwd_gru(&v, p, e.C, e.Hp, G, Gn, grads, ws, sb, ms, fuse_head ? ws.hg.p + (size_t)i * V : nullptr,
+                    w_o));                                              // bwdprop: the H chain
     STG_TRY(record(ev_gru[b], ms));
     const bool dl_chain = pipe && dl_on_chain();
     if (dl_chain) STG_TRY(bwd_dl(&v, p, e.C, e.Hp, grads, ws, sb, ms));   // dL after the GRU, off the A stream
     STG_TRY(wait(as, ev_gru[b], ms));
-    if (dtdg) STG_TRY(wait(as, ev_built[i & 1], ss));                 // the out-CSR of t
-    STG_TRY(bwd_grads(&v, p, X[i], e.C, e.Hp, grads, ws, sb, as, !dl_chain));   // parameter gradients
+    if (bgraph) STG_TRY(wait(as, ev_built[i & 1], ss));               // the out-CSR of t
+    STG_TRY(bwd_grads(&v, p, X[i], e.C, e.Hp, grads, ws, sb, as, !dl_chain, e.A));   // parameter gradients
     STG_TRY(record(ev_bdone[b], as));
     stack->entries.pop_back();
     stack->top -= e.bytes;

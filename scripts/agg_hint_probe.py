@@ -1,4 +1,5 @@
-"""Source-row cache hints in the production edge-stream aggregation (k_agg_stream,
+"""(Needs libstg at commit 63db492, where k_agg_stream had the HINT variants; the hints
+were measured slower and removed.)  Source-row cache hints in the edge-stream aggregation (k_agg_stream,
 stg_aggregate_set_param keys 3/4) on the C5 snapshot at W = 96: the view's column
 ids are replaced by hot-first labels (the rank of the source in out-degree order
 for the forward, in in-degree order for the backward), so rows u < hotk are the

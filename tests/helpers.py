@@ -18,10 +18,6 @@ def assert_graph_equal(gpu: dict, ref: dict, edge_ids: bool = True, tag=""):
             raise AssertionError("%s %s differs at %s: gpu %s ref %s" % (tag, k, bad, a[bad], b[bad]))
     if edge_ids:
         assert np.array_equal(gpu["out_eid"].cpu().numpy(), ref["out_eid"]), (tag, "out_eid")
-    # in_row / out_row are the COO row ids implied by the rowptrs
-    V = ref["V"]
-    assert np.array_equal(gpu["in_row"].cpu().numpy(), np.repeat(np.arange(V), np.diff(ref["in_rowptr"])))
-    assert np.array_equal(gpu["out_row"].cpu().numpy(), np.repeat(np.arange(V), np.diff(ref["out_rowptr"])))
     for k in ("norm_src", "norm_dst"):
         a = gpu[k].cpu().numpy().astype(np.float64)
         np.testing.assert_allclose(a, ref[k], rtol=2.5e-7, atol=0, err_msg=k)

@@ -7,6 +7,7 @@ sizes, the method's degenerate cases), each against the oracle or a closed form:
 * size limits: E >= 2^31 and V >= 2^30 rejected with STG_ERR_OUT_OF_RANGE before
   any device work."""
 import ctypes
+import os
 
 import numpy as np
 import pytest
@@ -148,3 +149,36 @@ def test_wrong_dtype_rejected(stg):
     with pytest.raises(stg.StgError) as e:
         stg.stg_gcn_aggregate_fwd(g.view(), x)
     assert e.value.status == 1
+
+
+def test_torch_allocator_hook(stg):
+    """Library-owned buffers come from torch's caching allocator (stg_set_allocator,
+    installed by the binding): creating objects calls the hook and shows up in
+    torch's memory statistics; destroying them returns every block."""
+    import gc
+    if os.environ.get("STG_TORCH_ALLOCATOR", "1") == "0":
+        pytest.skip("allocator hook disabled by the environment")
+    torch.cuda.synchronize()
+    s0 = stg.allocator_stats()
+    m0 = torch.cuda.memory_allocated()
+    cfg = gen.CONFIGS["C4"]
+    d = gen.dtdg(cfg)
+    g = stg.stg_dtdg_create(d.V, d.T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                            d.del_dst, stg.STG_SELF_LOOPS)
+    stack = stg.stg_state_stack_create(64 << 20)
+    v = stg.stg_dtdg_get_snapshot(g, 2)
+    x = to_gpu(gen.uniform_pm1(1, 2, cfg.V * 96).reshape(cfg.V, 96))
+    y = stg.stg_gcn_aggregate_fwd(v, x)
+    torch.cuda.synchronize()
+    s1 = stg.allocator_stats()
+    assert s1["alloc"] > s0["alloc"]
+    assert torch.cuda.memory_allocated() - m0 >= (64 << 20)       # at least the state stack arena
+    ref = oracle.csr(d.V, oracle.snapshot_set_window(d, 2, self_loops=True))
+    want = oracle.aggregate_fwd(ref, x.cpu().numpy().astype(np.float64))
+    assert np.max(np.abs(y.cpu().numpy() - want) / np.maximum(oracle.aggregate_scale(ref, x.cpu().numpy()), 1e-300)) <= 1e-5
+    live = (s1["alloc"] - s0["alloc"]) - (s1["free"] - s0["free"])     # blocks held (grown buffers were freed)
+    del v, stack, g
+    gc.collect()
+    torch.cuda.synchronize()
+    s2 = stg.allocator_stats()
+    assert s2["free"] - s1["free"] >= live

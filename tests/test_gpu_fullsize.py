@@ -1,4 +1,4 @@
-"""Parity at BASELINE.json's full size (configs[4], C5: 2^20 vertices, ~9 M edges per
+r"""Parity at BASELINE.json's full size (configs[4], C5: 2^20 vertices, ~9 M edges per
 snapshot, F = 64, H = 32) in the configuration bench.py times (STG_SELF_LOOPS |
 STG_EDGE_IDS, default aggregation strategy, W = 3H = 96, the pipelined Algorithm-1
 driver):

@@ -89,7 +89,7 @@ def test_sum_parts_parallel_is_bit_identical(stg, nb, n):
     bit for bit, and both == the fp32 sum in the documented order (blocks of 16 in
     order, then the block sums in order)."""
     rng = np.random.default_rng(nb * 7919 + n)
-    part = rng.standard_normal((nb, n)).astype(np.float32) * np.float32(1e3) ** rng.integers(-1, 2, (nb, n))
+    part = (rng.standard_normal((nb, n)) * 1e3 ** rng.integers(-1, 2, (nb, n))).astype(np.float32)
     pg = to_gpu(part)
     a = stg.stg_debug_sum_parts(pg, 0).cpu().numpy()
     b = stg.stg_debug_sum_parts(pg, 1).cpu().numpy()

@@ -281,8 +281,14 @@ def test_mse_head_hand_derived_golden(stg):
     import os
     spec = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "mse_head_hand.json")))
     for c in spec["cases"]:
-        Hn = to_gpu(np.array(c["H"]))
-        V, H = Hn.shape
+        # the GPU head needs H % 4 == 0: pad with zero hidden units (ReLU(0) = 0 and w_o = 0
+        # there, so the loss and every other entry are unchanged; their gradients are 0)
+        H0 = len(c["w_o"])
+        H = (H0 + 3) // 4 * 4
+        pad = lambda a: np.pad(np.array(a, np.float64), [(0, 0)] * (np.ndim(a) - 1) + [(0, H - H0)])
+        c = dict(c, H=pad(c["H"]), w_o=pad(c["w_o"]), dH=pad(c["dH"]), dw_o=pad(c["dw_o"]))
+        Hn = to_gpu(c["H"])
+        V = Hn.shape[0]
         loss = torch.zeros(1, device="cuda")
         dH = torch.full((V, H), 7.0, device="cuda")
         dw = torch.zeros(H, device="cuda")
@@ -293,3 +299,80 @@ def test_mse_head_hand_derived_golden(stg):
         np.testing.assert_allclose(dH.cpu().numpy(), np.array(c["dH"]), rtol=1e-6, atol=0, err_msg=c["name"])
         np.testing.assert_allclose(dw.cpu().numpy(), np.array(c["dw_o"]), rtol=1e-6, atol=0, err_msg=c["name"])
         assert db.item() == pytest.approx(c["db_o"], rel=1e-6), c["name"]
+
+
+@pytest.fixture
+def agg_first(stg):
+    """Run a test under the aggregate-first convolution order (NEXT-1), restoring the default."""
+    stg.stg_set_conv_order(1)
+    yield
+    stg.stg_set_conv_order(0)
+
+
+@pytest.mark.parametrize("name,H", [("C2", 32), ("C5s", 32), ("C1", 16)])
+def test_tgcn_step_parity_aggregate_first(stg, agg_first, name, H):
+    """(ÂX)W + b (NEXT-1) is the same model as the oracle's Â(XW) + b: the step and its
+    gradients match the fp64 oracle element-wise (condition scales of DESIGN.md §7)."""
+    cfg, g, ref = _graph(stg, name)
+    V, F = cfg.V, cfg.F
+    X = gen.features(cfg, 5)
+    p, pg = _params(F, H, 11)
+    Hp = gen.uniform_pm1(3, 3, V * H).reshape(V, H)
+    Xg, Hg = to_gpu(X), to_gpu(Hp)       # (the state stack keeps H_{t-1} by reference)
+    stack = stg.stg_state_stack_create(64 << 20)
+    Hn = stg.stg_tgcn_step(g.view(), pg, Xg, Hg, stack=stack)
+    f = oracle.tgcn_fwd(ref, p, X, Hp)
+    fs = tgcn_fwd_scale(ref, p, X, Hp, np.abs(Hp), f)
+    eH = elementwise_err(Hn.cpu().numpy(), f["Hn"], fs["Hn"])
+    G = gen.uniform_pm1(4, 4, V * H).reshape(V, H)
+    grads = _zero_grads(F, H)
+    dHp = stg.stg_tgcn_step_backward(g.view(), pg, Xg, to_gpu(G), grads, stack)
+    rg = oracle.zero_grads(F, H)
+    rdH = oracle.tgcn_bwd(ref, p, X, Hp, f, G, rg)
+    sc = {}
+    s_dH = tgcn_bwd_scales(ref, p, X, Hp, np.abs(Hp), f, fs, G, np.abs(G), sc)
+    edH = elementwise_err(dHp.cpu().numpy(), rdH, s_dH)
+    parity_log(("step_aggfirst", name, H), H=eH, dH=edH)
+    assert eH <= TAU_TGCN and edH <= TAU_TGCN, (eH, edH)
+    check_sequence(("step_aggfirst", name, H), {k: grads[k].cpu().numpy() for k in ("W", "b", "L", "l")}, rg, sc,
+                   normwise=g_tol(V))
+
+
+def test_train_sequence_dtdg_aggregate_first(stg, agg_first):
+    """Algorithm 1 over DTDG sequences in aggregate-first order: no backward snapshots
+    are built, and loss, H_t and every gradient match the oracle sequence."""
+    cfg = gen.CONFIGS["C5s"]
+    d = gen.dtdg(cfg)
+    g = stg.stg_dtdg_create(d.V, d.T, d.src0, d.dst0, d.add_off, d.add_src, d.add_dst, d.del_off, d.del_src,
+                            d.del_dst, stg.STG_SELF_LOOPS)
+    snaps = [oracle.csr(d.V, S) for S in oracle.snapshot_sets_fold(d, self_loops=True)]
+    p, pg = _params(cfg.F, cfg.H, 3)
+    H0 = np.zeros((cfg.V, cfg.H))
+    Hc = to_gpu(H0)
+    S = 4
+    for t0 in (0, S):
+        Xs = [gen.features(cfg, t0 + i) for i in range(S)]
+        Ys = [gen.labels(cfg, t0 + i) for i in range(S)]
+        grads = _zero_grads(cfg.F, cfg.H)
+        dw, db, loss = torch.zeros(cfg.H, device="cuda"), torch.zeros(1, device="cuda"), torch.zeros(1, device="cuda")
+        Hseq = torch.empty(S, cfg.V, cfg.H, device="cuda")
+        stack = stg.stg_state_stack_create(S * cfg.V * (3 * cfg.H + cfg.F) * 4 + (1 << 20))
+        stg.stg_tgcn_train_sequence(g, t0, S, pg, pg["w_o"], pg["b_o"], [to_gpu(x) for x in Xs],
+                                    [to_gpu(y) for y in Ys], Hc, Hseq, torch.empty(2, cfg.V, cfg.H, device="cuda"),
+                                    grads, dw, db, loss, stack)
+        assert stack.depth == 0
+        rl, rg, rH = oracle.train_sequence(snaps[t0:t0 + S], snaps[t0:t0 + S], p, Xs, Ys, H0)
+        _check_seq(("seq_aggfirst", t0), snaps[t0:t0 + S], p, Xs, Ys, H0, loss.item(), grads, dw, db, Hseq, rl, rg,
+                   rH, cfg.V * S)
+        H0 = rH
+        Hc = Hseq[-1].clone()
+
+
+def test_aggregate_first_rejects_unsupported(stg, agg_first):
+    cfg, g, ref = _graph(stg, "C2")
+    p, pg = _params(cfg.F, 64, 1)                 # H = 64: no tensor-core path
+    with pytest.raises(stg.StgError) as e:
+        stg.stg_tgcn_step(g.view(), pg, to_gpu(gen.features(cfg, 0)), torch.zeros(cfg.V, 64, device="cuda"))
+    assert e.value.status == 1
+    with pytest.raises(stg.StgError):
+        stg.stg_set_conv_order(2)

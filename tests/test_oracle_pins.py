@@ -350,3 +350,32 @@ def test_mse_head_hand_derived_golden():
         np.testing.assert_allclose(dH, np.array(c["dH"]), rtol=1e-15, atol=1e-15, err_msg=c["name"])
         np.testing.assert_allclose(grads["w_o"], np.array(c["dw_o"]), rtol=1e-15, atol=1e-15, err_msg=c["name"])
         assert grads["b_o"][0] == pytest.approx(c["db_o"], rel=1e-15, abs=1e-15), c["name"]
+
+
+def test_openmp_timing_build_matches_plain():
+    """The OpenMP build of the same source (bench.py's all-core CPU baseline only)
+    computes the same step: row-parallel results bit-identical, thread-reduced
+    parameter gradients equal up to fp64 reassociation."""
+    cfg = gen.CONFIGS["C2"]
+    s, d = gen.static_edges(cfg)
+    g = oracle.static_graph(cfg.V, s, d, self_loops=True)
+    p = gen.tgcn_params(cfg.F, cfg.H, 5)
+    X = gen.features(cfg, 3)
+    Hp = gen.uniform_pm1(2, 2, cfg.V * cfg.H).reshape(cfg.V, cfg.H)
+    G = gen.uniform_pm1(3, 3, cfg.V * cfg.H).reshape(cfg.V, cfg.H)
+    out = []
+    try:
+        for omp in (False, True):
+            oracle.use_openmp(omp)
+            f = oracle.tgcn_fwd(g, p, X, Hp)
+            gr = oracle.zero_grads(cfg.F, cfg.H)
+            dH = oracle.tgcn_bwd(g, p, X, Hp, f, G, gr)
+            out.append((f, gr, dH))
+    finally:
+        oracle.use_openmp(False)
+    (f0, g0, d0), (f1, g1, d1) = out
+    for k in ("C", "Z", "R", "Hh", "Hn"):
+        assert np.array_equal(f0[k], f1[k]), k
+    assert np.array_equal(d0, d1)
+    for k in ("W", "b", "L", "l"):
+        np.testing.assert_allclose(g1[k], g0[k], rtol=1e-12, atol=1e-12 * np.abs(g0[k]).max(), err_msg=k)
