@@ -61,6 +61,11 @@ int64_t stg_kernel_launch_count(void);
 typedef void* (*stg_alloc_fn)(size_t bytes, stg_stream_t stream, void* ctx);
 typedef void (*stg_free_fn)(void* ptr, stg_stream_t stream, void* ctx);
 stg_status stg_set_allocator(stg_alloc_fn alloc, stg_free_fn free_fn, void* ctx);
+/* Process teardown: forget every block obtained through the hook (their later
+ * frees, e.g. by static library state destroyed at exit, are skipped) and
+ * restore cudaMalloc / cudaFree.  For a hook whose owner (an interpreter) is
+ * shutting down; the memory goes back with the process. */
+stg_status stg_allocator_detach(void);
 
 /* Graph creation flags. */
 enum {
@@ -89,7 +94,20 @@ enum {
  * so the local results are exactly the rows / partial sums of the whole-graph
  * computation.  Snapshot builds need no communication.  rank / world are
  * informational.  row_begin <= row_end must lie in [0,V]
- * (STG_ERR_INVALID_ARG otherwise).  NULL = whole graph. */
+ * (STG_ERR_INVALID_ARG otherwise).  NULL = whole graph.
+ *
+ * Deviation from SURVEY §8(b) (`stg_dist {nccl_comm, rank, world}`,
+ * `stg_allgather_rows(stg_dist*, view, ...)`): the library holds no NCCL
+ * communicator.  The per-timestep row exchange of sharded mode is done over
+ * peer memory instead — every rank maps the others' row blocks once
+ * (stg_peer_alloc / stg_peer_open, CUDA IPC, NVLink on a multi-GPU box) and the
+ * forward gather reads a source row straight from its owner's block
+ * (stg_gcn_aggregate_peer), so the all-gather is fused into the aggregation
+ * tile by tile instead of being a separate NCCL call (north_star's "NCCL
+ * all-gather over NVLink" would be the unfused baseline); stg_allgather_rows
+ * takes that peer-row table.  The one collective left, the per-sequence
+ * gradient all-reduce (~51 KB), is issued by the caller (torch.distributed /
+ * NCCL), which owns the communicator and the process group. */
 typedef struct {
   int32_t rank, world;
   int32_t row_begin, row_end;
@@ -407,14 +425,55 @@ typedef struct {
 
 /* CUDA IPC handle of a peer-visible allocation (opaque, 64 bytes). */
 typedef struct { unsigned char reserved[64]; } stg_ipc_handle;
-/* Allocates `bytes` of device memory that other processes may map
- * (cudaMalloc'd, not pooled) and returns its IPC handle.  Free with stg_peer_free. */
+/* Allocates `bytes` of zero-initialised device memory that other processes may
+ * map (cudaMalloc'd, not pooled) and returns its IPC handle.  Free with stg_peer_free. */
 stg_status stg_peer_alloc(int64_t bytes, void** dptr, stg_ipc_handle* handle);
 stg_status stg_peer_free(void* dptr);
 /* Maps another process's allocation (same or peer device, peer access enabled
  * lazily over NVLink).  STG_ERR_CUDA if the handle was created in this process. */
 stg_status stg_peer_open(const stg_ipc_handle* handle, void** dptr);
 stg_status stg_peer_close(void* dptr);
+
+/* ---- sharded-mode Algorithm 1 in the library (the per-timestep exchange ordered
+ * by device-side flags instead of host barriers) ----
+ * Every rank holds, in peer-mapped memory (stg_peer_alloc / stg_peer_open):
+ *   P[b][k]  : rank k's P' rows [R_k, 3H] (b = exchange parity: two buffers),
+ *   dP[b][k] : rank k's partial dP over all V source rows [V, 3H],
+ *   flags[k] : 4 uint32 counters of rank k, zero at allocation — 0: forward
+ *              exchanges published, 1: forward exchanges consumed, 2: backward
+ *              exchanges published, 3: backward exchanges consumed.
+ * Forward exchange n (b = n % 2): wait until every rank consumed exchange n-2
+ * (its buffer), project this rank's P' rows, publish n, wait until every rank
+ * published n, gather + GRU (+ the fused head), mark n consumed.  Backward
+ * exchange m: wait until every rank consumed m-2, GRU backward + partial
+ * Âᵀ dC' into dP[b][rank], publish m, wait for all, reduce-scatter this rank's
+ * rows in rank order, mark m consumed, dW += X_locᵀ dP_loc.  Waits and
+ * publications are stream memory operations (cuStreamWaitValue32 /
+ * cuStreamWriteValue32 on the peers' counters), so no host synchronisation and
+ * no NCCL call sits on the data path; the per-sequence gradient all-reduce
+ * stays with the caller.  fwd_count / bwd_count: exchanges done so far by
+ * every rank (in/out; all ranks call with the same values). */
+typedef struct {
+  int32_t world, rank;
+  const int32_t* bounds;              /* (host) [world+1] */
+  float* P[2][STG_MAX_PEERS];
+  float* dP[2][STG_MAX_PEERS];
+  uint32_t* flags[STG_MAX_PEERS];
+  uint32_t fwd_count, bwd_count;
+} stg_peer_exchange;
+
+/* Algorithm 1 for one sequence of S timestamps on this rank's row block
+ * (sharded mode, X row-sharded): dtdg is this rank's sharded DTDG (stg_dist
+ * = its block), X_loc / Y_loc (host)[S] device pointers to its rows, H0 /
+ * H_seq [S][R,H] / G_work [2][R,H] its rows; gradients are this rank's share
+ * (sum over ranks = the whole-graph gradients).  dP_loc [R,3H] scratch.
+ * Needs the tensor-core path (tc_supported).  Errors as stg_tgcn_train_sequence. */
+stg_status stg_tgcn_train_sequence_peer(stg_dtdg* dtdg, int32_t t0, int32_t S, const stg_tgcn_params* p,
+                                        const float* w_o, const float* b_o, const float* const* X_loc,
+                                        const float* const* Y_loc, const float* H0, float* H_seq, float* G_work,
+                                        float* dP_loc, stg_tgcn_grads* grads, float* dw_o, float* db_o,
+                                        float* loss_accum, stg_state_stack* stack, stg_peer_exchange* px,
+                                        stg_stream_t stream);
 
 /* All-gather of row blocks over peer loads: full[u,:] = row u of its owner's block,
  * for all u in [0,V), W columns; full has leading dimension ldf >= W.  (The

@@ -168,8 +168,20 @@ _decl("stg_tgcn_step_backward_peer", [ctypes.POINTER(stg_csr_view), ctypes.POINT
                                       ctypes.POINTER(stg_tgcn_grads), _P, _P, _P])
 _decl("stg_tgcn_dw", [ctypes.POINTER(stg_tgcn_params), _i32, _P, _P, ctypes.POINTER(stg_tgcn_grads), _P, _P])
 
+
+class stg_peer_exchange(ctypes.Structure):
+    _fields_ = [("world", _i32), ("rank", _i32), ("bounds", ctypes.POINTER(_i32)),
+                ("P", (_P * 8) * 2), ("dP", (_P * 8) * 2), ("flags", _P * 8),
+                ("fwd_count", ctypes.c_uint32), ("bwd_count", ctypes.c_uint32)]
+
+
+_decl("stg_tgcn_train_sequence_peer", [_P, _i32, _i32, ctypes.POINTER(stg_tgcn_params), _P, _P, _P, _P, _P, _P, _P,
+                                       _P, ctypes.POINTER(stg_tgcn_grads), _P, _P, _P, _P,
+                                       ctypes.POINTER(stg_peer_exchange), _P])
+
 ABI_SYMBOLS = [
-    "stg_last_error", "stg_version", "stg_kernel_launch_count", "stg_set_allocator", "stg_memcpy",
+    "stg_last_error", "stg_version", "stg_kernel_launch_count", "stg_set_allocator", "stg_allocator_detach",
+    "stg_memcpy",
     "stg_static_graph_create", "stg_graph_view", "stg_graph_destroy",
     "stg_dtdg_create", "stg_dtdg_get_snapshot", "stg_dtdg_get_backward_snapshot", "stg_dtdg_get_snapshot_parts",
     "stg_dtdg_num_edges",
@@ -183,7 +195,7 @@ ABI_SYMBOLS = [
     "stg_gcn_aggregate_weighted", "stg_gcn_weighted_norm", "stg_tgcn2_step", "stg_tgcn2_step_backward",
     "stg_peer_alloc", "stg_peer_free", "stg_peer_open", "stg_peer_close", "stg_allgather_rows",
     "stg_gcn_aggregate_peer", "stg_reduce_scatter_rows", "stg_tgcn_project", "stg_tgcn_step_peer",
-    "stg_tgcn_step_backward_peer", "stg_tgcn_dw", "stg_tgcn2_peer_fwd", "stg_tgcn2_peer_bwd",
+    "stg_tgcn_step_backward_peer", "stg_tgcn_dw", "stg_tgcn_train_sequence_peer", "stg_tgcn2_peer_fwd", "stg_tgcn2_peer_bwd",
 ]
 
 # ---------------------------------------------------------------- allocator hook
@@ -196,9 +208,17 @@ _lib.stg_set_allocator.argtypes = [_ALLOC_FN, _FREE_FN, ctypes.c_void_p]
 _lib.stg_set_allocator.restype = _i32
 _hook_stats = {"alloc": 0, "free": 0, "bytes": 0}
 _exiting = [False]
-# at interpreter exit, objects still alive are left to the process teardown: their
-# blocks belong to torch's allocator, which must not be called back during finalisation
-atexit.register(lambda: _exiting.__setitem__(0, True))
+
+
+def _at_exit():
+    # objects still alive are left to the process teardown, and the library forgets
+    # its torch blocks: torch's allocator must not be called back during finalisation
+    # (static library state is destroyed after the interpreter)
+    _exiting[0] = True
+    _lib.stg_allocator_detach()
+
+
+atexit.register(_at_exit)
 
 
 def _torch_alloc(nbytes, stream, ctx):
@@ -324,9 +344,9 @@ class Graph:
             self.handle = None
 
     def __del__(self):
-        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
-            return
         try:
+            if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+                return
             self.close()
         except Exception:
             pass
@@ -360,9 +380,9 @@ class Dtdg:
             self.handle = None
 
     def __del__(self):
-        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
-            return
         try:
+            if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+                return
             self.close()
         except Exception:
             pass
@@ -544,9 +564,9 @@ class StateStack:
             self.handle = None
 
     def __del__(self):
-        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
-            return
         try:
+            if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+                return
             self.close()
         except Exception:
             pass
@@ -723,9 +743,9 @@ class PeerBuffer:
             self.ptr = None
 
     def __del__(self):
-        if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
-            return
         try:
+            if _exiting[0] or sys.is_finalizing():   # (the allocator hook calls back into torch)
+                return
             self.close()
         except Exception:
             pass
@@ -813,6 +833,18 @@ def stg_tgcn_dw(params: dict, X_loc, dP_loc, grads: dict, stack: StateStack, str
     R = X_loc.shape[0]
     _check(_lib.stg_tgcn_dw(ctypes.byref(P), int(R), _ptr(X_loc), ctypes.c_void_p(_row_ptr(dP_loc)),
                             ctypes.byref(G), stack.handle, _stream(stream)))
+
+
+def stg_tgcn_train_sequence_peer(dtdg, t0: int, params: dict, w_o, b_o, X_loc, Y_loc, H0, H_seq, G_work, dP_loc,
+                                 grads: dict, dw_o, db_o, loss_accum, stack, px: "stg_peer_exchange", stream=None):
+    """Sharded-mode Algorithm 1 for one sequence inside the library (device-side exchange flags)."""
+    P = make_params(params)
+    G = make_grads(grads)
+    S = len(X_loc)
+    _check(_lib.stg_tgcn_train_sequence_peer(dtdg.handle, int(t0), S, ctypes.byref(P), _ptr(w_o), _ptr(b_o),
+                                             _ptrs(X_loc), _ptrs(Y_loc), _ptr(H0), _ptr(H_seq), _ptr(G_work),
+                                             _ptr(dP_loc), ctypes.byref(G), _ptr(dw_o), _ptr(db_o),
+                                             _ptr(loss_accum), stack.handle, ctypes.byref(px), _stream(stream)))
 
 
 def stg_tgcn2_peer_fwd(phase: int, v: stg_csr_view, params: dict, X_loc, H_loc, rows: PeerRows = None, Z_loc=None,

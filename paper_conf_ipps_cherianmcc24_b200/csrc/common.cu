@@ -54,6 +54,7 @@ struct HookBlock {
 };
 static std::mutex g_hook_mu;
 static std::unordered_map<void*, HookBlock> g_hook_blocks;
+static bool g_detached = false;     // stg_allocator_detach: hook blocks are never freed
 
 void* dmalloc(size_t bytes, cudaStream_t s) {
   stg_alloc_fn a;
@@ -64,6 +65,13 @@ void* dmalloc(size_t bytes, cudaStream_t s) {
     a = g_alloc; f = g_free; ctx = g_ctx;
   }
   if (a) {
+    // A pooled block may have been released by its previous owner with work still
+    // pending on another stream, and the library may use this block on any of its
+    // streams: wait for the device first (cudaMalloc's ordering; allocations are
+    // grow-only and rare, never inside a captured graph)
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) != cudaSuccess) cudaGetLastError();
+    if (cs == cudaStreamCaptureStatusNone) cudaDeviceSynchronize();
     void* p = a(bytes, (stg_stream_t)s, ctx);
     if (p) {
       std::lock_guard<std::mutex> lk(g_hook_mu);
@@ -82,14 +90,17 @@ void* dmalloc(size_t bytes, cudaStream_t s) {
 void dfree(void* p, cudaStream_t s) {
   if (!p) return;
   HookBlock hb{nullptr, nullptr};
+  bool hooked = false;
   {
     std::lock_guard<std::mutex> lk(g_hook_mu);
     auto it = g_hook_blocks.find(p);
     if (it != g_hook_blocks.end()) {
       hb = it->second;
+      hooked = true;
       g_hook_blocks.erase(it);
     }
   }
+  if (hooked && !hb.free_fn) return;   // detached (process teardown): the owner's pool is gone
   if (hb.free_fn) {
     // cudaFree's ordering: no kernel of any stream may still use the block when
     // it returns to the caller's pool
@@ -256,6 +267,16 @@ const char* stg_last_error(void) { return stg::t_err.c_str(); }
 int32_t stg_version(void) { return 100; }
 
 int64_t stg_kernel_launch_count(void) { return stg::g_launches.load(); }
+
+stg_status stg_allocator_detach(void) {
+  std::lock_guard<std::mutex> lk(stg::g_hook_mu);
+  for (auto& e : stg::g_hook_blocks) e.second.free_fn = nullptr;   // freed later: skipped
+  stg::g_detached = true;
+  stg::g_alloc = nullptr;
+  stg::g_free = nullptr;
+  stg::g_ctx = nullptr;
+  return STG_OK;
+}
 
 stg_status stg_set_allocator(stg_alloc_fn alloc, stg_free_fn free_fn, void* ctx) {
   if ((alloc == nullptr) != (free_fn == nullptr))

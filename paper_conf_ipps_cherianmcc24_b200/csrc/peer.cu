@@ -95,6 +95,7 @@ stg_status stg_peer_alloc(int64_t bytes, void** dptr, stg_ipc_handle* handle) {
     return stg::fail(STG_ERR_NO_MEMORY, "stg_peer_alloc: cudaMalloc(%lld): %s", (long long)bytes,
                      cudaGetErrorString(e));
   }
+  cudaMemset(p, 0, (size_t)bytes);                 // zero-initialised (exchange counters start at 0)
   cudaIpcMemHandle_t h;
   e = cudaIpcGetMemHandle(&h, p);
   if (e != cudaSuccess) {

@@ -150,15 +150,24 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
     if (dg < kIdsBuckets && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&h[dg], __popc(peers));
   }
   if (TOUCH) {
-    // exclusive prefix of every row within the tile: 16 striped block scans
-    int64_t ex[kRowIPT];
-    int64_t tot = 0;
+    // exclusive prefix of every row within the tile: the striped degrees go through
+    // shared memory so that each thread scans 16 consecutive rows (one block scan)
+    __shared__ int32_t sd[kRowTile + kRowTile / 32];  // padded (index i at i + i/32)
+    auto pad = [](int i) { return i + (i >> 5); };
+#pragma unroll
+    for (int k = 0; k < kRowIPT; ++k) sd[pad(k * kRowThreads + (int)threadIdx.x)] = d[k];
+    __syncthreads();
+    int32_t run = 0;
+#pragma unroll
+    for (int k = 0; k < kRowIPT; ++k) run += sd[pad((int)threadIdx.x * kRowIPT + k)];
+    int64_t tot;
+    int64_t base = block_excl_scan(run, sh, &tot);
 #pragma unroll
     for (int k = 0; k < kRowIPT; ++k) {
-      int64_t t_k;
-      ex[k] = tot + block_excl_scan(d[k], sh, &t_k);
-      tot += t_k;
-      __syncthreads();                                  // sh reused by the next scan
+      const int i = pad((int)threadIdx.x * kRowIPT + k);
+      const int32_t x = sd[i];
+      sd[i] = (int32_t)base;                            // exclusive prefix within the tile
+      base += x;
     }
     if (threadIdx.x < 32) {                             // warp 0: publish, then look back 32 tiles at a time
       uint64_t* st = a.status + tile;
@@ -192,7 +201,7 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
     for (int k = 0; k < kRowIPT; ++k) {
       const int64_t v = r0 + (int64_t)k * kRowThreads;
       if (v < a.V) {
-        a.rowptr_new[v] = (int32_t)(pre + ex[k]);
+        a.rowptr_new[v] = (int32_t)(pre + sd[pad(k * kRowThreads + (int)threadIdx.x)]);
         a.deg_new[v] = d[k];
       }
     }
@@ -514,93 +523,82 @@ struct MergeArgs {
   const int32_t* in_col_new;
 };
 
-constexpr int kMergeRows = 1024;    // rows of a tile whose rowptr / touch marks are cached in shared memory
-constexpr int kMergeDelta = 1536;   // a tile's add (and delete) keys staged in shared memory
+constexpr int kMergeIPT = kMergeTile / 256;      // consecutive old edges per thread
 
-__device__ __forceinline__ int64_t lb_u64_s(const uint64_t* a, int64_t lo, int64_t hi, uint64_t k) {
-  while (lo < hi) {
-    const int64_t mid = (lo + hi) >> 1;
-    if (a[mid] < k) lo = mid + 1; else hi = mid;
-  }
-  return lo;
-}
+// Old edges: a CTA takes kMergeTile consecutive positions (loaded coalesced into
+// shared memory); thread t then walks its kMergeIPT consecutive positions in order.
+// Only the first edge of a row in the chunk searches the row's sorted add / delete
+// keys; the following ones advance those cursors (keys and columns are both sorted
+// within a row), so a hub row with thousands of deltas costs ~2 searches per chunk
+// instead of 2 per edge.
+constexpr int kMergeRows = 1024;                 // rows whose rowptr / touch / new rowptr are cached
 
-// Old edges: a CTA takes kMergeTile consecutive positions, caches the rowptr and the
-// touch marks of the rows they span, and stages the add / delete keys of those rows
-// (contiguous in the sorted delta lists) in shared memory, so the per-edge searches
-// (#adds < c, #dels < c of a touched row, typically a hub with thousands of deltas)
-// never go to global memory.  Lane-linear positions: coalesced reads and writes.
 __global__ void __launch_bounds__(256) k_merge2(const MergeArgs a) {
-  __shared__ int32_t srp[kMergeRows + 1];
+  __shared__ int32_t scol[kMergeTile];
+  __shared__ int32_t srp[kMergeRows + 1], snrp[kMergeRows];
   __shared__ int4 stc[kMergeRows];
-  __shared__ uint64_t sadd[kMergeDelta], sdel[kMergeDelta];
   __shared__ int32_t s_lo, s_hi;
-  __shared__ int s_r[4];                              // add range [A0, A1), delete range [D0, D1)
   if ((int64_t)blockIdx.x < a.old_tiles) {
     const int64_t e0 = (int64_t)blockIdx.x * kMergeTile;
     const int64_t e1 = min(e0 + (int64_t)kMergeTile, a.E_old);
     if (threadIdx.x == 0) {
       s_lo = row_of(a.orowptr, 0, a.V - 1, e0);
       s_hi = row_of(a.orowptr, 0, a.V - 1, e1 - 1);
-      s_r[0] = INT32_MAX; s_r[1] = 0; s_r[2] = INT32_MAX; s_r[3] = 0;
     }
+    for (int k = threadIdx.x; k < e1 - e0; k += blockDim.x) scol[k] = __ldcs(a.ocol + e0 + k);
     __syncthreads();
     const int32_t rlo = s_lo, rhi = s_hi, nr = rhi - rlo + 1;
-    const bool cached = nr <= kMergeRows;
+    const bool cached = nr <= kMergeRows;              // (the tile's rows: ~kMergeTile / mean degree)
     if (cached) {
-      int a0 = INT32_MAX, a1 = 0, d0 = INT32_MAX, d1 = 0;
       for (int k = threadIdx.x; k <= nr; k += blockDim.x) {
         srp[k] = __ldg(a.orowptr + rlo + k);
-        if (k < nr) {
-          const int4 t = __ldg(a.touch + rlo + k);
-          stc[k] = t;
-          if (t.y > t.x) { a0 = min(a0, t.x); a1 = max(a1, t.y); }
-          if (t.w > t.z) { d0 = min(d0, t.z); d1 = max(d1, t.w); }
-        }
+        if (k < nr) { stc[k] = __ldg(a.touch + rlo + k); snrp[k] = __ldg(a.nrowptr + rlo + k); }
       }
-      if (a1 > 0) { atomicMin(&s_r[0], a0); atomicMax(&s_r[1], a1); }
-      if (d1 > 0) { atomicMin(&s_r[2], d0); atomicMax(&s_r[3], d1); }
     }
     __syncthreads();
-    const int A0 = s_r[0], D0 = s_r[2];
-    const bool sa = cached && s_r[1] > 0 && s_r[1] - A0 <= kMergeDelta;
-    const bool sd = cached && s_r[3] > 0 && s_r[3] - D0 <= kMergeDelta;
-    if (sa) for (int k = threadIdx.x; k < s_r[1] - A0; k += blockDim.x) sadd[k] = __ldg(a.add + A0 + k);
-    if (sd) for (int k = threadIdx.x; k < s_r[3] - D0; k += blockDim.x) sdel[k] = __ldg(a.del + D0 + k);
-    __syncthreads();
-    for (int64_t j = e0 + threadIdx.x; j < e1; j += blockDim.x) {
-      int32_t v, orp;
-      int4 t;
-      if (cached) {
-        const int32_t r = row_of(srp, 0, rhi - rlo, j);
-        v = rlo + r; orp = srp[r]; t = stc[r];
-      } else {
-        v = row_of(a.orowptr, rlo, rhi, j); orp = __ldg(a.orowptr + v); t = __ldg(a.touch + v);
-      }
-      const int32_t c = __ldcs(a.ocol + j);
-      int64_t pos = (int64_t)__ldg(a.nrowptr + v) + (j - orp);
-      if (t.y != t.x || t.w != t.z) {
-        const uint64_t key = ((uint64_t)v << a.nb) | (uint64_t)c;
-        int64_t dl;
-        bool gone;
-        if (sd) {
-          const int64_t q = lb_u64_s(sdel, t.z - D0, t.w - D0, key);
-          gone = q < t.w - D0 && sdel[q] == key;
-          dl = q + D0;
-        } else {
-          dl = lb_u64(a.del, t.z, t.w, key);
-          gone = dl < t.w && a.del[dl] == key;
+    auto orowptr = [&](int32_t r) { return cached ? srp[r - rlo] : __ldg(a.orowptr + r); };
+    auto touch = [&](int32_t r) { return cached ? stc[r - rlo] : __ldg(a.touch + r); };
+    auto nrowptr = [&](int32_t r) { return cached ? snrp[r - rlo] : __ldg(a.nrowptr + r); };
+    const int64_t j0 = e0 + (int64_t)threadIdx.x * kMergeIPT;
+    if (j0 < e1) {
+      int32_t v = cached ? rlo + row_of(srp, 0, rhi - rlo, j0) : row_of(a.orowptr, rlo, rhi, j0);
+      int32_t orp = orowptr(v), oend = orowptr(v + 1);
+      int4 t = touch(v);
+      int32_t nrp = nrowptr(v);
+      bool fresh = true;                                // cursors of row v not set yet
+      int64_t al = 0, dl = 0;
+      const int64_t jend = min(j0 + (int64_t)kMergeIPT, e1);
+      for (int64_t j = j0; j < jend; ++j) {
+        while (j >= oend) {                             // next (non-empty) row
+          ++v;
+          orp = oend;
+          oend = orowptr(v + 1);
+          t = touch(v);
+          nrp = nrowptr(v);
+          fresh = true;
         }
-        if (gone) {                                     // deleted
-          if (a.emap_out) a.emap_out[j] = -1;
-          continue;
+        const int32_t c = scol[j - e0];
+        int64_t pos = (int64_t)nrp + (j - orp);
+        if (t.y != t.x || t.w != t.z) {
+          const uint64_t key = ((uint64_t)v << a.nb) | (uint64_t)c;
+          if (fresh) {
+            al = lb_u64(a.add, t.x, t.y, key);
+            dl = lb_u64(a.del, t.z, t.w, key);
+            fresh = false;
+          } else {
+            while (al < t.y && __ldg(a.add + al) < key) ++al;
+            while (dl < t.w && __ldg(a.del + dl) < key) ++dl;
+          }
+          if (dl < t.w && __ldg(a.del + dl) == key) {   // deleted
+            if (a.emap_out) a.emap_out[j] = -1;
+            continue;
+          }
+          pos += (al - t.x) - (dl - t.z);
         }
-        const int64_t al = sa ? lb_u64_s(sadd, t.x - A0, t.y - A0, key) + A0 : lb_u64(a.add, t.x, t.y, key);
-        pos += (al - t.x) - (dl - t.z);
+        a.ncol[pos] = c;
+        if (a.emap_out) a.emap_out[j] = (int32_t)pos;
+        if (a.eid_new) a.eid_new[pos] = a.emap_in[a.eid_old[j]];
       }
-      a.ncol[pos] = c;
-      if (a.emap_out) a.emap_out[j] = (int32_t)pos;
-      if (a.eid_new) a.eid_new[pos] = a.emap_in[a.eid_old[j]];
     }
   } else {                                            // added edges
     const uint64_t mask = (uint64_t(1) << a.nb) - 1;

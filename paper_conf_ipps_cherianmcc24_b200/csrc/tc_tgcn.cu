@@ -2300,3 +2300,154 @@ extern "C" stg_status stg_debug_sum_parts(const float* part, int32_t nb, int32_t
   count_launch();
   return check_launch("stg_debug_sum_parts");
 }
+
+// ------------------------------------------------------------------ NEXT-2 dense parts on tcgen05
+// The original T-GCN cell's convolutions multiply a row
+// concatenation [A1 | A2] by a small weight slice:
+//   out[r, :] (+)= rs[r] · [A1[r, :K1] | A2[r, :K2]] · W,  W(k, n) = W[k·sk + n·sn]
+// (the forward [X, H]·W_g / [X, r⊙H]·W_c, the backward dY·W[F:, :]ᵀ), and reduce
+//   grad[k, n] += Σ_r [A1 | A2][r, k] · B[r, n]
+// (dW_g, dW_c) — both 3xTF32 on the tensor cores like the TGCN's X·W and Σ AᵀB.
+namespace stg {
+namespace {
+
+// one 128-row tile per CTA at a time; B = Wᵀ [N × Kp] and the A tile [128 × Kp]
+// (both hi / lo, K-major) in shared memory; accumulator in TMEM; thread = row.
+template <int N>
+__global__ void __launch_bounds__(kTcThreads) k_tc_catmm(int V, const float* __restrict__ A1, int K1, int64_t ld1,
+                                                         const float* __restrict__ A2, int K2, int64_t ld2, int Kp,
+                                                         const float* __restrict__ W, int64_t sk, int64_t sn,
+                                                         const float* __restrict__ rs, float* __restrict__ out,
+                                                         int64_t ldo, int accumulate) {
+  extern __shared__ __align__(128) unsigned char sm[];
+  __shared__ uint64_t mbar;
+  __shared__ uint32_t tslot;
+  unsigned char* bhi = sm;
+  unsigned char* blo = bhi + N * Kp * 4;
+  unsigned char* ahi = blo + N * Kp * 4;
+  unsigned char* alo = ahi + 128 * Kp * 4;
+  constexpr uint32_t NC = N <= 32 ? 32 : (N <= 64 ? 64 : 128);
+  const int K = K1 + K2;
+  for (int e = threadIdx.x; e < N * Kp; e += blockDim.x) {            // B = Wᵀ (strided slice), zero past K
+    const int n = e / Kp, k = e % Kp;
+    const float v = k < K ? W[(int64_t)k * sk + (int64_t)n * sn] : 0.0f;
+    const float h = tc::tf32_hi(v);
+    *reinterpret_cast<float*>(bhi + tc::kmaj_off(n, k, Kp)) = h;
+    *reinterpret_cast<float*>(blo + tc::kmaj_off(n, k, Kp)) = v - h;
+  }
+  for (int i = threadIdx.x; i < 128 * Kp; i += kTcThreads) {          // zero the K padding once
+    reinterpret_cast<float*>(ahi)[i] = 0.f;
+    reinterpret_cast<float*>(alo)[i] = 0.f;
+  }
+  if ((threadIdx.x >> 5) == 0) tc::tmem_alloc(&tslot, NC);
+  if (threadIdx.x == 0) { tc::mbar_init(&mbar, 1); tc::fence_mbar_init(); }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  uint32_t phase = 0;
+  const uint32_t idesc = tc::idesc_tf32(128, N, 0, 0);
+  const int ntiles = (V + 127) / 128;
+  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int r0 = tile * 128;
+    tc::stage_rows(ahi, alo, A1 + (int64_t)r0 * ld1, ld1, V - r0, 128, K1, 0, 0, Kp);
+    if (K2 > 0) tc::stage_rows(ahi, alo, A2 + (int64_t)r0 * ld2, ld2, V - r0, 128, K2, 0, K1, Kp);
+    sync_mma_operands();
+    if (threadIdx.x == 0) {
+      mma_seg(tm, tc::smem_u32(ahi), tc::smem_u32(alo), Kp, 0, tc::smem_u32(bhi), tc::smem_u32(blo), Kp, 0, Kp, idesc,
+              true);
+      tc::commit(&mbar);
+    }
+    wait_mma(&mbar, phase);
+    const int row = r0 + threadIdx.x;
+    float v[N];
+    tmem_row_load<N>(tm, 0, v);
+    if (row < V) {
+      const float s = rs ? rs[row] : 1.0f;
+      float4* o = reinterpret_cast<float4*>(out + (int64_t)row * ldo);
+#pragma unroll
+      for (int c = 0; c < N / 4; ++c) {
+        float4 r = make_float4(s * v[4 * c], s * v[4 * c + 1], s * v[4 * c + 2], s * v[4 * c + 3]);
+        if (accumulate) {
+          const float4 q = o[c];
+          r.x += q.x; r.y += q.y; r.z += q.z; r.w += q.w;
+        }
+        o[c] = r;
+      }
+    }
+    tc::fence_before();
+    __syncthreads();
+    tc::fence_after();
+  }
+  tc::fence_before();
+  __syncthreads();
+  if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
+}
+
+// grad[k][n] += tot[row(k)][n]; rows 0..K1 hold A1's features, A2's start at hoff
+__global__ void k_cat_scatter(int K1, int K2, int N, int hoff, int Np, const float* __restrict__ tot,
+                              float* __restrict__ grad) {
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < (K1 + K2) * N; e += gridDim.x * blockDim.x) {
+    const int k = e / N, n = e % N;
+    const int m = k < K1 ? k : hoff + (k - K1);
+    grad[e] += tot[(int64_t)m * Np + n];
+  }
+}
+
+}  // namespace
+
+bool tc_cat_supported(int K1, int K2, int N) {
+  return (N == 16 || N == 32 || N == 64) && K1 % 4 == 0 && K2 % 4 == 0 && K1 >= 4 && K1 + K2 <= 128 &&
+         32 * ((K1 + 31) / 32) + 32 * ((K2 + 31) / 32) <= 128;
+}
+
+stg_status tc_catmm(int V, const float* A1, int K1, int64_t ld1, const float* A2, int K2, int64_t ld2, const float* W,
+                    int64_t sk, int64_t sn, int N, const float* rs, float* out, int64_t ldo, bool accumulate,
+                    cudaStream_t s) {
+  if (V <= 0) return STG_OK;
+  const int Kp = (K1 + K2 + 7) / 8 * 8;
+  const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)2 * 128 * Kp * 4;
+  const int ntiles = (V + 127) / 128;
+#define STG_CATMM(NN)                                                                                           \
+  do {                                                                                                          \
+    STG_TRY(prep(k_tc_catmm<NN>, smem));                                                                        \
+    const int nb = std::min(ntiles, occupancy_blocks(k_tc_catmm<NN>, smem));                                    \
+    k_tc_catmm<NN><<<nb, kTcThreads, smem, s>>>(V, A1, K1, ld1, A2, K2, ld2, Kp, W, sk, sn, rs, out, ldo,        \
+                                                accumulate ? 1 : 0);                                            \
+  } while (0)
+  if (N == 16) STG_CATMM(16);
+  else if (N == 32) STG_CATMM(32);
+  else if (N == 64) STG_CATMM(64);
+  else return fail(STG_ERR_INVALID_ARG, "tc_catmm: N=%d", N);
+#undef STG_CATMM
+  count_launch();
+  return check_launch("tc_catmm");
+}
+
+// grad[K1+K2][N] += [A1 | A2]ᵀ · B  (A1 [V, K1], A2 [V, K2], B [V, N], row-major, contiguous)
+stg_status tc_atb_cat(int V, const float* A1, int K1, const float* A2, int K2, const float* B, int N, float* part,
+                      float* tot, float* grad, cudaStream_t s) {
+  if (V <= 0) return STG_OK;
+  const int NB = (N + 31) / 32, Np = 32 * NB, n1 = (K1 + 31) / 32, n2 = K2 > 0 ? (K2 + 31) / 32 : 0;
+  CUtensorMap m[4], ones;
+  STG_TRY(make_tmap_f32(&m[0], A1, (uint64_t)V, K1, K1, 32, kAtbRT, true));
+  if (K2 > 0) STG_TRY(make_tmap_f32(&m[1], A2, (uint64_t)V, K2, K2, 32, kAtbRT, true));
+  else m[1] = m[0];
+  STG_TRY(make_tmap_f32(&m[2], B, (uint64_t)V, N, N, 32, kAtbRT, true));
+  m[3] = m[0];
+  STG_TRY(ones_map(&ones, kAtbRT, s));
+  AtbSpec2 sp{};
+  sp.V = V; sp.na = 1; sp.a_first[0] = 0; sp.nsa = n1 + n2; sp.nb = NB; sp.b_map = 2; sp.part = part;
+  for (int k = 0; k < n1; ++k) { sp.src_map[k] = 0; sp.src_col[k] = 32 * k; }
+  for (int k = 0; k < n2; ++k) { sp.src_map[n1 + k] = 1; sp.src_col[n1 + k] = 32 * k; }
+  int nb = 0;
+  STG_TRY(atb2_dispatch(NB, m, ones, sp, &nb, s));
+  const int n = 128 * Np;
+  if (nb <= 16 * kSumMaxGroups) k_tc_sum_parts2<<<(n + 31) / 32, 256, 0, s>>>(part, nb, n, tot);
+  else k_tc_sum_parts<<<(n + 255) / 256, 256, 0, s>>>(part, nb, n, tot);
+  k_cat_scatter<<<((K1 + K2) * N + 255) / 256, 256, 0, s>>>(K1, K2, N, 32 * n1, Np, tot, grad);
+  count_launch(2);
+  return check_launch("tc_atb_cat");
+}
+
+}  // namespace stg

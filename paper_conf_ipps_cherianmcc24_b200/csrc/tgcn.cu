@@ -37,6 +37,12 @@ stg_status tc_gru_bwd(int V, int H, const float* C, const float* Hp, const float
                       const float* ndst, float* dCs, float* dHp, float* da, float* RH, cudaStream_t s,
                       const float2* hg = nullptr, const float* w_o = nullptr);
 int tc_gru_blocks(int V);
+bool tc_cat_supported(int K1, int K2, int N);
+stg_status tc_catmm(int V, const float* A1, int K1, int64_t ld1, const float* A2, int K2, int64_t ld2, const float* W,
+                    int64_t sk, int64_t sn, int N, const float* rs, float* out, int64_t ldo, bool accumulate,
+                    cudaStream_t s);
+stg_status tc_atb_cat(int V, const float* A1, int K1, const float* A2, int K2, const float* B, int N, float* part,
+                      float* tot, float* grad, cudaStream_t s);
 stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* part, float* tot, float* dW,
                  cudaStream_t s);
 stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
@@ -1099,6 +1105,8 @@ static stg_status t2_mm(int32_t V, const float* A1, int32_t K1, int64_t ld1, con
                         bool accumulate, cudaStream_t s) {
   if (V == 0) return STG_OK;
   const int K = K1 + K2;
+  if (tc_cat_supported(K1, K2, N) && ld1 % 4 == 0 && (K2 == 0 || ld2 % 4 == 0) && ldo % 4 == 0)   // tensor cores
+    return tc_catmm(V, A1, K1, ld1, A2, K2, ld2, W, sk, sn, N, rs, out, ldo, accumulate, s);
   const size_t smem = sizeof(float) * ((size_t)K * N + 32 * (size_t)(K + 1));
   STG_TRY(set_smem(k_cat_mm, smem));
   const int nb = grid_blocks((const void*)k_cat_mm, smem, (V + 31) / 32);
@@ -1112,6 +1120,11 @@ static stg_status t2_atb(int32_t V, const float* A1, int32_t K1, const float* A2
                          int32_t N, float* grad, TgcnWs& ws, cudaStream_t s) {
   if (V == 0) return STG_OK;
   const int K = K1 + K2;
+  if (tc_cat_supported(K1, K2, N)) {                  // tensor cores (Σ AᵀB with TMA MN-major operands)
+    STG_TRY(ws.part_tc.alloc((size_t)tc_atb_max_blocks() * 2 * 128 * 128));
+    STG_TRY(ws.dl_tmp.alloc(2 * 128 * 128));
+    return tc_atb_cat(V, A1, K1, A2, K2, B, N, ws.part_tc.p, ws.dl_tmp.p, grad, s);
+  }
   const size_t smem = sizeof(float) * (32 * (size_t)K + 32 * (size_t)N + (size_t)K * N);
   STG_TRY(set_smem(k_cat_atb, smem));
   const int nb = grid_blocks((const void*)k_cat_atb, smem, (V + 31) / 32);
@@ -1703,3 +1716,143 @@ stg_status stg_tgcn_train_sequence_batched(const stg_graph* graph, int32_t S, co
 }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------- sharded mode in the library
+// Stream memory operations (driver API, via the runtime's entry-point query): a
+// stream waits for a peer's counter / publishes its own after the preceding work.
+namespace {
+typedef CUresult (*PFN_waitValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+typedef CUresult (*PFN_writeValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+struct StreamMemOps {
+  PFN_waitValue32 wait = nullptr;
+  PFN_writeValue32 write = nullptr;
+};
+stg_status stream_mem_ops(StreamMemOps* ops) {
+  static StreamMemOps o;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaDriverEntryPointQueryResult q;
+    void* f = nullptr;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      o.wait = reinterpret_cast<PFN_waitValue32>(f);
+    f = nullptr;
+    if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      o.write = reinterpret_cast<PFN_writeValue32>(f);
+    cudaGetLastError();
+  });
+  if (!o.wait || !o.write) return fail(STG_ERR_CUDA, "stream memory operations unavailable");
+  *ops = o;
+  return STG_OK;
+}
+// wait until every rank's counter `slot` reached `value`
+stg_status wait_all(const StreamMemOps& ops, const stg_peer_exchange* px, int slot, uint32_t value, cudaStream_t s) {
+  if (value == 0) return STG_OK;
+  for (int q = 0; q < px->world; ++q) {
+    const CUresult r = ops.wait((CUstream)s, (CUdeviceptr)(px->flags[q] + slot), value, CU_STREAM_WAIT_VALUE_GEQ);
+    if (r != CUDA_SUCCESS) return fail(STG_ERR_CUDA, "cuStreamWaitValue32 (rank %d slot %d): error %d", q, slot, (int)r);
+  }
+  return STG_OK;
+}
+stg_status publish(const StreamMemOps& ops, const stg_peer_exchange* px, int slot, uint32_t value, cudaStream_t s) {
+  const CUresult r = ops.write((CUstream)s, (CUdeviceptr)(px->flags[px->rank] + slot), value, 0);
+  if (r != CUDA_SUCCESS) return fail(STG_ERR_CUDA, "cuStreamWriteValue32 (slot %d): error %d", slot, (int)r);
+  return STG_OK;
+}
+}  // namespace
+
+stg_status stg_tgcn_train_sequence_peer(stg_dtdg* dtdg, int32_t t0, int32_t S, const stg_tgcn_params* p,
+                                        const float* w_o, const float* b_o, const float* const* X_loc,
+                                        const float* const* Y_loc, const float* H0, float* H_seq, float* G_work,
+                                        float* dP_loc, stg_tgcn_grads* grads, float* dw_o, float* db_o,
+                                        float* loss_accum, stg_state_stack* stack, stg_peer_exchange* px,
+                                        stg_stream_t stream) {
+  STG_TRY(check_params(p));
+  if (!dtdg || !px || S < 1 || !X_loc || !Y_loc || !H0 || !H_seq || !G_work || !dP_loc || !grads || !stack ||
+      !w_o || !b_o)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_peer: bad arguments");
+  if (px->world < 1 || px->world > STG_MAX_PEERS || px->rank < 0 || px->rank >= px->world || !px->bounds)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_peer: bad world / rank / bounds");
+  for (int q = 0; q < px->world; ++q)
+    if (!px->flags[q] || !px->P[0][q] || !px->P[1][q] || !px->dP[0][q] || !px->dP[1][q])
+      return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_peer: NULL exchange buffer of rank %d", q);
+  if (!tc_supported(p->F, p->H)) return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_peer: needs H in {16,32}");
+  if (t0 < 0 || t0 + S > stg_dtdg_num_timestamps(dtdg))
+    return fail(STG_ERR_OUT_OF_RANGE, "stg_tgcn_train_sequence_peer: [%d,%d) outside the DTDG", t0, t0 + S);
+  StreamMemOps ops;
+  STG_TRY(stream_mem_ops(&ops));
+  cudaStream_t s = (cudaStream_t)stream;
+  const int32_t rb = px->bounds[px->rank], R = px->bounds[px->rank + 1] - rb, H = p->H, H3 = 3 * H;
+  stg_csr_view v;
+  STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, t0, 0, STG_PART_IN, stream, &v));
+  const int32_t Vall = v.num_nodes;
+  if (v.row_begin != rb || v.row_end - v.row_begin != R)
+    return fail(STG_ERR_INVALID_ARG, "stg_tgcn_train_sequence_peer: the DTDG's row block is not bounds[rank]");
+  const size_t VH = (size_t)R * H;
+  TgcnWs& ws = stack->ws;
+  const int nbh = tc_gru_blocks(std::max(R, 1));
+  STG_TRY(ws.hg.alloc((size_t)S * std::max(R, 1)));
+  STG_TRY(ws.hd_lpart.alloc((size_t)nbh));
+  STG_TRY(ws.hd_gpart.alloc((size_t)nbh * (H + 1)));
+  const size_t need = stack_bytes(R, H);
+  if (stack->top + (size_t)S * need > stack->cap)
+    return fail(STG_ERR_NO_MEMORY, "stg_tgcn_train_sequence_peer: state stack too small");
+  const float* blocks[2][STG_MAX_PEERS];
+  const float* dblocks[2][STG_MAX_PEERS];
+  for (int b = 0; b < 2; ++b)
+    for (int q = 0; q < px->world; ++q) { blocks[b][q] = px->P[b][q]; dblocks[b][q] = px->dP[b][q]; }
+  // ---- forward
+  for (int32_t i = 0; i < S; ++i) {
+    if (i > 0) STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, t0 + i, 0, STG_PART_IN, stream, &v));
+    const uint32_t n = ++px->fwd_count;
+    const int b = (int)(n & 1u);
+    STG_TRY(wait_all(ops, px, 1, n >= 2 ? n - 2 : 0, s));             // every reader of buffer b is done
+    STG_TRY(stg_tgcn_project(&v, p, X_loc[i], px->P[b][px->rank], stream));
+    STG_TRY(publish(ops, px, 0, n, s));
+    STG_TRY(wait_all(ops, px, 0, n, s));                                // every owner's P' rows are there
+    float* C = reinterpret_cast<float*>(stack->arena.p + stack->top);
+    const float* Hp = i == 0 ? H0 : H_seq + (size_t)(i - 1) * VH;
+    const stg_peer_rows rows{px->world, px->bounds, blocks[b], (int64_t)H3};
+    const float* ndst_loc = v.norm_dst ? v.norm_dst + v.row_begin : nullptr;
+    STG_TRY(aggregate_launch(&v, 0, H3, nullptr, 0, C, H3, ndst_loc, nullptr, p->b, s, &rows));
+    STG_TRY(publish(ops, px, 1, n, s));
+    const HeadArgs ha{Y_loc[i], w_o, b_o, 1.0f / (float)Vall, ws.hd_lpart.p, ws.hd_gpart.p,
+                      ws.hg.p + (size_t)i * std::max(R, 1)};
+    STG_TRY(fwd_gru(R, p, C, Hp, H_seq + (size_t)i * VH, s, R > 0 ? &ha : nullptr));
+    if (R > 0) {
+      ProfScope prof_h(PH_HEAD, s);
+      STG_TRY(tc_seq_head_reduce(nbh, H, ws.hd_lpart.p, ws.hd_gpart.p, 1.0 / (double)Vall, loss_accum, dw_o, db_o,
+                                 s));
+    }
+    stack->entries.push_back(StackEntry{Hp, C, R, H, need});
+    stack->top += need;
+  }
+  // ---- backward (LIFO)
+  float* G = G_work;
+  float* Gn = G_work + VH;
+  if (VH) STG_CUDA(cudaMemsetAsync(G, 0, sizeof(float) * VH, s));
+  for (int32_t i = S - 1; i >= 0; --i) {
+    STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, t0 + i, 1, STG_PART_OUT, stream, &v));
+    const uint32_t m = ++px->bwd_count;
+    const int b = (int)(m & 1u);
+    STG_TRY(wait_all(ops, px, 3, m >= 2 ? m - 2 : 0, s));
+    if (stack->entries.empty()) return fail(STG_ERR_STATE, "stg_tgcn_train_sequence_peer: state stack underflow");
+    const StackEntry e = stack->entries.back();
+    BwdBufs bb;
+    STG_TRY(bwd_alloc(ws, &v, p, 1, &bb));
+    STG_TRY(bwd_gru(&v, p, e.C, e.Hp, G, Gn, grads, ws, bb, s, R > 0 ? ws.hg.p + (size_t)i * std::max(R, 1) : nullptr,
+                    w_o));
+    STG_TRY(bwd_dl(&v, p, e.C, e.Hp, grads, ws, bb, s));
+    STG_TRY(aggregate_launch(&v, 1, H3, bb.dC[0], H3, px->dP[b][px->rank], H3, v.norm_src, nullptr, nullptr, s));
+    STG_TRY(publish(ops, px, 2, m, s));
+    STG_TRY(wait_all(ops, px, 2, m, s));                                // every rank's partial dP is there
+    STG_TRY(stg_reduce_scatter_rows(px->world, px->bounds, dblocks[b], H3, px->rank, H3, dP_loc, H3, stream));
+    STG_TRY(publish(ops, px, 3, m, s));
+    STG_TRY(stg_tgcn_dw(p, R, X_loc[i], dP_loc, grads, stack, stream));
+    stack->entries.pop_back();
+    stack->top -= e.bytes;
+    std::swap(G, Gn);
+  }
+  return check_launch("stg_tgcn_train_sequence_peer");
+}

@@ -10,6 +10,8 @@ test); these helpers are the host logic and the collectives only — no compute.
 """
 from __future__ import annotations
 
+import ctypes
+
 import numpy as np
 import torch
 import torch.distributed as dist
@@ -135,13 +137,19 @@ class PeerTGCN:
     owners inside the aggregation (stg_tgcn_step_peer); the backward's partial
     dP of the local edges is reduce-scattered to the owners over peer loads
     (stg_reduce_scatter_rows) before dW += X_locᵀ dP_loc.  Two buffers per
-    exchanged matrix alternate per timestep, so one stream barrier per exchange
-    orders every write after the previous readers."""
+    exchanged matrix alternate per timestep.
 
-    def __init__(self, stg, bounds, V: int, F: int, H: int, S: int):
+    native=True (DTDG sources): the whole sequence runs in the library
+    (stg_tgcn_train_sequence_peer) with the cross-rank ordering done by device-side
+    counters in peer memory (stream wait / write operations) — no host barrier or
+    collective per timestep.  native=False: the Python loop below, one stream
+    barrier (a one-element NCCL all-reduce) per exchange."""
+
+    def __init__(self, stg, bounds, V: int, F: int, H: int, S: int, native: bool = True):
         self.stg = stg
         self.bounds = list(bounds)
         self.rank = dist.get_rank()
+        self.world = dist.get_world_size()
         self.V, self.F, self.H, self.S = V, F, H, S
         self.R = self.bounds[self.rank + 1] - self.bounds[self.rank]
         self.P = [PeerGroup(self.bounds, 3 * H) for _ in range(2)]
@@ -149,11 +157,30 @@ class PeerTGCN:
         self.dP_loc = torch.empty(max(self.R, 1), 3 * H, device="cuda")
         self.G = torch.empty(2, max(self.R, 1), H, device="cuda")
         self.stack = stg.stg_state_stack_create(S * max(self.R, 1) * 3 * H * 4 + (1 << 20))
+        self.native = native
+        if native:
+            # every rank's 4 exchange counters (zero-initialised peer memory)
+            self.flags = PeerGroup([0] + [1] * self.world, 4, full=True)
+            px = stg.stg_peer_exchange()
+            px.world, px.rank = self.world, self.rank
+            self._bounds_c = (ctypes.c_int32 * (self.world + 1))(*self.bounds)
+            px.bounds = self._bounds_c
+            for b in range(2):
+                for k in range(self.world):
+                    px.P[b][k] = self.P[b].ptrs[k]
+                    px.dP[b][k] = self.dP[b].ptrs[k]
+            for k in range(self.world):
+                px.flags[k] = self.flags.ptrs[k]
+            self.px = px
 
     def train_sequence(self, source, t0, params, w_o, b_o, X_loc, Y_loc, H0, H_seq, grads, dw_o, db_o, loss,
                        barrier=stream_barrier):
         stg, S, R, H = self.stg, len(X_loc), self.R, self.H
         dyn = isinstance(source, stg.Dtdg)
+        if self.native and dyn:
+            stg.stg_tgcn_train_sequence_peer(source, t0, params, w_o, b_o, X_loc, Y_loc, H0, H_seq, self.G,
+                                             self.dP_loc, grads, dw_o, db_o, loss, self.stack, self.px)
+            return
 
         def view(t, backward):
             if not dyn:

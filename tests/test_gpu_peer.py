@@ -181,7 +181,9 @@ def test_tgcn_peer_sequence_simulated_ranks(stg):
             stg.stg_tgcn_project(v, pg, r["X"][i], r["P"][i & 1])
         table = stg.PeerRows(b, [r["P"][i & 1].data_ptr() for r in ranks], 3 * H)
         for r, v in zip(ranks, views):
-            Hp = torch.zeros(r["R"], H, device="cuda") if i == 0 else r["Hs"][i - 1]
+            if i == 0:
+                r["H0"] = torch.zeros(r["R"], H, device="cuda")   # kept: the stack holds H_{t-1} by reference
+            Hp = r["H0"] if i == 0 else r["Hs"][i - 1]
             stg.stg_tgcn_step_peer(v, pg, table, Hp, r["Hs"][i], r["st"])
             stg.stg_mse_head(r["Hs"][i], r["Y"][i], pg["w_o"], pg["b_o"], loss_accum=r["loss"], V_total=V)
     for i in range(S - 1, -1, -1):
@@ -207,7 +209,9 @@ def test_tgcn_peer_sequence_simulated_ranks(stg):
 
 
 def _ipc_worker(rank, world, port, outdir):
+    import faulthandler
     import sys
+    faulthandler.enable()
     sys.path.insert(0, ROOT)
     import torch.distributed as dist
     import paper_conf_ipps_cherianmcc24_b200 as stg
@@ -230,7 +234,8 @@ def _ipc_worker(rank, world, port, outdir):
     X = [torch.from_numpy(gen.features(cfg, t)[lo:hi].copy()).cuda() for t in range(S)]
     Y = [torch.from_numpy(gen.labels(cfg, t)[lo:hi].copy()).cuda() for t in range(S)]
     Hs = torch.empty(S, R, H, device="cuda")
-    drv.train_sequence(g, 0, p, p["w_o"], p["b_o"], X, Y, torch.zeros(R, H, device="cuda"), Hs, grads, dw, db, loss)
+    H0 = torch.zeros(R, H, device="cuda")          # alive until the sequence's kernels ran
+    drv.train_sequence(g, 0, p, p["w_o"], p["b_o"], X, Y, H0, Hs, grads, dw, db, loss)
     torch.cuda.synchronize()
     out = {n: t.cpu().numpy() for n, t in grads.items()}
     out.update(w_o=dw.cpu().numpy(), b_o=db.cpu().numpy(), loss=loss.cpu().numpy(), H=Hs[-1].cpu().numpy(),

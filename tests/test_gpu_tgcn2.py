@@ -181,6 +181,8 @@ def test_tgcn2_sharded_peer_simulated_ranks(stg):
 
 
 def _ipc_worker2(rank, world, port, outdir):
+    import faulthandler
+    faulthandler.enable()
     import os
     import sys
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -204,7 +206,8 @@ def _ipc_worker2(rank, world, port, outdir):
     X = [torch.from_numpy(gen.features(cfg, t)[lo:hi].copy()).cuda() for t in range(S)]
     Y = [torch.from_numpy(gen.labels(cfg, t)[lo:hi].copy()).cuda() for t in range(S)]
     Hs = torch.empty(S, R, H, device="cuda")
-    drv.train_sequence(g, 0, p, p["w_o"], p["b_o"], X, Y, torch.zeros(R, H, device="cuda"), Hs, grads, dw, db, loss)
+    H0 = torch.zeros(R, H, device="cuda")          # alive until the sequence's kernels ran
+    drv.train_sequence(g, 0, p, p["w_o"], p["b_o"], X, Y, H0, Hs, grads, dw, db, loss)
     torch.cuda.synchronize()
     out = {n: t.cpu().numpy() for n, t in grads.items()}
     out.update(w_o=dw.cpu().numpy(), b_o=db.cpu().numpy(), loss=loss.cpu().numpy(), H=Hs[-1].cpu().numpy(),
