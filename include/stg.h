@@ -262,7 +262,7 @@ stg_status stg_aggregate_set_strategy(int32_t strategy);
  * key 0: neighbour rows in flight per warp, 4 | 8 | 16 (default 4);
  * key 1: minimum resident blocks per SM (register budget), 2..6 (default 6;
  *        supported pairs (rows, blocks): (4,6) (8,4) (16,2) (16,3));
- * key 2: 32 | 64 (default 32): strategy 2 serves launch widths above this. */
+ * key 2: 0 | 8 | 16 | 32 | 64 (default 0): strategy 2 serves launch widths above this. */
 stg_status stg_aggregate_set_param(int32_t key, int64_t value);
 
 /* ---- TGCN (GCN + GRU; reading C13-C15) ----

@@ -9,7 +9,7 @@
 // (hub rows are cut into 64-edge chunks).  Three decompositions
 // (stg_aggregate_set_strategy; DESIGN.md §Aggregation has the measurements):
 //
-//  2 (default, 64 < W <= 128 per launch) k_agg_stream: a warp takes 32 items
+//  2 (default, W <= 128 per launch) k_agg_stream: a warp takes 32 items
 //    at a time from a work queue, scans their edge counts and walks their
 //    concatenated edge lists in 32-edge batches, gathering D neighbour rows at
 //    once ACROSS row boundaries (lane c holds float4 column c of a row), with
@@ -813,7 +813,9 @@ struct AggTune {
   // 24 x 16 (C5 W = 96: 0.443 vs 0.477 ms; W = 64: 0.357 vs 0.418 ms)
   int d = 4;
   int minb = 6;
-  int wmin = 32;     // stream kernel for wmin < W_launch <= 128
+  // stream kernel for wmin < W_launch <= 128: it beats the row items at every width
+  // on C5 (scripts/agg_width_probe.py: W = 16 0.353 vs 0.452 ms, 32 0.364 vs 0.561, 64 0.392 vs 0.756)
+  int wmin = 0;
 };
 static AggTune g_tune;
 
@@ -1094,7 +1096,7 @@ stg_status stg_aggregate_set_param(int32_t key, int64_t value) {
       stg::g_tune.minb = (int)value;
       return STG_OK;
     case 2:
-      if (value != 32 && value != 64) break;
+      if (value != 0 && value != 8 && value != 16 && value != 32 && value != 64) break;
       stg::g_tune.wmin = (int)value;
       return STG_OK;
 

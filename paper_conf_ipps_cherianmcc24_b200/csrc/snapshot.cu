@@ -32,13 +32,15 @@ namespace stg {
 
 namespace {
 
-constexpr int kRowTile = 4096;                   // rows per scan / scatter tile
+constexpr int kRowTile = 4096;                   // rows per scan / scatter tile (1024: no faster on C5, offsets 2x slower)
 constexpr int kRowThreads = 256;
-constexpr int kRowIPT = kRowTile / kRowThreads;  // 16 rows per thread
+constexpr int kRowIPT = kRowTile / kRowThreads;  // rows per thread
+constexpr int kScatRounds = kRowTile / kRowThreads;   // 32-row rounds per warp in k_ids_scatter
 constexpr int kIdsSat = 1023;                    // degrees >= this share bucket 0
 constexpr int kIdsBuckets = kIdsSat + 2;         // 0..kIdsSat: degree buckets, kIdsSat+1: outside the block
 constexpr int kIdsOut = kIdsSat + 1;
 constexpr int kSatSortMax = 8192;                // saturated prefix sorted in shared memory
+constexpr int kSatRankMax = 2048;                // ... ranked by counting up to this size (O(m²/1024) per thread)
 constexpr int kMergeTile = 2048;                 // old edges per merge CTA
 
 __device__ __forceinline__ int ids_digit(int32_t v, int32_t d, int32_t rb, int32_t re) {
@@ -110,6 +112,9 @@ struct RowScanArgs {
   int dgl_both;
   float* norm_src;
   float* norm_dst;
+  // (TOUCH) the old CSR's row pointer: tile_row[t] = row of old edge t·kMergeTile
+  const int32_t* orowptr;
+  int32_t* tile_row;
 };
 
 template <bool TOUCH>
@@ -139,6 +144,42 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
       }
     }
     d[k] = x;
+  }
+  if (a.norm_dst) {                                    // (independent of the scan: issued first)
+    int32_t gi[kRowIPT], go[kRowIPT];
+#pragma unroll
+    for (int k = 0; k < kRowIPT; ++k) {
+      const int64_t v = r0 + (int64_t)k * kRowThreads;
+      gi[k] = v < a.V ? __ldg(a.gin + v) : 0;
+      go[k] = (v < a.V && a.dgl_both) ? __ldg(a.gout + v) : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < kRowIPT; ++k) {
+      const int64_t v = r0 + (int64_t)k * kRowThreads;
+      if (v >= a.V) continue;
+      const float nd = gi[k] > 0 ? 1.0f / sqrtf((float)gi[k]) : 0.0f;
+      a.norm_dst[v] = nd;
+      a.norm_src[v] = a.dgl_both ? (go[k] > 0 ? 1.0f / sqrtf((float)go[k]) : 0.0f) : nd;
+    }
+  }
+  if (TOUCH) {                                          // merge tile starts inside these (old) rows
+    const int ln = threadIdx.x & 31;
+    int32_t ob[kRowIPT], oe31[kRowIPT];
+#pragma unroll
+    for (int k = 0; k < kRowIPT; ++k) {                 // row v + 1 is the next lane's row (lane 31 loads it)
+      const int64_t v = r0 + (int64_t)k * kRowThreads;
+      ob[k] = v <= a.V ? __ldg(a.orowptr + v) : 0;     // (row V: the end of the last row)
+      oe31[k] = (ln == 31 && v < a.V) ? __ldg(a.orowptr + v + 1) : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < kRowIPT; ++k) {
+      const int64_t v = r0 + (int64_t)k * kRowThreads;
+      const int32_t nx = __shfl_down_sync(0xffffffffu, ob[k], 1);
+      const int32_t oe = ln == 31 ? oe31[k] : nx;
+      if (v < a.V)
+        for (int32_t t = (ob[k] + kMergeTile - 1) / kMergeTile; (int64_t)t * kMergeTile < oe; ++t)
+          a.tile_row[t] = (int32_t)v;
+    }
   }
   // node_ids key histogram (shared atomics, warp-aggregated by match_any)
   const int lane = threadIdx.x & 31;
@@ -206,22 +247,6 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
       }
     }
   }
-  if (a.norm_dst) {
-#pragma unroll
-    for (int k = 0; k < kRowIPT; ++k) {
-      const int64_t v = r0 + (int64_t)k * kRowThreads;
-      if (v >= a.V) break;
-      const int32_t di = __ldg(a.gin + v);
-      const float nd = di > 0 ? 1.0f / sqrtf((float)di) : 0.0f;
-      a.norm_dst[v] = nd;
-      if (a.dgl_both) {
-        const int32_t dout = __ldg(a.gout + v);
-        a.norm_src[v] = dout > 0 ? 1.0f / sqrtf((float)dout) : 0.0f;
-      } else {
-        a.norm_src[v] = nd;
-      }
-    }
-  }
   __syncthreads();
   for (int dg = threadIdx.x; dg < kIdsBuckets; dg += kRowThreads) a.hist[(int64_t)dg * a.ntiles + tile] = h[dg];
 }
@@ -273,8 +298,8 @@ __device__ __forceinline__ void bucket_bases(const int32_t* __restrict__ totals,
   }
 }
 
-// Stable scatter of one 4096-row tile: warp w owns rows [w·512, w·512+512) of the
-// tile in 16 rounds of 32; ranks from match_any, per-warp bucket counters.
+// Stable scatter of one kRowTile-row tile: warp w owns rows [w·kRowTile/8, (w+1)·kRowTile/8)
+// of the tile in kScatRounds rounds of 32; ranks from match_any, per-warp bucket counters.
 __global__ void __launch_bounds__(kRowThreads) k_ids_scatter(const int32_t* __restrict__ deg, int32_t V, int32_t rb,
                                                              int32_t re, const int32_t* __restrict__ offs,
                                                              const int32_t* __restrict__ totals, int32_t ntiles,
@@ -288,9 +313,9 @@ __global__ void __launch_bounds__(kRowThreads) k_ids_scatter(const int32_t* __re
   __syncwarp();
   const int64_t base = (int64_t)blockIdx.x * kRowTile + (int64_t)w * (kRowTile / 8);
   const unsigned lt = (1u << lane) - 1u;
-  int dig[16], rank[16];
+  int dig[kScatRounds], rank[kScatRounds];
 #pragma unroll
-  for (int r = 0; r < 16; ++r) {
+  for (int r = 0; r < kScatRounds; ++r) {
     const int64_t v = base + r * 32 + lane;
     const bool ok = v < V;
     const int dg = ok ? ids_digit((int32_t)v, __ldg(deg + v), rb, re) : kIdsBuckets + lane;
@@ -314,7 +339,7 @@ __global__ void __launch_bounds__(kRowThreads) k_ids_scatter(const int32_t* __re
   }
   __syncthreads();
 #pragma unroll
-  for (int r = 0; r < 16; ++r) {
+  for (int r = 0; r < kScatRounds; ++r) {
     const int64_t v = base + r * 32 + lane;
     if (v < V) ids[wcnt[w][dig[r]] + rank[r]] = (int32_t)v;
   }
@@ -353,7 +378,19 @@ __global__ void __launch_bounds__(1024) k_ids_finish(int32_t* __restrict__ ids, 
     if ((threadIdx.x & 31) == 0) { atomicAdd(&s_cnt[0], c0); atomicAdd(&s_cnt[1], c1); atomicAdd(&s_cnt[2], c2); }
   }
   if (m > 1) {
-    if (m <= kSatSortMax) {                             // bitonic sort of (~deg, id) in shared memory
+    if (m <= kSatRankMax) {                             // rank by counting over the keys in shared memory
+      for (int i = threadIdx.x; i < m; i += nt) {
+        const int32_t v = ids[i];
+        sk[i] = ((uint64_t)(uint32_t)(0x7fffffff - deg[v]) << 32) | (uint32_t)v;
+      }
+      __syncthreads();
+      for (int i = threadIdx.x; i < m; i += nt) {
+        const uint64_t ki = sk[i];
+        int r = 0;
+        for (int j = 0; j < m; ++j) r += sk[j] < ki;   // same j in every lane: broadcast reads
+        ids[r] = (int32_t)(uint32_t)ki;
+      }
+    } else if (m <= kSatSortMax) {                      // bitonic sort of (~deg, id) in shared memory
       int P = 1;
       while (P < m) P <<= 1;
       for (int i = threadIdx.x; i < P; i += nt) {
@@ -521,89 +558,145 @@ struct MergeArgs {
   int32_t* eid_new;
   const int32_t* in_rowptr_new;
   const int32_t* in_col_new;
+  const int32_t* tile_row;      // row of the first old edge of every tile (k_rowscan)
 };
 
-constexpr int kMergeIPT = kMergeTile / 256;      // consecutive old edges per thread
-
-// Old edges: a CTA takes kMergeTile consecutive positions (loaded coalesced into
-// shared memory); thread t then walks its kMergeIPT consecutive positions in order.
-// Only the first edge of a row in the chunk searches the row's sorted add / delete
-// keys; the following ones advance those cursors (keys and columns are both sorted
-// within a row), so a hub row with thousands of deltas costs ~2 searches per chunk
-// instead of 2 per edge.
-constexpr int kMergeRows = 1024;                 // rows whose rowptr / touch / new rowptr are cached
+// Old edges: a CTA takes kMergeTile consecutive positions.  The tile's rows
+// (rows [tile_row[t], tile_row[t+1]], from k_rowscan) have their old / new row
+// pointers, touch marks and add / delete keys cached in shared memory; the row of
+// every position comes from a max-scan of the row-start marks; then every edge is
+// independent: new position = rowptr'[v] + (j - rowptr[v]) + #adds < key - #dels <
+// key (a binary search in the row's few cached keys), or -1 when deleted.
+// Consecutive threads take consecutive positions, so loads and stores coalesce.
+constexpr int kMergeRows = 512;                  // rows whose rowptr / touch / new rowptr are cached
+constexpr int kMergeKeys = 512;                  // add / delete keys of the tile's rows cached in shared memory
+constexpr int kMergeIPT = kMergeTile / 256;      // positions per thread
 
 __global__ void __launch_bounds__(256) k_merge2(const MergeArgs a) {
-  __shared__ int32_t scol[kMergeTile];
+  __shared__ int32_t scol[kMergeTile], srow[kMergeTile];
   __shared__ int32_t srp[kMergeRows + 1], snrp[kMergeRows];
   __shared__ int4 stc[kMergeRows];
-  __shared__ int32_t s_lo, s_hi;
-  if ((int64_t)blockIdx.x < a.old_tiles) {
-    const int64_t e0 = (int64_t)blockIdx.x * kMergeTile;
+  __shared__ uint64_t sadd[kMergeKeys], sdel[kMergeKeys];
+  __shared__ int32_t s_lo, s_hi, s_rng[4], s_wmax[8];
+  const int64_t add_blocks = (int64_t)gridDim.x - a.old_tiles;      // added edges first: their searches
+  const int64_t tile = (int64_t)blockIdx.x - add_blocks;             // overlap the tiles instead of trailing
+  if (tile >= 0) {
+    const int64_t e0 = tile * kMergeTile;
     const int64_t e1 = min(e0 + (int64_t)kMergeTile, a.E_old);
-    if (threadIdx.x == 0) {
-      s_lo = row_of(a.orowptr, 0, a.V - 1, e0);
-      s_hi = row_of(a.orowptr, 0, a.V - 1, e1 - 1);
+    const int n = (int)(e1 - e0);
+    if (threadIdx.x == 0) {                            // rows [s_lo, s_hi] hold the tile's edges
+      s_lo = __ldg(a.tile_row + tile);
+      s_hi = tile + 1 < a.old_tiles ? __ldg(a.tile_row + tile + 1) : a.V - 1;
+      s_rng[0] = INT32_MAX; s_rng[1] = INT32_MIN; s_rng[2] = INT32_MAX; s_rng[3] = INT32_MIN;
     }
-    for (int k = threadIdx.x; k < e1 - e0; k += blockDim.x) scol[k] = __ldcs(a.ocol + e0 + k);
+#pragma unroll
+    for (int i = 0; i < kMergeIPT; ++i) {
+      const int k = threadIdx.x + i * 256;
+      if (k < n) scol[k] = __ldcs(a.ocol + e0 + k);
+      srow[k] = -1;
+    }
     __syncthreads();
     const int32_t rlo = s_lo, rhi = s_hi, nr = rhi - rlo + 1;
     const bool cached = nr <= kMergeRows;              // (the tile's rows: ~kMergeTile / mean degree)
     if (cached) {
+      int32_t a0 = INT32_MAX, a1 = INT32_MIN, d0 = INT32_MAX, d1 = INT32_MIN;
       for (int k = threadIdx.x; k <= nr; k += blockDim.x) {
         srp[k] = __ldg(a.orowptr + rlo + k);
-        if (k < nr) { stc[k] = __ldg(a.touch + rlo + k); snrp[k] = __ldg(a.nrowptr + rlo + k); }
+        if (k < nr) {
+          const int4 t = __ldg(a.touch + rlo + k);
+          stc[k] = t;
+          snrp[k] = __ldg(a.nrowptr + rlo + k);
+          if (t.y > t.x) { a0 = min(a0, t.x); a1 = max(a1, t.y); }
+          if (t.w > t.z) { d0 = min(d0, t.z); d1 = max(d1, t.w); }
+        }
+      }
+      if (a1 > a0) { atomicMin(&s_rng[0], a0); atomicMax(&s_rng[1], a1); }
+      if (d1 > d0) { atomicMin(&s_rng[2], d0); atomicMax(&s_rng[3], d1); }
+      __syncthreads();
+      for (int k = threadIdx.x; k < nr; k += blockDim.x) {   // row-start marks (non-empty rows)
+        const int32_t b = srp[k], e = srp[k + 1];
+        if (e > b && b < e1) srow[max((int64_t)b - e0, (int64_t)0)] = k;
       }
     }
     __syncthreads();
-    auto orowptr = [&](int32_t r) { return cached ? srp[r - rlo] : __ldg(a.orowptr + r); };
-    auto touch = [&](int32_t r) { return cached ? stc[r - rlo] : __ldg(a.touch + r); };
-    auto nrowptr = [&](int32_t r) { return cached ? snrp[r - rlo] : __ldg(a.nrowptr + r); };
-    const int64_t j0 = e0 + (int64_t)threadIdx.x * kMergeIPT;
-    if (j0 < e1) {
-      int32_t v = cached ? rlo + row_of(srp, 0, rhi - rlo, j0) : row_of(a.orowptr, rlo, rhi, j0);
-      int32_t orp = orowptr(v), oend = orowptr(v + 1);
-      int4 t = touch(v);
-      int32_t nrp = nrowptr(v);
-      bool fresh = true;                                // cursors of row v not set yet
-      int64_t al = 0, dl = 0;
-      const int64_t jend = min(j0 + (int64_t)kMergeIPT, e1);
-      for (int64_t j = j0; j < jend; ++j) {
-        while (j >= oend) {                             // next (non-empty) row
-          ++v;
-          orp = oend;
-          oend = orowptr(v + 1);
-          t = touch(v);
-          nrp = nrowptr(v);
-          fresh = true;
-        }
-        const int32_t c = scol[j - e0];
-        int64_t pos = (int64_t)nrp + (j - orp);
-        if (t.y != t.x || t.w != t.z) {
-          const uint64_t key = ((uint64_t)v << a.nb) | (uint64_t)c;
-          if (fresh) {
-            al = lb_u64(a.add, t.x, t.y, key);
-            dl = lb_u64(a.del, t.z, t.w, key);
-            fresh = false;
-          } else {
-            while (al < t.y && __ldg(a.add + al) < key) ++al;
-            while (dl < t.w && __ldg(a.del + dl) < key) ++dl;
-          }
-          if (dl < t.w && __ldg(a.del + dl) == key) {   // deleted
-            if (a.emap_out) a.emap_out[j] = -1;
-            continue;
-          }
-          pos += (al - t.x) - (dl - t.z);
-        }
-        a.ncol[pos] = c;
-        if (a.emap_out) a.emap_out[j] = (int32_t)pos;
-        if (a.eid_new) a.eid_new[pos] = a.emap_in[a.eid_old[j]];
+    // the tile rows' add / delete keys are contiguous ranges of the sorted lists
+    const int32_t ka0 = s_rng[0], kd0 = s_rng[2];
+    const int32_t na = s_rng[1] > ka0 ? s_rng[1] - ka0 : 0, nd = s_rng[3] > kd0 ? s_rng[3] - kd0 : 0;
+    const bool sa = cached && na <= kMergeKeys, sd = cached && nd <= kMergeKeys;
+    if (sa) for (int k = threadIdx.x; k < na; k += blockDim.x) sadd[k] = __ldg(a.add + ka0 + k);
+    if (sd) for (int k = threadIdx.x; k < nd; k += blockDim.x) sdel[k] = __ldg(a.del + kd0 + k);
+    if (cached) {                                      // inclusive max-scan of the marks: row of every position
+      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+      int32_t m[kMergeIPT];
+      int32_t run = -1;
+#pragma unroll
+      for (int i = 0; i < kMergeIPT; ++i) { run = max(run, srow[threadIdx.x * kMergeIPT + i]); m[i] = run; }
+      int32_t inc = run;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc = max(inc, y);
       }
+      if (lane == 31) s_wmax[w] = inc;
+      int32_t ex = __shfl_up_sync(0xffffffffu, inc, 1);
+      if (lane == 0) ex = -1;
+      __syncthreads();
+      for (int ww = 0; ww < w; ++ww) ex = max(ex, s_wmax[ww]);
+#pragma unroll
+      for (int i = 0; i < kMergeIPT; ++i) srow[threadIdx.x * kMergeIPT + i] = max(ex, m[i]);
+    }
+    __syncthreads();
+    // generic pointers (shared or global) indexed by the global key index: one code path
+    const uint64_t* A = sa ? sadd - ka0 : a.add;
+    const uint64_t* D = sd ? sdel - kd0 : a.del;
+#pragma unroll 2
+    for (int i = 0; i < kMergeIPT; ++i) {
+      const int k = threadIdx.x + i * 256;
+      if (k >= n) break;
+      const int64_t j = e0 + k;
+      int32_t v, orp, nrp;
+      int4 t;
+      if (cached) {
+        const int32_t r = srow[k];
+        v = rlo + r; orp = srp[r]; nrp = snrp[r]; t = stc[r];
+      } else {
+        v = row_of(a.orowptr, rlo, rhi, j);
+        orp = __ldg(a.orowptr + v); nrp = __ldg(a.nrowptr + v); t = __ldg(a.touch + v);
+      }
+      int64_t pos = (int64_t)nrp + (j - orp);
+      if (t.y != t.x || t.w != t.z) {
+        const uint64_t key = ((uint64_t)v << a.nb) | (uint64_t)scol[k];
+        // #adds / #dels of the row below key: a row has ~1 of each on average, so short
+        // ranges are counted directly; long ones (hubs) are searched
+        int32_t na_below = 0, nd_below = 0;
+        bool del = false;
+        if (t.y - t.x <= 4) {
+          for (int32_t q = t.x; q < t.y; ++q) na_below += A[q] < key;
+        } else {
+          int32_t lo = t.x, hi = t.y;
+          while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (A[mid] < key) lo = mid + 1; else hi = mid; }
+          na_below = lo - t.x;
+        }
+        if (t.w - t.z <= 4) {
+          for (int32_t q = t.z; q < t.w; ++q) { const uint64_t x = D[q]; nd_below += x < key; del |= x == key; }
+        } else {
+          int32_t lo = t.z, hi = t.w;
+          while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (D[mid] < key) lo = mid + 1; else hi = mid; }
+          nd_below = lo - t.z;
+          del = lo < t.w && D[lo] == key;
+        }
+        if (del) pos = -1;                              // deleted
+        else pos += na_below - nd_below;
+      }
+      if (a.emap_out) a.emap_out[j] = (int32_t)pos;
+      if (pos < 0) continue;
+      a.ncol[pos] = scol[k];
+      if (a.eid_new) a.eid_new[pos] = __ldg(a.emap_in + __ldcs(a.eid_old + j));
     }
   } else {                                            // added edges
     const uint64_t mask = (uint64_t(1) << a.nb) - 1;
-    const int64_t nthr = (int64_t)(gridDim.x - a.old_tiles) * blockDim.x;
-    for (int64_t i = (int64_t)(blockIdx.x - a.old_tiles) * blockDim.x + threadIdx.x; i < a.nadd; i += nthr) {
+    const int64_t nthr = add_blocks * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.nadd; i += nthr) {
       const uint64_t key = a.add[i];
       const int32_t v = (int32_t)(key >> a.nb), c = (int32_t)(key & mask);
       const int4 t = __ldg(a.touch + v);
@@ -646,6 +739,7 @@ stg_status ids_ws_reserve(BuildWs& ws, int32_t V, int64_t cap, cudaStream_t s) {
     STG_CUDA(cudaMemsetAsync(ws.lb_status.p, 0, sizeof(uint64_t) * ws.lb_status.n, s));
   }
   STG_TRY(ws.lb_ticket.alloc(1, s));
+  STG_TRY(ws.merge_rows.alloc((size_t)ceil_div(cap > 0 ? cap : 1, kMergeTile) + 1, s));
   return STG_OK;
 }
 
@@ -730,6 +824,8 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
     a.gin = dst.gin_deg.p; a.gout = dst.gout_deg.p; a.dgl_both = dst.dgl_both;
     a.norm_src = dst.norm_src.p; a.norm_dst = dst.norm_dst.p;
   }
+  a.orowptr = in_dir ? src.in_rowptr.p : src.out_rowptr.p;
+  a.tile_row = ws.merge_rows.p;
   STG_CUDA(cudaMemsetAsync(ws.lb_ticket.p, 0, sizeof(uint32_t), s));
   k_rowscan<true><<<ntiles, kRowThreads, 0, s>>>(a);
   count_launch();
@@ -745,6 +841,7 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
   m.old_tiles = ceil_div(src.E, kMergeTile);
   m.emap_out = emap_out; m.emap_in = emap_in; m.eid_old = eid_old; m.eid_new = eid_new;
   m.in_rowptr_new = in_rowptr_new; m.in_col_new = in_col_new;
+  m.tile_row = ws.merge_rows.p;
   const int64_t add_blocks = d.nadd > 0 ? std::min<int64_t>(ceil_div(d.nadd, 256), 4 * 148) : 0;
   if (m.old_tiles + add_blocks > 0) {
     k_merge2<<<(unsigned)(m.old_tiles + add_blocks), 256, 0, s>>>(m);

@@ -431,6 +431,14 @@ __device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, int c0, int
                "r"(c0), "r"(r0), "r"(z), "r"(smem_u32(src))
                : "memory");
 }
+// out[box] += smem box (fp32 add in the memory system; one add per element, so the
+// result is out + v rounded once, as a load-add-store would give)
+__device__ __forceinline__ void tma_reduce_add_2d(const CUtensorMap* map, int c0, int r0, const void* src) {
+  asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.tile.bulk_group [%0, {%1, %2}], [%3];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(c0), "r"(r0), "r"(smem_u32(src))
+               : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
@@ -440,7 +448,7 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 // bytes, 1024-aligned); `slot` alternates 0/1 across calls of this warp.
 // Writes v*s (this lane's row) into the free buffer, then lane 0 issues the
 // TMA store of box (c0, r0).  Rows past the tensor end are clipped by TMA.
-template <int NCOL>
+template <int NCOL, bool ADD = false>
 __device__ __forceinline__ void warp_box_store(unsigned char* buf0, int& slot, const float (&v)[NCOL], float s,
                                                const CUtensorMap* map, int c0, int r0) {
   constexpr int BYTES = 32 * NCOL * 4;
@@ -458,7 +466,8 @@ __device__ __forceinline__ void warp_box_store(unsigned char* buf0, int& slot, c
   fence_proxy_async();
   __syncwarp();
   if (lane == 0) {
-    tma_store_2d(map, c0, r0, buf);
+    if constexpr (ADD) tma_reduce_add_2d(map, c0, r0, buf);
+    else tma_store_2d(map, c0, r0, buf);
     bulk_commit();
   }
   slot ^= 1;

@@ -1829,8 +1829,13 @@ static stg_status atb2_stages(const CUtensorMap* m, const CUtensorMap& ones, con
   return atb2_launch<NB, RT, 2>(m, ones, sp, nb, s);
 }
 
-static stg_status atb2_dispatch(int NB, const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& sp, int* nb,
+static stg_status atb2_dispatch(int NB, const CUtensorMap* m, const CUtensorMap& ones, const AtbSpec2& spec, int* nb,
                                 cudaStream_t s) {
+  // an M = 128 A operand spans 4 consecutive box slots from a_first: pad the stage with
+  // empty slots (src_map -1: never loaded, hi and lo stay 0) until they exist
+  AtbSpec2 sp = spec;
+  while (sp.nsa + NB < sp.a_first[sp.na - 1] + 4 && sp.nsa < 8) sp.src_map[sp.nsa++] = -1;
+  if (sp.nsa + NB < sp.a_first[sp.na - 1] + 4) return fail(STG_ERR_INVALID_ARG, "atb2: %d A slots", sp.nsa);
   switch (NB) {
     case 1: return atb2_stages<1>(m, ones, sp, nb, s);
     case 2: return atb2_stages<2>(m, ones, sp, nb, s);
@@ -2384,6 +2389,149 @@ __global__ void __launch_bounds__(kTcThreads) k_tc_catmm(int V, const float* __r
   if ((threadIdx.x >> 5) == 0) tc::tmem_free(tm, NC);
 }
 
+// A 128-row tile of [A1 | A2] (K1 + K2 <= 128 columns, K1 % 4 == 0) as float4 chunks
+// of the concatenated row, nthr threads, at most 16 chunks per thread: load into
+// registers, then split into hi / lo at K-major column 4j.  Rows >= nvalid are 0.
+__device__ __forceinline__ void cat_load(float4 (&v)[16], const float* __restrict__ A1, int64_t ld1, int K1,
+                                         const float* __restrict__ A2, int64_t ld2, int K2, int nvalid, int tid,
+                                         int nthr) {
+  const int lane = tid & 31, warp = tid >> 5, nw = nthr >> 5;
+  const int nj = (K1 + K2) / 4, njb = (nj + 3) / 4, total = 16 * njb, j1 = K1 / 4;
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {
+    const int it = warp + i * nw;
+    const int r = (it % 16) * 8 + (lane & 7);
+    const int j = (it / 16) * 4 + (lane >> 3);
+    v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (it < total && j < nj && r < nvalid)
+      v[i] = __ldg(reinterpret_cast<const float4*>(j < j1 ? A1 + (int64_t)r * ld1 + 4 * j
+                                                          : A2 + (int64_t)r * ld2 + 4 * (j - j1)));
+  }
+}
+__device__ __forceinline__ void cat_store(const float4 (&v)[16], unsigned char* hi, unsigned char* lo, int K, int Kp,
+                                          int tid, int nthr) {
+  const int lane = tid & 31, warp = tid >> 5, nw = nthr >> 5;
+  const int nj = K / 4, njb = (nj + 3) / 4, total = 16 * njb;
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {
+    const int it = warp + i * nw;
+    const int r = (it % 16) * 8 + (lane & 7);
+    const int j = (it / 16) * 4 + (lane >> 3);
+    if (it < total && j < nj) tc::st_split4(hi, lo, r, j, Kp, v[i]);
+  }
+}
+
+// The same product, warp-specialised like k_tc_xw_pipe:
+//   warps 4-11  producers: NST groups of 256/NST threads (NST = ring slots, 2 when
+//               shared memory allows, else 1) take alternate tiles; a group holds its
+//               next tile in registers while it waits for its slot, then splits it;
+//   warp 12     one lane issues the 3xTF32 MMAs into one of two TMEM accumulators;
+//   warps 0-3   epilogue: tcgen05.ld, row scale, per-warp TMA box store, or a TMA
+//               reduce-add into out when accumulating.
+template <int N, int NST>
+__global__ void __launch_bounds__(kXwThreads, 1) k_tc_catmm_pipe(int V, const float* __restrict__ A1, int K1,
+                                                                 int64_t ld1, const float* __restrict__ A2, int K2,
+                                                                 int64_t ld2, int Kp,
+                                                                 const float* __restrict__ W, int64_t sk, int64_t sn,
+                                                                 const float* __restrict__ rs,
+                                                                 const __grid_constant__ CUtensorMap tmO,
+                                                                 int accumulate) {
+  extern __shared__ __align__(128) unsigned char sm[];
+  __shared__ uint64_t full[NST], empty[NST], tfull[2], tempty[2];
+  __shared__ uint32_t tslot;
+  constexpr uint32_t NC = N <= 32 ? 32 : 64;
+  constexpr int NT = 256 / NST;                      // producer threads per group
+  const int ABYTES = 128 * Kp * 4;
+  unsigned char* bhi = sm;
+  unsigned char* blo = bhi + N * Kp * 4;
+  unsigned char* abase = blo + N * Kp * 4;
+  auto ahi = [&](int st) { return abase + (size_t)st * 2 * ABYTES; };
+  auto alo = [&](int st) { return abase + (size_t)st * 2 * ABYTES + ABYTES; };
+  const int warp = threadIdx.x >> 5;
+  const int K = K1 + K2;
+  for (int e = threadIdx.x; e < N * Kp; e += blockDim.x) {            // B = Wᵀ (strided slice), zero past K
+    const int n = e / Kp, k = e % Kp;
+    const float v = k < K ? W[(int64_t)k * sk + (int64_t)n * sn] : 0.0f;
+    const float h = tc::tf32_hi(v);
+    *reinterpret_cast<float*>(bhi + tc::kmaj_off(n, k, Kp)) = h;
+    *reinterpret_cast<float*>(blo + tc::kmaj_off(n, k, Kp)) = v - h;
+  }
+  for (int i = threadIdx.x; i < NST * 2 * 128 * Kp; i += blockDim.x)   // zero the K padding once
+    reinterpret_cast<float*>(abase)[i] = 0.f;
+  if (warp == 12) tc::tmem_alloc(&tslot, 2 * NC);
+  if (threadIdx.x == 0) {
+    for (int st = 0; st < NST; ++st) { tc::mbar_init(&full[st], NT); tc::mbar_init(&empty[st], 1); }
+    for (int b = 0; b < 2; ++b) { tc::mbar_init(&tfull[b], 1); tc::mbar_init(&tempty[b], 128); }
+    tc::fence_mbar_init();
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tm = tslot;
+  const int ntiles = (V + 127) / 128;
+  if (warp >= 4 && warp < 12) {                      // ---- producers (group = slot)
+    const int grp = (warp - 4) / (NT / 32), tid = threadIdx.x - 128 - NT * grp;
+    float4 v[16];
+    int tile = blockIdx.x + grp * gridDim.x;
+    auto load = [&](int t) {
+      cat_load(v, A1 + (int64_t)t * 128 * ld1, ld1, K1, A2 + (int64_t)t * 128 * ld2, ld2, K2, V - t * 128, tid, NT);
+    };
+    if (tile < ntiles) load(tile);
+    for (int k = 0; tile < ntiles; tile += NST * gridDim.x, ++k) {
+      if (k > 0) tc::mbar_wait(&empty[grp], (k - 1) & 1);
+      cat_store(v, ahi(grp), alo(grp), K, Kp, tid, NT);
+      tc::fence_proxy_async();
+      tc::mbar_arrive(&full[grp]);
+      const int nt = tile + NST * gridDim.x;
+      if (nt < ntiles) load(nt);
+    }
+  } else if (warp == 12) {                           // ---- MMA issuer
+    if ((threadIdx.x & 31) == 0) {
+      const uint32_t idesc = tc::idesc_tf32(128, N, 0, 0);
+      int i = 0;
+      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+        const int st = i % NST, ks = i / NST;        // tile i: ring slot i % NST, accumulator i % 2
+        const int b = i & 1, kb = i >> 1;
+        tc::mbar_wait(&full[st], ks & 1);
+        if (kb > 0) tc::mbar_wait(&tempty[b], (kb - 1) & 1);
+        tc::fence_after();
+        mma_seg(tm + b * NC, tc::smem_u32(ahi(st)), tc::smem_u32(alo(st)), Kp, 0, tc::smem_u32(bhi),
+                tc::smem_u32(blo), Kp, 0, Kp, idesc, true);
+        tc::commit(&empty[st]);
+        tc::commit(&tfull[b]);
+      }
+    }
+  } else if (warp < 4) {                             // ---- epilogue, TMA box stores / reduce-adds
+    unsigned char* obuf = reinterpret_cast<unsigned char*>(
+        (reinterpret_cast<uintptr_t>(abase + (size_t)NST * 2 * ABYTES) + 1023) & ~uintptr_t(1023)) + warp * 4096;
+    int oslot = 0;
+    int i = 0;
+    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+      const int b = i & 1, kb = i >> 1;
+      const int row = tile * 128 + threadIdx.x;
+      const float sc = (rs && row < V) ? __ldg(rs + row) : 1.0f;
+      tc::mbar_wait(&tfull[b], kb & 1);
+      tc::fence_after();
+      const int wr0 = tile * 128 + warp * 32;
+#pragma unroll
+      for (int c0 = 0; c0 < N; c0 += 16) {
+        float v[16];
+        tmem_row_load<16>(tm + b * NC, c0, v);
+        if (c0 + 16 >= N) {                          // accumulator b fully read: release it early
+          tc::fence_before();
+          tc::mbar_arrive(&tempty[b]);
+        }
+        if (accumulate) tc::warp_box_store<16, true>(obuf, oslot, v, sc, &tmO, c0, wr0);
+        else tc::warp_box_store<16>(obuf, oslot, v, sc, &tmO, c0, wr0);
+      }
+    }
+    if ((threadIdx.x & 31) == 0) tc::bulk_wait_all();  // output boxes written before the CTA exits
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 12) tc::tmem_free(tm, 2 * NC);
+}
+
 // grad[k][n] += tot[row(k)][n]; rows 0..K1 hold A1's features, A2's start at hoff
 __global__ void k_cat_scatter(int K1, int K2, int N, int hoff, int Np, const float* __restrict__ tot,
                               float* __restrict__ grad) {
@@ -2406,8 +2554,36 @@ stg_status tc_catmm(int V, const float* A1, int K1, int64_t ld1, const float* A2
                     cudaStream_t s) {
   if (V <= 0) return STG_OK;
   const int Kp = (K1 + K2 + 7) / 8 * 8;
-  const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)2 * 128 * Kp * 4;
   const int ntiles = (V + 127) / 128;
+  if (K1 + K2 <= 128 && N % 16 == 0 && ((uintptr_t)out) % 16 == 0) {   // warp-specialised pipeline
+    const auto need = [&](int nst) { return (size_t)2 * N * Kp * 4 + (size_t)nst * 2 * 128 * Kp * 4 + 1024 + 4 * 4096; };
+    const int nst = need(2) <= 227 * 1024 ? 2 : (need(1) <= 227 * 1024 ? 1 : 0);
+    if (nst) {
+      const size_t smem = need(nst);
+      CUtensorMap tmO;
+      STG_TRY(make_tmap_f32_store(&tmO, out, (uint64_t)V, (uint64_t)N, (uint64_t)ldo, 16, 32));
+      const int nb = std::min(ntiles, num_sms());
+#define STG_CATMM_PIPE(NN, NS)                                                                                   \
+  do {                                                                                                           \
+    STG_TRY(prep(k_tc_catmm_pipe<NN, NS>, smem));                                                                \
+    k_tc_catmm_pipe<NN, NS><<<nb, kXwThreads, smem, s>>>(V, A1, K1, ld1, A2, K2, ld2, Kp, W, sk, sn, rs, tmO,    \
+                                                         accumulate ? 1 : 0);                                    \
+  } while (0)
+      if (nst == 2) {
+        if (N == 16) STG_CATMM_PIPE(16, 2);
+        else if (N == 32) STG_CATMM_PIPE(32, 2);
+        else STG_CATMM_PIPE(64, 2);
+      } else {
+        if (N == 16) STG_CATMM_PIPE(16, 1);
+        else if (N == 32) STG_CATMM_PIPE(32, 1);
+        else STG_CATMM_PIPE(64, 1);
+      }
+#undef STG_CATMM_PIPE
+      count_launch();
+      return check_launch("tc_catmm_pipe");
+    }
+  }
+  const size_t smem = (size_t)2 * N * Kp * 4 + (size_t)2 * 128 * Kp * 4;
 #define STG_CATMM(NN)                                                                                           \
   do {                                                                                                          \
     STG_TRY(prep(k_tc_catmm<NN>, smem));                                                                        \

@@ -71,10 +71,17 @@ def test_tgcn2_zero_parameters_halve_state(stg):
     assert torch.equal(Hn, 0.5 * Hp)
 
 
-def test_tgcn2_sequence_over_dtdg(stg):
+@pytest.mark.parametrize("name", ["C5s", "C4"])
+def test_tgcn2_sequence_over_dtdg(stg, name):
     """Algorithm 1 with the original T-GCN cell over DTDG snapshots (Get-Graph forward,
-    Get-Backward-Graph in LIFO order), surrogate head, BPTT."""
-    cfg = gen.CONFIGS["C5s"]
+    Get-Backward-Graph in LIFO order), BPTT.  The loss goes through the surrogate head;
+    the upstream gradient of step t is a fixed random G_t plus the gradient carried back
+    from step t+1.  (The head's ReLU is a decision: an H entry within the fp32 error of 0
+    flips its mask between fp32 and fp64 and moves a whole row's contribution to dW by
+    O(1/√rows) normwise -- measured 5e-4 on C5s -- so the gradient chain is driven by G_t,
+    not by the head; the head's gradient has its own element-wise tests.)  C4 (F = 8)
+    runs the Σ AᵀB reductions with padded operand slots at 2 CTAs per SM."""
+    cfg = gen.CONFIGS[name]
     dd = gen.dtdg(cfg)
     V, F, H, S = cfg.V, cfg.F, cfg.H, 3
     dg = stg.stg_dtdg_create(dd.V, dd.T, dd.src0, dd.dst0, dd.add_off, dd.add_src, dd.add_dst, dd.del_off,
@@ -83,11 +90,12 @@ def test_tgcn2_sequence_over_dtdg(stg):
     pg = {k: torch.from_numpy(v).cuda() for k, v in p.items()}
     Xs = [gen.features(cfg, t) for t in range(S)]
     Ys = [gen.labels(cfg, t) for t in range(S)]
+    Gs = [gen.uniform_pm1(cfg.seed, 80 + t, V * H).reshape(V, H) for t in range(S)]
     Xg = [torch.from_numpy(x).cuda() for x in Xs]
     Yg = [torch.from_numpy(y).cuda() for y in Ys]
     st = stg.stg_state_stack_create(S * V * 3 * H * 4 + (1 << 20))
     grads = _zero2(F, H)
-    dw, db, loss = torch.zeros(H, device="cuda"), torch.zeros(1, device="cuda"), torch.zeros(1, device="cuda")
+    loss = torch.zeros(1, device="cuda")
     Hs = [torch.zeros(V, H, device="cuda")]
     for t in range(S):
         v = stg.stg_dtdg_get_snapshot(dg, t)
@@ -96,16 +104,26 @@ def test_tgcn2_sequence_over_dtdg(stg):
     G = torch.zeros(V, H, device="cuda")
     for t in range(S - 1, -1, -1):
         v = stg.stg_dtdg_get_backward_snapshot(dg, t)
-        stg.stg_mse_head(Hs[t + 1], Yg[t], pg["w_o"], pg["b_o"], dH=G, accumulate=True, dw_o=dw, db_o=db)
-        G = stg.stg_tgcn2_step_backward(v, pg, Xg[t], G, grads, st)
+        G = stg.stg_tgcn2_step_backward(v, pg, Xg[t], G + torch.from_numpy(Gs[t]).cuda(), grads, st)
     torch.cuda.synchronize()
     sets = list(oracle.snapshot_sets_fold(dd, self_loops=True))
-    rl, rg, rH = oracle.train_sequence2([oracle.csr(V, sets[t]) for t in range(S)], p, Xs, Ys, np.zeros((V, H)))
+    graphs = [oracle.csr(V, sets[t]) for t in range(S)]
+    rg = oracle.zero_grads2(F, H)
+    Hc, fs, rl = np.zeros((V, H)), [], 0.0
+    for t in range(S):
+        f = oracle.tgcn2_fwd(graphs[t], p, Xs[t], Hc)
+        fs.append((Hc, f))
+        rl += oracle.mse_head(f["Hn"], Ys[t], p["w_o"], p["b_o"], {"w_o": np.zeros(H), "b_o": np.zeros(1)})[0]
+        Hc = f["Hn"]
+    rdH = np.zeros((V, H))
+    for t in range(S - 1, -1, -1):
+        Hp, f = fs[t]
+        rdH = oracle.tgcn2_bwd(graphs[t], p, Xs[t], Hp, f, rdH + Gs[t], rg)
     assert abs(loss.item() - rl) <= 1e-5 * abs(rl), (loss.item(), rl)
-    assert np.max(np.abs(Hs[-1].cpu().numpy() - rH)) <= 2e-5
-    gd = dict(grads)
-    gd["w_o"], gd["b_o"] = dw, db
-    _check(gd, rg, V * S, keys=("Wg", "bg", "Wc", "bc", "w_o", "b_o"))
+    assert np.max(np.abs(Hs[-1].cpu().numpy() - Hc)) <= 2e-5
+    _check(dict(grads), rg, V * S, keys=("Wg", "bg", "Wc", "bc"))
+    err = np.max(np.abs(G.cpu().numpy() - rdH)) / np.max(np.abs(rdH))
+    assert err <= 1e-4, err
 
 
 def test_tgcn2_sharded_peer_simulated_ranks(stg):
