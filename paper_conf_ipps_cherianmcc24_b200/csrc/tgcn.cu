@@ -584,86 +584,121 @@ __global__ void __launch_bounds__(kT) k_cat_atb(int32_t V, const float* __restri
   for (int e = threadIdx.x; e < K * N; e += kT) part[(int64_t)blockIdx.x * K * N + e] = sAcc[e];
 }
 
-// part[b][c] = Σ_{rows of block b} D[r, c] (fixed order: thread slices, then a fixed tree)
-__global__ void __launch_bounds__(kT) k_colsum_part(int32_t V, const float* __restrict__ D, int32_t N,
-                                                    float* __restrict__ part) {
-  __shared__ float red[kT];
-  const int slices = kT / N;                       // N divides kT (N = H or 2H, powers of two)
-  const int c = threadIdx.x % N, sl = threadIdx.x / N;
-  float acc = 0.0f;
-  if (sl < slices)
-    for (int64_t r = (int64_t)blockIdx.x * slices + sl; r < V; r += (int64_t)gridDim.x * slices)
-      acc += D[r * N + c];
-  red[threadIdx.x] = acc;
-  __syncthreads();
-  if (threadIdx.x < N) {
-    float t = 0.0f;
-    for (int q = 0; q < slices; ++q) t += red[q * N + threadIdx.x];
-    part[(int64_t)blockIdx.x * N + threadIdx.x] = t;
-  }
-}
-
 __device__ __forceinline__ float t2_sig(float a) { return 1.0f / (1.0f + expf(-a)); }
 
+// The cell's element-wise parts, one float4 of a row per thread (Q = H/4 float4 per
+// row; a thread's column group jq = index % Q is fixed under the grid stride, as
+// 256 % Q == 0).  The backward kernels also form the bias-gradient column sums of
+// what they produce (fixed order: the thread's rows in stride order, then the
+// block's threads of a column group in index order; k_reduce_part adds the blocks).
+__device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
+__device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+__device__ __forceinline__ float4 sig4(float4 a) { return make_float4(t2_sig(a.x), t2_sig(a.y), t2_sig(a.z), t2_sig(a.w)); }
+__device__ __forceinline__ float4 add4(float4 a, float4 b) { return make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w); }
+
 // r = σ(A[:, :H]), u = σ(A[:, H:]) -> RUC[:, 0:H), [H:2H); rH = r ⊙ Hp
-__global__ void k_t2_gates(int32_t V, int32_t H, const float* __restrict__ A, const float* __restrict__ Hp,
-                           float* __restrict__ RUC, float* __restrict__ rH) {
-  const int64_t n = (int64_t)V * H;
+template <int Q>
+__global__ void __launch_bounds__(256) k_t2_gates(int32_t V, const float* __restrict__ A, const float* __restrict__ Hp,
+                                                  float* __restrict__ RUC, float* __restrict__ rH) {
+  constexpr int H = 4 * Q;
+  const int64_t n = (int64_t)V * Q;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t v = i / H;
-    const int j = (int)(i % H);
-    const float r = t2_sig(A[v * 2 * H + j]), u = t2_sig(A[v * 2 * H + H + j]);
-    RUC[v * 3 * H + j] = r;
-    RUC[v * 3 * H + H + j] = u;
-    rH[i] = r * Hp[i];
+    const int64_t v = i / Q;
+    const int c = 4 * (int)(i % Q);
+    const float4 r = sig4(ld4(A + v * 2 * H + c)), u = sig4(ld4(A + v * 2 * H + H + c)), h = ld4(Hp + v * H + c);
+    st4(RUC + v * 3 * H + c, r);
+    st4(RUC + v * 3 * H + H + c, u);
+    st4(rH + v * H + c, make_float4(r.x * h.x, r.y * h.y, r.z * h.z, r.w * h.w));
   }
 }
 
 // c = tanh(A) -> RUC[:, 2H:3H);  H' = u ⊙ Hp + (1 − u) ⊙ c
-__global__ void k_t2_cand(int32_t V, int32_t H, const float* __restrict__ A, const float* __restrict__ Hp,
-                          float* __restrict__ RUC, float* __restrict__ Hn) {
-  const int64_t n = (int64_t)V * H;
+template <int Q>
+__global__ void __launch_bounds__(256) k_t2_cand(int32_t V, const float* __restrict__ A, const float* __restrict__ Hp,
+                                                 float* __restrict__ RUC, float* __restrict__ Hn) {
+  constexpr int H = 4 * Q;
+  const int64_t n = (int64_t)V * Q;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t v = i / H;
-    const int j = (int)(i % H);
-    const float c = tanhf(A[i]);
-    const float u = RUC[v * 3 * H + H + j];
-    RUC[v * 3 * H + 2 * H + j] = c;
-    Hn[i] = u * Hp[i] + (1.0f - u) * c;
+    const int64_t v = i / Q;
+    const int c = 4 * (int)(i % Q);
+    const float4 a = ld4(A + v * H + c), u = ld4(RUC + v * 3 * H + H + c), h = ld4(Hp + v * H + c);
+    const float4 cc = make_float4(tanhf(a.x), tanhf(a.y), tanhf(a.z), tanhf(a.w));
+    st4(RUC + v * 3 * H + 2 * H + c, cc);
+    st4(Hn + v * H + c, make_float4(u.x * h.x + (1.0f - u.x) * cc.x, u.y * h.y + (1.0f - u.y) * cc.y,
+                                    u.z * h.z + (1.0f - u.z) * cc.z, u.w * h.w + (1.0f - u.w) * cc.w));
   }
 }
 
-// du = G ⊙ (Hp − c); dAc = G ⊙ (1 − u) ⊙ (1 − c²); dHp = G ⊙ u; rH = r ⊙ Hp
-__global__ void k_t2_cand_bwd(int32_t V, int32_t H, const float* __restrict__ G, const float* __restrict__ Hp,
-                              const float* __restrict__ RUC, float* __restrict__ dAc, float* __restrict__ du,
-                              float* __restrict__ dHp, float* __restrict__ rH) {
-  const int64_t n = (int64_t)V * H;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t v = i / H;
-    const int j = (int)(i % H);
-    const float r = RUC[v * 3 * H + j], u = RUC[v * 3 * H + H + j], c = RUC[v * 3 * H + 2 * H + j];
-    const float g = G[i], h = Hp[i];
-    du[i] = g * (h - c);
-    dAc[i] = g * (1.0f - u) * (1.0f - c * c);
-    dHp[i] = g * u;
-    rH[i] = r * h;
+// block partial of NG float4 column groups per thread-column jq: part[b][g·H + 4jq ..]
+template <int Q, int NG>
+__device__ __forceinline__ void t2_block_colsum(const float4 (&acc)[NG], float* __restrict__ part) {
+  constexpr int H = 4 * Q;
+  __shared__ float4 red[NG][256];
+#pragma unroll
+  for (int g = 0; g < NG; ++g) red[g][threadIdx.x] = acc[g];
+  __syncthreads();
+  if (threadIdx.x < NG * Q) {
+    const int g = threadIdx.x / Q, jq = threadIdx.x % Q;
+    float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int sl = 0; sl < 256 / Q; ++sl) t = add4(t, red[g][sl * Q + jq]);
+    st4(part + (int64_t)blockIdx.x * NG * H + g * H + 4 * jq, t);
   }
 }
 
-// dr = d(rH) ⊙ Hp;  dHp += d(rH) ⊙ r;  dAg = [dr ⊙ r(1−r) | du ⊙ u(1−u)]
-__global__ void k_t2_gate_bwd(int32_t V, int32_t H, const float* __restrict__ drH, const float* __restrict__ Hp,
-                              const float* __restrict__ RUC, const float* __restrict__ du, float* __restrict__ dHp,
-                              float* __restrict__ dAg) {
-  const int64_t n = (int64_t)V * H;
+// du = G ⊙ (Hp − c); dAc = G ⊙ (1 − u) ⊙ (1 − c²); dHp = G ⊙ u; rH = r ⊙ Hp; part: colsum dAc
+template <int Q>
+__global__ void __launch_bounds__(256) k_t2_cand_bwd(int32_t V, const float* __restrict__ G,
+                                                     const float* __restrict__ Hp, const float* __restrict__ RUC,
+                                                     float* __restrict__ dAc, float* __restrict__ du,
+                                                     float* __restrict__ dHp, float* __restrict__ rH,
+                                                     float* __restrict__ part) {
+  constexpr int H = 4 * Q;
+  const int64_t n = (int64_t)V * Q;
+  float4 acc[1] = {make_float4(0.f, 0.f, 0.f, 0.f)};
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t v = i / H;
-    const int j = (int)(i % H);
-    const float r = RUC[v * 3 * H + j], u = RUC[v * 3 * H + H + j];
-    const float d = drH[i];
-    dHp[i] += d * r;
-    dAg[v * 2 * H + j] = d * Hp[i] * r * (1.0f - r);
-    dAg[v * 2 * H + H + j] = du[i] * u * (1.0f - u);
+    const int64_t v = i / Q;
+    const int c = 4 * (int)(i % Q);
+    const float* ruc = RUC + v * 3 * H + c;
+    const float4 r = ld4(ruc), u = ld4(ruc + H), cc = ld4(ruc + 2 * H);
+    const float4 g = ld4(G + v * H + c), h = ld4(Hp + v * H + c);
+    st4(du + v * H + c, make_float4(g.x * (h.x - cc.x), g.y * (h.y - cc.y), g.z * (h.z - cc.z), g.w * (h.w - cc.w)));
+    const float4 da = make_float4(g.x * (1.0f - u.x) * (1.0f - cc.x * cc.x), g.y * (1.0f - u.y) * (1.0f - cc.y * cc.y),
+                                  g.z * (1.0f - u.z) * (1.0f - cc.z * cc.z), g.w * (1.0f - u.w) * (1.0f - cc.w * cc.w));
+    st4(dAc + v * H + c, da);
+    acc[0] = add4(acc[0], da);
+    st4(dHp + v * H + c, make_float4(g.x * u.x, g.y * u.y, g.z * u.z, g.w * u.w));
+    st4(rH + v * H + c, make_float4(r.x * h.x, r.y * h.y, r.z * h.z, r.w * h.w));
   }
+  t2_block_colsum<Q, 1>(acc, part);
+}
+
+// dr = d(rH) ⊙ Hp;  dHp += d(rH) ⊙ r;  dAg = [dr ⊙ r(1−r) | du ⊙ u(1−u)]; part: colsum dAg
+template <int Q>
+__global__ void __launch_bounds__(256) k_t2_gate_bwd(int32_t V, const float* __restrict__ drH,
+                                                     const float* __restrict__ Hp, const float* __restrict__ RUC,
+                                                     const float* __restrict__ du, float* __restrict__ dHp,
+                                                     float* __restrict__ dAg, float* __restrict__ part) {
+  constexpr int H = 4 * Q;
+  const int64_t n = (int64_t)V * Q;
+  float4 acc[2] = {make_float4(0.f, 0.f, 0.f, 0.f), make_float4(0.f, 0.f, 0.f, 0.f)};
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = i / Q;
+    const int c = 4 * (int)(i % Q);
+    const float4 r = ld4(RUC + v * 3 * H + c), u = ld4(RUC + v * 3 * H + H + c);
+    const float4 d = ld4(drH + v * H + c), h = ld4(Hp + v * H + c), w = ld4(du + v * H + c);
+    float4 o = ld4(dHp + v * H + c);
+    o = make_float4(o.x + d.x * r.x, o.y + d.y * r.y, o.z + d.z * r.z, o.w + d.w * r.w);
+    st4(dHp + v * H + c, o);
+    const float4 gr = make_float4(d.x * h.x * r.x * (1.0f - r.x), d.y * h.y * r.y * (1.0f - r.y),
+                                  d.z * h.z * r.z * (1.0f - r.z), d.w * h.w * r.w * (1.0f - r.w));
+    const float4 gu = make_float4(w.x * u.x * (1.0f - u.x), w.y * u.y * (1.0f - u.y), w.z * u.z * (1.0f - u.z),
+                                  w.w * u.w * (1.0f - u.w));
+    st4(dAg + v * 2 * H + c, gr);
+    st4(dAg + v * 2 * H + H + c, gu);
+    acc[0] = add4(acc[0], gr);
+    acc[1] = add4(acc[1], gu);
+  }
+  t2_block_colsum<Q, 2>(acc, part);
 }
 
 int grid_blocks(const void* fn, size_t smem, int64_t tiles) {
@@ -1135,17 +1170,88 @@ static stg_status t2_atb(int32_t V, const float* A1, int32_t K1, const float* A2
   return check_launch("tgcn2 atb");
 }
 
-static stg_status t2_colsum(int32_t V, const float* D, int32_t N, float* grad, TgcnWs& ws, cudaStream_t s) {
-  if (V == 0) return STG_OK;
-  const int nb = (int)std::min<int64_t>((V + 63) / 64, (int64_t)num_sms() * 4);
-  STG_TRY(ws.t2part.alloc((size_t)nb * N));
-  k_colsum_part<<<nb, kT, 0, s>>>(V, D, N, ws.t2part.p);
-  k_reduce_part<<<(N + 255) / 256, 256, 0, s>>>(ws.t2part.p, nb, N, grad, N, nullptr, 0, nullptr);
-  count_launch(2);
-  return check_launch("tgcn2 colsum");
+// out[e] += Σ_b part[b][e] for many blocks b and few columns e: a block owns 32 columns,
+// warp w sums the blocks b ≡ w (mod 8) in ascending order (loads unrolled 8 deep),
+// then one lane adds the 8 warp sums in order (fixed order, run to run).
+__global__ void __launch_bounds__(256) k_reduce_part_wide(const float* __restrict__ part, int32_t nb, int32_t n,
+                                                          float* __restrict__ out) {
+  __shared__ float ws[8][33];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int e = blockIdx.x * 32 + lane;
+  float t = 0.0f;
+  if (e < n) {
+    int b = w;
+    for (; b + 56 < nb; b += 64) {
+      float x[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) x[k] = __ldg(part + (int64_t)(b + 8 * k) * n + e);
+#pragma unroll
+      for (int k = 0; k < 8; ++k) t += x[k];
+    }
+    for (; b < nb; b += 8) t += __ldg(part + (int64_t)b * n + e);
+  }
+  ws[w][lane] = t;
+  __syncthreads();
+  if (w == 0 && e < n) {
+    float tot = 0.0f;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) tot += ws[k][lane];
+    out[e] += tot;
+  }
 }
 
-static unsigned t2_grid(int64_t n) { return (unsigned)std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 16); }
+// element-wise parts of the cell (H = 4Q, Q in {1, 2, 4, 8, 16})
+static unsigned t2_blocks(int64_t n4) {
+  return (unsigned)std::min<int64_t>(std::max<int64_t>((n4 + 255) / 256, 1), (int64_t)num_sms() * 8);
+}
+#define STG_T2_LAUNCH(H, KERNEL, NB, ...)                                 \
+  switch (H) {                                                            \
+    case 4: KERNEL<1><<<NB, 256, 0, s>>>(__VA_ARGS__); break;             \
+    case 8: KERNEL<2><<<NB, 256, 0, s>>>(__VA_ARGS__); break;             \
+    case 16: KERNEL<4><<<NB, 256, 0, s>>>(__VA_ARGS__); break;            \
+    case 32: KERNEL<8><<<NB, 256, 0, s>>>(__VA_ARGS__); break;            \
+    default: KERNEL<16><<<NB, 256, 0, s>>>(__VA_ARGS__); break;           \
+  }
+
+static stg_status t2_gates(int32_t V, int32_t H, const float* A, const float* Hp, float* RUC, float* rH,
+                           cudaStream_t s) {
+  if (V == 0) return STG_OK;
+  STG_T2_LAUNCH(H, k_t2_gates, t2_blocks((int64_t)V * H / 4), V, A, Hp, RUC, rH);
+  count_launch();
+  return check_launch("tgcn2 gates");
+}
+
+static stg_status t2_cand(int32_t V, int32_t H, const float* A, const float* Hp, float* RUC, float* Hn,
+                          cudaStream_t s) {
+  if (V == 0) return STG_OK;
+  STG_T2_LAUNCH(H, k_t2_cand, t2_blocks((int64_t)V * H / 4), V, A, Hp, RUC, Hn);
+  count_launch();
+  return check_launch("tgcn2 candidate");
+}
+
+// ... and their gradients, with db_c += Σ_rows dA_c and db_g += Σ_rows dA_g
+static stg_status t2_cand_bwd(int32_t V, int32_t H, const float* G, const float* Hp, const float* RUC, float* dAc,
+                              float* du, float* dHp, float* rH, float* gbc, TgcnWs& ws, cudaStream_t s) {
+  if (V == 0) return STG_OK;
+  const unsigned nb = t2_blocks((int64_t)V * H / 4);
+  STG_TRY(ws.t2part.alloc((size_t)nb * H));
+  STG_T2_LAUNCH(H, k_t2_cand_bwd, nb, V, G, Hp, RUC, dAc, du, dHp, rH, ws.t2part.p);
+  k_reduce_part_wide<<<(H + 31) / 32, 256, 0, s>>>(ws.t2part.p, (int32_t)nb, H, gbc);
+  count_launch(2);
+  return check_launch("tgcn2 candidate backward");
+}
+
+static stg_status t2_gate_bwd(int32_t V, int32_t H, const float* drH, const float* Hp, const float* RUC,
+                              const float* du, float* dHp, float* dAg, float* gbg, TgcnWs& ws, cudaStream_t s) {
+  if (V == 0) return STG_OK;
+  const unsigned nb = t2_blocks((int64_t)V * H / 4);
+  STG_TRY(ws.t2part.alloc((size_t)nb * 2 * H));
+  STG_T2_LAUNCH(H, k_t2_gate_bwd, nb, V, drH, Hp, RUC, du, dHp, dAg, ws.t2part.p);
+  k_reduce_part_wide<<<(2 * H + 31) / 32, 256, 0, s>>>(ws.t2part.p, (int32_t)nb, 2 * H, gbg);
+  count_launch(2);
+  return check_launch("tgcn2 gate backward");
+}
+#undef STG_T2_LAUNCH
 
 static stg_status check_tgcn2(const stg_csr_view* g, const stg_tgcn2_params* p) {
   if (!g || !p || !p->Wg || !p->bg || !p->Wc || !p->bc) return fail(STG_ERR_INVALID_ARG, "tgcn2: NULL argument");
@@ -1188,13 +1294,11 @@ stg_status stg_tgcn2_step(const stg_csr_view* g, const stg_tgcn2_params* p, cons
   // gates: A = Â([X, H]·Wg) + bg  (P'-style: rows pre-scaled by n_src, n_dst per output row)
   STG_TRY(t2_mm(V, X, F, F, H_prev, H, H, p->Wg, H2, 1, H2, g->norm_src, Z, H2, false, s));
   STG_TRY(aggregate_launch(g, 0, H2, Z, H2, A, H2, g->norm_dst, nullptr, p->bg, s));
-  k_t2_gates<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, A, H_prev, RUC, rH);
-  count_launch();
+  STG_TRY(t2_gates(V, H, A, H_prev, RUC, rH, s));
   // candidate: A = Â([X, r⊙H]·Wc) + bc
   STG_TRY(t2_mm(V, X, F, F, rH, H, H, p->Wc, H, 1, H, g->norm_src, Z, H, false, s));
   STG_TRY(aggregate_launch(g, 0, H, Z, H, A, H, g->norm_dst, nullptr, p->bc, s));
-  k_t2_cand<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, A, H_prev, RUC, H_next);
-  count_launch();
+  STG_TRY(t2_cand(V, H, A, H_prev, RUC, H_next, s));
   if (stack) {
     stack->entries.push_back(StackEntry{H_prev, RUC, V, H, need});
     stack->top += need;
@@ -1219,17 +1323,13 @@ stg_status stg_tgcn2_step_backward(const stg_csr_view* g, const stg_tgcn2_params
   const float* RUC = e.C;
   const float* Hp = e.Hp;
   float *dAg = ws.t2z.p, *Y = ws.t2a.p, *rH = ws.t2b.p, *D1 = ws.t2c.p, *du = ws.t2d.p;
-  k_t2_cand_bwd<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, dH_next, Hp, RUC, D1, du, dH_prev, rH);
-  count_launch();
+  STG_TRY(t2_cand_bwd(V, H, dH_next, Hp, RUC, D1, du, dH_prev, rH, grads->bc, ws, s));
   // candidate convolution: dbc, dY = Âᵀ dAc, dWc += [X, r⊙H]ᵀ dY, d(r⊙H) = dY · Wc[F:, :]ᵀ
-  STG_TRY(t2_colsum(V, D1, H, grads->bc, ws, s));
   STG_TRY(aggregate_launch(g, 1, H, D1, H, Y, H, g->norm_src, g->norm_dst, nullptr, s));
   STG_TRY(t2_atb(V, X, F, rH, H, Y, H, grads->Wc, ws, s));
   STG_TRY(t2_mm(V, Y, H, H, nullptr, 0, 0, p->Wc + (size_t)F * H, 1, H, H, nullptr, D1, H, false, s));
-  k_t2_gate_bwd<<<t2_grid((int64_t)V * H), 256, 0, s>>>(V, H, D1, Hp, RUC, du, dH_prev, dAg);
-  count_launch();
+  STG_TRY(t2_gate_bwd(V, H, D1, Hp, RUC, du, dH_prev, dAg, grads->bg, ws, s));
   // gate convolution: dbg, dY = Âᵀ dAg, dWg += [X, H]ᵀ dY, dH += dY · Wg[F:, :]ᵀ
-  STG_TRY(t2_colsum(V, dAg, H2, grads->bg, ws, s));
   STG_TRY(aggregate_launch(g, 1, H2, dAg, H2, Y, H2, g->norm_src, g->norm_dst, nullptr, s));
   STG_TRY(t2_atb(V, X, F, Hp, H, Y, H2, grads->Wg, ws, s));
   STG_TRY(t2_mm(V, Y, H2, H2, nullptr, 0, 0, p->Wg + (size_t)F * H2, 1, H2, H, nullptr, dH_prev, H, true, s));
@@ -1276,15 +1376,13 @@ stg_status stg_tgcn2_peer_fwd(int32_t phase, const stg_csr_view* g, const stg_tg
     if (R == 0) return STG_OK;
     if (!Z_loc) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_fwd: Z_loc is NULL");
     STG_TRY(aggregate_launch(g, 0, H2, nullptr, 0, A, H2, nd_loc, nullptr, p->bg, s, Z));
-    k_t2_gates<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, A, H_loc, RUC, ws.t2b.p);
-    count_launch();
+    STG_TRY(t2_gates(R, H, A, H_loc, RUC, ws.t2b.p, s));
     return t2_mm(R, X_loc, F, F, ws.t2b.p, H, H, p->Wc, H, 1, H, ns_loc, Z_loc, H, false, s);
   }
   if (!H_next && R > 0) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_fwd: H_next is NULL");
   if (R > 0) {                               // candidate from the gathered Zc, H_next; push
     STG_TRY(aggregate_launch(g, 0, H, nullptr, 0, A, H, nd_loc, nullptr, p->bc, s, Z));
-    k_t2_cand<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, A, H_loc, RUC, H_next);
-    count_launch();
+    STG_TRY(t2_cand(R, H, A, H_loc, RUC, H_next, s));
   }
   stack->entries.push_back(StackEntry{H_loc, RUC, R, H, need});
   stack->top += need;
@@ -1313,9 +1411,7 @@ stg_status stg_tgcn2_peer_bwd(int32_t phase, const stg_csr_view* g, const stg_tg
   if (phase == 0) {                          // candidate backward; partial dY_c of the local edges for all V
     if (!dH_next || !part_out) return fail(STG_ERR_INVALID_ARG, "stg_tgcn2_peer_bwd: NULL dH_next / part_out");
     if (R > 0) {
-      k_t2_cand_bwd<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, dH_next, Hp, RUC, D1, du, dH_prev, rH);
-      count_launch();
-      STG_TRY(t2_colsum(R, D1, H, grads->bc, ws, s));
+      STG_TRY(t2_cand_bwd(R, H, dH_next, Hp, RUC, D1, du, dH_prev, rH, grads->bc, ws, s));
     }
     return aggregate_launch(g, 1, H, D1, H, part_out, H, g->norm_src, nd_loc, nullptr, s);
   }
@@ -1327,9 +1423,7 @@ stg_status stg_tgcn2_peer_bwd(int32_t phase, const stg_csr_view* g, const stg_tg
       STG_TRY(stg_reduce_scatter_rows(world, bounds, parts, H, rank, H, Yl, H, stream));
       STG_TRY(t2_atb(R, X_loc, F, rH, H, Yl, H, grads->Wc, ws, s));
       STG_TRY(t2_mm(R, Yl, H, H, nullptr, 0, 0, p->Wc + (size_t)F * H, 1, H, H, nullptr, D1, H, false, s));
-      k_t2_gate_bwd<<<t2_grid((int64_t)R * H), 256, 0, s>>>(R, H, D1, Hp, RUC, du, dH_prev, dAg);
-      count_launch();
-      STG_TRY(t2_colsum(R, dAg, H2, grads->bg, ws, s));
+      STG_TRY(t2_gate_bwd(R, H, D1, Hp, RUC, du, dH_prev, dAg, grads->bg, ws, s));
     }
     (void)V;
     return aggregate_launch(g, 1, H2, dAg, H2, part_out, H2, g->norm_src, nd_loc, nullptr, s);

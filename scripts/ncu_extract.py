@@ -18,13 +18,15 @@ for rep in sorted(glob.glob(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/nc
     rows = list(csv.reader(io.StringIO(txt)))
     if len(rows) < 3:
         continue
-    h, u, v = rows[0], rows[1], rows[2]
-    d = {"Kernel Name": v[h.index("Kernel Name")]}
-    for k in KEYS:
-        if k in h:
-            d[k] = (v[h.index(k)] + " " + u[h.index(k)]).strip()
-    stalls = sorted(((h[i], float(v[i].replace(",", "") or 0)) for i in range(len(h))
-                     if "pcsamp_warps_issue_stalled" in h[i] and not h[i].endswith("not_issued")), key=lambda x: -x[1])
-    d["top_stalls"] = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): x for k, x in stalls[:5]}
-    out[rep.split("/")[-1]] = d
+    h, u = rows[0], rows[1]
+    for n, v in enumerate(rows[2:]):
+        d = {"Kernel Name": v[h.index("Kernel Name")]}
+        for k in KEYS:
+            if k in h:
+                d[k] = (v[h.index(k)] + " " + u[h.index(k)]).strip()
+        stalls = sorted(((h[i], float(v[i].replace(",", "") or 0)) for i in range(len(h))
+                         if "pcsamp_warps_issue_stalled" in h[i] and not h[i].endswith("not_issued")),
+                        key=lambda x: -x[1])
+        d["top_stalls"] = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): x for k, x in stalls[:5]}
+        out[rep.split("/")[-1] + ("" if n == 0 else "#%d" % n)] = d
 print(json.dumps(out, indent=1))
