@@ -563,27 +563,33 @@ struct MergeArgs {
 
 // Old edges: a CTA takes kMergeTile consecutive positions.  The tile's rows
 // (rows [tile_row[t], tile_row[t+1]], from k_rowscan) have their old / new row
-// pointers, touch marks and add / delete keys cached in shared memory; the row of
-// every position comes from a max-scan of the row-start marks; then every edge is
-// independent: new position = rowptr'[v] + (j - rowptr[v]) + #adds < key - #dels <
-// key (a binary search in the row's few cached keys), or -1 when deleted.
-// Consecutive threads take consecutive positions, so loads and stores coalesce.
+// pointers and touch marks cached in shared memory, and the row of every position
+// comes from a max-scan of the row-start marks.  Merge path: old edges, adds and
+// deletes are all sorted by key = (row << nb) | col, so each add / delete key of the
+// tile's rows finds its rank among the tile's old keys ONCE (binary search in shared
+// memory) and leaves a mark there; an inclusive scan of the marks gives, for every
+// position k, #adds < key_k and #dels < key_k over the tile's rows; subtracting the
+// earlier rows' counts (contiguous in the sorted lists, from the touch marks) leaves
+// the row-local counts of the shift
+//     new position = rowptr'[v] + (j − rowptr[v]) + #adds_v < key_j − #dels_v < key_j.
+// Consecutive threads take consecutive positions, so the stores coalesce.  Tiles
+// spanning more than kMergeRows rows (mean degree < 4) take a per-edge search path.
 constexpr int kMergeRows = 512;                  // rows whose rowptr / touch / new rowptr are cached
-constexpr int kMergeKeys = 512;                  // add / delete keys of the tile's rows cached in shared memory
 constexpr int kMergeIPT = kMergeTile / 256;      // positions per thread
 
 __global__ void __launch_bounds__(256) k_merge2(const MergeArgs a) {
-  __shared__ int32_t scol[kMergeTile], srow[kMergeTile];
+  __shared__ int32_t scol[kMergeTile], srow[kMergeTile], smark[kMergeTile];   // marks: adds | dels << 16
+  __shared__ uint8_t sdl[kMergeTile];                                          // old edge deleted
   __shared__ int32_t srp[kMergeRows + 1], snrp[kMergeRows];
   __shared__ int4 stc[kMergeRows];
-  __shared__ uint64_t sadd[kMergeKeys], sdel[kMergeKeys];
-  __shared__ int32_t s_lo, s_hi, s_rng[4], s_wmax[8];
+  __shared__ int32_t s_lo, s_hi, s_rng[4], s_wsum[8];
   const int64_t add_blocks = (int64_t)gridDim.x - a.old_tiles;      // added edges first: their searches
   const int64_t tile = (int64_t)blockIdx.x - add_blocks;             // overlap the tiles instead of trailing
   if (tile >= 0) {
     const int64_t e0 = tile * kMergeTile;
     const int64_t e1 = min(e0 + (int64_t)kMergeTile, a.E_old);
     const int n = (int)(e1 - e0);
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     if (threadIdx.x == 0) {                            // rows [s_lo, s_hi] hold the tile's edges
       s_lo = __ldg(a.tile_row + tile);
       s_hi = tile + 1 < a.old_tiles ? __ldg(a.tile_row + tile + 1) : a.V - 1;
@@ -594,10 +600,12 @@ __global__ void __launch_bounds__(256) k_merge2(const MergeArgs a) {
       const int k = threadIdx.x + i * 256;
       if (k < n) scol[k] = __ldcs(a.ocol + e0 + k);
       srow[k] = -1;
+      smark[k] = 0;
+      sdl[k] = 0;
     }
     __syncthreads();
     const int32_t rlo = s_lo, rhi = s_hi, nr = rhi - rlo + 1;
-    const bool cached = nr <= kMergeRows;              // (the tile's rows: ~kMergeTile / mean degree)
+    bool cached = nr <= kMergeRows;                    // (the tile's rows: ~kMergeTile / mean degree)
     if (cached) {
       int32_t a0 = INT32_MAX, a1 = INT32_MIN, d0 = INT32_MAX, d1 = INT32_MIN;
       for (int k = threadIdx.x; k <= nr; k += blockDim.x) {
@@ -619,14 +627,11 @@ __global__ void __launch_bounds__(256) k_merge2(const MergeArgs a) {
       }
     }
     __syncthreads();
-    // the tile rows' add / delete keys are contiguous ranges of the sorted lists
-    const int32_t ka0 = s_rng[0], kd0 = s_rng[2];
-    const int32_t na = s_rng[1] > ka0 ? s_rng[1] - ka0 : 0, nd = s_rng[3] > kd0 ? s_rng[3] - kd0 : 0;
-    const bool sa = cached && na <= kMergeKeys, sd = cached && nd <= kMergeKeys;
-    if (sa) for (int k = threadIdx.x; k < na; k += blockDim.x) sadd[k] = __ldg(a.add + ka0 + k);
-    if (sd) for (int k = threadIdx.x; k < nd; k += blockDim.x) sdel[k] = __ldg(a.del + kd0 + k);
-    if (cached) {                                      // inclusive max-scan of the marks: row of every position
-      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    // the tile rows' add / delete keys are the contiguous ranges [A0, A1), [D0, D1)
+    const int32_t A0 = s_rng[0], D0 = s_rng[2];
+    const int32_t na = s_rng[1] > A0 ? s_rng[1] - A0 : 0, nd = s_rng[3] > D0 ? s_rng[3] - D0 : 0;
+    cached = cached && na < 65536 && nd < 32768;       // 16-bit mark fields
+    if (cached) {                                      // inclusive max-scan of the row-start marks
       int32_t m[kMergeIPT];
       int32_t run = -1;
 #pragma unroll
@@ -637,56 +642,81 @@ __global__ void __launch_bounds__(256) k_merge2(const MergeArgs a) {
         const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
         if (lane >= o) inc = max(inc, y);
       }
-      if (lane == 31) s_wmax[w] = inc;
+      if (lane == 31) s_wsum[w] = inc;
       int32_t ex = __shfl_up_sync(0xffffffffu, inc, 1);
       if (lane == 0) ex = -1;
       __syncthreads();
-      for (int ww = 0; ww < w; ++ww) ex = max(ex, s_wmax[ww]);
+      for (int ww = 0; ww < w; ++ww) ex = max(ex, s_wsum[ww]);
 #pragma unroll
       for (int i = 0; i < kMergeIPT; ++i) srow[threadIdx.x * kMergeIPT + i] = max(ex, m[i]);
     }
     __syncthreads();
-    // generic pointers (shared or global) indexed by the global key index: one code path
-    const uint64_t* A = sa ? sadd - ka0 : a.add;
-    const uint64_t* D = sd ? sdel - kd0 : a.del;
+    if (cached) {                                      // ranks of the delta keys among the tile's old keys
+      const int nb = a.nb;
+      auto key_at = [&](int i) { return ((uint64_t)(rlo + srow[i]) << nb) | (uint64_t)(uint32_t)scol[i]; };
+      auto rank = [&](uint64_t key) {                  // # old tile keys < key
+        int lo = 0, hi = n;
+        while (lo < hi) { const int mid = (lo + hi) >> 1; if (key_at(mid) < key) lo = mid + 1; else hi = mid; }
+        return lo;
+      };
+      for (int i = threadIdx.x; i < na; i += blockDim.x) {   // add a counts for positions with key > a
+        const int r = rank(__ldg(a.add + A0 + i));
+        if (r < n) atomicAdd(&smark[r], 1);
+      }
+      for (int i = threadIdx.x; i < nd; i += blockDim.x) {   // delete d: removes its old edge, counts after it
+        const uint64_t key = __ldg(a.del + D0 + i);
+        const int r = rank(key);
+        if (r < n && key_at(r) == key) {
+          sdl[r] = 1;
+          if (r + 1 < n) atomicAdd(&smark[r + 1], 1 << 16);
+        } else if (r == 0) {
+          atomicAdd(&smark[0], 1 << 16);              // an old edge of the first row before the tile
+        }
+      }
+    }
+    __syncthreads();
+    if (cached) {                                      // inclusive scan of the packed marks
+      int32_t m[kMergeIPT];
+      int32_t run = 0;
+#pragma unroll
+      for (int i = 0; i < kMergeIPT; ++i) { run += smark[threadIdx.x * kMergeIPT + i]; m[i] = run; }
+      int32_t inc = run;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+      }
+      if (lane == 31) s_wsum[w] = inc;
+      int32_t ex = inc - run;
+      __syncthreads();
+      for (int ww = 0; ww < w; ++ww) ex += s_wsum[ww];
+#pragma unroll
+      for (int i = 0; i < kMergeIPT; ++i) smark[threadIdx.x * kMergeIPT + i] = ex + m[i];
+    }
+    __syncthreads();
 #pragma unroll 2
     for (int i = 0; i < kMergeIPT; ++i) {
       const int k = threadIdx.x + i * 256;
       if (k >= n) break;
       const int64_t j = e0 + k;
-      int32_t v, orp, nrp;
-      int4 t;
+      int64_t pos;
       if (cached) {
         const int32_t r = srow[k];
-        v = rlo + r; orp = srp[r]; nrp = snrp[r]; t = stc[r];
-      } else {
-        v = row_of(a.orowptr, rlo, rhi, j);
-        orp = __ldg(a.orowptr + v); nrp = __ldg(a.nrowptr + v); t = __ldg(a.touch + v);
-      }
-      int64_t pos = (int64_t)nrp + (j - orp);
-      if (t.y != t.x || t.w != t.z) {
-        const uint64_t key = ((uint64_t)v << a.nb) | (uint64_t)scol[k];
-        // #adds / #dels of the row below key: a row has ~1 of each on average, so short
-        // ranges are counted directly; long ones (hubs) are searched
-        int32_t na_below = 0, nd_below = 0;
-        bool del = false;
-        if (t.y - t.x <= 4) {
-          for (int32_t q = t.x; q < t.y; ++q) na_below += A[q] < key;
-        } else {
-          int32_t lo = t.x, hi = t.y;
-          while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (A[mid] < key) lo = mid + 1; else hi = mid; }
-          na_below = lo - t.x;
+        const int4 t = stc[r];
+        const int32_t mk = smark[k];
+        const int32_t adds = t.y > t.x ? (mk & 0xffff) - (t.x - A0) : 0;
+        const int32_t dels = t.w > t.z ? (mk >> 16) - (t.z - D0) : 0;
+        pos = sdl[k] ? -1 : (int64_t)snrp[r] + (j - srp[r]) + adds - dels;
+      } else {                                         // per-edge searches in the global lists
+        const int32_t v = row_of(a.orowptr, rlo, rhi, j);
+        const int4 t = __ldg(a.touch + v);
+        pos = (int64_t)__ldg(a.nrowptr + v) + (j - __ldg(a.orowptr + v));
+        if (t.y != t.x || t.w != t.z) {
+          const uint64_t key = ((uint64_t)v << a.nb) | (uint64_t)(uint32_t)scol[k];
+          const int64_t al = lb_u64(a.add, t.x, t.y, key), dl = lb_u64(a.del, t.z, t.w, key);
+          if (dl < t.w && __ldg(a.del + dl) == key) pos = -1;
+          else pos += (al - t.x) - (dl - t.z);
         }
-        if (t.w - t.z <= 4) {
-          for (int32_t q = t.z; q < t.w; ++q) { const uint64_t x = D[q]; nd_below += x < key; del |= x == key; }
-        } else {
-          int32_t lo = t.z, hi = t.w;
-          while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (D[mid] < key) lo = mid + 1; else hi = mid; }
-          nd_below = lo - t.z;
-          del = lo < t.w && D[lo] == key;
-        }
-        if (del) pos = -1;                              // deleted
-        else pos += na_below - nd_below;
       }
       if (a.emap_out) a.emap_out[j] = (int32_t)pos;
       if (pos < 0) continue;

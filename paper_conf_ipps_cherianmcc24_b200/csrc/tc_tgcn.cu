@@ -449,6 +449,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
   int i = 0;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
     const int b = i & 1, r0 = tile * 128;
+    const float yv = (HEAD && r0 + lr < V) ? __ldg(hd.y + r0 + lr) : 0.f;   // issued before the waits
     tc::mbar_wait(&full[b], (i >> 1) & 1);
     // raw tile -> tensor-memory A operands; this thread's half of H stays in registers
     float h[HH];
@@ -524,7 +525,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
         __syncthreads();
         const int row = r0 + lr;
         if (row < V) {
-          const float e = (s_dot[0][lr] + s_dot[1][lr] + bo) - __ldg(hd.y + row);
+          const float e = (s_dot[0][lr] + s_dot[1][lr] + bo) - yv;
           const float g = 2.0f * e * hd.inv_v;
           if (hf == 0) {
             lacc += (double)e * (double)e;
@@ -834,10 +835,14 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
   };
   uint32_t mph = 0;
   int i = 0;
+  float wog[HEADG ? HH : 1];                           // this thread's columns of w_o (head gradient)
+#pragma unroll
+  for (int j = 0; j < (HEADG ? HH : 1); ++j) wog[j] = HEADG ? __ldg(w_o + c0 + j) : 0.f;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
     const int r0 = tile * 128, wr0 = r0 + q * 32;
     const int row = r0 + lr;
     const float nd = row < V ? (ndst ? __ldg(ndst + row) : 1.0f) : 0.f;   // (NULL: dC unscaled, aggregate-first)
+    const float2 hv = (HEADG && row < V) ? __ldg(hg + row) : make_float2(0.f, 0.f);   // issued before the waits
     tc::mbar_wait(&full, i & 1);
     float h[HH], g[HH];
     {
@@ -853,11 +858,10 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
         g[4 * qq] = x.x; g[4 * qq + 1] = x.y; g[4 * qq + 2] = x.z; g[4 * qq + 3] = x.w;
       }
       if (HEADG && row < V) {            // G = dH from step t+1 + the head's g·w_o ⊙ [H' > 0]
-        const float2 hv = __ldg(hg + row);
         const uint32_t mk = __float_as_uint(hv.y) >> c0;
 #pragma unroll
         for (int j = 0; j < HH; ++j)
-          if ((mk >> j) & 1u) g[j] = __fadd_rn(g[j], __fmul_rn(hv.x, __ldg(w_o + c0 + j)));
+          if ((mk >> j) & 1u) g[j] = __fadd_rn(g[j], __fmul_rn(hv.x, wog[j]));
       }
     }
     sync_tmem();
