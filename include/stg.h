@@ -556,12 +556,22 @@ stg_status stg_tgcn2_peer_bwd(int32_t phase, const stg_csr_view* g, const stg_tg
 stg_status stg_profile_enable(int32_t on);
 stg_status stg_profile_read(int32_t phase, double* total_ms, int64_t* count, int32_t reset);
 
-/* Schedule of stg_tgcn_train_sequence(_ev): 1 (default; env STG_SEQ_PIPELINE=0
- * sets 0 at load) = the three-stream pipeline (snapshot builds and the
+/* Schedule of stg_tgcn_train_sequence(_ev): 1 (default) = the three-stream pipeline (snapshot builds and the
  * H-independent work overlap the GRU chain); 0 = everything on the caller's
  * stream, one kernel after another (same arithmetic, same results; used to
  * measure the per-phase split). */
 stg_status stg_set_pipeline(int32_t on);
+
+/* Environment schedule tunables, read once when the library first needs them.
+ * None changes the arithmetic or skips work; each selects between measured
+ * schedules (defaults are the measured best on C5):
+ *   STG_ATB_SMEM_KB (220)  ring budget of the Σ AᵀB reduction kernel, KB
+ *   STG_ATB_CTAS (1)       allow 2 CTAs per SM for it when 3 stages fit twice
+ *   STG_ATB_L1 (0)         its 2-hi-stage / 1-lo-slot variant at 2 CTAs per SM
+ *   STG_SMALL_RB (auto)    rows per CTA of the small-graph sequence kernels
+ *   STG_DL_STREAM (0)      dL/dl reductions on the H-chain stream (1) or aux stream
+ *   STG_AUX_STREAM (1)     H-independent work on an aux stream (0: caller's stream)
+ *   STG_TORCH_ALLOCATOR    (binding) 0 keeps cudaMalloc instead of torch's pool */
 
 /* Order of the graph convolution in the TGCN step (reading C14; SURVEY §8(f)
  * NEXT-1): 0 (default) = linear-first C = Â(XW) + b — the forward aggregates

@@ -577,140 +577,6 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
   if (warp == 0) tc::tmem_free(tm, G::TCOLS);
 }
 
-// Ping-pong variant of k_tc_gru_fwd2: warps 0-3 and 4-7 are two independent groups
-// (thread = row, all H columns), each with its own raw buffer, TMEM half (256
-// columns) and barriers, working on alternate tiles — one group's MMA round trips
-// overlap the other's conversions and gate math.  TMEM per group: phase 1
-// [C_z hi | C_r hi | H hi | C_z lo | C_r lo | H lo | a_z | a_r]; phase 2 reuses
-// [0, 5H) as [C_h hi | C_h lo | rH hi | rH lo | a_h] once the phase-1 MMAs are done
-// (C_h stays in the raw buffer until then; the group's next TMA follows).
-__device__ __forceinline__ void group_sync(int g) { asm volatile("bar.sync %0, 128;" ::"r"(1 + g) : "memory"); }
-
-template <int H>
-__global__ void __launch_bounds__(256, 1) k_tc_gru_fwd3(int V, const __grid_constant__ CUtensorMap tmC,
-                                                        const __grid_constant__ CUtensorMap tmH,
-                                                        const float* __restrict__ L, const float* __restrict__ l,
-                                                        const __grid_constant__ CUtensorMap tmHn) {
-  using G = GruF2<H>;
-  constexpr int HH = G::HH;                      // column chunk (raw_to_tmem width, output box width)
-  extern __shared__ unsigned char sm_raw[];
-  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
-  __shared__ uint64_t full[2], mma_bar[2];
-  __shared__ uint32_t tslot;
-  unsigned char* bz_hi = sm + G::WOFF;  unsigned char* bz_lo = bz_hi + G::BG;
-  unsigned char* br_hi = bz_lo + G::BG; unsigned char* br_lo = br_hi + G::BG;
-  unsigned char* bh_hi = br_lo + G::BG; unsigned char* bh_lo = bh_hi + G::BG;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = warp & 3, g = warp >> 2;
-  const int lr = q * 32 + lane;
-  unsigned char* rawC = sm + (size_t)g * G::RAW;
-  unsigned char* rawH = rawC + G::NBC * kBox;
-  unsigned char* obuf = bh_lo + G::BG + warp * G::OBUF;
-  int oslot = 0;
-  const int LG = 2 * H * H;
-  stage_gate_weights<H>(bz_hi, bz_lo, L);
-  stage_gate_weights<H>(br_hi, br_lo, L + LG);
-  stage_gate_weights<H>(bh_hi, bh_lo, L + 2 * LG);
-  if (warp == 0) tc::tmem_alloc(&tslot, 512);
-  if (threadIdx.x == 0) {
-    tc::mbar_init(&full[0], 1); tc::mbar_init(&full[1], 1);
-    tc::mbar_init(&mma_bar[0], 1); tc::mbar_init(&mma_bar[1], 1);
-    tc::fence_mbar_init();
-  }
-  tc::fence_proxy_async();
-  tc::fence_before();
-  __syncthreads();
-  tc::fence_after();
-  const uint32_t tg = tslot + (uint32_t)(g * 256);         // this group's TMEM half
-  const uint32_t tq = tg + ((uint32_t)(q * 32) << 16);      // this thread's lane
-  const int ntiles = (V + 127) / 128;
-  const bool leader = (threadIdx.x & 127) == 0;
-  auto issue = [&](int tile) {
-    if (tile >= ntiles) return;
-    tc::mbar_expect_tx(&full[g], (uint32_t)(G::NBC + G::NBH) * kBox);
-#pragma unroll
-    for (int k = 0; k < G::NBC; ++k) tc::tma_load_2d(rawC + k * kBox, &tmC, 32 * k, tile * 128, &full[g]);
-    tc::tma_load_2d(rawH, &tmH, 0, tile * 128, &full[g]);
-  };
-  if (leader) issue(blockIdx.x + g * gridDim.x);
-  const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0);
-  uint32_t mph = 0;
-  for (int i = 0;; ++i) {
-    const int tile = blockIdx.x + (2 * i + g) * gridDim.x;
-    if (tile >= ntiles) break;
-    const int r0 = tile * 128;
-    tc::mbar_wait(&full[g], i & 1);
-    float h[H];
-#pragma unroll
-    for (int c = 0; c < H; c += HH) {
-      float t[HH];
-      raw_to_tmem<HH>(rawC, lr, c, tq + c, tq + 3 * H + c, t);                 // C_z
-      raw_to_tmem<HH>(rawC, lr, H + c, tq + H + c, tq + 4 * H + c, t);         // C_r
-      raw_to_tmem<HH>(rawH, lr, c, tq + 2 * H + c, tq + 5 * H + c, t);         // H
-#pragma unroll
-      for (int j = 0; j < HH; ++j) h[c + j] = t[j];
-    }
-    tc::tmem_wait_st();
-    tc::fence_before();
-    group_sync(g);
-    if (leader) {
-      tc::fence_after();
-      const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
-      mma_ts_seg(tg + 7 * H, tg + H, tg + 4 * H, rh_, rl, 2 * H, 0, H, idesc, true);        // r first
-      mma_ts_seg(tg + 7 * H, tg + 2 * H, tg + 5 * H, rh_, rl, 2 * H, H, H, idesc, false);
-      mma_ts_seg(tg + 6 * H, tg + 0, tg + 3 * H, zh, zl, 2 * H, 0, H, idesc, true);         // z
-      mma_ts_seg(tg + 6 * H, tg + 2 * H, tg + 5 * H, zh, zl, 2 * H, H, H, idesc, false);
-      tc::commit(&mma_bar[g]);
-    }
-    tc::mbar_wait(&mma_bar[g], mph);
-    mph ^= 1;
-    tc::fence_after();
-    float z[H];
-#pragma unroll
-    for (int c = 0; c < H; c += HH) {
-      float az[HH], ar[HH], rh[HH], lo[HH], t[HH];
-      tmem_row_load<HH>(tg + 6 * H, c, az);
-      tmem_row_load<HH>(tg + 7 * H, c, ar);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) {
-        z[c + j] = sigm(az[j] + __ldg(l + c + j));
-        rh[j] = sigm(ar[j] + __ldg(l + H + c + j)) * h[c + j];
-        lo[j] = rh[j] - tc::tf32_hi(rh[j]);
-      }
-      raw_to_tmem<HH>(rawC, lr, 2 * H + c, tq + c, tq + H + c, t);             // C_h over C_z / C_r hi
-      if constexpr (HH == 16) { tc::tmem_st16(tq + 2 * H + c, rh); tc::tmem_st16(tq + 3 * H + c, lo); }
-      else { tc::tmem_st8(tq + 2 * H + c, rh); tc::tmem_st8(tq + 3 * H + c, lo); }
-    }
-    tc::tmem_wait_st();
-    tc::fence_before();
-    group_sync(g);
-    if (leader) {
-      tc::fence_after();
-      issue(tile + 2 * gridDim.x);                     // raw buffer g fully read
-      const uint32_t hh_ = tc::smem_u32(bh_hi), hl = tc::smem_u32(bh_lo);
-      mma_ts_seg(tg + 4 * H, tg + 0, tg + H, hh_, hl, 2 * H, 0, H, idesc, true);           // h: C_h part
-      mma_ts_seg(tg + 4 * H, tg + 2 * H, tg + 3 * H, hh_, hl, 2 * H, H, H, idesc, false);  //    rH part
-      tc::commit(&mma_bar[g]);
-    }
-    tc::mbar_wait(&mma_bar[g], mph);
-    mph ^= 1;
-    tc::fence_after();
-#pragma unroll
-    for (int c = 0; c < H; c += HH) {
-      float ah[HH], o[HH];
-      tmem_row_load<HH>(tg + 4 * H, c, ah);
-#pragma unroll
-      for (int j = 0; j < HH; ++j) {
-        const float hh = tanhf(ah[j] + __ldg(l + 2 * H + c + j));
-        o[j] = z[c + j] * h[c + j] + (1.0f - z[c + j]) * hh;
-      }
-      tc::warp_box_store<HH>(obuf, oslot, o, 1.0f, &tmHn, c, r0 + q * 32);   // H'
-    }
-    tc::fence_before();
-  }
-  if (lane == 0) tc::bulk_wait_all();
-  __syncthreads();
-  if (warp == 0) tc::tmem_free(tslot, 512);
-}
 
 // ------------------------------------------------------------------ GRU backward, v2
 // Same data path as k_tc_gru_fwd2 (TMA boxes -> swizzled raw tile -> tensor
@@ -1730,10 +1596,6 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
   STG_TRY(make_tmap_f32(&tmC, C, (uint64_t)V, 3 * H, 3 * H, 32, 128));
   STG_TRY(make_tmap_f32(&tmH, Hp, (uint64_t)V, H, H, 32, 128));
   STG_TRY(make_tmap_f32_store(&tmHn, Hn, (uint64_t)V, H, H, (uint32_t)H / 2, 32));
-  static const int pp = [] {                       // ping-pong kernel (two 4-warp groups), opt-in:
-    const char* v = getenv("STG_GRU_FWD3");         // measured neutral on C5 (12.3 ms/epoch both)
-    return v ? atoi(v) : 0;
-  }();
   if (head) {                                      // fused surrogate head
     if (H == 32) {
       STG_TRY(prep(k_tc_gru_fwd2<32, true>, GruF2<32>::SMEM));
@@ -1742,12 +1604,6 @@ stg_status tc_gru_fwd(int V, int H, const float* C, const float* Hp, const float
       STG_TRY(prep(k_tc_gru_fwd2<16, true>, GruF2<16>::SMEM));
       k_tc_gru_fwd2<16, true><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn, *head);
     }
-  } else if (pp && H == 32) {
-    STG_TRY(prep(k_tc_gru_fwd3<32>, GruF2<32>::SMEM));
-    k_tc_gru_fwd3<32><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
-  } else if (pp) {
-    STG_TRY(prep(k_tc_gru_fwd3<16>, GruF2<16>::SMEM));
-    k_tc_gru_fwd3<16><<<nb, 256, GruF2<16>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn);
   } else if (H == 32) {
     STG_TRY(prep(k_tc_gru_fwd2<32, false>, GruF2<32>::SMEM));
     k_tc_gru_fwd2<32, false><<<nb, 256, GruF2<32>::SMEM, s>>>(V, tmC, tmH, L, l, tmHn, HeadArgs{});

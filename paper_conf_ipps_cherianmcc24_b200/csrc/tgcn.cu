@@ -1527,10 +1527,7 @@ int dl_on_chain() {
   }();
   return v;
 }
-std::atomic<int> g_pipeline{[] {
-  const char* v = getenv("STG_SEQ_PIPELINE");
-  return (v && v[0] == '0') ? 0 : 1;
-}()};
+std::atomic<int> g_pipeline{1};                   // stg_set_pipeline
 bool pipeline_enabled() { return g_pipeline.load(std::memory_order_relaxed) != 0; }
 // compute on an aux stream beside the H chain (1, default) or on the caller's
 // stream with only the snapshot builds overlapped (0)
