@@ -158,13 +158,11 @@ struct stg_dtdg {
     const uint64_t* gd = sharded ? gdel.p : del_out.p;
     const std::vector<int64_t>& gao = sharded ? ga_off : a_off;
     const std::vector<int64_t>& gdo = sharded ? gd_off : d_off;
-    const size_t vb = sizeof(int32_t) * (size_t)V;
-    STG_CUDA(cudaMemcpyAsync(st.gin_deg.p, sf.gin_deg.p, vb, cudaMemcpyDeviceToDevice, s));
-    STG_CUDA(cudaMemcpyAsync(st.gout_deg.p, sf.gout_deg.p, vb, cudaMemcpyDeviceToDevice, s));
-    STG_TRY(degree_hist2(DirDelta{ga + gao[td], gao[td + 1] - gao[td], gd + gdo[td], gdo[td + 1] - gdo[td]}, nb,
-                         rev ? -1 : 1, st.gin_deg.p, st.gout_deg.p, s));
+    // the whole-graph degrees (norms) follow inside the first direction's pass
+    const GDegStep gdeg{DirDelta{ga + gao[td], gao[td + 1] - gao[td], gd + gdo[td], gdo[td + 1] - gdo[td]},
+                        rev ? -1 : 1, sf.gin_deg.p, sf.gout_deg.p, st.gin_deg.p, st.gout_deg.p};
     return apply_delta(sf, st, dir(td, true, rev), dir(td, false, rev), E[t1], t1, touch_in.p,
-                       touch_out.p, *ws, s, parts & (PART_IN | PART_OUT));
+                       touch_out.p, *ws, s, parts & (PART_IN | PART_OUT), &gdeg);
   }
 
   // Walk from the best cached slot to t, writing into the pair {p0, p0+1}, for

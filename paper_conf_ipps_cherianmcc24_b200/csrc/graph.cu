@@ -353,7 +353,7 @@ stg_status complete_parts(Snapshot& g, uint32_t want, BuildWs& ws, cudaStream_t 
 // (the per-direction kernels are in snapshot.cu)
 stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
                        int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws, cudaStream_t s,
-                       uint32_t parts) {
+                       uint32_t parts, const GDegStep* gdeg) {
   const bool do_in = (parts & PART_IN) != 0, do_out = (parts & PART_OUT) != 0;
   if ((do_in && !(src.parts & PART_IN)) || (do_out && !(src.parts & PART_OUT)))
     return fail(STG_ERR_STATE, "apply_delta: source snapshot lacks a requested direction");
@@ -366,13 +366,19 @@ stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_di
     STG_TRY(ws.emap.alloc((size_t)src.E, s));
     emap = ws.emap.p;
   }
+  if (gdeg && !do_in && !do_out) {                  // no direction pass to carry the degree update
+    const size_t vb = sizeof(int32_t) * (size_t)src.V;
+    STG_CUDA(cudaMemcpyAsync(gdeg->gin_dst, gdeg->gin_src, vb, cudaMemcpyDeviceToDevice, s));
+    STG_CUDA(cudaMemcpyAsync(gdeg->gout_dst, gdeg->gout_src, vb, cudaMemcpyDeviceToDevice, s));
+    STG_TRY(degree_hist2(gdeg->keys, src.nb, gdeg->sign, gdeg->gin_dst, gdeg->gout_dst, s));
+  }
   if (do_in)
     STG_TRY(apply_dir2(src, dst, true, in_dir, touch_in, ws, s, true, emap, nullptr, nullptr, nullptr, nullptr,
-                       nullptr));
+                       nullptr, gdeg));
   if (do_out)
     STG_TRY(apply_dir2(src, dst, false, out_dir, touch_out, ws, s, !do_in, nullptr, carry ? emap : nullptr,
                        carry ? src.out_eid.p : nullptr, carry ? dst.out_eid.p : nullptr,
-                       carry ? dst.in_rowptr.p : nullptr, carry ? dst.in_col.p : nullptr));
+                       carry ? dst.in_rowptr.p : nullptr, carry ? dst.in_col.p : nullptr, do_in ? nullptr : gdeg));
   dst.E = E_new;
   dst.t = t_new;
   dst.parts = (do_in ? PART_IN : 0u) | (do_out ? PART_OUT : 0u);

@@ -27,7 +27,8 @@ inline int64_t sched_cap(int64_t E) { return E / (kHubChunk + 1) + 2; }
 //   sched[3] = n_items  = n_chunks + V - n_hub
 //   sched[4] = first item of the light rows with n <= kTierB (items are in degree order)
 //   sched[5] = first item of the light rows with n <= kTierC
-//   sched[6], sched[7]  unused (items stay 16-byte aligned)
+//   sched[6] = m        rows of the saturated node_ids prefix (degree >= 1023, snapshot.cu)
+//   sched[7] = their hub chunks (cptr[m]); build-time only (items stay 16-byte aligned)
 //   sched[8 ..]         = items, int4 {v, beg, n, hub} in node_ids order: hub
 //                         chunks first (hub = index into ids / cptr), then the
 //                         light rows (hub = -1).  n <= kHubChunk.
@@ -148,18 +149,29 @@ stg_status ids_sched_build(const int32_t* deg, const int32_t* rowptr, int32_t V,
                            int32_t* ids, int32_t* sched, int64_t cap, BuildWs& ws, cudaStream_t s);
 // whole-graph degree histogram of one delta batch (adds +sign, deletes -sign)
 stg_status degree_hist2(const DirDelta& d, int nb, int sign, int32_t* gin, int32_t* gout, cudaStream_t s);
+// whole-graph degree update of one delta step, fused into the first direction's pass:
+// dst's gin / gout = src's + the ±1 histogram of the whole-graph (src << nb | dst) keys
+struct GDegStep {
+  DirDelta keys;                 // whole-graph effective deltas (add = +sign, del = -sign)
+  int sign;
+  const int32_t* gin_src;
+  const int32_t* gout_src;
+  int32_t* gin_dst;
+  int32_t* gout_dst;
+};
 // one delta step of one CSR direction of src into dst (rowptr, col, degrees,
 // node_ids, schedule; the GCN norms too if `norms`); labels as in apply_delta
 stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const DirDelta& d, int4* touch, BuildWs& ws,
                       cudaStream_t s, bool norms, int32_t* emap_out, const int32_t* emap_in, const int32_t* eid_old,
-                      int32_t* eid_new, const int32_t* in_rowptr_new, const int32_t* in_col_new);
+                      int32_t* eid_new, const int32_t* in_rowptr_new, const int32_t* in_col_new,
+                      const GDegStep* gdeg = nullptr);
 
 // Applies the delta to the directions in `parts` (src must hold them; labels
 // are carried when both directions and src's labels are present).  The caller
 // has already updated dst's whole-graph degrees (gin_deg / gout_deg).
 stg_status apply_delta(const Snapshot& src, Snapshot& dst, const DirDelta& in_dir, const DirDelta& out_dir,
                        int64_t E_new, int32_t t_new, int4* touch_in, int4* touch_out, BuildWs& ws,
-                       cudaStream_t s, uint32_t parts = PART_ALL);
+                       cudaStream_t s, uint32_t parts = PART_ALL, const GDegStep* gdeg = nullptr);
 
 }  // namespace stg
 

@@ -27,11 +27,14 @@ struct BuildWs {
   DArray<int32_t> emap;        // delta apply: old in-CSR position -> new position (-1 = deleted)
   // node_ids counting sort and the single-pass row scan (snapshot.cu)
   DArray<int32_t> ids_hist, ids_offs, ids_tot, sat_tmp;
-  DArray<int32_t> merge_rows;  // row of the first old edge of every merge tile
+  DArray<int32_t> mpos;        // old-CSR positions of one step's adds | deletes (merge path)
+  DArray<int32_t> mbnd;        // per merge tile: first add | first delete placed in it
   DArray<int32_t> rows;        // COO row ids of one direction (transposes / labels only)
   DArray<uint64_t> lb_status;  // decoupled look-back words, one per row tile
   DArray<uint32_t> lb_ticket;  // tile counter (zeroed before each scan)
+  DArray<int32_t> gdeg;        // [2V] whole-graph degree deltas of one step (zero between steps)
   uint32_t lb_epoch = 0;
+  uint32_t lb_base = 0;        // lb_ticket's value when the next row scan starts (tickets are never reset)
 };
 
 namespace {

@@ -3,19 +3,25 @@
 // schedule builder (the degree presort), in few launches:
 //
 //   one delta step of one CSR direction (apply_dir2):
-//     k_touch2       mark the sorted add / delete ranges of every touched row
+//     k_touch3       mark the sorted add / delete ranges of every touched row;
+//                    place every delta key in the OLD CSR (its merge-path
+//                    position) and the merge tiles' first add / delete; the
+//                    whole-graph degree deltas of the step (GCN norms)
 //     k_rowscan      single-pass scan (decoupled look-back) of the new degrees
-//                    deg' = deg + |adds| - |dels| -> rowptr', deg', the GCN
-//                    norms, and the per-tile histogram of the node_ids key
-//     k_merge2       old edges move to rowptr'[v] + i - #dels<c + #adds<c (deleted
-//                    ones dropped), added edges are inserted; the row of an old
-//                    edge comes from the old rowptr (no COO row array is kept)
+//                    deg' = deg + |adds| - |dels| -> rowptr', deg', the
+//                    whole-graph degrees and GCN norms, and the per-tile
+//                    histogram of the node_ids key
+//     k_merge3       global merge path over the sorted (row, col) keys: old
+//                    edge j -> j - #dels before j + #adds placed <= j, add i at
+//                    old position p -> p - #dels before p + i (no row lookups)
 //   node_ids + schedule (ids_sched_build):
 //     k_ids_offsets  one CTA: digit-major exclusive scan of the tile histograms
 //     k_ids_scatter  stable counting-sort scatter (warp match_any ranks)
 //     k_ids_finish   one CTA: exact order of the saturated prefix (degree >=
-//                    kIdsSat), hub-chunk pointers, schedule header and tiers
-//     k_items2       work items in node_ids order; clears the touch marks
+//                    kIdsSat), its hub-chunk pointers, the per-bucket chunk
+//                    bases, schedule header and tiers
+//     k_items2       work items in node_ids order (the other hub-chunk
+//                    pointers in closed form); clears the step's marks
 //
 // node_ids = rows by (degree desc, id asc) (reading C4): a stable
 // counting sort on the key min(deg, kIdsSat) (kIdsSat + 1 buckets, plus one
@@ -41,7 +47,6 @@ constexpr int kIdsBuckets = kIdsSat + 2;         // 0..kIdsSat: degree buckets, 
 constexpr int kIdsOut = kIdsSat + 1;
 constexpr int kSatSortMax = 8192;                // saturated prefix sorted in shared memory
 constexpr int kSatRankMax = 2048;                // ... ranked by counting up to this size (O(m²/1024) per thread)
-constexpr int kMergeTile = 2048;                 // old edges per merge CTA
 
 __device__ __forceinline__ int ids_digit(int32_t v, int32_t d, int32_t rb, int32_t re) {
   if (v < rb || v >= re) return kIdsOut;
@@ -49,21 +54,105 @@ __device__ __forceinline__ int ids_digit(int32_t v, int32_t d, int32_t rb, int32
 }
 
 // ------------------------------------------------------------ delta marks
-// touch[row] = {add_lo, add_hi, del_lo, del_hi} (ranges in the sorted delta lists)
-__global__ void k_touch2(const uint64_t* __restrict__ add, int64_t nadd, const uint64_t* __restrict__ del,
-                         int64_t ndel, int nb, int4* __restrict__ touch) {
-  const int64_t n = nadd + ndel;
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
-    const bool is_add = k < nadd;
-    const uint64_t* d = is_add ? add : del;
-    const int64_t m = is_add ? nadd : ndel;
-    const int64_t i = is_add ? k : k - nadd;
-    const int32_t r = (int32_t)(d[i] >> nb);
-    const bool first = i == 0 || (int32_t)(d[i - 1] >> nb) != r;
-    const bool last = i == m - 1 || (int32_t)(d[i + 1] >> nb) != r;
-    int* t = reinterpret_cast<int*>(touch + r);
-    if (first) t[is_add ? 0 : 2] = (int)i;
-    if (last) t[is_add ? 1 : 3] = (int)(i + 1);
+// One launch over the step's delta keys (sorted, effective: adds absent from the
+// old CSR, deletes present):
+//   touch[row] = {add_lo, add_hi, del_lo, del_hi} (ranges in the sorted lists);
+//   padd[i] / pdel[i] = the key's position in the OLD CSR (insertion point of an
+//     add = number of old keys below it; a delete's own position) — old CSR
+//     positions are the global (row, col) key order, so these are the merge
+//     path of k_merge3;
+//   abnd[t] / dbnd[t] = adds / deletes whose position lies in merge tiles < t
+//     (positions are monotone in the sorted lists: each key writes the tiles
+//     between its predecessor's and its own; t in [0, ntm]);
+//   (gdeg) the whole-graph degree deltas into the zeroed scratch din / dout.
+struct TouchArgs {
+  const uint64_t* add;
+  int64_t nadd;
+  const uint64_t* del;
+  int64_t ndel;
+  int nb;
+  int4* touch;
+  const int32_t* orowptr;
+  const int32_t* ocol;
+  int32_t* padd;
+  int32_t* pdel;
+  int32_t* abnd;
+  int32_t* dbnd;
+  int32_t ntm;                  // merge tiles (positions [0, E_old] map to tiles [0, ntm))
+  const uint64_t* gadd;         // whole-graph keys (may be NULL)
+  int64_t ngadd;
+  const uint64_t* gdel;
+  int64_t ngdel;
+  int sign;
+  int32_t* din;
+  int32_t* dout;
+};
+
+constexpr int kMergeShift = 11;
+constexpr int kMergeTile = 1 << kMergeShift;     // old edges per merge CTA
+
+__device__ __forceinline__ int32_t old_pos(const int32_t* __restrict__ orowptr, const int32_t* __restrict__ ocol,
+                                           uint64_t key, int nb) {
+  const int32_t r = (int32_t)(key >> nb), c = (int32_t)(key & ((uint64_t(1) << nb) - 1));
+  int32_t b = __ldg(orowptr + r), e = __ldg(orowptr + r + 1);
+  while (b < e) {
+    const int32_t mid = (b + e) >> 1;
+    if (__ldg(ocol + mid) < c) b = mid + 1; else e = mid;
+  }
+  return b;
+}
+
+__global__ void __launch_bounds__(256) k_touch3(const TouchArgs a) {
+  const int64_t n = a.nadd + a.ndel, ng = a.ngadd + a.ngdel;
+  const uint64_t gmask = (uint64_t(1) << a.nb) - 1;
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  if (n == 0 && blockIdx.x == 0) {                     // no keys: every tile starts at entry 0
+    for (int t = threadIdx.x; t <= a.ntm; t += blockDim.x) { a.abnd[t] = 0; a.dbnd[t] = 0; }
+  }
+  const int64_t kend = max(n, ng);
+  for (int64_t k0 = blockIdx.x * (int64_t)blockDim.x; k0 < kend; k0 += stride) {   // warp-uniform trip count
+    const int64_t k = k0 + threadIdx.x;
+    if (k < ng) {
+      const uint64_t key = k < a.ngadd ? a.gadd[k] : a.gdel[k - a.ngadd];
+      const int sg = k < a.ngadd ? a.sign : -a.sign;
+      atomicAdd(a.din + (int32_t)(key & gmask), sg);
+      atomicAdd(a.dout + (int32_t)(key >> a.nb), sg);
+    }
+    const bool on = k < n;
+    const bool is_add = k < a.nadd;
+    const uint64_t* d = is_add ? a.add : a.del;
+    const int64_t m = is_add ? a.nadd : a.ndel;
+    const int64_t i = is_add ? k : k - a.nadd;
+    int32_t p = 0;
+    if (on) {
+      const uint64_t key = d[i];
+      const int32_t r = (int32_t)(key >> a.nb);
+      const bool first = i == 0 || (int32_t)(d[i - 1] >> a.nb) != r;
+      const bool last = i == m - 1 || (int32_t)(d[i + 1] >> a.nb) != r;
+      int* t = reinterpret_cast<int*>(a.touch + r);
+      if (first) t[is_add ? 0 : 2] = (int)i;
+      if (last) t[is_add ? 1 : 3] = (int)(i + 1);
+      p = old_pos(a.orowptr, a.ocol, key, a.nb);
+      (is_add ? a.padd : a.pdel)[i] = p;
+    }
+    // tile boundaries: the predecessor's position from the previous lane (same list), else searched
+    const int32_t pl = __shfl_up_sync(0xffffffffu, p, 1);
+    if (on) {
+      int32_t tp = -1;
+      if (i > 0) tp = (lane > 0 && k - 1 >= (is_add ? 0 : a.nadd)) ? (pl >> kMergeShift)
+                                                                  : (old_pos(a.orowptr, a.ocol, d[i - 1], a.nb) >> kMergeShift);
+      int32_t* bnd = is_add ? a.abnd : a.dbnd;
+      const int32_t ti = p >> kMergeShift;
+      for (int32_t t = tp + 1; t <= ti; ++t) bnd[t] = (int32_t)i;
+      if (i == m - 1)
+        for (int32_t t = ti + 1; t <= a.ntm; ++t) bnd[t] = (int32_t)m;
+    }
+  }
+  // one list empty (the other not): its tiles all start at entry 0
+  if (n > 0 && blockIdx.x == 0) {
+    if (a.nadd == 0) for (int t = threadIdx.x; t <= a.ntm; t += blockDim.x) a.abnd[t] = 0;
+    if (a.ndel == 0) for (int t = threadIdx.x; t <= a.ntm; t += blockDim.x) a.dbnd[t] = 0;
   }
 }
 
@@ -104,7 +193,8 @@ struct RowScanArgs {
   int32_t* hist;                // [kIdsBuckets][ntiles]
   int32_t ntiles;
   uint64_t* status;             // [ntiles] look-back words (TOUCH only)
-  uint32_t* ticket;             // tile counter, zero at launch (TOUCH only)
+  uint32_t* ticket;             // tile counter (TOUCH only), equal to tbase at launch
+  uint32_t tbase;
   uint32_t epoch;
   // GCN norms from the whole-graph degrees (may be NULL: not computed)
   const int32_t* gin;
@@ -112,9 +202,12 @@ struct RowScanArgs {
   int dgl_both;
   float* norm_src;
   float* norm_dst;
-  // (TOUCH) the old CSR's row pointer: tile_row[t] = row of old edge t·kMergeTile
-  const int32_t* orowptr;
-  int32_t* tile_row;
+  // fused whole-graph degree step (may be NULL): gin / gout are the source slot's,
+  // the degrees are gin + din, gout + dout, written to gin_w / gout_w
+  const int32_t* din;
+  const int32_t* dout;
+  int32_t* gin_w;
+  int32_t* gout_w;
 };
 
 template <bool TOUCH>
@@ -125,7 +218,7 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
   __shared__ int64_t s_prefix;
   for (int d = threadIdx.x; d < kIdsBuckets; d += kRowThreads) h[d] = 0;
   if (TOUCH) {
-    if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u);   // tiles in start order: look-back never waits on an unstarted tile
+    if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u) - a.tbase;   // tiles in start order: look-back never waits on an unstarted tile
   }
   __syncthreads();
   const int32_t tile = TOUCH ? (int32_t)s_tile : (int32_t)blockIdx.x;
@@ -147,11 +240,31 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
   }
   if (a.norm_dst) {                                    // (independent of the scan: issued first)
     int32_t gi[kRowIPT], go[kRowIPT];
+    if (a.din) {                                       // whole-graph degrees of this step (both kept current)
+      int32_t di[kRowIPT], dd[kRowIPT];
 #pragma unroll
-    for (int k = 0; k < kRowIPT; ++k) {
-      const int64_t v = r0 + (int64_t)k * kRowThreads;
-      gi[k] = v < a.V ? __ldg(a.gin + v) : 0;
-      go[k] = (v < a.V && a.dgl_both) ? __ldg(a.gout + v) : 0;
+      for (int k = 0; k < kRowIPT; ++k) {
+        const int64_t v = r0 + (int64_t)k * kRowThreads;
+        const bool ok = v < a.V;
+        gi[k] = ok ? __ldg(a.gin + v) : 0;
+        go[k] = ok ? __ldg(a.gout + v) : 0;
+        di[k] = ok ? __ldcg(a.din + v) : 0;
+        dd[k] = ok ? __ldcg(a.dout + v) : 0;
+      }
+#pragma unroll
+      for (int k = 0; k < kRowIPT; ++k) {
+        const int64_t v = r0 + (int64_t)k * kRowThreads;
+        gi[k] += di[k];
+        go[k] += dd[k];
+        if (v < a.V) { a.gin_w[v] = gi[k]; a.gout_w[v] = go[k]; }
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < kRowIPT; ++k) {
+        const int64_t v = r0 + (int64_t)k * kRowThreads;
+        gi[k] = v < a.V ? __ldg(a.gin + v) : 0;
+        go[k] = (v < a.V && a.dgl_both) ? __ldg(a.gout + v) : 0;
+      }
     }
 #pragma unroll
     for (int k = 0; k < kRowIPT; ++k) {
@@ -160,25 +273,6 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
       const float nd = gi[k] > 0 ? 1.0f / sqrtf((float)gi[k]) : 0.0f;
       a.norm_dst[v] = nd;
       a.norm_src[v] = a.dgl_both ? (go[k] > 0 ? 1.0f / sqrtf((float)go[k]) : 0.0f) : nd;
-    }
-  }
-  if (TOUCH) {                                          // merge tile starts inside these (old) rows
-    const int ln = threadIdx.x & 31;
-    int32_t ob[kRowIPT], oe31[kRowIPT];
-#pragma unroll
-    for (int k = 0; k < kRowIPT; ++k) {                 // row v + 1 is the next lane's row (lane 31 loads it)
-      const int64_t v = r0 + (int64_t)k * kRowThreads;
-      ob[k] = v <= a.V ? __ldg(a.orowptr + v) : 0;     // (row V: the end of the last row)
-      oe31[k] = (ln == 31 && v < a.V) ? __ldg(a.orowptr + v + 1) : 0;
-    }
-#pragma unroll
-    for (int k = 0; k < kRowIPT; ++k) {
-      const int64_t v = r0 + (int64_t)k * kRowThreads;
-      const int32_t nx = __shfl_down_sync(0xffffffffu, ob[k], 1);
-      const int32_t oe = ln == 31 ? oe31[k] : nx;
-      if (v < a.V)
-        for (int32_t t = (ob[k] + kMergeTile - 1) / kMergeTile; (int64_t)t * kMergeTile < oe; ++t)
-          a.tile_row[t] = (int32_t)v;
     }
   }
   // node_ids key histogram (shared atomics, warp-aggregated by match_any)
@@ -346,18 +440,51 @@ __global__ void __launch_bounds__(kRowThreads) k_ids_scatter(const int32_t* __re
 }
 
 // One CTA: (1) the saturated prefix ids[0, m) (degree >= kIdsSat, ascending id)
-// re-ordered by (degree desc, id asc); (2) n_hub = rows with degree > kHubChunk,
-// their chunk pointers cptr[0..n_hub] and n_chunks; (3) the schedule header and
-// the light-row tier boundaries (degree order makes them bucket-count prefixes).
+// re-ordered by (degree desc, id asc); (2) n_hub = rows with degree > kHubChunk
+// and the schedule header / light-row tiers (degree order makes them bucket-count
+// prefixes); (3) the hub-chunk pointers of the saturated prefix (a scan over its m
+// rows) and, for every other hub bucket b (all of its rows have degree exactly
+// kIdsSat - b, so ceil(deg / kHubChunk) chunks each), the bucket's first chunk
+// bk[b] and first row bk[kIdsBuckets + b]: k_items2 derives the rest of cptr in
+// closed form, so no per-hub pass runs in this single CTA.
 __global__ void __launch_bounds__(1024) k_ids_finish(int32_t* __restrict__ ids, const int32_t* __restrict__ deg,
                                                      const int32_t* __restrict__ totals, int32_t R, int64_t coff,
-                                                     int32_t* __restrict__ sched, int32_t* __restrict__ tmp) {
+                                                     int32_t* __restrict__ sched, int32_t* __restrict__ tmp,
+                                                     int32_t* __restrict__ bk) {
   extern __shared__ uint64_t sk[];                      // [kSatSortMax] sort keys
   __shared__ int32_t s_wsum[32];
   __shared__ int32_t s_btot;
   __shared__ int32_t s_cnt[3];
   const int m = totals[0];
   const int nt = blockDim.x;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  // block-wide exclusive scan (nt threads); *tot = the block total
+  auto bscan = [&](int32_t x, int32_t* tot) -> int32_t {
+    int32_t inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += y;
+    }
+    if (lane == 31) s_wsum[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+      const int32_t sv = lane < (nt >> 5) ? s_wsum[lane] : 0;
+      int32_t si = sv;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int32_t y = __shfl_up_sync(0xffffffffu, si, o);
+        if (lane >= o) si += y;
+      }
+      s_wsum[lane] = si - sv;                           // exclusive warp offsets
+      if (lane == 31) s_btot = si;                      // block total
+    }
+    __syncthreads();
+    const int32_t ex = s_wsum[w] + inc - x;
+    *tot = s_btot;
+    __syncthreads();                                    // s_wsum / s_btot reused by the next scan
+    return ex;
+  };
   if (threadIdx.x < 3) s_cnt[threadIdx.x] = 0;
   __syncthreads();
   {    // rows with degree > kHubChunk / > kTierB / > kTierC: bucket-count prefixes
@@ -429,49 +556,35 @@ __global__ void __launch_bounds__(1024) k_ids_finish(int32_t* __restrict__ ids, 
       __syncthreads();
       for (int i = threadIdx.x; i < m; i += nt) ids[i] = tmp[i];
     }
-    __syncthreads();
   }
   __syncthreads();
   const int32_t n_hub = s_cnt[0], n_b = s_cnt[1], n_c = s_cnt[2];
-  // chunk pointers over the hub rows: exclusive scan of ceil(deg / kHubChunk); each
-  // round's kFinishPT loads per thread are issued together (independent chains)
-  constexpr int kFinishPT = 16;
+  // (3a) chunk pointers over the saturated prefix (every row of it is a hub)
   int32_t* cptr = sched + coff;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   int32_t carry = 0;
-  for (int h0 = 0; h0 < n_hub; h0 += nt * kFinishPT) {
-    int32_t x[kFinishPT];
-#pragma unroll
-    for (int k = 0; k < kFinishPT; ++k) {
-      const int h = h0 + k * nt + threadIdx.x;
-      x[k] = h < n_hub ? (__ldg(deg + __ldg(ids + h)) + kHubChunk - 1) / kHubChunk : 0;
+  for (int h0 = 0; h0 < m; h0 += nt) {
+    const int h = h0 + threadIdx.x;
+    const int32_t x = h < m ? (__ldg(deg + __ldg(ids + h)) + kHubChunk - 1) / kHubChunk : 0;
+    int32_t tot;
+    const int32_t ex = bscan(x, &tot);
+    if (h < m) cptr[h] = carry + ex;
+    carry += tot;
+  }
+  const int32_t csat = carry;
+  // (3b) the other hub buckets b in [1, kIdsSat - kHubChunk): first chunk and first row
+  {
+    const int b = threadIdx.x;                          // nt >= kIdsSat + 1 threads
+    const bool hubb = b >= 1 && b < kIdsSat - kHubChunk;
+    const int32_t cnt = hubb ? __ldg(totals + b) : 0;
+    const int32_t nc = hubb ? (kIdsSat - b + kHubChunk - 1) / kHubChunk : 0;
+    int32_t tchunks, trows;
+    const int32_t exc = bscan(cnt * nc, &tchunks);
+    const int32_t exr = bscan(cnt, &trows);
+    if (b < kIdsBuckets) {
+      bk[b] = carry + exc;
+      bk[kIdsBuckets + b] = m + exr;
     }
-    for (int k = 0; k < kFinishPT && h0 + k * nt < n_hub; ++k) {
-      const int h = h0 + k * nt + threadIdx.x;
-      int32_t inc = x[k];
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc += y;
-      }
-      if (lane == 31) s_wsum[w] = inc;
-      __syncthreads();
-      if (w == 0) {
-        const int32_t sv = lane < (nt >> 5) ? s_wsum[lane] : 0;
-        int32_t si = sv;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int32_t y = __shfl_up_sync(0xffffffffu, si, o);
-          if (lane >= o) si += y;
-        }
-        s_wsum[lane] = si - sv;                         // exclusive warp offsets
-        if (lane == 31) s_btot = si;                    // block total
-      }
-      __syncthreads();
-      if (h < n_hub) cptr[h] = carry + s_wsum[w] + inc - x[k];
-      carry += s_btot;
-      __syncthreads();
-    }
+    carry += tchunks;
   }
   if (threadIdx.x == 0) {
     cptr[n_hub] = carry;
@@ -483,29 +596,53 @@ __global__ void __launch_bounds__(1024) k_ids_finish(int32_t* __restrict__ ids, 
     sched[3] = total;
     sched[4] = n_chunks + n_b - n_hub;
     sched[5] = n_chunks + n_c - n_hub;
+    sched[6] = m;                                       // saturated rows (cptr[0..m) written here)
+    sched[7] = csat;                                    // their chunks
   }
 }
 
 // Work items in node_ids order (layout in graph.cuh); then clear the touch marks
-// of this step's deltas (the next step starts from zero marks).
+// of this step's deltas (the next step starts from zero marks).  A hub chunk item
+// finds its row in the saturated prefix by a search over cptr[0..m], else through
+// the bucket tables of k_ids_finish (closed form: every row of bucket b has the
+// same chunk count); the first chunk of each such row writes its cptr entry.
 __global__ void k_items2(const int32_t* __restrict__ ids, const int32_t* __restrict__ rowptr, int64_t cap_items,
-                         int32_t* __restrict__ sched, const uint64_t* __restrict__ add, int64_t nadd,
-                         const uint64_t* __restrict__ del, int64_t ndel, int nb, int4* __restrict__ touch) {
-  const int32_t n_hub = sched[0], n_chunks = sched[1];
-  const int32_t* cptr = sched + sched[2];
+                         int32_t* __restrict__ sched, const int32_t* __restrict__ bk, const uint64_t* __restrict__ add,
+                         int64_t nadd, const uint64_t* __restrict__ del, int64_t ndel, int nb,
+                         int4* __restrict__ touch, const uint64_t* __restrict__ gadd, int64_t ngadd,
+                         const uint64_t* __restrict__ gdel, int64_t ngdel, int32_t* __restrict__ din,
+                         int32_t* __restrict__ dout) {
+  const int32_t n_hub = sched[0], n_chunks = sched[1], m = sched[6], csat = sched[7];
+  int32_t* cptr = sched + sched[2];
   const int64_t total = sched[3];
   int4* items = reinterpret_cast<int4*>(sched + kSchedHdr);
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total && i < cap_items; i += stride) {
     if (i < n_chunks) {
-      int32_t lo = 0, hi = n_hub;      // largest h with cptr[h] <= i
-      while (lo < hi) {
-        const int32_t mid = (lo + hi + 1) >> 1;
-        if (cptr[mid] <= i) lo = mid; else hi = mid - 1;
+      int32_t h, j;
+      if (i < csat) {
+        int32_t lo = 0, hi = m - 1;                     // largest h with cptr[h] <= i
+        while (lo < hi) {
+          const int32_t mid = (lo + hi + 1) >> 1;
+          if (cptr[mid] <= i) lo = mid; else hi = mid - 1;
+        }
+        h = lo;
+        j = (int32_t)i - cptr[lo];
+      } else {
+        int32_t lo = 1, hi = kIdsSat - kHubChunk - 1;   // largest hub bucket b with bk[b] <= i
+        while (lo < hi) {
+          const int32_t mid = (lo + hi + 1) >> 1;
+          if (__ldg(bk + mid) <= i) lo = mid; else hi = mid - 1;
+        }
+        const int32_t nc = (kIdsSat - lo + kHubChunk - 1) / kHubChunk;
+        const int32_t off = (int32_t)i - __ldg(bk + lo);
+        h = __ldg(bk + kIdsBuckets + lo) + off / nc;
+        j = off % nc;
+        if (j == 0) cptr[h] = (int32_t)i;
       }
-      const int32_t v = ids[lo], rb = rowptr[v], re = rowptr[v + 1];
-      const int32_t beg = rb + (int32_t)(i - cptr[lo]) * kHubChunk;
-      items[i] = make_int4(v, beg, min(kHubChunk, re - beg), lo);
+      const int32_t v = ids[h], rb = rowptr[v], re = rowptr[v + 1];
+      const int32_t beg = rb + j * kHubChunk;
+      items[i] = make_int4(v, beg, min(kHubChunk, re - beg), h);
     } else {
       const int32_t v = ids[n_hub + (i - n_chunks)];
       const int32_t rb = rowptr[v];
@@ -518,37 +655,37 @@ __global__ void k_items2(const int32_t* __restrict__ ids, const int32_t* __restr
       touch[(int32_t)(key >> nb)] = make_int4(0, 0, 0, 0);
     }
   }
+  if (din) {
+    const uint64_t mask = (uint64_t(1) << nb) - 1;
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < ngadd + ngdel; k += stride) {
+      const uint64_t key = k < ngadd ? gadd[k] : gdel[k - ngadd];
+      din[(int32_t)(key & mask)] = 0;
+      dout[(int32_t)(key >> nb)] = 0;
+    }
+  }
 }
 
 // ------------------------------------------------------------ merge
-__device__ __forceinline__ int64_t lb_u64(const uint64_t* a, int64_t lo, int64_t hi, uint64_t k) {
-  while (lo < hi) {
-    const int64_t mid = (lo + hi) >> 1;
-    if (a[mid] < k) lo = mid + 1; else hi = mid;
-  }
-  return lo;
-}
-// the row of CSR position j: largest r in [lo, hi] with rowptr[r] <= j
-__device__ __forceinline__ int32_t row_of(const int32_t* rp, int32_t lo, int32_t hi, int64_t j) {
-  while (lo < hi) {
-    const int32_t mid = (lo + hi + 1) >> 1;
-    if (rp[mid] <= j) lo = mid; else hi = mid - 1;
-  }
-  return lo;
-}
-
+// The CSR of one direction, read in position order, is the sorted key sequence
+// (row << nb | col); the new CSR is the merge of the surviving old keys and the
+// added keys (both sorted), so with D(j) = deletes at old positions < j and
+// A(j) = adds whose insertion point p <= j (k_touch3):
+//   surviving old edge j  ->  j − D(j) + A(j)
+//   added key i (point p) ->  p − D(p) + i
+// (rows need not be known: rowptr' comes from the degree scan).  A CTA owns
+// kMergeTile old positions plus the adds / deletes placed in them (contiguous
+// ranges of the sorted lists, from abnd / dbnd): marks in shared memory, one
+// block scan, then coalesced stores of the old edges and the adds.
 struct MergeArgs {
-  int32_t V, nb;
-  const int32_t* orowptr;
+  int nb;
   const int32_t* ocol;
   int64_t E_old;
-  const int32_t* nrowptr;
-  const int4* touch;
   const uint64_t* add;
-  int64_t nadd;
-  const uint64_t* del;
+  const int32_t* padd;
+  const int32_t* pdel;
+  const int32_t* abnd;
+  const int32_t* dbnd;
   int32_t* ncol;
-  int64_t old_tiles;
   // edge labels: in-direction pass records emap[old pos] = new pos
   // (-1 deleted); out-direction pass sets eid_new[new pos] = emap_in[eid_old[old pos]]
   // and searches the label of an added out-edge in the new in-CSR
@@ -558,194 +695,94 @@ struct MergeArgs {
   int32_t* eid_new;
   const int32_t* in_rowptr_new;
   const int32_t* in_col_new;
-  const int32_t* tile_row;      // row of the first old edge of every tile (k_rowscan)
 };
 
-// Old edges: a CTA takes kMergeTile consecutive positions.  The tile's rows
-// (rows [tile_row[t], tile_row[t+1]], from k_rowscan) have their old / new row
-// pointers and touch marks cached in shared memory, and the row of every position
-// comes from a max-scan of the row-start marks.  Merge path: old edges, adds and
-// deletes are all sorted by key = (row << nb) | col, so each add / delete key of the
-// tile's rows finds its rank among the tile's old keys ONCE (binary search in shared
-// memory) and leaves a mark there; an inclusive scan of the marks gives, for every
-// position k, #adds < key_k and #dels < key_k over the tile's rows; subtracting the
-// earlier rows' counts (contiguous in the sorted lists, from the touch marks) leaves
-// the row-local counts of the shift
-//     new position = rowptr'[v] + (j − rowptr[v]) + #adds_v < key_j − #dels_v < key_j.
-// Consecutive threads take consecutive positions, so the stores coalesce.  Tiles
-// spanning more than kMergeRows rows (mean degree < 4) take a per-edge search path.
-constexpr int kMergeRows = 512;                  // rows whose rowptr / touch / new rowptr are cached
 constexpr int kMergeIPT = kMergeTile / 256;      // positions per thread
 
-__global__ void __launch_bounds__(256) k_merge2(const MergeArgs a) {
-  __shared__ int32_t scol[kMergeTile], srow[kMergeTile], smark[kMergeTile];   // marks: adds | dels << 16
-  __shared__ uint8_t sdl[kMergeTile];                                          // old edge deleted
-  __shared__ int32_t srp[kMergeRows + 1], snrp[kMergeRows];
-  __shared__ int4 stc[kMergeRows];
-  __shared__ int32_t s_lo, s_hi, s_rng[4], s_wsum[8];
-  const int64_t add_blocks = (int64_t)gridDim.x - a.old_tiles;      // added edges first: their searches
-  const int64_t tile = (int64_t)blockIdx.x - add_blocks;             // overlap the tiles instead of trailing
-  if (tile >= 0) {
-    const int64_t e0 = tile * kMergeTile;
-    const int64_t e1 = min(e0 + (int64_t)kMergeTile, a.E_old);
-    const int n = (int)(e1 - e0);
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    if (threadIdx.x == 0) {                            // rows [s_lo, s_hi] hold the tile's edges
-      s_lo = __ldg(a.tile_row + tile);
-      s_hi = tile + 1 < a.old_tiles ? __ldg(a.tile_row + tile + 1) : a.V - 1;
-      s_rng[0] = INT32_MAX; s_rng[1] = INT32_MIN; s_rng[2] = INT32_MAX; s_rng[3] = INT32_MIN;
-    }
+__global__ void __launch_bounds__(256) k_merge3(const MergeArgs a) {
+  __shared__ int32_t scol[kMergeTile];
+  __shared__ int32_t sa[kMergeTile];             // adds placed before position k; then A (global count)
+  __shared__ int32_t sd[kMergeTile];             // position k deleted; then D (global count)
+  __shared__ int32_t s_wa[8], s_wd[8], s_dend;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t t = blockIdx.x;
+  const int64_t e0 = t << kMergeShift;
+  const int64_t rem = a.E_old - e0;
+  const int n = rem <= 0 ? 0 : (rem < kMergeTile ? (int)rem : kMergeTile);
+  const int32_t a0 = __ldg(a.abnd + t), a1 = __ldg(a.abnd + t + 1);
+  const int32_t d0 = __ldg(a.dbnd + t), d1 = __ldg(a.dbnd + t + 1);
+#pragma unroll
+  for (int i = 0; i < kMergeIPT; ++i) {
+    const int k = threadIdx.x + i * 256;
+    if (k < n) scol[k] = __ldcs(a.ocol + e0 + k);
+    sa[k] = 0;
+    sd[k] = 0;
+  }
+  __syncthreads();
+  for (int32_t i = a0 + threadIdx.x; i < a1; i += 256) {   // (an add at the tile end: last tile only, k = n < kMergeTile)
+    const int k = (int)(__ldg(a.padd + i) - e0);
+    if (k < kMergeTile) atomicAdd(&sa[k], 1);
+  }
+  for (int32_t i = d0 + threadIdx.x; i < d1; i += 256) sd[__ldg(a.pdel + i) - e0] = 1;
+  __syncthreads();
+  {                                                  // A inclusive, D exclusive (thread: 8 consecutive positions)
+    int32_t ma[kMergeIPT], md[kMergeIPT];
+    int32_t ra = 0, rd = 0;
 #pragma unroll
     for (int i = 0; i < kMergeIPT; ++i) {
-      const int k = threadIdx.x + i * 256;
-      if (k < n) scol[k] = __ldcs(a.ocol + e0 + k);
-      srow[k] = -1;
-      smark[k] = 0;
-      sdl[k] = 0;
+      const int k = threadIdx.x * kMergeIPT + i;
+      ra += sa[k];
+      ma[i] = ra;                                    // inclusive
+      md[i] = rd;                                    // exclusive
+      rd += sd[k];
     }
-    __syncthreads();
-    const int32_t rlo = s_lo, rhi = s_hi, nr = rhi - rlo + 1;
-    bool cached = nr <= kMergeRows;                    // (the tile's rows: ~kMergeTile / mean degree)
-    if (cached) {
-      int32_t a0 = INT32_MAX, a1 = INT32_MIN, d0 = INT32_MAX, d1 = INT32_MIN;
-      for (int k = threadIdx.x; k <= nr; k += blockDim.x) {
-        srp[k] = __ldg(a.orowptr + rlo + k);
-        if (k < nr) {
-          const int4 t = __ldg(a.touch + rlo + k);
-          stc[k] = t;
-          snrp[k] = __ldg(a.nrowptr + rlo + k);
-          if (t.y > t.x) { a0 = min(a0, t.x); a1 = max(a1, t.y); }
-          if (t.w > t.z) { d0 = min(d0, t.z); d1 = max(d1, t.w); }
-        }
-      }
-      if (a1 > a0) { atomicMin(&s_rng[0], a0); atomicMax(&s_rng[1], a1); }
-      if (d1 > d0) { atomicMin(&s_rng[2], d0); atomicMax(&s_rng[3], d1); }
-      __syncthreads();
-      for (int k = threadIdx.x; k < nr; k += blockDim.x) {   // row-start marks (non-empty rows)
-        const int32_t b = srp[k], e = srp[k + 1];
-        if (e > b && b < e1) srow[max((int64_t)b - e0, (int64_t)0)] = k;
-      }
+    int32_t ia = ra, id = rd;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t ya = __shfl_up_sync(0xffffffffu, ia, o), yd = __shfl_up_sync(0xffffffffu, id, o);
+      if (lane >= o) { ia += ya; id += yd; }
     }
+    if (lane == 31) { s_wa[w] = ia; s_wd[w] = id; }
+    int32_t xa = ia - ra + a0, xd = id - rd + d0;
     __syncthreads();
-    // the tile rows' add / delete keys are the contiguous ranges [A0, A1), [D0, D1)
-    const int32_t A0 = s_rng[0], D0 = s_rng[2];
-    const int32_t na = s_rng[1] > A0 ? s_rng[1] - A0 : 0, nd = s_rng[3] > D0 ? s_rng[3] - D0 : 0;
-    cached = cached && na < 65536 && nd < 32768;       // 16-bit mark fields
-    if (cached) {                                      // inclusive max-scan of the row-start marks
-      int32_t m[kMergeIPT];
-      int32_t run = -1;
+    for (int ww = 0; ww < w; ++ww) { xa += s_wa[ww]; xd += s_wd[ww]; }
+    if (threadIdx.x == 255) s_dend = xd + rd;          // D at the tile end
 #pragma unroll
-      for (int i = 0; i < kMergeIPT; ++i) { run = max(run, srow[threadIdx.x * kMergeIPT + i]); m[i] = run; }
-      int32_t inc = run;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc = max(inc, y);
-      }
-      if (lane == 31) s_wsum[w] = inc;
-      int32_t ex = __shfl_up_sync(0xffffffffu, inc, 1);
-      if (lane == 0) ex = -1;
-      __syncthreads();
-      for (int ww = 0; ww < w; ++ww) ex = max(ex, s_wsum[ww]);
-#pragma unroll
-      for (int i = 0; i < kMergeIPT; ++i) srow[threadIdx.x * kMergeIPT + i] = max(ex, m[i]);
+    for (int i = 0; i < kMergeIPT; ++i) {
+      const int k = threadIdx.x * kMergeIPT + i;
+      sa[k] = xa + ma[i];
+      sd[k] = xd + md[i];
     }
-    __syncthreads();
-    if (cached) {                                      // ranks of the delta keys among the tile's old keys
-      const int nb = a.nb;
-      auto key_at = [&](int i) { return ((uint64_t)(rlo + srow[i]) << nb) | (uint64_t)(uint32_t)scol[i]; };
-      auto rank = [&](uint64_t key) {                  // # old tile keys < key
-        int lo = 0, hi = n;
-        while (lo < hi) { const int mid = (lo + hi) >> 1; if (key_at(mid) < key) lo = mid + 1; else hi = mid; }
-        return lo;
-      };
-      for (int i = threadIdx.x; i < na; i += blockDim.x) {   // add a counts for positions with key > a
-        const int r = rank(__ldg(a.add + A0 + i));
-        if (r < n) atomicAdd(&smark[r], 1);
-      }
-      for (int i = threadIdx.x; i < nd; i += blockDim.x) {   // delete d: removes its old edge, counts after it
-        const uint64_t key = __ldg(a.del + D0 + i);
-        const int r = rank(key);
-        if (r < n && key_at(r) == key) {
-          sdl[r] = 1;
-          if (r + 1 < n) atomicAdd(&smark[r + 1], 1 << 16);
-        } else if (r == 0) {
-          atomicAdd(&smark[0], 1 << 16);              // an old edge of the first row before the tile
-        }
-      }
-    }
-    __syncthreads();
-    if (cached) {                                      // inclusive scan of the packed marks
-      int32_t m[kMergeIPT];
-      int32_t run = 0;
-#pragma unroll
-      for (int i = 0; i < kMergeIPT; ++i) { run += smark[threadIdx.x * kMergeIPT + i]; m[i] = run; }
-      int32_t inc = run;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc += y;
-      }
-      if (lane == 31) s_wsum[w] = inc;
-      int32_t ex = inc - run;
-      __syncthreads();
-      for (int ww = 0; ww < w; ++ww) ex += s_wsum[ww];
-#pragma unroll
-      for (int i = 0; i < kMergeIPT; ++i) smark[threadIdx.x * kMergeIPT + i] = ex + m[i];
-    }
-    __syncthreads();
+  }
+  __syncthreads();
+  const int32_t dend = s_dend;
 #pragma unroll 2
-    for (int i = 0; i < kMergeIPT; ++i) {
-      const int k = threadIdx.x + i * 256;
-      if (k >= n) break;
-      const int64_t j = e0 + k;
-      int64_t pos;
-      if (cached) {
-        const int32_t r = srow[k];
-        const int4 t = stc[r];
-        const int32_t mk = smark[k];
-        const int32_t adds = t.y > t.x ? (mk & 0xffff) - (t.x - A0) : 0;
-        const int32_t dels = t.w > t.z ? (mk >> 16) - (t.z - D0) : 0;
-        pos = sdl[k] ? -1 : (int64_t)snrp[r] + (j - srp[r]) + adds - dels;
-      } else {                                         // per-edge searches in the global lists
-        const int32_t v = row_of(a.orowptr, rlo, rhi, j);
-        const int4 t = __ldg(a.touch + v);
-        pos = (int64_t)__ldg(a.nrowptr + v) + (j - __ldg(a.orowptr + v));
-        if (t.y != t.x || t.w != t.z) {
-          const uint64_t key = ((uint64_t)v << a.nb) | (uint64_t)(uint32_t)scol[k];
-          const int64_t al = lb_u64(a.add, t.x, t.y, key), dl = lb_u64(a.del, t.z, t.w, key);
-          if (dl < t.w && __ldg(a.del + dl) == key) pos = -1;
-          else pos += (al - t.x) - (dl - t.z);
-        }
+  for (int i = 0; i < kMergeIPT; ++i) {              // surviving old edges (coalesced)
+    const int k = threadIdx.x + i * 256;
+    if (k >= n) break;
+    const int64_t j = e0 + k;
+    const int32_t dk = sd[k], dk1 = k + 1 < kMergeTile ? sd[k + 1] : dend;
+    const int64_t pos = dk1 > dk ? -1 : j - dk + sa[k];
+    if (a.emap_out) a.emap_out[j] = (int32_t)pos;
+    if (pos < 0) continue;
+    a.ncol[pos] = scol[k];
+    if (a.eid_new) a.eid_new[pos] = __ldg(a.emap_in + __ldcs(a.eid_old + j));
+  }
+  const uint64_t mask = (uint64_t(1) << a.nb) - 1;
+  for (int32_t i = a0 + threadIdx.x; i < a1; i += 256) {   // the adds of this tile
+    const int32_t p = __ldg(a.padd + i);
+    const int k = (int)(p - e0);
+    const int64_t q = (int64_t)p - (k < kMergeTile ? sd[k] : dend) + i;
+    const uint64_t key = __ldg(a.add + i);
+    const int32_t v = (int32_t)(key >> a.nb), c = (int32_t)(key & mask);
+    a.ncol[q] = c;
+    if (a.eid_new) {                                  // label = position of (v -> c) in the new in-CSR
+      int32_t l2 = a.in_rowptr_new[c], h2 = a.in_rowptr_new[c + 1];
+      while (l2 < h2) {
+        const int32_t mid = (l2 + h2) >> 1;
+        if (a.in_col_new[mid] < v) l2 = mid + 1; else h2 = mid;
       }
-      if (a.emap_out) a.emap_out[j] = (int32_t)pos;
-      if (pos < 0) continue;
-      a.ncol[pos] = scol[k];
-      if (a.eid_new) a.eid_new[pos] = __ldg(a.emap_in + __ldcs(a.eid_old + j));
-    }
-  } else {                                            // added edges
-    const uint64_t mask = (uint64_t(1) << a.nb) - 1;
-    const int64_t nthr = add_blocks * blockDim.x;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.nadd; i += nthr) {
-      const uint64_t key = a.add[i];
-      const int32_t v = (int32_t)(key >> a.nb), c = (int32_t)(key & mask);
-      const int4 t = __ldg(a.touch + v);
-      int32_t lo = __ldg(a.orowptr + v), b = lo, e = __ldg(a.orowptr + v + 1);
-      while (b < e) {
-        const int32_t mid = (b + e) >> 1;
-        if (a.ocol[mid] < c) b = mid + 1; else e = mid;
-      }
-      const int64_t dl = lb_u64(a.del, t.z, t.w, key);
-      const int64_t pos = (int64_t)__ldg(a.nrowptr + v) + (i - t.x) + (b - lo) - (dl - t.z);
-      a.ncol[pos] = c;
-      if (a.eid_new) {                                // label = position of (v -> c) in the new in-CSR
-        int32_t l2 = a.in_rowptr_new[c], h2 = a.in_rowptr_new[c + 1];
-        while (l2 < h2) {
-          const int32_t mid = (l2 + h2) >> 1;
-          if (a.in_col_new[mid] < v) l2 = mid + 1; else h2 = mid;
-        }
-        a.eid_new[pos] = l2;
-      }
+      a.eid_new[q] = l2;
     }
   }
 }
@@ -762,21 +799,29 @@ stg_status ids_ws_reserve(BuildWs& ws, int32_t V, int64_t cap, cudaStream_t s) {
   const int64_t ntiles = ceil_div(V > 0 ? V : 1, kRowTile);
   STG_TRY(ws.ids_hist.alloc((size_t)kIdsBuckets * ntiles, s));
   STG_TRY(ws.ids_offs.alloc((size_t)kIdsBuckets * ntiles, s));
-  STG_TRY(ws.ids_tot.alloc(kIdsBuckets, s));
+  STG_TRY(ws.ids_tot.alloc(3 * kIdsBuckets, s));   // totals | bucket chunk bases | bucket row bases
   STG_TRY(ws.sat_tmp.alloc((size_t)std::min<int64_t>(V, cap / kIdsSat + 1), s));
   if (ws.lb_status.n < (size_t)ntiles || !ws.lb_status.p) {     // fresh status words: never a valid epoch
     STG_TRY(ws.lb_status.alloc((size_t)ntiles, s));
     STG_CUDA(cudaMemsetAsync(ws.lb_status.p, 0, sizeof(uint64_t) * ws.lb_status.n, s));
   }
-  STG_TRY(ws.lb_ticket.alloc(1, s));
-  STG_TRY(ws.merge_rows.alloc((size_t)ceil_div(cap > 0 ? cap : 1, kMergeTile) + 1, s));
+  if (!ws.lb_ticket.p) {                                // a monotone ticket counter: no reset per scan
+    STG_TRY(ws.lb_ticket.alloc(1, s));
+    STG_CUDA(cudaMemsetAsync(ws.lb_ticket.p, 0, sizeof(uint32_t), s));
+    ws.lb_base = 0;
+  }
+  if (ws.gdeg.n < 2 * (size_t)V || !ws.gdeg.p) {        // whole-graph degree deltas: zero between steps
+    STG_TRY(ws.gdeg.alloc(2 * (size_t)(V > 0 ? V : 1), s));
+    STG_CUDA(cudaMemsetAsync(ws.gdeg.p, 0, sizeof(int32_t) * ws.gdeg.n, s));
+  }
   return STG_OK;
 }
 
 // node_ids + schedule of one direction whose key histogram is already in ws.ids_hist
 static stg_status ids_sched_from_hist(const int32_t* deg, const int32_t* rowptr, int32_t V, int32_t R, int32_t* ids,
                                       int32_t* sched, int64_t cap, BuildWs& ws, cudaStream_t s, int32_t rb,
-                                      int32_t re, const DirDelta* clear, int nb, int4* touch) {
+                                      int32_t re, const DirDelta* clear, int nb, int4* touch,
+                                      const DirDelta* gclear = nullptr) {
   const int32_t ntiles = (int32_t)ceil_div(V, kRowTile);
   k_ids_offsets<<<(kIdsBuckets + 31) / 32, 1024, 0, s>>>(ws.ids_hist.p, ntiles, ws.ids_offs.p, ws.ids_tot.p);
   k_ids_scatter<<<ntiles, kRowThreads, 0, s>>>(deg, V, rb, re, ws.ids_offs.p, ws.ids_tot.p, ntiles, ids);
@@ -793,12 +838,14 @@ static stg_status ids_sched_from_hist(const int32_t* deg, const int32_t* rowptr,
   }
   const int64_t coff = sched_cptr_off(V, cap);
   k_ids_finish<<<1, 1024, kSatSortMax * sizeof(uint64_t), s>>>(ids, deg, ws.ids_tot.p, R, coff, sched,
-                                                                ws.sat_tmp.p);
+                                                                ws.sat_tmp.p, ws.ids_tot.p + kIdsBuckets);
   const int64_t icap = sched_items_cap(V, cap);
-  const int64_t nclr = clear ? clear->nadd + clear->ndel : 0;
+  const int64_t nclr = std::max<int64_t>(clear ? clear->nadd + clear->ndel : 0, gclear ? gclear->nadd + gclear->ndel : 0);
   k_items2<<<grid_n(std::max<int64_t>(std::min<int64_t>(icap, (int64_t)R + cap / kHubChunk + 2), nclr)), 256, 0, s>>>(
-      ids, rowptr, icap, sched, clear ? clear->add : nullptr, clear ? clear->nadd : 0, clear ? clear->del : nullptr,
-      clear ? clear->ndel : 0, nb, touch);
+      ids, rowptr, icap, sched, ws.ids_tot.p + kIdsBuckets, clear ? clear->add : nullptr, clear ? clear->nadd : 0,
+      clear ? clear->del : nullptr, clear ? clear->ndel : 0, nb, touch, gclear ? gclear->add : nullptr,
+      gclear ? gclear->nadd : 0, gclear ? gclear->del : nullptr, gclear ? gclear->ndel : 0,
+      gclear ? ws.gdeg.p : nullptr, gclear ? ws.gdeg.p + V : nullptr);
   count_launch(4);
   return check_launch("ids_sched");
 }
@@ -828,12 +875,30 @@ stg_status degree_hist2(const DirDelta& d, int nb, int sign, int32_t* gin, int32
 // write the GCN norms of dst from its whole-graph degrees (gin / gout).
 stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const DirDelta& d, int4* touch, BuildWs& ws,
                       cudaStream_t s, bool norms, int32_t* emap_out, const int32_t* emap_in, const int32_t* eid_old,
-                      int32_t* eid_new, const int32_t* in_rowptr_new, const int32_t* in_col_new) {
+                      int32_t* eid_new, const int32_t* in_rowptr_new, const int32_t* in_col_new,
+                      const GDegStep* gdeg) {
   const int32_t V = src.V;
   STG_TRY(ids_ws_reserve(ws, V, dst.cap, s));
   const int32_t ntiles = (int32_t)ceil_div(V, kRowTile);
-  if (d.nadd + d.ndel > 0) {
-    k_touch2<<<grid_n(d.nadd + d.ndel), 256, 0, s>>>(d.add, d.nadd, d.del, d.ndel, src.nb, touch);
+  if (gdeg && !norms) return fail(STG_ERR_STATE, "apply_dir2: the degree step rides on the norms pass");
+  const int64_t ng = gdeg ? gdeg->keys.nadd + gdeg->keys.ndel : 0;
+  const int64_t nk = d.nadd + d.ndel;
+  const int32_t ntm = (int32_t)(src.E >> kMergeShift) + 1;    // merge tiles: positions [0, E_old]
+  STG_TRY(ws.mpos.alloc((size_t)std::max<int64_t>(nk, 1), s));
+  STG_TRY(ws.mbnd.alloc(2 * ((size_t)ntm + 1), s));
+  const int32_t* orowptr = in_dir ? src.in_rowptr.p : src.out_rowptr.p;
+  const int32_t* ocol = in_dir ? src.in_col.p : src.out_col.p;
+  {                                                      // touch marks, merge positions, (whole-graph degrees)
+    TouchArgs t{};
+    t.add = d.add; t.nadd = d.nadd; t.del = d.del; t.ndel = d.ndel; t.nb = src.nb;
+    t.touch = touch; t.orowptr = orowptr; t.ocol = ocol;
+    t.padd = ws.mpos.p; t.pdel = ws.mpos.p + d.nadd;
+    t.abnd = ws.mbnd.p; t.dbnd = ws.mbnd.p + ntm + 1; t.ntm = ntm;
+    if (ng > 0) {
+      t.gadd = gdeg->keys.add; t.ngadd = gdeg->keys.nadd; t.gdel = gdeg->keys.del; t.ngdel = gdeg->keys.ndel;
+      t.sign = gdeg->sign; t.din = ws.gdeg.p; t.dout = ws.gdeg.p + V;
+    }
+    k_touch3<<<grid_n(std::max<int64_t>(std::max<int64_t>(nk, ng), 1)), 256, 0, s>>>(t);
     count_launch();
   }
   const bool blk = in_dir && dst.sharded;
@@ -853,34 +918,32 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
   if (norms) {
     a.gin = dst.gin_deg.p; a.gout = dst.gout_deg.p; a.dgl_both = dst.dgl_both;
     a.norm_src = dst.norm_src.p; a.norm_dst = dst.norm_dst.p;
+    if (gdeg) {                                          // dst's degrees = src's + this step's deltas
+      a.gin = gdeg->gin_src; a.gout = gdeg->gout_src;
+      a.din = ws.gdeg.p; a.dout = ws.gdeg.p + V;
+      a.gin_w = gdeg->gin_dst; a.gout_w = gdeg->gout_dst;
+    }
   }
-  a.orowptr = in_dir ? src.in_rowptr.p : src.out_rowptr.p;
-  a.tile_row = ws.merge_rows.p;
-  STG_CUDA(cudaMemsetAsync(ws.lb_ticket.p, 0, sizeof(uint32_t), s));
+  a.tbase = ws.lb_base;
+  ws.lb_base += (uint32_t)ntiles;                        // every tile claims one ticket
   k_rowscan<true><<<ntiles, kRowThreads, 0, s>>>(a);
   count_launch();
   MergeArgs m{};
-  m.V = V; m.nb = src.nb;
-  m.orowptr = in_dir ? src.in_rowptr.p : src.out_rowptr.p;
-  m.ocol = in_dir ? src.in_col.p : src.out_col.p;
+  m.nb = src.nb;
+  m.ocol = ocol;
   m.E_old = src.E;
-  m.nrowptr = a.rowptr_new;
-  m.touch = touch;
-  m.add = d.add; m.nadd = d.nadd; m.del = d.del;
+  m.add = d.add;
+  m.padd = ws.mpos.p; m.pdel = ws.mpos.p + d.nadd;
+  m.abnd = ws.mbnd.p; m.dbnd = ws.mbnd.p + ntm + 1;
   m.ncol = in_dir ? dst.in_col.p : dst.out_col.p;
-  m.old_tiles = ceil_div(src.E, kMergeTile);
   m.emap_out = emap_out; m.emap_in = emap_in; m.eid_old = eid_old; m.eid_new = eid_new;
   m.in_rowptr_new = in_rowptr_new; m.in_col_new = in_col_new;
-  m.tile_row = ws.merge_rows.p;
-  const int64_t add_blocks = d.nadd > 0 ? std::min<int64_t>(ceil_div(d.nadd, 256), 4 * 148) : 0;
-  if (m.old_tiles + add_blocks > 0) {
-    k_merge2<<<(unsigned)(m.old_tiles + add_blocks), 256, 0, s>>>(m);
-    count_launch();
-  }
+  k_merge3<<<(unsigned)ntm, 256, 0, s>>>(m);
+  count_launch();
   const int32_t R = blk ? dst.rows() : V;
   return ids_sched_from_hist(a.deg_new, a.rowptr_new, V, R, in_dir ? dst.in_ids.p : dst.out_ids.p,
                              in_dir ? dst.in_sched.p : dst.out_sched.p, dst.cap, ws, s, a.rb, a.re, &d, src.nb,
-                             touch);
+                             touch, gdeg ? &gdeg->keys : nullptr);
 }
 
 }  // namespace stg

@@ -200,3 +200,59 @@ def test_snapshot_parts_rejects_bad_mask(stg):
         with pytest.raises(stg.StgError) as e:
             stg.stg_dtdg_get_snapshot_parts(g, 1, bad)
         assert e.value.status == 1
+
+
+def _merge_cases(seed=0, V=5000):
+    """Batches aimed at the snapshot merge (snapshot.cu k_touch3 / k_merge3): a base of
+    exactly 3 merge tiles (3·2048 unique edges), thousands of adds at ONE insertion point
+    (a row gaining edges past its last one, the last row of the graph: adds at the very
+    end), deletes at merge-tile boundaries and of whole rows, a step that empties the
+    graph and one that refills it from nothing."""
+    rng = np.random.default_rng(seed)
+    flat = rng.choice(V * V, 3 * 2048, replace=False)
+    s0, d0 = (flat // V).astype(np.int64), (flat % V).astype(np.int64)
+    key0 = np.sort(d0 * V + s0)                 # in-CSR order (dst, src)
+    A, D = [(np.zeros(0, int), np.zeros(0, int))], [(np.zeros(0, int), np.zeros(0, int))]
+    # t=1: row 17 (in-CSR row = dst) gains 3000 sources > all of its current ones; the last
+    # row V-1 gains 2500 (adds at the very end of the old CSR); 200 random adds
+    A.append((np.concatenate([np.arange(V - 3000, V), np.arange(V - 2500, V), rng.integers(0, V, 200)]),
+              np.concatenate([np.full(3000, 17), np.full(2500, V - 1), rng.integers(0, V, 200)])))
+    D.append((np.zeros(0, int), np.zeros(0, int)))
+    # t=2: delete the edges at old in-CSR positions 0, 2047, 2048, 4095, 4096 (tile boundaries, t=0
+    # order is a superset here: pick them from the base keys) and all of row 17's new sources
+    pick = key0[[0, 2047, 2048, 4095, 4096, 6143]]
+    D.append((np.concatenate([pick % V, np.arange(V - 3000, V)]), np.concatenate([pick // V, np.full(3000, 17)])))
+    A.append((rng.integers(0, V, 100), rng.integers(0, V, 100)))
+    # t=3: delete everything that can exist (the oracle normalises absent deletes away)
+    allk = np.unique(np.concatenate([key0, (A[1][1] * V + A[1][0]), (A[2][1] * V + A[2][0])]))
+    D.append((allk % V, allk // V))
+    A.append((np.zeros(0, int), np.zeros(0, int)))
+    # t=4: refill from an empty graph; t=5: a mixed step
+    A.append((rng.integers(0, V, 4000), rng.integers(0, V, 4000)))
+    D.append((np.zeros(0, int), np.zeros(0, int)))
+    A.append((rng.integers(0, V, 3000), rng.integers(0, V, 3000)))
+    D.append((rng.integers(0, V, 3000), rng.integers(0, V, 3000)))
+    off = lambda L: np.concatenate([[0], np.cumsum([x[0].size for x in L])]).astype(np.int64)
+    cat = lambda L, i: np.concatenate([x[i] for x in L]).astype(np.int32)
+    return gen.DTDG(V=V, T=len(A), W=0, slide=0, ev_src=None, ev_dst=None, src0=s0.astype(np.int32),
+                    dst0=d0.astype(np.int32), add_off=off(A), add_src=cat(A, 0), add_dst=cat(A, 1),
+                    del_off=off(D), del_src=cat(D, 0), del_dst=cat(D, 1))
+
+
+@pytest.mark.parametrize("loops", [False, True])
+def test_merge_edge_cases(stg, loops):
+    d = _merge_cases()
+    refs = _oracle_snaps(d, loops)
+    assert refs[3]["E"] == (d.V if loops else 0)          # the emptied snapshot
+    g = _create(stg, d, stg.STG_EDGE_IDS | (stg.STG_SELF_LOOPS if loops else 0))
+    for t in range(d.T):
+        assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_snapshot(g, t)), refs[t], tag=("merge", t))
+    for t in reversed(range(d.T)):
+        assert_graph_equal(stg.view_arrays(stg.stg_dtdg_get_backward_snapshot(g, t)), refs[t], tag=("merge", "b", t))
+    IN, OUT = stg.STG_PART_IN, stg.STG_PART_OUT
+    g2 = _create(stg, d, stg.STG_SELF_LOOPS if loops else 0)
+    for t in range(d.T):
+        _check_parts(stg.view_arrays(stg.stg_dtdg_get_snapshot_parts(g2, t, IN)), refs[t], IN, ("min", t))
+    for t in reversed(range(d.T)):
+        _check_parts(stg.view_arrays(stg.stg_dtdg_get_snapshot_parts(g2, t, OUT, backward=True)), refs[t], OUT,
+                     ("mout", t))
