@@ -5,15 +5,16 @@
 //   one delta step of one CSR direction (apply_dir2):
 //     k_touch3       mark the sorted add / delete ranges of every touched row;
 //                    place every delta key in the OLD CSR (its merge-path
-//                    position) and the merge tiles' first add / delete; the
-//                    whole-graph degree deltas of the step (GCN norms)
+//                    position); the whole-graph degree deltas of the step
 //     k_rowscan      single-pass scan (decoupled look-back) of the new degrees
 //                    deg' = deg + |adds| - |dels| -> rowptr', deg', the
-//                    whole-graph degrees and GCN norms, and the per-tile
-//                    histogram of the node_ids key
-//     k_merge3       global merge path over the sorted (row, col) keys: old
+//                    whole-graph degrees and GCN norms, the per-tile
+//                    histogram of the node_ids key, and the merge tiles'
+//                    first add / delete
+//     k_merge4       global merge path over the sorted (row, col) keys: old
 //                    edge j -> j - #dels before j + #adds placed <= j, add i at
-//                    old position p -> p - #dels before p + i (no row lookups)
+//                    old position p -> p - #dels before p + i (a warp per 256
+//                    old positions; no row lookups, no shared memory)
 //   node_ids + schedule (ids_sched_build):
 //     k_ids_offsets  one CTA: digit-major exclusive scan of the tile histograms
 //     k_ids_scatter  stable counting-sort scatter (warp match_any ranks)
@@ -60,10 +61,7 @@ __device__ __forceinline__ int ids_digit(int32_t v, int32_t d, int32_t rb, int32
 //   padd[i] / pdel[i] = the key's position in the OLD CSR (insertion point of an
 //     add = number of old keys below it; a delete's own position) — old CSR
 //     positions are the global (row, col) key order, so these are the merge
-//     path of k_merge3;
-//   abnd[t] / dbnd[t] = adds / deletes whose position lies in merge tiles < t
-//     (positions are monotone in the sorted lists: each key writes the tiles
-//     between its predecessor's and its own; t in [0, ntm]);
+//     path of k_merge4;
 //   (gdeg) the whole-graph degree deltas into the zeroed scratch din / dout.
 struct TouchArgs {
   const uint64_t* add;
@@ -76,9 +74,6 @@ struct TouchArgs {
   const int32_t* ocol;
   int32_t* padd;
   int32_t* pdel;
-  int32_t* abnd;
-  int32_t* dbnd;
-  int32_t ntm;                  // merge tiles (positions [0, E_old] map to tiles [0, ntm))
   const uint64_t* gadd;         // whole-graph keys (may be NULL)
   int64_t ngadd;
   const uint64_t* gdel;
@@ -88,8 +83,8 @@ struct TouchArgs {
   int32_t* dout;
 };
 
-constexpr int kMergeShift = 11;
-constexpr int kMergeTile = 1 << kMergeShift;     // old edges per merge CTA
+constexpr int kMergeShift = 8;
+constexpr int kMergeTile = 1 << kMergeShift;     // old positions per merge warp task
 
 __device__ __forceinline__ int32_t old_pos(const int32_t* __restrict__ orowptr, const int32_t* __restrict__ ocol,
                                            uint64_t key, int nb) {
@@ -105,14 +100,9 @@ __device__ __forceinline__ int32_t old_pos(const int32_t* __restrict__ orowptr, 
 __global__ void __launch_bounds__(256) k_touch3(const TouchArgs a) {
   const int64_t n = a.nadd + a.ndel, ng = a.ngadd + a.ngdel;
   const uint64_t gmask = (uint64_t(1) << a.nb) - 1;
-  const int lane = threadIdx.x & 31;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  if (n == 0 && blockIdx.x == 0) {                     // no keys: every tile starts at entry 0
-    for (int t = threadIdx.x; t <= a.ntm; t += blockDim.x) { a.abnd[t] = 0; a.dbnd[t] = 0; }
-  }
   const int64_t kend = max(n, ng);
-  for (int64_t k0 = blockIdx.x * (int64_t)blockDim.x; k0 < kend; k0 += stride) {   // warp-uniform trip count
-    const int64_t k = k0 + threadIdx.x;
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < kend; k += stride) {
     if (k < ng) {
       const uint64_t key = k < a.ngadd ? a.gadd[k] : a.gdel[k - a.ngadd];
       const int sg = k < a.ngadd ? a.sign : -a.sign;
@@ -124,7 +114,6 @@ __global__ void __launch_bounds__(256) k_touch3(const TouchArgs a) {
     const uint64_t* d = is_add ? a.add : a.del;
     const int64_t m = is_add ? a.nadd : a.ndel;
     const int64_t i = is_add ? k : k - a.nadd;
-    int32_t p = 0;
     if (on) {
       const uint64_t key = d[i];
       const int32_t r = (int32_t)(key >> a.nb);
@@ -133,28 +122,11 @@ __global__ void __launch_bounds__(256) k_touch3(const TouchArgs a) {
       int* t = reinterpret_cast<int*>(a.touch + r);
       if (first) t[is_add ? 0 : 2] = (int)i;
       if (last) t[is_add ? 1 : 3] = (int)(i + 1);
-      p = old_pos(a.orowptr, a.ocol, key, a.nb);
-      (is_add ? a.padd : a.pdel)[i] = p;
+      (is_add ? a.padd : a.pdel)[i] = old_pos(a.orowptr, a.ocol, key, a.nb);
     }
-    // tile boundaries: the predecessor's position from the previous lane (same list), else searched
-    const int32_t pl = __shfl_up_sync(0xffffffffu, p, 1);
-    if (on) {
-      int32_t tp = -1;
-      if (i > 0) tp = (lane > 0 && k - 1 >= (is_add ? 0 : a.nadd)) ? (pl >> kMergeShift)
-                                                                  : (old_pos(a.orowptr, a.ocol, d[i - 1], a.nb) >> kMergeShift);
-      int32_t* bnd = is_add ? a.abnd : a.dbnd;
-      const int32_t ti = p >> kMergeShift;
-      for (int32_t t = tp + 1; t <= ti; ++t) bnd[t] = (int32_t)i;
-      if (i == m - 1)
-        for (int32_t t = ti + 1; t <= a.ntm; ++t) bnd[t] = (int32_t)m;
-    }
-  }
-  // one list empty (the other not): its tiles all start at entry 0
-  if (n > 0 && blockIdx.x == 0) {
-    if (a.nadd == 0) for (int t = threadIdx.x; t <= a.ntm; t += blockDim.x) a.abnd[t] = 0;
-    if (a.ndel == 0) for (int t = threadIdx.x; t <= a.ntm; t += blockDim.x) a.dbnd[t] = 0;
   }
 }
+
 
 // whole-graph degree histogram of the add (+sign) and delete (-sign) batches
 __global__ void k_degree_hist2(const uint64_t* __restrict__ add, int64_t nadd, const uint64_t* __restrict__ del,
@@ -208,7 +180,28 @@ struct RowScanArgs {
   const int32_t* dout;
   int32_t* gin_w;
   int32_t* gout_w;
+  // (TOUCH) merge-tile boundaries from the old-CSR positions of k_touch3:
+  // abnd[t] / dbnd[t] = adds / deletes placed in merge tiles < t, t in [0, ntm]
+  const int32_t* padd;
+  int64_t nadd;
+  const int32_t* pdel;
+  int64_t ndel;
+  int32_t* abnd;
+  int32_t* dbnd;
+  int32_t ntm;
 };
+
+// B[t] = entries of the sorted position list P[0, n) in tiles < t (t in [0, ntm]):
+// positions are monotone, so entry i writes the tiles between its predecessor's and
+// its own (entry n: up to ntm)
+__device__ __forceinline__ void tile_bounds(const int32_t* __restrict__ P, int64_t n, int32_t ntm,
+                                            int32_t* __restrict__ B, int64_t gid, int64_t gstride) {
+  for (int64_t i = gid; i <= n; i += gstride) {
+    const int32_t tp = i > 0 ? (__ldg(P + i - 1) >> kMergeShift) : -1;
+    const int32_t ti = i < n ? (__ldg(P + i) >> kMergeShift) : ntm;
+    for (int32_t t = tp + 1; t <= ti; ++t) B[t] = (int32_t)i;
+  }
+}
 
 template <bool TOUCH>
 __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
@@ -329,6 +322,11 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
         s_prefix = prefix;
         if ((int64_t)(tile + 1) * kRowTile >= a.V) a.rowptr_new[a.V] = (int32_t)(prefix + tot);
       }
+    } else if (a.abnd) {                                // warps 1..7 meanwhile: the merge-tile boundaries
+      constexpr int kB = kRowThreads - 32;
+      const int64_t gid = (int64_t)tile * kB + (threadIdx.x - 32), gs = (int64_t)a.ntiles * kB;
+      tile_bounds(a.padd, a.nadd, a.ntm, a.abnd, gid, gs);
+      tile_bounds(a.pdel, a.ndel, a.ntm, a.dbnd, gid, gs);
     }
     __syncthreads();
     const int64_t pre = s_prefix;
@@ -672,10 +670,7 @@ __global__ void k_items2(const int32_t* __restrict__ ids, const int32_t* __restr
 // A(j) = adds whose insertion point p <= j (k_touch3):
 //   surviving old edge j  ->  j − D(j) + A(j)
 //   added key i (point p) ->  p − D(p) + i
-// (rows need not be known: rowptr' comes from the degree scan).  A CTA owns
-// kMergeTile old positions plus the adds / deletes placed in them (contiguous
-// ranges of the sorted lists, from abnd / dbnd): marks in shared memory, one
-// block scan, then coalesced stores of the old edges and the adds.
+// (rows need not be known: rowptr' comes from the degree scan).
 struct MergeArgs {
   int nb;
   const int32_t* ocol;
@@ -697,92 +692,105 @@ struct MergeArgs {
   const int32_t* in_col_new;
 };
 
-constexpr int kMergeIPT = kMergeTile / 256;      // positions per thread
+// One warp per merge tile of kMergeTile old positions, in rounds of 32 (lane =
+// position, so loads and stores coalesce).  The tile's adds / deletes are the
+// contiguous ranges [a0, a1) / [d0, d1) of the sorted lists (k_rowscan); the warp
+// loads all its old columns and the first 32 entries of each range (with the
+// add keys) in one go, then per round every lane counts the entries before its
+// own position with a warp-uniform loop over the round's entries (typically 0-2;
+// a range longer than 32 reloads its next 32).  The list index where a round
+// starts is the count of entries before it, so
+//   D(j) = deletes before j,  A(j) = adds placed at or before j
+// are global without any scan.  No shared memory, no block synchronisation.
+constexpr int kMergeRounds = kMergeTile / 32;
 
-__global__ void __launch_bounds__(256) k_merge3(const MergeArgs a) {
-  __shared__ int32_t scol[kMergeTile];
-  __shared__ int32_t sa[kMergeTile];             // adds placed before position k; then A (global count)
-  __shared__ int32_t sd[kMergeTile];             // position k deleted; then D (global count)
-  __shared__ int32_t s_wa[8], s_wd[8], s_dend;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t t = blockIdx.x;
-  const int64_t e0 = t << kMergeShift;
-  const int64_t rem = a.E_old - e0;
-  const int n = rem <= 0 ? 0 : (rem < kMergeTile ? (int)rem : kMergeTile);
-  const int32_t a0 = __ldg(a.abnd + t), a1 = __ldg(a.abnd + t + 1);
-  const int32_t d0 = __ldg(a.dbnd + t), d1 = __ldg(a.dbnd + t + 1);
-#pragma unroll
-  for (int i = 0; i < kMergeIPT; ++i) {
-    const int k = threadIdx.x + i * 256;
-    if (k < n) scol[k] = __ldcs(a.ocol + e0 + k);
-    sa[k] = 0;
-    sd[k] = 0;
-  }
-  __syncthreads();
-  for (int32_t i = a0 + threadIdx.x; i < a1; i += 256) {   // (an add at the tile end: last tile only, k = n < kMergeTile)
-    const int k = (int)(__ldg(a.padd + i) - e0);
-    if (k < kMergeTile) atomicAdd(&sa[k], 1);
-  }
-  for (int32_t i = d0 + threadIdx.x; i < d1; i += 256) sd[__ldg(a.pdel + i) - e0] = 1;
-  __syncthreads();
-  {                                                  // A inclusive, D exclusive (thread: 8 consecutive positions)
-    int32_t ma[kMergeIPT], md[kMergeIPT];
-    int32_t ra = 0, rd = 0;
-#pragma unroll
-    for (int i = 0; i < kMergeIPT; ++i) {
-      const int k = threadIdx.x * kMergeIPT + i;
-      ra += sa[k];
-      ma[i] = ra;                                    // inclusive
-      md[i] = rd;                                    // exclusive
-      rd += sd[k];
-    }
-    int32_t ia = ra, id = rd;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int32_t ya = __shfl_up_sync(0xffffffffu, ia, o), yd = __shfl_up_sync(0xffffffffu, id, o);
-      if (lane >= o) { ia += ya; id += yd; }
-    }
-    if (lane == 31) { s_wa[w] = ia; s_wd[w] = id; }
-    int32_t xa = ia - ra + a0, xd = id - rd + d0;
-    __syncthreads();
-    for (int ww = 0; ww < w; ++ww) { xa += s_wa[ww]; xd += s_wd[ww]; }
-    if (threadIdx.x == 255) s_dend = xd + rd;          // D at the tile end
-#pragma unroll
-    for (int i = 0; i < kMergeIPT; ++i) {
-      const int k = threadIdx.x * kMergeIPT + i;
-      sa[k] = xa + ma[i];
-      sd[k] = xd + md[i];
-    }
-  }
-  __syncthreads();
-  const int32_t dend = s_dend;
-#pragma unroll 2
-  for (int i = 0; i < kMergeIPT; ++i) {              // surviving old edges (coalesced)
-    const int k = threadIdx.x + i * 256;
-    if (k >= n) break;
-    const int64_t j = e0 + k;
-    const int32_t dk = sd[k], dk1 = k + 1 < kMergeTile ? sd[k + 1] : dend;
-    const int64_t pos = dk1 > dk ? -1 : j - dk + sa[k];
-    if (a.emap_out) a.emap_out[j] = (int32_t)pos;
-    if (pos < 0) continue;
-    a.ncol[pos] = scol[k];
-    if (a.eid_new) a.eid_new[pos] = __ldg(a.emap_in + __ldcs(a.eid_old + j));
-  }
+struct MergeChunk {              // 32 consecutive entries of a sorted position list, one per lane
+  int32_t base;                  // list index of lane 0's entry
+  int32_t off;                   // entries of the chunk consumed
+  int32_t p;                     // this lane's position (INT32_MAX past the range)
+  int32_t idx;                   // this lane's list index
+};
+
+__device__ __forceinline__ void chunk_load(MergeChunk& ch, const int32_t* __restrict__ P, int32_t base, int32_t end,
+                                           int lane) {
+  ch.base = base;
+  ch.off = 0;
+  ch.idx = base + lane;
+  ch.p = ch.idx < end ? __ldg(P + ch.idx) : INT32_MAX;
+}
+
+template <bool LABELS>
+__global__ void __launch_bounds__(256, LABELS ? 5 : 8) k_merge4(const MergeArgs a, int32_t ntm) {
+  const unsigned FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const int32_t t = (int32_t)(blockIdx.x * 8 + (threadIdx.x >> 5));
+  if (t >= ntm) return;                               // (warp-uniform)
+  const int64_t e0 = (int64_t)t << kMergeShift;
+  const int32_t a1 = __ldg(a.abnd + t + 1), d1 = __ldg(a.dbnd + t + 1);
+  const int32_t a0 = __ldg(a.abnd + t), d0 = __ldg(a.dbnd + t);
   const uint64_t mask = (uint64_t(1) << a.nb) - 1;
-  for (int32_t i = a0 + threadIdx.x; i < a1; i += 256) {   // the adds of this tile
-    const int32_t p = __ldg(a.padd + i);
-    const int k = (int)(p - e0);
-    const int64_t q = (int64_t)p - (k < kMergeTile ? sd[k] : dend) + i;
-    const uint64_t key = __ldg(a.add + i);
-    const int32_t v = (int32_t)(key >> a.nb), c = (int32_t)(key & mask);
-    a.ncol[q] = c;
-    if (a.eid_new) {                                  // label = position of (v -> c) in the new in-CSR
-      int32_t l2 = a.in_rowptr_new[c], h2 = a.in_rowptr_new[c + 1];
-      while (l2 < h2) {
-        const int32_t mid = (l2 + h2) >> 1;
-        if (a.in_col_new[mid] < v) l2 = mid + 1; else h2 = mid;
+  int32_t c[kMergeRounds], eo[LABELS ? kMergeRounds : 1];
+#pragma unroll
+  for (int r = 0; r < kMergeRounds; ++r) {            // every old column of the tile in flight
+    const int64_t j = e0 + r * 32 + lane;
+    c[r] = j < a.E_old ? __ldcs(a.ocol + j) : 0;
+    if (LABELS) eo[r] = j < a.E_old ? __ldcs(a.eid_old + j) : 0;
+  }
+  MergeChunk cd, ca;
+  chunk_load(cd, a.pdel, d0, d1, lane);
+  chunk_load(ca, a.padd, a0, a1, lane);
+  uint64_t key = ca.idx < a1 ? __ldg(a.add + ca.idx) : 0;
+#pragma unroll
+  for (int r = 0; r < kMergeRounds; ++r) {
+    const int64_t base = e0 + r * 32;
+    const int64_t j = base + lane;
+    // deletes of this round
+    int32_t D = cd.base + cd.off;                     // deletes before the round
+    bool deleted = false;
+    while (true) {
+      const int nin = __popc(__ballot_sync(FULL, lane >= cd.off && cd.p < base + 32));
+      for (int l = cd.off; l < cd.off + nin; ++l) {
+        const int32_t ql = __shfl_sync(FULL, cd.p, l);
+        D += ql < j;
+        deleted |= ql == j;
       }
-      a.eid_new[q] = l2;
+      cd.off += nin;
+      if (cd.off < 32 || cd.base + 32 >= d1) break;
+      chunk_load(cd, a.pdel, cd.base + 32, d1, lane);  // (a range longer than 32)
+    }
+    // adds of this round: count, and place them (the deletes before an add's point
+    // p are lane (p - base)'s D)
+    int32_t A = ca.base + ca.off;
+    while (true) {
+      const bool in = lane >= ca.off && ca.p < base + 32;
+      const int nin = __popc(__ballot_sync(FULL, in));
+      for (int l = ca.off; l < ca.off + nin; ++l) A += __shfl_sync(FULL, ca.p, l) <= j;
+      const int32_t Dp = __shfl_sync(FULL, D, in ? (int)(ca.p - base) : 0);
+      if (in) {
+        const int64_t q = (int64_t)ca.p - Dp + ca.idx;
+        const int32_t v = (int32_t)(key >> a.nb), cc = (int32_t)(key & mask);
+        a.ncol[q] = cc;
+        if (LABELS) {                                 // label = position of (v -> cc) in the new in-CSR
+          int32_t l2 = a.in_rowptr_new[cc], h2 = a.in_rowptr_new[cc + 1];
+          while (l2 < h2) {
+            const int32_t mid = (l2 + h2) >> 1;
+            if (a.in_col_new[mid] < v) l2 = mid + 1; else h2 = mid;
+          }
+          a.eid_new[q] = l2;
+        }
+      }
+      ca.off += nin;
+      if (ca.off < 32 || ca.base + 32 >= a1) break;
+      chunk_load(ca, a.padd, ca.base + 32, a1, lane);
+      key = ca.idx < a1 ? __ldg(a.add + ca.idx) : 0;
+    }
+    if (j < a.E_old) {                                // the surviving old edges
+      const int64_t pos = deleted ? -1 : j - D + A;
+      if (a.emap_out) a.emap_out[j] = (int32_t)pos;
+      if (!deleted) {
+        a.ncol[pos] = c[r];
+        if (LABELS) a.eid_new[pos] = __ldg(a.emap_in + eo[LABELS ? r : 0]);
+      }
     }
   }
 }
@@ -893,7 +901,6 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
     t.add = d.add; t.nadd = d.nadd; t.del = d.del; t.ndel = d.ndel; t.nb = src.nb;
     t.touch = touch; t.orowptr = orowptr; t.ocol = ocol;
     t.padd = ws.mpos.p; t.pdel = ws.mpos.p + d.nadd;
-    t.abnd = ws.mbnd.p; t.dbnd = ws.mbnd.p + ntm + 1; t.ntm = ntm;
     if (ng > 0) {
       t.gadd = gdeg->keys.add; t.ngadd = gdeg->keys.nadd; t.gdel = gdeg->keys.del; t.ngdel = gdeg->keys.ndel;
       t.sign = gdeg->sign; t.din = ws.gdeg.p; t.dout = ws.gdeg.p + V;
@@ -924,6 +931,8 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
       a.gin_w = gdeg->gin_dst; a.gout_w = gdeg->gout_dst;
     }
   }
+  a.padd = ws.mpos.p; a.nadd = d.nadd; a.pdel = ws.mpos.p + d.nadd; a.ndel = d.ndel;
+  a.abnd = ws.mbnd.p; a.dbnd = ws.mbnd.p + ntm + 1; a.ntm = ntm;
   a.tbase = ws.lb_base;
   ws.lb_base += (uint32_t)ntiles;                        // every tile claims one ticket
   k_rowscan<true><<<ntiles, kRowThreads, 0, s>>>(a);
@@ -938,7 +947,8 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
   m.ncol = in_dir ? dst.in_col.p : dst.out_col.p;
   m.emap_out = emap_out; m.emap_in = emap_in; m.eid_old = eid_old; m.eid_new = eid_new;
   m.in_rowptr_new = in_rowptr_new; m.in_col_new = in_col_new;
-  k_merge3<<<(unsigned)ntm, 256, 0, s>>>(m);
+  if (m.eid_new) k_merge4<true><<<(unsigned)ceil_div(ntm, 8), 256, 0, s>>>(m, ntm);
+  else k_merge4<false><<<(unsigned)ceil_div(ntm, 8), 256, 0, s>>>(m, ntm);
   count_launch();
   const int32_t R = blk ? dst.rows() : V;
   return ids_sched_from_hist(a.deg_new, a.rowptr_new, V, R, in_dir ? dst.in_ids.p : dst.out_ids.p,
