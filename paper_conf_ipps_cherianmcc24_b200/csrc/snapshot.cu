@@ -90,6 +90,17 @@ __device__ __forceinline__ int32_t old_pos(const int32_t* __restrict__ orowptr, 
                                            uint64_t key, int nb) {
   const int32_t r = (int32_t)(key >> nb), c = (int32_t)(key & ((uint64_t(1) << nb) - 1));
   int32_t b = __ldg(orowptr + r), e = __ldg(orowptr + r + 1);
+  // lower bound of c in ocol[b, e): 8-ary steps (7 independent probes per level, so a
+  // hub row of 10^5 edges takes 6 dependent rounds instead of 17), binary below 8
+  while (e - b > 8) {
+    const int32_t len = e - b;
+    int32_t lt = 0;                                   // probes below c (they are monotone)
+#pragma unroll
+    for (int k = 1; k < 8; ++k) lt += __ldg(ocol + b + (int32_t)(((int64_t)len * k) >> 3)) < c;
+    const int32_t nb_ = lt ? b + (int32_t)(((int64_t)len * lt) >> 3) + 1 : b;
+    e = lt < 7 ? b + (int32_t)(((int64_t)len * (lt + 1)) >> 3) : e;
+    b = nb_;
+  }
   while (b < e) {
     const int32_t mid = (b + e) >> 1;
     if (__ldg(ocol + mid) < c) b = mid + 1; else e = mid;

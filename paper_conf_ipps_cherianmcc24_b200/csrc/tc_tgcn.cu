@@ -999,6 +999,177 @@ __global__ void __launch_bounds__(192, 1) k_tc_atb2(const __grid_constant__ CUte
   if (warp == 1) tc::tmem_free(tm, tcols);
 }
 
+// ------------------------------------------------------------------ dL, gate-blocked (H = 32)
+// Only the gate-diagonal blocks of Σ_rows [C|H]ᵀ·da are parameter gradients:
+//   D_g = Σ_rows [C_g | H_g' | ones]ᵀ · da_g,   H_z' = H_r' = H, H_h' = RH,
+// rows 0..H-1 → dL_g¹, rows H..2H-1 → dL_g², row 2H → dl_g (the ones feature).
+// Three M = 128, N = 32 products per tile instead of two M = 128, N = 96 ones
+// (half the 3xTF32 tensor work, TMEM 96 columns).  Each A operand is 4 box slots
+// LBO apart in the stage (slots 0..10, BOX bytes each):
+//   0 C_z  1 C_r  2 H  3 ones  4 ones  5 C_h  6 RH  7 ones  8 da_z  9 da_r  10 da_h
+//   A_z = slots 0, 2, 4, 6 (LBO 2 boxes)   A_r = 1, 2, 3, 4   A_h = 5, 6, 7, 8
+// (the 4th chunk of each is another operand: D rows 96..127, never read).  The
+// ones boxes are static (hi = 1.0 in feature 0, lo = 0); warp 0 issues the TMA,
+// warp 1 the MMAs, warps 2-5 convert (lo = x − trunc x) and run the epilogue.
+constexpr int kDl3Slots = 11;
+template <int RT, int S, int L>
+__global__ void __launch_bounds__(192, 1) k_tc_dl3(const __grid_constant__ CUtensorMap mC,
+                                                   const __grid_constant__ CUtensorMap mH,
+                                                   const __grid_constant__ CUtensorMap mRH,
+                                                   const __grid_constant__ CUtensorMap mDA,
+                                                   const __grid_constant__ CUtensorMap m_ones, int V,
+                                                   float* __restrict__ part) {
+  constexpr int BOX = RT * 32 * 4;
+  constexpr int NS = kDl3Slots;
+  constexpr uint32_t ONES = (1u << 3) | (1u << 4) | (1u << 7);
+  extern __shared__ unsigned char sm_raw[];
+  unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t full[S], empty[S], conv[L], lfree[L], done, init_bar;
+  __shared__ uint32_t tslot;
+  constexpr size_t half = (size_t)NS * BOX;          // one stage (hi ring) or one lo slot
+  auto hi = [&](int st, int bx) { return sm + (size_t)st * half + (size_t)bx * BOX; };
+  auto lo = [&](int ls, int bx) { return sm + (size_t)(S + ls) * half + (size_t)bx * BOX; };
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (size_t e = threadIdx.x; e < (size_t)(S + L) * half / 16; e += blockDim.x)   // lo of the ones boxes stays 0
+    reinterpret_cast<float4*>(sm)[e] = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (warp == 1) tc::tmem_alloc(&tslot, 128);
+  if (threadIdx.x == 0) {
+    for (int st = 0; st < S; ++st) { tc::mbar_init(&full[st], 1); tc::mbar_init(&empty[st], 1); }
+    for (int ls = 0; ls < L; ++ls) { tc::mbar_init(&conv[ls], 128); tc::mbar_init(&lfree[ls], 1); }
+    tc::mbar_init(&done, 1); tc::mbar_init(&init_bar, 1);
+    tc::fence_mbar_init();
+  }
+  tc::fence_proxy_async();
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  if (threadIdx.x == 0) {                            // the static ones boxes of every stage
+    tc::mbar_expect_tx(&init_bar, (uint32_t)(3 * S * BOX));
+    for (int st = 0; st < S; ++st)
+      for (int k = 0; k < NS; ++k)
+        if ((ONES >> k) & 1u) tc::tma_load_2d(hi(st, k), &m_ones, 0, 0, &init_bar);
+  }
+  tc::mbar_wait(&init_bar, 0);
+  const uint32_t tm = tslot;
+  const int ntiles = (V + RT - 1) / RT;
+  int my_tiles = 0;
+  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) ++my_tiles;
+  if (warp == 0) {                                   // ---- TMA producer
+    if (lane == 0) {
+      for (int i = 0; i < my_tiles; ++i) {
+        const int st = i % S, kk = i / S, r0 = (blockIdx.x + i * gridDim.x) * RT;
+        if (kk > 0) tc::mbar_wait(&empty[st], (kk - 1) & 1);
+        tc::mbar_expect_tx(&full[st], (uint32_t)(8 * BOX));
+        tc::tma_load_2d(hi(st, 0), &mC, 0, r0, &full[st]);
+        tc::tma_load_2d(hi(st, 1), &mC, 32, r0, &full[st]);
+        tc::tma_load_2d(hi(st, 5), &mC, 64, r0, &full[st]);
+        tc::tma_load_2d(hi(st, 2), &mH, 0, r0, &full[st]);
+        tc::tma_load_2d(hi(st, 6), &mRH, 0, r0, &full[st]);
+        tc::tma_load_2d(hi(st, 8), &mDA, 0, r0, &full[st]);
+        tc::tma_load_2d(hi(st, 9), &mDA, 32, r0, &full[st]);
+        tc::tma_load_2d(hi(st, 10), &mDA, 64, r0, &full[st]);
+      }
+    }
+  } else if (warp == 1) {                            // ---- MMA issuer
+    if (lane == 0) {
+      const uint32_t idesc = tc::idesc_tf32(128, 32, 1, 1);
+      const int a_slot[3] = {0, 1, 5}, b_slot[3] = {8, 9, 10};
+      const uint32_t lbo[3] = {2u * BOX, (uint32_t)BOX, (uint32_t)BOX};
+      for (int i = 0; i < my_tiles; ++i) {
+        const int st = i % S, ls = i % L;
+        tc::mbar_wait(&conv[ls], (i / L) & 1);
+        tc::fence_after();
+#pragma unroll
+        for (int g = 0; g < 3; ++g) {
+          const uint32_t ah = tc::smem_u32(hi(st, a_slot[g])), al = tc::smem_u32(lo(ls, a_slot[g]));
+          const uint32_t bh = tc::smem_u32(hi(st, b_slot[g])), bl = tc::smem_u32(lo(ls, b_slot[g]));
+          const uint32_t d = tm + 32 * g;
+          for (int k = 0; k < RT; k += 8) {              // 8 K-rows (1024 B) per MMA
+            const uint32_t o = (uint32_t)k * 128;
+            const uint64_t dah = tc::desc_mn_sw128_32b(ah + o, lbo[g]), dal = tc::desc_mn_sw128_32b(al + o, lbo[g]);
+            const uint64_t dbh = tc::desc_mn_sw128_32b(bh + o, BOX), dbl = tc::desc_mn_sw128_32b(bl + o, BOX);
+            tc::mma_tf32(d, dal, dbh, idesc, (i > 0 || k > 0) ? 1u : 0u);
+            tc::mma_tf32(d, dah, dbl, idesc, 1u);
+            tc::mma_tf32(d, dah, dbh, idesc, 1u);
+          }
+        }
+        tc::commit(&empty[st]);
+        tc::commit(&lfree[ls]);
+      }
+      tc::commit(&done);
+    }
+  } else {                                           // ---- converters (warps 2-5), then epilogue
+    const int ct = threadIdx.x - 64;
+    for (int i = 0; i < my_tiles; ++i) {
+      const int st = i % S, ls = i % L;
+      tc::mbar_wait(&full[st], (i / S) & 1);
+      if (i >= L) tc::mbar_wait(&lfree[ls], ((i / L) - 1) & 1);   // MMAs of tile i-L done with slot ls
+      const uint32_t hb = tc::smem_u32(hi(st, 0)), lb = tc::smem_u32(lo(ls, 0));
+      constexpr int B4 = BOX / 16;                    // float4 per box
+      for (int e0 = ct; e0 < NS * B4; e0 += 8 * 128) {
+        float4 v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          if (e0 + 128 * j < NS * B4) v[j] = tc::lds128(hb + 16u * (uint32_t)(e0 + 128 * j));
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int e = e0 + 128 * j;
+          if (e < NS * B4 && !((ONES >> (e / B4)) & 1u))
+            tc::sts128(lb + 16u * (uint32_t)e,
+                       make_float4(v[j].x - tc::tf32_hi(v[j].x), v[j].y - tc::tf32_hi(v[j].y),
+                                   v[j].z - tc::tf32_hi(v[j].z), v[j].w - tc::tf32_hi(v[j].w)));
+        }
+      }
+      tc::fence_proxy_async();
+      tc::mbar_arrive(&conv[ls]);
+    }
+    // epilogue: rows 0..2H of each gate's D (lane quarter warp % 4), part[cta][g][row][32]
+    tc::mbar_wait(&done, 0);
+    tc::fence_after();
+    const int q = warp & 3, row = q * 32 + lane;
+    float* out = part + (size_t)blockIdx.x * 3 * 65 * 32;
+    for (int c = 0; c < 96; c += 8) {
+      float v[8];
+      if (my_tiles == 0 || q > 2) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = 0.f;
+      } else {
+        tc::tmem_ld8(tm + ((uint32_t)(q * 32) << 16) + (uint32_t)c, v);
+        tc::tmem_wait_ld();
+      }
+      const int g = c / 32, cc = c % 32;
+      if (row <= 64) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) out[((size_t)g * 65 + row) * 32 + cc + e] = v[e];
+      }
+    }
+  }
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 1) tc::tmem_free(tm, 128);
+}
+
+// dL / dl / db from the gate blocks tot[g][row][j] (rows 0..2H-1: [C_g | H_g'], row 2H: ones)
+__global__ void k_dl3_scatter(const float* __restrict__ tot, const float* __restrict__ L, float* __restrict__ dL,
+                              float* __restrict__ dl, float* __restrict__ db) {
+  constexpr int H = 32, LG = 2 * H * H;
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < 6 * H * H + 6 * H; e += gridDim.x * blockDim.x) {
+    if (e < 6 * H * H) {
+      const int g = e / LG, rem = e % LG, i = rem / H, j = rem % H;
+      dL[e] += tot[((size_t)g * 65 + i) * 32 + j];
+    } else if (e < 6 * H * H + 3 * H) {
+      const int c = e - 6 * H * H, g = c / H, j = c % H;
+      dl[c] += tot[((size_t)g * 65 + 64) * 32 + j];
+    } else {
+      const int c = e - 6 * H * H - 3 * H, g = c / H, i = c % H;      // db_g = dl_g · L_g¹ᵀ
+      const float* Lg = L + (int64_t)g * LG;
+      float s = 0.f;
+      for (int j = 0; j < H; ++j) s = fmaf(tot[((size_t)g * 65 + 64) * 32 + j], Lg[i * H + j], s);
+      db[c] += s;
+    }
+  }
+}
+
 // Fixed-order sum of the per-CTA partials: tot[e] = Σ_b part[b][e] (blocks of 16).
 __global__ void k_tc_sum_parts(const float* __restrict__ part, int nb, int n, float* __restrict__ tot) {
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
@@ -1746,8 +1917,34 @@ stg_status tc_dw(int V, int F, int H, const float* X, const float* dP, float* pa
 // dL, dl, db from C, H, RH, da (see k_tc_gru_bwd2) with ONE reduction kernel:
 //   D1 = [C_z|C_r|C_h | H]ᵀ·da  (C in feature boxes 0.., H at feature 32·ceil(3H/32)),
 //   D2 = [RH | ones]ᵀ·da        (RH features 0..H, the ones feature at 32).
+static stg_status tc_dl3(int V, const float* C, const float* Hp, const float* RH, const float* da, float* part,
+                         float* tot, float* dL, float* dl, float* db, const float* L, cudaStream_t s) {
+  constexpr int H = 32, RT = kAtbRT, S = 3, Ls = 2;
+  CUtensorMap mC, mH, mRH, mDA, ones;
+  STG_TRY(make_tmap_f32(&mC, C, (uint64_t)V, 3 * H, 3 * H, 32, RT, true));
+  STG_TRY(make_tmap_f32(&mH, Hp, (uint64_t)V, H, H, 32, RT, true));
+  STG_TRY(make_tmap_f32(&mRH, RH, (uint64_t)V, H, H, 32, RT, true));
+  STG_TRY(make_tmap_f32(&mDA, da, (uint64_t)V, 3 * H, 3 * H, 32, RT, true));
+  STG_TRY(ones_map(&ones, RT, s));
+  const size_t smem = (size_t)(S + Ls) * kDl3Slots * RT * 32 * 4 + 1024;
+  STG_CUDA(cudaFuncSetAttribute(k_tc_dl3<RT, S, Ls>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int ntiles = (V + RT - 1) / RT;
+  const int nb = std::max(1, std::min(ntiles, num_sms()));
+  k_tc_dl3<RT, S, Ls><<<nb, 192, smem, s>>>(mC, mH, mRH, mDA, ones, V, part);
+  const int n = 3 * 65 * 32;
+  k_tc_sum_parts2<<<(n + 31) / 32, 256, 0, s>>>(part, nb, n, tot);
+  k_dl3_scatter<<<(6 * H * H + 6 * H + 255) / 256, 256, 0, s>>>(tot, L, dL, dl, db);
+  count_launch(3);
+  return check_launch("tc_dl3");
+}
+
 stg_status tc_dl(int V, int H, const float* C, const float* Hp, const float* RH, const float* da, float* part,
                  float* tot, float* dL, float* dl, float* db, const float* L, cudaStream_t s) {
+  static const int gate_blocked = [] {               // (A/B switch: STG_DL3=0 restores the full products)
+    const char* v = getenv("STG_DL3");
+    return v ? atoi(v) : 1;
+  }();
+  if (H == 32 && gate_blocked) return tc_dl3(V, C, Hp, RH, da, part, tot, dL, dl, db, L, s);
   const int H3 = 3 * H, NBC = (H3 + 31) / 32;
   CUtensorMap m[4], ones;
   STG_TRY(make_tmap_f32(&m[0], C, (uint64_t)V, H3, H3, 32, kAtbRT, true));

@@ -1906,7 +1906,10 @@ stg_status stg_tgcn_train_sequence_peer(stg_dtdg* dtdg, int32_t t0, int32_t S, c
     const float* Hp = i == 0 ? H0 : H_seq + (size_t)(i - 1) * VH;
     const stg_peer_rows rows{px->world, px->bounds, blocks[b], (int64_t)H3};
     const float* ndst_loc = v.norm_dst ? v.norm_dst + v.row_begin : nullptr;
-    STG_TRY(aggregate_launch(&v, 0, H3, nullptr, 0, C, H3, ndst_loc, nullptr, p->b, s, &rows));
+    if (px->world == 1)                                                 // one owner: a plain local gather
+      STG_TRY(aggregate_launch(&v, 0, H3, px->P[b][0], H3, C, H3, ndst_loc, nullptr, p->b, s));
+    else
+      STG_TRY(aggregate_launch(&v, 0, H3, nullptr, 0, C, H3, ndst_loc, nullptr, p->b, s, &rows));
     STG_TRY(publish(ops, px, 1, n, s));
     const HeadArgs ha{Y_loc[i], w_o, b_o, 1.0f / (float)Vall, ws.hd_lpart.p, ws.hd_gpart.p,
                       ws.hg.p + (size_t)i * std::max(R, 1)};
@@ -1935,10 +1938,13 @@ stg_status stg_tgcn_train_sequence_peer(stg_dtdg* dtdg, int32_t t0, int32_t S, c
     STG_TRY(bwd_gru(&v, p, e.C, e.Hp, G, Gn, grads, ws, bb, s, R > 0 ? ws.hg.p + (size_t)i * std::max(R, 1) : nullptr,
                     w_o));
     STG_TRY(bwd_dl(&v, p, e.C, e.Hp, grads, ws, bb, s));
-    STG_TRY(aggregate_launch(&v, 1, H3, bb.dC[0], H3, px->dP[b][px->rank], H3, v.norm_src, nullptr, nullptr, s));
+    // one rank: its partial dP is the whole dP (no reduce-scatter copy)
+    STG_TRY(aggregate_launch(&v, 1, H3, bb.dC[0], H3, px->world == 1 ? dP_loc : px->dP[b][px->rank], H3, v.norm_src,
+                             nullptr, nullptr, s));
     STG_TRY(publish(ops, px, 2, m, s));
     STG_TRY(wait_all(ops, px, 2, m, s));                                // every rank's partial dP is there
-    STG_TRY(stg_reduce_scatter_rows(px->world, px->bounds, dblocks[b], H3, px->rank, H3, dP_loc, H3, stream));
+    if (px->world > 1)
+      STG_TRY(stg_reduce_scatter_rows(px->world, px->bounds, dblocks[b], H3, px->rank, H3, dP_loc, H3, stream));
     STG_TRY(publish(ops, px, 3, m, s));
     STG_TRY(stg_tgcn_dw(p, R, X_loc[i], dP_loc, grads, stack, stream));
     stack->entries.pop_back();
