@@ -117,8 +117,8 @@ __global__ void __launch_bounds__(256) k_touch3(const TouchArgs a) {
     if (k < ng) {
       const uint64_t key = k < a.ngadd ? a.gadd[k] : a.gdel[k - a.ngadd];
       const int sg = k < a.ngadd ? a.sign : -a.sign;
-      atomicAdd(a.din + (int32_t)(key & gmask), sg);
-      atomicAdd(a.dout + (int32_t)(key >> a.nb), sg);
+      if (a.din) atomicAdd(a.din + (int32_t)(key & gmask), sg);
+      if (a.dout) atomicAdd(a.dout + (int32_t)(key >> a.nb), sg);
     }
     const bool on = k < n;
     const bool is_add = k < a.nadd;
@@ -187,8 +187,9 @@ struct RowScanArgs {
   float* norm_dst;
   // fused whole-graph degree step (may be NULL): gin / gout are the source slot's,
   // the degrees are gin + din, gout + dout, written to gin_w / gout_w
-  const int32_t* din;
-  const int32_t* dout;
+  const int32_t* din;           // (NULL with self_dir 1: the in-degrees are this scan's own)
+  const int32_t* dout;          // (NULL with self_dir 2: the out-degrees are this scan's own)
+  int self_dir;                 // unsharded: 1 = this is the in-CSR, 2 = the out-CSR (its deg' is whole-graph)
   int32_t* gin_w;
   int32_t* gout_w;
   // (TOUCH) merge-tile boundaries from the old-CSR positions of k_touch3:
@@ -244,22 +245,22 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
   }
   if (a.norm_dst) {                                    // (independent of the scan: issued first)
     int32_t gi[kRowIPT], go[kRowIPT];
-    if (a.din) {                                       // whole-graph degrees of this step (both kept current)
+    if (a.gin_w) {                                     // whole-graph degrees of this step (both kept current)
       int32_t di[kRowIPT], dd[kRowIPT];
 #pragma unroll
       for (int k = 0; k < kRowIPT; ++k) {
         const int64_t v = r0 + (int64_t)k * kRowThreads;
         const bool ok = v < a.V;
-        gi[k] = ok ? __ldg(a.gin + v) : 0;
-        go[k] = ok ? __ldg(a.gout + v) : 0;
-        di[k] = ok ? __ldcg(a.din + v) : 0;
-        dd[k] = ok ? __ldcg(a.dout + v) : 0;
+        gi[k] = (ok && a.self_dir != 1) ? __ldg(a.gin + v) : 0;
+        go[k] = (ok && a.self_dir != 2) ? __ldg(a.gout + v) : 0;
+        di[k] = (ok && a.self_dir != 1) ? __ldcg(a.din + v) : 0;
+        dd[k] = (ok && a.self_dir != 2) ? __ldcg(a.dout + v) : 0;
       }
 #pragma unroll
       for (int k = 0; k < kRowIPT; ++k) {
         const int64_t v = r0 + (int64_t)k * kRowThreads;
-        gi[k] += di[k];
-        go[k] += dd[k];
+        gi[k] = a.self_dir == 1 ? d[k] : gi[k] + di[k];
+        go[k] = a.self_dir == 2 ? d[k] : go[k] + dd[k];
         if (v < a.V) { a.gin_w[v] = gi[k]; a.gout_w[v] = go[k]; }
       }
     } else {
@@ -664,12 +665,12 @@ __global__ void k_items2(const int32_t* __restrict__ ids, const int32_t* __restr
       touch[(int32_t)(key >> nb)] = make_int4(0, 0, 0, 0);
     }
   }
-  if (din) {
+  if (din || dout) {
     const uint64_t mask = (uint64_t(1) << nb) - 1;
     for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < ngadd + ngdel; k += stride) {
       const uint64_t key = k < ngadd ? gadd[k] : gdel[k - ngadd];
-      din[(int32_t)(key & mask)] = 0;
-      dout[(int32_t)(key >> nb)] = 0;
+      if (din) din[(int32_t)(key & mask)] = 0;
+      if (dout) dout[(int32_t)(key >> nb)] = 0;
     }
   }
 }
@@ -751,6 +752,67 @@ __global__ void __launch_bounds__(256, LABELS ? 5 : 8) k_merge4(const MergeArgs 
   chunk_load(cd, a.pdel, d0, d1, lane);
   chunk_load(ca, a.padd, a0, a1, lane);
   uint64_t key = ca.idx < a1 ? __ldg(a.add + ca.idx) : 0;
+  // Fast path (the common tile: at most 32 adds and 32 deletes, no two adds at one
+  // point): per round a 32-bit mask of deleted positions and one of add points
+  // (warp OR-reductions), lane r < 8 holding round r's masks and the counts before
+  // it; every position then needs a popcount, every add a shuffle.
+  const int32_t p_prev = __shfl_up_sync(FULL, ca.p, 1);
+  const bool dup = (ca.idx < a1) && lane > 0 && p_prev == ca.p;
+  if (d1 - d0 <= 32 && a1 - a0 <= 32 && !__any_sync(FULL, dup)) {
+    const int32_t e0i = (int32_t)e0;
+    const bool vd = cd.idx < d1, va = ca.idx < a1;
+    const int rd = vd ? (cd.p - e0i) >> 5 : -1, ra = va ? (ca.p - e0i) >> 5 : -1;
+    uint32_t md = 0, ma = 0;                          // lane r < 8: round r's masks
+#pragma unroll
+    for (int r = 0; r < kMergeRounds; ++r) {
+      const uint32_t xd = __reduce_or_sync(FULL, rd == r ? 1u << (cd.p & 31) : 0u);
+      const uint32_t xa = __reduce_or_sync(FULL, ra == r ? 1u << (ca.p & 31) : 0u);
+      if (lane == r) { md = xd; ma = xa; }
+    }
+    // counts before round `lane` (exclusive scan over the 8 rounds), as global list indices
+    int32_t sd = __popc(md), sa = __popc(ma);
+#pragma unroll
+    for (int o = 1; o < 8; o <<= 1) {
+      const int32_t yd = __shfl_up_sync(FULL, sd, o), ya = __shfl_up_sync(FULL, sa, o);
+      if (lane >= o) { sd += yd; sa += ya; }
+    }
+    const int32_t Dr = d0 + sd - __popc(md), Ar = a0 + sa - __popc(ma);
+    const uint32_t lt = (1u << lane) - 1u, le = lt | (1u << lane);
+#pragma unroll
+    for (int r = 0; r < kMergeRounds; ++r) {          // the surviving old edges
+      const int32_t j = e0i + r * 32 + lane;
+      const uint32_t mdr = __shfl_sync(FULL, md, r), mar = __shfl_sync(FULL, ma, r);
+      const int32_t D = __shfl_sync(FULL, Dr, r) + __popc(mdr & lt);
+      const int32_t A = __shfl_sync(FULL, Ar, r) + __popc(mar & le);
+      if ((int64_t)j < a.E_old) {
+        const bool deleted = (mdr >> lane) & 1u;
+        const int32_t pos = deleted ? -1 : j - D + A;
+        if (a.emap_out) a.emap_out[j] = pos;
+        if (!deleted) {
+          a.ncol[pos] = c[r];
+          if (LABELS) a.eid_new[pos] = __ldg(a.emap_in + eo[LABELS ? r : 0]);
+        }
+      }
+    }
+    // the adds: deletes before point p = round (p >> 5)'s count + the mask bits below p
+    const int rr = ra < 0 ? 0 : ra;
+    const uint32_t mdp = __shfl_sync(FULL, md, rr);
+    const int32_t Dp = __shfl_sync(FULL, Dr, rr) + __popc(mdp & ((1u << (ca.p & 31)) - 1u));
+    if (va) {
+      const int64_t q = (int64_t)ca.p - Dp + ca.idx;
+      const int32_t v = (int32_t)(key >> a.nb), cc = (int32_t)(key & mask);
+      a.ncol[q] = cc;
+      if (LABELS) {                                   // label = position of (v -> cc) in the new in-CSR
+        int32_t l2 = a.in_rowptr_new[cc], h2 = a.in_rowptr_new[cc + 1];
+        while (l2 < h2) {
+          const int32_t mid = (l2 + h2) >> 1;
+          if (a.in_col_new[mid] < v) l2 = mid + 1; else h2 = mid;
+        }
+        a.eid_new[q] = l2;
+      }
+    }
+    return;
+  }
 #pragma unroll
   for (int r = 0; r < kMergeRounds; ++r) {
     const int64_t base = e0 + r * 32;
@@ -840,7 +902,7 @@ stg_status ids_ws_reserve(BuildWs& ws, int32_t V, int64_t cap, cudaStream_t s) {
 static stg_status ids_sched_from_hist(const int32_t* deg, const int32_t* rowptr, int32_t V, int32_t R, int32_t* ids,
                                       int32_t* sched, int64_t cap, BuildWs& ws, cudaStream_t s, int32_t rb,
                                       int32_t re, const DirDelta* clear, int nb, int4* touch,
-                                      const DirDelta* gclear = nullptr) {
+                                      const DirDelta* gclear = nullptr, int self_dir = 0) {
   const int32_t ntiles = (int32_t)ceil_div(V, kRowTile);
   k_ids_offsets<<<(kIdsBuckets + 31) / 32, 1024, 0, s>>>(ws.ids_hist.p, ntiles, ws.ids_offs.p, ws.ids_tot.p);
   k_ids_scatter<<<ntiles, kRowThreads, 0, s>>>(deg, V, rb, re, ws.ids_offs.p, ws.ids_tot.p, ntiles, ids);
@@ -864,7 +926,7 @@ static stg_status ids_sched_from_hist(const int32_t* deg, const int32_t* rowptr,
       ids, rowptr, icap, sched, ws.ids_tot.p + kIdsBuckets, clear ? clear->add : nullptr, clear ? clear->nadd : 0,
       clear ? clear->del : nullptr, clear ? clear->ndel : 0, nb, touch, gclear ? gclear->add : nullptr,
       gclear ? gclear->nadd : 0, gclear ? gclear->del : nullptr, gclear ? gclear->ndel : 0,
-      gclear ? ws.gdeg.p : nullptr, gclear ? ws.gdeg.p + V : nullptr);
+      gclear && self_dir != 1 ? ws.gdeg.p : nullptr, gclear && self_dir != 2 ? ws.gdeg.p + V : nullptr);
   count_launch(4);
   return check_launch("ids_sched");
 }
@@ -902,6 +964,8 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
   if (gdeg && !norms) return fail(STG_ERR_STATE, "apply_dir2: the degree step rides on the norms pass");
   const int64_t ng = gdeg ? gdeg->keys.nadd + gdeg->keys.ndel : 0;
   const int64_t nk = d.nadd + d.ndel;
+  // unsharded: this direction's new degrees are the whole graph's (in- or out-degrees)
+  const int self_dir = dst.sharded ? 0 : (in_dir ? 1 : 2);
   const int32_t ntm = (int32_t)(src.E >> kMergeShift) + 1;    // merge tiles: positions [0, E_old]
   STG_TRY(ws.mpos.alloc((size_t)std::max<int64_t>(nk, 1), s));
   STG_TRY(ws.mbnd.alloc(2 * ((size_t)ntm + 1), s));
@@ -914,7 +978,9 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
     t.padd = ws.mpos.p; t.pdel = ws.mpos.p + d.nadd;
     if (ng > 0) {
       t.gadd = gdeg->keys.add; t.ngadd = gdeg->keys.nadd; t.gdel = gdeg->keys.del; t.ngdel = gdeg->keys.ndel;
-      t.sign = gdeg->sign; t.din = ws.gdeg.p; t.dout = ws.gdeg.p + V;
+      t.sign = gdeg->sign;
+      t.din = self_dir == 1 ? nullptr : ws.gdeg.p;
+      t.dout = self_dir == 2 ? nullptr : ws.gdeg.p + V;
     }
     k_touch3<<<grid_n(std::max<int64_t>(std::max<int64_t>(nk, ng), 1)), 256, 0, s>>>(t);
     count_launch();
@@ -938,7 +1004,9 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
     a.norm_src = dst.norm_src.p; a.norm_dst = dst.norm_dst.p;
     if (gdeg) {                                          // dst's degrees = src's + this step's deltas
       a.gin = gdeg->gin_src; a.gout = gdeg->gout_src;
-      a.din = ws.gdeg.p; a.dout = ws.gdeg.p + V;
+      a.din = self_dir == 1 ? nullptr : ws.gdeg.p;
+      a.dout = self_dir == 2 ? nullptr : ws.gdeg.p + V;
+      a.self_dir = self_dir;
       a.gin_w = gdeg->gin_dst; a.gout_w = gdeg->gout_dst;
     }
   }
@@ -964,7 +1032,7 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
   const int32_t R = blk ? dst.rows() : V;
   return ids_sched_from_hist(a.deg_new, a.rowptr_new, V, R, in_dir ? dst.in_ids.p : dst.out_ids.p,
                              in_dir ? dst.in_sched.p : dst.out_sched.p, dst.cap, ws, s, a.rb, a.re, &d, src.nb,
-                             touch, gdeg ? &gdeg->keys : nullptr);
+                             touch, gdeg ? &gdeg->keys : nullptr, self_dir);
 }
 
 }  // namespace stg
