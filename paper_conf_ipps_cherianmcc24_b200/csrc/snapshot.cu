@@ -412,6 +412,13 @@ __global__ void __launch_bounds__(kRowThreads) k_ids_scatter(const int32_t* __re
   __shared__ int32_t s_base[kIdsBuckets];
   __shared__ int64_t sh[32];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  constexpr int kOffPT = (kIdsBuckets + kRowThreads - 1) / kRowThreads;
+  int32_t toff[kOffPT];                                   // this tile's bucket offsets, issued first
+#pragma unroll
+  for (int k = 0; k < kOffPT; ++k) {
+    const int d = threadIdx.x + k * kRowThreads;
+    toff[k] = d < kIdsBuckets ? __ldg(offs + (int64_t)d * ntiles + blockIdx.x) : 0;
+  }
   for (int d = lane; d < kIdsBuckets; d += 32) wcnt[w][d] = 0;
   bucket_bases(totals, s_base, sh);
   __syncwarp();
@@ -419,10 +426,15 @@ __global__ void __launch_bounds__(kRowThreads) k_ids_scatter(const int32_t* __re
   const unsigned lt = (1u << lane) - 1u;
   int dig[kScatRounds], rank[kScatRounds];
 #pragma unroll
+  for (int r = 0; r < kScatRounds; ++r) {             // every degree of the warp's rows in flight first
+    const int64_t v = base + r * 32 + lane;
+    dig[r] = v < V ? __ldg(deg + v) : 0;
+  }
+#pragma unroll
   for (int r = 0; r < kScatRounds; ++r) {
     const int64_t v = base + r * 32 + lane;
     const bool ok = v < V;
-    const int dg = ok ? ids_digit((int32_t)v, __ldg(deg + v), rb, re) : kIdsBuckets + lane;
+    const int dg = ok ? ids_digit((int32_t)v, dig[r], rb, re) : kIdsBuckets + lane;
     const unsigned peers = __match_any_sync(0xffffffffu, dg);
     const int before = ok ? wcnt[w][dg] : 0;
     rank[r] = before + __popc(peers & lt);
@@ -432,8 +444,11 @@ __global__ void __launch_bounds__(kRowThreads) k_ids_scatter(const int32_t* __re
     __syncwarp();
   }
   __syncthreads();
-  for (int d = threadIdx.x; d < kIdsBuckets; d += kRowThreads) {   // exclusive prefix over warps + tile offset
-    int32_t run = s_base[d] + offs[(int64_t)d * ntiles + blockIdx.x];
+#pragma unroll
+  for (int k = 0; k < kOffPT; ++k) {                      // exclusive prefix over warps + tile offset
+    const int d = threadIdx.x + k * kRowThreads;
+    if (d >= kIdsBuckets) break;
+    int32_t run = s_base[d] + toff[k];
 #pragma unroll
     for (int ww = 0; ww < kRowThreads / 32; ++ww) {
       const int32_t c = wcnt[ww][d];

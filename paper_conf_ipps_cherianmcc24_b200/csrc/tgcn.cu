@@ -1527,6 +1527,14 @@ int dl_on_chain() {
   }();
   return v;
 }
+// forward: the snapshot build of t+1 starts after conv(t) (default) or after conv(t-1)
+int snap_after_conv() {
+  static const int v = [] {
+    const char* e = getenv("STG_SNAP_AFTER_CONV");
+    return e ? atoi(e) : 1;
+  }();
+  return v;
+}
 std::atomic<int> g_pipeline{1};                   // stg_set_pipeline
 bool pipeline_enabled() { return g_pipeline.load(std::memory_order_relaxed) != 0; }
 // compute on an aux stream beside the H chain (1, default) or on the caller's
@@ -1664,7 +1672,11 @@ stg_status stg_tgcn_train_sequence_ev(const stg_graph* graph, stg_dtdg* dtdg, in
     STG_TRY(fwd_conv(&views[k], p, X[i], ws.P.p, C, as, A));            // P', C (H-independent)
     STG_TRY(record(ev_conv[i & 1], as));
     if (dtdg && i + 1 < S) {                                            // prefetch Get-Graph(t+1)
-      if (i >= 1) STG_TRY(wait(ss, ev_conv[(i + 1) & 1], as));          // conv(t-1) done with that slot
+      // after conv(t) (which implies conv(t-1) is done with that slot): the build of t+1
+      // then runs beside the GRU of t rather than beside the aggregation (two
+      // memory-bound gathers side by side slow each other; STG_SNAP_AFTER_CONV=0: old order)
+      if (snap_after_conv()) STG_TRY(wait(ss, ev_conv[i & 1], as));
+      else if (i >= 1) STG_TRY(wait(ss, ev_conv[(i + 1) & 1], as));     // conv(t-1) done with that slot
       STG_TRY(stg_dtdg_get_snapshot_parts(dtdg, t + 1, 0, STG_PART_IN, ss, &views[(i + 1) & 1]));
       STG_TRY(record(ev_built[(i + 1) & 1], ss));
     }
