@@ -509,69 +509,96 @@ def main():
     if not args.no_e2e:
         Xpin = [x.pin_memory() for x in Xh]
         Ypin = [y.pin_memory() for y in Yh]
-        copy = torch.cuda.Stream(device=dev)
-        stage = [[torch.empty(R if peer else V, F, device=dev) for _ in range(S)] for _ in range(2)]
-        ystage = [[torch.empty(R, device=dev) for _ in range(S)] for _ in range(2)]
-        loss_h = torch.empty(1, pin_memory=True)
+        # a copy stream (STG_E2E_COPY_STREAMS > 1 alternates timestamps over several: measured
+        # slower, 208 vs 205 ms per C5 epoch) and three staging buffer sets, so the copies of
+        # the next sequence — across epoch boundaries too — run while the current one
+        # computes; a sequence's set is refilled once the sequence three back is done
+        ncs = max(1, int(os.environ.get("STG_E2E_COPY_STREAMS", "1")))
+        copies = [torch.cuda.Stream(device=dev) for _ in range(ncs)]
+        NB = 3
+        stage = [[torch.empty(R if peer else V, F, device=dev) for _ in range(S)] for _ in range(NB)]
+        ystage = [[torch.empty(R, device=dev) for _ in range(S)] for _ in range(NB)]
+        loss_h = [torch.empty(1, pin_memory=True) for _ in range(2)]
+        vals = []
         h2d = 0
+        nseq = len(seqs)
+        done = [None] * NB
 
-        def e2e_epoch():
+        def issue(gk):
+            """H2D copies of global sequence gk (sequence gk % nseq of its epoch) into set gk % NB."""
             nonlocal h2d
-            done = [None, None]
-            # prefetch sequence 0
-            def issue(k):
-                nonlocal h2d
-                t0, n = seqs[k]
-                evs = []
-                with torch.cuda.stream(copy):
-                    if done[k % 2] is not None:
-                        copy.wait_event(done[k % 2])
-                    for i in range(n):
-                        stage[k % 2][i].copy_(Xpin[(t0 + i) % NX], non_blocking=True)
-                        ystage[k % 2][i].copy_(Ypin[t0 + i], non_blocking=True)
-                        h2d += Xpin[0].numel() * 4 + Ypin[0].numel() * 4
-                        ev = torch.cuda.Event()          # per timestamp: its step starts when X_t landed
-                        ev.record(copy)
-                        evs.append(ev)
-                return evs
+            t0, n = seqs[gk % nseq]
+            buf = gk % NB
+            evs = []
+            for i in range(n):
+                cs = copies[(t0 + i) % ncs]
+                with torch.cuda.stream(cs):
+                    if done[buf] is not None:
+                        cs.wait_event(done[buf])
+                    stage[buf][i].copy_(Xpin[(t0 + i) % NX], non_blocking=True)
+                    ystage[buf][i].copy_(Ypin[t0 + i], non_blocking=True)
+                    h2d += Xpin[0].numel() * 4 + Ypin[0].numel() * 4
+                    ev = torch.cuda.Event()              # per timestamp: its step starts when X_t landed
+                    ev.record(cs)
+                    evs.append(ev)
+            return evs
+
+        def e2e_run(nepochs):
+            """nepochs epochs back to back; every epoch reads its loss back (D2H) before the
+            next one's result is needed; returns the last loss."""
+            nonlocal done
+            done = [None] * NB
+            total = nepochs * nseq
             ready = issue(0)
             Hprev = H0
-            for k, (t0, n) in enumerate(seqs):
+            last = None
+            vals.clear()
+            for gk in range(total):
+                k = gk % nseq
+                t0, n = seqs[k]
+                buf = gk % NB
+                if k == 0:
+                    Hprev = H0
                 per_step = (not peer) and (not batched)
                 if not per_step:
                     stream.wait_event(ready[-1])
-                if k + 1 < len(seqs):
-                    nxt = issue(k + 1) if True else None
+                nxt = issue(gk + 1) if gk + 1 < total else None
                 Hs = Hbuf[k % 2]
                 if peer:
-                    peer_drv.train_sequence(g, t0, p, p["w_o"], p["b_o"], stage[k % 2][:n], ystage[k % 2][:n],
+                    peer_drv.train_sequence(g, t0, p, p["w_o"], p["b_o"], stage[buf][:n], ystage[buf][:n],
                                             Hprev, Hs, grads, dw_o, db_o, loss)
                 elif batched:
-                    stg.stg_tgcn_train_sequence_batched(g, n, p, p["w_o"], p["b_o"], stage[k % 2][:n],
-                                                        ystage[k % 2][:n], Hprev, Hs, grads, dw_o, db_o, loss, stack)
+                    stg.stg_tgcn_train_sequence_batched(g, n, p, p["w_o"], p["b_o"], stage[buf][:n],
+                                                        ystage[buf][:n], Hprev, Hs, grads, dw_o, db_o, loss, stack)
                 else:
-                    stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], stage[k % 2][:n], ystage[k % 2][:n],
+                    stg.stg_tgcn_train_sequence(g, t0, n, p, p["w_o"], p["b_o"], stage[buf][:n], ystage[buf][:n],
                                                 Hprev, Hs, Gw, grads, dw_o, db_o, loss, stack, xy_ready=ready)
                 sgd()
                 ev = torch.cuda.Event()
                 ev.record(stream)
-                done[k % 2] = ev
+                done[buf] = ev
                 Hprev = Hs[n - 1]
-                if k + 1 < len(seqs):
-                    ready = nxt
-            loss_h.copy_(loss, non_blocking=True)
+                if k == nseq - 1:                        # the epoch's result: D2H now, read one epoch later
+                    lb = loss_h[(gk // nseq) % 2]
+                    lb.copy_(loss, non_blocking=True)
+                    lev = torch.cuda.Event()
+                    lev.record(stream)
+                    if last is not None:
+                        last[1].synchronize()
+                        vals.append(float(last[0].item()))
+                    last = (lb, lev)
+                ready = nxt
             torch.cuda.synchronize()
-            return float(loss_h.item())
+            vals.append(float(last[0].item()))
+            return vals[-1]
 
-        for _ in range(1):
-            e2e_epoch()
+        e2e_run(1)
         h2d = 0
         torch.cuda.synchronize()
         if pg:
             dist.barrier()
         t0w = time.perf_counter()
-        for _ in range(args.steps):
-            e2e_epoch()
+        e2e_run(args.steps)
         e2e_s = time.perf_counter() - t0w
         if pg:
             tt = torch.tensor([e2e_s], device=dev)
@@ -580,9 +607,10 @@ def main():
         e2e = {"value": edges_all * args.steps / e2e_s, "unit": UNIT,
                "h2d_bytes_per_step": int(h2d / args.steps), "d2h_bytes_per_step": 4,
                "ms_per_step": 1e3 * e2e_s / args.steps,
-               "note": "X_t (this rank's rows in sharded mode) and y_t copied H2D per timestamp (an event each; "
-                       "a step waits only for its own inputs) from pinned host memory every timestep on a copy "
-                       "stream overlapped with the previous sequence; loss read back every epoch"}
+               "note": "X_t (this rank's rows in sharded mode) and y_t copied H2D per timestamp from pinned host "
+                       "memory on %d copy stream(s), timestamps alternating; three staging sets so the next "
+                       "sequence's copies (across epoch boundaries too) overlap the current one; every "
+                       "epoch's loss read back D2H; wall clock over the K epochs" % ncs}
 
     # ---------------- CPU baseline: the oracle on one C5 timestep, 1 core and all cores (rank 0, N=1 only)
     cpu = None
