@@ -571,6 +571,10 @@ stg_status stg_set_pipeline(int32_t on);
  *   STG_SMALL_RB (auto)    rows per CTA of the small-graph sequence kernels
  *   STG_DL_STREAM (0)      dL/dl reductions on the H-chain stream (1) or aux stream
  *   STG_AUX_STREAM (1)     H-independent work on an aux stream (0: caller's stream)
+ *   STG_SNAP_AFTER_CONV (1) the forward build of Get-Graph(t+1) starts after the
+ *                          convolution of t (0: after that of t-1, beside the gather)
+ *   STG_DL3 (1)            H = 32 dL/dl as three gate-blocked products (0: the two
+ *                          full [C|H]ᵀda, [RH|1]ᵀda products; same gradients to fp32)
  *   STG_TORCH_ALLOCATOR    (binding) 0 keeps cudaMalloc instead of torch's pool */
 
 /* Order of the graph convolution in the TGCN step (reading C14; SURVEY §8(f)
