@@ -390,9 +390,18 @@ def main():
     run_epoch = lambda: epoch(Xdev, Ydev)
     launches_per_epoch = None
     if use_graphs:
+        # capture on a stream that has already run an epoch: the library's per-stream
+        # scratch (aggregation work queues, partials) exists before the capture, so
+        # nothing is allocated while capturing
+        cap_s = torch.cuda.Stream(device=dev)
+        cap_s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(cap_s):
+            epoch(Xdev, Ydev)
+        torch.cuda.current_stream().wait_stream(cap_s)
+        torch.cuda.synchronize()
         cg = torch.cuda.CUDAGraph()
         l0 = stg.kernel_launch_count()
-        with torch.cuda.graph(cg, capture_error_mode="relaxed"):
+        with torch.cuda.graph(cg, stream=cap_s, capture_error_mode="relaxed"):
             epoch(Xdev, Ydev)
         launches_per_epoch = stg.kernel_launch_count() - l0
         cg.replay()
