@@ -376,3 +376,49 @@ def test_aggregate_first_rejects_unsupported(stg, agg_first):
     assert e.value.status == 1
     with pytest.raises(stg.StgError):
         stg.stg_set_conv_order(2)
+
+
+@pytest.mark.parametrize("name,S", [("C2", 8), ("C5s", 4)])
+def test_static_sequence_cuda_graph_replay(stg, name, S):
+    """A sequence-batched training sequence captured as one CUDA graph (on a stream that
+    already ran it, as bench.py does) replays to the eager run's losses, gradients and
+    states bit for bit (every kernel is deterministic; nothing allocates while capturing)."""
+    cfg = gen.CONFIGS[name]
+    if name == "C5s":                                   # a static graph of the DTDG's base edges
+        dd = gen.dtdg(cfg)
+        s, d = dd.src0, dd.dst0
+    else:
+        s, d = gen.static_edges(cfg)
+    g = stg.stg_static_graph_create(cfg.V, s, d, stg.STG_SELF_LOOPS)
+    _, pg = _params(cfg.F, cfg.H, 3)
+    H = cfg.H
+    Xg = [to_gpu(gen.features(cfg, 40 + i)) for i in range(S)]
+    Yg = [to_gpu(gen.labels(cfg, 40 + i)) for i in range(S)]
+    H0 = to_gpu(gen.uniform_pm1(9, 9, cfg.V * H).reshape(cfg.V, H))
+    grads = _zero_grads(cfg.F, H)
+    dw, db, loss = torch.zeros(H, device="cuda"), torch.zeros(1, device="cuda"), torch.zeros(1, device="cuda")
+    Hseq = torch.empty(S, cfg.V, H, device="cuda")
+    stack = stg.stg_state_stack_create(1 << 20)
+
+    def run():
+        for t in (*grads.values(), dw, db, loss):
+            t.zero_()
+        stg.stg_tgcn_train_sequence_batched(g, S, pg, pg["w_o"], pg["b_o"], Xg, Yg, H0, Hseq, grads, dw, db, loss,
+                                            stack)
+
+    cs = torch.cuda.Stream()
+    cs.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(cs):
+        run()
+    torch.cuda.synchronize()
+    ref = {k: v.clone() for k, v in {**grads, "dw": dw, "db": db, "loss": loss, "H": Hseq}.items()}
+    for t in (*grads.values(), dw, db, loss, Hseq):
+        t.fill_(float("nan"))
+    cg = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(cg, stream=cs, capture_error_mode="relaxed"):
+        run()
+    cg.replay()
+    torch.cuda.synchronize()
+    got = {**grads, "dw": dw, "db": db, "loss": loss, "H": Hseq}
+    for k in ref:
+        assert torch.equal(got[k], ref[k]), k
