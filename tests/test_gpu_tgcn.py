@@ -422,3 +422,59 @@ def test_static_sequence_cuda_graph_replay(stg, name, S):
     got = {**grads, "dw": dw, "db": db, "loss": loss, "H": Hseq}
     for k in ref:
         assert torch.equal(got[k], ref[k]), k
+
+
+@pytest.mark.parametrize("order", [0, 1])
+def test_dtdg_sequences_cuda_graph_replay(stg, order):
+    """Two Algorithm-1 sequences over a DTDG (on-demand snapshots on the library's side
+    stream, the three-stream pipeline) captured as one CUDA graph on a stream that already
+    ran them: the replay reproduces an eager run with the same snapshot-cache walk pattern
+    bit for bit.  (A graph replays GPU work only: it is valid while the host-side cache
+    state at replay equals the state at capture, which a fixed per-epoch walk keeps.)"""
+    cfg = gen.CONFIGS["C5s"]
+    dd = gen.dtdg(cfg)
+    g = stg.stg_dtdg_create(dd.V, dd.T, dd.src0, dd.dst0, dd.add_off, dd.add_src, dd.add_dst, dd.del_off,
+                            dd.del_src, dd.del_dst, stg.STG_SELF_LOOPS | stg.STG_EDGE_IDS)
+    _, pg = _params(cfg.F, cfg.H, 3)
+    V, H, F, S = cfg.V, cfg.H, cfg.F, 4
+    seqs = [(0, S), (S, S)]
+    Xg = [to_gpu(gen.features(cfg, 40 + i)) for i in range(2 * S)]
+    Yg = [to_gpu(gen.labels(cfg, 40 + i)) for i in range(2 * S)]
+    H0 = torch.zeros(V, H, device="cuda")
+    grads = _zero_grads(F, H)
+    dw, db, loss = torch.zeros(H, device="cuda"), torch.zeros(1, device="cuda"), torch.zeros(1, device="cuda")
+    Hbuf = [torch.empty(S, V, H, device="cuda") for _ in range(2)]
+    Gw = torch.empty(2, V, H, device="cuda")
+    stack = stg.stg_state_stack_create(S * V * (3 * H + F) * 4 + (1 << 20))
+    stg.stg_set_conv_order(order)
+    try:
+        def run():
+            for t in (*grads.values(), dw, db, loss):
+                t.zero_()
+            Hp = H0
+            for k, (t0, n) in enumerate(seqs):
+                stg.stg_tgcn_train_sequence(g, t0, n, pg, pg["w_o"], pg["b_o"], Xg[t0:t0 + n], Yg[t0:t0 + n], Hp,
+                                            Hbuf[k], Gw, grads, dw, db, loss, stack)
+                Hp = Hbuf[k][n - 1]
+
+        cs = torch.cuda.Stream()
+        cs.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(cs):
+            run()                                       # warm-up: scratch, slots and cache heads settle
+            run()                                       # the reference, in the steady walk pattern
+        torch.cuda.synchronize()
+        ref = {k: v.clone() for k, v in {**grads, "dw": dw, "db": db, "loss": loss, "H0": Hbuf[0],
+                                          "H1": Hbuf[1]}.items()}
+        for t in (*grads.values(), dw, db, loss, *Hbuf):
+            t.fill_(float("nan"))
+        cg = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(cg, stream=cs, capture_error_mode="relaxed"):
+            run()
+        cg.replay()
+        torch.cuda.synchronize()
+        got = {**grads, "dw": dw, "db": db, "loss": loss, "H0": Hbuf[0], "H1": Hbuf[1]}
+        for k in ref:
+            assert torch.equal(got[k], ref[k]), k
+        assert stack.depth == 0
+    finally:
+        stg.stg_set_conv_order(0)
