@@ -385,7 +385,11 @@ def main():
         epoch(Xdev, Ydev)
     torch.cuda.synchronize()
     # CUDA graph of one whole epoch (static graphs: no host-side snapshot state), replayed
-    use_graphs = (args.graphs == 1) or (args.graphs < 0 and static and not pg)
+    # (DTDGs too when the epoch is launch-bound — its features fit in L2, e.g. C4: the
+    # snapshot cache walk is the same every epoch, and the row scan's tile claims and
+    # status tags are device-side, so replays are exact; tests/test_gpu_tgcn.py)
+    small = V * 3 * H * 4 <= 64 * (1 << 20)
+    use_graphs = (args.graphs == 1) or (args.graphs < 0 and (static or small) and not pg and not peer)
     cg = None
     run_epoch = lambda: epoch(Xdev, Ydev)
     launches_per_epoch = None
@@ -471,6 +475,12 @@ def main():
     alg_bytes = 4 * E_mean + 2 * (V + 1) + 2 * (R + 1) + 4 * (V + R) + 4 * Wagg * (V + R)
     f_ms, f_n = prof_timed["agg_fwd"]
     b_ms, b_n = prof_timed["agg_bwd"]
+    agg_timing = "CUDA events around every aggregation launch on its stream, over the timed region"
+    if f_n + b_n == 0:                  # graph replay: no per-launch events, take the single-stream pass
+        f_ms, f_n = prof["agg_fwd"]
+        b_ms, b_n = prof["agg_bwd"]
+        agg_timing = ("CUDA events around every aggregation launch in the single-stream pass (the timed "
+                      "region replays a CUDA graph: no per-launch events)")
     agg_avg_s = ((f_ms + b_ms) / (f_n + b_n)) / 1e3 if (f_n + b_n) else float("nan")
     agg_fwd_s = (f_ms / f_n) / 1e3 if f_n else float("nan")
     agg_bwd_s = (b_ms / b_n) / 1e3 if b_n else float("nan")
@@ -682,7 +692,7 @@ def main():
                          "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": agg_avg_s * 1e3,
                          "avg_fwd_ms": agg_fwd_s * 1e3, "avg_bwd_ms": agg_bwd_s * 1e3,
                          "launches_timed": f_n + b_n,
-                         "timing": "CUDA events around every aggregation launch on its stream, over the timed region",
+                         "timing": agg_timing,
                          "traffic_source": traffic_src, "peak_source": peak_src},
             "aggregation_edges_per_s": (2 * E_mean / (agg_fwd_s + agg_bwd_s)) if f_n and b_n else None,
             "aggregation_metric": "SURVEY §8(d): 2E / (t_fwd + t_bwd) at W = 3H for one snapshot (mean E_t), "

@@ -31,10 +31,8 @@ struct BuildWs {
   DArray<int32_t> mbnd;        // per merge tile: first add | first delete placed in it
   DArray<int32_t> rows;        // COO row ids of one direction (transposes / labels only)
   DArray<uint64_t> lb_status;  // decoupled look-back words, one per row tile
-  DArray<uint32_t> lb_ticket;  // tile counter (zeroed before each scan)
+  DArray<uint32_t> lb_ticket;  // [tile claims, finished tiles, generation] of the row scan (self-resetting)
   DArray<int32_t> gdeg;        // [2V] whole-graph degree deltas of one step (zero between steps)
-  uint32_t lb_epoch = 0;
-  uint32_t lb_base = 0;        // lb_ticket's value when the next row scan starts (tickets are never reset)
 };
 
 namespace {

@@ -176,9 +176,8 @@ struct RowScanArgs {
   int32_t* hist;                // [kIdsBuckets][ntiles]
   int32_t ntiles;
   uint64_t* status;             // [ntiles] look-back words (TOUCH only)
-  uint32_t* ticket;             // tile counter (TOUCH only), equal to tbase at launch
-  uint32_t tbase;
-  uint32_t epoch;
+  uint32_t* ticket;             // (TOUCH) [tile claims, finished tiles, generation], zero-initialised;
+                                // each launch's last tile resets the counts and bumps the generation
   // GCN norms from the whole-graph degrees (may be NULL: not computed)
   const int32_t* gin;
   const int32_t* gout;
@@ -219,14 +218,20 @@ template <bool TOUCH>
 __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
   __shared__ int32_t h[kIdsBuckets];
   __shared__ int64_t sh[32];
-  __shared__ uint32_t s_tile;
+  __shared__ uint32_t s_tile, s_epoch;
   __shared__ int64_t s_prefix;
   for (int d = threadIdx.x; d < kIdsBuckets; d += kRowThreads) h[d] = 0;
   if (TOUCH) {
-    if (threadIdx.x == 0) s_tile = atomicAdd(a.ticket, 1u) - a.tbase;   // tiles in start order: look-back never waits on an unstarted tile
+    if (threadIdx.x == 0) {
+      s_tile = atomicAdd(a.ticket, 1u);                // tiles in start order: look-back never waits on an unstarted tile
+      // this launch's status-word tag: the generation the previous launch left, plus one
+      // (device-side, so a CUDA-graph replay of the launch gets a fresh tag too)
+      s_epoch = *reinterpret_cast<volatile uint32_t*>(a.ticket + 2) % 0x3fffffffu + 1u;
+    }
   }
   __syncthreads();
   const int32_t tile = TOUCH ? (int32_t)s_tile : (int32_t)blockIdx.x;
+  const uint32_t epoch = TOUCH ? s_epoch : 0u;
   // striped rows (coalesced): row k of this thread = tile·kRowTile + k·kRowThreads + t
   const int64_t r0 = (int64_t)tile * kRowTile + threadIdx.x;
   int32_t d[kRowIPT];
@@ -311,14 +316,14 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
     }
     if (threadIdx.x < 32) {                             // warp 0: publish, then look back 32 tiles at a time
       uint64_t* st = a.status + tile;
-      if (threadIdx.x == 0) lb_store(st, lb_pack(a.epoch, tile == 0 ? 2u : 1u, (uint32_t)tot));
+      if (threadIdx.x == 0) lb_store(st, lb_pack(epoch, tile == 0 ? 2u : 1u, (uint32_t)tot));
       int64_t prefix = 0;
       for (int32_t j0 = tile - 1; j0 >= 0; j0 -= 32) {
         const int32_t j = j0 - lane;
         uint64_t w = 0;
         uint32_t fl = 2u;                               // lanes past tile 0 act as an inclusive zero
         if (j >= 0) {
-          do { w = lb_load(a.status + j); } while ((uint32_t)(w >> 34) != a.epoch || ((w >> 32) & 3u) == 0);
+          do { w = lb_load(a.status + j); } while ((uint32_t)(w >> 34) != epoch || ((w >> 32) & 3u) == 0);
           fl = (uint32_t)(w >> 32) & 3u;
         }
         const unsigned incl = __ballot_sync(0xffffffffu, fl == 2u);
@@ -330,7 +335,7 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
         if (first >= 0) break;
       }
       if (threadIdx.x == 0) {
-        if (tile > 0) lb_store(st, lb_pack(a.epoch, 2u, (uint32_t)(prefix + tot)));
+        if (tile > 0) lb_store(st, lb_pack(epoch, 2u, (uint32_t)(prefix + tot)));
         s_prefix = prefix;
         if ((int64_t)(tile + 1) * kRowTile >= a.V) a.rowptr_new[a.V] = (int32_t)(prefix + tot);
       }
@@ -353,6 +358,14 @@ __global__ void __launch_bounds__(kRowThreads) k_rowscan(const RowScanArgs a) {
   }
   __syncthreads();
   for (int dg = threadIdx.x; dg < kIdsBuckets; dg += kRowThreads) a.hist[(int64_t)dg * a.ntiles + tile] = h[dg];
+  if (TOUCH && threadIdx.x == 0) {                      // last tile out: reset the claims, publish the generation
+    __threadfence();
+    if (atomicAdd(a.ticket + 1, 1u) == gridDim.x - 1) {
+      a.ticket[0] = 0;
+      a.ticket[1] = 0;
+      a.ticket[2] = epoch;
+    }
+  }
 }
 
 // ------------------------------------------------------------ node_ids
@@ -901,10 +914,9 @@ stg_status ids_ws_reserve(BuildWs& ws, int32_t V, int64_t cap, cudaStream_t s) {
     STG_TRY(ws.lb_status.alloc((size_t)ntiles, s));
     STG_CUDA(cudaMemsetAsync(ws.lb_status.p, 0, sizeof(uint64_t) * ws.lb_status.n, s));
   }
-  if (!ws.lb_ticket.p) {                                // a monotone ticket counter: no reset per scan
-    STG_TRY(ws.lb_ticket.alloc(1, s));
-    STG_CUDA(cudaMemsetAsync(ws.lb_ticket.p, 0, sizeof(uint32_t), s));
-    ws.lb_base = 0;
+  if (!ws.lb_ticket.p) {                                // self-resetting claim counters + generation
+    STG_TRY(ws.lb_ticket.alloc(3, s));
+    STG_CUDA(cudaMemsetAsync(ws.lb_ticket.p, 0, 3 * sizeof(uint32_t), s));
   }
   if (ws.gdeg.n < 2 * (size_t)V || !ws.gdeg.p) {        // whole-graph degree deltas: zero between steps
     STG_TRY(ws.gdeg.alloc(2 * (size_t)(V > 0 ? V : 1), s));
@@ -1013,7 +1025,6 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
   a.ntiles = ntiles;
   a.status = ws.lb_status.p;
   a.ticket = ws.lb_ticket.p;
-  a.epoch = (++ws.lb_epoch) & 0x3fffffffu;
   if (norms) {
     a.gin = dst.gin_deg.p; a.gout = dst.gout_deg.p; a.dgl_both = dst.dgl_both;
     a.norm_src = dst.norm_src.p; a.norm_dst = dst.norm_dst.p;
@@ -1027,8 +1038,6 @@ stg_status apply_dir2(const Snapshot& src, Snapshot& dst, bool in_dir, const Dir
   }
   a.padd = ws.mpos.p; a.nadd = d.nadd; a.pdel = ws.mpos.p + d.nadd; a.ndel = d.ndel;
   a.abnd = ws.mbnd.p; a.dbnd = ws.mbnd.p + ntm + 1; a.ntm = ntm;
-  a.tbase = ws.lb_base;
-  ws.lb_base += (uint32_t)ntiles;                        // every tile claims one ticket
   k_rowscan<true><<<ntiles, kRowThreads, 0, s>>>(a);
   count_launch();
   MergeArgs m{};

@@ -417,11 +417,12 @@ def test_static_sequence_cuda_graph_replay(stg, name, S):
     cg = torch.cuda.CUDAGraph()
     with torch.cuda.graph(cg, stream=cs, capture_error_mode="relaxed"):
         run()
-    cg.replay()
-    torch.cuda.synchronize()
     got = {**grads, "dw": dw, "db": db, "loss": loss, "H": Hseq}
-    for k in ref:
-        assert torch.equal(got[k], ref[k]), k
+    for rep in range(3):
+        cg.replay()
+        torch.cuda.synchronize()
+        for k in ref:
+            assert torch.equal(got[k], ref[k]), (rep, k)
 
 
 @pytest.mark.parametrize("order", [0, 1])
@@ -470,11 +471,17 @@ def test_dtdg_sequences_cuda_graph_replay(stg, order):
         cg = torch.cuda.CUDAGraph()
         with torch.cuda.graph(cg, stream=cs, capture_error_mode="relaxed"):
             run()
-        cg.replay()
-        torch.cuda.synchronize()
         got = {**grads, "dw": dw, "db": db, "loss": loss, "H0": Hbuf[0], "H1": Hbuf[1]}
-        for k in ref:
-            assert torch.equal(got[k], ref[k]), k
+        for rep in range(3):                            # repeated replays: no host-side state baked in
+            cg.replay()
+            torch.cuda.synchronize()
+            for k in ref:
+                assert torch.equal(got[k], ref[k]), (rep, k)
         assert stack.depth == 0
+        with torch.cuda.stream(cs):                     # and eager calls after the replays still agree
+            run()
+        torch.cuda.synchronize()
+        for k in ref:
+            assert torch.equal(got[k], ref[k]), ("eager after replays", k)
     finally:
         stg.stg_set_conv_order(0)
