@@ -396,8 +396,10 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(sm_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full[2], mma_bar;
   __shared__ uint32_t tslot;
-  unsigned char* bz_hi = sm + G::WOFF;  unsigned char* bz_lo = bz_hi + G::BG;
-  unsigned char* br_hi = bz_lo + G::BG; unsigned char* br_lo = br_hi + G::BG;
+  // [Bz; Br] hi and lo are each one contiguous N = 2H operand (the z and r gates' H parts
+  // run as one N = 2H product into the adjacent accumulators z | r)
+  unsigned char* bz_hi = sm + G::WOFF;  unsigned char* br_hi = bz_hi + G::BG;
+  unsigned char* bz_lo = br_hi + G::BG; unsigned char* br_lo = bz_lo + G::BG;
   unsigned char* bh_hi = br_lo + G::BG; unsigned char* bh_lo = bh_hi + G::BG;
   auto rawC = [&](int b) { return sm + (size_t)b * G::RAW; };
   auto rawH = [&](int b) { return sm + (size_t)b * G::RAW + G::NBC * kBox; };
@@ -444,7 +446,7 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
     issue(blockIdx.x, 0);
     issue(blockIdx.x + gridDim.x, 1);
   }
-  const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0);
+  const uint32_t idesc = tc::idesc_tf32(128, H, 0, 0), idesc2 = tc::idesc_tf32(128, 2 * H, 0, 0);
   uint32_t mph = 0;
   int i = 0;
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
@@ -467,9 +469,8 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_fwd2(int V, const __grid_cons
       tc::fence_after();
       const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
       mma_ts_seg(tm + 8 * H, tm + 0, tm + 3 * H, zh, zl, 2 * H, 0, H, idesc, true);          // z: C_z part
-      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, idesc, false);     //    H part
       mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, idesc, true);         // r: C_r part
-      mma_ts_seg(tm + 9 * H, tm + 2 * H, tm + 5 * H, rh_, rl, 2 * H, H, H, idesc, false);    //    H part
+      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, idesc2, false);    // z | r: H part
       tc::commit(&mma_bar);
       issue(tile + 2 * gridDim.x, b);                  // raw buffer b is free
     }
@@ -645,8 +646,8 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
   __shared__ uint64_t full, mma_bar;
   __shared__ uint32_t tslot;
   unsigned char* w0 = sm + G::WOFF;
-  unsigned char* bz_hi = w0;              unsigned char* bz_lo = w0 + 1 * G::BG;
-  unsigned char* br_hi = w0 + 2 * G::BG;  unsigned char* br_lo = w0 + 3 * G::BG;
+  unsigned char* bz_hi = w0;              unsigned char* br_hi = w0 + 1 * G::BG;   // [Bz; Br] contiguous (as fwd2)
+  unsigned char* bz_lo = w0 + 2 * G::BG;  unsigned char* br_lo = w0 + 3 * G::BG;
   unsigned char* bh_hi = w0 + 4 * G::BG;  unsigned char* bh_lo = w0 + 5 * G::BG;
   unsigned char* lz_hi = w0 + 6 * G::BG;  unsigned char* lz_lo = w0 + 7 * G::BG;
   unsigned char* lr_hi = w0 + 8 * G::BG;  unsigned char* lr_lo = w0 + 9 * G::BG;
@@ -734,10 +735,9 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_bwd2(int V, const __grid_cons
     if (threadIdx.x == 0) {                             // P1; then request the next tile
       tc::fence_after();
       const uint32_t zh = tc::smem_u32(bz_hi), zl = tc::smem_u32(bz_lo), rh_ = tc::smem_u32(br_hi), rl = tc::smem_u32(br_lo);
-      mma_ts_seg(tm + 8 * H, tm + 0, tm + 3 * H, zh, zl, 2 * H, 0, H, id_h, true);
-      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, id_h, false);
-      mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, id_h, true);
-      mma_ts_seg(tm + 9 * H, tm + 2 * H, tm + 5 * H, rh_, rl, 2 * H, H, H, id_h, false);
+      mma_ts_seg(tm + 8 * H, tm + 0, tm + 3 * H, zh, zl, 2 * H, 0, H, id_h, true);          // z: C_z part
+      mma_ts_seg(tm + 9 * H, tm + H, tm + 4 * H, rh_, rl, 2 * H, 0, H, id_h, true);         // r: C_r part
+      mma_ts_seg(tm + 8 * H, tm + 2 * H, tm + 5 * H, zh, zl, 2 * H, H, H, id_2h, false);    // z | r: H part
       tc::commit(&mma_bar);
       issue(tile + gridDim.x);
     }
@@ -1460,8 +1460,8 @@ __global__ void __launch_bounds__(256, 1) k_tc_gru_seq_bwd(int V, int S, const _
   __shared__ float s_dot[2][128];
   __shared__ float s_g[4][H + 1];
   unsigned char* w0 = sm + G::WOFF;
-  unsigned char* bz_hi = w0;              unsigned char* bz_lo = w0 + 1 * G::BG;
-  unsigned char* br_hi = w0 + 2 * G::BG;  unsigned char* br_lo = w0 + 3 * G::BG;
+  unsigned char* bz_hi = w0;              unsigned char* br_hi = w0 + 1 * G::BG;   // [Bz; Br] contiguous (as fwd2)
+  unsigned char* bz_lo = w0 + 2 * G::BG;  unsigned char* br_lo = w0 + 3 * G::BG;
   unsigned char* bh_hi = w0 + 4 * G::BG;  unsigned char* bh_lo = w0 + 5 * G::BG;
   unsigned char* lz_hi = w0 + 6 * G::BG;  unsigned char* lz_lo = w0 + 7 * G::BG;
   unsigned char* lr_hi = w0 + 8 * G::BG;  unsigned char* lr_lo = w0 + 9 * G::BG;
