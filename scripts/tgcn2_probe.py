@@ -64,7 +64,7 @@ for _ in range(a.epochs):
     epoch()
 e1.record()
 torch.cuda.synchronize()
-ms = e0.elapsed_time(e1) / a.epochs
+ms = e0.elapsed_time(e1) / max(1, a.epochs)
 prof = stg.stg_profile_read(reset=True)
 E = sum(g.num_edges(t) for t in range(T))
 print(json.dumps({"model": "original T-GCN (NEXT-2), per-step library calls, one stream", "config": a.config,
