@@ -71,4 +71,4 @@ print(json.dumps({"model": "original T-GCN (NEXT-2), per-step library calls, one
                   "ms_per_epoch": ms, "timesteps_per_s": T / (ms / 1e3),
                   "aggregated_edges_per_s": 4 * E / (ms / 1e3),
                   "note": "4 aggregations per timestep (2 fwd: widths 2H, H; 2 bwd)",
-                  "phases_ms_per_epoch": {k: v[0] / a.epochs for k, v in prof.items()}}), flush=True)
+                  "phases_ms_per_epoch": {k: v[0] / max(1, a.epochs) for k, v in prof.items()}}), flush=True)
